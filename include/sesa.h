@@ -1,0 +1,212 @@
+/*
+ * sesa.h — C ABI of the B200-native concrete race checker (SESA hot path).
+ *
+ * Paper: P. Li, G. Li, G. Gopalakrishnan, "Practical Symbolic Race Checking of GPU Programs", SC'14.
+ * Citations "P:<line>" refer to /root/reference/PAPER.md (the paper's extracted text) and name the
+ * section they fall in.  The paper checks races symbolically, instantiating a barrier interval's read
+ * and write sets at two thread ids t1 != t2 (§II; §IV-B).  This library decides the
+ * same question exhaustively on CONCRETE access records ("race state" entries `cond ? r|w(addr)` of one
+ * thread in one barrier interval, §IV-A), every thread of the real launch geometry at once.
+ *
+ * Race definition implemented (README of the method, DESIGN.md §2 "readings"):
+ *   two access records r != s race at location λ iff
+ *     (1) they come from different threads: (block,thread) differ            P:79 (t1 != t2)
+ *     (2) at least one is a write (plain WRITE or ATOMIC)                     P:43 (§I definition)
+ *     (3) they are not both ATOMIC                                            P:573, P:447 (§VI)
+ *     (4) they are unordered: shared memory: same block and same interval
+ *         (λ fixes both); global: different blocks, or same block and same
+ *         interval                                                            P:73, P:79, P:97 (§II)
+ *     (5) lockstep mode only: not (same block, same interval, same warp, one
+ *         of them a READ)                                                     P:281 (§IV-B warp execution)
+ *     (6) not (both plain WRITE with equal value_hash)  — benign W/W          P:467 Table IV
+ *   λ = (SHARED, block, interval, granule) or (GLOBAL, granule); granule = addr / granularity;
+ *   a record of `size` bytes covers granules [addr/G, (addr+size-1)/G].     P:43 "same memory location",
+ *                                                                            P:269 "address overlapping"
+ *   kind = RW if one of them is a READ, else WW (W/W or W/A).              P:79 (WW / WR checks)
+ *   One race record per (λ, kind), witnessed by the lexicographically smallest (first, second) pair of
+ *   record indices (first < second).  The paper's witnesses are "a solution" of the solver; this
+ *   library fixes the canonical one so that results are reproducible (reading R12).
+ *   Output order: (space, block, interval, addr, kind), SHARED < GLOBAL; a global race has
+ *   block = interval = 0xFFFFFFFF.
+ *
+ * Conventions
+ *   - Every function returns sesa_status (0 == SESA_OK) unless stated.  Thread-compatible: one handle per
+ *     host thread; distinct handles may be used concurrently.
+ *   - All-or-nothing: on any error the handle's previous race list is dropped and sesa_races_get returns
+ *     SESA_ESTATE until the next successful check.  sesa_last_error() gives a one-line detail.
+ *   - Device pointers are plain CUDA device pointers (e.g. torch.Tensor.data_ptr()); streams are
+ *     cudaStream_t passed as void* (NULL = legacy default stream).
+ */
+#ifndef SESA_H
+#define SESA_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SESA_ABI_VERSION 1
+
+typedef enum {
+  SESA_OK = 0,
+  SESA_EINVAL = 1, /* bad argument, bad config, or bad record (sesa_last_error names the lowest bad index) */
+  SESA_ERANGE = 2, /* a field range does not fit the packed 64-bit sort key, or n / entries >= 2^31      */
+  SESA_ENOMEM = 3, /* device or host allocation failed                                                   */
+  SESA_ECUDA = 4,  /* a CUDA runtime error; sesa_last_error carries cudaGetErrorString                     */
+  SESA_ENCCL = 5,  /* an NCCL error (distributed handles)                                                */
+  SESA_ESTATE = 6, /* call not valid in the handle's current state (e.g. races_get with no result)      */
+  SESA_ETRUNC = 7  /* sesa_races_get: cap < number of races; cap records copied, *n_races = total       */
+} sesa_status;
+
+/* memory spaces (Fig. 3 memory sorts τl / τg; shared vs global) */
+enum { SESA_SPACE_SHARED = 0, SESA_SPACE_GLOBAL = 1 };
+/* access kinds: load -> READ, store -> WRITE (Fig. 3); any atomic RMW intrinsic -> ATOMIC */
+enum { SESA_READ = 0, SESA_WRITE = 1, SESA_ATOMIC = 2 };
+/* race kinds ("WW (Write-Write)" and "WR" checks) */
+enum { SESA_RACE_RW = 1, SESA_RACE_WW = 2 };
+
+typedef struct {
+  uint32_t warp_size;   /* >= 1.  32 = CUDA warp ("groups of 32 consecutively numbered threads");
+                           1 = no warp semantics.  warp(r) = r.thread / warp_size              */
+  uint32_t lockstep;    /* 0 | 1.  1 = exempt intra-warp pairs with a READ (R6-R8)    */
+  uint32_t granularity; /* power of two in [1, 4096]: bytes per comparison unit; 1 = exact byte overlap */
+  uint32_t flags;       /* must be 0 in ABI v1                                                          */
+} sesa_config;
+
+/* One concrete access: the paper's race-state entry `c ? r|w(a)` of one thread.
+ * 32 bytes, 8-byte aligned, array-of-structs in device memory. */
+typedef struct {
+  uint64_t addr;       /* SHARED: byte offset in the block's shared window; GLOBAL: device byte address    */
+  uint64_t value_hash; /* WRITE: 64-bit hash of the bytes written (producers fold size/offset in if writes
+                          of different sizes overlap); ignored for READ/ATOMIC                           */
+  uint32_t block;      /* linear blockIdx (x + y*gdx + z*gdx*gdy)                                    */
+  uint32_t thread;     /* linear threadIdx (x + y*bdx + z*bdx*bdy)                                   */
+  uint32_t interval;   /* number of __syncthreads the block executed before the access ("the code
+                          from the beginning to the barrier constitutes the first barrier interval" = 0) */
+  uint16_t size;       /* bytes accessed, >= 1                                                             */
+  uint8_t space;       /* SESA_SPACE_*                                                                     */
+  uint8_t rw;          /* SESA_READ / SESA_WRITE / SESA_ATOMIC                                             */
+} sesa_access;
+
+/* One race: one per (location, kind).  40 bytes. */
+typedef struct {
+  uint64_t addr;            /* granule base address = granule * granularity                              */
+  uint64_t first, second;   /* witness record indices (index_base-adjusted), first < second; lexicographic
+                               minimum over all racing pairs at this (location, kind)                      */
+  uint32_t block, interval; /* SHARED: the location's block and interval; GLOBAL: 0xFFFFFFFF, 0xFFFFFFFF  */
+  uint8_t space, kind;      /* SESA_SPACE_*, SESA_RACE_*                                                   */
+  uint8_t reserved[6];      /* zero                                                                        */
+} sesa_race;
+
+/* Parametric access descriptor: one access of one parametric flow (§IV).  The paper instantiates
+ * a flow's race history at two symbolic thread ids; sesa_expand instantiates it at EVERY thread id of every
+ * block of the flow ("replacing every occurrence of i with j").
+ *   active(t)  = (t & pmask) == pval  &&  (pmod == 0 || t % pmod == prem)  &&  plo <= t < phi  && t < nthreads
+ *                (conditional access `c(i) ? access`; flow condition)
+ *   f(t)       = t | (t + fc) % fm | t ^ fc | t >> fc | (t >> fc) * fm + (t & (2^fc - 1))
+ *                (fkind = SESA_F_ID / MODADD / XOR / SHR / ROW2D; ROW2D maps a linear tid onto a row-major
+ *                 2-D tile: ty = t >> fc, tx = t & (2^fc - 1), f = ty * fm + tx)
+ *   invalid: fkind > 4, MODADD with fm == 0, SHR/ROW2D with fc >= 32  -> SESA_EINVAL
+ *   addr       = base + bstride*block + tstride*f(t) + istride*k      (mod 2^64, signed strides), k < count
+ *   value_hash = rw != SESA_WRITE ? 0 : (flags & SESA_FLOW_CONST_VALUE) ? value_seed
+ *                : sesa_mix(sesa_mix(sesa_mix(value_seed ^ block) ^ t) ^ k)
+ *                with sesa_mix(x) = splitmix64 finaliser of (x + 0x9E3779B97F4A7C15).
+ * Output order is the paper's canonical sequential schedule: ascending block, then ascending
+ * interval, then ascending thread t, then descriptor index (program order), then k. */
+typedef struct {
+  uint64_t base;
+  int64_t bstride, tstride, istride;
+  uint64_t value_seed;
+  uint32_t block_lo, block_hi; /* blocks [block_lo, block_hi)                        */
+  uint32_t nthreads;           /* threads per block of the flow: t in [0, nthreads)  */
+  uint32_t interval;
+  uint32_t pmask, pval;
+  uint32_t pmod, prem;
+  uint32_t plo, phi;
+  uint32_t fkind, fc, fm;
+  uint32_t count;
+  uint16_t size;
+  uint8_t space, rw;
+  uint32_t flags;
+} sesa_flow; /* 104 bytes */
+
+enum { SESA_F_ID = 0, SESA_F_MODADD = 1, SESA_F_XOR = 2, SESA_F_SHR = 3, SESA_F_ROW2D = 4 };
+enum { SESA_FLOW_CONST_VALUE = 1 };
+
+typedef struct sesa_trace sesa_trace; /* opaque; owns device scratch and the last race list */
+
+/* Per-kernel timing of the last sesa_race_check (only when profiling is enabled). */
+typedef struct {
+  char name[32];        /* kernel family, e.g. "onesweep_pass"                                            */
+  uint32_t launches;    /* launches in the last check                                                      */
+  float ms;             /* summed CUDA-event time of those launches on the check's stream                  */
+  double bytes;         /* algorithmic bytes those launches must move (DESIGN.md §6 per-unit figures)       */
+} sesa_kernel_stat;
+
+typedef struct {
+  uint64_t n_records, n_entries, n_races;
+  uint32_t sort_bits, pos_bits, digit_bits, sort_passes; /* key layout chosen by the extents pass   */
+  uint32_t sorted_input;    /* records were (block, interval)-ordered                               */
+  uint32_t launches;        /* kernels launched by the last check (all families)                    */
+  uint32_t crossing_tiles;  /* conflict tiles with a location run crossing a tile boundary          */
+  uint32_t n_stats;         /* valid entries of sesa_trace_kernel_stats                             */
+} sesa_check_info;
+
+/* Create a single-GPU handle on the current CUDA device.  cfg is validated (EINVAL on warp_size 0,
+ * lockstep > 1, granularity not a power of 2 or > 4096, flags != 0).  *out = NULL on error. */
+sesa_status sesa_trace_create(const sesa_config *cfg, sesa_trace **out);
+
+/* Collective: create a handle that is rank `rank` of `world` (one process per GPU).  nccl_unique_id is the
+ * 128-byte ncclUniqueId produced by rank 0 (sesa_nccl_unique_id) and broadcast by the caller (e.g. with
+ * torch.distributed).  Records are then exchanged by location hash. */
+sesa_status sesa_trace_create_dist(const sesa_config *cfg, int rank, int world, const uint8_t nccl_unique_id[128],
+                                   sesa_trace **out);
+/* Fill a fresh ncclUniqueId (rank 0 only). */
+sesa_status sesa_nccl_unique_id(uint8_t out_id[128]);
+
+/* Race-check n records in DEVICE memory (borrowed; must stay valid until return).  Record i has global index
+ * index_base + i.  Enqueues on cuda_stream and returns when the race list is complete (it synchronises the
+ * stream).  A host pointer is EINVAL.  n == 0 is valid (no races).  Distributed handles: collective; every
+ * rank passes its shard and the exclusive prefix of shard sizes as index_base; rank 0 receives the merged
+ * list, identical to a 1-GPU check of the concatenated trace; other ranks receive 0 races. */
+sesa_status sesa_race_check(sesa_trace *t, const sesa_access *d_records, uint64_t n, uint64_t index_base,
+                            void *cuda_stream);
+
+/* Same, for records in HOST memory: the library copies them to the device (chunked through pinned staging
+ * when h_records is pageable) inside the call.  This is the end-to-end entry point. */
+sesa_status sesa_race_check_host(sesa_trace *t, const sesa_access *h_records, uint64_t n, uint64_t index_base,
+                                 void *cuda_stream);
+
+/* Copy the last race list to host memory (caller-owned).  cap == 0: only *n_races is set.  cap < count:
+ * copies cap races, sets *n_races = count, returns SESA_ETRUNC.  ESTATE when no successful check. */
+sesa_status sesa_races_get(sesa_trace *t, sesa_race *host_out, uint64_t cap, uint64_t *n_races);
+
+/* Device pointer to the last race list (owned by the handle, valid until the next check or destroy). */
+sesa_status sesa_races_device(sesa_trace *t, const sesa_race **d_races, uint64_t *n_races);
+
+/* Expand n_flows descriptors (device memory) into records at d_out (device, capacity cap records).
+ * *n_out = number of records the descriptors produce; if it exceeds cap nothing is written and SESA_ETRUNC
+ * is returned (call with cap = 0 to size the output).  Synchronises cuda_stream. */
+sesa_status sesa_expand(sesa_trace *t, const sesa_flow *d_flows, uint64_t n_flows, sesa_access *d_out, uint64_t cap,
+                        uint64_t *n_out, void *cuda_stream);
+
+/* Profiling: when enabled, every kernel of a check is bracketed by CUDA events on the check's stream. */
+sesa_status sesa_trace_set_profiling(sesa_trace *t, int enable);
+sesa_status sesa_trace_info(const sesa_trace *t, sesa_check_info *out);
+sesa_status sesa_trace_kernel_stats(const sesa_trace *t, sesa_kernel_stat *out, uint32_t cap, uint32_t *n_out);
+
+/* Tuning knob for tests: conflict-tile size exponent (0 = default).  Small tiles force location runs to
+ * cross tile boundaries so that the carry path is exercised on small traces. */
+sesa_status sesa_trace_set_tile_shift(sesa_trace *t, uint32_t conflict_tile_shift);
+
+void sesa_trace_destroy(sesa_trace *t); /* NULL-safe; frees all device scratch */
+const char *sesa_status_str(sesa_status s);
+const char *sesa_last_error(const sesa_trace *t); /* "" if none; valid until the next call on t */
+int sesa_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SESA_H */

@@ -1,0 +1,364 @@
+"""Pins for the CPU oracle (oracle/sesa_oracle.c) against what the paper and the mathematics fix.
+
+Every expected value here is either printed in the paper (cited PAPER.md line), a closed form derived in the
+test from the kernel's text, or brute force on tiny inputs; none comes from the CUDA path.
+"""
+import itertools
+
+import numpy as np
+import pytest
+
+import sesagen as G
+from oracle import oracle as O
+
+SH, GL = 0, 1
+RW, WW = 1, 2
+NOBI = 0xFFFFFFFF
+
+
+def tuples(races):
+    return O.race_tuples(races)
+
+
+def keyset(races):
+    """(λ, kind) projection: independent of record order / witnesses."""
+    return {(int(r["space"]), int(r["block"]), int(r["interval"]), int(r["addr"]), int(r["kind"])) for r in races}
+
+
+def idx_of(recs, **kw):
+    m = np.ones(len(recs), bool)
+    for k, v in kw.items():
+        m &= recs[k] == v
+    w = np.flatnonzero(m)
+    assert len(w) == 1, (kw, w)
+    return int(w[0])
+
+
+# ------------------------------------------------------------------------------------------------ layouts
+def test_layouts_agree():
+    assert O.REC_DTYPE == G.REC_DTYPE and O.RACE_DTYPE == G.RACE_DTYPE and O.FLOW_DTYPE == G.FLOW_DTYPE
+    O._load()  # asserts the C struct sizes
+
+
+# ------------------------------------------------------------------------------------------------ F1 race()
+def f1_closed_form(B=64, ls=False, distinct=True, ws=32):
+    """Expected races of race() derived by hand from P:75 (see tests/golden/f1_race.txt)."""
+    r = G.f1_race(B, distinct)
+    out = set()
+    # interval 0: v[k] written by thread k, read by thread k-1 (mod B): one RW per k (t1=k, t2=k-1).
+    for k in range(B):
+        w, rd = k, (k - 1) % B
+        if ls and w // ws == rd // ws:
+            continue
+        i = idx_of(r, thread=w, interval=0, rw=1)
+        j = idx_of(r, thread=rd, interval=0, rw=0)
+        out.add((SH, 0, 0, 4 * k, RW, min(i, j), max(i, j)))
+    # interval 1: odd t writes v[t>>2]; even t reads v[t].  v[j] (j < B/4) has writers 4j+1, 4j+3.
+    for j in range(B // 4):
+        writers = [t for t in (4 * j + 1, 4 * j + 3) if t < B]
+        widx = sorted(idx_of(r, thread=t, interval=1, rw=1) for t in writers)
+        if distinct and len(writers) == 2:  # WW, no warp exemption for write-write (reading R7)
+            out.add((SH, 0, 1, 4 * j, WW, widx[0], widx[1]))
+        if j % 2 == 0:  # reader thread j (even) reads v[j]
+            ridx = idx_of(r, thread=j, interval=1, rw=0)
+            racing = [idx_of(r, thread=t, interval=1, rw=1) for t in writers if not (ls and t // ws == j // ws)]
+            if racing:
+                cands = sorted((min(ridx, w), max(ridx, w)) for w in racing)
+                out.add((SH, 0, 1, 4 * j, RW) + cands[0])
+    return out
+
+
+@pytest.mark.parametrize("method", ["brute", "grouped"])
+def test_f1_paper_witnesses(method):
+    r = G.f1_race()
+    got = tuples(O.check(r, method=method))
+    # first interval, WR race on v[0], witness t1.x = 0 (writes v[0]) and t2.x = bdim.x - 1 (reads it)
+    i0 = idx_of(r, thread=0, interval=0, rw=1)
+    i63 = idx_of(r, thread=63, interval=0, rw=0)
+    assert (SH, 0, 0, 0, RW, i0, i63) in got
+    # second interval, RW race, e.g. t1.x = 0 (then-part read of v[0]) and t2.x = 1 (else-part write
+    # v[1 >> 2] = v[0]); it happens "no matter whether t1 and t2 are within a warp" -> lockstep off.
+    a = idx_of(r, thread=0, interval=1, rw=0)
+    b = idx_of(r, thread=1, interval=1, rw=1)
+    assert (SH, 0, 1, 0, RW, a, b) in got
+
+
+@pytest.mark.parametrize("method", ["brute", "grouped"])
+@pytest.mark.parametrize("ls", [0, 1])
+@pytest.mark.parametrize("distinct", [True, False])
+def test_f1_closed_form(method, ls, distinct):
+    got = set(tuples(O.check(G.f1_race(distinct=distinct), lockstep=ls, method=method)))
+    assert got == f1_closed_form(ls=bool(ls), distinct=distinct)
+    # counts quoted in DESIGN.md (88 / 22 / 72)
+    if not ls:
+        assert len(got) == (88 if distinct else 72)
+    elif distinct:
+        assert len(got) == 22
+
+
+def test_f1_golden_file():
+    """tests/golden/f1_race.txt was written by tests/golden/make_golden.py (oracle only) and is checked
+    here against the closed form, so the stored file is pinned by the paper's kernel text."""
+    rows = set()
+    for line in open("tests/golden/f1_race.txt"):
+        if line.startswith("#") or not line.strip():
+            continue
+        rows.add(tuple(int(x) for x in line.split()))
+    assert rows == f1_closed_form()
+
+
+# ------------------------------------------------------------------------------------------------ F2 / F3
+@pytest.mark.parametrize("method", ["brute", "grouped"])
+def test_f2_reduction_race_free(method):
+    # the WW and RW queries of the reduction interval are unsat -> no race
+    r = G.f2_reduction()
+    assert len(r) == 189
+    for ls in (0, 1):
+        assert len(O.check(r, lockstep=ls, method=method)) == 0
+
+
+@pytest.mark.parametrize("B", [16, 32, 64, 128, 256])
+def test_f3_bitonic_race_free(B):
+    # Table II: bitonic2.0 reports no races (RR column "-") at #T = 16 ... 256
+    r = G.f3_bitonic(B)
+    assert len(O.check(r)) == 0
+    if B <= 64:
+        assert len(O.check(r, method="brute")) == 0
+
+
+def test_f3_bitonic_mutant_races():
+    # deleting the barrier between two steps (merging intervals) must produce races: sanity of the fixture
+    r = G.f3_bitonic(32)
+    r2 = r.copy()
+    r2["interval"] = np.where(r2["interval"] == 3, 2, r2["interval"])
+    assert len(O.check(r2)) > 0
+
+
+# ------------------------------------------------------------------------------------------------ F4 prescan
+@pytest.mark.parametrize("method", ["grouped", "brute"])
+def test_f4_histo_prescan(method):
+    r = G.f4_histo_prescan()
+    got = tuples(O.check(r, method=method))
+    # closed form: SUM(32) writes Avg/StdDev[16..31] (threads 16..31), SUM(16) in the same interval reads
+    # them (threads 0..15 read [t+16]): 16 + 16 RW races, nothing else (each [0..15] is touched by its own
+    # thread only, [32..63] only read).
+    assert len(got) == 32
+    assert {(x[0], x[2], x[3], x[4]) for x in got} == {(SH, 4, base + 4 * k, RW)
+                                                       for base in (0, G.F4_STD) for k in range(16, 32)}
+    # the write in SUM(stride) by thread <17,0,0> races with the read in SUM(16) by thread <1,0,0>
+    w17 = idx_of(r, thread=17, interval=4, rw=1, addr=4 * 17)
+    r1 = np.flatnonzero((r["thread"] == 1) & (r["addr"] == 4 * 17) & (r["rw"] == 0))
+    assert len(r1) == 1
+    assert (SH, 0, 4, 4 * 17, RW, int(r1[0]), w17) in got
+    # lockstep: all participants of the last interval are threads < 32 = warp 0 -> the warp-synchronous
+    # idiom is exempt (refs [25], [26])
+    assert len(O.check(r, lockstep=1, method=method)) == 0
+    # but with warp size 1 the race is reported even in lockstep mode
+    assert len(O.check(r, lockstep=1, warp_size=1, method=method)) == 32
+
+
+# ------------------------------------------------------------------------------------------------ F5 binning
+def test_f5_binning():
+    r = G.f5_binning()
+    assert len(r) == 3 * 16896  # Table IV: 16,896 threads
+    got = tuples(O.check(r))
+    i_r = idx_of(r, block=0, thread=0, rw=0, addr=G.F5_BINCOUNT)
+    i_a = idx_of(r, block=0, thread=1, rw=2)
+    # exactly one race: RW at binCount_g[0]; atomic-atomic pairs excluded; sample reads unique
+    assert got == [(GL, NOBI, NOBI, G.F5_BINCOUNT, RW, i_r, i_a)]
+    # the paper's witness (thread bid 32 tid 64 reads, bid 0 tid 0 atomicAdds) is a racing pair
+    p = r[idx_of(r, block=32, thread=64, rw=0, addr=G.F5_BINCOUNT)]
+    q = r[idx_of(r, block=0, thread=0, rw=2)]
+    assert O.pair_kind(p, q) == RW
+    got1 = tuples(O.check(r, lockstep=1))
+    assert got1 == [(GL, NOBI, NOBI, G.F5_BINCOUNT, RW, i_r, idx_of(r, block=0, thread=32, rw=2))]
+
+
+# ------------------------------------------------------------------------------------------------ C1
+def test_c1_truth_by_construction():
+    r = G.c1()
+    assert len(r) == 959
+    for method in ("brute", "grouped"):
+        assert tuples(O.check(r, method=method)) == [(SH, 0, 5, 4, WW, 833, 836)]
+
+
+# ------------------------------------------------------------------------------------------------ expansion
+@pytest.mark.parametrize("name", ["f1", "f1c", "f2", "f5", "c1"])
+def test_expand_matches_direct(name):
+    direct, fl = {
+        "f1": (G.f1_race(), G.f1_flows()),
+        "f1c": (G.f1_race(distinct=False), G.f1_flows(distinct=False)),
+        "f2": (G.f2_reduction(), G.f2_flows()),
+        "f5": (G.f5_binning(), G.f5_flows()),
+        "c1": (G.c1(), G.c1_flows()),
+    }[name]
+    ex = O.expand(fl)
+    assert len(ex) == len(direct)
+    assert ex.tobytes() == direct.tobytes()
+
+
+def test_expand_c2_counts_and_race_free():
+    fl = G.c2_flows(gx=2, gy=2, K=64)
+    ex = O.expand(fl)
+    per_thread = 4 + 36 * (64 // 16 - 1) + 33
+    assert len(ex) == 4 * 256 * per_thread
+    assert len(O.check(ex)) == 0
+    mut = O.expand(G.c2_mutant_flows(drop_barrier=2, gx=2, gy=2, K=64))
+    assert len(O.check(mut)) > 0
+
+
+def test_expand_full_c2_count():
+    assert len(G.c2_flows()) == 628
+    # 16,384 threads x 1,117 records: count without materialising through the C loop
+    import ctypes
+    lib = O._load()
+    f = np.ascontiguousarray(G.c2_flows())
+    n = lib.oracle_expand(f.ctypes.data, len(f), None, 0)
+    assert n == 16384 * 1117 == 18300928
+
+
+# ------------------------------------------------------------------------------------------------ brute == grouped
+CONFIGS = [dict(ws=32, ls=0, G=4), dict(ws=32, ls=1, G=4), dict(ws=4, ls=1, G=1), dict(ws=1, ls=1, G=2),
+           dict(ws=2, ls=0, G=8), dict(ws=8, ls=1, G=16)]
+
+
+@pytest.mark.parametrize("cfg", CONFIGS)
+def test_brute_equals_grouped_random(cfg):
+    for seed in range(60):
+        n = 1 + (seed * 7) % 90
+        r = G.random_trace(n, seed, threads=12 + seed % 50, sort=seed % 3 != 0)
+        a = O.check(r, warp_size=cfg["ws"], lockstep=cfg["ls"], granularity=cfg["G"], method="brute")
+        b = O.check(r, warp_size=cfg["ws"], lockstep=cfg["ls"], granularity=cfg["G"], method="grouped")
+        assert a.tobytes() == b.tobytes(), (cfg, seed)
+
+
+def test_index_base_shifts_witnesses():
+    r = G.f1_race()
+    a = O.check(r)
+    b = O.check(r, index_base=1000)
+    assert np.array_equal(a["first"] + 1000, b["first"]) and np.array_equal(a["second"] + 1000, b["second"])
+
+
+# ------------------------------------------------------------------------------------------------ invariants
+def _rand(seed, n=70):
+    return G.random_trace(n, seed, threads=40)
+
+
+@pytest.mark.parametrize("seed", range(25))
+def test_invariants(seed):
+    r = _rand(seed)
+    base = O.check(r)
+    # witness validity: P(first, second) holds with the race's kind, both records cover the location
+    for x in base:
+        a, b = r[int(x["first"])], r[int(x["second"])]
+        assert O.pair_kind(a, b) == x["kind"]
+        for q in (a, b):
+            assert q["space"] == x["space"]
+            assert q["addr"] // 4 <= x["addr"] // 4 <= (int(q["addr"]) + int(q["size"]) - 1) // 4
+            if x["space"] == SH:
+                assert (q["block"], q["interval"]) == (x["block"], x["interval"])
+    # lockstep only removes races
+    assert keyset(O.check(r, lockstep=1)) <= keyset(base)
+    # warp size 1 makes lockstep a no-op
+    assert O.check(r, warp_size=1, lockstep=1).tobytes() == O.check(r, warp_size=1).tobytes()
+    # permutation invariance of the (λ, kind) projection
+    rng = np.random.default_rng(seed)
+    assert keyset(O.check(r[rng.permutation(len(r))])) == keyset(base)
+    # monotonicity: adding records never removes a (λ, kind)... except benign/ordering are pairwise, so it holds
+    extra = _rand(seed + 1000, 20)
+    assert keyset(base) <= keyset(O.check(np.concatenate([r, extra])))
+    # the witness is the lexicographic minimum: no racing pair at (λ, K) is smaller (brute enumeration)
+    for x in base:
+        lam = (x["space"], x["block"], x["interval"], x["addr"] // 4)
+        for i, j in itertools.combinations(range(int(x["second"]) + 1), 2):
+            if (i, j) >= (int(x["first"]), int(x["second"])):
+                continue
+            a, b = r[i], r[j]
+            cover = all(q["space"] == lam[0] and q["addr"] // 4 <= lam[3] <= (int(q["addr"]) + int(q["size"]) - 1) // 4
+                        and (q["space"] == GL or (q["block"], q["interval"]) == (lam[1], lam[2])) for q in (a, b))
+            assert not (cover and O.pair_kind(a, b) == x["kind"])
+
+
+def test_all_writes_distinct_values_closed_form():
+    """One block, one interval, every record a plain write by its own thread with a distinct value: every
+    granule touched by >= 2 records is a WW race witnessed by its two lowest record indices."""
+    rng = np.random.default_rng(7)
+    n = 300
+    r = np.zeros(n, G.REC_DTYPE)
+    r["thread"] = np.arange(n)
+    r["rw"] = 1
+    r["space"] = SH
+    r["size"] = 4
+    r["addr"] = 4 * rng.integers(0, 90, n)
+    r["value_hash"] = np.arange(n) + 1
+    exp = []
+    for w in sorted(set(r["addr"].tolist())):
+        ids = np.flatnonzero(r["addr"] == w)
+        if len(ids) >= 2:
+            exp.append((SH, 0, 0, w, WW, int(ids[0]), int(ids[1])))
+    assert tuples(O.check(r)) == exp
+    # same values everywhere: all benign (Table IV "W/W (Benign)")
+    r["value_hash"] = 5
+    assert len(O.check(r)) == 0
+
+
+def test_global_ordering_rule():
+    """Same block, different intervals of global memory: ordered by __syncthreads (reading R2); different
+    blocks: unordered."""
+    rows = [(0x1000, 1, 0, 0, 0, 4, GL, 1),   # b0 t0 iv0 W
+            (0x1000, 0, 0, 1, 1, 4, GL, 0),   # b0 t1 iv1 R   -> ordered after the barrier, no race
+            (0x2000, 1, 0, 0, 0, 4, GL, 1),   # b0 t0 iv0 W
+            (0x2000, 0, 1, 1, 1, 4, GL, 0),   # b1 t1 iv1 R   -> other block: race
+            (0x3000, 0, 0, 0, 0, 4, GL, 1),   # b0 t0 iv0 W
+            (0x3000, 0, 0, 0, 1, 4, GL, 0)]   # same thread, any interval: never a race
+    got = tuples(O.check(G.recs(rows)))
+    assert got == [(GL, NOBI, NOBI, 0x2000, RW, 2, 3)]
+
+
+def test_atomics_and_benign_rules():
+    rows = [(0x10, 0, 0, 0, 0, 4, GL, 2), (0x10, 0, 1, 0, 0, 4, GL, 2),      # A-A: never
+            (0x20, 9, 0, 0, 0, 4, GL, 1), (0x20, 0, 1, 0, 0, 4, GL, 2),      # W-A: WW (A never benign)
+            (0x30, 9, 0, 0, 0, 4, GL, 1), (0x30, 9, 1, 0, 0, 4, GL, 1),      # W-W same value: benign
+            (0x40, 9, 0, 0, 0, 4, GL, 1), (0x40, 8, 1, 0, 0, 4, GL, 1),      # W-W different values: WW
+            (0x50, 0, 0, 0, 0, 4, GL, 0), (0x50, 0, 1, 0, 0, 4, GL, 2)]      # R-A: RW
+    got = tuples(O.check(G.recs(rows)))
+    assert got == [(GL, NOBI, NOBI, 0x20, WW, 2, 3), (GL, NOBI, NOBI, 0x40, WW, 6, 7),
+                   (GL, NOBI, NOBI, 0x50, RW, 8, 9)]
+
+
+def test_granularity_byte_overlap():
+    # G = 1: a 4-byte write at 0x100 and a 1-byte read at 0x103 overlap in byte 0x103 only
+    rows = [(0x100, 1, 0, 0, 0, 4, GL, 1), (0x103, 0, 1, 0, 0, 1, GL, 0), (0x104, 0, 2, 0, 0, 1, GL, 0)]
+    got = tuples(O.check(G.recs(rows), granularity=1))
+    assert got == [(GL, NOBI, NOBI, 0x103, RW, 0, 1)]
+    # G = 8: all three share granule 0x100/8 = 0x20
+    got8 = tuples(O.check(G.recs(rows), granularity=8))
+    assert got8 == [(GL, NOBI, NOBI, 0x100, RW, 0, 1)]
+
+
+# ------------------------------------------------------------------------------------------------ validation
+def test_validation_lowest_bad_index():
+    r = G.f1_race()
+    r[40]["rw"] = 3
+    r[17]["size"] = 0
+    assert O.validate(r) == 17
+    with pytest.raises(O.OracleError) as e:
+        O.check(r)
+    assert e.value.code == 1 and e.value.detail == 17
+    r2 = G.f1_race()
+    r2[5]["addr"] = 2**64 - 2  # addr + size - 1 wraps
+    assert O.validate(r2) == 5
+    r3 = G.f1_race()
+    r3[9]["space"] = 2
+    assert O.validate(r3) == 9
+
+
+def test_bad_config():
+    r = G.f1_race()
+    for kw in (dict(warp_size=0), dict(lockstep=2), dict(granularity=3), dict(granularity=8192)):
+        with pytest.raises(O.OracleError):
+            O.check(r, **kw)
+
+
+def test_empty():
+    assert len(O.check(np.zeros(0, G.REC_DTYPE))) == 0
