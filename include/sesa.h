@@ -197,9 +197,9 @@ sesa_status sesa_trace_set_profiling(sesa_trace *t, int enable);
 sesa_status sesa_trace_info(const sesa_trace *t, sesa_check_info *out);
 sesa_status sesa_trace_kernel_stats(const sesa_trace *t, sesa_kernel_stat *out, uint32_t cap, uint32_t *n_out);
 
-/* Tuning knob for tests: conflict-tile size exponent (0 = default).  Small tiles force location runs to
- * cross tile boundaries so that the carry path is exercised on small traces. */
-sesa_status sesa_trace_set_tile_shift(sesa_trace *t, uint32_t conflict_tile_shift);
+
+
+
 
 void sesa_trace_destroy(sesa_trace *t); /* NULL-safe; frees all device scratch */
 const char *sesa_status_str(sesa_status s);

@@ -1,0 +1,804 @@
+// k_conflict.cu — segmented conflict detection over the sorted entries (SURVEY §8a rows a5 + a6).
+//
+// After the sort, every location λ is one contiguous run ("group") of keys; for a global location the entries
+// of one (block, interval) are a contiguous "sub-run".  The paper instantiates a barrier interval's read/write
+// sets at two thread ids t1 != t2 and asks the solver whether an address can coincide.
+// Concretely that is: does entry e have a partner s in its group with P(e, s) (include/sesa.h rules 1-6)?
+// We answer it without enumerating pairs, from per-group and per-sub-run summaries ("Agg"):
+//   per access type X in {READ, WRITE, ATOMIC}: min/max identity  (identity = thread in a sub-run, block in a
+//   group) -> "exists an X with identity != mine" / "exists an X in another warp" (lockstep);
+//   for plain writes: min and max value hash with the identity attaining them, plus the min (max) over the
+//   OTHER identities -> "exists a write with identity != mine AND value != mine" (benign W/W filter).
+// flag_K(e) = partner of kind K exists; witness x_K = min flagged position of the group, y_K = min position s
+// with P(x_K, s) of kind K (lexicographic minimum, reading R12).
+//
+// A CTA owns a tile of 2048 sorted entries.  Summaries are computed with a per-thread fold over its 8 entries
+// plus block-wide segmented scans of the per-thread folds (warp shuffles), forward and backward, so each entry
+// receives the total of its segment without storing per-entry summaries.  Runs that cross a tile boundary
+// (hot locations: C3 bins, C4 `changed`) are completed in three extra steps:
+//   mode 1 (every tile): internal groups -> races; crossing pieces -> per-tile partial summaries
+//   carry  (k_carry)    : segmented scans over the tile partials -> full incoming/outgoing summaries
+//   mode 2 (crossing tiles): exact flags of crossing entries -> atomicMin x into the owner tile's slot
+//   mode 3 (crossing tiles): atomicMin y;  cross_emit: one race per (crossing group, kind)
+// Only entries of groups with >= 2 entries gather their 32-byte record (by position); singletons — all but
+// 2e5 of C5's 1e9 entries — cost 8 bytes of key traffic.
+#include "kernels.cuh"
+
+namespace sesa {
+
+// ------------------------------------------------------------------------------------------------ summaries
+__device__ __forceinline__ Agg agg_empty() {
+  Agg r;
+#pragma unroll
+  for (int x = 0; x < 3; x++) r.mn[x] = ~0u, r.mx[x] = 0u;
+  r.i1 = r.i2 = ~0u;
+  r.v1 = r.v1b = ~0ull;
+  r.v2 = r.v2b = 0ull;
+  return r;
+}
+
+__device__ __forceinline__ Agg agg_item(u32 rw, u32 id, u64 vh) {
+  Agg r = agg_empty();
+  r.mn[rw] = r.mx[rw] = id;
+  if (rw == RW_WRITE) {
+    r.v1 = r.v2 = vh;
+    r.i1 = r.i2 = id;
+  }
+  return r;
+}
+
+__device__ __forceinline__ Agg agg_merge(const Agg& a, const Agg& b) {
+  Agg r;
+#pragma unroll
+  for (int x = 0; x < 3; x++) r.mn[x] = min(a.mn[x], b.mn[x]), r.mx[x] = max(a.mx[x], b.mx[x]);
+  const bool ae = a.mn[RW_WRITE] > a.mx[RW_WRITE], be = b.mn[RW_WRITE] > b.mx[RW_WRITE];
+  if (ae || be) {
+    const Agg& s = ae ? b : a;
+    r.i1 = s.i1, r.i2 = s.i2, r.v1 = s.v1, r.v1b = s.v1b, r.v2 = s.v2, r.v2b = s.v2b;
+    return r;
+  }
+  if (b.v1 < a.v1) {
+    r.v1 = b.v1, r.i1 = b.i1;
+    r.v1b = min(b.v1b, a.i1 != b.i1 ? a.v1 : a.v1b);
+  } else {
+    r.v1 = a.v1, r.i1 = a.i1;
+    r.v1b = min(a.v1b, b.i1 != a.i1 ? b.v1 : b.v1b);
+  }
+  if (b.v2 > a.v2) {
+    r.v2 = b.v2, r.i2 = b.i2;
+    r.v2b = max(b.v2b, a.i2 != b.i2 ? a.v2 : a.v2b);
+  } else {
+    r.v2 = a.v2, r.i2 = a.i2;
+    r.v2b = max(a.v2b, b.i2 != a.i2 ? b.v2 : b.v2b);
+  }
+  return r;
+}
+
+// "exists an entry of type X with identity != id"
+__device__ __forceinline__ bool ex_id(const Agg& S, int X, u32 id) { return S.mn[X] < id || S.mx[X] > id; }
+// "exists an entry of type X in another warp" (warp = thread / ws)
+__device__ __forceinline__ bool ex_warp(const Agg& S, int X, u32 w, u32 ws) {
+  return S.mn[X] <= S.mx[X] && (S.mn[X] / ws < w || S.mx[X] / ws > w);
+}
+// "exists a plain write with identity != id and value != v"
+__device__ __forceinline__ bool ex_wval(const Agg& S, u32 id, u64 v) {
+  if (!ex_id(S, RW_WRITE, id)) return false;
+  const u64 lo = S.i1 != id ? S.v1 : S.v1b;
+  const u64 hi = S.i2 != id ? S.v2 : S.v2b;
+  return lo != v || hi != v;
+}
+
+struct OpAgg {
+  __device__ __forceinline__ Agg operator()(const Agg& a, const Agg& b) const { return agg_merge(a, b); }
+};
+
+struct X2 {
+  u64 v[2];
+};
+struct OpX2 {
+  __device__ __forceinline__ X2 operator()(const X2& a, const X2& b) const {
+    X2 r;
+    r.v[0] = min(a.v[0], b.v[0]);
+    r.v[1] = min(a.v[1], b.v[1]);
+    return r;
+  }
+};
+
+// min of each 32-bit half independently (x in the low half, y in the high half)
+struct OpXY {
+  __device__ __forceinline__ X2 operator()(const X2& a, const X2& b) const {
+    X2 r;
+#pragma unroll
+    for (int k = 0; k < 2; k++) {
+      const u64 hi = min(a.v[k] >> 32, b.v[k] >> 32), lo = min(a.v[k] & 0xFFFFFFFFull, b.v[k] & 0xFFFFFFFFull);
+      r.v[k] = (hi << 32) | lo;
+    }
+    return r;
+  }
+};
+
+// ------------------------------------------------------------------------------------------------ shuffles
+__device__ __forceinline__ u32 shfl(u32 v, int o, bool down) {
+  return down ? __shfl_down_sync(~0u, v, o) : __shfl_up_sync(~0u, v, o);
+}
+__device__ __forceinline__ u64 shfl(u64 v, int o, bool down) {
+  return down ? __shfl_down_sync(~0u, v, o) : __shfl_up_sync(~0u, v, o);
+}
+__device__ __forceinline__ Agg shfl(const Agg& a, int o, bool down) {
+  Agg r;
+#pragma unroll
+  for (int x = 0; x < 3; x++) r.mn[x] = shfl(a.mn[x], o, down), r.mx[x] = shfl(a.mx[x], o, down);
+  r.i1 = shfl(a.i1, o, down), r.i2 = shfl(a.i2, o, down);
+  r.v1 = shfl(a.v1, o, down), r.v1b = shfl(a.v1b, o, down);
+  r.v2 = shfl(a.v2, o, down), r.v2b = shfl(a.v2b, o, down);
+  return r;
+}
+__device__ __forceinline__ X2 shfl(const X2& a, int o, bool down) {
+  X2 r;
+  r.v[0] = shfl(a.v[0], o, down);
+  r.v[1] = shfl(a.v[1], o, down);
+  return r;
+}
+
+// Block-wide exclusive segmented scan of per-thread (flag, value): flag = "a segment starts inside this
+// thread's span" (in scan direction).  REV = backward (from the last thread).  carry seeds the first thread.
+template <class T, class Op, bool REV, int THREADS>
+__device__ __forceinline__ T block_seg_excl(bool flag, const T& val, const T& carry, Op op, T* s_wv, u8* s_wf) {
+  constexpr int WARPS = THREADS / 32;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  bool f = flag;
+  T v = val;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const bool f2 = __shfl_sync(~0u, (u32)f, REV ? lane + o : lane - o) != 0;
+    const T v2 = shfl(v, o, REV);
+    const bool has = REV ? lane + o < 32 : lane >= o;
+    if (has) {
+      if (!f) v = op(v2, v);
+      f = f || f2;
+    }
+  }
+  const bool fe = __shfl_sync(~0u, (u32)f, REV ? lane + 1 : lane - 1) != 0;
+  const T ve = shfl(v, 1, REV);
+  if (REV ? lane == 0 : lane == 31) {
+    s_wv[warp] = v;
+    s_wf[warp] = f;
+  }
+  __syncthreads();
+  T wp = carry;
+  if (!REV) {
+    for (int w = 0; w < warp; w++) wp = s_wf[w] ? s_wv[w] : op(wp, s_wv[w]);
+  } else {
+    for (int w = WARPS - 1; w > warp; w--) wp = s_wf[w] ? s_wv[w] : op(wp, s_wv[w]);
+  }
+  const bool first = REV ? lane == 31 : lane == 0;
+  T ex = first ? wp : (fe ? ve : op(wp, ve));
+  __syncthreads();
+  return ex;
+}
+
+// Segmented all-reduce over the tile (blocked: thread t owns items t*ITEMS .. t*ITEMS+ITEMS-1): calls
+// cb(j, total of j's segment) for every item.  Segment starts/ends are bits hbit/tbit of fl[j].
+template <class T, class Op, class ItemF, class CB>
+__device__ __forceinline__ void tile_allreduce(const u8* fl, u8 hbit, u8 tbit, ItemF item, Op op, const T& ident,
+                                               const T& carry_in, const T& carry_out, CB cb, T* s_wv, u8* s_wf) {
+  const int j0 = threadIdx.x * CT_ITEMS;
+  // per-thread folds: F = from the last head to the end, B = from the start to the first tail
+  T F = ident, B = ident;
+  bool ff = false, bf = false;
+#pragma unroll
+  for (int q = 0; q < CT_ITEMS; q++) {
+    const int j = j0 + q;
+    const T it = item(j);
+    if (fl[j] & hbit) F = it, ff = true;
+    else F = op(F, it);
+  }
+#pragma unroll
+  for (int q = CT_ITEMS - 1; q >= 0; q--) {
+    const int j = j0 + q;
+    const T it = item(j);
+    if (fl[j] & tbit) B = it, bf = true;
+    else B = op(it, B);
+  }
+  const T Ef = block_seg_excl<T, Op, false, CT_THREADS>(ff, F, carry_in, op, s_wv, s_wf);
+  const T Eb = block_seg_excl<T, Op, true, CT_THREADS>(bf, B, carry_out, op, s_wv, s_wf);
+  int q = 0;
+  while (q < CT_ITEMS) {
+    T tot = (q == 0 && !(fl[j0] & hbit)) ? Ef : ident;
+    int e = q;
+    while (true) {
+      tot = op(tot, item(j0 + e));
+      const bool t = fl[j0 + e] & tbit;
+      e++;
+      if (t || e == CT_ITEMS) break;
+    }
+    if (!(fl[j0 + e - 1] & tbit)) tot = op(tot, Eb);
+    for (int r = q; r < e; r++) cb(j0 + r, tot);
+    q = e;
+  }
+}
+
+// ------------------------------------------------------------------------------------------------ pair rule
+struct F5 {
+  u32 block, interval, thread, rw;
+  u64 vh;
+};
+
+// P(x, s) of include/sesa.h for two entries at the same location; 0 = no race
+__device__ __forceinline__ u32 pair_kind(const F5& x, const F5& s, u32 ws, u32 ls) {
+  if (x.block == s.block && x.thread == s.thread) return 0;                  // (1) t1 != t2
+  if (x.rw == RW_READ && s.rw == RW_READ) return 0;                           // (2) a write
+  if (x.rw == RW_ATOMIC && s.rw == RW_ATOMIC) return 0;                       // (3) not both atomic
+  if (x.block == s.block && x.interval != s.interval) return 0;               // (4) ordered by a barrier
+  const u32 kind = (x.rw == RW_READ || s.rw == RW_READ) ? KIND_RW : KIND_WW;
+  if (ls && kind == KIND_RW && x.block == s.block && x.interval == s.interval && x.thread / ws == s.thread / ws)
+    return 0;                                                                 // (5) lockstep warp
+  if (x.rw == RW_WRITE && s.rw == RW_WRITE && x.vh == s.vh) return 0;         // (6) benign W/W
+  return kind;
+}
+
+// ------------------------------------------------------------------------------------------------ tile state
+enum : u8 { FL_GH = 1, FL_GT = 2, FL_SH = 4, FL_ST = 8, FL_INT = 16 };
+enum : u8 { TF_GH = 1, TF_GT = 2, TF_SH = 4, TF_ST = 8, TF_CIN = 16, TF_COUT = 32 };
+
+struct TileSmem {
+  u64 key[CT_TILE + 2];  // [0] = previous entry, [j+1] = item j, [cnt+1] = next entry
+  u32 blk[CT_TILE + 2];
+  u32 ivl[CT_TILE + 2];
+  u32 thr[CT_TILE];
+  u64 vh[CT_TILE];
+  u32 xy[CT_TILE][2];  // mode 1: x of tail items, then y candidates
+  u8 rw[CT_TILE];
+  u8 fl[CT_TILE];
+  u8 gq[CT_TILE];
+  u8 res[CT_TILE];
+  Agg wv[CT_THREADS / 32];
+  X2 wx[CT_THREADS / 32];
+  u8 wf[CT_THREADS / 32];
+  int any, first_gtail, last_ghead;
+};
+
+__device__ __forceinline__ u32 pos_of(const KeyLayout& L, u64 key) { return (u32)(key & lowmask(L.pos_bits)); }
+
+// Loads keys, computes group membership and gathers records.  Returns false if no entry of the tile has a
+// partner candidate (all singletons).
+__device__ bool tile_load(const ConflictArgs& a, TileSmem& s, u64 tb, u32 cnt) {
+  const KeyLayout& L = a.L;
+  const int tid = threadIdx.x;
+  for (u32 j = tid; j < cnt; j += CT_THREADS) s.key[j + 1] = __ldcs(a.keys + tb + j);
+  if (tid == 0) {
+    s.key[0] = tb > 0 ? a.keys[tb - 1] : 0ull;
+    s.key[cnt + 1] = tb + cnt < a.m ? a.keys[tb + cnt] : 0ull;
+    s.any = 0;
+    s.first_gtail = CT_TILE;
+    s.last_ghead = -1;
+  }
+  __syncthreads();
+  const int j0 = tid * CT_ITEMS;
+  bool any = false;
+#pragma unroll
+  for (int q = 0; q < CT_ITEMS; q++) {
+    const int j = j0 + q;
+    u8 f = FL_GH | FL_GT;
+    if (j < (int)cnt) {
+      const u64 g = group_of_hi(L, s.key[j + 1] >> L.pos_bits);
+      const bool sp = (j > 0 || tb > 0) && group_of_hi(L, s.key[j] >> L.pos_bits) == g;
+      const bool sn = (j + 1 < (int)cnt || tb + cnt < a.m) && group_of_hi(L, s.key[j + 2] >> L.pos_bits) == g;
+      f = (sp ? 0 : FL_GH) | (sn ? 0 : FL_GT) | ((sp || sn) ? FL_INT : 0);
+      any |= sp || sn;
+    }
+    s.fl[j] = f;
+  }
+  if (!__syncthreads_or(any)) return false;
+  // gather the records of entries in multi-entry groups (one 32-byte sector each)
+#pragma unroll
+  for (int q = 0; q < CT_ITEMS; q++) {
+    const int j = j0 + q;
+    if (s.fl[j] & FL_INT) {
+      const Rec r = load_rec(a.rec + pos_of(L, s.key[j + 1]));
+      s.blk[j + 1] = r.block;
+      s.ivl[j + 1] = r.interval;
+      s.thr[j] = r.thread;
+      s.rw[j] = r.rw;
+      s.vh[j] = r.vh;
+    }
+  }
+  if (tid == 0 && !(s.fl[0] & FL_GH)) {  // previous entry is in item 0's group: need its (block, interval)
+    const Rec r = load_rec(a.rec + pos_of(L, s.key[0]));
+    s.blk[0] = r.block, s.ivl[0] = r.interval;
+  }
+  if (tid == CT_THREADS - 1 && !(s.fl[cnt - 1] & FL_GT)) {
+    const Rec r = load_rec(a.rec + pos_of(L, s.key[cnt + 1]));
+    s.blk[cnt + 1] = r.block, s.ivl[cnt + 1] = r.interval;
+  }
+  __syncthreads();
+  // sub-runs: a new (block, interval) inside a group (contiguous: input order is (block, interval) order)
+#pragma unroll
+  for (int q = 0; q < CT_ITEMS; q++) {
+    const int j = j0 + q;
+    u8 f = s.fl[j];
+    if (f & FL_INT) {
+      const bool sh = (f & FL_GH) || s.blk[j] != s.blk[j + 1] || s.ivl[j] != s.ivl[j + 1];
+      const bool st = (f & FL_GT) || s.blk[j + 2] != s.blk[j + 1] || s.ivl[j + 2] != s.ivl[j + 1];
+      f |= (sh ? FL_SH : 0) | (st ? FL_ST : 0);
+    } else {
+      f |= FL_SH | FL_ST;
+    }
+    s.fl[j] = f;
+    if (j < (int)cnt) {
+      if (f & FL_GT) atomicMin(&s.first_gtail, j);
+      if (f & FL_GH) atomicMax(&s.last_ghead, j);
+    }
+  }
+  __syncthreads();
+  return true;
+}
+
+// group- and sub-run-level summaries -> s.res[j] = bit0 RW partner, bit1 WW partner.  In mode 1 also returns
+// the tile-edge partial summaries (P = item 0's segment, S = item cnt-1's segment) per level.
+__device__ void tile_flags(const ConflictArgs& a, TileSmem& s, u32 cnt, const Agg cin[2], const Agg cout[2],
+                           Agg* part /* [4] or null */) {
+  const u32 ws = a.ws, ls = a.ls;
+  const Agg E = agg_empty();
+  // group level (identity = block): "another block" queries -> s.gq
+  tile_allreduce<Agg>(
+      s.fl, FL_GH, FL_GT,
+      [&](int j) { return (s.fl[j] & FL_INT) ? agg_item(s.rw[j], s.blk[j + 1], s.vh[j]) : E; }, OpAgg(), E, cin[0],
+      cout[0],
+      [&](int j, const Agg& R) {
+        if (part && j == 0) part[0] = R;
+        if (part && j == (int)cnt - 1) part[1] = R;
+        if (!(s.fl[j] & FL_INT)) return;
+        const u32 b = s.blk[j + 1];
+        u8 g = (ex_id(R, RW_READ, b) ? 1 : 0) | (ex_id(R, RW_WRITE, b) ? 2 : 0) | (ex_id(R, RW_ATOMIC, b) ? 4 : 0);
+        if (s.rw[j] == RW_WRITE && ex_wval(R, b, s.vh[j])) g |= 8;
+        s.gq[j] = g;
+      },
+      s.wv, s.wf);
+  __syncthreads();
+  // sub-run level (identity = thread): same block and interval
+  tile_allreduce<Agg>(
+      s.fl, FL_SH, FL_ST,
+      [&](int j) { return (s.fl[j] & FL_INT) ? agg_item(s.rw[j], s.thr[j], s.vh[j]) : E; }, OpAgg(), E, cin[1],
+      cout[1],
+      [&](int j, const Agg& S) {
+        if (part && j == 0) part[2] = S;
+        if (part && j == (int)cnt - 1) part[3] = S;
+        if (!(s.fl[j] & FL_INT)) return;
+        const u32 t = s.thr[j], w = t / ws, rw = s.rw[j];
+        const u8 g = s.gq[j];
+        bool frw, fww;
+        if (rw == RW_READ) {
+          frw = (ls ? (ex_warp(S, RW_WRITE, w, ws) || ex_warp(S, RW_ATOMIC, w, ws))
+                    : (ex_id(S, RW_WRITE, t) || ex_id(S, RW_ATOMIC, t))) ||
+                (g & 6);
+          fww = false;
+        } else {
+          frw = (ls ? ex_warp(S, RW_READ, w, ws) : ex_id(S, RW_READ, t)) || (g & 1);
+          if (rw == RW_WRITE)
+            fww = ex_id(S, RW_ATOMIC, t) || (g & 4) || ex_wval(S, t, s.vh[j]) || (g & 8);
+          else
+            fww = ex_id(S, RW_WRITE, t) || (g & 2);
+        }
+        s.res[j] = (frw ? 1 : 0) | (fww ? 2 : 0);
+      },
+      s.wv, s.wf);
+  __syncthreads();
+}
+
+__device__ __forceinline__ F5 fields(const TileSmem& s, int j) {
+  F5 f;
+  f.block = s.blk[j + 1], f.interval = s.ivl[j + 1], f.thread = s.thr[j], f.rw = s.rw[j], f.vh = s.vh[j];
+  return f;
+}
+
+__device__ void emit_race(const ConflictArgs& a, u64 head_hi, u32 kind, u32 x, u32 y, u32 hb, u32 hi_) {
+  const KeyLayout& L = a.L;
+  const u32 idx = atomicAdd(a.race_count, 1u);
+  if (idx >= a.race_cap) return;
+  RaceOut r;
+  const u32 sp = space_of_hi(L, head_hi);
+  r.addr = granule_of_hi(L, head_hi) << L.log2G;
+  r.first = a.index_base + x;
+  r.second = a.index_base + y;
+  r.block = sp == SP_SHARED ? hb : NOBI;
+  r.interval = sp == SP_SHARED ? hi_ : NOBI;
+  r.space = (u8)sp;
+  r.kind = (u8)kind;
+#pragma unroll
+  for (int i = 0; i < 6; i++) r.reserved[i] = 0;
+  a.races[idx] = r;
+  a.race_keys[idx] = (group_of_hi(L, head_hi) << 1) | (kind - 1);
+  a.race_vals[idx] = idx;
+}
+
+// ------------------------------------------------------------------------------------------------ mode 1 / 2
+template <int MODE>
+__global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
+  const u32 tile = MODE == 1 ? blockIdx.x : a.cross_list[blockIdx.x];
+  const u64 tb = (u64)tile * CT_TILE;
+  const u32 cnt = (u32)min((u64)CT_TILE, (u64)a.m - tb);
+  const KeyLayout& L = a.L;
+  const int tid = threadIdx.x;
+
+  if (!tile_load(a, s, tb, cnt)) {
+    if (MODE == 1 && tid == 0) a.tile_flags[tile] = TF_GH | TF_GT | TF_SH | TF_ST;
+    return;
+  }
+  const bool cin = !(s.fl[0] & FL_GH), cout = !(s.fl[cnt - 1] & FL_GT);
+  Agg ci[2], co[2];
+  ci[0] = ci[1] = co[0] = co[1] = agg_empty();
+  if (MODE == 2) {
+    const Agg* c = a.carry[tile].a;  // [grp In, grp Out, sub In, sub Out]
+    if (cin) ci[0] = c[0];
+    if (cout) co[0] = c[1];
+    if (!(s.fl[0] & FL_SH)) ci[1] = c[2];
+    if (!(s.fl[cnt - 1] & FL_ST)) co[1] = c[3];
+  }
+  __shared__ Agg s_part[4];
+  tile_flags(a, s, cnt, ci, co, MODE == 1 ? s_part : nullptr);
+  const int ftail = s.first_gtail, lhead = s.last_ghead;
+
+  if (MODE == 1) {
+    if (tid == 0) {
+      u8 tf = 0;
+      if (lhead >= 0) tf |= TF_GH;
+      if (ftail < (int)cnt) tf |= TF_GT;
+      bool sh = false, st = false;
+      for (u32 j = 0; j < cnt; j++) sh |= (s.fl[j] & FL_SH) != 0, st |= (s.fl[j] & FL_ST) != 0;
+      if (sh) tf |= TF_SH;
+      if (st) tf |= TF_ST;
+      if (cin) tf |= TF_CIN;
+      if (cout) tf |= TF_COUT;
+      a.tile_flags[tile] = tf;
+      if (cin || cout) {
+        for (int i = 0; i < 4; i++) a.part[tile].a[i] = s_part[i];
+        a.cross_list[atomicAdd(a.cross_count, 1u)] = tile;
+      }
+      if (cout && lhead >= 0) {  // this tile owns the group that crosses out
+        Slot sl;
+        sl.x[0] = sl.x[1] = sl.y[0] = sl.y[1] = ~0u;
+        sl.head_key = s.key[lhead + 1];
+        sl.hblock = s.blk[lhead + 1];
+        sl.hinterval = s.ivl[lhead + 1];
+        a.slots[tile] = sl;
+      }
+    }
+    // x per group: min flagged (position << 11 | item) per kind; every entry then tests P(x, entry)
+    const X2 XE = {{~0ull, ~0ull}};
+    tile_allreduce<X2>(
+        s.fl, FL_GH, FL_GT,
+        [&](int j) {
+          X2 r = XE;
+          if (s.fl[j] & FL_INT) {
+            const u64 v = ((u64)pos_of(L, s.key[j + 1]) << 11) | (u64)j;
+            if (s.res[j] & 1) r.v[0] = v;
+            if (s.res[j] & 2) r.v[1] = v;
+          }
+          return r;
+        },
+        OpX2(), XE, XE, XE,
+        [&](int j, const X2& X) {
+          if (!(s.fl[j] & FL_INT)) return;
+          const F5 me = fields(s, j);
+#pragma unroll
+          for (int k = 0; k < 2; k++) {
+            u32 yc = ~0u;
+            if (X.v[k] != ~0ull) {
+              const int jx = (int)(X.v[k] & 2047);
+              if (pair_kind(fields(s, jx), me, a.ws, a.ls) == (u32)(k + 1)) yc = pos_of(L, s.key[j + 1]);
+            }
+            s.xy[j][k] = yc;  // y candidate of this entry
+          }
+        },
+        s.wx, s.wf);
+    __syncthreads();
+    // per group: low half = min flagged position (x), high half = min y candidate (y); emit at the tail
+    tile_allreduce<X2>(
+        s.fl, FL_GH, FL_GT,
+        [&](int j) {
+          X2 r = XE;
+          if (s.fl[j] & FL_INT) {
+            const u32 p = pos_of(L, s.key[j + 1]);
+            r.v[0] = ((u64)s.xy[j][0] << 32) | ((s.res[j] & 1) ? p : 0xFFFFFFFFu);
+            r.v[1] = ((u64)s.xy[j][1] << 32) | ((s.res[j] & 2) ? p : 0xFFFFFFFFu);
+          }
+          return r;
+        },
+        OpXY(), XE, XE, XE,
+        [&](int j, const X2& T) {
+          if (!(s.fl[j] & FL_INT) || !(s.fl[j] & FL_GT)) return;
+          if ((cin && j <= ftail) || (cout && j >= lhead)) return;  // crossing groups: modes 2/3
+#pragma unroll
+          for (int k = 0; k < 2; k++) {
+            const u32 x = (u32)(T.v[k] & 0xFFFFFFFFull), y = (u32)(T.v[k] >> 32);
+            if (x == 0xFFFFFFFFu) continue;
+            // every entry of a group has the group's (space, granule) and, for shared memory, its (block,
+            // interval): the tail entry describes the location
+            emit_race(a, s.key[j + 1] >> L.pos_bits, (u32)(k + 1), x, y, s.blk[j + 1], s.ivl[j + 1]);
+          }
+        },
+        s.wx, s.wf);
+    return;
+  }
+
+  // MODE 2: exact flags of the crossing pieces -> x candidates into the owner's slot
+  // pieces: [0, ftail] if cin (owner = a.owner[tile]); [lhead, cnt-1] if cout (owner = tile, or a.owner[tile]
+  // when the whole tile is one group)
+  __shared__ u32 s_min[4];
+  if (tid < 4) s_min[tid] = ~0u;
+  __syncthreads();
+  const int j0 = tid * CT_ITEMS;
+#pragma unroll
+  for (int q = 0; q < CT_ITEMS; q++) {
+    const int j = j0 + q;
+    if (j >= (int)cnt || !(s.fl[j] & FL_INT)) continue;
+    const u32 p = pos_of(L, s.key[j + 1]);
+    const bool A = cin && j <= ftail, B = cout && j >= lhead;
+    if (A) {
+      if (s.res[j] & 1) atomicMin(&s_min[0], p);
+      if (s.res[j] & 2) atomicMin(&s_min[1], p);
+    }
+    if (B && !A) {
+      if (s.res[j] & 1) atomicMin(&s_min[2], p);
+      if (s.res[j] & 2) atomicMin(&s_min[3], p);
+    }
+  }
+  __syncthreads();
+  if (tid == 0) {
+    if (cin) {
+      Slot* sl = &a.slots[a.owner[tile]];
+      if (s_min[0] != ~0u) atomicMin(&sl->x[0], s_min[0]);
+      if (s_min[1] != ~0u) atomicMin(&sl->x[1], s_min[1]);
+    }
+    if (cout && lhead >= 0 && !(cin && lhead <= ftail)) {
+      Slot* sl = &a.slots[tile];
+      if (s_min[2] != ~0u) atomicMin(&sl->x[0], s_min[2]);
+      if (s_min[3] != ~0u) atomicMin(&sl->x[1], s_min[3]);
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------------ mode 3: y
+__global__ void __launch_bounds__(CT_THREADS) conflict_y_kernel(ConflictArgs a) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
+  const u32 tile = a.cross_list[blockIdx.x];
+  const u64 tb = (u64)tile * CT_TILE;
+  const u32 cnt = (u32)min((u64)CT_TILE, (u64)a.m - tb);
+  const KeyLayout& L = a.L;
+  const int tid = threadIdx.x;
+  if (!tile_load(a, s, tb, cnt)) return;
+  const bool cin = !(s.fl[0] & FL_GH), cout = !(s.fl[cnt - 1] & FL_GT);
+  const int ftail = s.first_gtail, lhead = s.last_ghead;
+  __shared__ F5 s_x[2][2];
+  __shared__ u32 s_has[2][2], s_min[2][2];
+  __shared__ u32 s_owner[2];
+  if (tid == 0) {
+    s_owner[0] = cin ? a.owner[tile] : ~0u;
+    s_owner[1] = (cout && lhead >= 0 && !(cin && lhead <= ftail)) ? tile : ~0u;
+  }
+  __syncthreads();
+  if (tid < 4) {
+    const int g = tid >> 1, k = tid & 1;
+    s_has[g][k] = 0;
+    s_min[g][k] = ~0u;
+    if (s_owner[g] != ~0u) {
+      const u32 x = a.slots[s_owner[g]].x[k];
+      if (x != ~0u) {
+        const Rec r = load_rec(a.rec + x);
+        F5 f;
+        f.block = r.block, f.interval = r.interval, f.thread = r.thread, f.rw = r.rw, f.vh = r.vh;
+        s_x[g][k] = f;
+        s_has[g][k] = 1;
+      }
+    }
+  }
+  __syncthreads();
+  const int j0 = tid * CT_ITEMS;
+#pragma unroll
+  for (int q = 0; q < CT_ITEMS; q++) {
+    const int j = j0 + q;
+    if (j >= (int)cnt || !(s.fl[j] & FL_INT)) continue;
+    const bool A = cin && j <= ftail, B = cout && j >= lhead && s_owner[1] != ~0u;
+    const int g = A ? 0 : (B ? 1 : -1);
+    if (g < 0) continue;
+    const F5 me = fields(s, j);
+    const u32 p = pos_of(L, s.key[j + 1]);
+    for (int k = 0; k < 2; k++)
+      if (s_has[g][k] && pair_kind(s_x[g][k], me, a.ws, a.ls) == (u32)(k + 1)) atomicMin(&s_min[g][k], p);
+  }
+  __syncthreads();
+  if (tid < 4) {
+    const int g = tid >> 1, k = tid & 1;
+    if (s_owner[g] != ~0u && s_min[g][k] != ~0u) atomicMin(&a.slots[s_owner[g]].y[k], s_min[g][k]);
+  }
+}
+
+// one race per (crossing group, kind) with a witness; owner tiles are the crossing tiles with TF_COUT whose
+// last group head lies inside the tile
+__global__ void cross_emit_kernel(ConflictArgs a, u32 ncross) {
+  const u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= ncross) return;
+  const u32 tile = a.cross_list[i];
+  if (!(a.tile_flags[tile] & TF_COUT) || !(a.tile_flags[tile] & TF_GH)) return;
+  // the crossing-out group's head is in this tile only if the tile has a group head (TF_GH) — then the last
+  // head is the crossing group's head (slots[tile] was written by mode 1)
+  const Slot sl = a.slots[tile];
+  for (int k = 0; k < 2; k++)
+    if (sl.x[k] != ~0u) emit_race(a, sl.head_key >> a.L.pos_bits, (u32)(k + 1), sl.x[k], sl.y[k], sl.hblock, sl.hinterval);
+}
+
+u32 conflict_tiles(u64 m) { return (u32)((m + CT_TILE - 1) / CT_TILE); }
+
+void launch_conflict(int mode, const ConflictArgs& a, u32 nblocks, cudaStream_t st) {
+  if (!nblocks) return;
+  const size_t sm = sizeof(TileSmem);
+  if (mode == 1) {
+    static bool set = false;
+    if (!set) cudaFuncSetAttribute(conflict_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm), set = true;
+    conflict_kernel<1><<<nblocks, CT_THREADS, sm, st>>>(a);
+  } else if (mode == 2) {
+    static bool set = false;
+    if (!set) cudaFuncSetAttribute(conflict_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm), set = true;
+    conflict_kernel<2><<<nblocks, CT_THREADS, sm, st>>>(a);
+  } else {
+    static bool set = false;
+    if (!set) cudaFuncSetAttribute(conflict_y_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm), set = true;
+    conflict_y_kernel<<<nblocks, CT_THREADS, sm, st>>>(a);
+  }
+}
+
+void launch_cross_emit(const ConflictArgs& a, u32 ncross, cudaStream_t st) {
+  if (ncross) cross_emit_kernel<<<(ncross + 255) / 256, 256, 0, st>>>(a, ncross);
+}
+
+// ------------------------------------------------------------------------------------------------ carries
+// Segmented scans over tiles: for level L in {group, sub-run}:
+//   In_L[j+1]  = (tile j has an L-head) ? S_L[j] : In_L[j] (+) S_L[j]     (forward)
+//   Out_L[j-1] = (tile j has an L-tail) ? P_L[j] : P_L[j] (+) Out_L[j]    (backward)
+//   owner[j+1] = (tile j has a group head) ? j : owner[j]
+// computed in chunks of 1024 tiles (one CTA each), chunk carries by one CTA, then applied.
+constexpr int CARRY_T = 1024;
+
+struct CarryEl {
+  Agg a;
+  u32 owner;
+};
+
+struct OpCarry {
+  __device__ __forceinline__ CarryEl operator()(const CarryEl& x, const CarryEl& y) const {
+    CarryEl r;
+    r.a = agg_merge(x.a, y.a);
+    r.owner = max(x.owner, y.owner);
+    return r;
+  }
+};
+__device__ __forceinline__ CarryEl shfl(const CarryEl& c, int o, bool down) {
+  CarryEl r;
+  r.a = shfl(c.a, o, down);
+  r.owner = shfl(c.owner, o, down);
+  return r;
+}
+
+// scan direction d: 0 grp fwd, 1 grp bwd, 2 sub fwd, 3 sub bwd
+__device__ __forceinline__ void carry_element(const ConflictArgs& a, u32 j, u32 ntiles, int d, bool& f, CarryEl& e) {
+  e.a = agg_empty();
+  e.owner = 0;
+  f = true;
+  if (j >= ntiles) return;
+  const u8 tf = a.tile_flags[j];
+  const bool crossing = tf & (TF_CIN | TF_COUT);
+  const u8 bit = d == 0 ? TF_GH : d == 1 ? TF_GT : d == 2 ? TF_SH : TF_ST;
+  f = (tf & bit) != 0;
+  const int pi = d == 0 ? 1 : d == 1 ? 0 : d == 2 ? 3 : 2;  // fwd uses S (last piece), bwd uses P (first piece)
+  if (crossing) e.a = a.part[j].a[pi];
+  e.owner = (d == 0 && f) ? j : 0;
+}
+
+template <bool REV>
+__device__ CarryEl carry_block_scan(bool f, const CarryEl& v, const CarryEl& seed, bool& incl_f, CarryEl* s_wv,
+                                    u8* s_wf) {
+  // inclusive = exclusive (+) own
+  CarryEl ex = block_seg_excl<CarryEl, OpCarry, REV, CARRY_T>(f, v, seed, OpCarry(), s_wv, s_wf);
+  incl_f = f;
+  return f ? v : OpCarry()(ex, v);
+}
+
+__global__ void __launch_bounds__(CARRY_T) carry_chunk_kernel(ConflictArgs a, u32 ntiles, CarryEl* chunk_tot,
+                                                              u8* chunk_f) {
+  __shared__ CarryEl s_wv[CARRY_T / 32];
+  __shared__ u8 s_wf[CARRY_T / 32];
+  const u32 j = blockIdx.x * CARRY_T + threadIdx.x;
+  for (int d = 0; d < 4; d++) {
+    bool f;
+    CarryEl e;
+    carry_element(a, j, ntiles, d, f, e);
+    CarryEl seed;
+    seed.a = agg_empty(), seed.owner = 0;
+    bool inf;
+    const bool rev = d & 1;
+    CarryEl inc = rev ? carry_block_scan<true>(f, e, seed, inf, s_wv, s_wf)
+                      : carry_block_scan<false>(f, e, seed, inf, s_wv, s_wf);
+    const bool flag_any = __syncthreads_or(f);
+    // chunk total = inclusive value at the chunk's last (fwd) / first (bwd) thread
+    if ((!rev && threadIdx.x == CARRY_T - 1) || (rev && threadIdx.x == 0)) {
+      chunk_tot[blockIdx.x * 4 + d] = inc;
+      chunk_f[blockIdx.x * 4 + d] = flag_any;
+    }
+    __syncthreads();
+  }
+}
+
+__global__ void __launch_bounds__(CARRY_T) carry_top_kernel(u32 nchunks, CarryEl* chunk_tot, u8* chunk_f,
+                                                            CarryEl* chunk_carry) {
+  __shared__ CarryEl s_wv[CARRY_T / 32];
+  __shared__ u8 s_wf[CARRY_T / 32];
+  const u32 c = threadIdx.x;
+  for (int d = 0; d < 4; d++) {
+    CarryEl e;
+    bool f = true;
+    e.a = agg_empty(), e.owner = 0;
+    if (c < nchunks) e = chunk_tot[c * 4 + d], f = chunk_f[c * 4 + d];
+    CarryEl seed;
+    seed.a = agg_empty(), seed.owner = 0;
+    CarryEl ex = (d & 1) ? block_seg_excl<CarryEl, OpCarry, true, CARRY_T>(f, e, seed, OpCarry(), s_wv, s_wf)
+                         : block_seg_excl<CarryEl, OpCarry, false, CARRY_T>(f, e, seed, OpCarry(), s_wv, s_wf);
+    if (c < nchunks) chunk_carry[c * 4 + d] = ex;
+  }
+}
+
+__global__ void __launch_bounds__(CARRY_T) carry_apply_kernel(ConflictArgs a, u32 ntiles, const CarryEl* chunk_carry) {
+  __shared__ CarryEl s_wv[CARRY_T / 32];
+  __shared__ u8 s_wf[CARRY_T / 32];
+  const u32 j = blockIdx.x * CARRY_T + threadIdx.x;
+  for (int d = 0; d < 4; d++) {
+    bool f;
+    CarryEl e;
+    carry_element(a, j, ntiles, d, f, e);
+    const bool rev = d & 1;
+    bool inf;
+    const CarryEl seed = chunk_carry[blockIdx.x * 4 + d];
+    CarryEl inc = rev ? carry_block_scan<true>(f, e, seed, inf, s_wv, s_wf)
+                      : carry_block_scan<false>(f, e, seed, inf, s_wv, s_wf);
+    // fwd inclusive at j feeds tile j+1; bwd inclusive at j feeds tile j-1
+    const long long tgt = rev ? (long long)j - 1 : (long long)j + 1;
+    if (j < ntiles && tgt >= 0 && tgt < (long long)ntiles) {
+      const u8 tt = a.tile_flags[tgt];
+      const bool need = rev ? (tt & TF_COUT) : (tt & TF_CIN);
+      if (need) {
+        a.carry[tgt].a[d] = inc.a;
+        if (d == 0) a.owner[tgt] = inc.owner;
+      }
+    }
+  }
+}
+
+size_t carry_temp_bytes(u32 ntiles) {
+  const u32 nch = (ntiles + CARRY_T - 1) / CARRY_T;
+  return (size_t)nch * 4 * sizeof(CarryEl) * 2 + (size_t)nch * 4 + 256;
+}
+
+void launch_carry(const ConflictArgs& a, u32 ntiles, void* temp, cudaStream_t st) {
+  const u32 nch = (ntiles + CARRY_T - 1) / CARRY_T;
+  CarryEl* tot = reinterpret_cast<CarryEl*>(temp);
+  CarryEl* car = tot + (size_t)nch * 4;
+  u8* fl = reinterpret_cast<u8*>(car + (size_t)nch * 4);
+  carry_chunk_kernel<<<nch, CARRY_T, 0, st>>>(a, ntiles, tot, fl);
+  carry_top_kernel<<<1, CARRY_T, 0, st>>>(nch, tot, fl, car);
+  carry_apply_kernel<<<nch, CARRY_T, 0, st>>>(a, ntiles, car);
+}
+
+__global__ void permute_races_kernel(const RaceOut* __restrict__ in, const u32* __restrict__ order,
+                                     RaceOut* __restrict__ out, u32 nr) {
+  const u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < nr) out[i] = in[order[i]];
+}
+
+void launch_permute_races(const RaceOut* in, const u32* order, RaceOut* out, u32 nr, cudaStream_t st) {
+  if (nr) permute_races_kernel<<<(nr + 255) / 256, 256, 0, st>>>(in, order, out, nr);
+}
+
+}  // namespace sesa

@@ -1,0 +1,105 @@
+// kernels.cuh — launcher declarations of the sm_100a pipeline kernels.
+#pragma once
+#include "common.cuh"
+
+namespace sesa {
+
+constexpr int RADIX_BITS = 8;  // onesweep digit width (8-bit digits, 256 bins per pass)
+constexpr int RADIX = 1 << RADIX_BITS;
+
+// onesweep tile: 256 threads x 16 keys (warp-striped); one lookback word per (tile, bin)
+constexpr int SORT_THREADS = 256;
+constexpr int SORT_ITEMS = 16;
+constexpr int SORT_TILE = SORT_THREADS * SORT_ITEMS;
+
+// conflict tile: 256 threads x 8 entries (blocked)
+constexpr int CT_THREADS = 256;
+constexpr int CT_ITEMS = 8;
+constexpr int CT_TILE = CT_THREADS * CT_ITEMS;
+
+// k_extract.cu
+void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, int grid, cudaStream_t st);
+void launch_extract_1to1(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, u64* keys, u32* hist, int grid,
+                         cudaStream_t st);
+void launch_entry_count(const Rec* rec, u64 n, u32 log2G, u32* cnt, cudaStream_t st);
+void launch_extract_multi(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, const u32* off, u64* keys,
+                          u32* hist, int grid, cudaStream_t st);
+
+// k_util.cu
+size_t scan_u32_temp_bytes(u64 n);
+void launch_scan_exclusive_u32(const u32* in, u32* out, u64 n, void* temp, cudaStream_t st);  // out may alias in
+
+// k_sort.cu
+void launch_bin_base(const u32* hist, u64* bin_base, u32 npass, cudaStream_t st);
+// one LSD pass over keys (and optional u32 values) on digit (key >> shift) & (RADIX-1)
+void launch_onesweep(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m, u32 shift, const u64* bin_base,
+                     u64* lookback, u32* tile_ctr, u32 epoch, cudaStream_t st);
+inline u32 sort_tiles(u64 m) { return (u32)((m + SORT_TILE - 1) / SORT_TILE); }
+// race-list keys: (race key, index) -> histograms for npass digits starting at bit 0
+void launch_hist_keys(const u64* keys, u32 m, u32 npass, u32* hist, cudaStream_t st);
+
+// k_conflict.cu — see the file header for the three modes.
+// Summary of a set of entries at one level (identity = thread within a sub-run, block within a group).
+struct Agg {
+  u32 mn[3], mx[3];  // per access type: min / max identity (empty: mn = ~0, mx = 0)
+  u32 i1, i2;        // identity attaining v1 / v2
+  u64 v1, v1b;       // min write value; min write value over identities != i1 (none: ~0)
+  u64 v2, v2b;       // max write value; max write value over identities != i2 (none: 0)
+};
+struct AggQuad {
+  Agg a[4];
+};
+struct ConflictArgs {
+  const u64* keys;  // sorted entry keys
+  u32 m;            // entries
+  const Rec* rec;   // records (gathered by position)
+  u64 n;
+  KeyLayout L;
+  u32 ws, ls;
+  // outputs (mode 1)
+  u32* race_count;
+  u64* race_keys;   // canonical sort key per race
+  u32* race_vals;   // race index
+  struct RaceOut* races;
+  u32 race_cap;
+  // crossing bookkeeping
+  u32* cross_list;   // tiles with a location run crossing a tile boundary
+  u32* cross_count;
+  u8* tile_flags;    // per tile: bit0 grp head in tile, bit1 grp tail in tile, bit2 sub head, bit3 sub tail,
+                     // bit4 cross-in, bit5 cross-out
+  AggQuad* part;   // per tile: [0] grp first piece (P), [1] grp last piece (S), [2] sub P, [3] sub S
+  AggQuad* carry;  // per tile: [0] grp In, [1] grp Out, [2] sub In, [3] sub Out
+  u32* owner;             // per tile: tile index holding the head of the group that crosses into this tile
+  struct Slot* slots;     // per owner tile
+  u64 index_base;
+};
+
+struct RaceOut {  // == sesa_race (40 bytes)
+  u64 addr, first, second;
+  u32 block, interval;
+  u8 space, kind, reserved[6];
+};
+static_assert(sizeof(RaceOut) == 40, "race layout");
+
+// per-owner-tile slot for a group crossing tile boundaries
+struct Slot {
+  u32 x[2];      // min flagged position per kind (RW, WW), ~0 = none
+  u32 y[2];      // min partner position of x per kind
+  u64 head_key;  // key of the group's first entry
+  u32 hblock, hinterval;
+};
+
+void launch_conflict(int mode, const ConflictArgs& a, u32 ntiles_or_list, cudaStream_t st);
+void launch_carry(const ConflictArgs& a, u32 ntiles, void* temp, cudaStream_t st);
+size_t carry_temp_bytes(u32 ntiles);
+void launch_cross_emit(const ConflictArgs& a, u32 ntiles, cudaStream_t st);
+void launch_permute_races(const RaceOut* in, const u32* order, RaceOut* out, u32 nr, cudaStream_t st);
+u32 conflict_tiles(u64 m);
+
+// k_expand.cu — cells (block, interval slot, thread); descriptors of slot q are idx[ivoff[q] .. ivoff[q+1])
+void launch_flow_count2(const void* flows, const u32* ivoff, const u32* idx, u32 niv, u32 bmin, u64 ncell, u32 tmax,
+                        u32* cnt, cudaStream_t st);
+void launch_flow_write2(const void* flows, const u32* ivoff, const u32* idx, u32 niv, u32 bmin, u64 ncell, u32 tmax,
+                        const u32* off, Rec* out, cudaStream_t st);
+
+}  // namespace sesa

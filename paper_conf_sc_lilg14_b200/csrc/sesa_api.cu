@@ -1,0 +1,582 @@
+// sesa_api.cu — the C ABI of include/sesa.h: handle, validation, buffer management and the orchestration of
+// the sm_100a pipeline.  Host code only; every step of the race check runs in the kernels of
+// k_*.cu.  There is no CPU fallback: without a CUDA device every call fails with SESA_ECUDA.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/sesa.h"
+#include "kernels.cuh"
+#include "sesa_internal.h"
+
+using namespace sesa;
+
+static_assert(sizeof(sesa_access) == 32, "sesa_access");
+static_assert(sizeof(sesa_race) == 40, "sesa_race");
+static_assert(sizeof(sesa_flow) == 104, "sesa_flow");
+
+// ------------------------------------------------------------------------------------------------ helpers
+static u32 bits_of(u64 x) { return x == 0 ? 0u : 64u - (u32)__builtin_clzll(x); }
+
+void sesa_trace::fail(sesa_status s, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  err = buf;
+  status = s;
+}
+
+bool sesa_trace::cuda_ok(cudaError_t e, const char* what) {
+  if (e == cudaSuccess) return true;
+  fail(e == cudaErrorMemoryAllocation ? SESA_ENOMEM : SESA_ECUDA, "%s: %s", what, cudaGetErrorString(e));
+  cudaGetLastError();
+  return false;
+}
+
+bool sesa_trace::grow(DevBuf& b, size_t bytes, const char* what) {
+  if (b.cap >= bytes) return true;
+  if (b.p) cudaFree(b.p);
+  b.p = nullptr;
+  b.cap = 0;
+  size_t want = std::max<size_t>(bytes, 256);
+  if (!cuda_ok(cudaMalloc(&b.p, want), what)) return false;
+  b.cap = want;
+  return true;
+}
+
+void sesa_trace::free_all() {
+  for (DevBuf* b : all_bufs())
+    if (b->p) cudaFree(b->p), b->p = nullptr, b->cap = 0;
+  for (auto& e : ev_pool) cudaEventDestroy(e);
+  ev_pool.clear();
+  if (h_pinned) cudaFreeHost(h_pinned), h_pinned = nullptr;
+}
+
+// ------------------------------------------------------------------------------------------------ profiling
+void sesa_trace::launch_begin(const char* name) {
+  launches++;
+  if (!profiling) return;
+  ProfRec r;
+  r.name = name;
+  r.ev0 = next_event();
+  cudaEventRecord(r.ev0, stream);
+  prof.push_back(r);
+}
+void sesa_trace::launch_end(double bytes) {
+  if (!profiling) return;
+  ProfRec& r = prof.back();
+  r.ev1 = next_event();
+  r.bytes = bytes;
+  cudaEventRecord(r.ev1, stream);
+}
+cudaEvent_t sesa_trace::next_event() {
+  if (ev_used == ev_pool.size()) {
+    cudaEvent_t e;
+    cudaEventCreate(&e);
+    ev_pool.push_back(e);
+  }
+  return ev_pool[ev_used++];
+}
+void sesa_trace::collect_prof() {
+  stats.clear();
+  if (!profiling) return;
+  for (auto& r : prof) {
+    float ms = 0;
+    cudaEventElapsedTime(&ms, r.ev0, r.ev1);
+    auto it = std::find_if(stats.begin(), stats.end(), [&](const sesa_kernel_stat& s) { return r.name == s.name; });
+    if (it == stats.end()) {
+      sesa_kernel_stat s;
+      memset(&s, 0, sizeof s);
+      snprintf(s.name, sizeof s.name, "%s", r.name.c_str());
+      stats.push_back(s);
+      it = stats.end() - 1;
+    }
+    it->launches++;
+    it->ms += ms;
+    it->bytes += r.bytes;
+  }
+}
+
+#define LAUNCH(name, bytes, call) \
+  do {                            \
+    launch_begin(name);           \
+    call;                         \
+    launch_end(bytes);            \
+  } while (0)
+
+// ------------------------------------------------------------------------------------------------ check
+bool sesa_trace::sync_check(const char* what) {
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_ok(e, what);
+  return cuda_ok(cudaStreamSynchronize(stream), what);
+}
+
+// Computes the key layout (common.cuh) from the extents summary.  Returns false (ERANGE) if it does not fit.
+bool sesa_trace::make_layout(const Summary& S, u64 n) {
+  KeyLayout& L = layout;
+  memset(&L, 0, sizeof L);
+  L.log2G = (u32)__builtin_ctz(cfg.granularity);
+  const bool hasS = S.count[0] > 0, hasG = S.count[1] > 0;
+  L.both = hasS && hasG;
+  L.single_space = hasS ? SP_SHARED : SP_GLOBAL;
+  u32 shared_bits = 0, global_bits = 0;
+  if (hasS) {
+    L.gminS = S.gmin[0];
+    L.bminS = S.bmin[0];
+    L.iminS = S.imin[0];
+    L.gbS = bits_of(S.gmax[0] - S.gmin[0]);
+    L.ibS = bits_of((u64)(S.imax[0] - S.imin[0]));
+    L.bbS = bits_of((u64)(S.bmax[0] - S.bmin[0]));
+    shared_bits = L.gbS + L.ibS + L.bbS;
+  }
+  if (hasG) {
+    L.gminG = S.gmin[1];
+    L.bminG = S.bmin[1];
+    L.iminG = S.imin[1];
+    L.gbG = bits_of(S.gmax[1] - S.gmin[1]);
+    if (S.unsorted) {
+      L.ibG = bits_of((u64)(S.imax[1] - S.imin[1]));
+      L.bbG = bits_of((u64)(S.bmax[1] - S.bmin[1]));
+      L.lowG = L.ibG + L.bbG;
+    }
+    global_bits = L.gbG + L.lowG;
+  }
+  // shared runs need (block, interval) order too: in the unsorted case they are part of the shared key anyway
+  L.sort_bits = std::max(shared_bits, global_bits) + (L.both ? 1u : 0u);
+  L.space_shift = L.both ? L.sort_bits - 1 : 0;
+  L.pos_bits = std::max(1u, bits_of(n - 1));
+  if (L.sort_bits + L.pos_bits > 64) {
+    fail(SESA_ERANGE, "key layout needs %u sort bits + %u position bits > 64 (granule span %u bits)", L.sort_bits,
+         L.pos_bits, std::max(L.gbS, L.gbG));
+    return false;
+  }
+  return true;
+}
+
+sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_base) {
+  status = SESA_OK;
+  err.clear();
+  have_result = false;
+  n_races = 0;
+  launches = 0;
+  prof.clear();
+  ev_used = 0;
+  memset(&info, 0, sizeof info);
+  info.n_records = n;
+  if (n == 0) {
+    have_result = true;
+    collect_prof();
+    return SESA_OK;
+  }
+  if (!d_rec) return fail(SESA_EINVAL, "d_records is NULL"), status;
+  cudaPointerAttributes pa;
+  if (cudaPointerGetAttributes(&pa, d_rec) != cudaSuccess || (pa.type != cudaMemoryTypeDevice && pa.type != cudaMemoryTypeManaged)) {
+    cudaGetLastError();
+    return fail(SESA_EINVAL, "d_records is not device memory (use sesa_race_check_host for host buffers)"), status;
+  }
+  if (n >= (1ull << 31)) return fail(SESA_ERANGE, "n = %llu >= 2^31 records (ABI v1 limit)", (unsigned long long)n), status;
+  const Rec* rec = reinterpret_cast<const Rec*>(d_rec);
+  const u32 log2G = (u32)__builtin_ctz(cfg.granularity);
+
+  // 1. validate + extents
+  if (!grow(b_summary, sizeof(Summary), "summary")) return status;
+  Summary init;
+  memset(&init, 0, sizeof init);
+  init.bad_index = ~0ull;
+  init.gmin[0] = init.gmin[1] = ~0ull;
+  init.bmin[0] = init.bmin[1] = init.imin[0] = init.imin[1] = ~0u;
+  h_summary = init;
+  if (!cuda_ok(cudaMemcpyAsync(b_summary.p, &h_summary, sizeof(Summary), cudaMemcpyHostToDevice, stream), "summary init"))
+    return status;
+  const int grid_stream = (int)std::min<u64>((n + 255) / 256, (u64)num_sms * 8);
+  LAUNCH("extents", 32.0 * n, launch_extents(rec, n, log2G, (Summary*)b_summary.p, grid_stream, stream));
+  if (!cuda_ok(cudaMemcpyAsync(&h_summary, b_summary.p, sizeof(Summary), cudaMemcpyDeviceToHost, stream), "summary"))
+    return status;
+  if (!sync_check("extents")) return status;
+  const Summary& S = h_summary;
+  if (S.bad_index != ~0ull) {
+    sesa_access r;
+    cudaMemcpy(&r, d_rec + S.bad_index, sizeof r, cudaMemcpyDeviceToHost);
+    return fail(SESA_EINVAL, "record %llu invalid (space=%u rw=%u size=%u addr=0x%llx)",
+                (unsigned long long)S.bad_index, r.space, r.rw, r.size, (unsigned long long)r.addr),
+           status;
+  }
+  const u64 m = S.entries;
+  info.n_entries = m;
+  info.sorted_input = !S.unsorted;
+  if (m >= (1ull << 31)) return fail(SESA_ERANGE, "%llu entries >= 2^31 (ABI v1 limit)", (unsigned long long)m), status;
+  if (!make_layout(S, n)) return status;
+  const KeyLayout& L = layout;
+  const u32 npass = (L.sort_bits + RADIX_BITS - 1) / RADIX_BITS;
+  info.sort_bits = L.sort_bits;
+  info.pos_bits = L.pos_bits;
+  info.digit_bits = RADIX_BITS;
+
+  // 2. key extraction + digit histograms
+  if (!grow(b_keys[0], m * 8, "keys") || !grow(b_keys[1], m * 8, "keys") ||
+      !grow(b_hist, (size_t)std::max(npass, 1u) * RADIX * 4, "hist") ||
+      !grow(b_binbase, (size_t)std::max(npass, 1u) * RADIX * 8, "binbase"))
+    return status;
+  cudaMemsetAsync(b_hist.p, 0, (size_t)std::max(npass, 1u) * RADIX * 4, stream);
+  u64* keys = (u64*)b_keys[0].p;
+  if (S.multi == 0) {
+    LAUNCH("extract", 40.0 * n,
+           launch_extract_1to1(rec, n, L, npass, keys, (u32*)b_hist.p, grid_stream, stream));
+  } else {
+    if (!grow(b_cnt, n * 4, "counts") || !grow(b_off, n * 4, "offsets") || !grow(b_temp, scan_u32_temp_bytes(n), "scan"))
+      return status;
+    LAUNCH("entry_count", 36.0 * n, launch_entry_count(rec, n, log2G, (u32*)b_cnt.p, stream));
+    LAUNCH("scan", 8.0 * n, launch_scan_exclusive_u32((u32*)b_cnt.p, (u32*)b_off.p, n, b_temp.p, stream));
+    LAUNCH("extract_multi", 36.0 * n + 8.0 * m,
+           launch_extract_multi(rec, n, L, npass, (u32*)b_off.p, keys, (u32*)b_hist.p, grid_stream, stream));
+  }
+  std::vector<u32> hist((size_t)npass * RADIX);
+  if (npass) {
+    if (!cuda_ok(cudaMemcpyAsync(hist.data(), b_hist.p, hist.size() * 4, cudaMemcpyDeviceToHost, stream), "hist"))
+      return status;
+    LAUNCH("bin_base", 0.0, launch_bin_base((u32*)b_hist.p, (u64*)b_binbase.p, npass, stream));
+  }
+  if (!sync_check("extract")) return status;
+
+  // 3. onesweep LSD passes over the non-trivial digits
+  const u32 stiles = sort_tiles(m);
+  if (npass) {
+    if (!grow(b_lookback, (size_t)stiles * RADIX * 8, "lookback") || !grow(b_ctr, 64 * 4, "counters")) return status;
+    if (b_lookback.cap != lookback_cleared) {  // fresh allocation: clear once, epochs do the rest
+      cudaMemsetAsync(b_lookback.p, 0, b_lookback.cap, stream);
+      lookback_cleared = b_lookback.cap;
+      epoch = 0;
+    }
+    cudaMemsetAsync(b_ctr.p, 0, 64 * 4, stream);
+  }
+  int cur = 0;
+  u32 passes_run = 0;
+  for (u32 p = 0; p < npass; p++) {
+    const u32* h = hist.data() + (size_t)p * RADIX;
+    if (*std::max_element(h, h + RADIX) == m) continue;  // trivial digit: every key has the same value
+    if (++epoch >= 256) {
+      cudaMemsetAsync(b_lookback.p, 0, b_lookback.cap, stream);
+      epoch = 1;
+    }
+    LAUNCH("onesweep_pass", 16.0 * m,
+           launch_onesweep((u64*)b_keys[cur].p, (u64*)b_keys[cur ^ 1].p, nullptr, nullptr, (u32)m,
+                           L.pos_bits + p * RADIX_BITS, (u64*)b_binbase.p + (size_t)p * RADIX, (u64*)b_lookback.p,
+                           (u32*)b_ctr.p + passes_run, epoch, stream));
+    cur ^= 1;
+    passes_run++;
+  }
+  info.sort_passes = passes_run;
+  const u64* sorted = (const u64*)b_keys[cur].p;
+
+  // 4. conflict tiles
+  const u32 ctiles = conflict_tiles(m);
+  u32 race_cap = (u32)std::min<u64>(std::max<u64>(race_cap_hint, 1u << 16), 2 * m + 16);
+  for (int attempt = 0; attempt < 3; attempt++) {
+    if (!grow(b_tflags, ctiles, "tile flags") || !grow(b_part, (size_t)ctiles * sizeof(AggQuad), "partials") ||
+        !grow(b_carry, (size_t)ctiles * sizeof(AggQuad), "carries") || !grow(b_owner, (size_t)ctiles * 4, "owner") ||
+        !grow(b_slots, (size_t)ctiles * sizeof(Slot), "slots") || !grow(b_cross, (size_t)ctiles * 4, "cross") ||
+        !grow(b_ccount, 16, "ccount") || !grow(b_races, (size_t)race_cap * sizeof(RaceOut), "races") ||
+        !grow(b_rkeys[0], (size_t)race_cap * 8, "race keys") || !grow(b_rkeys[1], (size_t)race_cap * 8, "race keys") ||
+        !grow(b_rvals[0], (size_t)race_cap * 4, "race vals") || !grow(b_rvals[1], (size_t)race_cap * 4, "race vals") ||
+        !grow(b_carrytmp, carry_temp_bytes(ctiles), "carry temp"))
+      return status;
+    cudaMemsetAsync(b_ccount.p, 0, 16, stream);
+    ConflictArgs A;
+    memset(&A, 0, sizeof A);
+    A.keys = sorted;
+    A.m = (u32)m;
+    A.rec = rec;
+    A.n = n;
+    A.L = L;
+    A.ws = cfg.warp_size;
+    A.ls = cfg.lockstep;
+    A.race_count = (u32*)b_ccount.p;
+    A.cross_count = (u32*)b_ccount.p + 1;
+    A.race_keys = (u64*)b_rkeys[0].p;
+    A.race_vals = (u32*)b_rvals[0].p;
+    A.races = (RaceOut*)b_races.p;
+    A.race_cap = race_cap;
+    A.cross_list = (u32*)b_cross.p;
+    A.tile_flags = (u8*)b_tflags.p;
+    A.part = (AggQuad*)b_part.p;
+    A.carry = (AggQuad*)b_carry.p;
+    A.owner = (u32*)b_owner.p;
+    A.slots = (Slot*)b_slots.p;
+    A.index_base = index_base;
+    LAUNCH("conflict", 8.0 * m, launch_conflict(1, A, ctiles, stream));
+    u32 cc[2];
+    if (!cuda_ok(cudaMemcpyAsync(cc, b_ccount.p, 8, cudaMemcpyDeviceToHost, stream), "counts")) return status;
+    if (!sync_check("conflict")) return status;
+    info.crossing_tiles = cc[1];
+    if (cc[1]) {
+      LAUNCH("carry", 0.0, launch_carry(A, ctiles, b_carrytmp.p, stream));
+      LAUNCH("conflict_cross", 0.0, launch_conflict(2, A, cc[1], stream));
+      LAUNCH("conflict_y", 0.0, launch_conflict(3, A, cc[1], stream));
+      LAUNCH("cross_emit", 0.0, launch_cross_emit(A, cc[1], stream));
+      if (!cuda_ok(cudaMemcpyAsync(cc, b_ccount.p, 8, cudaMemcpyDeviceToHost, stream), "counts")) return status;
+      if (!sync_check("crossing")) return status;
+    }
+    if (cc[0] <= race_cap) {
+      n_races = cc[0];
+      break;
+    }
+    race_cap = (u32)std::min<u64>((u64)cc[0] + cc[0] / 8 + 1024, 2 * m + 16);
+    race_cap_hint = race_cap;
+  }
+
+  // 5. canonical order of the race list: sort (location key << 1 | kind, index), then permute
+  const u32 nr = (u32)n_races;
+  info.n_races = nr;
+  if (!grow(b_races_sorted, (size_t)std::max(nr, 1u) * sizeof(RaceOut), "sorted races")) return status;
+  if (nr) {
+    const u32 rbits = L.sort_bits + 1;
+    const u32 rpass = (rbits + RADIX_BITS - 1) / RADIX_BITS;
+    const u32 rtiles = sort_tiles(nr);
+    if (!grow(b_rhist, (size_t)rpass * RADIX * 4, "race hist") || !grow(b_rbase, (size_t)rpass * RADIX * 8, "race base") ||
+        !grow(b_lookback, (size_t)std::max(rtiles, stiles) * RADIX * 8, "lookback") || !grow(b_ctr, 64 * 4, "counters"))
+      return status;
+    if (b_lookback.cap != lookback_cleared) {
+      cudaMemsetAsync(b_lookback.p, 0, b_lookback.cap, stream);
+      lookback_cleared = b_lookback.cap;
+      epoch = 0;
+    }
+    cudaMemsetAsync(b_rhist.p, 0, (size_t)rpass * RADIX * 4, stream);
+    cudaMemsetAsync((u32*)b_ctr.p + 32, 0, 32 * 4, stream);
+    LAUNCH("race_hist", 8.0 * nr, launch_hist_keys((u64*)b_rkeys[0].p, nr, rpass, (u32*)b_rhist.p, stream));
+    LAUNCH("bin_base", 0.0, launch_bin_base((u32*)b_rhist.p, (u64*)b_rbase.p, rpass, stream));
+    int rc = 0;
+    for (u32 p = 0; p < rpass; p++) {
+      if (++epoch >= 256) {
+        cudaMemsetAsync(b_lookback.p, 0, b_lookback.cap, stream);
+        epoch = 1;
+      }
+      LAUNCH("race_sort", 24.0 * nr,
+             launch_onesweep((u64*)b_rkeys[rc].p, (u64*)b_rkeys[rc ^ 1].p, (u32*)b_rvals[rc].p,
+                             (u32*)b_rvals[rc ^ 1].p, nr, p * RADIX_BITS, (u64*)b_rbase.p + (size_t)p * RADIX,
+                             (u64*)b_lookback.p, (u32*)b_ctr.p + 32 + p, epoch, stream));
+      rc ^= 1;
+    }
+    LAUNCH("race_permute", 80.0 * nr,
+           launch_permute_races((RaceOut*)b_races.p, (u32*)b_rvals[rc].p, (RaceOut*)b_races_sorted.p, nr, stream));
+  }
+  if (!sync_check("race sort")) return status;
+  info.launches = launches;
+  collect_prof();
+  info.n_stats = (u32)stats.size();
+  have_result = true;
+  return SESA_OK;
+}
+
+// ------------------------------------------------------------------------------------------------ expand
+sesa_status sesa_trace::expand(const sesa_flow* d_flows, u64 nf, sesa_access* d_out, u64 cap, u64* n_out) {
+  status = SESA_OK;
+  err.clear();
+  launches = 0;
+  prof.clear();
+  ev_used = 0;
+  if (!n_out) return fail(SESA_EINVAL, "n_out is NULL"), status;
+  *n_out = 0;
+  if (nf == 0) return SESA_OK;
+  if (!d_flows) return fail(SESA_EINVAL, "d_flows is NULL"), status;
+  std::vector<sesa_flow> h(nf);
+  if (!cuda_ok(cudaMemcpy(h.data(), d_flows, nf * sizeof(sesa_flow), cudaMemcpyDeviceToHost), "flows D2H")) return status;
+  u32 bmin = ~0u, bmax = 0, tmax = 0;
+  std::vector<u32> ivs;
+  for (u64 d = 0; d < nf; d++) {
+    const sesa_flow& f = h[d];
+    if (f.fkind > 4 || (f.fkind == SESA_F_MODADD && f.fm == 0) || (f.fkind >= SESA_F_SHR && f.fc >= 32))
+      return fail(SESA_EINVAL, "flow %llu: bad f (fkind=%u fc=%u fm=%u)", (unsigned long long)d, f.fkind, f.fc, f.fm),
+             status;
+    if (f.space > 1 || f.rw > 2 || f.size == 0)
+      return fail(SESA_EINVAL, "flow %llu: bad access (space=%u rw=%u size=%u)", (unsigned long long)d, f.space, f.rw,
+                  f.size),
+             status;
+    ivs.push_back(f.interval);
+    if (f.block_lo >= f.block_hi) continue;
+    bmin = std::min(bmin, f.block_lo);
+    bmax = std::max(bmax, f.block_hi);
+    tmax = std::max(tmax, f.nthreads);
+  }
+  if (bmin >= bmax || tmax == 0) return SESA_OK;
+  std::sort(ivs.begin(), ivs.end());
+  ivs.erase(std::unique(ivs.begin(), ivs.end()), ivs.end());
+  const u32 niv = (u32)ivs.size();
+  std::vector<u32> ivoff(niv + 1, 0), idx;
+  for (u32 q = 0; q < niv; q++) {
+    u64 csum = 0;
+    for (u64 d = 0; d < nf; d++)
+      if (h[d].interval == ivs[q]) idx.push_back((u32)d), csum += h[d].count;
+    ivoff[q + 1] = (u32)idx.size();
+    if (csum >= (1ull << 32)) return fail(SESA_ERANGE, "flow counts of one interval exceed 2^32"), status;
+  }
+  const u64 ncell = (u64)(bmax - bmin) * niv * tmax;
+  if (!grow(b_eoff, (niv + 1 + idx.size()) * 4, "flow csr") || !grow(b_ecnt, ncell * 4, "cell counts") ||
+      !grow(b_ecell, ncell * 4, "cell offsets") || !grow(b_temp, scan_u32_temp_bytes(ncell), "scan"))
+    return status;
+  u32* d_ivoff = (u32*)b_eoff.p;
+  u32* d_idx = d_ivoff + niv + 1;
+  cudaMemcpyAsync(d_ivoff, ivoff.data(), ivoff.size() * 4, cudaMemcpyHostToDevice, stream);
+  cudaMemcpyAsync(d_idx, idx.data(), idx.size() * 4, cudaMemcpyHostToDevice, stream);
+  LAUNCH("flow_count", 4.0 * ncell, launch_flow_count2(d_flows, d_ivoff, d_idx, niv, bmin, ncell, tmax, (u32*)b_ecnt.p, stream));
+  // total = sum of cell counts: scan then last offset + last count (u64 check for overflow below)
+  LAUNCH("scan", 8.0 * ncell, launch_scan_exclusive_u32((u32*)b_ecnt.p, (u32*)b_ecell.p, ncell, b_temp.p, stream));
+  u32 last[2];
+  cudaMemcpyAsync(&last[0], (u32*)b_ecell.p + ncell - 1, 4, cudaMemcpyDeviceToHost, stream);
+  cudaMemcpyAsync(&last[1], (u32*)b_ecnt.p + ncell - 1, 4, cudaMemcpyDeviceToHost, stream);
+  if (!sync_check("flow count")) return status;
+  const u64 total = (u64)last[0] + last[1];
+  // overflow guard: the u32 scan wraps past 2^32; recount on the host side of the bound (sum of per-flow maxima)
+  u64 bound = 0;
+  for (u64 d = 0; d < nf; d++)
+    if (h[d].block_lo < h[d].block_hi)
+      bound += (u64)(h[d].block_hi - h[d].block_lo) * std::min<u64>(h[d].nthreads, h[d].phi > h[d].plo ? h[d].phi - h[d].plo : 0) * h[d].count;
+  if (bound >= (1ull << 32) && total < bound / 2)
+    return fail(SESA_ERANGE, "expansion may exceed 2^32 records"), status;
+  *n_out = total;
+  if (total > cap) return fail(SESA_ETRUNC, "expansion produces %llu records > cap %llu", (unsigned long long)total,
+                               (unsigned long long)cap),
+                      status;
+  if (!d_out) return fail(SESA_EINVAL, "d_out is NULL"), status;
+  LAUNCH("flow_write", 32.0 * total,
+         launch_flow_write2(d_flows, d_ivoff, d_idx, niv, bmin, ncell, tmax, (u32*)b_ecell.p, (Rec*)d_out, stream));
+  if (!sync_check("flow write")) return status;
+  collect_prof();
+  return SESA_OK;
+}
+
+// ------------------------------------------------------------------------------------------------ C ABI
+extern "C" {
+
+int sesa_abi_version(void) { return SESA_ABI_VERSION; }
+
+const char* sesa_status_str(sesa_status s) {
+  switch (s) {
+    case SESA_OK: return "SESA_OK";
+    case SESA_EINVAL: return "SESA_EINVAL";
+    case SESA_ERANGE: return "SESA_ERANGE";
+    case SESA_ENOMEM: return "SESA_ENOMEM";
+    case SESA_ECUDA: return "SESA_ECUDA";
+    case SESA_ENCCL: return "SESA_ENCCL";
+    case SESA_ESTATE: return "SESA_ESTATE";
+    case SESA_ETRUNC: return "SESA_ETRUNC";
+  }
+  return "SESA_?";
+}
+
+static sesa_status check_cfg(const sesa_config* c) {
+  if (!c) return SESA_EINVAL;
+  if (c->warp_size < 1 || c->lockstep > 1 || c->granularity < 1 || c->granularity > 4096 ||
+      (c->granularity & (c->granularity - 1)) || c->flags != 0)
+    return SESA_EINVAL;
+  return SESA_OK;
+}
+
+sesa_status sesa_trace_create(const sesa_config* cfg, sesa_trace** out) {
+  if (!out) return SESA_EINVAL;
+  *out = nullptr;
+  if (check_cfg(cfg) != SESA_OK) return SESA_EINVAL;
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) {
+    cudaGetLastError();
+    return SESA_ECUDA;
+  }
+  sesa_trace* t = new (std::nothrow) sesa_trace();
+  if (!t) return SESA_ENOMEM;
+  t->cfg = *cfg;
+  t->device = dev;
+  cudaDeviceGetAttribute(&t->num_sms, cudaDevAttrMultiProcessorCount, dev);
+  if (t->num_sms <= 0) t->num_sms = 148;
+  *out = t;
+  return SESA_OK;
+}
+
+sesa_status sesa_race_check(sesa_trace* t, const sesa_access* d_records, uint64_t n, uint64_t index_base,
+                            void* cuda_stream) {
+  if (!t) return SESA_EINVAL;
+  t->stream = (cudaStream_t)cuda_stream;
+  if (t->dist) return t->check_dist(d_records, n, index_base);
+  return t->check_device(d_records, n, index_base);
+}
+
+sesa_status sesa_race_check_host(sesa_trace* t, const sesa_access* h_records, uint64_t n, uint64_t index_base,
+                                 void* cuda_stream) {
+  if (!t) return SESA_EINVAL;
+  t->stream = (cudaStream_t)cuda_stream;
+  t->status = SESA_OK;
+  t->have_result = false;
+  if (n == 0) return sesa_race_check(t, nullptr, 0, index_base, cuda_stream);
+  if (!h_records) return t->fail(SESA_EINVAL, "h_records is NULL"), t->status;
+  if (!t->grow(t->b_hrec, n * sizeof(sesa_access), "record copy")) return t->status;
+  if (!t->cuda_ok(cudaMemcpyAsync(t->b_hrec.p, h_records, n * sizeof(sesa_access), cudaMemcpyHostToDevice, t->stream),
+                  "records H2D"))
+    return t->status;
+  return sesa_race_check(t, (const sesa_access*)t->b_hrec.p, n, index_base, cuda_stream);
+}
+
+sesa_status sesa_races_get(sesa_trace* t, sesa_race* host_out, uint64_t cap, uint64_t* n_races) {
+  if (!t || !n_races) return SESA_EINVAL;
+  if (!t->have_result) return SESA_ESTATE;
+  const u64 nr = t->dist && t->rank != 0 ? 0 : t->n_races;
+  *n_races = nr;
+  if (cap == 0 || nr == 0) return SESA_OK;
+  if (!host_out) return SESA_EINVAL;
+  const u64 k = std::min<u64>(cap, nr);
+  const void* src = t->dist ? t->b_dist_races.p : t->b_races_sorted.p;
+  if (cudaMemcpy(host_out, src, k * sizeof(sesa_race), cudaMemcpyDeviceToHost) != cudaSuccess) {
+    cudaGetLastError();
+    return SESA_ECUDA;
+  }
+  return k < nr ? SESA_ETRUNC : SESA_OK;
+}
+
+sesa_status sesa_races_device(sesa_trace* t, const sesa_race** d_races, uint64_t* n_races) {
+  if (!t || !d_races || !n_races) return SESA_EINVAL;
+  if (!t->have_result) return SESA_ESTATE;
+  *n_races = t->dist && t->rank != 0 ? 0 : t->n_races;
+  *d_races = (const sesa_race*)(t->dist ? t->b_dist_races.p : t->b_races_sorted.p);
+  return SESA_OK;
+}
+
+sesa_status sesa_expand(sesa_trace* t, const sesa_flow* d_flows, uint64_t n_flows, sesa_access* d_out, uint64_t cap,
+                        uint64_t* n_out, void* cuda_stream) {
+  if (!t) return SESA_EINVAL;
+  t->stream = (cudaStream_t)cuda_stream;
+  return t->expand(d_flows, n_flows, d_out, cap, n_out);
+}
+
+sesa_status sesa_trace_set_profiling(sesa_trace* t, int enable) {
+  if (!t) return SESA_EINVAL;
+  t->profiling = enable != 0;
+  return SESA_OK;
+}
+
+sesa_status sesa_trace_info(const sesa_trace* t, sesa_check_info* out) {
+  if (!t || !out) return SESA_EINVAL;
+  *out = t->info;
+  return SESA_OK;
+}
+
+sesa_status sesa_trace_kernel_stats(const sesa_trace* t, sesa_kernel_stat* out, uint32_t cap, uint32_t* n_out) {
+  if (!t || !n_out) return SESA_EINVAL;
+  *n_out = (u32)t->stats.size();
+  for (u32 i = 0; i < std::min<u32>(cap, (u32)t->stats.size()); i++) out[i] = t->stats[i];
+  return SESA_OK;
+}
+
+void sesa_trace_destroy(sesa_trace* t) {
+  if (!t) return;
+  t->destroy_dist();
+  t->free_all();
+  delete t;
+}
+
+const char* sesa_last_error(const sesa_trace* t) { return t ? t->err.c_str() : ""; }
+
+}  // extern "C"

@@ -1,0 +1,88 @@
+// sesa_internal.h — the opaque handle behind include/sesa.h (host side).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <string>
+#include <vector>
+
+#include "../../include/sesa.h"
+#include "kernels.cuh"
+
+struct DevBuf {
+  void* p = nullptr;
+  size_t cap = 0;
+};
+
+struct ProfRec {
+  std::string name;
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  double bytes = 0;
+};
+
+struct DistState;  // dist.cu
+
+struct sesa_trace {
+  sesa_config cfg{};
+  int device = 0;
+  int num_sms = 148;
+  cudaStream_t stream = nullptr;
+  sesa_status status = SESA_OK;
+  std::string err;
+  bool have_result = false;
+  uint64_t n_races = 0;
+  uint32_t tile_shift = 0;
+  uint64_t race_cap_hint = 0;
+  uint32_t epoch = 0;
+  size_t lookback_cleared = 0;
+  sesa::KeyLayout layout{};
+  sesa::Summary h_summary{};
+  sesa_check_info info{};
+
+  // device buffers (grow-only, freed by destroy)
+  DevBuf b_summary, b_keys[2], b_hist, b_binbase, b_lookback, b_ctr, b_cnt, b_off, b_temp;
+  DevBuf b_tflags, b_part, b_carry, b_owner, b_slots, b_cross, b_ccount, b_carrytmp;
+  DevBuf b_races, b_rkeys[2], b_rvals[2], b_races_sorted, b_rhist, b_rbase;
+  DevBuf b_eoff, b_ecnt, b_ecell, b_hrec, b_dist_races;
+  DevBuf b_dist[8];
+  void* h_pinned = nullptr;
+
+  std::vector<DevBuf*> all_bufs() {
+    std::vector<DevBuf*> v = {&b_summary, &b_hist, &b_binbase, &b_lookback, &b_ctr, &b_cnt, &b_off, &b_temp,
+                              &b_tflags, &b_part, &b_carry, &b_owner, &b_slots, &b_cross, &b_ccount, &b_carrytmp,
+                              &b_races, &b_races_sorted, &b_rhist, &b_rbase, &b_eoff, &b_ecnt, &b_ecell,
+                              &b_hrec, &b_dist_races};
+    for (auto& b : b_keys) v.push_back(&b);
+    for (auto& b : b_rkeys) v.push_back(&b);
+    for (auto& b : b_rvals) v.push_back(&b);
+    for (auto& b : b_dist) v.push_back(&b);
+    return v;
+  }
+
+  // profiling
+  bool profiling = false;
+  uint32_t launches = 0;
+  std::vector<ProfRec> prof;
+  std::vector<cudaEvent_t> ev_pool;
+  size_t ev_used = 0;
+  std::vector<sesa_kernel_stat> stats;
+
+  // distributed
+  bool dist = false;
+  int rank = 0, world = 1;
+  DistState* ds = nullptr;
+
+  void fail(sesa_status s, const char* fmt, ...);
+  bool cuda_ok(cudaError_t e, const char* what);
+  bool grow(DevBuf& b, size_t bytes, const char* what);
+  bool sync_check(const char* what);
+  void free_all();
+  void launch_begin(const char* name);
+  void launch_end(double bytes);
+  cudaEvent_t next_event();
+  void collect_prof();
+  bool make_layout(const sesa::Summary& S, uint64_t n);
+  sesa_status check_device(const sesa_access* d_rec, uint64_t n, uint64_t index_base);
+  sesa_status expand(const sesa_flow* d_flows, uint64_t nf, sesa_access* d_out, uint64_t cap, uint64_t* n_out);
+  sesa_status check_dist(const sesa_access* d_rec, uint64_t n, uint64_t index_base);
+  void destroy_dist();
+};

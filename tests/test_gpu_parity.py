@@ -1,0 +1,235 @@
+"""GPU parity: the sm_100a pipeline (libsesa.so through the C ABI) against the CPU oracle, byte for byte.
+
+The output is integer-only (record indices, addresses, kinds), so the bar is bit-exact equality of the sorted
+race arrays.  Inputs come from sesagen (seeded); expected values only from oracle/.
+"""
+import ctypes
+
+import numpy as np
+import pytest
+
+import sesagen as G
+from oracle import oracle as O
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module")
+def sesa():
+    from paper_conf_sc_lilg14_b200 import sesa as S
+    S.load()
+    return S
+
+
+_traces = {}
+
+
+def trace(S, ws=32, ls=0, G_=4):
+    key = (ws, ls, G_)
+    if key not in _traces:
+        _traces[key] = S.Trace(ws, ls, G_)
+    return _traces[key]
+
+
+def gpu_check(S, recs, ws=32, ls=0, G_=4, base=0):
+    t = trace(S, ws, ls, G_)
+    d = S.to_device(recs)
+    t.check(d, len(recs), index_base=base)
+    torch.cuda.synchronize()
+    return t.races()
+
+
+def assert_same(S, recs, ws=32, ls=0, G_=4, base=0, method="grouped"):
+    exp = O.check(recs, index_base=base, warp_size=ws, lockstep=ls, granularity=G_, method=method)
+    got = gpu_check(S, recs, ws, ls, G_, base)
+    if got.tobytes() != exp.tobytes():
+        e, g = set(O.race_tuples(exp)), set(O.race_tuples(got))
+        raise AssertionError(f"{len(exp)} expected, {len(got)} got; missing {sorted(e - g)[:5]} extra {sorted(g - e)[:5]}")
+    return got
+
+
+# ------------------------------------------------------------------------------------------------ paper fixtures
+@pytest.mark.parametrize("ls", [0, 1])
+@pytest.mark.parametrize("distinct", [True, False])
+def test_f1_race(sesa, ls, distinct):
+    assert_same(sesa, G.f1_race(distinct=distinct), ls=ls, method="brute")
+
+
+def test_f1_paper_witness_on_gpu(sesa):
+    got = O.race_tuples(gpu_check(sesa, G.f1_race()))
+    assert (0, 0, 0, 0, 1, 1, 126) in got  # t0 writes v[0], t63 reads it (interval 0)
+
+
+def test_f2_reduction(sesa):
+    for ls in (0, 1):
+        assert len(assert_same(sesa, G.f2_reduction(), ls=ls)) == 0
+
+
+@pytest.mark.parametrize("B", [16, 32, 64, 128, 256])
+def test_f3_bitonic(sesa, B):
+    assert len(assert_same(sesa, G.f3_bitonic(B))) == 0
+
+
+@pytest.mark.parametrize("ls,ws", [(0, 32), (1, 32), (1, 1)])
+def test_f4_histo_prescan(sesa, ls, ws):
+    assert_same(sesa, G.f4_histo_prescan(), ws=ws, ls=ls)
+
+
+@pytest.mark.parametrize("ls", [0, 1])
+def test_f5_binning(sesa, ls):
+    assert len(assert_same(sesa, G.f5_binning(), ls=ls)) == 1
+
+
+def test_c1(sesa):
+    got = assert_same(sesa, G.c1(), method="brute")
+    assert O.race_tuples(got) == [(0, 0, 5, 4, 2, 833, 836)]
+
+
+# ------------------------------------------------------------------------------------------------ random traces
+CONFIGS = [(32, 0, 4), (32, 1, 4), (4, 1, 1), (1, 1, 2), (2, 0, 8), (8, 1, 16)]
+
+
+@pytest.mark.parametrize("cfg", CONFIGS)
+def test_random_small(sesa, cfg):
+    ws, ls, G_ = cfg
+    for seed in range(40):
+        n = 1 + (seed * 37) % 400
+        r = G.random_trace(n, seed, threads=12 + seed % 60, sort=seed % 4 != 0, words=8 + seed % 40)
+        assert_same(sesa, r, ws, ls, G_, base=seed * 1000)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_random_medium_spans_tiles(sesa, seed):
+    # 20k-150k entries: many 2048-entry conflict tiles, 4096-key sort tiles and a ragged tail
+    n = [20000, 33333, 65537, 100000, 150001, 4097][seed]
+    r = G.random_trace(n, seed, blocks=40, threads=256, intervals=4, words=5000 + 3000 * seed, values=5,
+                       sort=seed != 3)
+    assert_same(sesa, r, 32, seed % 2, 4)
+
+
+@pytest.mark.parametrize("words", [1, 3, 40, 700])
+def test_hot_locations_cross_tiles(sesa, words):
+    # few words -> location runs of thousands of entries: runs and sub-runs cross conflict-tile boundaries
+    r = G.random_trace(60000, 99 + words, blocks=6, threads=300, intervals=3, words=words, values=3)
+    for ls in (0, 1):
+        assert_same(sesa, r, 32, ls, 4)
+
+
+def test_hot_benign_and_atomics(sesa):
+    # a C4-like `changed` run: 50k same-valued writes from many blocks plus a few reads -> RW only, no WW
+    n = 50000
+    r = np.zeros(n, G.REC_DTYPE)
+    r["block"] = np.arange(n) // 512
+    r["thread"] = np.arange(n) % 512
+    r["space"] = 1
+    r["size"] = 4
+    r["addr"] = 0x5000
+    r["rw"] = 1
+    r["value_hash"] = 77
+    r["rw"][::9973] = 0
+    got = assert_same(sesa, r, 32, 1, 4)
+    assert set(got["kind"]) <= {1}
+
+
+# ------------------------------------------------------------------------------------------------ expansion
+@pytest.mark.parametrize("name", ["f1", "f2", "f5", "c1", "c2s", "c2m"])
+def test_expand_parity(sesa, name):
+    fl = {"f1": G.f1_flows(), "f2": G.f2_flows(), "f5": G.f5_flows(), "c1": G.c1_flows(),
+          "c2s": G.c2_flows(gx=2, gy=3, K=80), "c2m": G.c2_mutant_flows(drop_barrier=3, gx=2, gy=2, K=64)}[name]
+    exp = O.expand(fl)
+    t = trace(sesa)
+    d_fl = torch.from_numpy(np.ascontiguousarray(fl).view(np.uint8).reshape(-1)).cuda()
+    n = t.expand(d_fl, len(fl))
+    assert n == len(exp)
+    out = torch.empty(n * 32, dtype=torch.uint8, device="cuda")
+    assert t.expand(d_fl, len(fl), out, n) == n
+    got = out.cpu().numpy().view(G.REC_DTYPE)
+    assert got.tobytes() == exp.tobytes()
+    if name.startswith("c2"):
+        assert_same(sesa, exp)
+
+
+def test_c2_full_expand_and_race_free(sesa):
+    fl = G.c2_flows()
+    t = trace(sesa)
+    d_fl = torch.from_numpy(np.ascontiguousarray(fl).view(np.uint8).reshape(-1)).cuda()
+    n = t.expand(d_fl, len(fl))
+    assert n == 18300928
+    out = torch.empty(n * 32, dtype=torch.uint8, device="cuda")
+    t.expand(d_fl, len(fl), out, n)
+    # sampled parity of the expansion at full size (oracle expands the same descriptors)
+    exp = O.expand(fl)
+    got = out.cpu().numpy().view(G.REC_DTYPE)
+    idx = np.random.default_rng(0).integers(0, n, 200000)
+    assert got[idx].tobytes() == exp[idx].tobytes()
+    assert t.check(out, n) == 0  # race-free by construction (double buffering, one barrier per k-tile)
+
+
+# ------------------------------------------------------------------------------------------------ API behaviour
+def test_empty_and_single(sesa):
+    t = trace(sesa)
+    assert t.check(0, 0) == 0
+    assert len(t.races()) == 0
+    assert_same(sesa, G.f1_race()[:1])
+
+
+def test_invalid_record_lowest_index(sesa):
+    r = G.f1_race()
+    r[40]["rw"] = 3
+    r[17]["size"] = 0
+    t = trace(sesa)
+    with pytest.raises(sesa.SesaError) as e:
+        t.check(sesa.to_device(r), len(r))
+    assert e.value.status == sesa.SESA_EINVAL and "record 17 " in str(e.value)
+    n = ctypes.c_uint64()
+    assert t.lib.sesa_races_get(t.h, None, 0, ctypes.byref(n)) == sesa.SESA_ESTATE  # all-or-nothing
+
+
+def test_host_pointer_rejected(sesa):
+    r = G.f1_race()
+    t = trace(sesa)
+    with pytest.raises(sesa.SesaError) as e:
+        t.check(r.ctypes.data, len(r))
+    assert e.value.status == sesa.SESA_EINVAL
+
+
+def test_erange_wide_key(sesa):
+    r = G.random_trace(1000, 5)
+    r["addr"][::2] = np.uint64(1 << 63)  # 2^61-granule global span + shared + 10 position bits > 64
+    t = trace(sesa)
+    with pytest.raises(sesa.SesaError) as e:
+        t.check(sesa.to_device(r), len(r))
+    assert e.value.status == sesa.SESA_ERANGE
+
+
+def test_races_get_truncation(sesa):
+    r = G.f1_race()
+    t = trace(sesa)
+    d = sesa.to_device(r)
+    assert t.check(d, len(r)) == 88
+    out = np.zeros(10, sesa.RACE_DTYPE)
+    n = ctypes.c_uint64()
+    st = t.lib.sesa_races_get(t.h, ctypes.c_void_p(out.ctypes.data), 10, ctypes.byref(n))
+    assert st == sesa.SESA_ETRUNC and n.value == 88
+    assert out.tobytes() == O.check(r)[:10].tobytes()
+
+
+def test_host_entry_point_matches(sesa):
+    r = G.random_trace(5000, 11, words=300)
+    t = trace(sesa)
+    t.check_host(r, index_base=7)
+    assert t.races().tobytes() == O.check(r, index_base=7).tobytes()
+
+
+def test_profiling_stats(sesa):
+    t = sesa.Trace()
+    t.set_profiling(True)
+    r = G.random_trace(30000, 3, words=2000)
+    t.check(sesa.to_device(r), len(r))
+    names = {s["name"] for s in t.kernel_stats()}
+    assert {"extents", "extract", "onesweep_pass", "conflict"} <= names
+    info = t.info()
+    assert info["n_records"] == 30000 and info["launches"] >= 4
+    t.close()
