@@ -229,7 +229,10 @@ def test_profiling_stats(sesa):
     r = G.random_trace(30000, 3, words=2000)
     t.check(sesa.to_device(r), len(r))
     names = {s["name"] for s in t.kernel_stats()}
-    assert {"extents", "extract", "onesweep_pass", "conflict"} <= names
+    assert {"extents", "extract_multi", "onesweep_pass", "conflict"} <= names  # sizes up to 8 B: multi-granule
+    r1 = G.random_trace(30000, 4, words=2000, sizes=(4,), unaligned=False)
+    t.check(sesa.to_device(r1), len(r1))
+    assert "extract" in {s["name"] for s in t.kernel_stats()}
     info = t.info()
     assert info["n_records"] == 30000 and info["launches"] >= 4
     t.close()
