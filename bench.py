@@ -1,0 +1,360 @@
+"""Benchmark: access records race-checked per second (Grec/s) on B200, with HBM roofline and CPU-oracle baseline.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c5|c4|c3|c2|c1] [--impl ours|reference]
+
+One step = one sesa_race_check over the whole trace (every §8(a) row: extents, key extract, onesweep sort,
+conflict tiles, carries, race sort) with the records already resident in HBM.  Default workload: BASELINE.json
+config 5 (1e9 records, the trace the 1/2/4/8-GPU metric is quoted on).  For N > 1 (torchrun) records are
+sharded by contiguous ranges and exchanged by location hash inside sesa_race_check (NCCL all-to-all).
+Prints ONE JSON line on rank 0 (contract in the task statement; fields explained in DESIGN.md §9).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "access records race-checked/sec (Grec/s) at 1/2/4/8 B200; % HBM roofline"
+CONFIGS = {
+    "c1": dict(workload="C1 tree reduction 1x64 threads, 6 intervals, 959 records, 1 injected WW", ws=32, ls=0),
+    "c2": dict(workload="C2 Parboil-sgemm-shaped 64 blocks x 256 threads, 32 intervals, 18,300,928 records",
+               ws=32, ls=0),
+    "c3": dict(workload="C3 Parboil-histo-shaped 1024 x 512 threads, Zipf bins + atomics, ~101.4M records",
+               ws=32, ls=0),
+    "c4": dict(workload="C4 Lonestar-bfs-shaped 2^24 nodes, power-law degrees, lockstep, ~392M records",
+               ws=32, ls=1),
+    "c5": dict(workload="C5 scaling sweep: 1e9 global records, 0.01% injected races", ws=32, ls=0),
+}
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+def make_records(cfg: str, n_override=None, rank=0, world=1):
+    """Device records for one rank: (tensor, n, index_base)."""
+    import numpy as np
+    import torch
+
+    import sesagen as G
+    from sesagen import configs as C
+    if cfg == "c5":
+        n = n_override or 10**9
+        lo, hi = rank * n // world, (rank + 1) * n // world
+        out = torch.empty((hi - lo) * 32, dtype=torch.uint8, device="cuda")
+        from sesagen.configs import _devlib, c5_cfg
+        import ctypes
+        c = c5_cfg(n)
+        rc = _devlib().gen_c5_dev(ctypes.byref(c), lo, hi, ctypes.c_void_p(out.data_ptr()),
+                                  ctypes.c_void_p(torch.cuda.current_stream().cuda_stream))
+        assert rc == 0
+        return out, hi - lo, lo, n
+    if cfg in ("c3", "c4"):
+        recs, n = (C.C3() if cfg == "c3" else C.C4()).device()
+        lo, hi = rank * n // world, (rank + 1) * n // world
+        return recs[lo * 32:hi * 32], hi - lo, lo, n
+    if cfg == "c2":
+        from paper_conf_sc_lilg14_b200 import sesa as S
+        fl = G.c2_flows()
+        t = S.Trace()
+        d_fl = torch.from_numpy(np.ascontiguousarray(fl).view(np.uint8).reshape(-1)).cuda()
+        n = t.expand(d_fl, len(fl))
+        out = torch.empty(n * 32, dtype=torch.uint8, device="cuda")
+        t.expand(d_fl, len(fl), out, n)
+        t.close()
+        lo, hi = rank * n // world, (rank + 1) * n // world
+        return out[lo * 32:hi * 32], hi - lo, lo, n
+    recs = G.c1()
+    n = len(recs)
+    lo, hi = rank * n // world, (rank + 1) * n // world
+    return torch.from_numpy(recs.view(np.uint8).reshape(-1)).cuda()[lo * 32:hi * 32], hi - lo, lo, n
+
+
+def host_sample(cfg: str, budget_records: int):
+    """A bounded host-generated sample of the same workload for the oracle (cpu_baseline / reference arm)."""
+    import sesagen as G
+    from sesagen import configs as C
+    if cfg == "c5":
+        n = budget_records
+        return C.c5_host(n), f"seeded C5 generator at n={n} (same recipe, {max(1, n // 10000)} injected races)"
+    if cfg == "c3":
+        b = max(1, budget_records // (512 * 2 * 96))
+        s = C.C3(blocks=b)
+        return s.host(), f"C3 recipe with {b} of 1024 blocks"
+    if cfg == "c4":
+        lg = 18
+        return C.C4(log2n=lg).host(), f"C4 recipe with 2^{lg} nodes"
+    if cfg == "c2":
+        from oracle import oracle as O
+        fl = G.c2_flows(gx=2, gy=4)
+        return O.expand(fl), "C2 recipe with 8 of 64 blocks (oracle-expanded flows)"
+    return G.c1(), "C1 (full)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        self.p = None
+
+    def __enter__(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "200"], stdout=self.f,
+                                      stderr=subprocess.DEVNULL)
+        except FileNotFoundError:
+            self.p = None
+        time.sleep(0.3)
+        return self
+
+    def __exit__(self, *a):
+        if self.p:
+            self.p.terminate()
+            self.p.wait()
+
+    def summary(self):
+        self.f.flush()
+        rows = []
+        for line in open(self.f.name):
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                rows.append(dict(sm=float(parts[1]), smax=float(parts[2]), power=float(parts[3]),
+                                 hw=parts[5], hwt=parts[6], swt=parts[7], pcap=parts[8]))
+            except ValueError:
+                continue
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
+        load = [r for r in rows if r["power"] > 200] or rows
+        reasons = set()
+        for r in load:
+            for k, name in (("hw", "hw_slowdown"), ("hwt", "hw_thermal_slowdown"), ("swt", "sw_thermal_slowdown"),
+                            ("pcap", "sw_power_cap")):
+                if r[k].lower() == "active":
+                    reasons.add(name)
+        return {"sm_mhz": statistics.median(r["sm"] for r in load), "sm_max_mhz": max(r["smax"] for r in rows),
+                "reasons": sorted(reasons), "samples": len(rows), "samples_under_load": len(load)}
+
+
+def measured_peak_hbm():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        return float(json.load(open(p))["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def ncu_traffic(cfg: str, kernel: str):
+    """DRAM bytes per launch of `kernel` from the committed ncu --set full summary, if one exists."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if not os.path.exists(p):
+        return None
+    d = json.load(open(p))
+    return d.get(cfg, {}).get(kernel)
+
+
+def run_cpu_baseline(cfg: str, budget_records: int):
+    from oracle import oracle as O
+    recs, sample = host_sample(cfg, budget_records)
+    c = CONFIGS[cfg]
+    t0 = time.perf_counter()
+    O.check(recs, warp_size=c["ws"], lockstep=c["ls"], granularity=4)
+    dt = time.perf_counter() - t0
+    return {"value": len(recs) / dt / 1e9, "unit": "Grec/s", "cores": 1, "kind": "oracle",
+            "sample": f"{sample}: {len(recs)} records in {dt:.2f} s (oracle_check_grouped, 1 thread)"}
+
+
+def reference_arm(args, rank, world):
+    """--impl reference: the CPU oracle as it stands, on bounded samples of the same workload (rank 0 only)."""
+    if rank != 0:
+        return
+    from oracle import oracle as O
+    c = CONFIGS[args.config]
+    budget = args.ref_records
+    recs, sample = host_sample(args.config, budget)
+    for _ in range(args.warmup):
+        O.check(recs[: min(len(recs), 100000)], warp_size=c["ws"], lockstep=c["ls"])
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        O.check(recs, warp_size=c["ws"], lockstep=c["ls"], granularity=4)
+        times.append(time.perf_counter() - t0)
+    tot = sum(times)
+    value = len(recs) * args.steps / tot / 1e9
+    line = {"metric": METRIC, "value": value, "unit": "Grec/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": 1000 * tot / args.steps, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+            "config": {"workload": c["workload"], "sample": sample}, "impl": "reference",
+            "cpu_baseline": {"value": value, "unit": "Grec/s", "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": "Grec/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="c5", choices=sorted(CONFIGS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--n", type=int, default=None, help="override the C5 record count")
+    ap.add_argument("--cpu-records", type=int, default=1 << 24)
+    ap.add_argument("--ref-records", type=int, default=1 << 23)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    args = ap.parse_args()
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        reference_arm(args, rank, world)
+        return
+
+    import torch
+    torch.cuda.set_device(local)
+    from paper_conf_sc_lilg14_b200 import sesa as S
+    S.load()
+    c = CONFIGS[args.config]
+    pg = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        pg = dist
+        uid = S.nccl_unique_id() if rank == 0 else bytes(128)
+        obj = [uid]
+        dist.broadcast_object_list(obj, src=0)
+        trace = S.Trace(c["ws"], c["ls"], 4, dist=(rank, world, obj[0]))
+    else:
+        trace = S.Trace(c["ws"], c["ls"], 4)
+
+    recs, n_local, base, n_total = make_records(args.config, args.n, rank, world)
+    torch.cuda.synchronize()
+    log(f"[bench] rank {rank}/{world}: {args.config} n={n_total} local={n_local}")
+    stream = torch.cuda.current_stream()
+
+    def step():
+        trace.check(recs, n_local, index_base=base, stream=stream)
+
+    for _ in range(args.warmup):
+        step()
+    trace.set_profiling(True)
+    kstats = {}
+    launches = 0
+    start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(torch.cuda.current_device()) as clk:
+        if pg:
+            pg.barrier()
+        torch.cuda.synchronize()
+        start.record(stream)
+        for _ in range(args.steps):
+            step()
+            for s in trace.kernel_stats():
+                a = kstats.setdefault(s["name"], dict(launches=0, ms=0.0, bytes=0.0))
+                a["launches"] += s["launches"]
+                a["ms"] += s["ms"]
+                a["bytes"] += s["bytes"]
+            launches += trace.info()["launches"]
+        end.record(stream)
+        torch.cuda.synchronize()
+        if pg:
+            pg.barrier()
+    trace.set_profiling(False)
+    ms = start.elapsed_time(end)
+    if pg:
+        t = torch.tensor([ms], device="cuda")
+        pg.all_reduce(t, op=pg.ReduceOp.MAX)
+        ms = float(t.item())
+    info = trace.info()
+    n_races = trace.n_races() if rank == 0 else 0
+    value = n_total * args.steps / (ms / 1e3) / 1e9
+
+    # full-size sanity of the bench's own output (C5: the races injected by construction)
+    check = None
+    if rank == 0 and args.config == "c5":
+        from sesagen.configs import c5_truth
+        got = trace.races()
+        exp = c5_truth(n_total)
+        check = bool(got.tobytes() == exp.tobytes())
+        log(f"[bench] C5 races {len(got)} (expected {len(exp)}), identical to construction truth: {check}")
+
+    # roofline of the dominant kernel (the onesweep pass): algorithmic bytes / CUDA-event time per launch
+    peak, peak_src = measured_peak_hbm()
+    dom = max(kstats, key=lambda k: kstats[k]["ms"]) if kstats else None
+    roof = None
+    if "onesweep_pass" in kstats and kstats["onesweep_pass"]["launches"]:
+        o = kstats["onesweep_pass"]
+        ach = o["bytes"] / (o["ms"] / 1e3) / 1e9
+        trf = ncu_traffic(args.config, "onesweep_pass")
+        roof = {"bound": "hbm", "kernel": "onesweep_pass", "achieved": ach, "peak": peak, "unit": "GB/s",
+                "frac": ach / peak, "traffic": trf, "bytes_per_launch": o["bytes"] / o["launches"],
+                "ms_per_launch": o["ms"] / o["launches"], "peak_source": peak_src,
+                "share_of_step": o["ms"] / max(1e-9, sum(v["ms"] for v in kstats.values()))}
+    step_bytes = sum(v["bytes"] for v in kstats.values()) / max(1, args.steps)
+
+    # end-to-end through the public API with host buffers (H2D of the records + D2H of the race list each step)
+    e2e = None
+    if not args.no_e2e and rank == 0 and world == 1:
+        pinned = torch.empty(n_local * 32, dtype=torch.uint8, pin_memory=True)
+        pinned.copy_(recs)
+        torch.cuda.synchronize()
+        e_steps = max(1, min(args.steps, 3))
+        trace.check_host_ptr(pinned.data_ptr(), n_local)  # warm-up
+        trace.races()
+        t0 = time.perf_counter()
+        for _ in range(e_steps):
+            trace.check_host_ptr(pinned.data_ptr(), n_local, index_base=base)
+            rr = trace.races()
+        dt = time.perf_counter() - t0
+        e2e = {"value": n_total * e_steps / dt / 1e9, "unit": "Grec/s", "h2d_bytes_per_step": n_local * 32,
+               "d2h_bytes_per_step": int(len(rr) * 40), "steps": e_steps}
+        del pinned
+
+    cpu = None
+    if not args.no_cpu and rank == 0 and world == 1:
+        cpu = run_cpu_baseline(args.config, args.cpu_records)
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": "Grec/s", "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+                "scaling": "strong", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+                "config": {"workload": c["workload"], "n_records": n_total, "warp_size": c["ws"],
+                           "lockstep": c["ls"], "granularity": 4,
+                           "parallelism": f"location-hash sharding x{world}" if world > 1 else "single GPU",
+                           "l2": f"inputs {n_total * 32 / 1e9:.1f} GB >> 126 MB L2 (no flush needed)"
+                           if n_total * 32 > 1e9 else "inputs smaller than L2 (latency-bound config)",
+                           "sort_bits": info["sort_bits"], "sort_passes": info["sort_passes"],
+                           "races": n_races, "crossing_tiles": info["crossing_tiles"]},
+                "gpu_launches": launches, "roofline": roof,
+                "honesty": {"record_bytes_per_step": n_total * 32, "achieved_gbs_vs_32B_per_record":
+                            n_total * 32 / (ms / args.steps / 1e3) / 1e9,
+                            "frac_32B_per_record": n_total * 32 / (ms / args.steps / 1e3) / 1e9 / peak,
+                            "algorithmic_bytes_per_step": step_bytes,
+                            "frac_algorithmic": step_bytes / (ms / args.steps / 1e3) / 1e9 / peak},
+                "kernels": {k: dict(launches=v["launches"], ms_per_step=v["ms"] / args.steps,
+                                    gbs=(v["bytes"] / (v["ms"] / 1e3) / 1e9) if v["ms"] > 0 else None)
+                            for k, v in sorted(kstats.items(), key=lambda kv: -kv[1]["ms"])},
+                "dominant_kernel": dom, "e2e": e2e, "cpu_baseline": cpu, "clocks": clk.summary(),
+                "full_size_check": check}
+        print(json.dumps(line), flush=True)
+    trace.close()
+    if pg:
+        pg.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()
