@@ -147,6 +147,7 @@ typedef struct {
 
 typedef struct {
   uint64_t n_records, n_entries, n_races;
+  uint64_t n_multi;         /* entries at locations touched >= 2 times (the only ones that can race) */
   uint32_t sort_bits, pos_bits, digit_bits, sort_passes; /* key layout chosen by the extents pass   */
   uint32_t sorted_input;    /* records were (block, interval)-ordered                               */
   uint32_t launches;        /* kernels launched by the last check (all families)                    */

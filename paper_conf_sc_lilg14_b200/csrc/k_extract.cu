@@ -10,42 +10,61 @@ namespace sesa {
 // wrap — the bounds P:73 and the memory sorts of Fig. 3), and reduce per space: min/max granule,
 // block, interval; count entries (granules) and multi-granule records; detect (block, interval) order.
 // ------------------------------------------------------------------------------------------------------------
-template <int THREADS>
+template <int THREADS, int U>
 __global__ void __launch_bounds__(THREADS) extents_kernel(const Rec* __restrict__ rec, u64 n, u32 log2G,
                                                           Summary* __restrict__ out) {
   u64 bad = ~0ull, ent = 0, multi = 0, cnt[2] = {0, 0};
   u64 gmin[2] = {~0ull, ~0ull}, gmax[2] = {0, 0};
   u32 bmin[2] = {~0u, ~0u}, bmax[2] = {0, 0}, imin[2] = {~0u, ~0u}, imax[2] = {0, 0};
   u32 unsorted = 0;
-  const u64 stride = (u64)gridDim.x * THREADS;
-  for (u64 k = (u64)blockIdx.x * THREADS + threadIdx.x; k < n; k += stride) {
-    Rec r = load_rec(rec + k);
-    bool ok = r.space <= 1 && r.rw <= 2 && r.size >= 1 && r.addr <= ~0ull - (u64)(r.size - 1);
-    if (!ok) {
-      bad = bad < k ? bad : k;
-      continue;
+  const int lane = threadIdx.x & 31;
+  const u64 stride = (u64)gridDim.x * THREADS, gt = (u64)blockIdx.x * THREADS + threadIdx.x;
+  const u64 rounds = (n + stride * U - 1) / (stride * U);
+  for (u64 it = 0; it < rounds; it++) {
+    Rec r[U];
+#pragma unroll
+    for (int j = 0; j < U; j++) {  // U independent 32-byte loads in flight per thread
+      const u64 k = (it * U + j) * stride + gt;
+      if (k < n) r[j] = load_rec(rec + k);
     }
-    u64 glo = r.addr >> log2G, ghi = (r.addr + (u64)(r.size - 1)) >> log2G;
-    ent += ghi - glo + 1;
-    multi += ghi != glo;
-    int s = r.space;
-    cnt[s]++;
-    gmin[s] = min(gmin[s], glo);
-    gmax[s] = max(gmax[s], ghi);
-    bmin[s] = min(bmin[s], r.block);
-    bmax[s] = max(bmax[s], r.block);
-    imin[s] = min(imin[s], r.interval);
-    imax[s] = max(imax[s], r.interval);
-    if (k > 0) {
-      const uint4* q = reinterpret_cast<const uint4*>(rec + k - 1) + 1;  // (block, thread, interval, ...)
-      uint4 p = __ldg(q);
-      if (r.block < p.x || (r.block == p.x && r.interval < p.z)) unsorted = 1;
+#pragma unroll
+    for (int j = 0; j < U; j++) {
+      const u64 k = (it * U + j) * stride + gt;
+      const bool in = k < n;
+      // (block, interval) of record k-1: held by the previous lane, or loaded for lane 0
+      u32 pb = __shfl_up_sync(~0u, in ? r[j].block : 0u, 1), pi = __shfl_up_sync(~0u, in ? r[j].interval : 0u, 1);
+      if (!in) continue;
+      if (lane == 0 && k > 0) {
+        const uint4 q = __ldg(reinterpret_cast<const uint4*>(rec + k - 1) + 1);
+        pb = q.x, pi = q.z;
+      }
+      const Rec& x = r[j];
+      const bool ok = x.space <= 1 && x.rw <= 2 && x.size >= 1 && x.addr <= ~0ull - (u64)(x.size - 1);
+      if (!ok) {
+        bad = min(bad, k);
+        continue;
+      }
+      if (k > 0 && (x.block < pb || (x.block == pb && x.interval < pi))) unsorted = 1;
+      const u64 glo = x.addr >> log2G, ghi = (x.addr + (u64)(x.size - 1)) >> log2G;
+      ent += ghi - glo + 1;
+      multi += ghi != glo;
+#pragma unroll
+      for (int sp = 0; sp < 2; sp++) {  // static indices: no local-memory arrays
+        if (x.space != sp) continue;
+        cnt[sp]++;
+        gmin[sp] = min(gmin[sp], glo);
+        gmax[sp] = max(gmax[sp], ghi);
+        bmin[sp] = min(bmin[sp], x.block);
+        bmax[sp] = max(bmax[sp], x.block);
+        imin[sp] = min(imin[sp], x.interval);
+        imax[sp] = max(imax[sp], x.interval);
+      }
     }
   }
   // block reduction through warp shuffles then one atomic per field per CTA
   __shared__ u64 s64[THREADS / 32][9];
   __shared__ u32 s32[THREADS / 32][9];
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int warp = threadIdx.x >> 5;
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) {
     bad = min(bad, __shfl_xor_sync(~0u, bad, o));
@@ -103,13 +122,13 @@ __global__ void __launch_bounds__(THREADS) extents_kernel(const Rec* __restrict_
 }
 
 void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, int grid, cudaStream_t st) {
-  extents_kernel<256><<<grid, 256, 0, st>>>(rec, n, log2G, d_sum);
+  extents_kernel<256, 4><<<grid, 256, 0, st>>>(rec, n, log2G, d_sum);
 }
 
 // ------------------------------------------------------------------------------------------------------------
 // key extraction, 1 entry per record (every record within one granule): key = key_hi << pos_bits | pos, plus
 // the histogram of every radix digit the sort will use (onesweep's upfront histogram), accumulated per CTA in
-// shared memory with warp-aggregated (match_any) increments and flushed with one global atomic per bin.
+// shared memory with warp-aggregated (ballot-matched) increments and flushed with one global atomic per bin.
 // ------------------------------------------------------------------------------------------------------------
 template <int THREADS, int RB>
 __global__ void __launch_bounds__(THREADS) extract_1to1_kernel(const Rec* __restrict__ rec, u64 n, KeyLayout L,
@@ -119,22 +138,38 @@ __global__ void __launch_bounds__(THREADS) extract_1to1_kernel(const Rec* __rest
   extern __shared__ u32 sh[];  // [npass][RADIX]
   for (u32 i = threadIdx.x; i < npass * RADIX; i += THREADS) sh[i] = 0;
   __syncthreads();
-  const u64 stride = (u64)gridDim.x * THREADS;
-  const u64 nround = (n + stride - 1) / stride;
+  constexpr int U = 2;
+  const u64 stride = (u64)gridDim.x * THREADS, gt = (u64)blockIdx.x * THREADS + threadIdx.x;
+  const u64 nround = (n + stride * U - 1) / (stride * U);
   for (u64 it = 0; it < nround; it++) {
-    u64 k = it * stride + (u64)blockIdx.x * THREADS + threadIdx.x;
-    bool valid = k < n;
-    u64 key = 0;
-    if (valid) {
-      Rec r = load_rec(rec + k);
-      u64 g = r.addr >> L.log2G;
-      key = (key_hi_of(L, r.space, r.block, r.interval, g) << L.pos_bits) | k;
-      keys[k] = key;
+    Rec r[U];
+#pragma unroll
+    for (int j = 0; j < U; j++) {
+      const u64 k = (it * U + j) * stride + gt;
+      if (k < n) r[j] = load_rec(rec + k);
     }
-    for (u32 p = 0; p < npass; p++) {
-      u32 d = valid ? (u32)((key >> (L.pos_bits + p * RB)) & (RADIX - 1)) : RADIX;
-      unsigned peers = __match_any_sync(~0u, d);
-      if (valid && (threadIdx.x & 31) == 31 - __clz(peers)) atomicAdd(&sh[p * RADIX + d], __popc(peers));
+#pragma unroll
+    for (int j = 0; j < U; j++) {
+      const u64 k = (it * U + j) * stride + gt;
+      const bool valid = k < n;
+      u64 key = 0;
+      if (valid) {
+        key = (key_hi_of(L, r[j].space, r[j].block, r[j].interval, r[j].addr >> L.log2G) << L.pos_bits) | k;
+        __stcs(keys + k, key);
+      }
+      // warp-aggregated histogram increments: lanes with equal digits found by ballots (ALU pipe)
+      const unsigned vmask = __ballot_sync(~0u, valid);
+      for (u32 p = 0; p < npass; p++) {
+        const u32 d = (u32)((key >> (L.pos_bits + p * RB)) & (RADIX - 1));
+        unsigned peers = vmask;
+#pragma unroll
+        for (int b = 0; b < RB; b++) {
+          const bool bit = (d >> b) & 1u;
+          const unsigned mm = __ballot_sync(~0u, bit);
+          peers &= bit ? mm : ~mm;
+        }
+        if (valid && (threadIdx.x & 31) == 31 - __clz(peers)) atomicAdd(&sh[p * RADIX + d], __popc(peers));
+      }
     }
   }
   __syncthreads();

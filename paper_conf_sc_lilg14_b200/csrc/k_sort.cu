@@ -2,7 +2,7 @@
 //
 // One pass = one kernel: a CTA takes the next tile in launch order (atomic tile counter, so every predecessor
 // tile is resident or done: forward progress for the look-back), loads 16 keys per thread warp-striped
-// (coalesced 256-byte rows), ranks them per warp with __match_any_sync (stable: item-major, lane-minor),
+// (coalesced 256-byte rows), ranks them per warp with ballot bit-matching (stable: item-major, lane-minor),
 // publishes its per-digit counts, obtains the exclusive per-digit prefix of all earlier tiles by decoupled
 // look-back (Merrill & Garland single-pass scan, one 64-bit status word per (tile, digit) tagged with a pass
 // epoch so the array never needs clearing), scatters the tile into shared memory in digit order, and writes it
@@ -24,6 +24,20 @@ __device__ __forceinline__ u64 ld_relaxed(const u64* p) {
   u64 v;
   asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
+}
+
+// Lanes holding the same digit (stable peers) without __match_any_sync: MATCH runs on the slow ADU pipe on
+// sm_100 (ncu: 65-96% ADU busy), ballots run on the ALU pipe.  NB = digit bits to compare.
+template <int NB>
+__device__ __forceinline__ unsigned peers_of(u32 d) {
+  unsigned p = ~0u;
+#pragma unroll
+  for (int b = 0; b < NB; b++) {
+    const bool bit = (d >> b) & 1u;
+    const unsigned m = __ballot_sync(~0u, bit);
+    p &= bit ? m : ~m;
+  }
+  return p;
 }
 
 // global exclusive prefix of each pass's digit histogram -> bin_base[pass][digit]
@@ -73,7 +87,7 @@ __device__ __forceinline__ u32 block_excl_sum(u32 v, u32* scratch /* [THREADS/32
 }
 
 template <int THREADS, int ITEMS, bool VALS>
-__global__ void __launch_bounds__(THREADS) onesweep_kernel(const u64* __restrict__ kin, u64* __restrict__ kout,
+__global__ void __launch_bounds__(THREADS, 3) onesweep_kernel(const u64* __restrict__ kin, u64* __restrict__ kout,
                                                            const u32* __restrict__ vin, u32* __restrict__ vout,
                                                            u32 m, u32 shift, const u64* __restrict__ bin_base,
                                                            u64* __restrict__ lookback, u32* __restrict__ tile_ctr,
@@ -113,11 +127,12 @@ __global__ void __launch_bounds__(THREADS) onesweep_kernel(const u64* __restrict
   }
   // warp-level ranking: rank = (warp's running count of the digit) + (lower peers in this row)
   u32* wh = whist + warp * RADIX;
+  const bool full = tbase + TILE <= m;
 #pragma unroll
   for (int i = 0; i < ITEMS; i++) {
-    const bool valid = wbase + (u64)i * 32 < m;
+    const bool valid = full || wbase + (u64)i * 32 < m;
     const u32 d = valid ? (u32)((k[i] >> shift) & (RADIX - 1)) : (u32)RADIX;
-    const unsigned peers = __match_any_sync(~0u, d);
+    const unsigned peers = full ? peers_of<RADIX_BITS>(d) : peers_of<RADIX_BITS + 1>(d);
     u32 c = valid ? wh[d] : 0u;
     rk[i] = c + __popc(peers & lanemask_lt());
     __syncwarp();

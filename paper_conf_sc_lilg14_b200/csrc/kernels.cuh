@@ -96,6 +96,11 @@ void launch_cross_emit(const ConflictArgs& a, u32 ntiles, cudaStream_t st);
 void launch_permute_races(const RaceOut* in, const u32* order, RaceOut* out, u32 nr, cudaStream_t st);
 u32 conflict_tiles(u64 m);
 
+// k_compact.cu — keep only entries of locations touched >= 2 times (order preserved); *total = count
+size_t compact_temp_bytes(u64 m);
+void launch_compact_multi(const u64* keys, u32 m, const KeyLayout& L, u64* out, void* temp, u32* total,
+                          cudaStream_t st);
+
 // k_expand.cu — cells (block, interval slot, thread); descriptors of slot q are idx[ivoff[q] .. ivoff[q+1])
 void launch_flow_count2(const void* flows, const u32* ivoff, const u32* idx, u32 niv, u32 bmin, u64 ncell, u32 tmax,
                         u32* cnt, cudaStream_t st);

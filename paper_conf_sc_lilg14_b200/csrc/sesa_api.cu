@@ -273,11 +273,21 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
     passes_run++;
   }
   info.sort_passes = passes_run;
-  const u64* sorted = (const u64*)b_keys[cur].p;
+
+  // 4a. keep only entries of locations touched at least twice (order-preserving compaction)
+  if (!grow(b_ctmp, compact_temp_bytes(m), "compact temp") || !grow(b_ctotal, 16, "compact count")) return status;
+  u64* comp = (u64*)b_keys[cur ^ 1].p;
+  LAUNCH("compact", 8.0 * m, launch_compact_multi((const u64*)b_keys[cur].p, (u32)m, L, comp, b_ctmp.p,
+                                                  (u32*)b_ctotal.p, stream));
+  u32 m2 = 0;
+  if (!cuda_ok(cudaMemcpyAsync(&m2, b_ctotal.p, 4, cudaMemcpyDeviceToHost, stream), "compact count")) return status;
+  if (!sync_check("compact")) return status;
+  info.n_multi = m2;
+  const u64* sorted = comp;
 
   // 4. conflict tiles
-  const u32 ctiles = conflict_tiles(m);
-  u32 race_cap = (u32)std::min<u64>(std::max<u64>(race_cap_hint, 1u << 16), 2 * m + 16);
+  const u32 ctiles = conflict_tiles(m2);
+  u32 race_cap = (u32)std::min<u64>(std::max<u64>(race_cap_hint, 1u << 16), 2 * (u64)m2 + 16);
   for (int attempt = 0; attempt < 3; attempt++) {
     if (!grow(b_tflags, ctiles, "tile flags") || !grow(b_part, (size_t)ctiles * sizeof(AggQuad), "partials") ||
         !grow(b_carry, (size_t)ctiles * sizeof(AggQuad), "carries") || !grow(b_owner, (size_t)ctiles * 4, "owner") ||
@@ -291,7 +301,7 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
     ConflictArgs A;
     memset(&A, 0, sizeof A);
     A.keys = sorted;
-    A.m = (u32)m;
+    A.m = m2;
     A.rec = rec;
     A.n = n;
     A.L = L;
@@ -310,7 +320,7 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
     A.owner = (u32*)b_owner.p;
     A.slots = (Slot*)b_slots.p;
     A.index_base = index_base;
-    LAUNCH("conflict", 8.0 * m, launch_conflict(1, A, ctiles, stream));
+    LAUNCH("conflict", 40.0 * m2, launch_conflict(1, A, ctiles, stream));
     u32 cc[2];
     if (!cuda_ok(cudaMemcpyAsync(cc, b_ccount.p, 8, cudaMemcpyDeviceToHost, stream), "counts")) return status;
     if (!sync_check("conflict")) return status;
@@ -327,7 +337,7 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
       n_races = cc[0];
       break;
     }
-    race_cap = (u32)std::min<u64>((u64)cc[0] + cc[0] / 8 + 1024, 2 * m + 16);
+    race_cap = (u32)std::min<u64>((u64)cc[0] + cc[0] / 8 + 1024, 2 * (u64)m2 + 16);
     race_cap_hint = race_cap;
   }
 

@@ -42,7 +42,7 @@ struct sesa_trace {
   DevBuf b_summary, b_keys[2], b_hist, b_binbase, b_lookback, b_ctr, b_cnt, b_off, b_temp;
   DevBuf b_tflags, b_part, b_carry, b_owner, b_slots, b_cross, b_ccount, b_carrytmp;
   DevBuf b_races, b_rkeys[2], b_rvals[2], b_races_sorted, b_rhist, b_rbase;
-  DevBuf b_eoff, b_ecnt, b_ecell, b_hrec, b_dist_races;
+  DevBuf b_eoff, b_ecnt, b_ecell, b_hrec, b_dist_races, b_ctmp, b_ctotal;
   DevBuf b_dist[8];
   void* h_pinned = nullptr;
 
@@ -50,7 +50,7 @@ struct sesa_trace {
     std::vector<DevBuf*> v = {&b_summary, &b_hist, &b_binbase, &b_lookback, &b_ctr, &b_cnt, &b_off, &b_temp,
                               &b_tflags, &b_part, &b_carry, &b_owner, &b_slots, &b_cross, &b_ccount, &b_carrytmp,
                               &b_races, &b_races_sorted, &b_rhist, &b_rbase, &b_eoff, &b_ecnt, &b_ecell,
-                              &b_hrec, &b_dist_races};
+                              &b_hrec, &b_dist_races, &b_ctmp, &b_ctotal};
     for (auto& b : b_keys) v.push_back(&b);
     for (auto& b : b_rkeys) v.push_back(&b);
     for (auto& b : b_rvals) v.push_back(&b);
