@@ -103,6 +103,38 @@ __host__ __device__ __forceinline__ u64 sesa_mix(u64 x) {
   return x ^ (x >> 31);
 }
 
+// ---- decoupled look-back (Merrill & Garland) for one scalar per tile, done by one whole warp ------------------
+// Status word: bits 63..62 = 1 (tile aggregate) | 2 (inclusive prefix), low 62 bits = value; 0 = not yet
+// published.  The warp inspects 32 predecessors per step (one per lane) instead of walking them one by one.
+// All 32 lanes of the calling warp must call it; returns the exclusive prefix of `tile`.
+__device__ __forceinline__ u64 warp_lookback(u64* lb, u32 tile, u64 agg) {
+  const int lane = threadIdx.x & 31;
+  volatile u64* v = lb;
+  if (lane == 0) v[tile] = ((tile == 0 ? 2ull : 1ull) << 62) | agg;
+  if (tile == 0) return 0;
+  u64 excl = 0;
+  long long base = (long long)tile - 1;
+  while (true) {
+    const long long p = base - lane;
+    u64 w = 2ull << 62;  // "prefix 0" before tile 0
+    if (p >= 0) {
+      do {
+        w = v[p];
+      } while ((w >> 62) == 0);
+    }
+    const unsigned pre = __ballot_sync(~0u, (w >> 62) == 2);
+    const int first = pre ? __ffs(pre) - 1 : 31;  // nearest predecessor holding an inclusive prefix
+    u64 x = lane <= first ? (w & ((1ull << 62) - 1)) : 0ull;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(~0u, x, o);
+    excl += x;
+    if (pre) break;
+    base -= 32;
+  }
+  if (lane == 0) v[tile] = (2ull << 62) | (excl + agg);
+  return excl;
+}
+
 // ---- device summary written by the extents pass ------------------------------------------------------------
 struct Summary {
   unsigned long long bad_index;  // lowest invalid record index (~0 = none)

@@ -49,34 +49,21 @@ __global__ void __launch_bounds__(CP_THREADS) compact_multi_kernel(const u64* __
   }
   if (lane == 31) s_w[warp] = x;
   __syncthreads();
-  if (tid == 0) {
+  if (warp == 0) {
     u32 acc = 0;
-    for (int w = 0; w < CP_THREADS / 32; w++) {
-      const u32 t = s_w[w];
-      s_w[w] = acc;
-      acc += t;
-    }
-    // look-back: status 1 = tile aggregate, 2 = inclusive prefix (value in the low 62 bits)
-    volatile u64* v = lb;
-    if (tile == 0) {
-      v[0] = (2ull << 62) | acc;
-      s_base = 0;
-    } else {
-      v[tile] = (1ull << 62) | acc;
-      u64 ex = 0;
-      long long p = (long long)tile - 1;
-      while (true) {
-        const u64 w = v[p];
-        const u64 st = w >> 62;
-        if (st == 0) continue;
-        ex += w & ((1ull << 62) - 1);
-        if (st == 2) break;
-        p--;
+    if (lane == 0) {
+      for (int w = 0; w < CP_THREADS / 32; w++) {
+        const u32 t = s_w[w];
+        s_w[w] = acc;
+        acc += t;
       }
-      v[tile] = (2ull << 62) | (ex + acc);
-      s_base = ex;
     }
-    if (tb + cnt >= m) *total = (u32)(s_base + acc);  // last tile publishes the count
+    acc = __shfl_sync(~0u, acc, 0);
+    const u64 ex = warp_lookback(lb, tile, acc);
+    if (lane == 0) {
+      s_base = ex;
+      if (tb + cnt >= m) *total = (u32)(ex + acc);  // the last tile publishes the count
+    }
   }
   __syncthreads();
   u32 o = s_w[warp] + x - c;

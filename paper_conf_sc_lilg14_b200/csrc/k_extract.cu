@@ -1,6 +1,8 @@
 // k_extract.cu — record validation + extents and key extraction with upfront digit
 // histograms (row a2).  Both are HBM-streaming passes over the 32-byte records: one 32-byte sector per record,
 // read with two 16-byte vector loads, grid sized to a multiple of the 148 SMs.
+#include <cstdlib>
+
 #include "kernels.cuh"
 
 namespace sesa {
@@ -130,14 +132,16 @@ void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, int grid, 
 // the histogram of every radix digit the sort will use (onesweep's upfront histogram), accumulated per CTA in
 // shared memory with warp-aggregated (ballot-matched) increments and flushed with one global atomic per bin.
 // ------------------------------------------------------------------------------------------------------------
-template <int THREADS, int RB>
+template <int THREADS, int RB, int HIST>
 __global__ void __launch_bounds__(THREADS) extract_1to1_kernel(const Rec* __restrict__ rec, u64 n, KeyLayout L,
                                                                 u32 npass, u64* __restrict__ keys,
                                                                 u32* __restrict__ hist /* [npass][1<<RB] */) {
   constexpr int RADIX = 1 << RB;
-  extern __shared__ u32 sh[];  // [npass][RADIX]
-  for (u32 i = threadIdx.x; i < npass * RADIX; i += THREADS) sh[i] = 0;
+  extern __shared__ u32 sh[];  // [npass][RADIX] (HIST 0) or [warps][npass][RADIX] (HIST 1)
+  const u32 nsh = HIST == 1 ? npass * RADIX * (THREADS / 32) : npass * RADIX;
+  for (u32 i = threadIdx.x; i < nsh; i += THREADS) sh[i] = 0;
   __syncthreads();
+  u32* wsh = sh + (HIST == 1 ? (threadIdx.x >> 5) * npass * RADIX : 0);
   constexpr int U = 2;
   const u64 stride = (u64)gridDim.x * THREADS, gt = (u64)blockIdx.x * THREADS + threadIdx.x;
   const u64 nround = (n + stride * U - 1) / (stride * U);
@@ -157,6 +161,11 @@ __global__ void __launch_bounds__(THREADS) extract_1to1_kernel(const Rec* __rest
         key = (key_hi_of(L, r[j].space, r[j].block, r[j].interval, r[j].addr >> L.log2G) << L.pos_bits) | k;
         __stcs(keys + k, key);
       }
+      if (HIST == 1) {  // per-warp private sub-histograms, plain shared-memory atomics
+        if (valid)
+          for (u32 p = 0; p < npass; p++) atomicAdd(&wsh[p * RADIX + ((key >> (L.pos_bits + p * RB)) & (RADIX - 1))], 1u);
+        continue;
+      }
       // warp-aggregated histogram increments: lanes with equal digits found by ballots (ALU pipe)
       const unsigned vmask = __ballot_sync(~0u, valid);
       for (u32 p = 0; p < npass; p++) {
@@ -173,14 +182,30 @@ __global__ void __launch_bounds__(THREADS) extract_1to1_kernel(const Rec* __rest
     }
   }
   __syncthreads();
-  for (u32 i = threadIdx.x; i < npass * RADIX; i += THREADS)
-    if (sh[i]) atomicAdd(&hist[i], sh[i]);
+  for (u32 i = threadIdx.x; i < npass * RADIX; i += THREADS) {
+    u32 v = sh[i];
+    if (HIST == 1)
+      for (int w = 1; w < THREADS / 32; w++) v += sh[w * npass * RADIX + i];
+    if (v) atomicAdd(&hist[i], v);
+  }
 }
 
 void launch_extract_1to1(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, u64* keys, u32* hist, int grid,
                          cudaStream_t st) {
-  size_t smem = (size_t)npass * (1 << RADIX_BITS) * sizeof(u32);
-  extract_1to1_kernel<256, RADIX_BITS><<<grid, 256, smem, st>>>(rec, n, L, npass, keys, hist);
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("SESA_HIST");
+    v = e ? atoi(e) : 1;
+  }
+  if (v == 1) {
+    size_t smem = (size_t)npass * (1 << RADIX_BITS) * sizeof(u32) * 8;
+    static bool set = false;
+    if (!set) cudaFuncSetAttribute(extract_1to1_kernel<256, RADIX_BITS, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024), set = true;
+    extract_1to1_kernel<256, RADIX_BITS, 1><<<grid, 256, smem, st>>>(rec, n, L, npass, keys, hist);
+  } else {
+    size_t smem = (size_t)npass * (1 << RADIX_BITS) * sizeof(u32);
+    extract_1to1_kernel<256, RADIX_BITS, 0><<<grid, 256, smem, st>>>(rec, n, L, npass, keys, hist);
+  }
 }
 
 // ------------------------------------------------------------------------------------------------------------

@@ -8,6 +8,8 @@
 // epoch so the array never needs clearing), scatters the tile into shared memory in digit order, and writes it
 // out so that each digit's run of the tile lands contiguously (coalesced stores).  Traffic per pass: 8 B read +
 // 8 B written per key (+4 + 4 with values); the look-back words add 8 B x 256 per 4096-key tile (~0.5 B/key).
+#include <cstdlib>
+
 #include "kernels.cuh"
 
 namespace sesa {
@@ -86,7 +88,7 @@ __device__ __forceinline__ u32 block_excl_sum(u32 v, u32* scratch /* [THREADS/32
   return scratch[warp] + x - v;
 }
 
-template <int THREADS, int ITEMS, bool VALS>
+template <int THREADS, int ITEMS, bool VALS, int MATCH>
 __global__ void __launch_bounds__(THREADS, 3) onesweep_kernel(const u64* __restrict__ kin, u64* __restrict__ kout,
                                                            const u32* __restrict__ vin, u32* __restrict__ vout,
                                                            u32 m, u32 shift, const u64* __restrict__ bin_base,
@@ -102,11 +104,14 @@ __global__ void __launch_bounds__(THREADS, 3) onesweep_kernel(const u64* __restr
   u32* bin_start = whist + WARPS * RADIX;                                       // [RADIX]
   long long* glob = reinterpret_cast<long long*>(bin_start + RADIX);            // [RADIX]
   u32* scratch = reinterpret_cast<u32*>(glob + RADIX);                          // [WARPS + 1]
+  u32* wmask = scratch + WARPS + 1;                                             // [WARPS][RADIX + 1] (MATCH 1)
   __shared__ u32 s_tile;
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   if (tid == 0) s_tile = atomicAdd(tile_ctr, 1u);
   for (int i = tid; i < WARPS * RADIX; i += THREADS) whist[i] = 0;
+  if (MATCH == 1)
+    for (int i = tid; i < WARPS * (RADIX + 1); i += THREADS) wmask[i] = 0;
   __syncthreads();
   const u32 tile = s_tile;
   const u64 tbase = (u64)tile * TILE;
@@ -132,7 +137,18 @@ __global__ void __launch_bounds__(THREADS, 3) onesweep_kernel(const u64* __restr
   for (int i = 0; i < ITEMS; i++) {
     const bool valid = full || wbase + (u64)i * 32 < m;
     const u32 d = valid ? (u32)((k[i] >> shift) & (RADIX - 1)) : (u32)RADIX;
-    const unsigned peers = full ? peers_of<RADIX_BITS>(d) : peers_of<RADIX_BITS + 1>(d);
+    unsigned peers;
+    if (MATCH == 0) {
+      peers = full ? peers_of<RADIX_BITS>(d) : peers_of<RADIX_BITS + 1>(d);
+    } else {
+      // each lane sets its bit in its digit's word of a per-warp mask array: the word becomes the peer set
+      u32* wm = wmask + warp * (RADIX + 1);
+      atomicOr(&wm[d], 1u << lane);
+      __syncwarp();
+      peers = wm[d];
+      __syncwarp();
+      if (lane == 31 - __clz(peers)) wm[d] = 0;
+    }
     u32 c = valid ? wh[d] : 0u;
     rk[i] = c + __popc(peers & lanemask_lt());
     __syncwarp();
@@ -197,32 +213,41 @@ template <bool VALS>
 static size_t onesweep_smem() {
   constexpr int WARPS = SORT_THREADS / 32;
   return (size_t)SORT_TILE * 8 + (VALS ? (size_t)SORT_TILE * 4 : 0) + (size_t)WARPS * RADIX * 4 + RADIX * 4 +
-         RADIX * 8 + (WARPS + 1) * 4;
+         RADIX * 8 + (WARPS + 1) * 4 + (size_t)WARPS * (RADIX + 1) * 4;
+}
+
+int sort_variant() {  // SESA_SORT_MATCH=0 ballots, 1 atomicOr masks (default)
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("SESA_SORT_MATCH");
+    v = e ? atoi(e) : 1;
+  }
+  return v;
+}
+
+template <bool VALS, int MATCH>
+static void launch_os(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m, u32 shift, const u64* bin_base,
+                      u64* lookback, u32* tile_ctr, u32 epoch, cudaStream_t st) {
+  auto kern = onesweep_kernel<SORT_THREADS, SORT_ITEMS, VALS, MATCH>;
+  const size_t sm = onesweep_smem<VALS>();
+  static bool set = false;
+  if (!set) {
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    set = true;
+  }
+  kern<<<sort_tiles(m), SORT_THREADS, sm, st>>>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch);
 }
 
 void launch_onesweep(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m, u32 shift, const u64* bin_base,
                      u64* lookback, u32* tile_ctr, u32 epoch, cudaStream_t st) {
-  const u32 tiles = sort_tiles(m);
-  if (!tiles) return;
+  if (!sort_tiles(m)) return;
+  const bool ballot = sort_variant() == 0;
   if (vin) {
-    auto kern = onesweep_kernel<SORT_THREADS, SORT_ITEMS, true>;
-    size_t sm = onesweep_smem<true>();
-    static bool set = false;
-    if (!set) {
-      cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-      set = true;
-    }
-    kern<<<tiles, SORT_THREADS, sm, st>>>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch);
+    if (ballot) launch_os<true, 0>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
+    else launch_os<true, 1>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
   } else {
-    auto kern = onesweep_kernel<SORT_THREADS, SORT_ITEMS, false>;
-    size_t sm = onesweep_smem<false>();
-    static bool set = false;
-    if (!set) {
-      cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-      set = true;
-    }
-    kern<<<tiles, SORT_THREADS, sm, st>>>(kin, kout, nullptr, nullptr, m, shift, bin_base, lookback, tile_ctr,
-                                          epoch);
+    if (ballot) launch_os<false, 0>(kin, kout, nullptr, nullptr, m, shift, bin_base, lookback, tile_ctr, epoch, st);
+    else launch_os<false, 1>(kin, kout, nullptr, nullptr, m, shift, bin_base, lookback, tile_ctr, epoch, st);
   }
 }
 

@@ -29,33 +29,18 @@ __global__ void __launch_bounds__(SCAN_THREADS) scan_u32_kernel(const u32* __res
   }
   if (lane == 31) s_w[warp] = x;
   __syncthreads();
-  if (tid == 0) {
+  if (warp == 0) {
     u32 acc = 0;
-    for (int w = 0; w < SCAN_THREADS / 32; w++) {
-      u32 c = s_w[w];
-      s_w[w] = acc;
-      acc += c;
-    }
-    // look-back: status 1 = aggregate, 2 = inclusive prefix (value in the low 62 bits)
-    volatile u64* vlb = lb;
-    if (tile == 0) {
-      vlb[0] = (2ull << 62) | acc;
-      s_prefix = 0;
-    } else {
-      vlb[tile] = (1ull << 62) | acc;
-      u64 ex = 0;
-      long long p = (long long)tile - 1;
-      while (true) {
-        const u64 w = vlb[p];
-        const u64 st = w >> 62;
-        if (st == 0) continue;
-        ex += w & ((1ull << 62) - 1);
-        if (st == 2) break;
-        p--;
+    if (lane == 0) {
+      for (int w = 0; w < SCAN_THREADS / 32; w++) {
+        u32 c = s_w[w];
+        s_w[w] = acc;
+        acc += c;
       }
-      vlb[tile] = (2ull << 62) | (ex + acc);
-      s_prefix = ex;
     }
+    acc = __shfl_sync(~0u, acc, 0);
+    const u64 ex = warp_lookback(lb, tile, acc);
+    if (lane == 0) s_prefix = ex;
   }
   __syncthreads();
   u32 run = (u32)s_prefix + s_w[warp] + x - sum;
