@@ -23,7 +23,11 @@ __global__ void __launch_bounds__(CP_THREADS) compact_multi_kernel(const u64* __
   const u32 tile = s_tile;
   const u64 tb = (u64)tile * CP_TILE;
   const u32 cnt = (u32)min((u64)CP_TILE, (u64)m - tb);
-  for (u32 j = tid; j < cnt; j += CP_THREADS) sk[j + 1] = __ldcs(keys + tb + j);
+#pragma unroll
+  for (int q = 0; q < CP_ITEMS; q++) {  // compile-time trip count: all 8 loads in flight
+    const u32 j = q * CP_THREADS + tid;
+    if (j < cnt) sk[j + 1] = __ldcs(keys + tb + j);
+  }
   if (tid == 0) {
     sk[0] = tb > 0 ? keys[tb - 1] : 0ull;
     sk[cnt + 1] = tb + cnt < m ? keys[tb + cnt] : 0ull;

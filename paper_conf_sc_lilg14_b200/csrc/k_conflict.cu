@@ -265,7 +265,11 @@ __device__ __forceinline__ u32 pos_of(const KeyLayout& L, u64 key) { return (u32
 __device__ bool tile_load(const ConflictArgs& a, TileSmem& s, u64 tb, u32 cnt) {
   const KeyLayout& L = a.L;
   const int tid = threadIdx.x;
-  for (u32 j = tid; j < cnt; j += CT_THREADS) s.key[j + 1] = __ldcs(a.keys + tb + j);
+#pragma unroll
+  for (int q = 0; q < CT_ITEMS; q++) {  // compile-time trip count: all loads in flight
+    const u32 j = q * CT_THREADS + tid;
+    if (j < cnt) s.key[j + 1] = __ldcs(a.keys + tb + j);
+  }
   if (tid == 0) {
     s.key[0] = tb > 0 ? a.keys[tb - 1] : 0ull;
     s.key[cnt + 1] = tb + cnt < a.m ? a.keys[tb + cnt] : 0ull;

@@ -130,9 +130,28 @@ __global__ void __launch_bounds__(THREADS, 3) onesweep_kernel(const u64* __restr
       k[i] = ~0ull;
     }
   }
-  // warp-level ranking: rank = (warp's running count of the digit) + (lower peers in this row)
   u32* wh = whist + warp * RADIX;
   const bool full = tbase + TILE <= m;
+  // (1) early counts: per-warp digit histogram with shared-memory atomics (no ordering needed for counts)
+#pragma unroll
+  for (int i = 0; i < ITEMS; i++)
+    if (full || wbase + (u64)i * 32 < m) atomicAdd(&wh[(u32)((k[i] >> shift) & (RADIX - 1))], 1u);
+  __syncthreads();
+  // (2) per-digit tile totals -> publish the tile aggregate BEFORE ranking, so that successor tiles find it
+  //     during their look-back; per-warp counts become exclusive offsets across warps
+  u32 tot = 0;
+  if (tid < RADIX) {
+#pragma unroll
+    for (int w = 0; w < WARPS; w++) {
+      u32 c = whist[w * RADIX + tid];
+      whist[w * RADIX + tid] = tot;
+      tot += c;
+    }
+    st_relaxed(lookback + (u64)tile * RADIX + tid, lb_pack(tile == 0 ? LB_PREFIX : LB_AGG, epoch, tot));
+  }
+  const u32 bs = block_excl_sum<THREADS>(tid < RADIX ? tot : 0u, scratch);  // (contains __syncthreads)
+  if (tid < RADIX) bin_start[tid] = bs;
+  // (3) stable warp-level ranking: running per-warp digit counter (starts at the warp's offset) + lower peers
 #pragma unroll
   for (int i = 0; i < ITEMS; i++) {
     const bool valid = full || wbase + (u64)i * 32 < m;
@@ -155,31 +174,18 @@ __global__ void __launch_bounds__(THREADS, 3) onesweep_kernel(const u64* __restr
     if (valid && lane == 31 - __clz(peers)) wh[d] = c + __popc(peers);
     __syncwarp();
   }
-  __syncthreads();
-  // per-digit tile totals; per-warp counts -> exclusive offsets across warps
-  u32 tot = 0;
+  // (4) look-back for the exclusive prefix of every digit over earlier tiles (by now mostly published)
   if (tid < RADIX) {
-#pragma unroll
-    for (int w = 0; w < WARPS; w++) {
-      u32 c = whist[w * RADIX + tid];
-      whist[w * RADIX + tid] = tot;
-      tot += c;
-    }
-    st_relaxed(lookback + (u64)tile * RADIX + tid, lb_pack(tile == 0 ? LB_PREFIX : LB_AGG, epoch, tot));
-  }
-  const u32 bs = block_excl_sum<THREADS>(tid < RADIX ? tot : 0u, scratch);
-  if (tid < RADIX) {
-    bin_start[tid] = bs;
     u64 excl = 0;
     if (tile > 0) {
       long long p = (long long)tile - 1;
       while (true) {
         const u64 w = ld_relaxed(lookback + (u64)p * RADIX + tid);
         const u32 e = (u32)((w >> 54) & 0xFF);
-        const u64 s = w & (3ull << 62);
-        if (e != epoch || s == 0) continue;  // predecessor has not published yet: spin
+        const u64 st = w & (3ull << 62);
+        if (e != epoch || st == 0) continue;  // predecessor has not published yet: spin
         excl += w & LB_VAL;
-        if (s == LB_PREFIX) break;
+        if (st == LB_PREFIX) break;
         p--;
       }
       st_relaxed(lookback + (u64)tile * RADIX + tid, lb_pack(LB_PREFIX, epoch, excl + tot));
@@ -192,7 +198,7 @@ __global__ void __launch_bounds__(THREADS, 3) onesweep_kernel(const u64* __restr
   for (int i = 0; i < ITEMS; i++) {
     if (wbase + (u64)i * 32 < m) {
       const u32 d = (u32)((k[i] >> shift) & (RADIX - 1));
-      const u32 pos = bin_start[d] + whist[warp * RADIX + d] + rk[i];
+      const u32 pos = bin_start[d] + rk[i];
       keys_s[pos] = k[i];
       if (VALS) vals_s[pos] = v[i];
     }
