@@ -12,6 +12,7 @@
 // run the entries of one (block, interval) — a "sub-run" — are contiguous.
 #pragma once
 #include <cstdint>
+#include <cstdlib>
 #include <cuda_runtime.h>
 
 typedef uint64_t u64;
@@ -84,6 +85,13 @@ __device__ __forceinline__ u64 group_of_hi(const KeyLayout& L, u64 hi) {
   return space_of_hi(L, hi) == SP_GLOBAL ? (hi & ~lowmask(L.lowG)) : hi;
 }
 
+// same location run?  (sorted keys a, b; the run key drops the position bits and, for an unsorted-input global
+// layout, the (block, interval) bits; different spaces differ in the space bit, which no mask clears)
+__device__ __forceinline__ bool same_group(const KeyLayout& L, u64 a, u64 b) {
+  const bool glob = L.both ? ((a >> (L.space_shift + L.pos_bits)) & 1ull) != 0 : L.single_space == SP_GLOBAL;
+  return ((a ^ b) >> (L.pos_bits + (glob ? L.lowG : 0u))) == 0;
+}
+
 __device__ __forceinline__ u64 granule_of_hi(const KeyLayout& L, u64 hi) {
   if (space_of_hi(L, hi) == SP_SHARED) return (hi & lowmask(L.gbS)) + L.gminS;
   return ((hi >> L.lowG) & lowmask(L.gbG)) + L.gminG;
@@ -103,11 +111,94 @@ __host__ __device__ __forceinline__ u64 sesa_mix(u64 x) {
   return x ^ (x >> 31);
 }
 
+// tile ids of the single-pass scans: 1 = atomic counter, 0 = blockIdx.x (dispatch order); env SESA_TILE_ATOMIC
+inline int tile_atomic_mode() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("SESA_TILE_ATOMIC");
+    v = e ? atoi(e) : 1;
+  }
+  return v;
+}
+
+// ---- TMA bulk copies (cp.async.bulk, 1-D: no tensor map) completing on an mbarrier -------------------------
+__device__ __forceinline__ u32 smem_u32(const void* p) { return (u32)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(u64* bar, u32 count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
+__device__ __forceinline__ void mbar_expect_tx(u64* bar, u32 bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+// bytes must be a multiple of 16, both addresses 16-byte aligned
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, u32 bytes, u64* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(u64* bar, u32 parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n WAIT_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra WAIT_%=;\n}" ::"r"(
+          smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+
+// ---- TMA streaming ring: a persistent CTA walks chunks c = blockIdx.x + j*gridDim.x, keeping STAGES chunks in
+// flight with cp.async.bulk (bytes in flight do not cost registers).  Usage:
+//   BulkRing<S> ring(smem_bufs, bars, chunk_bytes);  ring.start(src, nbytes_total)   (all threads)
+//   for (j = 0; ring.next(j); j++) { const char* data = ring.wait(j); ...; ring.release(j); }
+template <int STAGES>
+struct BulkRing {
+  unsigned char* buf;  // [STAGES][chunk]
+  u64* bar;            // [STAGES]
+  u32 chunk;           // bytes per chunk (multiple of 16)
+  const unsigned char* src;
+  u64 total;           // bytes
+  u64 nchunks;
+  __device__ __forceinline__ BulkRing(unsigned char* b, u64* br, u32 ch) : buf(b), bar(br), chunk(ch) {}
+  __device__ __forceinline__ void issue(u64 j) {  // thread 0: chunk #j of this CTA into slot j % STAGES
+    const u64 c = blockIdx.x + j * gridDim.x;
+    if (c >= nchunks) return;
+    const u64 off = c * chunk;
+    const u32 bytes = (u32)((min((u64)chunk, total - off) + 15) & ~15ull);
+    const int slot = (int)(j % STAGES);
+    mbar_expect_tx(&bar[slot], bytes);
+    bulk_g2s(buf + (size_t)slot * chunk, src + off, bytes, &bar[slot]);
+  }
+  __device__ __forceinline__ void start(const void* s, u64 nbytes) {
+    src = reinterpret_cast<const unsigned char*>(s);
+    total = nbytes;
+    nchunks = (nbytes + chunk - 1) / chunk;
+    if (threadIdx.x == 0) {
+      for (int i = 0; i < STAGES; i++) mbar_init(&bar[i], 1);
+      fence_mbar_init();
+      for (int i = 0; i < STAGES; i++) issue(i);
+    }
+    __syncthreads();
+  }
+  __device__ __forceinline__ bool next(u64 j) const { return blockIdx.x + j * gridDim.x < nchunks; }
+  __device__ __forceinline__ u64 chunk_index(u64 j) const { return blockIdx.x + j * gridDim.x; }
+  __device__ __forceinline__ u32 chunk_bytes(u64 j) const {
+    return (u32)min((u64)chunk, total - chunk_index(j) * chunk);
+  }
+  __device__ __forceinline__ const unsigned char* wait(u64 j) {
+    const int slot = (int)(j % STAGES);
+    mbar_wait(&bar[slot], (u32)((j / STAGES) & 1));
+    return buf + (size_t)slot * chunk;
+  }
+  __device__ __forceinline__ void release(u64 j) {  // all threads: slot j % STAGES may be refilled
+    __syncthreads();
+    if (threadIdx.x == 0) issue(j + STAGES);
+  }
+};
+
 // ---- decoupled look-back (Merrill & Garland) for one scalar per tile, done by one whole warp ------------------
 // Status word: bits 63..62 = 1 (tile aggregate) | 2 (inclusive prefix), low 62 bits = value; 0 = not yet
 // published.  The warp inspects 32 predecessors per step (one per lane) instead of walking them one by one.
 // All 32 lanes of the calling warp must call it; returns the exclusive prefix of `tile`.
-__device__ __forceinline__ u64 warp_lookback(u64* lb, u32 tile, u64 agg) {
+__device__ __forceinline__ u64 warp_lookback(u64* lb, u32 tile, u64 agg, unsigned long long* dbg = nullptr) {
   const int lane = threadIdx.x & 31;
   volatile u64* v = lb;
   if (lane == 0) v[tile] = ((tile == 0 ? 2ull : 1ull) << 62) | agg;
@@ -118,10 +209,16 @@ __device__ __forceinline__ u64 warp_lookback(u64* lb, u32 tile, u64 agg) {
     const long long p = base - lane;
     u64 w = 2ull << 62;  // "prefix 0" before tile 0
     if (p >= 0) {
-      do {
+      int spins = 0;
+      while (true) {
         w = v[p];
-      } while ((w >> 62) == 0);
+        spins++;
+        if ((w >> 62) != 0) break;
+        __nanosleep(spins < 4 ? 32 : 128);  // back off: spinning warps otherwise flood L2
+      }
+      if (dbg) atomicAdd(&dbg[1], (unsigned long long)spins);
     }
+    if (dbg && lane == 0) atomicAdd(&dbg[0], 1ull);
     const unsigned pre = __ballot_sync(~0u, (w >> 62) == 2);
     const int first = pre ? __ffs(pre) - 1 : 31;  // nearest predecessor holding an inclusive prefix
     u64 x = lane <= first ? (w & ((1ull << 62) - 1)) : 0ull;

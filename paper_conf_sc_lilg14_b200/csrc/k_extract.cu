@@ -1,6 +1,7 @@
 // k_extract.cu — record validation + extents and key extraction with upfront digit
 // histograms (row a2).  Both are HBM-streaming passes over the 32-byte records: one 32-byte sector per record,
 // read with two 16-byte vector loads, grid sized to a multiple of the 148 SMs.
+#include <algorithm>
 #include <cstdlib>
 
 #include "kernels.cuh"
@@ -12,6 +13,10 @@ namespace sesa {
 // wrap — the bounds P:73 and the memory sorts of Fig. 3), and reduce per space: min/max granule,
 // block, interval; count entries (granules) and multi-granule records; detect (block, interval) order.
 // ------------------------------------------------------------------------------------------------------------
+constexpr int EX_STAGES = 4, EX_CHUNK = 16384, EX_RECS = EX_CHUNK / 32;
+
+// Register version (measured faster than a TMA ring here: the per-record reductions are ALU-heavy and the ring's
+// strided shared-memory reads and barriers cost more than they save).
 template <int THREADS, int U>
 __global__ void __launch_bounds__(THREADS) extents_kernel(const Rec* __restrict__ rec, u64 n, u32 log2G,
                                                           Summary* __restrict__ out) {
@@ -67,6 +72,7 @@ __global__ void __launch_bounds__(THREADS) extents_kernel(const Rec* __restrict_
   __shared__ u64 s64[THREADS / 32][9];
   __shared__ u32 s32[THREADS / 32][9];
   const int warp = threadIdx.x >> 5;
+  (void)lane;
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) {
     bad = min(bad, __shfl_xor_sync(~0u, bad, o));
@@ -123,6 +129,15 @@ __global__ void __launch_bounds__(THREADS) extents_kernel(const Rec* __restrict_
   }
 }
 
+static int ring_grid(const void* kern, int threads, size_t smem, size_t smem_max) {
+  int dev = 0, sms = 148, per = 1;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_max);  // never lowered
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, kern, threads, smem);
+  return sms * (per > 0 ? per : 1);
+}
+
 void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, int grid, cudaStream_t st) {
   extents_kernel<256, 4><<<grid, 256, 0, st>>>(rec, n, log2G, d_sum);
 }
@@ -132,80 +147,53 @@ void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, int grid, 
 // the histogram of every radix digit the sort will use (onesweep's upfront histogram), accumulated per CTA in
 // shared memory with warp-aggregated (ballot-matched) increments and flushed with one global atomic per bin.
 // ------------------------------------------------------------------------------------------------------------
-template <int THREADS, int RB, int HIST>
+template <int THREADS, int RB>
 __global__ void __launch_bounds__(THREADS) extract_1to1_kernel(const Rec* __restrict__ rec, u64 n, KeyLayout L,
                                                                 u32 npass, u64* __restrict__ keys,
                                                                 u32* __restrict__ hist /* [npass][1<<RB] */) {
   constexpr int RADIX = 1 << RB;
-  extern __shared__ u32 sh[];  // [npass][RADIX] (HIST 0) or [warps][npass][RADIX] (HIST 1)
-  const u32 nsh = HIST == 1 ? npass * RADIX * (THREADS / 32) : npass * RADIX;
+  extern __shared__ __align__(128) unsigned char smem[];
+  __shared__ u64 bars[EX_STAGES];
+  u32* sh = reinterpret_cast<u32*>(smem + (size_t)EX_STAGES * EX_CHUNK);  // [warps][npass][RADIX]
+  const u32 nsh = npass * RADIX * (THREADS / 32);
   for (u32 i = threadIdx.x; i < nsh; i += THREADS) sh[i] = 0;
-  __syncthreads();
-  u32* wsh = sh + (HIST == 1 ? (threadIdx.x >> 5) * npass * RADIX : 0);
-  constexpr int U = 2;
-  const u64 stride = (u64)gridDim.x * THREADS, gt = (u64)blockIdx.x * THREADS + threadIdx.x;
-  const u64 nround = (n + stride * U - 1) / (stride * U);
-  for (u64 it = 0; it < nround; it++) {
-    Rec r[U];
+  u32* wsh = sh + (threadIdx.x >> 5) * npass * RADIX;  // per-warp private sub-histograms: plain smem atomics
+  BulkRing<EX_STAGES> ring(smem, bars, EX_CHUNK);
+  ring.start(rec, n * 32);  // (contains __syncthreads)
+  for (u64 j = 0; ring.next(j); j++) {
+    const Rec* R = reinterpret_cast<const Rec*>(ring.wait(j));
+    const u64 c0 = ring.chunk_index(j) * EX_RECS;
+    const u32 nr = ring.chunk_bytes(j) / 32;
 #pragma unroll
-    for (int j = 0; j < U; j++) {
-      const u64 k = (it * U + j) * stride + gt;
-      if (k < n) r[j] = load_rec(rec + k);
+    for (int h = 0; h < EX_RECS / THREADS; h++) {
+      const u32 t = h * THREADS + threadIdx.x;
+      if (t >= nr) continue;
+      const Rec& x = R[t];
+      const u64 key = (key_hi_of(L, x.space, x.block, x.interval, x.addr >> L.log2G) << L.pos_bits) | (c0 + t);
+      __stcs(keys + c0 + t, key);
+      for (u32 p = 0; p < npass; p++) atomicAdd(&wsh[p * RADIX + ((key >> (L.pos_bits + p * RB)) & (RADIX - 1))], 1u);
     }
-#pragma unroll
-    for (int j = 0; j < U; j++) {
-      const u64 k = (it * U + j) * stride + gt;
-      const bool valid = k < n;
-      u64 key = 0;
-      if (valid) {
-        key = (key_hi_of(L, r[j].space, r[j].block, r[j].interval, r[j].addr >> L.log2G) << L.pos_bits) | k;
-        __stcs(keys + k, key);
-      }
-      if (HIST == 1) {  // per-warp private sub-histograms, plain shared-memory atomics
-        if (valid)
-          for (u32 p = 0; p < npass; p++) atomicAdd(&wsh[p * RADIX + ((key >> (L.pos_bits + p * RB)) & (RADIX - 1))], 1u);
-        continue;
-      }
-      // warp-aggregated histogram increments: lanes with equal digits found by ballots (ALU pipe)
-      const unsigned vmask = __ballot_sync(~0u, valid);
-      for (u32 p = 0; p < npass; p++) {
-        const u32 d = (u32)((key >> (L.pos_bits + p * RB)) & (RADIX - 1));
-        unsigned peers = vmask;
-#pragma unroll
-        for (int b = 0; b < RB; b++) {
-          const bool bit = (d >> b) & 1u;
-          const unsigned mm = __ballot_sync(~0u, bit);
-          peers &= bit ? mm : ~mm;
-        }
-        if (valid && (threadIdx.x & 31) == 31 - __clz(peers)) atomicAdd(&sh[p * RADIX + d], __popc(peers));
-      }
-    }
+    ring.release(j);
   }
   __syncthreads();
   for (u32 i = threadIdx.x; i < npass * RADIX; i += THREADS) {
-    u32 v = sh[i];
-    if (HIST == 1)
-      for (int w = 1; w < THREADS / 32; w++) v += sh[w * npass * RADIX + i];
+    u32 v = 0;
+    for (int w = 0; w < THREADS / 32; w++) v += sh[w * npass * RADIX + i];
     if (v) atomicAdd(&hist[i], v);
   }
 }
 
-void launch_extract_1to1(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, u64* keys, u32* hist, int grid,
+void launch_extract_1to1(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, u64* keys, u32* hist, int,
                          cudaStream_t st) {
-  static int v = -1;
-  if (v < 0) {
-    const char* e = getenv("SESA_HIST");
-    v = e ? atoi(e) : 1;
-  }
-  if (v == 1) {
-    size_t smem = (size_t)npass * (1 << RADIX_BITS) * sizeof(u32) * 8;
-    static bool set = false;
-    if (!set) cudaFuncSetAttribute(extract_1to1_kernel<256, RADIX_BITS, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024), set = true;
-    extract_1to1_kernel<256, RADIX_BITS, 1><<<grid, 256, smem, st>>>(rec, n, L, npass, keys, hist);
-  } else {
-    size_t smem = (size_t)npass * (1 << RADIX_BITS) * sizeof(u32);
-    extract_1to1_kernel<256, RADIX_BITS, 0><<<grid, 256, smem, st>>>(rec, n, L, npass, keys, hist);
-  }
+  static int grids[9] = {0};
+  const size_t sm = (size_t)EX_STAGES * EX_CHUNK + (size_t)npass * 8 * RADIX * 4;  // ring + npass x 8 warps hist
+  if (!grids[npass])
+    grids[npass] = ring_grid((const void*)extract_1to1_kernel<256, RADIX_BITS>, 256, sm,
+                             (size_t)EX_STAGES * EX_CHUNK + (size_t)8 * 8 * RADIX * 4);
+  const int grid = grids[npass];
+  const u64 chunks = (n * 32 + EX_CHUNK - 1) / EX_CHUNK;
+  extract_1to1_kernel<256, RADIX_BITS><<<(unsigned)std::min<u64>(chunks, (u64)grid), 256, sm, st>>>(rec, n, L, npass,
+                                                                                                   keys, hist);
 }
 
 // ------------------------------------------------------------------------------------------------------------

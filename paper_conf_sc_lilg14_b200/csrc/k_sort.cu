@@ -8,7 +8,10 @@
 // epoch so the array never needs clearing), scatters the tile into shared memory in digit order, and writes it
 // out so that each digit's run of the tile lands contiguously (coalesced stores).  Traffic per pass: 8 B read +
 // 8 B written per key (+4 + 4 with values); the look-back words add 8 B x 256 per 4096-key tile (~0.5 B/key).
+#include <algorithm>
+#include <cstdio>
 #include <cstdlib>
+#include <vector>
 
 #include "kernels.cuh"
 
@@ -22,6 +25,13 @@ __device__ __forceinline__ u64 lb_pack(u64 status, u32 epoch, u64 v) { return st
 __device__ __forceinline__ void st_relaxed(u64* p, u64 v) {
   asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
+__device__ __forceinline__ u64 gtime() {
+  u64 t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ unsigned long long* g_prof = nullptr;  // optional per-tile phase stamps (SESA_SORT_PROF)
+
 __device__ __forceinline__ u64 ld_relaxed(const u64* p) {
   u64 v;
   asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
@@ -88,12 +98,12 @@ __device__ __forceinline__ u32 block_excl_sum(u32 v, u32* scratch /* [THREADS/32
   return scratch[warp] + x - v;
 }
 
-template <int THREADS, int ITEMS, bool VALS, int MATCH>
-__global__ void __launch_bounds__(THREADS, 3) onesweep_kernel(const u64* __restrict__ kin, u64* __restrict__ kout,
+template <int THREADS, int ITEMS, bool VALS, int MATCH, int MINB>
+__global__ void __launch_bounds__(THREADS, MINB) onesweep_kernel(const u64* __restrict__ kin, u64* __restrict__ kout,
                                                            const u32* __restrict__ vin, u32* __restrict__ vout,
                                                            u32 m, u32 shift, const u64* __restrict__ bin_base,
                                                            u64* __restrict__ lookback, u32* __restrict__ tile_ctr,
-                                                           u32 epoch) {
+                                                           u32 epoch, int g_tile_atomic) {
   constexpr int WARPS = THREADS / 32;
   constexpr int TILE = THREADS * ITEMS;
   static_assert(RADIX <= THREADS, "one bin per thread");
@@ -105,15 +115,21 @@ __global__ void __launch_bounds__(THREADS, 3) onesweep_kernel(const u64* __restr
   long long* glob = reinterpret_cast<long long*>(bin_start + RADIX);            // [RADIX]
   u32* scratch = reinterpret_cast<u32*>(glob + RADIX);                          // [WARPS + 1]
   u32* wmask = scratch + WARPS + 1;                                             // [WARPS][RADIX + 1] (MATCH 1)
-  __shared__ u32 s_tile;
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  if (tid == 0) s_tile = atomicAdd(tile_ctr, 1u);
+  const u32 ntiles = (u32)((m + TILE - 1) / TILE);
+  // one tile per CTA; tile ids from an atomic counter = execution order (blockIdx order measured 45% slower:
+  // a tile whose predecessor was dispatched later spins in the look-back)
+  __shared__ u32 s_tile;
+  if (tid == 0) s_tile = g_tile_atomic ? atomicAdd(tile_ctr, 1u) : blockIdx.x;
+  __syncthreads();
+  for (u32 tile = s_tile; tile < ntiles; tile = ntiles) {
+  unsigned long long* prof = g_prof ? g_prof + (u64)tile * 8 : nullptr;
+  if (prof && tid == 0) prof[0] = gtime();
   for (int i = tid; i < WARPS * RADIX; i += THREADS) whist[i] = 0;
   if (MATCH == 1)
     for (int i = tid; i < WARPS * (RADIX + 1); i += THREADS) wmask[i] = 0;
   __syncthreads();
-  const u32 tile = s_tile;
   const u64 tbase = (u64)tile * TILE;
 
   u64 k[ITEMS];
@@ -132,6 +148,14 @@ __global__ void __launch_bounds__(THREADS, 3) onesweep_kernel(const u64* __restr
   }
   u32* wh = whist + warp * RADIX;
   const bool full = tbase + TILE <= m;
+  if (prof) {  // all keys of this thread have arrived
+    u64 sum = 0;
+#pragma unroll
+    for (int i = 0; i < ITEMS; i++) sum += k[i];
+    if (sum == 12345) prof[7] = 0;  // keep the loads ordered before the stamp
+    __syncthreads();
+    if (tid == 0) prof[1] = gtime();
+  }
   // (1) early counts: per-warp digit histogram with shared-memory atomics (no ordering needed for counts)
 #pragma unroll
   for (int i = 0; i < ITEMS; i++)
@@ -151,7 +175,45 @@ __global__ void __launch_bounds__(THREADS, 3) onesweep_kernel(const u64* __restr
   }
   const u32 bs = block_excl_sum<THREADS>(tid < RADIX ? tot : 0u, scratch);  // (contains __syncthreads)
   if (tid < RADIX) bin_start[tid] = bs;
-  // (3) stable warp-level ranking: running per-warp digit counter (starts at the warp's offset) + lower peers
+  if (prof && tid == 0) prof[2] = gtime();
+  // (3) look-back for the exclusive prefix of every digit over earlier tiles, right after publishing the
+  //     aggregate so that inclusive prefixes propagate with minimal delay; each bin-owner thread inspects 4
+  //     predecessors per round trip and backs off while they are unpublished
+  if (tid < RADIX) {
+    u64 excl = 0;
+    if (tile > 0) {
+      long long p = (long long)tile - 1;
+      int spins = 0;
+      while (true) {
+        u64 w[4];
+#pragma unroll
+        for (int q = 0; q < 4; q++) w[q] = p - q >= 0 ? ld_relaxed(lookback + (u64)(p - q) * RADIX + tid) : 0ull;
+        // consume predecessors in order while they are published; stop at the first inclusive prefix
+        int q = 0;
+        bool done = false;
+        for (; q < 4 && p - q >= 0; q++) {
+          const u32 e = (u32)((w[q] >> 54) & 0xFF);
+          const u64 st = w[q] & (3ull << 62);
+          if (e != epoch || st == 0) break;
+          excl += w[q] & LB_VAL;
+          if (st == LB_PREFIX) {
+            done = true;
+            break;
+          }
+        }
+        if (done) break;
+        if (q == 0) __nanosleep(++spins < 4 ? 32 : 128);
+        p -= q;
+      }
+      st_relaxed(lookback + (u64)tile * RADIX + tid, lb_pack(LB_PREFIX, epoch, excl + tot));
+    }
+    glob[tid] = (long long)(bin_base[tid] + excl) - (long long)bs;
+  }
+  if (prof) {
+    __syncthreads();
+    if (tid == 0) prof[3] = gtime();
+  }
+  // (4) stable warp-level ranking: running per-warp digit counter (starts at the warp's offset) + lower peers
 #pragma unroll
   for (int i = 0; i < ITEMS; i++) {
     const bool valid = full || wbase + (u64)i * 32 < m;
@@ -174,25 +236,8 @@ __global__ void __launch_bounds__(THREADS, 3) onesweep_kernel(const u64* __restr
     if (valid && lane == 31 - __clz(peers)) wh[d] = c + __popc(peers);
     __syncwarp();
   }
-  // (4) look-back for the exclusive prefix of every digit over earlier tiles (by now mostly published)
-  if (tid < RADIX) {
-    u64 excl = 0;
-    if (tile > 0) {
-      long long p = (long long)tile - 1;
-      while (true) {
-        const u64 w = ld_relaxed(lookback + (u64)p * RADIX + tid);
-        const u32 e = (u32)((w >> 54) & 0xFF);
-        const u64 st = w & (3ull << 62);
-        if (e != epoch || st == 0) continue;  // predecessor has not published yet: spin
-        excl += w & LB_VAL;
-        if (st == LB_PREFIX) break;
-        p--;
-      }
-      st_relaxed(lookback + (u64)tile * RADIX + tid, lb_pack(LB_PREFIX, epoch, excl + tot));
-    }
-    glob[tid] = (long long)(bin_base[tid] + excl) - (long long)bs;
-  }
   __syncthreads();
+  if (prof && tid == 0) prof[4] = gtime();
   // scatter into shared memory in (digit, stable) order
 #pragma unroll
   for (int i = 0; i < ITEMS; i++) {
@@ -213,14 +258,31 @@ __global__ void __launch_bounds__(THREADS, 3) onesweep_kernel(const u64* __restr
     __stcs(kout + dst, key);
     if (VALS) __stcs(vout + dst, vals_s[j]);
   }
+  if (prof) {
+    __syncthreads();
+    if (tid == 0) prof[5] = gtime(), prof[6] = (u64)blockIdx.x;
+  }
+  }
 }
 
-template <bool VALS>
+template <int THREADS, int ITEMS, bool VALS>
 static size_t onesweep_smem() {
-  constexpr int WARPS = SORT_THREADS / 32;
-  return (size_t)SORT_TILE * 8 + (VALS ? (size_t)SORT_TILE * 4 : 0) + (size_t)WARPS * RADIX * 4 + RADIX * 4 +
-         RADIX * 8 + (WARPS + 1) * 4 + (size_t)WARPS * (RADIX + 1) * 4;
+  constexpr int WARPS = THREADS / 32, TILE = THREADS * ITEMS;
+  return (size_t)TILE * 8 + (VALS ? (size_t)TILE * 4 : 0) + (size_t)WARPS * RADIX * 4 + RADIX * 4 + RADIX * 8 +
+         (WARPS + 1) * 4 + (size_t)WARPS * (RADIX + 1) * 4;
 }
+
+int sort_cfg() {  // SESA_SORT_CFG: 0 = 256x16, 1 = 256x24, 2 = 512x16, 3 = TMA 256x16, 4 = TMA 256x24; default 1
+//   (measured on C5: 1 fastest; the persistent TMA-prefetch variants delay aggregates and lose badly)
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("SESA_SORT_CFG");
+    v = e ? atoi(e) : 1;
+  }
+  return v;
+}
+
+u32 sort_tile_keys() { return (sort_cfg() == 1 || sort_cfg() == 4) ? 256 * 24 : sort_cfg() == 2 ? 512 * 16 : 256 * 16; }
 
 int sort_variant() {  // SESA_SORT_MATCH=0 ballots, 1 atomicOr masks (default)
   static int v = -1;
@@ -231,30 +293,257 @@ int sort_variant() {  // SESA_SORT_MATCH=0 ballots, 1 atomicOr masks (default)
   return v;
 }
 
-template <bool VALS, int MATCH>
+
+// ------------------------------------------------------------------------------------------------------------
+// Persistent, TMA-pipelined onesweep pass (keys only).  Each CTA acquires tiles in increasing order from a
+// counter and, while it ranks / looks back / scatters tile i, the TMA engine (cp.async.bulk, mbarrier
+// completion) is already streaming its next tile into the other shared-memory stage, so loads stay in flight
+// through the look-back waits (ncu on the one-tile-per-CTA kernel: 49% long-scoreboard stalls).  Keys are read
+// from shared memory warp-striped (conflict-free) into registers; the consumed stage doubles as the scatter
+// buffer for the coalesced write-out.  Deadlock-free: a CTA holds at most {current, next} and the lowest
+// unfinished tile is always some CTA's current tile.
+// ------------------------------------------------------------------------------------------------------------
+template <int THREADS, int ITEMS, int MINB>
+__global__ void __launch_bounds__(THREADS, MINB) onesweep_tma_kernel(const u64* __restrict__ kin,
+                                                                     u64* __restrict__ kout, u32 m, u32 shift,
+                                                                     const u64* __restrict__ bin_base,
+                                                                     u64* __restrict__ lookback,
+                                                                     u32* __restrict__ tile_ctr, u32 epoch) {
+  constexpr int WARPS = THREADS / 32;
+  constexpr int TILE = THREADS * ITEMS;
+  static_assert(RADIX <= THREADS, "one bin per thread");
+  extern __shared__ __align__(128) unsigned char smem[];
+  u64* stage = reinterpret_cast<u64*>(smem);                          // [2][TILE]
+  u32* whist = reinterpret_cast<u32*>(stage + 2 * TILE);              // [WARPS][RADIX]
+  u32* wmask = whist + WARPS * RADIX;                                 // [WARPS][RADIX + 1]
+  u32* bin_start = wmask + WARPS * (RADIX + 1);                       // [RADIX]
+  long long* glob = reinterpret_cast<long long*>(bin_start + RADIX);  // [RADIX]
+  u32* scratch = reinterpret_cast<u32*>(glob + RADIX);                // [WARPS + 1]
+  u64* bar = reinterpret_cast<u64*>(scratch + WARPS + 2);             // [2] (8-byte aligned)
+  __shared__ u32 s_tile[2];
+
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const u32 ntiles = (u32)((m + TILE - 1) / TILE);
+  for (int i = tid; i < WARPS * (RADIX + 1); i += THREADS) wmask[i] = 0;
+  if (tid == 0) {
+    mbar_init(&bar[0], 1);
+    mbar_init(&bar[1], 1);
+    fence_mbar_init();
+    s_tile[0] = atomicAdd(tile_ctr, 1u);
+    if (s_tile[0] < ntiles) {
+      const u64 tb = (u64)s_tile[0] * TILE;
+      const u32 bytes = (u32)((min((u64)TILE, (u64)m - tb) * 8 + 15) & ~15ull);
+      mbar_expect_tx(&bar[0], bytes);
+      bulk_g2s(stage, kin + tb, bytes, &bar[0]);
+    }
+  }
+  __syncthreads();
+  for (u32 it = 0;; it++) {
+    const int sI = it & 1;
+    const u32 tile = s_tile[sI];
+    if (tile >= ntiles) break;
+    u64* st = stage + sI * TILE;
+    for (int i = tid; i < WARPS * RADIX; i += THREADS) whist[i] = 0;
+    __syncthreads();  // everyone is done with the other stage (previous tile's write-out) and saw s_tile
+    if (tid == 0) {   // prefetch the next tile into the other stage
+      const u32 nxt = atomicAdd(tile_ctr, 1u);
+      s_tile[sI ^ 1] = nxt;
+      if (nxt < ntiles) {
+        const u64 tb = (u64)nxt * TILE;
+        const u32 bytes = (u32)((min((u64)TILE, (u64)m - tb) * 8 + 15) & ~15ull);
+        mbar_expect_tx(&bar[sI ^ 1], bytes);
+        bulk_g2s(stage + (sI ^ 1) * TILE, kin + tb, bytes, &bar[sI ^ 1]);
+      }
+    }
+    const u64 tbase = (u64)tile * TILE;
+    const bool full = tbase + TILE <= m;
+    mbar_wait(&bar[sI], (it >> 1) & 1);
+    u64 k[ITEMS];
+    u32 rk[ITEMS];
+    const u32 wofs = warp * 32 * ITEMS + lane;
+#pragma unroll
+    for (int i = 0; i < ITEMS; i++) k[i] = (full || tbase + wofs + i * 32 < m) ? st[wofs + i * 32] : ~0ull;
+    u32* wh = whist + warp * RADIX;
+#pragma unroll
+    for (int i = 0; i < ITEMS; i++)
+      if (full || tbase + wofs + i * 32 < m) atomicAdd(&wh[(u32)((k[i] >> shift) & (RADIX - 1))], 1u);
+    __syncthreads();
+    u32 tot = 0;
+    if (tid < RADIX) {
+#pragma unroll
+      for (int w = 0; w < WARPS; w++) {
+        const u32 c = whist[w * RADIX + tid];
+        whist[w * RADIX + tid] = tot;
+        tot += c;
+      }
+      st_relaxed(lookback + (u64)tile * RADIX + tid, lb_pack(tile == 0 ? LB_PREFIX : LB_AGG, epoch, tot));
+    }
+    const u32 bs = block_excl_sum<THREADS>(tid < RADIX ? tot : 0u, scratch);
+    if (tid < RADIX) {
+      bin_start[tid] = bs;
+      u64 excl = 0;
+      if (tile > 0) {
+        long long p = (long long)tile - 1;
+        int spins = 0;
+        while (true) {
+          u64 w[4];
+#pragma unroll
+          for (int q = 0; q < 4; q++) w[q] = p - q >= 0 ? ld_relaxed(lookback + (u64)(p - q) * RADIX + tid) : 0ull;
+          int q = 0;
+          bool done = false;
+          for (; q < 4 && p - q >= 0; q++) {
+            const u32 e = (u32)((w[q] >> 54) & 0xFF);
+            const u64 sst = w[q] & (3ull << 62);
+            if (e != epoch || sst == 0) break;
+            excl += w[q] & LB_VAL;
+            if (sst == LB_PREFIX) {
+              done = true;
+              break;
+            }
+          }
+          if (done) break;
+          if (q == 0) __nanosleep(++spins < 4 ? 32 : 128);
+          p -= q;
+        }
+        st_relaxed(lookback + (u64)tile * RADIX + tid, lb_pack(LB_PREFIX, epoch, excl + tot));
+      }
+      glob[tid] = (long long)(bin_base[tid] + excl) - (long long)bs;
+    }
+    // stable warp-level ranking (atomicOr peer masks), running counter starts at the warp's offset
+#pragma unroll
+    for (int i = 0; i < ITEMS; i++) {
+      const bool valid = full || tbase + wofs + i * 32 < m;
+      const u32 d = valid ? (u32)((k[i] >> shift) & (RADIX - 1)) : (u32)RADIX;
+      u32* wm = wmask + warp * (RADIX + 1);
+      atomicOr(&wm[d], 1u << lane);
+      __syncwarp();
+      const unsigned peers = wm[d];
+      __syncwarp();
+      const bool leader = lane == 31 - __clz(peers);
+      if (leader) wm[d] = 0;
+      const u32 c = valid ? wh[d] : 0u;
+      rk[i] = c + __popc(peers & lanemask_lt());
+      __syncwarp();
+      if (valid && leader) wh[d] = c + __popc(peers);
+      __syncwarp();
+    }
+    __syncthreads();  // all keys are in registers and bin_start/glob are set: reuse the stage for the scatter
+#pragma unroll
+    for (int i = 0; i < ITEMS; i++)
+      if (full || tbase + wofs + i * 32 < m) st[bin_start[(u32)((k[i] >> shift) & (RADIX - 1))] + rk[i]] = k[i];
+    __syncthreads();
+    const u32 tcount = (u32)min((u64)TILE, (u64)m - tbase);
+#pragma unroll 4
+    for (u32 j = tid; j < tcount; j += THREADS) {
+      const u64 key = st[j];
+      const u32 d = (u32)((key >> shift) & (RADIX - 1));
+      __stcs(kout + (u64)(glob[d] + (long long)j), key);
+    }
+  }
+}
+
+template <int THREADS, int ITEMS, int MINB>
+static void launch_os_tma(const u64* kin, u64* kout, u32 m, u32 shift, const u64* bin_base, u64* lookback,
+                          u32* tile_ctr, u32 epoch, cudaStream_t st) {
+  constexpr int WARPS = THREADS / 32, TILE = THREADS * ITEMS;
+  auto kern = onesweep_tma_kernel<THREADS, ITEMS, MINB>;
+  const size_t sm = (size_t)2 * TILE * 8 + (size_t)WARPS * RADIX * 4 + (size_t)WARPS * (RADIX + 1) * 4 + RADIX * 4 +
+                    RADIX * 8 + (WARPS + 2) * 4 + 16 + 64;
+  static int grid = 0;
+  if (!grid) {
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    int dev = 0, sms = 148, per = 1;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, kern, THREADS, sm);
+    grid = sms * std::max(per, 1);
+  }
+  const u32 tiles = (u32)((m + TILE - 1) / TILE);
+  kern<<<std::min<u32>(tiles, (u32)grid), THREADS, sm, st>>>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch);
+}
+
+template <int THREADS, int ITEMS, int MINB, bool VALS, int MATCH>
 static void launch_os(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m, u32 shift, const u64* bin_base,
                       u64* lookback, u32* tile_ctr, u32 epoch, cudaStream_t st) {
-  auto kern = onesweep_kernel<SORT_THREADS, SORT_ITEMS, VALS, MATCH>;
-  const size_t sm = onesweep_smem<VALS>();
+  auto kern = onesweep_kernel<THREADS, ITEMS, VALS, MATCH, MINB>;
+  const size_t sm = onesweep_smem<THREADS, ITEMS, VALS>();
   static bool set = false;
   if (!set) {
     cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     set = true;
   }
-  kern<<<sort_tiles(m), SORT_THREADS, sm, st>>>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch);
+  const u32 tiles = (u32)((m + THREADS * ITEMS - 1) / (THREADS * ITEMS));
+  static int cap = 0;
+  if (!cap) {
+    int dev = 0, sms = 148, per = 1;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, kern, THREADS, sm);
+    cap = sms * std::max(per, 1);
+  }
+  (void)cap;
+  kern<<<tiles, THREADS, sm, st>>>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch,
+                                   tile_atomic_mode());
+}
+
+template <bool VALS, int MATCH>
+static void launch_os_cfg(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m, u32 shift,
+                          const u64* bin_base, u64* lookback, u32* tile_ctr, u32 epoch, cudaStream_t st) {
+  switch (sort_cfg()) {
+    case 1: launch_os<256, 24, 2, VALS, MATCH>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 2: launch_os<512, 16, 1, VALS, MATCH>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    default: launch_os<256, 16, 3, VALS, MATCH>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
+  }
+}
+
+static void sort_prof_dump(u32 m, cudaStream_t st, unsigned long long* d, u32 tile_keys) {
+  const u32 nt = (m + tile_keys - 1) / tile_keys;
+  std::vector<unsigned long long> h((size_t)nt * 8);
+  cudaMemcpyAsync(h.data(), d, h.size() * 8, cudaMemcpyDeviceToHost, st);
+  cudaStreamSynchronize(st);
+  double ph[5] = {0, 0, 0, 0, 0};
+  unsigned long long t0 = ~0ull, t1 = 0;
+  for (u32 t = 0; t < nt; t++) {
+    const unsigned long long* p = &h[(size_t)t * 8];
+    for (int q = 0; q < 5; q++) ph[q] += (double)(p[q + 1] - p[q]);
+    t0 = std::min(t0, p[0]);
+    t1 = std::max(t1, p[5]);
+  }
+  fprintf(stderr, "[sortprof] tiles %u span %.3f ms; mean ns: load %.0f counts %.0f lookback %.0f rank %.0f write %.0f\n", nt,
+          (t1 - t0) / 1e6, ph[0] / nt, ph[1] / nt, ph[2] / nt, ph[3] / nt, ph[4] / nt);
 }
 
 void launch_onesweep(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m, u32 shift, const u64* bin_base,
                      u64* lookback, u32* tile_ctr, u32 epoch, cudaStream_t st) {
-  if (!sort_tiles(m)) return;
-  const bool ballot = sort_variant() == 0;
-  if (vin) {
-    if (ballot) launch_os<true, 0>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
-    else launch_os<true, 1>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
-  } else {
-    if (ballot) launch_os<false, 0>(kin, kout, nullptr, nullptr, m, shift, bin_base, lookback, tile_ctr, epoch, st);
-    else launch_os<false, 1>(kin, kout, nullptr, nullptr, m, shift, bin_base, lookback, tile_ctr, epoch, st);
+  if (!m) return;
+  static unsigned long long* dprof = nullptr;
+  static size_t dcap = 0;
+  const bool want = getenv("SESA_SORT_PROF") && !vin;
+  if (want) {
+    const size_t need = ((size_t)m / 4096 + 2) * 64;
+    if (need > dcap) {
+      if (dprof) cudaFree(dprof);
+      cudaMalloc(&dprof, need);
+      dcap = need;
+    }
+    cudaMemcpyToSymbolAsync(g_prof, &dprof, sizeof(dprof), 0, cudaMemcpyHostToDevice, st);
+  } else if (dprof) {
+    unsigned long long* z = nullptr;
+    cudaMemcpyToSymbolAsync(g_prof, &z, sizeof(z), 0, cudaMemcpyHostToDevice, st);
   }
+  const bool ballot = sort_variant() == 0;
+  if (vin) {  // race lists are small: fixed config
+    if (ballot) launch_os<256, 16, 3, true, 0>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
+    else launch_os<256, 16, 3, true, 1>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
+  } else if (sort_cfg() == 3) {
+    launch_os_tma<256, 16, 2>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
+  } else if (sort_cfg() == 4) {
+    launch_os_tma<256, 24, 1>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
+  } else {
+    if (ballot) launch_os_cfg<false, 0>(kin, kout, nullptr, nullptr, m, shift, bin_base, lookback, tile_ctr, epoch, st);
+    else launch_os_cfg<false, 1>(kin, kout, nullptr, nullptr, m, shift, bin_base, lookback, tile_ctr, epoch, st);
+  }
+  if (want) sort_prof_dump(m, st, dprof, sort_tile_keys());
 }
 
 // digit histograms of plain keys (race list sort): npass 8-bit digits from bit 0

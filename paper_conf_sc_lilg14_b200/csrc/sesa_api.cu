@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
@@ -220,7 +221,7 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
   info.digit_bits = RADIX_BITS;
 
   // 2. key extraction + digit histograms
-  if (!grow(b_keys[0], m * 8, "keys") || !grow(b_keys[1], m * 8, "keys") ||
+  if (!grow(b_keys[0], m * 8 + 64, "keys") || !grow(b_keys[1], m * 8 + 64, "keys") ||
       !grow(b_hist, (size_t)std::max(npass, 1u) * RADIX * 4, "hist") ||
       !grow(b_binbase, (size_t)std::max(npass, 1u) * RADIX * 8, "binbase"))
     return status;
@@ -502,6 +503,7 @@ sesa_status sesa_trace_create(const sesa_config* cfg, sesa_trace** out) {
   t->cfg = *cfg;
   t->device = dev;
   cudaDeviceGetAttribute(&t->num_sms, cudaDevAttrMultiProcessorCount, dev);
+
   if (t->num_sms <= 0) t->num_sms = 148;
   *out = t;
   return SESA_OK;
