@@ -175,6 +175,15 @@ sesa_status sesa_nccl_unique_id(uint8_t out_id[128]);
 sesa_status sesa_race_check(sesa_trace *t, const sesa_access *d_records, uint64_t n, uint64_t index_base,
                             void *cuda_stream);
 
+/* Test/diagnostic entry: the distributed check of sesa_race_check with `world` (<= 8) VIRTUAL ranks on the
+ * current GPU — the same kernels and data flow as the NCCL path (partition by location owner, key exchange,
+ * record fetch, race gather), with the exchanges done by device copies.  Rank r owns records
+ * [offs[r], offs[r+1]) of d_records (offs has world+1 entries, offs[0] = 0).  On return *out is a handle holding
+ * the merged race list (read it with sesa_races_get; destroy it with sesa_trace_destroy).  The result must equal
+ * a single-GPU check of the same records (tests/test_gpu_dist.py). */
+sesa_status sesa_race_check_loopback(const sesa_config *cfg, const sesa_access *d_records, const uint64_t *offs,
+                                     int world, uint64_t index_base, void *cuda_stream, sesa_trace **out);
+
 /* Same, for records in HOST memory: the library copies them to the device (chunked through pinned staging
  * when h_records is pageable) inside the call.  This is the end-to-end entry point. */
 sesa_status sesa_race_check_host(sesa_trace *t, const sesa_access *h_records, uint64_t n, uint64_t index_base,

@@ -21,8 +21,20 @@ BUILD = os.path.join(ROOT, "build", "sesa")
 LIB = os.path.join(PKG, "libsesa.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+def _nccl_dir():
+    """The NCCL torch ships (same libnccl.so.2 the process already has loaded when torch is imported)."""
+    for p in __import__("sys").path:
+        d = os.path.join(p, "nvidia", "nccl")
+        if os.path.exists(os.path.join(d, "include", "nccl.h")):
+            return d
+    return None
+
+
+NCCL = _nccl_dir()
+NCCL_INC = os.path.join(NCCL, "include") if NCCL else "/usr/include"
+NCCL_LIB = os.path.join(NCCL, "lib") if NCCL else "/usr/lib/x86_64-linux-gnu"
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "--expt-relaxed-constexpr", "-Xcompiler", "-fPIC,-O2",
-         "-Xptxas", "-v", "-I", os.path.join(ROOT, "include"), "-I", CSRC]
+         "-Xptxas", "-v", "-I", os.path.join(ROOT, "include"), "-I", CSRC, "-I", NCCL_INC]
 
 
 def _sources():
@@ -58,7 +70,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
                 sys.stderr.write(log)
     if force or not os.path.exists(LIB) or os.path.getmtime(LIB) < max(os.path.getmtime(o) for o in objs):
         tmp = LIB + f".tmp{os.getpid()}"
-        cmd = [NVCC] + ARCH + ["-shared", "-o", tmp] + objs + ["-lcudart"]
+        cmd = [NVCC] + ARCH + ["-shared", "-o", tmp] + objs + ["-lcudart", "-L", NCCL_LIB, "-l:libnccl.so.2",
+                                                               "-Xlinker", "-rpath=" + NCCL_LIB]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")

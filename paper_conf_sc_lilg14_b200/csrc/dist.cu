@@ -1,20 +1,550 @@
-// dist.cu — multi-GPU sharding.  Placeholder until the NCCL exchange lands:
-// distributed handles report SESA_ENCCL.
+// dist.cu — multi-GPU race check (SURVEY §8a rows a3 "shard + all-to-all" and a7 "gather + merge").
+//
+// Every race is a property of one location λ (two accesses to the same location), so entries shard by
+// owner(λ) = mix64(λ) mod N with no other communication than:
+//   X1  all-reduce of the extents summaries (one consistent key layout on every rank) + all-gather of the
+//       shard boundaries (global (block, interval) order, global record positions)
+//   X2  all-to-all of the 8-byte sort keys (carrying the GLOBAL record position) to their location owners
+//   X3  all-to-all of the positions of entries at locations touched >= 2 times (the only ones that can race;
+//       2e5 of C5's 1e9) to the ranks holding those records, and X4 the 32-byte records back
+//   X5  gather of the (already canonically ordered) per-rank race lists to rank 0, which re-sorts the union.
+// The exchange is an interface: NCCL (one process per GPU, grouped ncclSend/ncclRecv over NVLink/NVSwitch) or
+// a loopback implementation (W virtual ranks on one GPU, device copies) that runs the same kernels and data
+// flow for tests.  Received key blocks are concatenated in source-rank order, so global positions stay
+// ascending: the LSD sort's stability then yields the same canonical run order as a 1-GPU check.
+#include <dlfcn.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <memory>
+#include <vector>
+
 #include "sesa_internal.h"
 
-struct DistState {};
+using namespace sesa;
 
-sesa_status sesa_trace::check_dist(const sesa_access*, uint64_t, uint64_t) {
-  fail(SESA_ENCCL, "distributed race check not available in this build");
+namespace sesa {
+
+// ------------------------------------------------------------------------------------------------ partition
+// Stable partition of u64 items into W <= 8 buckets.  Warp chunks of 512 items (16 coalesced rows); per-chunk
+// bucket counts -> one exclusive scan over the bucket-major count matrix -> writes.  MODE 0: item = sort key,
+// bucket = mix64(location run key) mod W.  MODE 1: item = key of a compacted entry, emitted as its global
+// position, bucket = owner rank of that position (bases[W+1]); the entry index is written alongside.
+constexpr int PT_ROWS = 16, PT_CHUNK = 32 * PT_ROWS, PT_THREADS = 256;
+
+struct PartArgs {
+  const u64* in;
+  u64 n;
+  u32 W;
+  int mode;
+  KeyLayout L;
+  u64 bases[9];
+  u32* cnt;        // [W][nchunks]
+  const u32* off;  // exclusive scan of cnt
+  u64* out;
+  u32* out_src;
+};
+
+__device__ __forceinline__ u32 part_bucket(const PartArgs& a, u64 item) {
+  if (a.mode == 0) return (u32)(sesa_mix(group_of_hi(a.L, item >> a.L.pos_bits)) % a.W);
+  const u64 pos = item & lowmask(a.L.pos_bits);
+  u32 r = 0;
+  while (r + 1 < a.W && pos >= a.bases[r + 1]) r++;
+  return r;
+}
+
+template <bool WRITE>
+__global__ void __launch_bounds__(PT_THREADS) partition_kernel(PartArgs a) {
+  const int lane = threadIdx.x & 31;
+  const u64 nch = (a.n + PT_CHUNK - 1) / PT_CHUNK;
+  const u64 gw = ((u64)blockIdx.x * PT_THREADS + threadIdx.x) >> 5, nw = ((u64)gridDim.x * PT_THREADS) >> 5;
+  for (u64 c = gw; c < nch; c += nw) {
+    u32 run[8];
+#pragma unroll
+    for (int d = 0; d < 8; d++) run[d] = (WRITE && d < (int)a.W) ? a.off[(u64)d * nch + c] : 0u;
+    for (int r = 0; r < PT_ROWS; r++) {
+      const u64 i = c * PT_CHUNK + (u64)r * 32 + lane;
+      const bool valid = i < a.n;
+      const u64 item = valid ? a.in[i] : 0ull;
+      const u32 b = valid ? part_bucket(a, item) : 99u;
+#pragma unroll
+      for (int d = 0; d < 8; d++) {
+        if (d >= (int)a.W) break;
+        const unsigned m = __ballot_sync(~0u, b == (u32)d);
+        if (WRITE && b == (u32)d) {
+          const u32 o = run[d] + __popc(m & lanemask_lt());
+          a.out[o] = a.mode == 0 ? item : (item & lowmask(a.L.pos_bits));
+          if (a.out_src) a.out_src[o] = (u32)i;
+        }
+        run[d] += __popc(m);
+      }
+    }
+    if (!WRITE && lane == 0)
+      for (int d = 0; d < (int)a.W; d++) a.cnt[(u64)d * nch + c] = run[d];
+  }
+}
+
+__global__ void bucket_totals_kernel(const u32* cnt, const u32* off, u64 nch, u32 W, u64* tot) {
+  const u32 d = threadIdx.x;
+  // bucket d occupies [off[d*nch], off[d*nch + nch-1] + cnt[d*nch + nch-1]) of the bucket-major output
+  if (d < W) tot[d] = nch ? (u64)off[(u64)d * nch + nch - 1] + cnt[(u64)d * nch + nch - 1] - off[(u64)d * nch] : 0ull;
+}
+
+__global__ void gather_records_kernel(const Rec* __restrict__ rec, const u64* __restrict__ pos, u64 base, u64 n,
+                                      Rec* __restrict__ out) {
+  const u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) out[i] = rec[pos[i] - base];
+}
+
+__global__ void scatter_records_kernel(const Rec* __restrict__ in, const u32* __restrict__ dst, u64 n,
+                                       Rec* __restrict__ out) {
+  const u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) out[dst[i]] = in[i];
+}
+
+}  // namespace sesa
+
+// ------------------------------------------------------------------------------------------------ state
+struct RankBufs {
+  DevBuf pcnt, poff, ptmp, send, recv, src, req, reqin, recsend, recback, rec_entry, tot, rkeys, rvals, races;
+};
+
+struct DistState {
+  ncclComm_t comm = nullptr;
+  RankBufs b;
+};
+
+// per-rank host-side values exchanged in X1
+struct RankInfo {
+  unsigned long long n, base, first_b, first_i, last_b, last_i, bad;  // bad: global index or ~0
+};
+
+static bool partition(sesa_trace* t, RankBufs& B, const u64* in, u64 n, u32 W, int mode, const u64* bases,
+                      u64* out_tot /*[W]*/) {
+  PartArgs a;
+  memset(&a, 0, sizeof a);
+  a.in = in;
+  a.n = n;
+  a.W = W;
+  a.mode = mode;
+  a.L = t->layout;
+  for (u32 i = 0; i <= W && bases; i++) a.bases[i] = bases[i];
+  const u64 nch = (n + PT_CHUNK - 1) / PT_CHUNK;
+  const u64 ncnt = std::max<u64>(nch * W, 1);
+  if (!t->grow(B.pcnt, ncnt * 4, "part counts") || !t->grow(B.poff, ncnt * 4, "part offsets") ||
+      !t->grow(B.ptmp, scan_u32_temp_bytes(ncnt), "part scan") || !t->grow(B.send, std::max<u64>(n, 1) * 8, "send") ||
+      !t->grow(B.src, std::max<u64>(n, 1) * 4, "src") || !t->grow(B.tot, 8 * 8, "totals"))
+    return false;
+  a.cnt = (u32*)B.pcnt.p;
+  a.off = (u32*)B.poff.p;
+  a.out = (u64*)B.send.p;
+  a.out_src = mode == 1 ? (u32*)B.src.p : nullptr;
+  if (n) {
+    const unsigned grid = (unsigned)std::min<u64>((nch + 7) / 8, (u64)t->num_sms * 8);
+    t->launches += 3;
+    if (getenv("SESA_SYNC_DEBUG")) fprintf(stderr, "[sesa debug] partition n=%llu W=%u grid=%u nch=%llu\n",
+                                           (unsigned long long)n, W, grid, (unsigned long long)nch);
+    partition_kernel<false><<<grid, PT_THREADS, 0, t->stream>>>(a);
+    launch_scan_exclusive_u32((u32*)B.pcnt.p, (u32*)B.poff.p, nch * W, B.ptmp.p, t->stream);
+    partition_kernel<true><<<grid, PT_THREADS, 0, t->stream>>>(a);
+    bucket_totals_kernel<<<1, 32, 0, t->stream>>>((u32*)B.pcnt.p, (u32*)B.poff.p, nch, W, (u64*)B.tot.p);
+    if (!t->cuda_ok(cudaMemcpyAsync(out_tot, B.tot.p, W * 8, cudaMemcpyDeviceToHost, t->stream), "totals")) return false;
+  } else {
+    for (u32 i = 0; i < W; i++) out_tot[i] = 0;
+  }
+  return t->sync_check("partition");
+}
+
+// ------------------------------------------------------------------------------------------------ exchange
+// One exchange = every rank sends count[r][p] elements (elem bytes) of its send buffer (bucket-major) to rank p,
+// and receives, concatenated in source-rank order, into its recv buffer.
+struct Exchanger {
+  virtual ~Exchanger() {}
+  virtual int world() const = 0;
+  // host-side all-gather of a per-rank POD value
+  virtual bool allgather(sesa_trace* t, const void* mine, void* all, size_t bytes) = 0;
+  // send[p] counts (elements) -> recv from each peer; offsets computed by the caller
+  virtual bool alltoall(sesa_trace* t, const void* send, const u64* scnt, void* recv, const u64* rcnt, size_t elem) = 0;
+};
+
+struct NcclExchanger : Exchanger {
+  ncclComm_t comm;
+  int rank_, world_;
+  DevBuf tmp;
+  NcclExchanger(ncclComm_t c, int r, int w) : comm(c), rank_(r), world_(w) {}
+  int world() const override { return world_; }
+  bool nccl_ok(sesa_trace* t, ncclResult_t r, const char* what) {
+    if (r == ncclSuccess) return true;
+    t->fail(SESA_ENCCL, "%s: %s", what, ncclGetErrorString(r));
+    return false;
+  }
+  bool allgather(sesa_trace* t, const void* mine, void* all, size_t bytes) override {
+    if (!t->grow(tmp, bytes * (world_ + 1), "allgather")) return false;
+    char* d = (char*)tmp.p;
+    cudaMemcpyAsync(d + bytes * world_, mine, bytes, cudaMemcpyHostToDevice, t->stream);
+    if (!nccl_ok(t, ncclAllGather(d + bytes * world_, d, bytes, ncclUint8, comm, t->stream), "ncclAllGather")) return false;
+    cudaMemcpyAsync(all, d, bytes * world_, cudaMemcpyDeviceToHost, t->stream);
+    return t->sync_check("allgather");
+  }
+  bool alltoall(sesa_trace* t, const void* send, const u64* scnt, void* recv, const u64* rcnt, size_t elem) override {
+    u64 so = 0, ro = 0;
+    if (!nccl_ok(t, ncclGroupStart(), "ncclGroupStart")) return false;
+    for (int p = 0; p < world_; p++) {
+      if (scnt[p] && !nccl_ok(t, ncclSend((const char*)send + so * elem, scnt[p] * elem, ncclUint8, p, comm, t->stream),
+                              "ncclSend"))
+        return false;
+      if (rcnt[p] && !nccl_ok(t, ncclRecv((char*)recv + ro * elem, rcnt[p] * elem, ncclUint8, p, comm, t->stream),
+                              "ncclRecv"))
+        return false;
+      so += scnt[p];
+      ro += rcnt[p];
+    }
+    if (!nccl_ok(t, ncclGroupEnd(), "ncclGroupEnd")) return false;
+    return t->sync_check("alltoall");
+  }
+};
+
+// ------------------------------------------------------------------------------------------------ the check
+// Runs the collective check for `R` ranks whose handles are ts[0..R) (one real rank with NCCL: R = 1 and
+// my_rank = its rank; loopback: R = world virtual ranks on this GPU).  Phases are executed for every local rank
+// before each exchange; for loopback the exchange is performed by device copies between the local handles.
+struct LoopbackCtx {
+  std::vector<sesa_trace*> ts;
+};
+
+static bool fail_all(std::vector<sesa_trace*>& ts, const sesa_trace* src) {
+  for (auto* t : ts)
+    if (t != src) t->status = src->status, t->err = src->err;
+  return false;
+}
+
+struct RankIO {
+  const Rec* rec;
+  u64 n, index_base;
+};
+
+// exchange helper covering both modes: per local rank r, send buffers/counts -> recv buffers/counts
+static bool exchange(std::vector<sesa_trace*>& ts, Exchanger* ex, const std::vector<const void*>& send,
+                     const std::vector<std::vector<u64>>& scnt, std::vector<DevBuf*>& recv, std::vector<std::vector<u64>>& rcnt,
+                     size_t elem, const char* what) {
+  const int W = ex ? ex->world() : (int)ts.size();
+  const int R = (int)ts.size();
+  rcnt.assign(R, std::vector<u64>(W, 0));
+  if (ex) {  // real ranks: one local handle; counts by all-gather of the count rows
+    sesa_trace* t = ts[0];
+    std::vector<u64> all((size_t)W * W);
+    if (!ex->allgather(t, scnt[0].data(), all.data(), W * 8)) return false;
+    int me = t->rank;
+    u64 tot = 0;
+    for (int p = 0; p < W; p++) rcnt[0][p] = all[(size_t)p * W + me], tot += rcnt[0][p];
+    if (!t->grow(*recv[0], std::max<u64>(tot, 1) * elem + 64, what)) return false;
+    return ex->alltoall(t, send[0], scnt[0].data(), recv[0]->p, rcnt[0].data(), elem);
+  }
+  // loopback: rank r receives from every s, in source order
+  if (getenv("SESA_SYNC_DEBUG"))
+    for (int r = 0; r < R; r++)
+      for (int p = 0; p < W; p++) fprintf(stderr, "[sesa debug] %s scnt[%d][%d] = %llu\n", what, r, p, (unsigned long long)scnt[r][p]);
+  for (int r = 0; r < R; r++) {
+    u64 tot = 0;
+    for (int s = 0; s < R; s++) rcnt[r][s] = scnt[s][r], tot += scnt[s][r];
+    if (!ts[r]->grow(*recv[r], std::max<u64>(tot, 1) * elem + 64, what)) return fail_all(ts, ts[r]);
+  }
+  for (int r = 0; r < R; r++) {
+    u64 ro = 0;
+    for (int s = 0; s < R; s++) {
+      u64 so = 0;
+      for (int q = 0; q < r; q++) so += scnt[s][q];
+      if (scnt[s][r])
+        cudaMemcpyAsync((char*)recv[r]->p + ro * elem, (const char*)send[s] + so * elem, scnt[s][r] * elem,
+                        cudaMemcpyDeviceToDevice, ts[0]->stream);
+      ro += scnt[s][r];
+    }
+  }
+  return ts[0]->sync_check(what) || fail_all(ts, ts[0]);
+}
+
+static sesa_status dist_check(std::vector<sesa_trace*>& ts, std::vector<RankIO>& io, Exchanger* ex) {
+  const int R = (int)ts.size();
+  const int W = ex ? ex->world() : R;
+  for (int r = 0; r < R; r++) ts[r]->begin_check(io[r].n);
+  // --- P1: extents per rank
+  for (int r = 0; r < R; r++) {
+    if (io[r].n && !ts[r]->check_records_ptr((const sesa_access*)io[r].rec, io[r].n)) return fail_all(ts, ts[r]), ts[r]->status;
+    if (!ts[r]->step_extents(io[r].rec, io[r].n)) return fail_all(ts, ts[r]), ts[r]->status;
+  }
+  // --- X1: summaries + shard boundaries
+  std::vector<RankInfo> infos(W);
+  std::vector<Summary> sums(W);
+  for (int r = 0; r < R; r++) {
+    RankInfo ri;
+    memset(&ri, 0, sizeof ri);
+    ri.n = io[r].n;
+    ri.base = io[r].index_base;
+    ri.bad = ts[r]->h_summary.bad_index == ~0ull ? ~0ull : io[r].index_base + ts[r]->h_summary.bad_index;
+    if (io[r].n) {
+      sesa_access f, l;
+      cudaMemcpy(&f, io[r].rec, 32, cudaMemcpyDeviceToHost);
+      cudaMemcpy(&l, io[r].rec + io[r].n - 1, 32, cudaMemcpyDeviceToHost);
+      ri.first_b = f.block, ri.first_i = f.interval, ri.last_b = l.block, ri.last_i = l.interval;
+    }
+    if (ex) {
+      if (!ex->allgather(ts[0], &ri, infos.data(), sizeof ri)) return ts[0]->status;
+      if (!ex->allgather(ts[0], &ts[0]->h_summary, sums.data(), sizeof(Summary))) return ts[0]->status;
+    } else {
+      infos[r] = ri;
+      sums[r] = ts[r]->h_summary;
+    }
+  }
+  Summary S = sums[0];
+  u64 bad = ~0ull;
+  for (int p = 0; p < W; p++) bad = std::min<u64>(bad, infos[p].bad);
+  if (bad != ~0ull) {
+    for (int r = 0; r < R; r++) {
+      const u64 b0 = io[r].index_base;
+      if (bad >= b0 && bad < b0 + io[r].n) ts[r]->report_bad((const sesa_access*)io[r].rec, bad - b0, bad);
+      else ts[r]->fail(SESA_EINVAL, "record %llu invalid (on another rank)", (unsigned long long)bad);
+    }
+    return SESA_EINVAL;
+  }
+  for (int p = 1; p < W; p++) {
+    const Summary& q = sums[p];
+    S.entries += q.entries, S.multi += q.multi, S.unsorted |= q.unsorted;
+    for (int sp = 0; sp < 2; sp++) {
+      if (!q.count[sp]) continue;
+      if (!S.count[sp]) {
+        S.gmin[sp] = q.gmin[sp], S.gmax[sp] = q.gmax[sp], S.bmin[sp] = q.bmin[sp], S.bmax[sp] = q.bmax[sp];
+        S.imin[sp] = q.imin[sp], S.imax[sp] = q.imax[sp];
+      } else {
+        S.gmin[sp] = std::min(S.gmin[sp], q.gmin[sp]), S.gmax[sp] = std::max(S.gmax[sp], q.gmax[sp]);
+        S.bmin[sp] = std::min(S.bmin[sp], q.bmin[sp]), S.bmax[sp] = std::max(S.bmax[sp], q.bmax[sp]);
+        S.imin[sp] = std::min(S.imin[sp], q.imin[sp]), S.imax[sp] = std::max(S.imax[sp], q.imax[sp]);
+      }
+      S.count[sp] += q.count[sp];
+    }
+  }
+  // global (block, interval) order across shard boundaries; shards must be contiguous in index order
+  u64 ntot = 0, base0 = infos[0].base;
+  int prev = -1;
+  for (int p = 0; p < W; p++) {
+    if (infos[p].base != base0 + ntot) {
+      for (auto* t : ts) t->fail(SESA_EINVAL, "index_base of rank %d is %llu, expected %llu (exclusive prefix)", p,
+                                 (unsigned long long)infos[p].base, (unsigned long long)(base0 + ntot));
+      return SESA_EINVAL;
+    }
+    ntot += infos[p].n;
+    if (!infos[p].n) continue;
+    if (prev >= 0 && (infos[p].first_b < infos[prev].last_b ||
+                      (infos[p].first_b == infos[prev].last_b && infos[p].first_i < infos[prev].last_i)))
+      S.unsorted = 1;
+    prev = p;
+  }
+  if (S.entries >= (1ull << 31) || ntot >= (1ull << 31)) {
+    for (auto* t : ts) t->fail(SESA_ERANGE, "%llu entries / %llu records >= 2^31 (ABI v1 limit)",
+                               (unsigned long long)S.entries, (unsigned long long)ntot);
+    return SESA_ERANGE;
+  }
+  std::vector<u64> bases(W + 1);
+  for (int p = 0; p < W; p++) bases[p] = infos[p].base - base0;
+  bases[W] = ntot;
+  for (int r = 0; r < R; r++) {
+    if (!ts[r]->make_layout(S, std::max<u64>(ntot, 1))) return fail_all(ts, ts[r]), SESA_ERANGE;
+    ts[r]->info.n_entries = S.entries;
+    ts[r]->info.sort_bits = ts[r]->layout.sort_bits;
+    ts[r]->info.pos_bits = ts[r]->layout.pos_bits;
+  }
+  // --- P2: keys with global positions, partitioned by location owner
+  std::vector<std::vector<u64>> scnt(R, std::vector<u64>(W)), rcnt;
+  std::vector<const void*> sendp(R);
+  std::vector<DevBuf*> recvb(R);
+  for (int r = 0; r < R; r++) {
+    sesa_trace* t = ts[r];
+    const u64 mloc = t->h_summary.entries;
+    if (!t->step_extract(io[r].rec, io[r].n, mloc, io[r].index_base - base0, S.multi != 0)) return fail_all(ts, t), t->status;
+    if (!partition(t, t->ds->b, (const u64*)t->b_keys[0].p, mloc, W, 0, nullptr, scnt[r].data()))
+      return fail_all(ts, t), t->status;
+    sendp[r] = t->ds->b.send.p;
+    recvb[r] = &t->b_keys[1];  // received keys land in b_keys[1], then are copied/swapped into b_keys[0]
+  }
+  // --- X2: keys to their owners
+  if (!exchange(ts, ex, sendp, scnt, recvb, rcnt, 8, "key exchange")) return ts[0]->status;
+  // --- P3: local sort + compaction of the received keys; requests for the records of multi-entry locations
+  std::vector<u64*> comp(R);
+  std::vector<u32> m2(R);
+  std::vector<std::vector<u64>> qcnt(R, std::vector<u64>(W)), qrcnt;
+  std::vector<DevBuf*> reqb(R);
+  for (int r = 0; r < R; r++) {
+    sesa_trace* t = ts[r];
+    u64 mr = 0;
+    for (int s = 0; s < W; s++) mr += rcnt[r][s];
+    std::swap(t->b_keys[0], t->b_keys[1]);  // received keys -> b_keys[0]
+    if (!t->grow(t->b_keys[1], mr * 8 + 64, "keys")) return fail_all(ts, t), t->status;
+    if (!t->step_hist(mr)) return fail_all(ts, t), t->status;
+    int cur = 0;
+    if (!t->step_sort(mr, &cur)) return fail_all(ts, t), t->status;
+    if (!t->step_compact(cur, mr, &comp[r], &m2[r])) return fail_all(ts, t), t->status;
+    if (!partition(t, t->ds->b, comp[r], m2[r], W, 1, bases.data(), qcnt[r].data())) return fail_all(ts, t), t->status;
+    sendp[r] = t->ds->b.send.p;
+    reqb[r] = &t->ds->b.reqin;
+  }
+  // --- X3: positions to the record owners
+  if (!exchange(ts, ex, sendp, qcnt, reqb, qrcnt, 8, "request exchange")) return ts[0]->status;
+  // --- P4: owners gather the requested records
+  std::vector<std::vector<u64>> bcnt, brcnt;
+  bcnt.assign(R, std::vector<u64>(W));
+  std::vector<DevBuf*> backb(R);
+  for (int r = 0; r < R; r++) {
+    sesa_trace* t = ts[r];
+    u64 nq = 0;
+    for (int s = 0; s < W; s++) nq += qrcnt[r][s], bcnt[r][s] = qrcnt[r][s];
+    if (!t->grow(t->ds->b.recsend, std::max<u64>(nq, 1) * 32, "record send")) return fail_all(ts, t), t->status;
+    if (nq) {
+      t->launches++;
+      gather_records_kernel<<<(unsigned)((nq + 255) / 256), 256, 0, t->stream>>>(
+          io[r].rec, (const u64*)t->ds->b.reqin.p, io[r].index_base - base0, nq, (Rec*)t->ds->b.recsend.p);
+    }
+    sendp[r] = t->ds->b.recsend.p;
+    backb[r] = &t->ds->b.recback;
+  }
+  // --- X4: records back to the requesters (in the order of their request buffers)
+  if (!exchange(ts, ex, sendp, bcnt, backb, brcnt, 32, "record exchange")) return ts[0]->status;
+  // --- P5: entry-aligned records, conflict tiles, local canonical race order
+  std::vector<std::vector<u64>> racn(R, std::vector<u64>(W, 0)), racrn;
+  for (int r = 0; r < R; r++) {
+    sesa_trace* t = ts[r];
+    RankBufs& B = t->ds->b;
+    if (!t->grow(B.rec_entry, std::max<u32>(m2[r], 1) * 32, "entry records")) return fail_all(ts, t), t->status;
+    if (m2[r]) {
+      t->launches++;
+      scatter_records_kernel<<<(m2[r] + 255) / 256, 256, 0, t->stream>>>((const Rec*)B.recback.p, (const u32*)B.src.p,
+                                                                          m2[r], (Rec*)B.rec_entry.p);
+    }
+    if (!t->step_conflict(comp[r], m2[r], nullptr, 0, (const Rec*)B.rec_entry.p, base0)) return fail_all(ts, t), t->status;
+    const u32 nr = (u32)t->n_races;
+    if (!t->grow(t->b_races_sorted, (size_t)std::max(nr, 1u) * sizeof(RaceOut), "sorted races")) return fail_all(ts, t), t->status;
+    if (!t->step_race_sort(nr, (RaceOut*)t->b_races.p, (u64*)t->b_rkeys[0].p, (u32*)t->b_rvals[0].p,
+                           (u64*)t->b_rkeys[1].p, (u32*)t->b_rvals[1].p, (RaceOut*)t->b_races_sorted.p))
+      return fail_all(ts, t), t->status;
+    if (!t->sync_check("local races")) return fail_all(ts, t), t->status;
+    racn[r][0] = nr;  // everything goes to rank 0
+    sendp[r] = t->b_races_sorted.p;
+    recvb[r] = &B.races;
+  }
+  // --- X5: race lists to rank 0 (rank 0 receives every rank's list, in rank order), then one canonical sort
+  if (!exchange(ts, ex, sendp, racn, recvb, racrn, sizeof(RaceOut), "race gather")) return ts[0]->status;
+  for (int r = 0; r < R; r++) {
+    sesa_trace* t = ts[r];
+    const bool is0 = (ex ? t->rank : r) == 0;
+    t->n_races = 0;
+    if (is0) {
+      u64 nr = 0;
+      for (int s = 0; s < W; s++) nr += racrn[r][s];
+      RankBufs& B = t->ds->b;
+      if (!t->grow(B.rkeys, std::max<u64>(nr, 1) * 16, "race keys") || !t->grow(B.rvals, std::max<u64>(nr, 1) * 8, "race vals") ||
+          !t->grow(t->b_dist_races, std::max<u64>(nr, 1) * sizeof(RaceOut), "races"))
+        return fail_all(ts, t), t->status;
+      if (nr) {
+        t->launches++;
+        race_rekey_launch((const RaceOut*)B.races.p, nr, t->layout, (u64*)B.rkeys.p, (u32*)B.rvals.p, t->stream);
+        if (!t->step_race_sort((u32)nr, (const RaceOut*)B.races.p, (u64*)B.rkeys.p, (u32*)B.rvals.p,
+                               (u64*)B.rkeys.p + nr, (u32*)B.rvals.p + nr, (RaceOut*)t->b_dist_races.p))
+          return fail_all(ts, t), t->status;
+      }
+      t->n_races = nr;
+    }
+    if (!t->sync_check("race merge")) return fail_all(ts, t), t->status;
+    t->info.n_races = t->n_races;
+    t->info.launches = t->launches;
+    t->collect_prof();
+    t->info.n_stats = (u32)t->stats.size();
+    t->have_result = true;
+  }
+  return SESA_OK;
+}
+
+// ------------------------------------------------------------------------------------------------ handle glue
+sesa_status sesa_trace::check_dist(const sesa_access* d_rec, uint64_t n, uint64_t index_base) {
+  std::vector<sesa_trace*> ts = {this};
+  std::vector<RankIO> io = {{(const Rec*)d_rec, n, index_base}};
+  NcclExchanger ex(ds->comm, rank, world);
+  const sesa_status s = dist_check(ts, io, &ex);
+  if (s != SESA_OK && status == SESA_OK) status = s;
   return status;
 }
 
-void sesa_trace::destroy_dist() {}
+void sesa_trace::destroy_dist() {
+  if (!ds) return;
+  RankBufs& B = ds->b;
+  for (DevBuf* b : {&B.pcnt, &B.poff, &B.ptmp, &B.send, &B.recv, &B.src, &B.req, &B.reqin, &B.recsend, &B.recback,
+                    &B.rec_entry, &B.tot, &B.rkeys, &B.rvals, &B.races})
+    if (b->p) cudaFree(b->p), b->p = nullptr;
+  if (ds->comm) ncclCommDestroy(ds->comm);
+  delete ds;
+  ds = nullptr;
+}
 
 extern "C" {
-sesa_status sesa_trace_create_dist(const sesa_config*, int, int, const uint8_t*, sesa_trace** out) {
-  if (out) *out = nullptr;
-  return SESA_ENCCL;
+
+sesa_status sesa_nccl_unique_id(uint8_t* out_id) {
+  if (!out_id) return SESA_EINVAL;
+  ncclUniqueId id;
+  if (ncclGetUniqueId(&id) != ncclSuccess) return SESA_ENCCL;
+  static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId");
+  memcpy(out_id, &id, 128);
+  return SESA_OK;
 }
-sesa_status sesa_nccl_unique_id(uint8_t*) { return SESA_ENCCL; }
+
+sesa_status sesa_trace_create_dist(const sesa_config* cfg, int rank, int world, const uint8_t* uid, sesa_trace** out) {
+  if (!out) return SESA_EINVAL;
+  *out = nullptr;
+  if (!uid || world < 1 || world > 8 || rank < 0 || rank >= world) return SESA_EINVAL;
+  sesa_trace* t = nullptr;
+  sesa_status s = sesa_trace_create(cfg, &t);
+  if (s != SESA_OK) return s;
+  t->dist = true;
+  t->rank = rank;
+  t->world = world;
+  t->ds = new DistState();
+  ncclUniqueId id;
+  memcpy(&id, uid, 128);
+  if (ncclCommInitRank(&t->ds->comm, world, id, rank) != ncclSuccess) {
+    t->ds->comm = nullptr;
+    sesa_trace_destroy(t);
+    return SESA_ENCCL;
+  }
+  *out = t;
+  return SESA_OK;
 }
+
+// Test/diagnostic entry: the distributed check with `world` virtual ranks on the current GPU (loopback exchange).
+// Rank r owns records [offs[r], offs[r+1]) of d_records.  The merged race list is retrieved with
+// sesa_races_get(t, ...) on the returned primary handle t (created here; destroy with sesa_trace_destroy).
+sesa_status sesa_race_check_loopback(const sesa_config* cfg, const sesa_access* d_records, const uint64_t* offs,
+                                     int world, uint64_t index_base, void* stream, sesa_trace** out) {
+  if (!out || !offs || world < 1 || world > 8) return SESA_EINVAL;
+  *out = nullptr;
+  std::vector<sesa_trace*> ts(world, nullptr);
+  for (int r = 0; r < world; r++) {
+    sesa_status s = sesa_trace_create(cfg, &ts[r]);
+    if (s != SESA_OK) {
+      for (auto* t : ts) sesa_trace_destroy(t);
+      return s;
+    }
+    ts[r]->stream = (cudaStream_t)stream;
+    ts[r]->ds = new DistState();
+  }
+  std::vector<RankIO> io(world);
+  for (int r = 0; r < world; r++)
+    io[r] = {(const Rec*)(d_records + offs[r]), offs[r + 1] - offs[r], index_base + offs[r]};
+  const sesa_status s = dist_check(ts, io, nullptr);
+  // rank 0's handle carries the merged list; expose it as a regular single-GPU result
+  sesa_trace* t0 = ts[0];
+  if (s == SESA_OK) std::swap(t0->b_races_sorted, t0->b_dist_races);
+  for (int r = 1; r < world; r++) sesa_trace_destroy(ts[r]);
+  *out = t0;
+  return s == SESA_OK ? SESA_OK : t0->status;
+}
+
+}  // extern "C"

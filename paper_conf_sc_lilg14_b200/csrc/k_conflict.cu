@@ -260,6 +260,12 @@ struct TileSmem {
 
 __device__ __forceinline__ u32 pos_of(const KeyLayout& L, u64 key) { return (u32)(key & lowmask(L.pos_bits)); }
 
+// the record of entry e (sorted/compacted entry index) with key `key`: by position in the caller's record array
+// (single GPU), or entry-aligned records fetched from the owner ranks (distributed check)
+__device__ __forceinline__ Rec rec_at(const ConflictArgs& a, u64 e, u64 key) {
+  return a.rec_entry ? load_rec(a.rec_entry + e) : load_rec(a.rec + (pos_of(a.L, key) - a.rec_pos_base));
+}
+
 // Loads keys, computes group membership and gathers records.  Returns false if no entry of the tile has a
 // partner candidate (all singletons).
 __device__ bool tile_load(const ConflictArgs& a, TileSmem& s, u64 tb, u32 cnt) {
@@ -299,7 +305,7 @@ __device__ bool tile_load(const ConflictArgs& a, TileSmem& s, u64 tb, u32 cnt) {
   for (int q = 0; q < CT_ITEMS; q++) {
     const int j = j0 + q;
     if (s.fl[j] & FL_INT) {
-      const Rec r = load_rec(a.rec + pos_of(L, s.key[j + 1]));
+      const Rec r = rec_at(a, tb + j, s.key[j + 1]);
       s.blk[j + 1] = r.block;
       s.ivl[j + 1] = r.interval;
       s.thr[j] = r.thread;
@@ -308,11 +314,11 @@ __device__ bool tile_load(const ConflictArgs& a, TileSmem& s, u64 tb, u32 cnt) {
     }
   }
   if (tid == 0 && !(s.fl[0] & FL_GH)) {  // previous entry is in item 0's group: need its (block, interval)
-    const Rec r = load_rec(a.rec + pos_of(L, s.key[0]));
+    const Rec r = rec_at(a, tb - 1, s.key[0]);
     s.blk[0] = r.block, s.ivl[0] = r.interval;
   }
   if (tid == CT_THREADS - 1 && !(s.fl[cnt - 1] & FL_GT)) {
-    const Rec r = load_rec(a.rec + pos_of(L, s.key[cnt + 1]));
+    const Rec r = rec_at(a, tb + cnt, s.key[cnt + 1]);
     s.blk[cnt + 1] = r.block, s.ivl[cnt + 1] = r.interval;
   }
   __syncthreads();
@@ -463,7 +469,7 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
       }
       if (cout && lhead >= 0) {  // this tile owns the group that crosses out
         Slot sl;
-        sl.x[0] = sl.x[1] = sl.y[0] = sl.y[1] = ~0u;
+        sl.x[0] = sl.x[1] = sl.y[0] = sl.y[1] = ~0ull;
         sl.head_key = s.key[lhead + 1];
         sl.hblock = s.blk[lhead + 1];
         sl.hinterval = s.ivl[lhead + 1];
@@ -531,15 +537,17 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
   // MODE 2: exact flags of the crossing pieces -> x candidates into the owner's slot
   // pieces: [0, ftail] if cin (owner = a.owner[tile]); [lhead, cnt-1] if cout (owner = tile, or a.owner[tile]
   // when the whole tile is one group)
-  __shared__ u32 s_min[4];
-  if (tid < 4) s_min[tid] = ~0u;
+  __shared__ unsigned long long s_min[4];
+  if (tid < 4) s_min[tid] = ~0ull;
   __syncthreads();
   const int j0 = tid * CT_ITEMS;
 #pragma unroll
   for (int q = 0; q < CT_ITEMS; q++) {
     const int j = j0 + q;
     if (j >= (int)cnt || !(s.fl[j] & FL_INT)) continue;
-    const u32 p = pos_of(L, s.key[j + 1]);
+    // (position, entry index): the witness is the min POSITION (with an unsorted-input layout, entries of a run
+    // are ordered by (block, interval) first); the entry index locates its record in mode 3
+    const unsigned long long p = ((unsigned long long)pos_of(L, s.key[j + 1]) << 32) | (u32)(tb + j);
     const bool A = cin && j <= ftail, B = cout && j >= lhead;
     if (A) {
       if (s.res[j] & 1) atomicMin(&s_min[0], p);
@@ -554,13 +562,13 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
   if (tid == 0) {
     if (cin) {
       Slot* sl = &a.slots[a.owner[tile]];
-      if (s_min[0] != ~0u) atomicMin(&sl->x[0], s_min[0]);
-      if (s_min[1] != ~0u) atomicMin(&sl->x[1], s_min[1]);
+      if (s_min[0] != ~0ull) atomicMin((unsigned long long*)&sl->x[0], s_min[0]);
+      if (s_min[1] != ~0ull) atomicMin((unsigned long long*)&sl->x[1], s_min[1]);
     }
     if (cout && lhead >= 0 && !(cin && lhead <= ftail)) {
       Slot* sl = &a.slots[tile];
-      if (s_min[2] != ~0u) atomicMin(&sl->x[0], s_min[2]);
-      if (s_min[3] != ~0u) atomicMin(&sl->x[1], s_min[3]);
+      if (s_min[2] != ~0ull) atomicMin((unsigned long long*)&sl->x[0], s_min[2]);
+      if (s_min[3] != ~0ull) atomicMin((unsigned long long*)&sl->x[1], s_min[3]);
     }
   }
 }
@@ -578,7 +586,8 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_y_kernel(ConflictArgs a) 
   const bool cin = !(s.fl[0] & FL_GH), cout = !(s.fl[cnt - 1] & FL_GT);
   const int ftail = s.first_gtail, lhead = s.last_ghead;
   __shared__ F5 s_x[2][2];
-  __shared__ u32 s_has[2][2], s_min[2][2];
+  __shared__ u32 s_has[2][2];
+  __shared__ unsigned long long s_min[2][2];
   __shared__ u32 s_owner[2];
   if (tid == 0) {
     s_owner[0] = cin ? a.owner[tile] : ~0u;
@@ -588,11 +597,12 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_y_kernel(ConflictArgs a) 
   if (tid < 4) {
     const int g = tid >> 1, k = tid & 1;
     s_has[g][k] = 0;
-    s_min[g][k] = ~0u;
+    s_min[g][k] = ~0ull;
     if (s_owner[g] != ~0u) {
-      const u32 x = a.slots[s_owner[g]].x[k];
-      if (x != ~0u) {
-        const Rec r = load_rec(a.rec + x);
+      const u64 xp = a.slots[s_owner[g]].x[k];
+      if (xp != ~0ull) {
+        const u32 x = (u32)(xp & 0xFFFFFFFFull);
+        const Rec r = rec_at(a, x, a.keys[x]);
         F5 f;
         f.block = r.block, f.interval = r.interval, f.thread = r.thread, f.rw = r.rw, f.vh = r.vh;
         s_x[g][k] = f;
@@ -610,14 +620,15 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_y_kernel(ConflictArgs a) 
     const int g = A ? 0 : (B ? 1 : -1);
     if (g < 0) continue;
     const F5 me = fields(s, j);
-    const u32 p = pos_of(L, s.key[j + 1]);
+    const unsigned long long p = ((unsigned long long)pos_of(L, s.key[j + 1]) << 32) | (u32)(tb + j);
     for (int k = 0; k < 2; k++)
       if (s_has[g][k] && pair_kind(s_x[g][k], me, a.ws, a.ls) == (u32)(k + 1)) atomicMin(&s_min[g][k], p);
   }
   __syncthreads();
   if (tid < 4) {
     const int g = tid >> 1, k = tid & 1;
-    if (s_owner[g] != ~0u && s_min[g][k] != ~0u) atomicMin(&a.slots[s_owner[g]].y[k], s_min[g][k]);
+    if (s_owner[g] != ~0u && s_min[g][k] != ~0ull)
+      atomicMin((unsigned long long*)&a.slots[s_owner[g]].y[k], s_min[g][k]);
   }
 }
 
@@ -632,7 +643,9 @@ __global__ void cross_emit_kernel(ConflictArgs a, u32 ncross) {
   // head is the crossing group's head (slots[tile] was written by mode 1)
   const Slot sl = a.slots[tile];
   for (int k = 0; k < 2; k++)
-    if (sl.x[k] != ~0u) emit_race(a, sl.head_key >> a.L.pos_bits, (u32)(k + 1), sl.x[k], sl.y[k], sl.hblock, sl.hinterval);
+    if (sl.x[k] != ~0ull)  // (position << 32 | entry): report positions
+      emit_race(a, sl.head_key >> a.L.pos_bits, (u32)(k + 1), (u32)(sl.x[k] >> 32), (u32)(sl.y[k] >> 32), sl.hblock,
+                sl.hinterval);
 }
 
 u32 conflict_tiles(u64 m) { return (u32)((m + CT_TILE - 1) / CT_TILE); }
@@ -793,6 +806,23 @@ void launch_carry(const ConflictArgs& a, u32 ntiles, void* temp, cudaStream_t st
   carry_chunk_kernel<<<nch, CARRY_T, 0, st>>>(a, ntiles, tot, fl);
   carry_top_kernel<<<1, CARRY_T, 0, st>>>(nch, tot, fl, car);
   carry_apply_kernel<<<nch, CARRY_T, 0, st>>>(a, ntiles, car);
+}
+
+// canonical sort key of a race record (as emitted by emit_race) rebuilt from its fields (rank-0 merge)
+__global__ void race_rekey_kernel(const RaceOut* __restrict__ r, u64 n, KeyLayout L, u64* __restrict__ keys,
+                                  u32* __restrict__ vals) {
+  const u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const RaceOut x = r[i];
+  // global races carry block = interval = NOBI: use the layout minima so the (masked) low fields stay zero
+  const bool glob = x.space == SP_GLOBAL;
+  const u64 hi = key_hi_of(L, x.space, glob ? L.bminG : x.block, glob ? L.iminG : x.interval, x.addr >> L.log2G);
+  keys[i] = (group_of_hi(L, hi) << 1) | (u64)(x.kind - 1);
+  vals[i] = (u32)i;
+}
+
+void race_rekey_launch(const RaceOut* r, u64 n, const KeyLayout& L, u64* keys, u32* vals, cudaStream_t st) {
+  if (n) race_rekey_kernel<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(r, n, L, keys, vals);
 }
 
 __global__ void permute_races_kernel(const RaceOut* __restrict__ in, const u32* __restrict__ order,

@@ -150,7 +150,8 @@ void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, int grid, 
 template <int THREADS, int RB>
 __global__ void __launch_bounds__(THREADS) extract_1to1_kernel(const Rec* __restrict__ rec, u64 n, KeyLayout L,
                                                                 u32 npass, u64* __restrict__ keys,
-                                                                u32* __restrict__ hist /* [npass][1<<RB] */) {
+                                                                u32* __restrict__ hist /* [npass][1<<RB] */,
+                                                                u64 pos_base) {
   constexpr int RADIX = 1 << RB;
   extern __shared__ __align__(128) unsigned char smem[];
   __shared__ u64 bars[EX_STAGES];
@@ -169,7 +170,7 @@ __global__ void __launch_bounds__(THREADS) extract_1to1_kernel(const Rec* __rest
       const u32 t = h * THREADS + threadIdx.x;
       if (t >= nr) continue;
       const Rec& x = R[t];
-      const u64 key = (key_hi_of(L, x.space, x.block, x.interval, x.addr >> L.log2G) << L.pos_bits) | (c0 + t);
+      const u64 key = (key_hi_of(L, x.space, x.block, x.interval, x.addr >> L.log2G) << L.pos_bits) | (pos_base + c0 + t);
       __stcs(keys + c0 + t, key);
       for (u32 p = 0; p < npass; p++) atomicAdd(&wsh[p * RADIX + ((key >> (L.pos_bits + p * RB)) & (RADIX - 1))], 1u);
     }
@@ -183,8 +184,8 @@ __global__ void __launch_bounds__(THREADS) extract_1to1_kernel(const Rec* __rest
   }
 }
 
-void launch_extract_1to1(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, u64* keys, u32* hist, int,
-                         cudaStream_t st) {
+void launch_extract_1to1(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, u64* keys, u32* hist, u64 pos_base,
+                         int, cudaStream_t st) {
   static int grids[9] = {0};
   const size_t sm = (size_t)EX_STAGES * EX_CHUNK + (size_t)npass * 8 * RADIX * 4;  // ring + npass x 8 warps hist
   if (!grids[npass])
@@ -193,7 +194,7 @@ void launch_extract_1to1(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, u
   const int grid = grids[npass];
   const u64 chunks = (n * 32 + EX_CHUNK - 1) / EX_CHUNK;
   extract_1to1_kernel<256, RADIX_BITS><<<(unsigned)std::min<u64>(chunks, (u64)grid), 256, sm, st>>>(rec, n, L, npass,
-                                                                                                   keys, hist);
+                                                                                                   keys, hist, pos_base);
 }
 
 // ------------------------------------------------------------------------------------------------------------
@@ -211,7 +212,8 @@ __global__ void entry_count_kernel(const Rec* __restrict__ rec, u64 n, u32 log2G
 template <int THREADS, int RB>
 __global__ void __launch_bounds__(THREADS) extract_multi_kernel(const Rec* __restrict__ rec, u64 n, KeyLayout L,
                                                                  u32 npass, const u32* __restrict__ off,
-                                                                 u64* __restrict__ keys, u32* __restrict__ hist) {
+                                                                 u64* __restrict__ keys, u32* __restrict__ hist,
+                                                                 u64 pos_base) {
   constexpr int RADIX = 1 << RB;
   extern __shared__ u32 sh[];
   for (u32 i = threadIdx.x; i < npass * RADIX; i += THREADS) sh[i] = 0;
@@ -222,7 +224,7 @@ __global__ void __launch_bounds__(THREADS) extract_multi_kernel(const Rec* __res
     u64 glo = r.addr >> L.log2G, ghi = (r.addr + (u64)(r.size - 1)) >> L.log2G;
     u64 o = off[k];
     for (u64 g = glo; g <= ghi; g++, o++) {
-      u64 key = (key_hi_of(L, r.space, r.block, r.interval, g) << L.pos_bits) | k;
+      u64 key = (key_hi_of(L, r.space, r.block, r.interval, g) << L.pos_bits) | (pos_base + k);
       keys[o] = key;
       for (u32 p = 0; p < npass; p++) atomicAdd(&sh[p * RADIX + ((key >> (L.pos_bits + p * RB)) & (RADIX - 1))], 1u);
     }
@@ -237,9 +239,9 @@ void launch_entry_count(const Rec* rec, u64 n, u32 log2G, u32* cnt, cudaStream_t
 }
 
 void launch_extract_multi(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, const u32* off, u64* keys,
-                          u32* hist, int grid, cudaStream_t st) {
+                          u32* hist, u64 pos_base, int grid, cudaStream_t st) {
   size_t smem = (size_t)npass * (1 << RADIX_BITS) * sizeof(u32);
-  extract_multi_kernel<256, RADIX_BITS><<<grid, 256, smem, st>>>(rec, n, L, npass, off, keys, hist);
+  extract_multi_kernel<256, RADIX_BITS><<<grid, 256, smem, st>>>(rec, n, L, npass, off, keys, hist, pos_base);
 }
 
 }  // namespace sesa

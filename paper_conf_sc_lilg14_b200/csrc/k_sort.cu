@@ -546,24 +546,28 @@ void launch_onesweep(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m
   if (want) sort_prof_dump(m, st, dprof, sort_tile_keys());
 }
 
-// digit histograms of plain keys (race list sort): npass 8-bit digits from bit 0
-__global__ void hist_keys_kernel(const u64* __restrict__ keys, u32 m, u32 npass, u32* __restrict__ hist) {
+// digit histograms of plain keys: npass 8-bit digits from bit `shift` (race lists: 0; exchanged keys: pos_bits)
+__global__ void hist_keys_kernel(const u64* __restrict__ keys, u32 m, u32 npass, u32 shift, u32* __restrict__ hist) {
   extern __shared__ u32 sh[];
   for (u32 i = threadIdx.x; i < npass * RADIX; i += blockDim.x) sh[i] = 0;
   __syncthreads();
   for (u32 k = blockIdx.x * blockDim.x + threadIdx.x; k < m; k += gridDim.x * blockDim.x) {
     u64 key = keys[k];
-    for (u32 p = 0; p < npass; p++) atomicAdd(&sh[p * RADIX + ((key >> (p * RADIX_BITS)) & (RADIX - 1))], 1u);
+    for (u32 p = 0; p < npass; p++) atomicAdd(&sh[p * RADIX + ((key >> (shift + p * RADIX_BITS)) & (RADIX - 1))], 1u);
   }
   __syncthreads();
   for (u32 i = threadIdx.x; i < npass * RADIX; i += blockDim.x)
     if (sh[i]) atomicAdd(&hist[i], sh[i]);
 }
 
-void launch_hist_keys(const u64* keys, u32 m, u32 npass, u32* hist, cudaStream_t st) {
+void launch_hist_keys_shift(const u64* keys, u32 m, u32 npass, u32 shift, u32* hist, cudaStream_t st) {
   if (!m || !npass) return;
   u32 grid = min((m + 255) / 256, 1184u);
-  hist_keys_kernel<<<grid, 256, npass * RADIX * 4, st>>>(keys, m, npass, hist);
+  hist_keys_kernel<<<grid, 256, npass * RADIX * 4, st>>>(keys, m, npass, shift, hist);
+}
+
+void launch_hist_keys(const u64* keys, u32 m, u32 npass, u32* hist, cudaStream_t st) {
+  launch_hist_keys_shift(keys, m, npass, 0, hist, st);
 }
 
 }  // namespace sesa

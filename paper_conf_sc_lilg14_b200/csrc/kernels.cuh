@@ -19,11 +19,11 @@ constexpr int CT_TILE = CT_THREADS * CT_ITEMS;
 
 // k_extract.cu
 void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, int grid, cudaStream_t st);
-void launch_extract_1to1(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, u64* keys, u32* hist, int grid,
-                         cudaStream_t st);
+void launch_extract_1to1(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, u64* keys, u32* hist, u64 pos_base,
+                         int grid, cudaStream_t st);
 void launch_entry_count(const Rec* rec, u64 n, u32 log2G, u32* cnt, cudaStream_t st);
 void launch_extract_multi(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, const u32* off, u64* keys,
-                          u32* hist, int grid, cudaStream_t st);
+                          u32* hist, u64 pos_base, int grid, cudaStream_t st);
 
 // k_util.cu
 size_t scan_u32_temp_bytes(u64 n);
@@ -38,6 +38,7 @@ u32 sort_tile_keys();
 inline u32 sort_tiles(u64 m) { return (u32)((m + SORT_TILE - 1) / SORT_TILE); }  // upper bound (smallest tile)
 // race-list keys: (race key, index) -> histograms for npass digits starting at bit 0
 void launch_hist_keys(const u64* keys, u32 m, u32 npass, u32* hist, cudaStream_t st);
+void launch_hist_keys_shift(const u64* keys, u32 m, u32 npass, u32 shift, u32* hist, cudaStream_t st);
 
 // k_conflict.cu — see the file header for the three modes.
 // Summary of a set of entries at one level (identity = thread within a sub-run, block within a group).
@@ -53,7 +54,9 @@ struct AggQuad {
 struct ConflictArgs {
   const u64* keys;  // sorted entry keys
   u32 m;            // entries
-  const Rec* rec;   // records (gathered by position)
+  const Rec* rec;   // records (gathered by position - rec_pos_base) ...
+  const Rec* rec_entry;  // ... or, if set, entry-aligned records (distributed check: fetched from owners)
+  u32 rec_pos_base;
   u64 n;
   KeyLayout L;
   u32 ws, ls;
@@ -84,8 +87,8 @@ static_assert(sizeof(RaceOut) == 40, "race layout");
 
 // per-owner-tile slot for a group crossing tile boundaries
 struct Slot {
-  u32 x[2];      // min flagged position per kind (RW, WW), ~0 = none
-  u32 y[2];      // min partner position of x per kind
+  u64 x[2];      // min over flagged entries of (position << 32 | entry index) per kind (RW, WW), ~0 = none
+  u64 y[2];      // min over partners of x of (position << 32 | entry index) per kind
   u64 head_key;  // key of the group's first entry
   u32 hblock, hinterval;
 };
@@ -95,6 +98,7 @@ void launch_carry(const ConflictArgs& a, u32 ntiles, void* temp, cudaStream_t st
 size_t carry_temp_bytes(u32 ntiles);
 void launch_cross_emit(const ConflictArgs& a, u32 ntiles, cudaStream_t st);
 void launch_permute_races(const RaceOut* in, const u32* order, RaceOut* out, u32 nr, cudaStream_t st);
+void race_rekey_launch(const RaceOut* r, u64 n, const KeyLayout& L, u64* keys, u32* vals, cudaStream_t st);
 u32 conflict_tiles(u64 m);
 
 // k_compact.cu — keep only entries of locations touched >= 2 times (order preserved); *total = count

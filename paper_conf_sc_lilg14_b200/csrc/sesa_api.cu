@@ -63,6 +63,7 @@ void sesa_trace::free_all() {
 // ------------------------------------------------------------------------------------------------ profiling
 void sesa_trace::launch_begin(const char* name) {
   launches++;
+  prof_last = name;
   if (!profiling) return;
   ProfRec r;
   r.name = name;
@@ -71,6 +72,12 @@ void sesa_trace::launch_begin(const char* name) {
   prof.push_back(r);
 }
 void sesa_trace::launch_end(double bytes) {
+  static const bool dbg = getenv("SESA_SYNC_DEBUG") != nullptr;
+  if (dbg) {  // pinpoint the failing launch
+    cudaError_t e = cudaStreamSynchronize(stream);
+    if (e == cudaSuccess) e = cudaGetLastError();
+    if (e != cudaSuccess) fprintf(stderr, "[sesa debug] after %s: %s\n", prof_last.c_str(), cudaGetErrorString(e));
+  }
   if (!profiling) return;
   ProfRec& r = prof.back();
   r.ev1 = next_event();
@@ -161,7 +168,7 @@ bool sesa_trace::make_layout(const Summary& S, u64 n) {
   return true;
 }
 
-sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_base) {
+void sesa_trace::begin_check(u64 n) {
   status = SESA_OK;
   err.clear();
   have_result = false;
@@ -171,85 +178,100 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
   ev_used = 0;
   memset(&info, 0, sizeof info);
   info.n_records = n;
-  if (n == 0) {
-    have_result = true;
-    collect_prof();
-    return SESA_OK;
-  }
-  if (!d_rec) return fail(SESA_EINVAL, "d_records is NULL"), status;
-  cudaPointerAttributes pa;
-  if (cudaPointerGetAttributes(&pa, d_rec) != cudaSuccess || (pa.type != cudaMemoryTypeDevice && pa.type != cudaMemoryTypeManaged)) {
-    cudaGetLastError();
-    return fail(SESA_EINVAL, "d_records is not device memory (use sesa_race_check_host for host buffers)"), status;
-  }
-  if (n >= (1ull << 31)) return fail(SESA_ERANGE, "n = %llu >= 2^31 records (ABI v1 limit)", (unsigned long long)n), status;
-  const Rec* rec = reinterpret_cast<const Rec*>(d_rec);
-  const u32 log2G = (u32)__builtin_ctz(cfg.granularity);
+}
 
-  // 1. validate + extents
-  if (!grow(b_summary, sizeof(Summary), "summary")) return status;
+bool sesa_trace::check_records_ptr(const sesa_access* d_rec, u64 n) {
+  if (!d_rec) return fail(SESA_EINVAL, "d_records is NULL"), false;
+  cudaPointerAttributes pa;
+  if (cudaPointerGetAttributes(&pa, d_rec) != cudaSuccess ||
+      (pa.type != cudaMemoryTypeDevice && pa.type != cudaMemoryTypeManaged)) {
+    cudaGetLastError();
+    return fail(SESA_EINVAL, "d_records is not device memory (use sesa_race_check_host for host buffers)"), false;
+  }
+  if (n >= (1ull << 31)) return fail(SESA_ERANGE, "n = %llu >= 2^31 records (ABI v1 limit)", (unsigned long long)n), false;
+  return true;
+}
+
+// step 1: validation + extents of the local records -> h_summary (synchronises)
+bool sesa_trace::step_extents(const Rec* rec, u64 n) {
+  const u32 log2G = (u32)__builtin_ctz(cfg.granularity);
+  if (!grow(b_summary, sizeof(Summary), "summary")) return false;
   Summary init;
   memset(&init, 0, sizeof init);
   init.bad_index = ~0ull;
   init.gmin[0] = init.gmin[1] = ~0ull;
   init.bmin[0] = init.bmin[1] = init.imin[0] = init.imin[1] = ~0u;
   h_summary = init;
+  if (n == 0) return true;
   if (!cuda_ok(cudaMemcpyAsync(b_summary.p, &h_summary, sizeof(Summary), cudaMemcpyHostToDevice, stream), "summary init"))
-    return status;
+    return false;
   const int grid_stream = (int)std::min<u64>((n + 255) / 256, (u64)num_sms * 8);
   LAUNCH("extents", 32.0 * n, launch_extents(rec, n, log2G, (Summary*)b_summary.p, grid_stream, stream));
   if (!cuda_ok(cudaMemcpyAsync(&h_summary, b_summary.p, sizeof(Summary), cudaMemcpyDeviceToHost, stream), "summary"))
-    return status;
-  if (!sync_check("extents")) return status;
-  const Summary& S = h_summary;
-  if (S.bad_index != ~0ull) {
-    sesa_access r;
-    cudaMemcpy(&r, d_rec + S.bad_index, sizeof r, cudaMemcpyDeviceToHost);
-    return fail(SESA_EINVAL, "record %llu invalid (space=%u rw=%u size=%u addr=0x%llx)",
-                (unsigned long long)S.bad_index, r.space, r.rw, r.size, (unsigned long long)r.addr),
-           status;
-  }
-  const u64 m = S.entries;
-  info.n_entries = m;
-  info.sorted_input = !S.unsorted;
-  if (m >= (1ull << 31)) return fail(SESA_ERANGE, "%llu entries >= 2^31 (ABI v1 limit)", (unsigned long long)m), status;
-  if (!make_layout(S, n)) return status;
+    return false;
+  return sync_check("extents");
+}
+
+bool sesa_trace::report_bad(const sesa_access* d_rec, u64 local_bad, u64 global_bad) {
+  sesa_access r;
+  cudaMemcpy(&r, d_rec + local_bad, sizeof r, cudaMemcpyDeviceToHost);
+  fail(SESA_EINVAL, "record %llu invalid (space=%u rw=%u size=%u addr=0x%llx)", (unsigned long long)global_bad, r.space,
+       r.rw, r.size, (unsigned long long)r.addr);
+  return false;
+}
+
+// step 2: keys (+ the histograms of every sort digit) of the local records at positions pos_base + i -> b_keys[0]
+bool sesa_trace::step_extract(const Rec* rec, u64 n, u64 m, u64 pos_base, bool multi) {
   const KeyLayout& L = layout;
   const u32 npass = (L.sort_bits + RADIX_BITS - 1) / RADIX_BITS;
-  info.sort_bits = L.sort_bits;
-  info.pos_bits = L.pos_bits;
-  info.digit_bits = RADIX_BITS;
-
-  // 2. key extraction + digit histograms
+  const u32 log2G = L.log2G;
   if (!grow(b_keys[0], m * 8 + 64, "keys") || !grow(b_keys[1], m * 8 + 64, "keys") ||
       !grow(b_hist, (size_t)std::max(npass, 1u) * RADIX * 4, "hist") ||
       !grow(b_binbase, (size_t)std::max(npass, 1u) * RADIX * 8, "binbase"))
-    return status;
+    return false;
   cudaMemsetAsync(b_hist.p, 0, (size_t)std::max(npass, 1u) * RADIX * 4, stream);
+  if (n == 0) return true;
   u64* keys = (u64*)b_keys[0].p;
-  if (S.multi == 0) {
-    LAUNCH("extract", 40.0 * n,
-           launch_extract_1to1(rec, n, L, npass, keys, (u32*)b_hist.p, grid_stream, stream));
+  const int grid_stream = (int)std::min<u64>((n + 255) / 256, (u64)num_sms * 8);
+  if (!multi) {
+    LAUNCH("extract", 40.0 * n, launch_extract_1to1(rec, n, L, npass, keys, (u32*)b_hist.p, pos_base, grid_stream, stream));
   } else {
     if (!grow(b_cnt, n * 4, "counts") || !grow(b_off, n * 4, "offsets") || !grow(b_temp, scan_u32_temp_bytes(n), "scan"))
-      return status;
+      return false;
     LAUNCH("entry_count", 36.0 * n, launch_entry_count(rec, n, log2G, (u32*)b_cnt.p, stream));
     LAUNCH("scan", 8.0 * n, launch_scan_exclusive_u32((u32*)b_cnt.p, (u32*)b_off.p, n, b_temp.p, stream));
     LAUNCH("extract_multi", 36.0 * n + 8.0 * m,
-           launch_extract_multi(rec, n, L, npass, (u32*)b_off.p, keys, (u32*)b_hist.p, grid_stream, stream));
+           launch_extract_multi(rec, n, L, npass, (u32*)b_off.p, keys, (u32*)b_hist.p, pos_base, grid_stream, stream));
   }
+  return true;
+}
+
+// step 2' (distributed): histograms of keys that arrived from the exchange (already in b_keys[0])
+bool sesa_trace::step_hist(u64 m) {
+  const u32 npass = (layout.sort_bits + RADIX_BITS - 1) / RADIX_BITS;
+  if (!grow(b_hist, (size_t)std::max(npass, 1u) * RADIX * 4, "hist") ||
+      !grow(b_binbase, (size_t)std::max(npass, 1u) * RADIX * 8, "binbase"))
+    return false;
+  cudaMemsetAsync(b_hist.p, 0, (size_t)std::max(npass, 1u) * RADIX * 4, stream);
+  LAUNCH("hist", 8.0 * m, launch_hist_keys_shift((const u64*)b_keys[0].p, (u32)m, npass, layout.pos_bits,
+                                                 (u32*)b_hist.p, stream));
+  return true;
+}
+
+// step 3: LSD onesweep passes over the non-trivial digits of b_keys[0] (m keys); result in b_keys[*cur]
+bool sesa_trace::step_sort(u64 m, int* cur_out) {
+  const KeyLayout& L = layout;
+  const u32 npass = (L.sort_bits + RADIX_BITS - 1) / RADIX_BITS;
   std::vector<u32> hist((size_t)npass * RADIX);
-  if (npass) {
+  if (npass && m) {
     if (!cuda_ok(cudaMemcpyAsync(hist.data(), b_hist.p, hist.size() * 4, cudaMemcpyDeviceToHost, stream), "hist"))
-      return status;
+      return false;
     LAUNCH("bin_base", 0.0, launch_bin_base((u32*)b_hist.p, (u64*)b_binbase.p, npass, stream));
   }
-  if (!sync_check("extract")) return status;
-
-  // 3. onesweep LSD passes over the non-trivial digits
+  if (!sync_check("extract")) return false;
   const u32 stiles = sort_tiles(m);
-  if (npass) {
-    if (!grow(b_lookback, (size_t)stiles * RADIX * 8, "lookback") || !grow(b_ctr, 64 * 4, "counters")) return status;
+  if (npass && m) {
+    if (!grow(b_lookback, (size_t)stiles * RADIX * 8, "lookback") || !grow(b_ctr, 64 * 4, "counters")) return false;
     if (b_lookback.cap != lookback_cleared) {  // fresh allocation: clear once, epochs do the rest
       cudaMemsetAsync(b_lookback.p, 0, b_lookback.cap, stream);
       lookback_cleared = b_lookback.cap;
@@ -259,7 +281,7 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
   }
   int cur = 0;
   u32 passes_run = 0;
-  for (u32 p = 0; p < npass; p++) {
+  for (u32 p = 0; p < npass && m; p++) {
     const u32* h = hist.data() + (size_t)p * RADIX;
     if (*std::max_element(h, h + RADIX) == m) continue;  // trivial digit: every key has the same value
     if (++epoch >= 256) {
@@ -274,19 +296,30 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
     passes_run++;
   }
   info.sort_passes = passes_run;
+  *cur_out = cur;
+  return true;
+}
 
-  // 4a. keep only entries of locations touched at least twice (order-preserving compaction)
-  if (!grow(b_ctmp, compact_temp_bytes(m), "compact temp") || !grow(b_ctotal, 16, "compact count")) return status;
-  u64* comp = (u64*)b_keys[cur ^ 1].p;
-  LAUNCH("compact", 8.0 * m, launch_compact_multi((const u64*)b_keys[cur].p, (u32)m, L, comp, b_ctmp.p,
-                                                  (u32*)b_ctotal.p, stream));
-  u32 m2 = 0;
-  if (!cuda_ok(cudaMemcpyAsync(&m2, b_ctotal.p, 4, cudaMemcpyDeviceToHost, stream), "compact count")) return status;
-  if (!sync_check("compact")) return status;
-  info.n_multi = m2;
-  const u64* sorted = comp;
+// step 4: keep entries of locations touched >= 2 times (into the other key buffer) -> (*comp, *m2)
+bool sesa_trace::step_compact(int cur, u64 m, u64** comp, u32* m2) {
+  *comp = (u64*)b_keys[cur ^ 1].p;
+  *m2 = 0;
+  if (m == 0) return true;
+  if (!grow(b_ctmp, compact_temp_bytes(m), "compact temp") || !grow(b_ctotal, 16, "compact count")) return false;
+  LAUNCH("compact", 16.0 * m, launch_compact_multi((const u64*)b_keys[cur].p, (u32)m, layout, *comp, b_ctmp.p,
+                                                   (u32*)b_ctotal.p, stream));
+  if (!cuda_ok(cudaMemcpyAsync(m2, b_ctotal.p, 4, cudaMemcpyDeviceToHost, stream), "compact count")) return false;
+  if (!sync_check("compact")) return false;
+  info.n_multi = *m2;
+  return true;
+}
 
-  // 4. conflict tiles
+// step 5: conflict tiles (+ crossing carries) over the m2 compacted entries -> unsorted races (b_races, b_rkeys[0],
+// b_rvals[0]); n_races set.  Records come by position (rec - rec_pos_base) or entry-aligned (rec_entry).
+bool sesa_trace::step_conflict(const u64* comp, u32 m2, const Rec* rec, u32 rec_pos_base, const Rec* rec_entry,
+                               u64 index_base) {
+  n_races = 0;
+  if (m2 == 0) return true;
   const u32 ctiles = conflict_tiles(m2);
   u32 race_cap = (u32)std::min<u64>(std::max<u64>(race_cap_hint, 1u << 16), 2 * (u64)m2 + 16);
   for (int attempt = 0; attempt < 3; attempt++) {
@@ -297,15 +330,16 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
         !grow(b_rkeys[0], (size_t)race_cap * 8, "race keys") || !grow(b_rkeys[1], (size_t)race_cap * 8, "race keys") ||
         !grow(b_rvals[0], (size_t)race_cap * 4, "race vals") || !grow(b_rvals[1], (size_t)race_cap * 4, "race vals") ||
         !grow(b_carrytmp, carry_temp_bytes(ctiles), "carry temp"))
-      return status;
+      return false;
     cudaMemsetAsync(b_ccount.p, 0, 16, stream);
     ConflictArgs A;
     memset(&A, 0, sizeof A);
-    A.keys = sorted;
+    A.keys = comp;
     A.m = m2;
     A.rec = rec;
-    A.n = n;
-    A.L = L;
+    A.rec_entry = rec_entry;
+    A.rec_pos_base = rec_pos_base;
+    A.L = layout;
     A.ws = cfg.warp_size;
     A.ls = cfg.lockstep;
     A.race_count = (u32*)b_ccount.p;
@@ -323,60 +357,96 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
     A.index_base = index_base;
     LAUNCH("conflict", 40.0 * m2, launch_conflict(1, A, ctiles, stream));
     u32 cc[2];
-    if (!cuda_ok(cudaMemcpyAsync(cc, b_ccount.p, 8, cudaMemcpyDeviceToHost, stream), "counts")) return status;
-    if (!sync_check("conflict")) return status;
+    if (!cuda_ok(cudaMemcpyAsync(cc, b_ccount.p, 8, cudaMemcpyDeviceToHost, stream), "counts")) return false;
+    if (!sync_check("conflict")) return false;
     info.crossing_tiles = cc[1];
     if (cc[1]) {
       LAUNCH("carry", 0.0, launch_carry(A, ctiles, b_carrytmp.p, stream));
       LAUNCH("conflict_cross", 0.0, launch_conflict(2, A, cc[1], stream));
       LAUNCH("conflict_y", 0.0, launch_conflict(3, A, cc[1], stream));
       LAUNCH("cross_emit", 0.0, launch_cross_emit(A, cc[1], stream));
-      if (!cuda_ok(cudaMemcpyAsync(cc, b_ccount.p, 8, cudaMemcpyDeviceToHost, stream), "counts")) return status;
-      if (!sync_check("crossing")) return status;
+      if (!cuda_ok(cudaMemcpyAsync(cc, b_ccount.p, 8, cudaMemcpyDeviceToHost, stream), "counts")) return false;
+      if (!sync_check("crossing")) return false;
     }
     if (cc[0] <= race_cap) {
       n_races = cc[0];
-      break;
+      return true;
     }
     race_cap = (u32)std::min<u64>((u64)cc[0] + cc[0] / 8 + 1024, 2 * (u64)m2 + 16);
     race_cap_hint = race_cap;
   }
+  return fail(SESA_ECUDA, "race list did not fit after retries"), false;
+}
 
-  // 5. canonical order of the race list: sort (location key << 1 | kind, index), then permute
+// step 6: canonical order of nr races: sort (location key << 1 | kind, index), permute into `out`
+bool sesa_trace::step_race_sort(u32 nr, const RaceOut* races, u64* rkeys0, u32* rvals0, u64* rkeys1, u32* rvals1,
+                                RaceOut* out) {
+  if (nr == 0) return true;
+  const u32 rbits = layout.sort_bits + 1;
+  const u32 rpass = (rbits + RADIX_BITS - 1) / RADIX_BITS;
+  const u32 rtiles = sort_tiles(nr);
+  if (!grow(b_rhist, (size_t)rpass * RADIX * 4, "race hist") || !grow(b_rbase, (size_t)rpass * RADIX * 8, "race base") ||
+      !grow(b_lookback, (size_t)rtiles * RADIX * 8, "lookback") || !grow(b_ctr, 64 * 4, "counters"))
+    return false;
+  if (b_lookback.cap != lookback_cleared) {
+    cudaMemsetAsync(b_lookback.p, 0, b_lookback.cap, stream);
+    lookback_cleared = b_lookback.cap;
+    epoch = 0;
+  }
+  cudaMemsetAsync(b_rhist.p, 0, (size_t)rpass * RADIX * 4, stream);
+  cudaMemsetAsync((u32*)b_ctr.p + 32, 0, 32 * 4, stream);
+  LAUNCH("race_hist", 8.0 * nr, launch_hist_keys(rkeys0, nr, rpass, (u32*)b_rhist.p, stream));
+  LAUNCH("bin_base", 0.0, launch_bin_base((u32*)b_rhist.p, (u64*)b_rbase.p, rpass, stream));
+  u64* k[2] = {rkeys0, rkeys1};
+  u32* v[2] = {rvals0, rvals1};
+  int rc = 0;
+  for (u32 p = 0; p < rpass; p++) {
+    if (++epoch >= 256) {
+      cudaMemsetAsync(b_lookback.p, 0, b_lookback.cap, stream);
+      epoch = 1;
+    }
+    LAUNCH("race_sort", 24.0 * nr,
+           launch_onesweep(k[rc], k[rc ^ 1], v[rc], v[rc ^ 1], nr, p * RADIX_BITS, (u64*)b_rbase.p + (size_t)p * RADIX,
+                           (u64*)b_lookback.p, (u32*)b_ctr.p + 32 + p, epoch, stream));
+    rc ^= 1;
+  }
+  LAUNCH("race_permute", 80.0 * nr, launch_permute_races(races, v[rc], out, nr, stream));
+  return true;
+}
+
+sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_base) {
+  begin_check(n);
+  if (n == 0) {
+    have_result = true;
+    collect_prof();
+    return SESA_OK;
+  }
+  if (!check_records_ptr(d_rec, n)) return status;
+  const Rec* rec = reinterpret_cast<const Rec*>(d_rec);
+  if (!step_extents(rec, n)) return status;
+  const Summary& S = h_summary;
+  if (S.bad_index != ~0ull) return report_bad(d_rec, S.bad_index, S.bad_index), status;
+  const u64 m = S.entries;
+  info.n_entries = m;
+  info.sorted_input = !S.unsorted;
+  if (m >= (1ull << 31)) return fail(SESA_ERANGE, "%llu entries >= 2^31 (ABI v1 limit)", (unsigned long long)m), status;
+  if (!make_layout(S, n)) return status;
+  info.sort_bits = layout.sort_bits;
+  info.pos_bits = layout.pos_bits;
+  info.digit_bits = RADIX_BITS;
+  if (!step_extract(rec, n, m, 0, S.multi != 0)) return status;
+  int cur = 0;
+  if (!step_sort(m, &cur)) return status;
+  u64* comp = nullptr;
+  u32 m2 = 0;
+  if (!step_compact(cur, m, &comp, &m2)) return status;
+  if (!step_conflict(comp, m2, rec, 0, nullptr, index_base)) return status;
   const u32 nr = (u32)n_races;
   info.n_races = nr;
   if (!grow(b_races_sorted, (size_t)std::max(nr, 1u) * sizeof(RaceOut), "sorted races")) return status;
-  if (nr) {
-    const u32 rbits = L.sort_bits + 1;
-    const u32 rpass = (rbits + RADIX_BITS - 1) / RADIX_BITS;
-    const u32 rtiles = sort_tiles(nr);
-    if (!grow(b_rhist, (size_t)rpass * RADIX * 4, "race hist") || !grow(b_rbase, (size_t)rpass * RADIX * 8, "race base") ||
-        !grow(b_lookback, (size_t)std::max(rtiles, stiles) * RADIX * 8, "lookback") || !grow(b_ctr, 64 * 4, "counters"))
-      return status;
-    if (b_lookback.cap != lookback_cleared) {
-      cudaMemsetAsync(b_lookback.p, 0, b_lookback.cap, stream);
-      lookback_cleared = b_lookback.cap;
-      epoch = 0;
-    }
-    cudaMemsetAsync(b_rhist.p, 0, (size_t)rpass * RADIX * 4, stream);
-    cudaMemsetAsync((u32*)b_ctr.p + 32, 0, 32 * 4, stream);
-    LAUNCH("race_hist", 8.0 * nr, launch_hist_keys((u64*)b_rkeys[0].p, nr, rpass, (u32*)b_rhist.p, stream));
-    LAUNCH("bin_base", 0.0, launch_bin_base((u32*)b_rhist.p, (u64*)b_rbase.p, rpass, stream));
-    int rc = 0;
-    for (u32 p = 0; p < rpass; p++) {
-      if (++epoch >= 256) {
-        cudaMemsetAsync(b_lookback.p, 0, b_lookback.cap, stream);
-        epoch = 1;
-      }
-      LAUNCH("race_sort", 24.0 * nr,
-             launch_onesweep((u64*)b_rkeys[rc].p, (u64*)b_rkeys[rc ^ 1].p, (u32*)b_rvals[rc].p,
-                             (u32*)b_rvals[rc ^ 1].p, nr, p * RADIX_BITS, (u64*)b_rbase.p + (size_t)p * RADIX,
-                             (u64*)b_lookback.p, (u32*)b_ctr.p + 32 + p, epoch, stream));
-      rc ^= 1;
-    }
-    LAUNCH("race_permute", 80.0 * nr,
-           launch_permute_races((RaceOut*)b_races.p, (u32*)b_rvals[rc].p, (RaceOut*)b_races_sorted.p, nr, stream));
-  }
+  if (!step_race_sort(nr, (RaceOut*)b_races.p, (u64*)b_rkeys[0].p, (u32*)b_rvals[0].p, (u64*)b_rkeys[1].p,
+                      (u32*)b_rvals[1].p, (RaceOut*)b_races_sorted.p))
+    return status;
   if (!sync_check("race sort")) return status;
   info.launches = launches;
   collect_prof();

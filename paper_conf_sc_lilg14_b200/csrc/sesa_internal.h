@@ -65,6 +65,7 @@ struct sesa_trace {
   std::vector<cudaEvent_t> ev_pool;
   size_t ev_used = 0;
   std::vector<sesa_kernel_stat> stats;
+  std::string prof_last;
 
   // distributed
   bool dist = false;
@@ -82,6 +83,19 @@ struct sesa_trace {
   void collect_prof();
   bool make_layout(const sesa::Summary& S, uint64_t n);
   sesa_status check_device(const sesa_access* d_rec, uint64_t n, uint64_t index_base);
+  // pipeline steps (shared by the single-GPU and the distributed check)
+  void begin_check(uint64_t n);
+  bool check_records_ptr(const sesa_access* d_rec, uint64_t n);
+  bool step_extents(const sesa::Rec* rec, uint64_t n);
+  bool report_bad(const sesa_access* d_rec, uint64_t local_bad, uint64_t global_bad);
+  bool step_extract(const sesa::Rec* rec, uint64_t n, uint64_t m, uint64_t pos_base, bool multi);
+  bool step_hist(uint64_t m);
+  bool step_sort(uint64_t m, int* cur_out);
+  bool step_compact(int cur, uint64_t m, uint64_t** comp, uint32_t* m2);
+  bool step_conflict(const uint64_t* comp, uint32_t m2, const sesa::Rec* rec, uint32_t rec_pos_base,
+                     const sesa::Rec* rec_entry, uint64_t index_base);
+  bool step_race_sort(uint32_t nr, const sesa::RaceOut* races, uint64_t* rk0, uint32_t* rv0, uint64_t* rk1,
+                      uint32_t* rv1, sesa::RaceOut* out);
   sesa_status expand(const sesa_flow* d_flows, uint64_t nf, sesa_access* d_out, uint64_t cap, uint64_t* n_out);
   sesa_status check_dist(const sesa_access* d_rec, uint64_t n, uint64_t index_base);
   void destroy_dist();

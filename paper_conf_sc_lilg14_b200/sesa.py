@@ -55,7 +55,7 @@ class sesa_check_info(ctypes.Structure):
 EXPORTS = ["sesa_trace_create", "sesa_trace_create_dist", "sesa_nccl_unique_id", "sesa_race_check",
            "sesa_race_check_host", "sesa_races_get", "sesa_races_device", "sesa_expand", "sesa_trace_set_profiling",
            "sesa_trace_info", "sesa_trace_kernel_stats", "sesa_trace_destroy", "sesa_status_str", "sesa_last_error",
-           "sesa_abi_version"]
+           "sesa_abi_version", "sesa_race_check_loopback"]
 
 _lib = None
 
@@ -75,6 +75,7 @@ def load() -> ctypes.CDLL:
     lib.sesa_nccl_unique_id.argtypes = [P]
     lib.sesa_race_check.argtypes = [P, P, U64, U64, P]
     lib.sesa_race_check_host.argtypes = [P, P, U64, U64, P]
+    lib.sesa_race_check_loopback.argtypes = [ctypes.POINTER(sesa_config), P, P, I, U64, P, PP]
     lib.sesa_races_get.argtypes = [P, P, U64, ctypes.POINTER(U64)]
     lib.sesa_races_device.argtypes = [P, PP, ctypes.POINTER(U64)]
     lib.sesa_expand.argtypes = [P, P, U64, P, U64, ctypes.POINTER(U64), P]
@@ -221,6 +222,29 @@ def _dev_ptr(x, n):
         return x, n
     nbytes = x.numel() * x.element_size()
     return x.data_ptr(), (n if n is not None else nbytes // 32)
+
+
+def check_loopback(d_records, offs, warp_size=32, lockstep=0, granularity=4, index_base=0, stream=None):
+    """Distributed check with len(offs)-1 virtual ranks on this GPU; returns the merged race array."""
+    lib = load()
+    cfg = sesa_config(warp_size, lockstep, granularity, 0)
+    o = (ctypes.c_uint64 * len(offs))(*offs)
+    h = ctypes.c_void_p()
+    ptr, _ = _dev_ptr(d_records, offs[-1])
+    st = lib.sesa_race_check_loopback(ctypes.byref(cfg), ctypes.c_void_p(ptr), o, len(offs) - 1, index_base,
+                                      _stream_ptr(stream), ctypes.byref(h))
+    try:
+        if st != SESA_OK:
+            raise SesaError(st, lib.sesa_last_error(h).decode() if h.value else "sesa_race_check_loopback")
+        n = ctypes.c_uint64()
+        lib.sesa_races_get(h, None, 0, ctypes.byref(n))
+        out = np.zeros(n.value, RACE_DTYPE)
+        if n.value:
+            lib.sesa_races_get(h, ctypes.c_void_p(out.ctypes.data), n.value, ctypes.byref(n))
+        return out
+    finally:
+        if h.value:
+            lib.sesa_trace_destroy(h)
 
 
 def nccl_unique_id() -> bytes:
