@@ -18,6 +18,9 @@ namespace sesa {
 constexpr int CP_STAGES = 4, CP_CHUNK_BYTES = 16384, CP_CHUNK = CP_CHUNK_BYTES / 8, CP_THREADS = 256;
 constexpr int CP_ROWS = CP_CHUNK / CP_THREADS;  // 8 rows per warp
 
+// Per key one comparison with its predecessor (sp); "same as successor" is the next lane's sp (row ballot shifted
+// by one, lane 31 takes bit 0 of the next row).  Keys outside [0, m) and the array edges use sentinel neighbours
+// whose top bit differs, so no 64-bit bounds tests are needed in the inner loop.
 template <bool WRITE>
 __global__ void __launch_bounds__(CP_THREADS) compact_kernel(const u64* __restrict__ keys, u32 m, KeyLayout L,
                                                              u32* __restrict__ chunk_cnt,
@@ -26,6 +29,10 @@ __global__ void __launch_bounds__(CP_THREADS) compact_kernel(const u64* __restri
   __shared__ u64 bars[CP_STAGES];
   __shared__ u32 s_w[CP_THREADS / 32];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  // run key shift: constant unless both spaces are present (then it depends on the key's space bit)
+  const u32 sh_shared = L.pos_bits, sh_global = L.pos_bits + L.lowG;
+  const u32 sh_fixed = L.both ? 0u : (L.single_space == SP_GLOBAL ? sh_global : sh_shared);
+  const u32 sbit = L.space_shift + L.pos_bits;
   BulkRing<CP_STAGES> ring(smem, bars, CP_CHUNK_BYTES);
   ring.start(keys, (u64)m * 8);
   for (u64 j = 0; ring.next(j); j++) {
@@ -37,30 +44,37 @@ __global__ void __launch_bounds__(CP_THREADS) compact_kernel(const u64* __restri
 #pragma unroll
     for (int r = 0; r < CP_ROWS; r++) {
       const u32 t = w0 + r * 32 + lane;
-      k[r] = t < nk ? K[t] : 0ull;
+      // past the end: a sentinel that differs from every real key in the top bit (and from each other's groups:
+      // those lanes are masked out of the ballots below anyway)
+      k[r] = t < nk ? K[t] : ~0ull;
     }
-    // neighbours of the warp's first / last key: inside the chunk from shared memory, else from global
-    const u64 before = w0 > 0 ? K[w0 - 1] : (base > 0 ? keys[base - 1] : 0ull);
+    const u64 first_key = __shfl_sync(~0u, k[0], 0);
+    u64 before = w0 > 0 ? K[w0 - 1] : (base > 0 ? keys[base - 1] : first_key ^ (1ull << 63));
     const u32 wend = w0 + 32 * CP_ROWS;
-    const u64 after = wend < nk ? K[wend] : (base + wend < m ? keys[base + wend] : 0ull);
-    u32 cnt = 0, slot = 0;
-    if (WRITE) {  // this warp's output offset: chunk offset + counts of the chunk's earlier warps
-      slot = chunk_off[c];
-    }
-    unsigned ball[CP_ROWS];
+    const u64 last_key = __shfl_sync(~0u, k[CP_ROWS - 1], 31);
+    const u64 after = wend < nk ? K[wend] : (base + wend < m ? keys[base + wend] : last_key ^ (1ull << 63));
+    unsigned bsp[CP_ROWS], vm[CP_ROWS];  // ballot of "same group as predecessor" (valid lanes only)
 #pragma unroll
     for (int r = 0; r < CP_ROWS; r++) {
-      const u64 i = base + w0 + r * 32 + lane;
-      const u64 up = __shfl_up_sync(~0u, k[r], 1), dn = __shfl_down_sync(~0u, k[r], 1);
-      const u64 pl = __shfl_sync(~0u, r > 0 ? k[r > 0 ? r - 1 : 0] : before, 31);
-      const u64 nf = __shfl_sync(~0u, r + 1 < CP_ROWS ? k[r + 1 < CP_ROWS ? r + 1 : r] : after, 0);
-      const u64 prev = lane > 0 ? up : (r > 0 ? pl : before);
-      const u64 next = lane < 31 ? dn : (r + 1 < CP_ROWS ? nf : after);
-      const bool valid = i < m;
-      const bool sp = valid && i > 0 && same_group(L, k[r], prev);
-      const bool sn = valid && i + 1 < m && same_group(L, k[r], next);
-      ball[r] = __ballot_sync(~0u, sp || sn);
-      cnt += __popc(ball[r]);
+      const u32 valid_rows = nk > w0 + r * 32 ? nk - (w0 + r * 32) : 0u;
+      vm[r] = valid_rows >= 32 ? ~0u : ((1u << valid_rows) - 1u);
+      const u64 up = __shfl_up_sync(~0u, k[r], 1);
+      const u64 prev = lane > 0 ? up : before;
+      const u32 sh = L.both ? ((k[r] >> sbit) & 1ull ? sh_global : sh_shared) : sh_fixed;
+      bsp[r] = __ballot_sync(~0u, ((k[r] ^ prev) >> sh) == 0) & vm[r];
+      before = __shfl_sync(~0u, k[r], 31);
+    }
+    // same as successor: bit (lane+1) of this row's sp ballot; lane 31 uses bit 0 of the next row (or `after`)
+    const u32 sh_last = L.both ? ((last_key >> sbit) & 1ull ? sh_global : sh_shared) : sh_fixed;
+    const bool last_sn = ((last_key ^ after) >> sh_last) == 0;
+    u32 cnt = 0;
+    unsigned keep[CP_ROWS];
+#pragma unroll
+    for (int r = 0; r < CP_ROWS; r++) {
+      const unsigned nxt = r + 1 < CP_ROWS ? (bsp[r + 1 < CP_ROWS ? r + 1 : r] & 1u) : (last_sn ? 1u : 0u);
+      const unsigned bsn = (bsp[r] >> 1) | (nxt << 31);
+      keep[r] = (bsp[r] | bsn) & vm[r];
+      cnt += __popc(keep[r]);
     }
     if (lane == 0) s_w[warp] = cnt;
     __syncthreads();
@@ -71,11 +85,12 @@ __global__ void __launch_bounds__(CP_THREADS) compact_kernel(const u64* __restri
         chunk_cnt[c] = t;
       }
     } else {
+      u32 slot = chunk_off[c];
       for (int w = 0; w < warp; w++) slot += s_w[w];
 #pragma unroll
       for (int r = 0; r < CP_ROWS; r++) {
-        if (ball[r] & (1u << lane)) out[slot + __popc(ball[r] & lanemask_lt())] = k[r];
-        slot += __popc(ball[r]);
+        if (keep[r] & (1u << lane)) out[slot + __popc(keep[r] & lanemask_lt())] = k[r];
+        slot += __popc(keep[r]);
       }
     }
     ring.release(j);  // (contains __syncthreads: s_w may be rewritten next chunk)

@@ -98,68 +98,49 @@ __device__ __forceinline__ u32 block_excl_sum(u32 v, u32* scratch /* [THREADS/32
   return scratch[warp] + x - v;
 }
 
-template <int THREADS, int ITEMS, bool VALS, int MATCH, int MINB>
-__global__ void __launch_bounds__(THREADS, MINB) onesweep_kernel(const u64* __restrict__ kin, u64* __restrict__ kout,
-                                                           const u32* __restrict__ vin, u32* __restrict__ vout,
-                                                           u32 m, u32 shift, const u64* __restrict__ bin_base,
-                                                           u64* __restrict__ lookback, u32* __restrict__ tile_ctr,
-                                                           u32 epoch, int g_tile_atomic) {
+// One tile (body templated on FULL: full tiles skip every validity test).  Per item the digit (9 bits; invalid
+// items of a partial tile use digit RADIX) and later its rank are packed into one register: rd = rank << 9 | d.
+template <int THREADS, int ITEMS, bool VALS, int MATCH, int LBW, bool FULL>
+__device__ __forceinline__ void onesweep_tile(const u64* __restrict__ kin, u64* __restrict__ kout,
+                                              const u32* __restrict__ vin, u32* __restrict__ vout, u32 m, u32 shift,
+                                              const u64* __restrict__ bin_base, u64* __restrict__ lookback,
+                                              u32 epoch, u32 tile, unsigned char* smem,
+                                              unsigned long long* prof) {
   constexpr int WARPS = THREADS / 32;
   constexpr int TILE = THREADS * ITEMS;
-  static_assert(RADIX <= THREADS, "one bin per thread");
-  extern __shared__ __align__(16) unsigned char smem[];
   u64* keys_s = reinterpret_cast<u64*>(smem);                                  // [TILE]
   u32* vals_s = reinterpret_cast<u32*>(keys_s + TILE);                          // [TILE] if VALS
   u32* whist = VALS ? vals_s + TILE : reinterpret_cast<u32*>(keys_s + TILE);    // [WARPS][RADIX]
   u32* bin_start = whist + WARPS * RADIX;                                       // [RADIX]
   long long* glob = reinterpret_cast<long long*>(bin_start + RADIX);            // [RADIX]
   u32* scratch = reinterpret_cast<u32*>(glob + RADIX);                          // [WARPS + 1]
-  u32* wmask = scratch + WARPS + 1;                                             // [WARPS][RADIX + 1] (MATCH 1)
-
+  u32* wmask = scratch + WARPS + 1;                                             // [WARPS][RADIX + 1]
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const u32 ntiles = (u32)((m + TILE - 1) / TILE);
-  // one tile per CTA; tile ids from an atomic counter = execution order (blockIdx order measured 45% slower:
-  // a tile whose predecessor was dispatched later spins in the look-back)
-  __shared__ u32 s_tile;
-  if (tid == 0) s_tile = g_tile_atomic ? atomicAdd(tile_ctr, 1u) : blockIdx.x;
-  __syncthreads();
-  for (u32 tile = s_tile; tile < ntiles; tile = ntiles) {
-  unsigned long long* prof = g_prof ? g_prof + (u64)tile * 8 : nullptr;
-  if (prof && tid == 0) prof[0] = gtime();
-  for (int i = tid; i < WARPS * RADIX; i += THREADS) whist[i] = 0;
-  if (MATCH == 1)
-    for (int i = tid; i < WARPS * (RADIX + 1); i += THREADS) wmask[i] = 0;
-  __syncthreads();
   const u64 tbase = (u64)tile * TILE;
-
+  const u64 wbase = tbase + (u64)warp * 32 * ITEMS + lane;
+  // number of valid items of this thread (items i < nv are inside the array)
+  const int nv = FULL ? ITEMS : (int)(wbase < m ? min((u64)ITEMS, ((u64)m - wbase + 31) / 32) : 0ull);
   u64 k[ITEMS];
   u32 v[ITEMS];
-  u32 rk[ITEMS];
-  const u64 wbase = tbase + (u64)warp * 32 * ITEMS + lane;
+  u32 rd[ITEMS];
 #pragma unroll
   for (int i = 0; i < ITEMS; i++) {
-    u64 idx = wbase + (u64)i * 32;
-    if (idx < m) {
-      k[i] = __ldcs(kin + idx);  // streaming: each key is read once per pass
-      if (VALS) v[i] = __ldcs(vin + idx);
-    } else {
-      k[i] = ~0ull;
+    if (FULL || i < nv) {
+      k[i] = __ldcs(kin + wbase + (u64)i * 32);  // streaming: each key is read once per pass
+      if (VALS) v[i] = __ldcs(vin + wbase + (u64)i * 32);
     }
   }
-  u32* wh = whist + warp * RADIX;
-  const bool full = tbase + TILE <= m;
-  if (prof) {  // all keys of this thread have arrived
-    u64 sum = 0;
 #pragma unroll
-    for (int i = 0; i < ITEMS; i++) sum += k[i];
-    if (sum == 12345) prof[7] = 0;  // keep the loads ordered before the stamp
+  for (int i = 0; i < ITEMS; i++) rd[i] = (FULL || i < nv) ? (u32)((k[i] >> shift) & (RADIX - 1)) : (u32)RADIX;
+  u32* wh = whist + warp * RADIX;
+  if (prof) {
     __syncthreads();
     if (tid == 0) prof[1] = gtime();
   }
   // (1) early counts: per-warp digit histogram with shared-memory atomics (no ordering needed for counts)
 #pragma unroll
   for (int i = 0; i < ITEMS; i++)
-    if (full || wbase + (u64)i * 32 < m) atomicAdd(&wh[(u32)((k[i] >> shift) & (RADIX - 1))], 1u);
+    if (FULL || i < nv) atomicAdd(&wh[rd[i]], 1u);
   __syncthreads();
   // (2) per-digit tile totals -> publish the tile aggregate BEFORE ranking, so that successor tiles find it
   //     during their look-back; per-warp counts become exclusive offsets across warps
@@ -167,7 +148,7 @@ __global__ void __launch_bounds__(THREADS, MINB) onesweep_kernel(const u64* __re
   if (tid < RADIX) {
 #pragma unroll
     for (int w = 0; w < WARPS; w++) {
-      u32 c = whist[w * RADIX + tid];
+      const u32 c = whist[w * RADIX + tid];
       whist[w * RADIX + tid] = tot;
       tot += c;
     }
@@ -177,34 +158,34 @@ __global__ void __launch_bounds__(THREADS, MINB) onesweep_kernel(const u64* __re
   if (tid < RADIX) bin_start[tid] = bs;
   if (prof && tid == 0) prof[2] = gtime();
   // (3) look-back for the exclusive prefix of every digit over earlier tiles, right after publishing the
-  //     aggregate so that inclusive prefixes propagate with minimal delay; each bin-owner thread inspects 4
-  //     predecessors per round trip and backs off while they are unpublished
+  //     aggregate so that inclusive prefixes propagate with minimal delay; each bin-owner thread inspects LBW
+  //     predecessors per L2 round trip and backs off while they are unpublished
   if (tid < RADIX) {
     u64 excl = 0;
     if (tile > 0) {
       long long p = (long long)tile - 1;
       int spins = 0;
       while (true) {
-        u64 w[4];
+        u64 w[LBW];
 #pragma unroll
-        for (int q = 0; q < 4; q++) w[q] = p - q >= 0 ? ld_relaxed(lookback + (u64)(p - q) * RADIX + tid) : 0ull;
-        // consume predecessors in order while they are published; stop at the first inclusive prefix
+        for (int q = 0; q < LBW; q++) w[q] = p - q >= 0 ? ld_relaxed(lookback + (u64)(p - q) * RADIX + tid) : 0ull;
         int q = 0;
         bool done = false;
-        for (; q < 4 && p - q >= 0; q++) {
-          const u32 e = (u32)((w[q] >> 54) & 0xFF);
-          const u64 st = w[q] & (3ull << 62);
-          if (e != epoch || st == 0) break;
-          excl += w[q] & LB_VAL;
-          if (st == LB_PREFIX) {
-            done = true;
-            break;
-          }
+#pragma unroll
+        for (int qq = 0; qq < LBW; qq++) {
+          if (done || q != qq || p - qq < 0) continue;
+          const u32 e = (u32)((w[qq] >> 54) & 0xFF);
+          const u64 st = w[qq] & (3ull << 62);
+          if (e != epoch || st == 0) continue;
+          excl += w[qq] & LB_VAL;
+          q = qq + 1;
+          if (st == LB_PREFIX) done = true;
         }
         if (done) break;
         if (q == 0) __nanosleep(++spins < 4 ? 32 : 128);
         p -= q;
       }
+      if (prof && tid == 0) prof[7] = ((u64)(tile - p) << 32) | (u64)spins;  // walk distance, spins (digit 0)
       st_relaxed(lookback + (u64)tile * RADIX + tid, lb_pack(LB_PREFIX, epoch, excl + tot));
     }
     glob[tid] = (long long)(bin_base[tid] + excl) - (long long)bs;
@@ -214,42 +195,41 @@ __global__ void __launch_bounds__(THREADS, MINB) onesweep_kernel(const u64* __re
     if (tid == 0) prof[3] = gtime();
   }
   // (4) stable warp-level ranking: running per-warp digit counter (starts at the warp's offset) + lower peers
+  u32* wm = wmask + warp * (RADIX + 1);
 #pragma unroll
   for (int i = 0; i < ITEMS; i++) {
-    const bool valid = full || wbase + (u64)i * 32 < m;
-    const u32 d = valid ? (u32)((k[i] >> shift) & (RADIX - 1)) : (u32)RADIX;
+    const u32 d = rd[i];
     unsigned peers;
     if (MATCH == 0) {
-      peers = full ? peers_of<RADIX_BITS>(d) : peers_of<RADIX_BITS + 1>(d);
+      peers = FULL ? peers_of<RADIX_BITS>(d) : peers_of<RADIX_BITS + 1>(d);
     } else {
       // each lane sets its bit in its digit's word of a per-warp mask array: the word becomes the peer set
-      u32* wm = wmask + warp * (RADIX + 1);
       atomicOr(&wm[d], 1u << lane);
       __syncwarp();
       peers = wm[d];
       __syncwarp();
-      if (lane == 31 - __clz(peers)) wm[d] = 0;
     }
-    u32 c = valid ? wh[d] : 0u;
-    rk[i] = c + __popc(peers & lanemask_lt());
+    const bool leader = lane == 31 - __clz(peers);
+    if (MATCH == 1 && leader) wm[d] = 0;
+    const u32 c = wh[d];
+    rd[i] |= (c + __popc(peers & lanemask_lt())) << 9;
     __syncwarp();
-    if (valid && lane == 31 - __clz(peers)) wh[d] = c + __popc(peers);
+    if ((FULL || d < RADIX) && leader) wh[d] = c + __popc(peers);
     __syncwarp();
   }
   __syncthreads();
   if (prof && tid == 0) prof[4] = gtime();
-  // scatter into shared memory in (digit, stable) order
+  // (5) scatter into shared memory in (digit, stable) order, then coalesced stores of each digit's run
 #pragma unroll
   for (int i = 0; i < ITEMS; i++) {
-    if (wbase + (u64)i * 32 < m) {
-      const u32 d = (u32)((k[i] >> shift) & (RADIX - 1));
-      const u32 pos = bin_start[d] + rk[i];
+    if (FULL || i < nv) {
+      const u32 pos = bin_start[rd[i] & 511] + (rd[i] >> 9);
       keys_s[pos] = k[i];
       if (VALS) vals_s[pos] = v[i];
     }
   }
   __syncthreads();
-  const u32 tcount = (u32)min((u64)TILE, (u64)m - tbase);
+  const u32 tcount = FULL ? (u32)TILE : (u32)min((u64)TILE, (u64)m - tbase);
 #pragma unroll 4
   for (u32 j = tid; j < tcount; j += THREADS) {
     const u64 key = keys_s[j];
@@ -262,7 +242,38 @@ __global__ void __launch_bounds__(THREADS, MINB) onesweep_kernel(const u64* __re
     __syncthreads();
     if (tid == 0) prof[5] = gtime(), prof[6] = (u64)blockIdx.x;
   }
-  }
+}
+
+template <int THREADS, int ITEMS, bool VALS, int MATCH, int MINB, int LBW>
+__global__ void __launch_bounds__(THREADS, MINB) onesweep_kernel(const u64* __restrict__ kin, u64* __restrict__ kout,
+                                                                 const u32* __restrict__ vin, u32* __restrict__ vout,
+                                                                 u32 m, u32 shift, const u64* __restrict__ bin_base,
+                                                                 u64* __restrict__ lookback, u32* __restrict__ tile_ctr,
+                                                                 u32 epoch, int g_tile_atomic) {
+  constexpr int WARPS = THREADS / 32;
+  constexpr int TILE = THREADS * ITEMS;
+  static_assert(RADIX <= THREADS, "one bin per thread");
+  extern __shared__ __align__(16) unsigned char smem[];
+  u32* whist = VALS ? reinterpret_cast<u32*>(smem) + 3 * TILE : reinterpret_cast<u32*>(smem) + 2 * TILE;
+  u32* wmask = whist + WARPS * RADIX + RADIX + 2 * RADIX + WARPS + 1;
+  __shared__ u32 s_tile;
+  const int tid = threadIdx.x;
+  // one tile per CTA; tile ids from an atomic counter = execution order (blockIdx order measured 45% slower:
+  // a tile whose predecessor was dispatched later spins in the look-back)
+  if (tid == 0) s_tile = g_tile_atomic ? atomicAdd(tile_ctr, 1u) : blockIdx.x;
+  for (int i = tid; i < WARPS * RADIX; i += THREADS) whist[i] = 0;
+  if (MATCH == 1)
+    for (int i = tid; i < WARPS * (RADIX + 1); i += THREADS) wmask[i] = 0;
+  __syncthreads();
+  const u32 tile = s_tile;
+  unsigned long long* prof = g_prof ? g_prof + (u64)tile * 8 : nullptr;
+  if (prof && tid == 0) prof[0] = gtime();
+  if ((u64)(tile + 1) * TILE <= m)
+    onesweep_tile<THREADS, ITEMS, VALS, MATCH, LBW, true>(kin, kout, vin, vout, m, shift, bin_base, lookback, epoch,
+                                                          tile, smem, prof);
+  else
+    onesweep_tile<THREADS, ITEMS, VALS, MATCH, LBW, false>(kin, kout, vin, vout, m, shift, bin_base, lookback, epoch,
+                                                           tile, smem, prof);
 }
 
 template <int THREADS, int ITEMS, bool VALS>
@@ -293,6 +304,171 @@ int sort_variant() {  // SESA_SORT_MATCH=0 ballots, 1 atomicOr masks (default)
   return v;
 }
 
+
+
+// ------------------------------------------------------------------------------------------------------------
+// Warp-specialized onesweep (cfg 8/9): 8 worker warps load, count, rank and scatter; one helper warp turns the
+// per-warp counts into tile totals and per-warp offsets, publishes the tile aggregate, walks the look-back for
+// all 256 digits (8 per lane, loads interleaved) and fills the global offsets — concurrently with the workers'
+// ranking (named barriers 1/2), so the look-back wait overlaps the ranking instead of preceding it.
+// ------------------------------------------------------------------------------------------------------------
+template <int ITEMS, int MINB>
+__global__ void __launch_bounds__(288, MINB) onesweep_ws_kernel(const u64* __restrict__ kin, u64* __restrict__ kout,
+                                                                u32 m, u32 shift, const u64* __restrict__ bin_base,
+                                                                u64* __restrict__ lookback, u32* __restrict__ tile_ctr,
+                                                                u32 epoch) {
+  constexpr int WARPS = 8, WT = 256, TILE = WT * ITEMS;
+  extern __shared__ __align__(16) unsigned char smem[];
+  u64* keys_s = reinterpret_cast<u64*>(smem);                          // [TILE]
+  u32* whist = reinterpret_cast<u32*>(keys_s + TILE);                  // [WARPS][RADIX] counts -> warp offsets
+  u32* wcnt = whist + WARPS * RADIX;                                   // [WARPS][RADIX + 1] local running counters
+  u32* wmask = wcnt + WARPS * (RADIX + 1);                             // [WARPS][RADIX + 1]
+  u32* bin_start = wmask + WARPS * (RADIX + 1);                        // [RADIX]
+  long long* glob = reinterpret_cast<long long*>(bin_start + RADIX + (RADIX & 1));  // [RADIX]
+  __shared__ u32 s_tile;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  if (tid == 0) s_tile = atomicAdd(tile_ctr, 1u);
+  for (int i = tid; i < WARPS * RADIX; i += 288) whist[i] = 0;
+  for (int i = tid; i < 2 * WARPS * (RADIX + 1); i += 288) wcnt[i] = 0;  // wcnt and wmask
+  __syncthreads();
+  const u32 tile = s_tile;
+  const u64 tbase = (u64)tile * TILE;
+  const bool full = tbase + TILE <= m;
+  u64 k[ITEMS];
+  u32 rd[ITEMS];
+  int nv = 0;
+  if (warp < WARPS) {
+    const u64 wbase = tbase + (u64)warp * 32 * ITEMS + lane;
+    nv = full ? ITEMS : (int)(wbase < m ? min((u64)ITEMS, ((u64)m - wbase + 31) / 32) : 0ull);
+#pragma unroll
+    for (int i = 0; i < ITEMS; i++)
+      if (i < nv) k[i] = __ldcs(kin + wbase + (u64)i * 32);
+#pragma unroll
+    for (int i = 0; i < ITEMS; i++) rd[i] = i < nv ? (u32)((k[i] >> shift) & (RADIX - 1)) : (u32)RADIX;
+    u32* wh = whist + warp * RADIX;
+#pragma unroll
+    for (int i = 0; i < ITEMS; i++)
+      if (i < nv) atomicAdd(&wh[rd[i]], 1u);
+  }
+  __syncthreads();  // counts complete
+  if (warp == WARPS) {
+    // ---- helper warp: 8 digits per lane (d = lane + 32 q)
+    u32 tot[8];
+#pragma unroll
+    for (int q = 0; q < 8; q++) {
+      const int d = lane + 32 * q;
+      u32 t = 0;
+#pragma unroll
+      for (int w = 0; w < WARPS; w++) {
+        const u32 c = whist[w * RADIX + d];
+        whist[w * RADIX + d] = t;
+        t += c;
+      }
+      tot[q] = t;
+      st_relaxed(lookback + (u64)tile * RADIX + d, lb_pack(tile == 0 ? LB_PREFIX : LB_AGG, epoch, t));
+    }
+    // bin_start: exclusive scan over d = 0..255 (lane-major order d = lane + 32 q: scan over q-rows of 32)
+    u32 carry = 0;
+#pragma unroll
+    for (int q = 0; q < 8; q++) {
+      u32 x = tot[q];
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const u32 y = __shfl_up_sync(~0u, x, o);
+        if (lane >= o) x += y;
+      }
+      bin_start[lane + 32 * q] = carry + x - tot[q];
+      carry += __shfl_sync(~0u, x, 31);
+    }
+    // look-back: 8 digits per lane walked together (independent loads in flight)
+    u64 excl[8];
+    long long p[8];
+    bool done[8];
+#pragma unroll
+    for (int q = 0; q < 8; q++) excl[q] = 0, p[q] = (long long)tile - 1, done[q] = tile == 0;
+    int spins = 0;
+    while (true) {
+      bool all = true;
+      u64 w[8];
+#pragma unroll
+      for (int q = 0; q < 8; q++) w[q] = (!done[q] && p[q] >= 0) ? ld_relaxed(lookback + (u64)p[q] * RADIX + lane + 32 * q) : 0ull;
+      bool progress = false;
+#pragma unroll
+      for (int q = 0; q < 8; q++) {
+        if (done[q]) continue;
+        const u32 e = (u32)((w[q] >> 54) & 0xFF);
+        const u64 st = w[q] & (3ull << 62);
+        if (e != epoch || st == 0) {
+          all = false;
+          continue;
+        }
+        progress = true;
+        excl[q] += w[q] & LB_VAL;
+        if (st == LB_PREFIX) done[q] = true;
+        else p[q]--, all = false;
+      }
+      if (all) break;
+      if (!progress) __nanosleep(++spins < 4 ? 32 : 128);
+    }
+#pragma unroll
+    for (int q = 0; q < 8; q++) {
+      const int d = lane + 32 * q;
+      if (tile > 0) st_relaxed(lookback + (u64)tile * RADIX + d, lb_pack(LB_PREFIX, epoch, excl[q] + tot[q]));
+      glob[d] = (long long)(bin_base[d] + excl[q]) - (long long)bin_start[d];
+    }
+    asm volatile("bar.arrive 1, 288;" ::: "memory");  // offsets ready
+  } else {
+    // ---- worker warps: stable ranking within the warp (local counters), concurrently with the look-back
+    u32* wm = wmask + warp * (RADIX + 1);
+    u32* wc = wcnt + warp * (RADIX + 1);
+#pragma unroll
+    for (int i = 0; i < ITEMS; i++) {
+      const u32 d = rd[i];
+      atomicOr(&wm[d], 1u << lane);
+      __syncwarp();
+      const unsigned peers = wm[d];
+      __syncwarp();
+      const bool leader = lane == 31 - __clz(peers);
+      if (leader) wm[d] = 0;
+      const u32 c = wc[d];
+      rd[i] |= (c + __popc(peers & lanemask_lt())) << 9;
+      __syncwarp();
+      if (leader) wc[d] = c + __popc(peers);
+      __syncwarp();
+    }
+    asm volatile("bar.sync 1, 288;" ::: "memory");  // wait for the helper's offsets
+    const u32* wo = whist + warp * RADIX;
+#pragma unroll
+    for (int i = 0; i < ITEMS; i++) {
+      if (i < nv) {
+        const u32 d = rd[i] & 511;
+        keys_s[bin_start[d] + wo[d] + (rd[i] >> 9)] = k[i];
+      }
+    }
+  }
+  __syncthreads();  // tile scattered into shared memory
+  const u32 tcount = full ? (u32)TILE : (u32)min((u64)TILE, (u64)m - tbase);
+#pragma unroll 4
+  for (u32 j = tid; j < tcount; j += 288) {
+    const u64 key = keys_s[j];
+    const u32 d = (u32)((key >> shift) & (RADIX - 1));
+    __stcs(kout + (u64)(glob[d] + (long long)j), key);
+  }
+}
+
+template <int ITEMS, int MINB>
+static void launch_os_ws(const u64* kin, u64* kout, u32 m, u32 shift, const u64* bin_base, u64* lookback,
+                         u32* tile_ctr, u32 epoch, cudaStream_t st) {
+  constexpr int TILE = 256 * ITEMS;
+  auto kern = onesweep_ws_kernel<ITEMS, MINB>;
+  const size_t sm = (size_t)TILE * 8 + 8 * RADIX * 4 + 2 * 8 * (RADIX + 1) * 4 + RADIX * 4 + 8 + RADIX * 8 + 64;
+  static bool set = false;
+  if (!set) {
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    set = true;
+  }
+  kern<<<(unsigned)((m + TILE - 1) / TILE), 288, sm, st>>>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch);
+}
 
 // ------------------------------------------------------------------------------------------------------------
 // Persistent, TMA-pipelined onesweep pass (keys only).  Each CTA acquires tiles in increasing order from a
@@ -462,10 +638,10 @@ static void launch_os_tma(const u64* kin, u64* kout, u32 m, u32 shift, const u64
   kern<<<std::min<u32>(tiles, (u32)grid), THREADS, sm, st>>>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch);
 }
 
-template <int THREADS, int ITEMS, int MINB, bool VALS, int MATCH>
+template <int THREADS, int ITEMS, int MINB, bool VALS, int MATCH, int LBW = 4>
 static void launch_os(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m, u32 shift, const u64* bin_base,
                       u64* lookback, u32* tile_ctr, u32 epoch, cudaStream_t st) {
-  auto kern = onesweep_kernel<THREADS, ITEMS, VALS, MATCH, MINB>;
+  auto kern = onesweep_kernel<THREADS, ITEMS, VALS, MATCH, MINB, LBW>;
   const size_t sm = onesweep_smem<THREADS, ITEMS, VALS>();
   static bool set = false;
   if (!set) {
@@ -491,6 +667,12 @@ static void launch_os_cfg(const u64* kin, u64* kout, const u32* vin, u32* vout, 
                           const u64* bin_base, u64* lookback, u32* tile_ctr, u32 epoch, cudaStream_t st) {
   switch (sort_cfg()) {
     case 1: launch_os<256, 24, 2, VALS, MATCH>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 5: launch_os<256, 24, 2, VALS, MATCH, 8>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 6: launch_os<256, 24, 2, VALS, MATCH, 16>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 7: launch_os<256, 8, 5, VALS, MATCH, 8>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 10: launch_os<256, 32, 2, VALS, MATCH, 4>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 11: launch_os<256, 32, 2, VALS, MATCH, 8>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 12: launch_os<256, 40, 1, VALS, MATCH, 8>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
     case 2: launch_os<512, 16, 1, VALS, MATCH>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
     default: launch_os<256, 16, 3, VALS, MATCH>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
   }
@@ -501,14 +683,17 @@ static void sort_prof_dump(u32 m, cudaStream_t st, unsigned long long* d, u32 ti
   std::vector<unsigned long long> h((size_t)nt * 8);
   cudaMemcpyAsync(h.data(), d, h.size() * 8, cudaMemcpyDeviceToHost, st);
   cudaStreamSynchronize(st);
-  double ph[5] = {0, 0, 0, 0, 0};
+  double ph[5] = {0, 0, 0, 0, 0}, dist = 0, spins = 0, dmax = 0;
   unsigned long long t0 = ~0ull, t1 = 0;
   for (u32 t = 0; t < nt; t++) {
     const unsigned long long* p = &h[(size_t)t * 8];
     for (int q = 0; q < 5; q++) ph[q] += (double)(p[q + 1] - p[q]);
     t0 = std::min(t0, p[0]);
     t1 = std::max(t1, p[5]);
+    dist += (double)(p[7] >> 32), spins += (double)(p[7] & 0xFFFFFFFFull);
+    dmax = std::max(dmax, (double)(p[7] >> 32));
   }
+  fprintf(stderr, "[sortprof] walk distance mean %.1f max %.0f tiles, spins mean %.2f\n", dist / nt, dmax, spins / nt);
   fprintf(stderr, "[sortprof] tiles %u span %.3f ms; mean ns: load %.0f counts %.0f lookback %.0f rank %.0f write %.0f\n", nt,
           (t1 - t0) / 1e6, ph[0] / nt, ph[1] / nt, ph[2] / nt, ph[3] / nt, ph[4] / nt);
 }
@@ -520,7 +705,7 @@ void launch_onesweep(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m
   static size_t dcap = 0;
   const bool want = getenv("SESA_SORT_PROF") && !vin;
   if (want) {
-    const size_t need = ((size_t)m / 4096 + 2) * 64;
+    const size_t need = ((size_t)m / 2048 + 2) * 64;
     if (need > dcap) {
       if (dprof) cudaFree(dprof);
       cudaMalloc(&dprof, need);
@@ -535,6 +720,10 @@ void launch_onesweep(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m
   if (vin) {  // race lists are small: fixed config
     if (ballot) launch_os<256, 16, 3, true, 0>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
     else launch_os<256, 16, 3, true, 1>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
+  } else if (sort_cfg() == 8) {
+    launch_os_ws<16, 2>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
+  } else if (sort_cfg() == 9) {
+    launch_os_ws<24, 1>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
   } else if (sort_cfg() == 3) {
     launch_os_tma<256, 16, 2>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
   } else if (sort_cfg() == 4) {

@@ -35,7 +35,7 @@ void launch_bin_base(const u32* hist, u64* bin_base, u32 npass, cudaStream_t st)
 void launch_onesweep(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m, u32 shift, const u64* bin_base,
                      u64* lookback, u32* tile_ctr, u32 epoch, cudaStream_t st);
 u32 sort_tile_keys();
-inline u32 sort_tiles(u64 m) { return (u32)((m + SORT_TILE - 1) / SORT_TILE); }  // upper bound (smallest tile)
+inline u32 sort_tiles(u64 m) { return (u32)((m + 2047) / 2048); }  // upper bound (smallest tile: 2048 keys)
 // race-list keys: (race key, index) -> histograms for npass digits starting at bit 0
 void launch_hist_keys(const u64* keys, u32 m, u32 npass, u32* hist, cudaStream_t st);
 void launch_hist_keys_shift(const u64* keys, u32 m, u32 npass, u32 shift, u32* hist, cudaStream_t st);
