@@ -16,15 +16,42 @@ namespace sesa {
 constexpr int EX_STAGES = 4, EX_CHUNK = 16384, EX_RECS = EX_CHUNK / 32;
 
 // Register version (measured faster than a TMA ring here: the per-record reductions are ALU-heavy and the ring's
-// strided shared-memory reads and barriers cost more than they save).
+// strided shared-memory reads and barriers cost more than they save).  Scalar accumulators per space (arrays
+// indexed by the record's space spilled to local memory), warp votes only in convergent code, and a warp-uniform
+// single-space fast path (traces are mostly single-space).
+struct SpaceAcc {
+  u64 cnt, gmin, gmax;
+  u32 bmin, bmax, imin, imax;
+  __device__ __forceinline__ void init() { cnt = 0, gmin = ~0ull, gmax = 0, bmin = ~0u, bmax = 0, imin = ~0u, imax = 0; }
+  __device__ __forceinline__ void add(u64 glo, u64 ghi, u32 b, u32 i) {
+    cnt++;
+    gmin = min(gmin, glo), gmax = max(gmax, ghi);
+    bmin = min(bmin, b), bmax = max(bmax, b);
+    imin = min(imin, i), imax = max(imax, i);
+  }
+  __device__ __forceinline__ void warp_reduce() {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      cnt += __shfl_xor_sync(~0u, cnt, o);
+      gmin = min(gmin, __shfl_xor_sync(~0u, gmin, o));
+      gmax = max(gmax, __shfl_xor_sync(~0u, gmax, o));
+      bmin = min(bmin, __shfl_xor_sync(~0u, bmin, o));
+      bmax = max(bmax, __shfl_xor_sync(~0u, bmax, o));
+      imin = min(imin, __shfl_xor_sync(~0u, imin, o));
+      imax = max(imax, __shfl_xor_sync(~0u, imax, o));
+    }
+  }
+};
+
 template <int THREADS, int U>
 __global__ void __launch_bounds__(THREADS) extents_kernel(const Rec* __restrict__ rec, u64 n, u32 log2G,
                                                           Summary* __restrict__ out) {
-  u64 bad = ~0ull, ent = 0, multi = 0, cnt[2] = {0, 0};
-  u64 gmin[2] = {~0ull, ~0ull}, gmax[2] = {0, 0};
-  u32 bmin[2] = {~0u, ~0u}, bmax[2] = {0, 0}, imin[2] = {~0u, ~0u}, imax[2] = {0, 0};
+  u64 bad = ~0ull, ent = 0, multi = 0;
+  SpaceAcc A0, A1;  // shared, global
+  A0.init();
+  A1.init();
   u32 unsorted = 0;
-  const int lane = threadIdx.x & 31;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const u64 stride = (u64)gridDim.x * THREADS, gt = (u64)blockIdx.x * THREADS + threadIdx.x;
   const u64 rounds = (n + stride * U - 1) / (stride * U);
   for (u64 it = 0; it < rounds; it++) {
@@ -38,94 +65,81 @@ __global__ void __launch_bounds__(THREADS) extents_kernel(const Rec* __restrict_
     for (int j = 0; j < U; j++) {
       const u64 k = (it * U + j) * stride + gt;
       const bool in = k < n;
-      // (block, interval) of record k-1: held by the previous lane, or loaded for lane 0
+      // (block, interval) of record k-1: held by the previous lane, or loaded for lane 0 (convergent shuffles)
       u32 pb = __shfl_up_sync(~0u, in ? r[j].block : 0u, 1), pi = __shfl_up_sync(~0u, in ? r[j].interval : 0u, 1);
-      if (!in) continue;
-      if (lane == 0 && k > 0) {
+      if (lane == 0 && in && k > 0) {
         const uint4 q = __ldg(reinterpret_cast<const uint4*>(rec + k - 1) + 1);
         pb = q.x, pi = q.z;
       }
       const Rec& x = r[j];
-      const bool ok = x.space <= 1 && x.rw <= 2 && x.size >= 1 && x.addr <= ~0ull - (u64)(x.size - 1);
-      if (!ok) {
-        bad = min(bad, k);
-        continue;
-      }
-      if (k > 0 && (x.block < pb || (x.block == pb && x.interval < pi))) unsorted = 1;
+      const bool ok = in && x.space <= 1 && x.rw <= 2 && x.size >= 1 && x.addr <= ~0ull - (u64)(x.size - 1);
+      if (in && !ok) bad = min(bad, k);
       const u64 glo = x.addr >> log2G, ghi = (x.addr + (u64)(x.size - 1)) >> log2G;
-      ent += ghi - glo + 1;
-      multi += ghi != glo;
-#pragma unroll
-      for (int sp = 0; sp < 2; sp++) {  // static indices: no local-memory arrays
-        if (x.space != sp) continue;
-        cnt[sp]++;
-        gmin[sp] = min(gmin[sp], glo);
-        gmax[sp] = max(gmax[sp], ghi);
-        bmin[sp] = min(bmin[sp], x.block);
-        bmax[sp] = max(bmax[sp], x.block);
-        imin[sp] = min(imin[sp], x.interval);
-        imax[sp] = max(imax[sp], x.interval);
+      if (ok) {
+        if (k > 0 && (x.block < pb || (x.block == pb && x.interval < pi))) unsorted = 1;
+        ent += ghi - glo + 1;
+        multi += ghi != glo;
+      }
+      const bool all_glob = __all_sync(~0u, !ok || x.space == SP_GLOBAL);
+      if (all_glob) {
+        if (ok) A1.add(glo, ghi, x.block, x.interval);
+      } else if (__all_sync(~0u, !ok || x.space == SP_SHARED)) {
+        if (ok) A0.add(glo, ghi, x.block, x.interval);
+      } else if (ok) {
+        if (x.space == SP_GLOBAL) A1.add(glo, ghi, x.block, x.interval);
+        else A0.add(glo, ghi, x.block, x.interval);
       }
     }
   }
   // block reduction through warp shuffles then one atomic per field per CTA
-  __shared__ u64 s64[THREADS / 32][9];
-  __shared__ u32 s32[THREADS / 32][9];
-  const int warp = threadIdx.x >> 5;
-  (void)lane;
+  __shared__ SpaceAcc sa[THREADS / 32][2];
+  __shared__ u64 s64[THREADS / 32][3];
+  __shared__ u32 s_uns[THREADS / 32];
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) {
     bad = min(bad, __shfl_xor_sync(~0u, bad, o));
     ent += __shfl_xor_sync(~0u, ent, o);
     multi += __shfl_xor_sync(~0u, multi, o);
-#pragma unroll
-    for (int s = 0; s < 2; s++) {
-      cnt[s] += __shfl_xor_sync(~0u, cnt[s], o);
-      gmin[s] = min(gmin[s], __shfl_xor_sync(~0u, gmin[s], o));
-      gmax[s] = max(gmax[s], __shfl_xor_sync(~0u, gmax[s], o));
-      bmin[s] = min(bmin[s], __shfl_xor_sync(~0u, bmin[s], o));
-      bmax[s] = max(bmax[s], __shfl_xor_sync(~0u, bmax[s], o));
-      imin[s] = min(imin[s], __shfl_xor_sync(~0u, imin[s], o));
-      imax[s] = max(imax[s], __shfl_xor_sync(~0u, imax[s], o));
-    }
     unsorted |= __shfl_xor_sync(~0u, unsorted, o);
   }
+  A0.warp_reduce();
+  A1.warp_reduce();
   if (lane == 0) {
-    s64[warp][0] = bad; s64[warp][1] = ent; s64[warp][2] = multi;
-    s64[warp][3] = cnt[0]; s64[warp][4] = cnt[1];
-    s64[warp][5] = gmin[0]; s64[warp][6] = gmin[1]; s64[warp][7] = gmax[0]; s64[warp][8] = gmax[1];
-    s32[warp][0] = bmin[0]; s32[warp][1] = bmin[1]; s32[warp][2] = bmax[0]; s32[warp][3] = bmax[1];
-    s32[warp][4] = imin[0]; s32[warp][5] = imin[1]; s32[warp][6] = imax[0]; s32[warp][7] = imax[1];
-    s32[warp][8] = unsorted;
+    s64[warp][0] = bad, s64[warp][1] = ent, s64[warp][2] = multi;
+    sa[warp][0] = A0, sa[warp][1] = A1;
+    s_uns[warp] = unsorted;
   }
   __syncthreads();
   if (threadIdx.x == 0) {
     for (int w = 1; w < THREADS / 32; w++) {
       s64[0][0] = min(s64[0][0], s64[w][0]);
-      s64[0][1] += s64[w][1]; s64[0][2] += s64[w][2]; s64[0][3] += s64[w][3]; s64[0][4] += s64[w][4];
-      s64[0][5] = min(s64[0][5], s64[w][5]); s64[0][6] = min(s64[0][6], s64[w][6]);
-      s64[0][7] = max(s64[0][7], s64[w][7]); s64[0][8] = max(s64[0][8], s64[w][8]);
-      for (int q = 0; q < 8; q += 2) {
-        bool isMin = q == 0 || q == 4;
-        s32[0][q] = isMin ? min(s32[0][q], s32[w][q]) : max(s32[0][q], s32[w][q]);
-        s32[0][q + 1] = isMin ? min(s32[0][q + 1], s32[w][q + 1]) : max(s32[0][q + 1], s32[w][q + 1]);
+      s64[0][1] += s64[w][1];
+      s64[0][2] += s64[w][2];
+      s_uns[0] |= s_uns[w];
+      for (int sp = 0; sp < 2; sp++) {
+        SpaceAcc& d = sa[0][sp];
+        const SpaceAcc& e = sa[w][sp];
+        d.cnt += e.cnt;
+        d.gmin = min(d.gmin, e.gmin), d.gmax = max(d.gmax, e.gmax);
+        d.bmin = min(d.bmin, e.bmin), d.bmax = max(d.bmax, e.bmax);
+        d.imin = min(d.imin, e.imin), d.imax = max(d.imax, e.imax);
       }
-      s32[0][8] |= s32[w][8];
     }
     if (s64[0][0] != ~0ull) atomicMin(&out->bad_index, (unsigned long long)s64[0][0]);
     if (s64[0][1]) atomicAdd(&out->entries, (unsigned long long)s64[0][1]);
     if (s64[0][2]) atomicAdd(&out->multi, (unsigned long long)s64[0][2]);
-    for (int s = 0; s < 2; s++) {
-      if (!s64[0][3 + s]) continue;
-      atomicAdd(&out->count[s], (unsigned long long)s64[0][3 + s]);
-      atomicMin(&out->gmin[s], (unsigned long long)s64[0][5 + s]);
-      atomicMax(&out->gmax[s], (unsigned long long)s64[0][7 + s]);
-      atomicMin(&out->bmin[s], s32[0][0 + s]);
-      atomicMax(&out->bmax[s], s32[0][2 + s]);
-      atomicMin(&out->imin[s], s32[0][4 + s]);
-      atomicMax(&out->imax[s], s32[0][6 + s]);
+    for (int sp = 0; sp < 2; sp++) {
+      const SpaceAcc& d = sa[0][sp];
+      if (!d.cnt) continue;
+      atomicAdd(&out->count[sp], (unsigned long long)d.cnt);
+      atomicMin(&out->gmin[sp], (unsigned long long)d.gmin);
+      atomicMax(&out->gmax[sp], (unsigned long long)d.gmax);
+      atomicMin(&out->bmin[sp], d.bmin);
+      atomicMax(&out->bmax[sp], d.bmax);
+      atomicMin(&out->imin[sp], d.imin);
+      atomicMax(&out->imax[sp], d.imax);
     }
-    if (s32[0][8]) atomicOr(&out->unsorted, 1u);
+    if (s_uns[0]) atomicOr(&out->unsorted, 1u);
   }
 }
 
