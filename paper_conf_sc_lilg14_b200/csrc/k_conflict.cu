@@ -88,8 +88,75 @@ __device__ __forceinline__ bool ex_wval(const Agg& S, u32 id, u64 v) {
   return lo != v || hi != v;
 }
 
+// tri-state "exists a plain write with identity != id and value != v": 0 no, 1 yes, 2 unknown (never for Agg)
+__device__ __forceinline__ int wval3(const Agg& S, u32 id, u64 v) { return ex_wval(S, id, v) ? 1 : 0; }
+
 struct OpAgg {
   __device__ __forceinline__ Agg operator()(const Agg& a, const Agg& b) const { return agg_merge(a, b); }
+};
+
+// ---- cheap summary (AggC): same identity fields, only min/max of the write values
+__device__ __forceinline__ bool ex_id(const AggC& S, int X, u32 id) { return S.mn[X] < id || S.mx[X] > id; }
+__device__ __forceinline__ bool ex_warp(const AggC& S, int X, u32 w, u32 ws) {
+  return S.mn[X] <= S.mx[X] && (S.mn[X] / ws < w || S.mx[X] / ws > w);
+}
+__device__ __forceinline__ int wval3(const AggC& S, u32 id, u64 v) {
+  if (!ex_id(S, RW_WRITE, id)) return 0;  // no writer with another identity
+  if (S.vlo == S.vhi) return 0;           // every write of the set has one value, which is mine (I am a writer)
+  return 2;                               // >= 2 identities and >= 2 values: needs the exact summary
+}
+struct OpAggC {
+  __device__ __forceinline__ AggC operator()(const AggC& a, const AggC& b) const {
+    AggC r;
+#pragma unroll
+    for (int x = 0; x < 3; x++) r.mn[x] = min(a.mn[x], b.mn[x]), r.mx[x] = max(a.mx[x], b.mx[x]);
+    r.vlo = min(a.vlo, b.vlo);
+    r.vhi = max(a.vhi, b.vhi);
+    return r;
+  }
+};
+template <class A>
+__device__ __forceinline__ A agg_empty_t();
+template <>
+__device__ __forceinline__ Agg agg_empty_t<Agg>() { return agg_empty(); }
+template <>
+__device__ __forceinline__ AggC agg_empty_t<AggC>() {
+  AggC r;
+#pragma unroll
+  for (int x = 0; x < 3; x++) r.mn[x] = ~0u, r.mx[x] = 0u;
+  r.vlo = ~0ull, r.vhi = 0ull;
+  return r;
+}
+template <class A>
+__device__ __forceinline__ A agg_item_t(u32 rw, u32 id, u64 vh);
+template <>
+__device__ __forceinline__ Agg agg_item_t<Agg>(u32 rw, u32 id, u64 vh) { return agg_item(rw, id, vh); }
+template <>
+__device__ __forceinline__ AggC agg_item_t<AggC>(u32 rw, u32 id, u64 vh) {
+  AggC r = agg_empty_t<AggC>();
+  r.mn[rw] = r.mx[rw] = id;
+  if (rw == RW_WRITE) r.vlo = r.vhi = vh;
+  return r;
+}
+template <class A>
+struct OpOf;
+template <>
+struct OpOf<Agg> {
+  typedef OpAgg type;
+};
+template <>
+struct OpOf<AggC> {
+  typedef OpAggC type;
+};
+template <class A>
+struct QuadOf;
+template <>
+struct QuadOf<Agg> {
+  typedef AggQuad type;
+};
+template <>
+struct QuadOf<AggC> {
+  typedef AggQuadC type;
 };
 
 struct X2 {
@@ -131,6 +198,13 @@ __device__ __forceinline__ Agg shfl(const Agg& a, int o, bool down) {
   r.i1 = shfl(a.i1, o, down), r.i2 = shfl(a.i2, o, down);
   r.v1 = shfl(a.v1, o, down), r.v1b = shfl(a.v1b, o, down);
   r.v2 = shfl(a.v2, o, down), r.v2b = shfl(a.v2b, o, down);
+  return r;
+}
+__device__ __forceinline__ AggC shfl(const AggC& a, int o, bool down) {
+  AggC r;
+#pragma unroll
+  for (int x = 0; x < 3; x++) r.mn[x] = shfl(a.mn[x], o, down), r.mx[x] = shfl(a.mx[x], o, down);
+  r.vlo = shfl(a.vlo, o, down), r.vhi = shfl(a.vhi, o, down);
   return r;
 }
 __device__ __forceinline__ X2 shfl(const X2& a, int o, bool down) {
@@ -253,9 +327,10 @@ struct TileSmem {
   u8 gq[CT_TILE];
   u8 res[CT_TILE];
   Agg wv[CT_THREADS / 32];
+  AggC wvc[CT_THREADS / 32];
   X2 wx[CT_THREADS / 32];
   u8 wf[CT_THREADS / 32];
-  int any, first_gtail, last_ghead;
+  int any, first_gtail, last_ghead, unknown;
 };
 
 __device__ __forceinline__ u32 pos_of(const KeyLayout& L, u64 key) { return (u32)(key & lowmask(L.pos_bits)); }
@@ -345,33 +420,46 @@ __device__ bool tile_load(const ConflictArgs& a, TileSmem& s, u64 tb, u32 cnt) {
 }
 
 // group- and sub-run-level summaries -> s.res[j] = bit0 RW partner, bit1 WW partner.  In mode 1 also returns
-// the tile-edge partial summaries (P = item 0's segment, S = item cnt-1's segment) per level.
-__device__ void tile_flags(const ConflictArgs& a, TileSmem& s, u32 cnt, const Agg cin[2], const Agg cout[2],
-                           Agg* part /* [4] or null */) {
+// the tile-edge partial summaries (P = item 0's segment, S = item cnt-1's segment) per level.  With the cheap
+// summary (A = AggC) a benign query that cannot be decided sets s.unknown (the check is then redone exactly).
+template <class A>
+__device__ A* scan_scratch(TileSmem& s);
+template <>
+__device__ __forceinline__ Agg* scan_scratch<Agg>(TileSmem& s) { return s.wv; }
+template <>
+__device__ __forceinline__ AggC* scan_scratch<AggC>(TileSmem& s) { return s.wvc; }
+
+template <class A>
+__device__ void tile_flags(const ConflictArgs& a, TileSmem& s, u32 cnt, const A cin[2], const A cout[2],
+                           A* part /* [4] or null */) {
+  typedef typename OpOf<A>::type Op;
   const u32 ws = a.ws, ls = a.ls;
-  const Agg E = agg_empty();
-  // group level (identity = block): "another block" queries -> s.gq
-  tile_allreduce<Agg>(
+  const A E = agg_empty_t<A>();
+  // group level (identity = block): "another block" queries -> s.gq (bit3: benign query yes, bit4: unknown)
+  tile_allreduce<A>(
       s.fl, FL_GH, FL_GT,
-      [&](int j) { return (s.fl[j] & FL_INT) ? agg_item(s.rw[j], s.blk[j + 1], s.vh[j]) : E; }, OpAgg(), E, cin[0],
+      [&](int j) { return (s.fl[j] & FL_INT) ? agg_item_t<A>(s.rw[j], s.blk[j + 1], s.vh[j]) : E; }, Op(), E, cin[0],
       cout[0],
-      [&](int j, const Agg& R) {
+      [&](int j, const A& R) {
         if (part && j == 0) part[0] = R;
         if (part && j == (int)cnt - 1) part[1] = R;
         if (!(s.fl[j] & FL_INT)) return;
         const u32 b = s.blk[j + 1];
         u8 g = (ex_id(R, RW_READ, b) ? 1 : 0) | (ex_id(R, RW_WRITE, b) ? 2 : 0) | (ex_id(R, RW_ATOMIC, b) ? 4 : 0);
-        if (s.rw[j] == RW_WRITE && ex_wval(R, b, s.vh[j])) g |= 8;
+        if (s.rw[j] == RW_WRITE) {
+          const int q = wval3(R, b, s.vh[j]);
+          g |= q == 1 ? 8 : q == 2 ? 16 : 0;
+        }
         s.gq[j] = g;
       },
-      s.wv, s.wf);
+      scan_scratch<A>(s), s.wf);
   __syncthreads();
   // sub-run level (identity = thread): same block and interval
-  tile_allreduce<Agg>(
+  tile_allreduce<A>(
       s.fl, FL_SH, FL_ST,
-      [&](int j) { return (s.fl[j] & FL_INT) ? agg_item(s.rw[j], s.thr[j], s.vh[j]) : E; }, OpAgg(), E, cin[1],
+      [&](int j) { return (s.fl[j] & FL_INT) ? agg_item_t<A>(s.rw[j], s.thr[j], s.vh[j]) : E; }, Op(), E, cin[1],
       cout[1],
-      [&](int j, const Agg& S) {
+      [&](int j, const A& S) {
         if (part && j == 0) part[2] = S;
         if (part && j == (int)cnt - 1) part[3] = S;
         if (!(s.fl[j] & FL_INT)) return;
@@ -385,14 +473,17 @@ __device__ void tile_flags(const ConflictArgs& a, TileSmem& s, u32 cnt, const Ag
           fww = false;
         } else {
           frw = (ls ? ex_warp(S, RW_READ, w, ws) : ex_id(S, RW_READ, t)) || (g & 1);
-          if (rw == RW_WRITE)
-            fww = ex_id(S, RW_ATOMIC, t) || (g & 4) || ex_wval(S, t, s.vh[j]) || (g & 8);
-          else
+          if (rw == RW_WRITE) {
+            const int q = wval3(S, t, s.vh[j]);
+            fww = ex_id(S, RW_ATOMIC, t) || (g & 4) || q == 1 || (g & 8);
+            if (!fww && (q == 2 || (g & 16))) s.unknown = 1;  // undecidable with the cheap summary
+          } else {
             fww = ex_id(S, RW_WRITE, t) || (g & 2);
+          }
         }
         s.res[j] = (frw ? 1 : 0) | (fww ? 2 : 0);
       },
-      s.wv, s.wf);
+      scan_scratch<A>(s), s.wf);
   __syncthreads();
 }
 
@@ -423,8 +514,9 @@ __device__ void emit_race(const ConflictArgs& a, u64 head_hi, u32 kind, u32 x, u
 }
 
 // ------------------------------------------------------------------------------------------------ mode 1 / 2
-template <int MODE>
+template <int MODE, class A>
 __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
+  typedef typename QuadOf<A>::type Q;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
   const u32 tile = MODE == 1 ? blockIdx.x : a.cross_list[blockIdx.x];
@@ -438,18 +530,24 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
     return;
   }
   const bool cin = !(s.fl[0] & FL_GH), cout = !(s.fl[cnt - 1] & FL_GT);
-  Agg ci[2], co[2];
-  ci[0] = ci[1] = co[0] = co[1] = agg_empty();
+  A ci[2], co[2];
+  ci[0] = ci[1] = co[0] = co[1] = agg_empty_t<A>();
+  if (tid == 0) s.unknown = 0;
   if (MODE == 2) {
-    const Agg* c = a.carry[tile].a;  // [grp In, grp Out, sub In, sub Out]
+    const A* c = reinterpret_cast<const Q*>(a.carry)[tile].a;  // [grp In, grp Out, sub In, sub Out]
     if (cin) ci[0] = c[0];
     if (cout) co[0] = c[1];
     if (!(s.fl[0] & FL_SH)) ci[1] = c[2];
     if (!(s.fl[cnt - 1] & FL_ST)) co[1] = c[3];
   }
-  __shared__ Agg s_part[4];
-  tile_flags(a, s, cnt, ci, co, MODE == 1 ? s_part : nullptr);
+  __shared__ A s_part[4];
+  tile_flags<A>(a, s, cnt, ci, co, MODE == 1 ? s_part : nullptr);
   const int ftail = s.first_gtail, lhead = s.last_ghead;
+  if (s.unknown) {  // a benign query the cheap summary cannot decide: the host reruns with exact summaries
+    if (tid == 0) atomicOr(a.need_exact, 1u);
+    if (MODE == 1 && tid == 0) a.tile_flags[tile] = TF_GH | TF_GT | TF_SH | TF_ST;
+    return;
+  }
 
   if (MODE == 1) {
     if (tid == 0) {
@@ -464,7 +562,7 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
       if (cout) tf |= TF_COUT;
       a.tile_flags[tile] = tf;
       if (cin || cout) {
-        for (int i = 0; i < 4; i++) a.part[tile].a[i] = s_part[i];
+        for (int i = 0; i < 4; i++) reinterpret_cast<Q*>(a.part)[tile].a[i] = s_part[i];
         a.cross_list[atomicAdd(a.cross_count, 1u)] = tile;
       }
       if (cout && lhead >= 0) {  // this tile owns the group that crosses out
@@ -650,17 +748,23 @@ __global__ void cross_emit_kernel(ConflictArgs a, u32 ncross) {
 
 u32 conflict_tiles(u64 m) { return (u32)((m + CT_TILE - 1) / CT_TILE); }
 
-void launch_conflict(int mode, const ConflictArgs& a, u32 nblocks, cudaStream_t st) {
+template <int MODE, class A>
+static void launch_ck(const ConflictArgs& a, u32 nblocks, cudaStream_t st) {
+  const size_t sm = sizeof(TileSmem);
+  static bool set = false;
+  if (!set) cudaFuncSetAttribute(conflict_kernel<MODE, A>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm), set = true;
+  conflict_kernel<MODE, A><<<nblocks, CT_THREADS, sm, st>>>(a);
+}
+
+void launch_conflict(int mode, bool exact, const ConflictArgs& a, u32 nblocks, cudaStream_t st) {
   if (!nblocks) return;
   const size_t sm = sizeof(TileSmem);
   if (mode == 1) {
-    static bool set = false;
-    if (!set) cudaFuncSetAttribute(conflict_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm), set = true;
-    conflict_kernel<1><<<nblocks, CT_THREADS, sm, st>>>(a);
+    if (exact) launch_ck<1, Agg>(a, nblocks, st);
+    else launch_ck<1, AggC>(a, nblocks, st);
   } else if (mode == 2) {
-    static bool set = false;
-    if (!set) cudaFuncSetAttribute(conflict_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm), set = true;
-    conflict_kernel<2><<<nblocks, CT_THREADS, sm, st>>>(a);
+    if (exact) launch_ck<2, Agg>(a, nblocks, st);
+    else launch_ck<2, AggC>(a, nblocks, st);
   } else {
     static bool set = false;
     if (!set) cudaFuncSetAttribute(conflict_y_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm), set = true;
@@ -680,29 +784,35 @@ void launch_cross_emit(const ConflictArgs& a, u32 ncross, cudaStream_t st) {
 // computed in chunks of 1024 tiles (one CTA each), chunk carries by one CTA, then applied.
 constexpr int CARRY_T = 1024;
 
+template <class A>
 struct CarryEl {
-  Agg a;
+  A a;
   u32 owner;
 };
 
+template <class A>
 struct OpCarry {
-  __device__ __forceinline__ CarryEl operator()(const CarryEl& x, const CarryEl& y) const {
-    CarryEl r;
-    r.a = agg_merge(x.a, y.a);
+  __device__ __forceinline__ CarryEl<A> operator()(const CarryEl<A>& x, const CarryEl<A>& y) const {
+    CarryEl<A> r;
+    r.a = typename OpOf<A>::type()(x.a, y.a);
     r.owner = max(x.owner, y.owner);
     return r;
   }
 };
-__device__ __forceinline__ CarryEl shfl(const CarryEl& c, int o, bool down) {
-  CarryEl r;
+template <class A>
+__device__ __forceinline__ CarryEl<A> shfl(const CarryEl<A>& c, int o, bool down) {
+  CarryEl<A> r;
   r.a = shfl(c.a, o, down);
   r.owner = shfl(c.owner, o, down);
   return r;
 }
 
 // scan direction d: 0 grp fwd, 1 grp bwd, 2 sub fwd, 3 sub bwd
-__device__ __forceinline__ void carry_element(const ConflictArgs& a, u32 j, u32 ntiles, int d, bool& f, CarryEl& e) {
-  e.a = agg_empty();
+template <class A>
+__device__ __forceinline__ void carry_element(const ConflictArgs& a, u32 j, u32 ntiles, int d, bool& f,
+                                              CarryEl<A>& e) {
+  typedef typename QuadOf<A>::type Q;
+  e.a = agg_empty_t<A>();
   e.owner = 0;
   f = true;
   if (j >= ntiles) return;
@@ -711,34 +821,33 @@ __device__ __forceinline__ void carry_element(const ConflictArgs& a, u32 j, u32 
   const u8 bit = d == 0 ? TF_GH : d == 1 ? TF_GT : d == 2 ? TF_SH : TF_ST;
   f = (tf & bit) != 0;
   const int pi = d == 0 ? 1 : d == 1 ? 0 : d == 2 ? 3 : 2;  // fwd uses S (last piece), bwd uses P (first piece)
-  if (crossing) e.a = a.part[j].a[pi];
+  if (crossing) e.a = reinterpret_cast<const Q*>(a.part)[j].a[pi];
   e.owner = (d == 0 && f) ? j : 0;
 }
 
-template <bool REV>
-__device__ CarryEl carry_block_scan(bool f, const CarryEl& v, const CarryEl& seed, bool& incl_f, CarryEl* s_wv,
-                                    u8* s_wf) {
+template <class A, bool REV>
+__device__ CarryEl<A> carry_block_scan(bool f, const CarryEl<A>& v, const CarryEl<A>& seed, CarryEl<A>* s_wv,
+                                       u8* s_wf) {
   // inclusive = exclusive (+) own
-  CarryEl ex = block_seg_excl<CarryEl, OpCarry, REV, CARRY_T>(f, v, seed, OpCarry(), s_wv, s_wf);
-  incl_f = f;
-  return f ? v : OpCarry()(ex, v);
+  CarryEl<A> ex = block_seg_excl<CarryEl<A>, OpCarry<A>, REV, CARRY_T>(f, v, seed, OpCarry<A>(), s_wv, s_wf);
+  return f ? v : OpCarry<A>()(ex, v);
 }
 
-__global__ void __launch_bounds__(CARRY_T) carry_chunk_kernel(ConflictArgs a, u32 ntiles, CarryEl* chunk_tot,
+template <class A>
+__global__ void __launch_bounds__(CARRY_T) carry_chunk_kernel(ConflictArgs a, u32 ntiles, CarryEl<A>* chunk_tot,
                                                               u8* chunk_f) {
-  __shared__ CarryEl s_wv[CARRY_T / 32];
+  __shared__ CarryEl<A> s_wv[CARRY_T / 32];
   __shared__ u8 s_wf[CARRY_T / 32];
   const u32 j = blockIdx.x * CARRY_T + threadIdx.x;
   for (int d = 0; d < 4; d++) {
     bool f;
-    CarryEl e;
-    carry_element(a, j, ntiles, d, f, e);
-    CarryEl seed;
-    seed.a = agg_empty(), seed.owner = 0;
-    bool inf;
+    CarryEl<A> e;
+    carry_element<A>(a, j, ntiles, d, f, e);
+    CarryEl<A> seed;
+    seed.a = agg_empty_t<A>(), seed.owner = 0;
     const bool rev = d & 1;
-    CarryEl inc = rev ? carry_block_scan<true>(f, e, seed, inf, s_wv, s_wf)
-                      : carry_block_scan<false>(f, e, seed, inf, s_wv, s_wf);
+    CarryEl<A> inc = rev ? carry_block_scan<A, true>(f, e, seed, s_wv, s_wf)
+                         : carry_block_scan<A, false>(f, e, seed, s_wv, s_wf);
     const bool flag_any = __syncthreads_or(f);
     // chunk total = inclusive value at the chunk's last (fwd) / first (bwd) thread
     if ((!rev && threadIdx.x == CARRY_T - 1) || (rev && threadIdx.x == 0)) {
@@ -749,44 +858,48 @@ __global__ void __launch_bounds__(CARRY_T) carry_chunk_kernel(ConflictArgs a, u3
   }
 }
 
-__global__ void __launch_bounds__(CARRY_T) carry_top_kernel(u32 nchunks, CarryEl* chunk_tot, u8* chunk_f,
-                                                            CarryEl* chunk_carry) {
-  __shared__ CarryEl s_wv[CARRY_T / 32];
+template <class A>
+__global__ void __launch_bounds__(CARRY_T) carry_top_kernel(u32 nchunks, CarryEl<A>* chunk_tot, u8* chunk_f,
+                                                            CarryEl<A>* chunk_carry) {
+  __shared__ CarryEl<A> s_wv[CARRY_T / 32];
   __shared__ u8 s_wf[CARRY_T / 32];
   const u32 c = threadIdx.x;
   for (int d = 0; d < 4; d++) {
-    CarryEl e;
+    CarryEl<A> e;
     bool f = true;
-    e.a = agg_empty(), e.owner = 0;
+    e.a = agg_empty_t<A>(), e.owner = 0;
     if (c < nchunks) e = chunk_tot[c * 4 + d], f = chunk_f[c * 4 + d];
-    CarryEl seed;
-    seed.a = agg_empty(), seed.owner = 0;
-    CarryEl ex = (d & 1) ? block_seg_excl<CarryEl, OpCarry, true, CARRY_T>(f, e, seed, OpCarry(), s_wv, s_wf)
-                         : block_seg_excl<CarryEl, OpCarry, false, CARRY_T>(f, e, seed, OpCarry(), s_wv, s_wf);
+    CarryEl<A> seed;
+    seed.a = agg_empty_t<A>(), seed.owner = 0;
+    CarryEl<A> ex =
+        (d & 1) ? block_seg_excl<CarryEl<A>, OpCarry<A>, true, CARRY_T>(f, e, seed, OpCarry<A>(), s_wv, s_wf)
+                : block_seg_excl<CarryEl<A>, OpCarry<A>, false, CARRY_T>(f, e, seed, OpCarry<A>(), s_wv, s_wf);
     if (c < nchunks) chunk_carry[c * 4 + d] = ex;
   }
 }
 
-__global__ void __launch_bounds__(CARRY_T) carry_apply_kernel(ConflictArgs a, u32 ntiles, const CarryEl* chunk_carry) {
-  __shared__ CarryEl s_wv[CARRY_T / 32];
+template <class A>
+__global__ void __launch_bounds__(CARRY_T) carry_apply_kernel(ConflictArgs a, u32 ntiles,
+                                                              const CarryEl<A>* chunk_carry) {
+  typedef typename QuadOf<A>::type Q;
+  __shared__ CarryEl<A> s_wv[CARRY_T / 32];
   __shared__ u8 s_wf[CARRY_T / 32];
   const u32 j = blockIdx.x * CARRY_T + threadIdx.x;
   for (int d = 0; d < 4; d++) {
     bool f;
-    CarryEl e;
-    carry_element(a, j, ntiles, d, f, e);
+    CarryEl<A> e;
+    carry_element<A>(a, j, ntiles, d, f, e);
     const bool rev = d & 1;
-    bool inf;
-    const CarryEl seed = chunk_carry[blockIdx.x * 4 + d];
-    CarryEl inc = rev ? carry_block_scan<true>(f, e, seed, inf, s_wv, s_wf)
-                      : carry_block_scan<false>(f, e, seed, inf, s_wv, s_wf);
+    const CarryEl<A> seed = chunk_carry[blockIdx.x * 4 + d];
+    CarryEl<A> inc = rev ? carry_block_scan<A, true>(f, e, seed, s_wv, s_wf)
+                         : carry_block_scan<A, false>(f, e, seed, s_wv, s_wf);
     // fwd inclusive at j feeds tile j+1; bwd inclusive at j feeds tile j-1
     const long long tgt = rev ? (long long)j - 1 : (long long)j + 1;
     if (j < ntiles && tgt >= 0 && tgt < (long long)ntiles) {
       const u8 tt = a.tile_flags[tgt];
       const bool need = rev ? (tt & TF_COUT) : (tt & TF_CIN);
       if (need) {
-        a.carry[tgt].a[d] = inc.a;
+        reinterpret_cast<Q*>(a.carry)[tgt].a[d] = inc.a;
         if (d == 0) a.owner[tgt] = inc.owner;
       }
     }
@@ -795,17 +908,23 @@ __global__ void __launch_bounds__(CARRY_T) carry_apply_kernel(ConflictArgs a, u3
 
 size_t carry_temp_bytes(u32 ntiles) {
   const u32 nch = (ntiles + CARRY_T - 1) / CARRY_T;
-  return (size_t)nch * 4 * sizeof(CarryEl) * 2 + (size_t)nch * 4 + 256;
+  return (size_t)nch * 4 * sizeof(CarryEl<Agg>) * 2 + (size_t)nch * 4 + 256;
 }
 
-void launch_carry(const ConflictArgs& a, u32 ntiles, void* temp, cudaStream_t st) {
+template <class A>
+static void launch_carry_t(const ConflictArgs& a, u32 ntiles, void* temp, cudaStream_t st) {
   const u32 nch = (ntiles + CARRY_T - 1) / CARRY_T;
-  CarryEl* tot = reinterpret_cast<CarryEl*>(temp);
-  CarryEl* car = tot + (size_t)nch * 4;
+  CarryEl<A>* tot = reinterpret_cast<CarryEl<A>*>(temp);
+  CarryEl<A>* car = tot + (size_t)nch * 4;
   u8* fl = reinterpret_cast<u8*>(car + (size_t)nch * 4);
-  carry_chunk_kernel<<<nch, CARRY_T, 0, st>>>(a, ntiles, tot, fl);
-  carry_top_kernel<<<1, CARRY_T, 0, st>>>(nch, tot, fl, car);
-  carry_apply_kernel<<<nch, CARRY_T, 0, st>>>(a, ntiles, car);
+  carry_chunk_kernel<A><<<nch, CARRY_T, 0, st>>>(a, ntiles, tot, fl);
+  carry_top_kernel<A><<<1, CARRY_T, 0, st>>>(nch, tot, fl, car);
+  carry_apply_kernel<A><<<nch, CARRY_T, 0, st>>>(a, ntiles, car);
+}
+
+void launch_carry(bool exact, const ConflictArgs& a, u32 ntiles, void* temp, cudaStream_t st) {
+  if (exact) launch_carry_t<Agg>(a, ntiles, temp, st);
+  else launch_carry_t<AggC>(a, ntiles, temp, st);
 }
 
 // canonical sort key of a race record (as emitted by emit_race) rebuilt from its fields (rank-0 merge)

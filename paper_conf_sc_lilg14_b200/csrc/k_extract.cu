@@ -43,8 +43,8 @@ struct SpaceAcc {
   }
 };
 
-template <int THREADS, int U>
-__global__ void __launch_bounds__(THREADS) extents_kernel(const Rec* __restrict__ rec, u64 n, u32 log2G,
+template <int THREADS, int U, int MINB>
+__global__ void __launch_bounds__(THREADS, MINB) extents_kernel(const Rec* __restrict__ rec, u64 n, u32 log2G,
                                                           Summary* __restrict__ out) {
   u64 bad = ~0ull, ent = 0, multi = 0;
   SpaceAcc A0, A1;  // shared, global
@@ -153,7 +153,23 @@ static int ring_grid(const void* kern, int threads, size_t smem, size_t smem_max
 }
 
 void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, int grid, cudaStream_t st) {
-  extents_kernel<256, 4><<<grid, 256, 0, st>>>(rec, n, log2G, d_sum);
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("SESA_EXT_CFG");
+    v = e ? atoi(e) : 1;  // measured best on C5: U=4 records in flight, 64 registers, 4 CTAs/SM
+  }
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const unsigned g = (unsigned)std::min<u64>((n + 255) / 256, (u64)sms * 8);
+  switch (v) {
+    case 1: extents_kernel<256, 4, 4><<<g, 256, 0, st>>>(rec, n, log2G, d_sum); break;
+    case 2: extents_kernel<256, 8, 2><<<g, 256, 0, st>>>(rec, n, log2G, d_sum); break;
+    case 3: extents_kernel<256, 2, 6><<<g, 256, 0, st>>>(rec, n, log2G, d_sum); break;
+    case 4: extents_kernel<256, 8, 3><<<g, 256, 0, st>>>(rec, n, log2G, d_sum); break;
+    default: extents_kernel<256, 4, 1><<<g, 256, 0, st>>>(rec, n, log2G, d_sum); break;
+  }
+  (void)grid;
 }
 
 // ------------------------------------------------------------------------------------------------------------

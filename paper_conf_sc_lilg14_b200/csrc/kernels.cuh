@@ -48,8 +48,18 @@ struct Agg {
   u64 v1, v1b;       // min write value; min write value over identities != i1 (none: ~0)
   u64 v2, v2b;       // max write value; max write value over identities != i2 (none: 0)
 };
+// Cheap summary: per type min/max identity + min/max write value.  Resolves every flag except "exists a write
+// with identity != mine and value != mine" when the set holds >= 2 writer identities and >= 2 distinct values
+// (then the query is "unknown" and the check is redone with the exact summary).
+struct AggC {
+  u32 mn[3], mx[3];
+  u64 vlo, vhi;  // min / max write value (empty: ~0 / 0)
+};
 struct AggQuad {
   Agg a[4];
+};
+struct AggQuadC {
+  AggC a[4];
 };
 struct ConflictArgs {
   const u64* keys;  // sorted entry keys
@@ -71,8 +81,9 @@ struct ConflictArgs {
   u32* cross_count;
   u8* tile_flags;    // per tile: bit0 grp head in tile, bit1 grp tail in tile, bit2 sub head, bit3 sub tail,
                      // bit4 cross-in, bit5 cross-out
-  AggQuad* part;   // per tile: [0] grp first piece (P), [1] grp last piece (S), [2] sub P, [3] sub S
-  AggQuad* carry;  // per tile: [0] grp In, [1] grp Out, [2] sub In, [3] sub Out
+  void* part;      // per tile AggQuad(C): [0] grp first piece (P), [1] grp last piece (S), [2] sub P, [3] sub S
+  void* carry;     // per tile AggQuad(C): [0] grp In, [1] grp Out, [2] sub In, [3] sub Out
+  u32* need_exact; // set by cheap-summary tiles that met an unknown benign query
   u32* owner;             // per tile: tile index holding the head of the group that crosses into this tile
   struct Slot* slots;     // per owner tile
   u64 index_base;
@@ -93,8 +104,8 @@ struct Slot {
   u32 hblock, hinterval;
 };
 
-void launch_conflict(int mode, const ConflictArgs& a, u32 ntiles_or_list, cudaStream_t st);
-void launch_carry(const ConflictArgs& a, u32 ntiles, void* temp, cudaStream_t st);
+void launch_conflict(int mode, bool exact, const ConflictArgs& a, u32 ntiles_or_list, cudaStream_t st);
+void launch_carry(bool exact, const ConflictArgs& a, u32 ntiles, void* temp, cudaStream_t st);
 size_t carry_temp_bytes(u32 ntiles);
 void launch_cross_emit(const ConflictArgs& a, u32 ntiles, cudaStream_t st);
 void launch_permute_races(const RaceOut* in, const u32* order, RaceOut* out, u32 nr, cudaStream_t st);

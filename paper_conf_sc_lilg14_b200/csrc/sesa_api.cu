@@ -331,7 +331,6 @@ bool sesa_trace::step_conflict(const u64* comp, u32 m2, const Rec* rec, u32 rec_
         !grow(b_rvals[0], (size_t)race_cap * 4, "race vals") || !grow(b_rvals[1], (size_t)race_cap * 4, "race vals") ||
         !grow(b_carrytmp, carry_temp_bytes(ctiles), "carry temp"))
       return false;
-    cudaMemsetAsync(b_ccount.p, 0, 16, stream);
     ConflictArgs A;
     memset(&A, 0, sizeof A);
     A.keys = comp;
@@ -344,29 +343,43 @@ bool sesa_trace::step_conflict(const u64* comp, u32 m2, const Rec* rec, u32 rec_
     A.ls = cfg.lockstep;
     A.race_count = (u32*)b_ccount.p;
     A.cross_count = (u32*)b_ccount.p + 1;
+    A.need_exact = (u32*)b_ccount.p + 2;
     A.race_keys = (u64*)b_rkeys[0].p;
     A.race_vals = (u32*)b_rvals[0].p;
     A.races = (RaceOut*)b_races.p;
     A.race_cap = race_cap;
     A.cross_list = (u32*)b_cross.p;
     A.tile_flags = (u8*)b_tflags.p;
-    A.part = (AggQuad*)b_part.p;
-    A.carry = (AggQuad*)b_carry.p;
+    A.part = b_part.p;
+    A.carry = b_carry.p;
     A.owner = (u32*)b_owner.p;
     A.slots = (Slot*)b_slots.p;
     A.index_base = index_base;
-    LAUNCH("conflict", 40.0 * m2, launch_conflict(1, A, ctiles, stream));
-    u32 cc[2];
-    if (!cuda_ok(cudaMemcpyAsync(cc, b_ccount.p, 8, cudaMemcpyDeviceToHost, stream), "counts")) return false;
-    if (!sync_check("conflict")) return false;
-    info.crossing_tiles = cc[1];
-    if (cc[1]) {
-      LAUNCH("carry", 0.0, launch_carry(A, ctiles, b_carrytmp.p, stream));
-      LAUNCH("conflict_cross", 0.0, launch_conflict(2, A, cc[1], stream));
-      LAUNCH("conflict_y", 0.0, launch_conflict(3, A, cc[1], stream));
-      LAUNCH("cross_emit", 0.0, launch_cross_emit(A, cc[1], stream));
-      if (!cuda_ok(cudaMemcpyAsync(cc, b_ccount.p, 8, cudaMemcpyDeviceToHost, stream), "counts")) return false;
-      if (!sync_check("crossing")) return false;
+    // cheap summaries first; a benign query they cannot decide (>= 2 writers with >= 2 values at one location)
+    // makes the whole check rerun with the exact summaries (mode 1 and, for crossing runs, mode 2 can detect it)
+    u32 cc[3] = {0, 0, 0};
+    for (int pass = 0; pass < 2; pass++) {
+      const bool exact = pass == 1;
+      cudaMemsetAsync(b_ccount.p, 0, 16, stream);
+      LAUNCH(exact ? "conflict_exact" : "conflict", 40.0 * m2, launch_conflict(1, exact, A, ctiles, stream));
+      if (!cuda_ok(cudaMemcpyAsync(cc, b_ccount.p, 12, cudaMemcpyDeviceToHost, stream), "counts")) return false;
+      if (!sync_check("conflict")) return false;
+      if (cc[2] && !exact) continue;
+      info.crossing_tiles = cc[1];
+      if (cc[1]) {
+        LAUNCH("carry", 0.0, launch_carry(exact, A, ctiles, b_carrytmp.p, stream));
+        LAUNCH("conflict_cross", 0.0, launch_conflict(2, exact, A, cc[1], stream));
+        if (!exact) {
+          if (!cuda_ok(cudaMemcpyAsync(cc, b_ccount.p, 12, cudaMemcpyDeviceToHost, stream), "counts")) return false;
+          if (!sync_check("crossing")) return false;
+          if (cc[2]) continue;
+        }
+        LAUNCH("conflict_y", 0.0, launch_conflict(3, exact, A, cc[1], stream));
+        LAUNCH("cross_emit", 0.0, launch_cross_emit(A, cc[1], stream));
+        if (!cuda_ok(cudaMemcpyAsync(cc, b_ccount.p, 12, cudaMemcpyDeviceToHost, stream), "counts")) return false;
+        if (!sync_check("crossing")) return false;
+      }
+      break;
     }
     if (cc[0] <= race_cap) {
       n_races = cc[0];
