@@ -211,11 +211,13 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="c5", choices=sorted(CONFIGS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--n", type=int, default=None, help="override the C5 record count")
+    ap.add_argument("--records", type=int, default=None, help="override the C5 record count")
     ap.add_argument("--cpu-records", type=int, default=1 << 24)
     ap.add_argument("--ref-records", type=int, default=1 << 23)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--force-dist", action="store_true",
+                    help="use the NCCL distributed handle even with one rank (exercises the N>1 code path)")
     args = ap.parse_args()
 
     rank = int(os.environ.get("RANK", "0"))
@@ -231,7 +233,7 @@ def main():
     S.load()
     c = CONFIGS[args.config]
     pg = None
-    if world > 1:
+    if world > 1 or args.force_dist:
         import torch.distributed as dist
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
         pg = dist
@@ -242,7 +244,7 @@ def main():
     else:
         trace = S.Trace(c["ws"], c["ls"], 4)
 
-    recs, n_local, base, n_total = make_records(args.config, args.n, rank, world)
+    recs, n_local, base, n_total = make_records(args.config, args.records, rank, world)
     torch.cuda.synchronize()
     log(f"[bench] rank {rank}/{world}: {args.config} n={n_total} local={n_local}")
     stream = torch.cuda.current_stream()
