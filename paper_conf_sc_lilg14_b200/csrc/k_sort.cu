@@ -112,7 +112,8 @@ __device__ __forceinline__ void onesweep_tile(const u64* __restrict__ kin, u64* 
   u32* vals_s = reinterpret_cast<u32*>(keys_s + TILE);                          // [TILE] if VALS
   u32* whist = VALS ? vals_s + TILE : reinterpret_cast<u32*>(keys_s + TILE);    // [WARPS][RADIX]
   u32* bin_start = whist + WARPS * RADIX;                                       // [RADIX]
-  long long* glob = reinterpret_cast<long long*>(bin_start + RADIX);            // [RADIX]
+  long long* glob = reinterpret_cast<long long*>(bin_start + RADIX);            // [RADIX] (8-byte slots)
+  u32* globu = reinterpret_cast<u32*>(glob);                                    // u32 view of the same slots
   u32* scratch = reinterpret_cast<u32*>(glob + RADIX);                          // [WARPS + 1]
   u32* wmask = scratch + WARPS + 1;                                             // [WARPS][RADIX + 1]
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -188,7 +189,7 @@ __device__ __forceinline__ void onesweep_tile(const u64* __restrict__ kin, u64* 
       if (prof && tid == 0) prof[7] = ((u64)(tile - p) << 32) | (u64)spins;  // walk distance, spins (digit 0)
       st_relaxed(lookback + (u64)tile * RADIX + tid, lb_pack(LB_PREFIX, epoch, excl + tot));
     }
-    glob[tid] = (long long)(bin_base[tid] + excl) - (long long)bs;
+    globu[tid] = (u32)(bin_base[tid] + excl) - bs;  // positions < m < 2^32: modular u32 offsets
   }
   if (prof) {
     __syncthreads();
@@ -206,15 +207,17 @@ __device__ __forceinline__ void onesweep_tile(const u64* __restrict__ kin, u64* 
       // each lane sets its bit in its digit's word of a per-warp mask array: the word becomes the peer set
       atomicOr(&wm[d], 1u << lane);
       __syncwarp();
-      peers = wm[d];
-      __syncwarp();
     }
-    const bool leader = lane == 31 - __clz(peers);
-    if (MATCH == 1 && leader) wm[d] = 0;
+    // the peer word and the running counter are read together: one shared-memory round trip per item
+    if (MATCH == 1) peers = wm[d];
     const u32 c = wh[d];
-    rd[i] |= (c + __popc(peers & lanemask_lt())) << 9;
     __syncwarp();
-    if ((FULL || d < RADIX) && leader) wh[d] = c + __popc(peers);
+    const bool leader = lane == 31 - __clz(peers);
+    rd[i] |= (c + __popc(peers & lanemask_lt())) << 9;
+    if (leader) {
+      if (MATCH == 1) wm[d] = 0;
+      if (FULL || d < RADIX) wh[d] = c + __popc(peers);
+    }
     __syncwarp();
   }
   __syncthreads();
@@ -234,7 +237,7 @@ __device__ __forceinline__ void onesweep_tile(const u64* __restrict__ kin, u64* 
   for (u32 j = tid; j < tcount; j += THREADS) {
     const u64 key = keys_s[j];
     const u32 d = (u32)((key >> shift) & (RADIX - 1));
-    const u64 dst = (u64)(glob[d] + (long long)j);
+    const u32 dst = globu[d] + j;
     __stcs(kout + dst, key);
     if (VALS) __stcs(vout + dst, vals_s[j]);
   }
@@ -276,6 +279,199 @@ __global__ void __launch_bounds__(THREADS, MINB) onesweep_kernel(const u64* __re
                                                            tile, smem, prof);
 }
 
+// ------------------------------------------------------------------------------------------------------------
+// onesweep2 (keys only): the tile-local position of every key is known once the tile's digit counts are (bin
+// start + the warp's offset within the bin + its stable rank in the warp), so ranking writes each key straight
+// into its shared-memory slot and keeps no per-item rank registers; the global offsets from the look-back are
+// only needed by the final coalesced write-out.  LATE_LB = walk the look-back after ranking (predecessors have
+// had the ranking time to publish their inclusive prefixes) instead of before.
+// ------------------------------------------------------------------------------------------------------------
+template <int THREADS, int ITEMS, int LBW, bool FULL, bool LATE_LB, int S, bool BAL>
+__device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64* __restrict__ kout, u32 m, u32 shift,
+                                               const u64* __restrict__ bin_base, u64* __restrict__ lookback,
+                                               u32 epoch, u32 tile, unsigned char* smem, unsigned long long* prof) {
+  constexpr int WARPS = THREADS / 32;
+  constexpr int TILE = THREADS * ITEMS;
+  constexpr int IPS = ITEMS / S;  // items per rank stream
+  static_assert(ITEMS % S == 0, "streams split the items evenly");
+  u64* keys_s = reinterpret_cast<u64*>(smem);                    // [TILE]
+  u32* whist = reinterpret_cast<u32*>(keys_s + TILE);             // [WARPS*S][RADIX]: counts -> tile-local bases
+  u32* globu = whist + WARPS * S * RADIX;                        // [RADIX]
+  u32* scratch = globu + RADIX;                                  // [WARPS + 1]
+  u32* wmask = scratch + WARPS + 1;                              // [WARPS*S][RADIX + 1]
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const u64 tbase = (u64)tile * TILE;
+  const u64 wbase = tbase + (u64)warp * 32 * ITEMS + lane;
+  const int nv = FULL ? ITEMS : (int)(wbase < m ? min((u64)ITEMS, ((u64)m - wbase + 31) / 32) : 0ull);
+  u64 k[ITEMS];
+#pragma unroll
+  for (int i = 0; i < ITEMS; i++)
+    if (FULL || i < nv) k[i] = __ldcs(kin + wbase + (u64)i * 32);
+  auto digit = [&](int i) -> u32 {
+    return (FULL || i < nv) ? (u32)((k[i] >> shift) & (RADIX - 1)) : (u32)RADIX;
+  };
+  // rank streams: items [s*IPS, (s+1)*IPS) of a warp form stream s (stable order = warp, stream, item, lane),
+  // each with its own counters and peer masks, so that S items are ranked per shared-memory round trip
+  u32* wh = whist + warp * S * RADIX;
+  if (prof) {
+    __syncthreads();
+    if (tid == 0) prof[1] = gtime();
+  }
+  // (1) per-(warp, stream) digit counts
+#pragma unroll
+  for (int i = 0; i < ITEMS; i++)
+    if (FULL || i < nv) atomicAdd(&wh[(i / IPS) * RADIX + digit(i)], 1u);
+  __syncthreads();
+  // (2) tile totals -> publish the aggregate; per-(warp, stream, digit) tile-local base = bin start + offset
+  u32 tot = 0;
+  if (tid < RADIX) {
+#pragma unroll
+    for (int w = 0; w < WARPS * S; w++) {
+      const u32 c = whist[w * RADIX + tid];
+      whist[w * RADIX + tid] = tot;
+      tot += c;
+    }
+    st_relaxed(lookback + (u64)tile * RADIX + tid, lb_pack(tile == 0 ? LB_PREFIX : LB_AGG, epoch, tot));
+  }
+  const u32 bs = block_excl_sum<THREADS>(tid < RADIX ? tot : 0u, scratch);  // (contains __syncthreads)
+  if (tid < RADIX) {
+#pragma unroll
+    for (int w = 0; w < WARPS * S; w++) whist[w * RADIX + tid] += bs;
+  }
+  auto look_back = [&]() {
+    if (tid < RADIX) {
+      u64 excl = 0;
+      if (tile > 0) {
+        long long p = (long long)tile - 1;
+        int spins = 0;
+        while (true) {
+          u64 w[LBW];
+#pragma unroll
+          for (int q = 0; q < LBW; q++) w[q] = p - q >= 0 ? ld_relaxed(lookback + (u64)(p - q) * RADIX + tid) : 0ull;
+          int q = 0;
+          bool done = false;
+#pragma unroll
+          for (int qq = 0; qq < LBW; qq++) {
+            if (done || q != qq || p - qq < 0) continue;
+            const u32 e = (u32)((w[qq] >> 54) & 0xFF);
+            const u64 st = w[qq] & (3ull << 62);
+            if (e != epoch || st == 0) continue;
+            excl += w[qq] & LB_VAL;
+            q = qq + 1;
+            if (st == LB_PREFIX) done = true;
+          }
+          if (done) break;
+          if (q == 0) __nanosleep(++spins < 4 ? 32 : 128);
+          p -= q;
+        }
+        if (prof && tid == 0) prof[7] = ((u64)(tile - p) << 32) | (u64)spins;
+        st_relaxed(lookback + (u64)tile * RADIX + tid, lb_pack(LB_PREFIX, epoch, excl + tot));
+      }
+      globu[tid] = (u32)(bin_base[tid] + excl) - bs;  // positions < m < 2^32: modular u32 offsets
+    }
+  };
+  if (!LATE_LB) look_back();
+  __syncthreads();
+  if (prof && tid == 0) prof[2] = gtime();
+  // (3) stable warp ranking, each key stored straight into its tile-local slot
+  u32* wm = wmask + warp * S * (RADIX + 1);
+  const unsigned lt = lanemask_lt();
+#pragma unroll
+  for (int i = 0; i < IPS; i++) {
+    u32 d[S];
+#pragma unroll
+    for (int q = 0; q < S; q++) {
+      d[q] = digit(q * IPS + i);
+      if (!BAL) atomicOr(&wm[q * (RADIX + 1) + d[q]], 1u << lane);
+    }
+    if (!BAL) __syncwarp();
+    unsigned peers[S];
+    u32 c[S];
+#pragma unroll
+    for (int q = 0; q < S; q++) {
+      // BAL: the peer set from one ballot per digit bit (ALU pipe, no shared-memory traffic)
+      peers[q] = BAL ? (FULL ? peers_of<RADIX_BITS>(d[q]) : peers_of<RADIX_BITS + 1>(d[q]))
+                     : wm[q * (RADIX + 1) + d[q]];
+      c[q] = wh[q * RADIX + d[q]];
+    }
+    __syncwarp();
+#pragma unroll
+    for (int q = 0; q < S; q++) {
+      const bool leader = lane == 31 - __clz(peers[q]);
+      if (FULL || d[q] < RADIX) keys_s[c[q] + __popc(peers[q] & lt)] = k[q * IPS + i];
+      if (leader) {
+        if (!BAL) wm[q * (RADIX + 1) + d[q]] = 0;
+        if (FULL || d[q] < RADIX) wh[q * RADIX + d[q]] = c[q] + __popc(peers[q]);
+      }
+    }
+    __syncwarp();
+  }
+  if (prof && tid == 0) prof[3] = gtime();
+  if (LATE_LB) look_back();
+  __syncthreads();
+  if (prof && tid == 0) prof[4] = gtime();
+  // (4) coalesced write-out of each digit's run
+  const u32 tcount = FULL ? (u32)TILE : (u32)min((u64)TILE, (u64)m - tbase);
+#pragma unroll 4
+  for (u32 j = tid; j < tcount; j += THREADS) {
+    const u64 key = keys_s[j];
+    const u32 d = (u32)((key >> shift) & (RADIX - 1));
+    __stcs(kout + (globu[d] + j), key);
+  }
+  if (prof) {
+    __syncthreads();
+    if (tid == 0) prof[5] = gtime(), prof[6] = (u64)blockIdx.x;
+  }
+}
+
+template <int THREADS, int ITEMS, int MINB, int LBW, bool LATE_LB, int S, bool BAL>
+__global__ void __launch_bounds__(THREADS, MINB) onesweep2_kernel(const u64* __restrict__ kin, u64* __restrict__ kout,
+                                                                  u32 m, u32 shift, const u64* __restrict__ bin_base,
+                                                                  u64* __restrict__ lookback,
+                                                                  u32* __restrict__ tile_ctr, u32 epoch) {
+  constexpr int WARPS = THREADS / 32;
+  constexpr int TILE = THREADS * ITEMS;
+  static_assert(RADIX <= THREADS, "one bin per thread");
+  extern __shared__ __align__(16) unsigned char smem[];
+  u32* whist = reinterpret_cast<u32*>(smem) + 2 * TILE;
+  u32* wmask = whist + WARPS * S * RADIX + RADIX + WARPS + 1;
+  __shared__ u32 s_tile;
+  const int tid = threadIdx.x;
+  if (tid == 0) s_tile = atomicAdd(tile_ctr, 1u);
+  for (int i = tid; i < WARPS * S * RADIX; i += THREADS) whist[i] = 0;
+  if (!BAL)
+    for (int i = tid; i < WARPS * S * (RADIX + 1); i += THREADS) wmask[i] = 0;
+  __syncthreads();
+  const u32 tile = s_tile;
+  unsigned long long* prof = g_prof ? g_prof + (u64)tile * 8 : nullptr;
+  if (prof && tid == 0) prof[0] = gtime();
+  if ((u64)(tile + 1) * TILE <= m)
+    onesweep2_tile<THREADS, ITEMS, LBW, true, LATE_LB, S, BAL>(kin, kout, m, shift, bin_base, lookback, epoch, tile, smem, prof);
+  else
+    onesweep2_tile<THREADS, ITEMS, LBW, false, LATE_LB, S, BAL>(kin, kout, m, shift, bin_base, lookback, epoch, tile, smem, prof);
+}
+
+template <int THREADS, int ITEMS, int S, bool BAL>
+static size_t onesweep2_smem() {
+  constexpr int WARPS = THREADS / 32, TILE = THREADS * ITEMS;
+  return (size_t)TILE * 8 + (size_t)WARPS * S * RADIX * 4 + RADIX * 4 + (WARPS + 1) * 4 +
+         (BAL ? 0 : (size_t)WARPS * S * (RADIX + 1) * 4);
+}
+
+template <int THREADS, int ITEMS, int MINB, int LBW, bool LATE_LB, int S = 1, bool BAL = false>
+static void launch_os2(const u64* kin, u64* kout, u32 m, u32 shift, const u64* bin_base, u64* lookback,
+                       u32* tile_ctr, u32 epoch, cudaStream_t st) {
+  auto kern = onesweep2_kernel<THREADS, ITEMS, MINB, LBW, LATE_LB, S, BAL>;
+  const size_t sm = onesweep2_smem<THREADS, ITEMS, S, BAL>();
+  static bool set = false;
+  if (!set) {
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    set = true;
+  }
+  const u32 tiles = (u32)((m + THREADS * ITEMS - 1) / (THREADS * ITEMS));
+  kern<<<tiles, THREADS, sm, st>>>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch);
+}
+
 template <int THREADS, int ITEMS, bool VALS>
 static size_t onesweep_smem() {
   constexpr int WARPS = THREADS / 32, TILE = THREADS * ITEMS;
@@ -283,17 +479,27 @@ static size_t onesweep_smem() {
          (WARPS + 1) * 4 + (size_t)WARPS * (RADIX + 1) * 4;
 }
 
-int sort_cfg() {  // SESA_SORT_CFG: 0 = 256x16, 1 = 256x24, 2 = 512x16, 3 = TMA 256x16, 4 = TMA 256x24; default 1
-//   (measured on C5: 1 fastest; the persistent TMA-prefetch variants delay aggregates and lose badly)
+// SESA_SORT_CFG selects the onesweep variant (all measured on C5, 1 B200; DESIGN.md §6 has the table):
+//   0 / 1   onesweep (ranks kept in registers, look-back before ranking), 256 x 16 / 256 x 24 keys
+//   13..16  onesweep2, 256 x 24: early / late look-back at 2 CTAs/SM (13/14), 3 CTAs/SM (15/16)
+//   19 / 20 onesweep2, 256 x 32, early / late look-back (20 = default: fastest)
+//   21      as 20 with 16 predecessors per look-back round trip;  26: two rank streams;  31: ballot peers
+int sort_cfg() {
   static int v = -1;
   if (v < 0) {
     const char* e = getenv("SESA_SORT_CFG");
-    v = e ? atoi(e) : 1;
+    v = e ? atoi(e) : 20;
   }
   return v;
 }
 
-u32 sort_tile_keys() { return (sort_cfg() == 1 || sort_cfg() == 4) ? 256 * 24 : sort_cfg() == 2 ? 512 * 16 : 256 * 16; }
+u32 sort_tile_keys() {
+  switch (sort_cfg()) {
+    case 1: case 13: case 14: case 15: case 16: return 256 * 24;
+    case 19: case 20: case 21: case 26: case 31: return 256 * 32;
+    default: return 256 * 16;
+  }
+}
 
 int sort_variant() {  // SESA_SORT_MATCH=0 ballots, 1 atomicOr masks (default)
   static int v = -1;
@@ -305,338 +511,6 @@ int sort_variant() {  // SESA_SORT_MATCH=0 ballots, 1 atomicOr masks (default)
 }
 
 
-
-// ------------------------------------------------------------------------------------------------------------
-// Warp-specialized onesweep (cfg 8/9): 8 worker warps load, count, rank and scatter; one helper warp turns the
-// per-warp counts into tile totals and per-warp offsets, publishes the tile aggregate, walks the look-back for
-// all 256 digits (8 per lane, loads interleaved) and fills the global offsets — concurrently with the workers'
-// ranking (named barriers 1/2), so the look-back wait overlaps the ranking instead of preceding it.
-// ------------------------------------------------------------------------------------------------------------
-template <int ITEMS, int MINB>
-__global__ void __launch_bounds__(288, MINB) onesweep_ws_kernel(const u64* __restrict__ kin, u64* __restrict__ kout,
-                                                                u32 m, u32 shift, const u64* __restrict__ bin_base,
-                                                                u64* __restrict__ lookback, u32* __restrict__ tile_ctr,
-                                                                u32 epoch) {
-  constexpr int WARPS = 8, WT = 256, TILE = WT * ITEMS;
-  extern __shared__ __align__(16) unsigned char smem[];
-  u64* keys_s = reinterpret_cast<u64*>(smem);                          // [TILE]
-  u32* whist = reinterpret_cast<u32*>(keys_s + TILE);                  // [WARPS][RADIX] counts -> warp offsets
-  u32* wcnt = whist + WARPS * RADIX;                                   // [WARPS][RADIX + 1] local running counters
-  u32* wmask = wcnt + WARPS * (RADIX + 1);                             // [WARPS][RADIX + 1]
-  u32* bin_start = wmask + WARPS * (RADIX + 1);                        // [RADIX]
-  long long* glob = reinterpret_cast<long long*>(bin_start + RADIX + (RADIX & 1));  // [RADIX]
-  __shared__ u32 s_tile;
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  if (tid == 0) s_tile = atomicAdd(tile_ctr, 1u);
-  for (int i = tid; i < WARPS * RADIX; i += 288) whist[i] = 0;
-  for (int i = tid; i < 2 * WARPS * (RADIX + 1); i += 288) wcnt[i] = 0;  // wcnt and wmask
-  __syncthreads();
-  const u32 tile = s_tile;
-  const u64 tbase = (u64)tile * TILE;
-  const bool full = tbase + TILE <= m;
-  u64 k[ITEMS];
-  u32 rd[ITEMS];
-  int nv = 0;
-  if (warp < WARPS) {
-    const u64 wbase = tbase + (u64)warp * 32 * ITEMS + lane;
-    nv = full ? ITEMS : (int)(wbase < m ? min((u64)ITEMS, ((u64)m - wbase + 31) / 32) : 0ull);
-#pragma unroll
-    for (int i = 0; i < ITEMS; i++)
-      if (i < nv) k[i] = __ldcs(kin + wbase + (u64)i * 32);
-#pragma unroll
-    for (int i = 0; i < ITEMS; i++) rd[i] = i < nv ? (u32)((k[i] >> shift) & (RADIX - 1)) : (u32)RADIX;
-    u32* wh = whist + warp * RADIX;
-#pragma unroll
-    for (int i = 0; i < ITEMS; i++)
-      if (i < nv) atomicAdd(&wh[rd[i]], 1u);
-  }
-  __syncthreads();  // counts complete
-  if (warp == WARPS) {
-    // ---- helper warp: 8 digits per lane (d = lane + 32 q)
-    u32 tot[8];
-#pragma unroll
-    for (int q = 0; q < 8; q++) {
-      const int d = lane + 32 * q;
-      u32 t = 0;
-#pragma unroll
-      for (int w = 0; w < WARPS; w++) {
-        const u32 c = whist[w * RADIX + d];
-        whist[w * RADIX + d] = t;
-        t += c;
-      }
-      tot[q] = t;
-      st_relaxed(lookback + (u64)tile * RADIX + d, lb_pack(tile == 0 ? LB_PREFIX : LB_AGG, epoch, t));
-    }
-    // bin_start: exclusive scan over d = 0..255 (lane-major order d = lane + 32 q: scan over q-rows of 32)
-    u32 carry = 0;
-#pragma unroll
-    for (int q = 0; q < 8; q++) {
-      u32 x = tot[q];
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const u32 y = __shfl_up_sync(~0u, x, o);
-        if (lane >= o) x += y;
-      }
-      bin_start[lane + 32 * q] = carry + x - tot[q];
-      carry += __shfl_sync(~0u, x, 31);
-    }
-    // look-back: 8 digits per lane walked together (independent loads in flight)
-    u64 excl[8];
-    long long p[8];
-    bool done[8];
-#pragma unroll
-    for (int q = 0; q < 8; q++) excl[q] = 0, p[q] = (long long)tile - 1, done[q] = tile == 0;
-    int spins = 0;
-    while (true) {
-      bool all = true;
-      u64 w[8];
-#pragma unroll
-      for (int q = 0; q < 8; q++) w[q] = (!done[q] && p[q] >= 0) ? ld_relaxed(lookback + (u64)p[q] * RADIX + lane + 32 * q) : 0ull;
-      bool progress = false;
-#pragma unroll
-      for (int q = 0; q < 8; q++) {
-        if (done[q]) continue;
-        const u32 e = (u32)((w[q] >> 54) & 0xFF);
-        const u64 st = w[q] & (3ull << 62);
-        if (e != epoch || st == 0) {
-          all = false;
-          continue;
-        }
-        progress = true;
-        excl[q] += w[q] & LB_VAL;
-        if (st == LB_PREFIX) done[q] = true;
-        else p[q]--, all = false;
-      }
-      if (all) break;
-      if (!progress) __nanosleep(++spins < 4 ? 32 : 128);
-    }
-#pragma unroll
-    for (int q = 0; q < 8; q++) {
-      const int d = lane + 32 * q;
-      if (tile > 0) st_relaxed(lookback + (u64)tile * RADIX + d, lb_pack(LB_PREFIX, epoch, excl[q] + tot[q]));
-      glob[d] = (long long)(bin_base[d] + excl[q]) - (long long)bin_start[d];
-    }
-    asm volatile("bar.arrive 1, 288;" ::: "memory");  // offsets ready
-  } else {
-    // ---- worker warps: stable ranking within the warp (local counters), concurrently with the look-back
-    u32* wm = wmask + warp * (RADIX + 1);
-    u32* wc = wcnt + warp * (RADIX + 1);
-#pragma unroll
-    for (int i = 0; i < ITEMS; i++) {
-      const u32 d = rd[i];
-      atomicOr(&wm[d], 1u << lane);
-      __syncwarp();
-      const unsigned peers = wm[d];
-      __syncwarp();
-      const bool leader = lane == 31 - __clz(peers);
-      if (leader) wm[d] = 0;
-      const u32 c = wc[d];
-      rd[i] |= (c + __popc(peers & lanemask_lt())) << 9;
-      __syncwarp();
-      if (leader) wc[d] = c + __popc(peers);
-      __syncwarp();
-    }
-    asm volatile("bar.sync 1, 288;" ::: "memory");  // wait for the helper's offsets
-    const u32* wo = whist + warp * RADIX;
-#pragma unroll
-    for (int i = 0; i < ITEMS; i++) {
-      if (i < nv) {
-        const u32 d = rd[i] & 511;
-        keys_s[bin_start[d] + wo[d] + (rd[i] >> 9)] = k[i];
-      }
-    }
-  }
-  __syncthreads();  // tile scattered into shared memory
-  const u32 tcount = full ? (u32)TILE : (u32)min((u64)TILE, (u64)m - tbase);
-#pragma unroll 4
-  for (u32 j = tid; j < tcount; j += 288) {
-    const u64 key = keys_s[j];
-    const u32 d = (u32)((key >> shift) & (RADIX - 1));
-    __stcs(kout + (u64)(glob[d] + (long long)j), key);
-  }
-}
-
-template <int ITEMS, int MINB>
-static void launch_os_ws(const u64* kin, u64* kout, u32 m, u32 shift, const u64* bin_base, u64* lookback,
-                         u32* tile_ctr, u32 epoch, cudaStream_t st) {
-  constexpr int TILE = 256 * ITEMS;
-  auto kern = onesweep_ws_kernel<ITEMS, MINB>;
-  const size_t sm = (size_t)TILE * 8 + 8 * RADIX * 4 + 2 * 8 * (RADIX + 1) * 4 + RADIX * 4 + 8 + RADIX * 8 + 64;
-  static bool set = false;
-  if (!set) {
-    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-    set = true;
-  }
-  kern<<<(unsigned)((m + TILE - 1) / TILE), 288, sm, st>>>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch);
-}
-
-// ------------------------------------------------------------------------------------------------------------
-// Persistent, TMA-pipelined onesweep pass (keys only).  Each CTA acquires tiles in increasing order from a
-// counter and, while it ranks / looks back / scatters tile i, the TMA engine (cp.async.bulk, mbarrier
-// completion) is already streaming its next tile into the other shared-memory stage, so loads stay in flight
-// through the look-back waits (ncu on the one-tile-per-CTA kernel: 49% long-scoreboard stalls).  Keys are read
-// from shared memory warp-striped (conflict-free) into registers; the consumed stage doubles as the scatter
-// buffer for the coalesced write-out.  Deadlock-free: a CTA holds at most {current, next} and the lowest
-// unfinished tile is always some CTA's current tile.
-// ------------------------------------------------------------------------------------------------------------
-template <int THREADS, int ITEMS, int MINB>
-__global__ void __launch_bounds__(THREADS, MINB) onesweep_tma_kernel(const u64* __restrict__ kin,
-                                                                     u64* __restrict__ kout, u32 m, u32 shift,
-                                                                     const u64* __restrict__ bin_base,
-                                                                     u64* __restrict__ lookback,
-                                                                     u32* __restrict__ tile_ctr, u32 epoch) {
-  constexpr int WARPS = THREADS / 32;
-  constexpr int TILE = THREADS * ITEMS;
-  static_assert(RADIX <= THREADS, "one bin per thread");
-  extern __shared__ __align__(128) unsigned char smem[];
-  u64* stage = reinterpret_cast<u64*>(smem);                          // [2][TILE]
-  u32* whist = reinterpret_cast<u32*>(stage + 2 * TILE);              // [WARPS][RADIX]
-  u32* wmask = whist + WARPS * RADIX;                                 // [WARPS][RADIX + 1]
-  u32* bin_start = wmask + WARPS * (RADIX + 1);                       // [RADIX]
-  long long* glob = reinterpret_cast<long long*>(bin_start + RADIX);  // [RADIX]
-  u32* scratch = reinterpret_cast<u32*>(glob + RADIX);                // [WARPS + 1]
-  u64* bar = reinterpret_cast<u64*>(scratch + WARPS + 2);             // [2] (8-byte aligned)
-  __shared__ u32 s_tile[2];
-
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const u32 ntiles = (u32)((m + TILE - 1) / TILE);
-  for (int i = tid; i < WARPS * (RADIX + 1); i += THREADS) wmask[i] = 0;
-  if (tid == 0) {
-    mbar_init(&bar[0], 1);
-    mbar_init(&bar[1], 1);
-    fence_mbar_init();
-    s_tile[0] = atomicAdd(tile_ctr, 1u);
-    if (s_tile[0] < ntiles) {
-      const u64 tb = (u64)s_tile[0] * TILE;
-      const u32 bytes = (u32)((min((u64)TILE, (u64)m - tb) * 8 + 15) & ~15ull);
-      mbar_expect_tx(&bar[0], bytes);
-      bulk_g2s(stage, kin + tb, bytes, &bar[0]);
-    }
-  }
-  __syncthreads();
-  for (u32 it = 0;; it++) {
-    const int sI = it & 1;
-    const u32 tile = s_tile[sI];
-    if (tile >= ntiles) break;
-    u64* st = stage + sI * TILE;
-    for (int i = tid; i < WARPS * RADIX; i += THREADS) whist[i] = 0;
-    __syncthreads();  // everyone is done with the other stage (previous tile's write-out) and saw s_tile
-    if (tid == 0) {   // prefetch the next tile into the other stage
-      const u32 nxt = atomicAdd(tile_ctr, 1u);
-      s_tile[sI ^ 1] = nxt;
-      if (nxt < ntiles) {
-        const u64 tb = (u64)nxt * TILE;
-        const u32 bytes = (u32)((min((u64)TILE, (u64)m - tb) * 8 + 15) & ~15ull);
-        mbar_expect_tx(&bar[sI ^ 1], bytes);
-        bulk_g2s(stage + (sI ^ 1) * TILE, kin + tb, bytes, &bar[sI ^ 1]);
-      }
-    }
-    const u64 tbase = (u64)tile * TILE;
-    const bool full = tbase + TILE <= m;
-    mbar_wait(&bar[sI], (it >> 1) & 1);
-    u64 k[ITEMS];
-    u32 rk[ITEMS];
-    const u32 wofs = warp * 32 * ITEMS + lane;
-#pragma unroll
-    for (int i = 0; i < ITEMS; i++) k[i] = (full || tbase + wofs + i * 32 < m) ? st[wofs + i * 32] : ~0ull;
-    u32* wh = whist + warp * RADIX;
-#pragma unroll
-    for (int i = 0; i < ITEMS; i++)
-      if (full || tbase + wofs + i * 32 < m) atomicAdd(&wh[(u32)((k[i] >> shift) & (RADIX - 1))], 1u);
-    __syncthreads();
-    u32 tot = 0;
-    if (tid < RADIX) {
-#pragma unroll
-      for (int w = 0; w < WARPS; w++) {
-        const u32 c = whist[w * RADIX + tid];
-        whist[w * RADIX + tid] = tot;
-        tot += c;
-      }
-      st_relaxed(lookback + (u64)tile * RADIX + tid, lb_pack(tile == 0 ? LB_PREFIX : LB_AGG, epoch, tot));
-    }
-    const u32 bs = block_excl_sum<THREADS>(tid < RADIX ? tot : 0u, scratch);
-    if (tid < RADIX) {
-      bin_start[tid] = bs;
-      u64 excl = 0;
-      if (tile > 0) {
-        long long p = (long long)tile - 1;
-        int spins = 0;
-        while (true) {
-          u64 w[4];
-#pragma unroll
-          for (int q = 0; q < 4; q++) w[q] = p - q >= 0 ? ld_relaxed(lookback + (u64)(p - q) * RADIX + tid) : 0ull;
-          int q = 0;
-          bool done = false;
-          for (; q < 4 && p - q >= 0; q++) {
-            const u32 e = (u32)((w[q] >> 54) & 0xFF);
-            const u64 sst = w[q] & (3ull << 62);
-            if (e != epoch || sst == 0) break;
-            excl += w[q] & LB_VAL;
-            if (sst == LB_PREFIX) {
-              done = true;
-              break;
-            }
-          }
-          if (done) break;
-          if (q == 0) __nanosleep(++spins < 4 ? 32 : 128);
-          p -= q;
-        }
-        st_relaxed(lookback + (u64)tile * RADIX + tid, lb_pack(LB_PREFIX, epoch, excl + tot));
-      }
-      glob[tid] = (long long)(bin_base[tid] + excl) - (long long)bs;
-    }
-    // stable warp-level ranking (atomicOr peer masks), running counter starts at the warp's offset
-#pragma unroll
-    for (int i = 0; i < ITEMS; i++) {
-      const bool valid = full || tbase + wofs + i * 32 < m;
-      const u32 d = valid ? (u32)((k[i] >> shift) & (RADIX - 1)) : (u32)RADIX;
-      u32* wm = wmask + warp * (RADIX + 1);
-      atomicOr(&wm[d], 1u << lane);
-      __syncwarp();
-      const unsigned peers = wm[d];
-      __syncwarp();
-      const bool leader = lane == 31 - __clz(peers);
-      if (leader) wm[d] = 0;
-      const u32 c = valid ? wh[d] : 0u;
-      rk[i] = c + __popc(peers & lanemask_lt());
-      __syncwarp();
-      if (valid && leader) wh[d] = c + __popc(peers);
-      __syncwarp();
-    }
-    __syncthreads();  // all keys are in registers and bin_start/glob are set: reuse the stage for the scatter
-#pragma unroll
-    for (int i = 0; i < ITEMS; i++)
-      if (full || tbase + wofs + i * 32 < m) st[bin_start[(u32)((k[i] >> shift) & (RADIX - 1))] + rk[i]] = k[i];
-    __syncthreads();
-    const u32 tcount = (u32)min((u64)TILE, (u64)m - tbase);
-#pragma unroll 4
-    for (u32 j = tid; j < tcount; j += THREADS) {
-      const u64 key = st[j];
-      const u32 d = (u32)((key >> shift) & (RADIX - 1));
-      __stcs(kout + (u64)(glob[d] + (long long)j), key);
-    }
-  }
-}
-
-template <int THREADS, int ITEMS, int MINB>
-static void launch_os_tma(const u64* kin, u64* kout, u32 m, u32 shift, const u64* bin_base, u64* lookback,
-                          u32* tile_ctr, u32 epoch, cudaStream_t st) {
-  constexpr int WARPS = THREADS / 32, TILE = THREADS * ITEMS;
-  auto kern = onesweep_tma_kernel<THREADS, ITEMS, MINB>;
-  const size_t sm = (size_t)2 * TILE * 8 + (size_t)WARPS * RADIX * 4 + (size_t)WARPS * (RADIX + 1) * 4 + RADIX * 4 +
-                    RADIX * 8 + (WARPS + 2) * 4 + 16 + 64;
-  static int grid = 0;
-  if (!grid) {
-    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-    int dev = 0, sms = 148, per = 1;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, kern, THREADS, sm);
-    grid = sms * std::max(per, 1);
-  }
-  const u32 tiles = (u32)((m + TILE - 1) / TILE);
-  kern<<<std::min<u32>(tiles, (u32)grid), THREADS, sm, st>>>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch);
-}
 
 template <int THREADS, int ITEMS, int MINB, bool VALS, int MATCH, int LBW = 4>
 static void launch_os(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m, u32 shift, const u64* bin_base,
@@ -667,13 +541,15 @@ static void launch_os_cfg(const u64* kin, u64* kout, const u32* vin, u32* vout, 
                           const u64* bin_base, u64* lookback, u32* tile_ctr, u32 epoch, cudaStream_t st) {
   switch (sort_cfg()) {
     case 1: launch_os<256, 24, 2, VALS, MATCH>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 5: launch_os<256, 24, 2, VALS, MATCH, 8>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 6: launch_os<256, 24, 2, VALS, MATCH, 16>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 7: launch_os<256, 8, 5, VALS, MATCH, 8>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 10: launch_os<256, 32, 2, VALS, MATCH, 4>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 11: launch_os<256, 32, 2, VALS, MATCH, 8>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 12: launch_os<256, 40, 1, VALS, MATCH, 8>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 2: launch_os<512, 16, 1, VALS, MATCH>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 13: launch_os2<256, 24, 2, 4, false>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 14: launch_os2<256, 24, 2, 4, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 15: launch_os2<256, 24, 3, 4, false>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 16: launch_os2<256, 24, 3, 4, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 19: launch_os2<256, 32, 2, 4, false>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 20: launch_os2<256, 32, 2, 4, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 21: launch_os2<256, 32, 2, 16, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 26: launch_os2<256, 32, 2, 4, true, 2>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 31: launch_os2<256, 32, 2, 4, true, 1, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
     default: launch_os<256, 16, 3, VALS, MATCH>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
   }
 }
@@ -720,14 +596,6 @@ void launch_onesweep(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m
   if (vin) {  // race lists are small: fixed config
     if (ballot) launch_os<256, 16, 3, true, 0>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
     else launch_os<256, 16, 3, true, 1>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
-  } else if (sort_cfg() == 8) {
-    launch_os_ws<16, 2>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
-  } else if (sort_cfg() == 9) {
-    launch_os_ws<24, 1>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
-  } else if (sort_cfg() == 3) {
-    launch_os_tma<256, 16, 2>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
-  } else if (sort_cfg() == 4) {
-    launch_os_tma<256, 24, 1>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
   } else {
     if (ballot) launch_os_cfg<false, 0>(kin, kout, nullptr, nullptr, m, shift, bin_base, lookback, tile_ctr, epoch, st);
     else launch_os_cfg<false, 1>(kin, kout, nullptr, nullptr, m, shift, bin_base, lookback, tile_ctr, epoch, st);
