@@ -143,6 +143,147 @@ __global__ void __launch_bounds__(THREADS, MINB) extents_kernel(const Rec* __res
   }
 }
 
+// extents2 (default): warp w streams the contiguous record range [w*rw, (w+1)*rw) in rows of 32 (U rows in
+// flight), all index arithmetic in 32 bits (n < 2^31, include/sesa.h).  Per record only what the layout needs:
+// min address and max last byte per space (granule = address >> log2G commutes with min/max, so the shifts
+// happen once per thread), block/interval min/max, the extra-granule count from the in-granule offset (32-bit),
+// validity, and (block, interval) order against the predecessor (previous lane, or the previous row's lane 31).
+struct SpaceAcc2 {
+  u32 cnt, bmin, bmax, imin, imax;
+  u64 amin, amax;
+  __device__ __forceinline__ void init() { cnt = 0, amin = ~0ull, amax = 0, bmin = ~0u, bmax = 0, imin = ~0u, imax = 0; }
+  __device__ __forceinline__ void add(u64 a, u64 last, u32 b, u32 i) {
+    cnt++;
+    amin = min(amin, a), amax = max(amax, last);
+    bmin = min(bmin, b), bmax = max(bmax, b);
+    imin = min(imin, i), imax = max(imax, i);
+  }
+  __device__ __forceinline__ SpaceAcc to_acc(u32 log2G) const {
+    SpaceAcc A;
+    A.init();
+    if (cnt) {
+      A.cnt = cnt, A.gmin = amin >> log2G, A.gmax = amax >> log2G;
+      A.bmin = bmin, A.bmax = bmax, A.imin = imin, A.imax = imax;
+    }
+    return A;
+  }
+};
+
+template <int U>
+__global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ rec, u32 n, u32 log2G, u32 rw,
+                                                       Summary* __restrict__ out) {
+  constexpr int THREADS = 256;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const u32 gw = (blockIdx.x * THREADS + threadIdx.x) >> 5;
+  const u64 start64 = (u64)gw * rw;
+  const u32 start = (u32)min(start64, (u64)n), end = (u32)min((u64)n, start64 + rw);
+  const u32 gmask = (1u << log2G) - 1u;
+  u32 bad = ~0u, extra = 0, multi = 0, unsorted = 0;
+  SpaceAcc2 A0, A1;
+  A0.init();
+  A1.init();
+  const uint4* q = reinterpret_cast<const uint4*>(rec);
+  u64 prev_bi = 0;  // (block << 32 | interval) of the record before the current row's lane 0
+  if (start > 0 && start < end) {
+    const uint4 p = __ldg(q + 2 * (u64)(start - 1) + 1);
+    prev_bi = ((u64)p.x << 32) | p.z;
+  }
+  for (u32 r0 = start; r0 < end; r0 += 32 * U) {
+    uint4 a[U], b[U];
+#pragma unroll
+    for (int u = 0; u < U; u++) {
+      const u32 i = r0 + u * 32 + lane;
+      if (i < end) a[u] = __ldcs(q + 2 * (u64)i), b[u] = __ldcs(q + 2 * (u64)i + 1);
+      else a[u] = make_uint4(0, 0, 0, 0), b[u] = make_uint4(0, 0, 0, 0);
+    }
+    bool ok[U];
+    bool allg = true, alls = true;
+#pragma unroll
+    for (int u = 0; u < U; u++) {
+      const u32 i = r0 + u * 32 + lane;
+      const u64 bi = ((u64)b[u].x << 32) | b[u].z;
+      const u64 up = __shfl_up_sync(~0u, bi, 1);
+      const u64 pbi = lane ? up : prev_bi;
+      prev_bi = __shfl_sync(~0u, bi, 31);
+      const u32 size = b[u].w & 0xFFFFu, sp = (b[u].w >> 16) & 0xFFu, rwv = b[u].w >> 24;
+      const u64 addr = ((u64)a[u].y << 32) | a[u].x;
+      const bool in = i < end;
+      ok[u] = in && sp <= 1u && rwv <= 2u && size >= 1u && addr + (u64)size - 1ull >= addr;
+      bad = (in && !ok[u]) ? min(bad, i) : bad;
+      const u32 e = ((a[u].x & gmask) + size - 1u) >> log2G;  // granules beyond the first
+      extra += ok[u] ? e : 0u;
+      multi += (ok[u] && e != 0u) ? 1u : 0u;
+      unsorted |= (ok[u] && bi < pbi) ? 1u : 0u;
+      allg = allg && (!ok[u] || sp == SP_GLOBAL);
+      alls = alls && (!ok[u] || sp == SP_SHARED);
+    }
+    // one space decision per batch (traces are mostly single-space)
+    const bool bg = __all_sync(~0u, allg), bs = !bg && __all_sync(~0u, alls);
+#pragma unroll
+    for (int u = 0; u < U; u++) {
+      const u64 addr = ((u64)a[u].y << 32) | a[u].x;
+      const u64 last = addr + (u64)(b[u].w & 0xFFFFu) - 1ull;
+      const bool glob = bg || (!bs && ((b[u].w >> 16) & 0xFFu) == SP_GLOBAL);
+      if (ok[u]) {
+        if (glob) A1.add(addr, last, b[u].x, b[u].z);
+        else A0.add(addr, last, b[u].x, b[u].z);
+      }
+    }
+  }
+  // block reduction (warp shuffles, then one atomic per field per CTA)
+  u64 bad64 = bad == ~0u ? ~0ull : (u64)bad, ent = (u64)extra + A0.cnt + A1.cnt, mul = multi;
+  SpaceAcc S0 = A0.to_acc(log2G), S1 = A1.to_acc(log2G);
+  __shared__ SpaceAcc sa[THREADS / 32][2];
+  __shared__ u64 s64[THREADS / 32][3];
+  __shared__ u32 s_uns[THREADS / 32];
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    bad64 = min(bad64, __shfl_xor_sync(~0u, bad64, o));
+    ent += __shfl_xor_sync(~0u, ent, o);
+    mul += __shfl_xor_sync(~0u, mul, o);
+    unsorted |= __shfl_xor_sync(~0u, unsorted, o);
+  }
+  S0.warp_reduce();
+  S1.warp_reduce();
+  if (lane == 0) {
+    s64[warp][0] = bad64, s64[warp][1] = ent, s64[warp][2] = mul;
+    sa[warp][0] = S0, sa[warp][1] = S1;
+    s_uns[warp] = unsorted;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    for (int w = 1; w < THREADS / 32; w++) {
+      s64[0][0] = min(s64[0][0], s64[w][0]);
+      s64[0][1] += s64[w][1];
+      s64[0][2] += s64[w][2];
+      s_uns[0] |= s_uns[w];
+      for (int x = 0; x < 2; x++) {
+        SpaceAcc& d = sa[0][x];
+        const SpaceAcc& e = sa[w][x];
+        d.cnt += e.cnt;
+        d.gmin = min(d.gmin, e.gmin), d.gmax = max(d.gmax, e.gmax);
+        d.bmin = min(d.bmin, e.bmin), d.bmax = max(d.bmax, e.bmax);
+        d.imin = min(d.imin, e.imin), d.imax = max(d.imax, e.imax);
+      }
+    }
+    if (s64[0][0] != ~0ull) atomicMin(&out->bad_index, (unsigned long long)s64[0][0]);
+    if (s64[0][1]) atomicAdd(&out->entries, (unsigned long long)s64[0][1]);
+    if (s64[0][2]) atomicAdd(&out->multi, (unsigned long long)s64[0][2]);
+    for (int x = 0; x < 2; x++) {
+      const SpaceAcc& d = sa[0][x];
+      if (!d.cnt) continue;
+      atomicAdd(&out->count[x], (unsigned long long)d.cnt);
+      atomicMin(&out->gmin[x], (unsigned long long)d.gmin);
+      atomicMax(&out->gmax[x], (unsigned long long)d.gmax);
+      atomicMin(&out->bmin[x], d.bmin);
+      atomicMax(&out->bmax[x], d.bmax);
+      atomicMin(&out->imin[x], d.imin);
+      atomicMax(&out->imax[x], d.imax);
+    }
+    if (s_uns[0]) atomicOr(&out->unsorted, 1u);
+  }
+}
+
 static int ring_grid(const void* kern, int threads, size_t smem, size_t smem_max) {
   int dev = 0, sms = 148, per = 1;
   cudaGetDevice(&dev);
@@ -156,12 +297,25 @@ void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, int grid, 
   static int v = -1;
   if (v < 0) {
     const char* e = getenv("SESA_EXT_CFG");
-    v = e ? atoi(e) : 1;  // measured best on C5: U=4 records in flight, 64 registers, 4 CTAs/SM
+    v = e ? atoi(e) : 0;  // 0 = extents2; 1..4 = the round-1 grid-stride kernel (U=4, 64 registers, 4 CTAs/SM: 7.7 ms on C5)
   }
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   const unsigned g = (unsigned)std::min<u64>((n + 255) / 256, (u64)sms * 8);
+  if (v == 0) {  // extents2: contiguous warp ranges, one full wave of resident warps
+    static int per = 0;
+    if (!per) {
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, extents2_kernel<4>, 256, 0);
+      per = std::max(per, 1);
+    }
+    const u64 warps = (u64)sms * per * 8;
+    u64 rw = (n + warps - 1) / warps;
+    rw = std::max<u64>(128, (rw + 127) / 128 * 128);
+    const u64 nw = (n + rw - 1) / rw;
+    extents2_kernel<4><<<(unsigned)((nw + 7) / 8), 256, 0, st>>>(rec, (u32)n, log2G, (u32)rw, d_sum);
+    return;
+  }
   switch (v) {
     case 1: extents_kernel<256, 4, 4><<<g, 256, 0, st>>>(rec, n, log2G, d_sum); break;
     case 2: extents_kernel<256, 8, 2><<<g, 256, 0, st>>>(rec, n, log2G, d_sum); break;

@@ -114,7 +114,9 @@ u32 conflict_tiles(u64 m);
 
 // k_compact.cu — keep only entries of locations touched >= 2 times (order preserved); *total = count
 size_t compact_temp_bytes(u64 m);
-void launch_compact_multi(const u64* keys, u32 m, const KeyLayout& L, u64* out, void* temp, u32* total,
+// keys: sorted (m); seg: free buffer of m keys; out: where the result goes (may alias keys, which is dead after);
+// returns the array holding the m2 compacted keys (out, or seg for SESA_COMPACT=1)
+u64* launch_compact_multi(const u64* keys, u32 m, const KeyLayout& L, u64* seg, u64* out, void* temp, u32* total,
                           cudaStream_t st);
 
 // k_expand.cu — cells (block, interval slot, thread); descriptors of slot q are idx[ivoff[q] .. ivoff[q+1])

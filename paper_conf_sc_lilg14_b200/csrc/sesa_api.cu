@@ -302,12 +302,14 @@ bool sesa_trace::step_sort(u64 m, int* cur_out) {
 
 // step 4: keep entries of locations touched >= 2 times (into the other key buffer) -> (*comp, *m2)
 bool sesa_trace::step_compact(int cur, u64 m, u64** comp, u32* m2) {
-  *comp = (u64*)b_keys[cur ^ 1].p;
+  // the sorted keys are dead after compaction: the result is concatenated back into their buffer
+  *comp = (u64*)b_keys[cur].p;
   *m2 = 0;
   if (m == 0) return true;
   if (!grow(b_ctmp, compact_temp_bytes(m), "compact temp") || !grow(b_ctotal, 16, "compact count")) return false;
-  LAUNCH("compact", 16.0 * m, launch_compact_multi((const u64*)b_keys[cur].p, (u32)m, layout, *comp, b_ctmp.p,
-                                                   (u32*)b_ctotal.p, stream));
+  LAUNCH("compact", 8.0 * m, *comp = launch_compact_multi((const u64*)b_keys[cur].p, (u32)m, layout,
+                                                          (u64*)b_keys[cur ^ 1].p, (u64*)b_keys[cur].p, b_ctmp.p,
+                                                          (u32*)b_ctotal.p, stream));
   if (!cuda_ok(cudaMemcpyAsync(m2, b_ctotal.p, 4, cudaMemcpyDeviceToHost, stream), "compact count")) return false;
   if (!sync_check("compact")) return false;
   info.n_multi = *m2;
