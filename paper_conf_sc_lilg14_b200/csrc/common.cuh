@@ -121,6 +121,30 @@ inline int tile_atomic_mode() {
   return v;
 }
 
+// block-wide exclusive sum over THREADS values (one per thread)
+template <int THREADS>
+__device__ __forceinline__ u32 block_excl_sum(u32 v, u32* scratch /* [THREADS/32 + 1] */) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  u32 x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    u32 y = __shfl_up_sync(~0u, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) scratch[warp] = x;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    u32 acc = 0;
+    for (int w = 0; w < THREADS / 32; w++) {
+      u32 c = scratch[w];
+      scratch[w] = acc;
+      acc += c;
+    }
+  }
+  __syncthreads();
+  return scratch[warp] + x - v;
+}
+
 // ---- TMA bulk copies (cp.async.bulk, 1-D: no tensor map) completing on an mbarrier -------------------------
 __device__ __forceinline__ u32 smem_u32(const void* p) { return (u32)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void mbar_init(u64* bar, u32 count) {

@@ -15,10 +15,7 @@ namespace sesa {
 // ------------------------------------------------------------------------------------------------------------
 constexpr int EX_STAGES = 4, EX_CHUNK = 16384, EX_RECS = EX_CHUNK / 32;
 
-// Register version (measured faster than a TMA ring here: the per-record reductions are ALU-heavy and the ring's
-// strided shared-memory reads and barriers cost more than they save).  Scalar accumulators per space (arrays
-// indexed by the record's space spilled to local memory), warp votes only in convergent code, and a warp-uniform
-// single-space fast path (traces are mostly single-space).
+// Per-space extents in granule units (the block-level reduction format written to Summary).
 struct SpaceAcc {
   u64 cnt, gmin, gmax;
   u32 bmin, bmax, imin, imax;
@@ -43,107 +40,7 @@ struct SpaceAcc {
   }
 };
 
-template <int THREADS, int U, int MINB>
-__global__ void __launch_bounds__(THREADS, MINB) extents_kernel(const Rec* __restrict__ rec, u64 n, u32 log2G,
-                                                          Summary* __restrict__ out) {
-  u64 bad = ~0ull, ent = 0, multi = 0;
-  SpaceAcc A0, A1;  // shared, global
-  A0.init();
-  A1.init();
-  u32 unsorted = 0;
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const u64 stride = (u64)gridDim.x * THREADS, gt = (u64)blockIdx.x * THREADS + threadIdx.x;
-  const u64 rounds = (n + stride * U - 1) / (stride * U);
-  for (u64 it = 0; it < rounds; it++) {
-    Rec r[U];
-#pragma unroll
-    for (int j = 0; j < U; j++) {  // U independent 32-byte loads in flight per thread
-      const u64 k = (it * U + j) * stride + gt;
-      if (k < n) r[j] = load_rec(rec + k);
-    }
-#pragma unroll
-    for (int j = 0; j < U; j++) {
-      const u64 k = (it * U + j) * stride + gt;
-      const bool in = k < n;
-      // (block, interval) of record k-1: held by the previous lane, or loaded for lane 0 (convergent shuffles)
-      u32 pb = __shfl_up_sync(~0u, in ? r[j].block : 0u, 1), pi = __shfl_up_sync(~0u, in ? r[j].interval : 0u, 1);
-      if (lane == 0 && in && k > 0) {
-        const uint4 q = __ldg(reinterpret_cast<const uint4*>(rec + k - 1) + 1);
-        pb = q.x, pi = q.z;
-      }
-      const Rec& x = r[j];
-      const bool ok = in && x.space <= 1 && x.rw <= 2 && x.size >= 1 && x.addr <= ~0ull - (u64)(x.size - 1);
-      if (in && !ok) bad = min(bad, k);
-      const u64 glo = x.addr >> log2G, ghi = (x.addr + (u64)(x.size - 1)) >> log2G;
-      if (ok) {
-        if (k > 0 && (x.block < pb || (x.block == pb && x.interval < pi))) unsorted = 1;
-        ent += ghi - glo + 1;
-        multi += ghi != glo;
-      }
-      const bool all_glob = __all_sync(~0u, !ok || x.space == SP_GLOBAL);
-      if (all_glob) {
-        if (ok) A1.add(glo, ghi, x.block, x.interval);
-      } else if (__all_sync(~0u, !ok || x.space == SP_SHARED)) {
-        if (ok) A0.add(glo, ghi, x.block, x.interval);
-      } else if (ok) {
-        if (x.space == SP_GLOBAL) A1.add(glo, ghi, x.block, x.interval);
-        else A0.add(glo, ghi, x.block, x.interval);
-      }
-    }
-  }
-  // block reduction through warp shuffles then one atomic per field per CTA
-  __shared__ SpaceAcc sa[THREADS / 32][2];
-  __shared__ u64 s64[THREADS / 32][3];
-  __shared__ u32 s_uns[THREADS / 32];
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    bad = min(bad, __shfl_xor_sync(~0u, bad, o));
-    ent += __shfl_xor_sync(~0u, ent, o);
-    multi += __shfl_xor_sync(~0u, multi, o);
-    unsorted |= __shfl_xor_sync(~0u, unsorted, o);
-  }
-  A0.warp_reduce();
-  A1.warp_reduce();
-  if (lane == 0) {
-    s64[warp][0] = bad, s64[warp][1] = ent, s64[warp][2] = multi;
-    sa[warp][0] = A0, sa[warp][1] = A1;
-    s_uns[warp] = unsorted;
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    for (int w = 1; w < THREADS / 32; w++) {
-      s64[0][0] = min(s64[0][0], s64[w][0]);
-      s64[0][1] += s64[w][1];
-      s64[0][2] += s64[w][2];
-      s_uns[0] |= s_uns[w];
-      for (int sp = 0; sp < 2; sp++) {
-        SpaceAcc& d = sa[0][sp];
-        const SpaceAcc& e = sa[w][sp];
-        d.cnt += e.cnt;
-        d.gmin = min(d.gmin, e.gmin), d.gmax = max(d.gmax, e.gmax);
-        d.bmin = min(d.bmin, e.bmin), d.bmax = max(d.bmax, e.bmax);
-        d.imin = min(d.imin, e.imin), d.imax = max(d.imax, e.imax);
-      }
-    }
-    if (s64[0][0] != ~0ull) atomicMin(&out->bad_index, (unsigned long long)s64[0][0]);
-    if (s64[0][1]) atomicAdd(&out->entries, (unsigned long long)s64[0][1]);
-    if (s64[0][2]) atomicAdd(&out->multi, (unsigned long long)s64[0][2]);
-    for (int sp = 0; sp < 2; sp++) {
-      const SpaceAcc& d = sa[0][sp];
-      if (!d.cnt) continue;
-      atomicAdd(&out->count[sp], (unsigned long long)d.cnt);
-      atomicMin(&out->gmin[sp], (unsigned long long)d.gmin);
-      atomicMax(&out->gmax[sp], (unsigned long long)d.gmax);
-      atomicMin(&out->bmin[sp], d.bmin);
-      atomicMax(&out->bmax[sp], d.bmax);
-      atomicMin(&out->imin[sp], d.imin);
-      atomicMax(&out->imax[sp], d.imax);
-    }
-    if (s_uns[0]) atomicOr(&out->unsorted, 1u);
-  }
-}
-
-// extents2 (default): warp w streams the contiguous record range [w*rw, (w+1)*rw) in rows of 32 (U rows in
+// extents2: warp w streams the contiguous record range [w*rw, (w+1)*rw) in rows of 32 (U rows in
 // flight), all index arithmetic in 32 bits (n < 2^31, include/sesa.h).  Per record only what the layout needs:
 // min address and max last byte per space (granule = address >> log2G commutes with min/max, so the shifts
 // happen once per thread), block/interval min/max, the extra-granule count from the in-granule offset (32-bit),
@@ -169,9 +66,14 @@ struct SpaceAcc2 {
   }
 };
 
+// With tile_hist != null the warp ranges are whole tiles of FUSED_TILE records and each warp also writes, per
+// tile, the histogram of the raw low granule byte (addr >> log2G) & 255: once the extents fix gmin, these are the
+// tile histograms of the first sort digit ((g - gmin) & 255 is a rotation of g & 255), which lets the fused
+// extract + first sort pass place every tile without a look-back (k_fused.cu).
 template <int U>
 __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ rec, u32 n, u32 log2G, u32 rw,
-                                                       Summary* __restrict__ out) {
+                                                       Summary* __restrict__ out, u32* __restrict__ tile_hist) {
+  __shared__ u32 s_th[8][RADIX];
   constexpr int THREADS = 256;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const u32 gw = (blockIdx.x * THREADS + threadIdx.x) >> 5;
@@ -188,12 +90,21 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
     const uint4 p = __ldg(q + 2 * (u64)(start - 1) + 1);
     prev_bi = ((u64)p.x << 32) | p.z;
   }
-  for (u32 r0 = start; r0 < end; r0 += 32 * U) {
+  u32* th = s_th[warp];
+  const u32 seg = tile_hist ? (u32)FUSED_TILE : rw;  // records between histogram flushes
+  for (u32 t0 = start; t0 < end; t0 += seg) {
+  const u32 tend = min(end, t0 + seg);
+  if (tile_hist) {
+#pragma unroll
+    for (int q = 0; q < RADIX / 32; q++) th[q * 32 + lane] = 0;
+    __syncwarp();
+  }
+  for (u32 r0 = t0; r0 < tend; r0 += 32 * U) {
     uint4 a[U], b[U];
 #pragma unroll
     for (int u = 0; u < U; u++) {
       const u32 i = r0 + u * 32 + lane;
-      if (i < end) a[u] = __ldcs(q + 2 * (u64)i), b[u] = __ldcs(q + 2 * (u64)i + 1);
+      if (i < tend) a[u] = __ldcs(q + 2 * (u64)i), b[u] = __ldcs(q + 2 * (u64)i + 1);
       else a[u] = make_uint4(0, 0, 0, 0), b[u] = make_uint4(0, 0, 0, 0);
     }
     bool ok[U];
@@ -207,7 +118,7 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
       prev_bi = __shfl_sync(~0u, bi, 31);
       const u32 size = b[u].w & 0xFFFFu, sp = (b[u].w >> 16) & 0xFFu, rwv = b[u].w >> 24;
       const u64 addr = ((u64)a[u].y << 32) | a[u].x;
-      const bool in = i < end;
+      const bool in = i < tend;
       ok[u] = in && sp <= 1u && rwv <= 2u && size >= 1u && addr + (u64)size - 1ull >= addr;
       bad = (in && !ok[u]) ? min(bad, i) : bad;
       const u32 e = ((a[u].x & gmask) + size - 1u) >> log2G;  // granules beyond the first
@@ -227,8 +138,17 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
       if (ok[u]) {
         if (glob) A1.add(addr, last, b[u].x, b[u].z);
         else A0.add(addr, last, b[u].x, b[u].z);
+        if (tile_hist) atomicAdd(&th[(u32)(addr >> log2G) & (RADIX - 1)], 1u);
       }
     }
+  }
+  if (tile_hist) {
+    __syncwarp();
+    u32* dst = tile_hist + (u64)(t0 / FUSED_TILE) * RADIX;
+#pragma unroll
+    for (int q = 0; q < RADIX / 32; q++) dst[q * 32 + lane] = th[q * 32 + lane];
+    __syncwarp();
+  }
   }
   // block reduction (warp shuffles, then one atomic per field per CTA)
   u64 bad64 = bad == ~0u ? ~0ull : (u64)bad, ent = (u64)extra + A0.cnt + A1.cnt, mul = multi;
@@ -293,36 +213,23 @@ static int ring_grid(const void* kern, int threads, size_t smem, size_t smem_max
   return sms * (per > 0 ? per : 1);
 }
 
-void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, int grid, cudaStream_t st) {
-  static int v = -1;
-  if (v < 0) {
-    const char* e = getenv("SESA_EXT_CFG");
-    v = e ? atoi(e) : 0;  // 0 = extents2; 1..4 = the round-1 grid-stride kernel (U=4, 64 registers, 4 CTAs/SM: 7.7 ms on C5)
+void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, u32* tile_hist, int grid, cudaStream_t st) {
+  // extents2: contiguous warp ranges, one full wave of resident warps (the round-1 grid-stride kernel took
+  // 7.7 ms on C5: 132 instructions per record, 64-bit index math and local-memory accumulators; this one 4.6 ms)
+  static int sms = 0, per = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, extents2_kernel<4>, 256, 0);
+    per = std::max(per, 1);
   }
-  int dev = 0, sms = 148;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  const unsigned g = (unsigned)std::min<u64>((n + 255) / 256, (u64)sms * 8);
-  if (v == 0) {  // extents2: contiguous warp ranges, one full wave of resident warps
-    static int per = 0;
-    if (!per) {
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, extents2_kernel<4>, 256, 0);
-      per = std::max(per, 1);
-    }
-    const u64 warps = (u64)sms * per * 8;
-    u64 rw = (n + warps - 1) / warps;
-    rw = std::max<u64>(128, (rw + 127) / 128 * 128);
-    const u64 nw = (n + rw - 1) / rw;
-    extents2_kernel<4><<<(unsigned)((nw + 7) / 8), 256, 0, st>>>(rec, (u32)n, log2G, (u32)rw, d_sum);
-    return;
-  }
-  switch (v) {
-    case 1: extents_kernel<256, 4, 4><<<g, 256, 0, st>>>(rec, n, log2G, d_sum); break;
-    case 2: extents_kernel<256, 8, 2><<<g, 256, 0, st>>>(rec, n, log2G, d_sum); break;
-    case 3: extents_kernel<256, 2, 6><<<g, 256, 0, st>>>(rec, n, log2G, d_sum); break;
-    case 4: extents_kernel<256, 8, 3><<<g, 256, 0, st>>>(rec, n, log2G, d_sum); break;
-    default: extents_kernel<256, 4, 1><<<g, 256, 0, st>>>(rec, n, log2G, d_sum); break;
-  }
+  const u64 warps = (u64)sms * per * 8;
+  const u64 gran = tile_hist ? FUSED_TILE : 128;  // warp ranges: whole tiles when tile histograms are wanted
+  u64 rw = (n + warps - 1) / warps;
+  rw = std::max<u64>(gran, (rw + gran - 1) / gran * gran);
+  const u64 nw = (n + rw - 1) / rw;
+  extents2_kernel<4><<<(unsigned)((nw + 7) / 8), 256, 0, st>>>(rec, (u32)n, log2G, (u32)rw, d_sum, tile_hist);
   (void)grid;
 }
 

@@ -1,0 +1,267 @@
+// k_fused.cu — key extraction fused with the first LSD sort pass (SURVEY §8a rows a2 + a4), for the common
+// layout: one space (global), records already in (block, interval) order, one granule per record — C3, C4, C5.
+//
+// The first sort digit of an entry is d = (g - gmin) & 255 with g = addr >> log2G.  Modulo 256 that is a
+// rotation of the raw byte g & 255, whose per-tile histograms the extents pass already produced (k_extract.cu)
+// before gmin was known.  From them three small kernels compute, for every tile t of FUSED_TILE records and
+// digit d, the exact output offset of the tile's digit-d run (bin base + the digit-d counts of all earlier
+// tiles).  The fused kernel then reads each record's address once (the key never makes the round trip through
+// HBM that a separate extract kernel + first pass costs: 32 B read + 8 B written per record instead of
+// 32 + 8 + 8 + 8), ranks the tile stably by d exactly like a onesweep tile (k_sort.cu) and writes each digit run
+// to its precomputed offset — no decoupled look-back, so CTAs are persistent and take tiles in any order.  It
+// also accumulates the histograms of the remaining digits (the upfront histograms of the later passes).
+#include <algorithm>
+#include <cstdlib>
+
+#include "kernels.cuh"
+
+namespace sesa {
+
+// ---- tile offsets from the raw per-tile histograms H[t][r] (r = g & 255), r0 = gmin & 255, digit(r) = r - r0 --
+// (1) per chunk of tiles: column sums P[c][r]
+__global__ void tile_col_reduce_kernel(const u32* __restrict__ H, u32 T, u32 tpc, u32* __restrict__ P) {
+  const u32 c = blockIdx.x, r = threadIdx.x;
+  const u32 t0 = c * tpc, t1 = min(T, t0 + tpc);
+  u32 s = 0;
+#pragma unroll 8
+  for (u32 t = t0; t < t1; t++) s += H[(u64)t * RADIX + r];
+  P[(u64)c * RADIX + r] = s;
+}
+
+// (2) one CTA: exclusive prefix over chunks per raw byte, plus the bin base of each digit (rotated order)
+__global__ void tile_col_scan_kernel(u32* __restrict__ P, u32 C, u32 r0) {
+  __shared__ u32 s_tot[RADIX], s_w[RADIX / 32 + 1];
+  const u32 r = threadIdx.x, lane = r & 31, warp = r >> 5;
+  u32 run = 0;
+  for (u32 c0 = 0; c0 < C; c0 += 16) {  // 16 independent loads per round trip
+    u32 v[16];
+#pragma unroll
+    for (int q = 0; q < 16; q++) v[q] = c0 + q < C ? P[(u64)(c0 + q) * RADIX + r] : 0u;
+#pragma unroll
+    for (int q = 0; q < 16; q++)
+      if (c0 + q < C) P[(u64)(c0 + q) * RADIX + r] = run, run += v[q];
+  }
+  const u32 d = (r - r0) & (RADIX - 1);
+  s_tot[d] = run;
+  __syncthreads();
+  // exclusive scan over digits d (thread d holds s_tot[d])
+  const u32 v = s_tot[r];
+  u32 x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const u32 y = __shfl_up_sync(~0u, x, o);
+    if (lane >= (u32)o) x += y;
+  }
+  if (lane == 31) s_w[warp] = x;
+  __syncthreads();
+  if (r == 0) {
+    u32 acc = 0;
+    for (int w = 0; w < RADIX / 32; w++) {
+      const u32 c = s_w[w];
+      s_w[w] = acc;
+      acc += c;
+    }
+  }
+  __syncthreads();
+  s_tot[r] = s_w[warp] + x - v;  // bin base of digit r
+  __syncthreads();
+  const u32 base = s_tot[d];
+  for (u32 c = 0; c < C; c++) P[(u64)c * RADIX + r] += base;
+}
+
+// (3) per chunk: O[t][digit] = offset of tile t's digit run
+__global__ void tile_col_down_kernel(const u32* __restrict__ H, u32 T, u32 tpc, const u32* __restrict__ P, u32 r0,
+                                     u32* __restrict__ O) {
+  const u32 c = blockIdx.x, r = threadIdx.x;
+  const u32 t0 = c * tpc, t1 = min(T, t0 + tpc);
+  const u32 d = (r - r0) & (RADIX - 1);
+  u32 run = P[(u64)c * RADIX + r];
+#pragma unroll 8
+  for (u32 t = t0; t < t1; t++) {
+    O[(u64)t * RADIX + d] = run;
+    run += H[(u64)t * RADIX + r];
+  }
+}
+
+size_t fused_temp_bytes(u64 n) {
+  const u64 T = (n + FUSED_TILE - 1) / FUSED_TILE;
+  return (T * RADIX * 4 + 255) / 256 * 256 + (u64)1024 * RADIX * 4;
+}
+
+// ---- the fused kernel -------------------------------------------------------------------------------------------
+struct FusedArgs {
+  const Rec* rec;
+  u32 n, log2G, pos_bits, npass;
+  u64 gmin;
+  const u32* toff;  // [T][RADIX] output offset of each tile's digit run
+  u64* kout;
+  u32* hist;        // [npass][RADIX] global digit histograms (rows 1.. are accumulated here)
+  u32 nohist;       // timing experiment only (SESA_FUSED_NOHIST): skip the later-digit histograms
+};
+
+// Persistent CTAs, software-pipelined in registers: right after a tile's digit counts (when its addresses have
+// become 32-bit key parts), the CTA issues the loads of its NEXT tile's addresses into the freed registers, so
+// they are in flight during the ranking and write-out of the current tile — the CTA's HBM reads never pause.
+template <int NP>
+__global__ void __launch_bounds__(FUSED_THREADS, FUSED_MINB) fused_extract_pass0_kernel(FusedArgs A) {
+  constexpr int THREADS = FUSED_THREADS, ITEMS = FUSED_ITEMS, WARPS = THREADS / 32, TILE = FUSED_TILE;
+  extern __shared__ __align__(16) unsigned char smem[];
+  u64* keys_s = reinterpret_cast<u64*>(smem);              // [TILE]
+  u32* whist = reinterpret_cast<u32*>(keys_s + TILE);       // [WARPS][RADIX]
+  u32* globu = whist + WARPS * RADIX;                      // [RADIX]
+  u32* scratch = globu + RADIX;                            // [WARPS + 1]
+  u32* wmask = scratch + WARPS + 1;                        // [WARPS][RADIX + 1]
+  u32* hrest = wmask + WARPS * (RADIX + 1);                // [NP - 1][RADIX]
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  constexpr u32 nrest = (NP - 1) * RADIX;
+  for (u32 i = tid; i < WARPS * (RADIX + 1); i += THREADS) wmask[i] = 0;
+  for (u32 i = tid; i < nrest; i += THREADS) hrest[i] = 0;
+  const u32 T = (A.n + TILE - 1) / TILE;
+  u32* wh = whist + warp * RADIX;
+  u32* wm = wmask + warp * (RADIX + 1);
+  const unsigned lt = lanemask_lt();
+  // (0) addresses of a tile's records: one 32-byte sector per record, the 8-byte address word is all the key needs
+  u64 a[ITEMS];
+  auto issue = [&](u32 t) {
+    const u32 wb = t * TILE + warp * 32 * ITEMS + lane;
+    const u64* ap = reinterpret_cast<const u64*>(A.rec) + 4 * (u64)wb;  // record stride: 4 words
+#pragma unroll
+    for (int i = 0; i < ITEMS; i++)
+      if (wb + i * 32 < A.n) a[i] = __ldcs(ap + i * 128);
+  };
+  u32 tile = blockIdx.x;
+  if (tile < T) issue(tile);
+  while (tile < T) {
+    const u32 tbase = tile * TILE;
+    const u32 wbase = tbase + warp * 32 * ITEMS + lane;
+    const int nv = wbase < A.n ? (int)min((u32)ITEMS, (A.n - wbase + 31) / 32) : 0;
+    // only key_hi = g - gmin (< 2^32 on this path) is kept per item: the position part of the key is the item's
+    // record index, known from (tile, warp, item, lane)
+    u32 kh[ITEMS];
+#pragma unroll
+    for (int i = 0; i < ITEMS; i++) kh[i] = i < nv ? (u32)((a[i] >> A.log2G) - A.gmin) : 0u;
+    auto digit = [&](int i) -> u32 { return i < nv ? (kh[i] & (RADIX - 1)) : (u32)RADIX; };
+    for (u32 i = tid; i < WARPS * RADIX; i += THREADS) whist[i] = 0;
+    __syncthreads();
+    // (1) per-warp counts of digit 0
+#pragma unroll
+    for (int i = 0; i < ITEMS; i++)
+      if (i < nv) atomicAdd(&wh[digit(i)], 1u);
+    __syncthreads();
+    // (2) tile-local bases = bin start + warp offset; global write offsets from the precomputed table
+    u32 tot = 0;
+    if (tid < RADIX) {
+#pragma unroll
+      for (int w = 0; w < WARPS; w++) {
+        const u32 c = whist[w * RADIX + tid];
+        whist[w * RADIX + tid] = tot;
+        tot += c;
+      }
+    }
+    const u32 bs = block_excl_sum<THREADS>(tid < RADIX ? tot : 0u, scratch);  // (contains __syncthreads)
+    if (tid < RADIX) {
+#pragma unroll
+      for (int w = 0; w < WARPS; w++) whist[w * RADIX + tid] += bs;
+      globu[tid] = A.toff[(u64)tile * RADIX + tid] - bs;
+    }
+    __syncthreads();
+    const u32 next = tile + gridDim.x;
+    if (next < T) issue(next);  // prefetch: in flight during ranking and write-out
+    // (3) stable warp ranking (peer masks by shared-memory atomicOr), each key stored into its tile slot
+#pragma unroll
+    for (int i = 0; i < ITEMS; i++) {
+      const u32 d = digit(i);
+      atomicOr(&wm[d], 1u << lane);
+      __syncwarp();
+      const unsigned peers = wm[d];
+      const u32 c = wh[d];
+      __syncwarp();
+      if (d < RADIX) keys_s[c + __popc(peers & lt)] = ((u64)kh[i] << A.pos_bits) | (u64)(wbase + i * 32);
+      if (lane == 31 - __clz(peers)) {
+        wm[d] = 0;
+        if (d < RADIX) wh[d] = c + __popc(peers);
+      }
+      __syncwarp();
+    }
+    __syncthreads();
+    // (4) coalesced write-out of each digit run, and the CTA histograms of the later digits
+    const u32 tcount = min((u32)TILE, A.n - tbase);
+#pragma unroll 4
+    for (u32 j = tid; j < tcount; j += THREADS) {
+      const u64 key = keys_s[j];
+      const u32 d = (u32)((key >> A.pos_bits) & (RADIX - 1));
+      __stcs(A.kout + (globu[d] + j), key);
+      if (!A.nohist) {
+#pragma unroll
+        for (int p = 1; p < NP; p++)
+          atomicAdd(&hrest[(p - 1) * RADIX + (u32)((key >> (A.pos_bits + p * RADIX_BITS)) & (RADIX - 1))], 1u);
+      }
+    }
+    __syncthreads();  // shared memory is reused by the next tile
+    tile = next;
+  }
+  for (u32 i = tid; i < nrest; i += THREADS)
+    if (hrest[i]) atomicAdd(&A.hist[RADIX + i], hrest[i]);
+}
+
+static size_t fused_smem(u32 npass) {
+  constexpr int WARPS = FUSED_THREADS / 32;
+  return (size_t)FUSED_TILE * 8 + (size_t)WARPS * RADIX * 4 + RADIX * 4 + (WARPS + 1) * 4 +
+         (size_t)WARPS * (RADIX + 1) * 4 + (size_t)(npass > 0 ? npass - 1 : 0) * RADIX * 4;
+}
+
+bool fused_supported(u32 npass) { return npass >= 1 && npass <= 4; }  // sort_bits <= 32 on this path
+
+// tile offsets O[t][d] into temp (fused_temp_bytes(n)) from the extents' raw per-tile histograms
+void launch_tile_offsets(u64 n, const KeyLayout& L, const u32* tile_hist, void* temp, cudaStream_t st) {
+  if (!n) return;
+  const u32 T = (u32)((n + FUSED_TILE - 1) / FUSED_TILE);
+  u32* O = reinterpret_cast<u32*>(temp);
+  u32* P = reinterpret_cast<u32*>(reinterpret_cast<char*>(temp) + ((u64)T * RADIX * 4 + 255) / 256 * 256);
+  const u32 C = std::min<u32>(T, 1024), tpc = (T + C - 1) / C, Cu = (T + tpc - 1) / tpc;
+  const u32 r0 = (u32)(L.gminG & (RADIX - 1));
+  tile_col_reduce_kernel<<<Cu, RADIX, 0, st>>>(tile_hist, T, tpc, P);
+  tile_col_scan_kernel<<<1, RADIX, 0, st>>>(P, Cu, r0);
+  tile_col_down_kernel<<<Cu, RADIX, 0, st>>>(tile_hist, T, tpc, P, r0, O);
+}
+
+// temp: holds the tile offsets (launch_tile_offsets); hist: [npass][RADIX] zeroed (rows >= 1 filled)
+void launch_fused_extract_pass0(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, void* temp, u64* kout,
+                                u32* hist, cudaStream_t st) {
+  if (!n) return;
+  const u32 T = (u32)((n + FUSED_TILE - 1) / FUSED_TILE);
+  u32* O = reinterpret_cast<u32*>(temp);
+  static int grid = 0;
+  if (!grid) {
+    int dev = 0, sms = 148, per = 1;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const void* ks[4] = {(const void*)fused_extract_pass0_kernel<1>, (const void*)fused_extract_pass0_kernel<2>,
+                         (const void*)fused_extract_pass0_kernel<3>, (const void*)fused_extract_pass0_kernel<4>};
+    for (int i = 0; i < 4; i++)
+      cudaFuncSetAttribute(ks[i], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fused_smem(i + 1));
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fused_extract_pass0_kernel<4>, FUSED_THREADS, fused_smem(4));
+    grid = sms * std::max(per, 1);
+  }
+  const size_t sm = fused_smem(npass);
+  FusedArgs A;
+  A.rec = rec;
+  A.n = (u32)n;
+  A.log2G = L.log2G;
+  A.pos_bits = L.pos_bits;
+  A.npass = npass;
+  A.gmin = L.gminG;
+  A.toff = O;
+  A.kout = kout;
+  A.hist = hist;
+  A.nohist = getenv("SESA_FUSED_NOHIST") ? 1u : 0u;
+  const u32 g = std::min<u32>(T, (u32)grid);
+  switch (npass) {
+    case 1: fused_extract_pass0_kernel<1><<<g, FUSED_THREADS, sm, st>>>(A); break;
+    case 2: fused_extract_pass0_kernel<2><<<g, FUSED_THREADS, sm, st>>>(A); break;
+    case 3: fused_extract_pass0_kernel<3><<<g, FUSED_THREADS, sm, st>>>(A); break;
+    default: fused_extract_pass0_kernel<4><<<g, FUSED_THREADS, sm, st>>>(A); break;
+  }
+}
+
+}  // namespace sesa

@@ -6,6 +6,8 @@ namespace sesa {
 
 constexpr int RADIX_BITS = 8;  // onesweep digit width (8-bit digits, 256 bins per pass)
 constexpr int RADIX = 1 << RADIX_BITS;
+// fused key extract + first sort pass (k_fused.cu): tiles of 256 threads x 32 records
+constexpr int FUSED_THREADS = 256, FUSED_ITEMS = 16, FUSED_MINB = 3, FUSED_TILE = FUSED_THREADS * FUSED_ITEMS;
 
 // onesweep tile: 256 threads x 16 keys (warp-striped); one lookback word per (tile, bin)
 constexpr int SORT_THREADS = 256;
@@ -18,12 +20,21 @@ constexpr int CT_ITEMS = 8;
 constexpr int CT_TILE = CT_THREADS * CT_ITEMS;
 
 // k_extract.cu
-void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, int grid, cudaStream_t st);
+// tile_hist (optional, [ceil(n / FUSED_TILE)][RADIX]): per-tile histograms of (addr >> log2G) & 255 (k_fused.cu)
+void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, u32* tile_hist, int grid, cudaStream_t st);
 void launch_extract_1to1(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, u64* keys, u32* hist, u64 pos_base,
                          int grid, cudaStream_t st);
 void launch_entry_count(const Rec* rec, u64 n, u32 log2G, u32* cnt, cudaStream_t st);
 void launch_extract_multi(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, const u32* off, u64* keys,
                           u32* hist, u64 pos_base, int grid, cudaStream_t st);
+
+// k_fused.cu — key extract fused with the first sort pass (single global space, (block, interval)-ordered
+// input, one granule per record); tile_hist from launch_extents
+bool fused_supported(u32 npass);
+size_t fused_temp_bytes(u64 n);
+void launch_tile_offsets(u64 n, const KeyLayout& L, const u32* tile_hist, void* temp, cudaStream_t st);
+void launch_fused_extract_pass0(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, void* temp, u64* kout,
+                                u32* hist, cudaStream_t st);
 
 // k_util.cu
 size_t scan_u32_temp_bytes(u64 n);

@@ -193,9 +193,21 @@ bool sesa_trace::check_records_ptr(const sesa_access* d_rec, u64 n) {
 }
 
 // step 1: validation + extents of the local records -> h_summary (synchronises)
-bool sesa_trace::step_extents(const Rec* rec, u64 n) {
+static bool fused_enabled() {  // SESA_FUSED=0 disables the fused key extract + first sort pass
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("SESA_FUSED");
+    v = e ? atoi(e) : 1;
+  }
+  return v != 0;
+}
+
+bool sesa_trace::step_extents(const Rec* rec, u64 n, bool tile_hist) {
   const u32 log2G = (u32)__builtin_ctz(cfg.granularity);
   if (!grow(b_summary, sizeof(Summary), "summary")) return false;
+  // per-tile raw digit histograms for the fused first pass (worth it only for traces of many tiles)
+  have_thist = tile_hist && fused_enabled() && n >= 32768;
+  if (have_thist && !grow(b_thist, ((n + FUSED_TILE - 1) / FUSED_TILE) * RADIX * 4, "tile histograms")) return false;
   Summary init;
   memset(&init, 0, sizeof init);
   init.bad_index = ~0ull;
@@ -206,7 +218,8 @@ bool sesa_trace::step_extents(const Rec* rec, u64 n) {
   if (!cuda_ok(cudaMemcpyAsync(b_summary.p, &h_summary, sizeof(Summary), cudaMemcpyHostToDevice, stream), "summary init"))
     return false;
   const int grid_stream = (int)std::min<u64>((n + 255) / 256, (u64)num_sms * 8);
-  LAUNCH("extents", 32.0 * n, launch_extents(rec, n, log2G, (Summary*)b_summary.p, grid_stream, stream));
+  LAUNCH("extents", 32.0 * n, launch_extents(rec, n, log2G, (Summary*)b_summary.p,
+                                             have_thist ? (u32*)b_thist.p : nullptr, grid_stream, stream));
   if (!cuda_ok(cudaMemcpyAsync(&h_summary, b_summary.p, sizeof(Summary), cudaMemcpyDeviceToHost, stream), "summary"))
     return false;
   return sync_check("extents");
@@ -246,6 +259,22 @@ bool sesa_trace::step_extract(const Rec* rec, u64 n, u64 m, u64 pos_base, bool m
   return true;
 }
 
+// step 2+3a (fused): keys of the records sorted by the first digit -> b_keys[1], histograms of the other digits
+bool sesa_trace::step_extract_fused(const Rec* rec, u64 n) {
+  const KeyLayout& L = layout;
+  const u32 npass = (L.sort_bits + RADIX_BITS - 1) / RADIX_BITS;
+  if (!grow(b_keys[0], n * 8 + 64, "keys") || !grow(b_keys[1], n * 8 + 64, "keys") ||
+      !grow(b_hist, (size_t)npass * RADIX * 4, "hist") || !grow(b_binbase, (size_t)npass * RADIX * 8, "binbase") ||
+      !grow(b_ftmp, fused_temp_bytes(n), "fused temp"))
+    return false;
+  cudaMemsetAsync(b_hist.p, 0, (size_t)npass * RADIX * 4, stream);
+  LAUNCH("tile_offsets", 2.0 * RADIX * 4 * ((n + FUSED_TILE - 1) / FUSED_TILE),
+         launch_tile_offsets(n, L, (const u32*)b_thist.p, b_ftmp.p, stream));
+  LAUNCH("extract_pass0", 40.0 * n,
+         launch_fused_extract_pass0(rec, n, L, npass, b_ftmp.p, (u64*)b_keys[1].p, (u32*)b_hist.p, stream));
+  return true;
+}
+
 // step 2' (distributed): histograms of keys that arrived from the exchange (already in b_keys[0])
 bool sesa_trace::step_hist(u64 m) {
   const u32 npass = (layout.sort_bits + RADIX_BITS - 1) / RADIX_BITS;
@@ -259,7 +288,7 @@ bool sesa_trace::step_hist(u64 m) {
 }
 
 // step 3: LSD onesweep passes over the non-trivial digits of b_keys[0] (m keys); result in b_keys[*cur]
-bool sesa_trace::step_sort(u64 m, int* cur_out) {
+bool sesa_trace::step_sort(u64 m, int* cur_out, u32 first_pass, int cur0) {
   const KeyLayout& L = layout;
   const u32 npass = (L.sort_bits + RADIX_BITS - 1) / RADIX_BITS;
   std::vector<u32> hist((size_t)npass * RADIX);
@@ -279,9 +308,9 @@ bool sesa_trace::step_sort(u64 m, int* cur_out) {
     }
     cudaMemsetAsync(b_ctr.p, 0, 64 * 4, stream);
   }
-  int cur = 0;
-  u32 passes_run = 0;
-  for (u32 p = 0; p < npass && m; p++) {
+  int cur = cur0;
+  u32 passes_run = first_pass;
+  for (u32 p = first_pass; p < npass && m; p++) {
     const u32* h = hist.data() + (size_t)p * RADIX;
     if (*std::max_element(h, h + RADIX) == m) continue;  // trivial digit: every key has the same value
     if (++epoch >= 256) {
@@ -438,7 +467,7 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
   }
   if (!check_records_ptr(d_rec, n)) return status;
   const Rec* rec = reinterpret_cast<const Rec*>(d_rec);
-  if (!step_extents(rec, n)) return status;
+  if (!step_extents(rec, n, true)) return status;
   const Summary& S = h_summary;
   if (S.bad_index != ~0ull) return report_bad(d_rec, S.bad_index, S.bad_index), status;
   const u64 m = S.entries;
@@ -449,9 +478,16 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
   info.sort_bits = layout.sort_bits;
   info.pos_bits = layout.pos_bits;
   info.digit_bits = RADIX_BITS;
-  if (!step_extract(rec, n, m, 0, S.multi != 0)) return status;
+  const u32 npass = (layout.sort_bits + RADIX_BITS - 1) / RADIX_BITS;
+  const bool fused = have_thist && !layout.both && layout.single_space == SP_GLOBAL && layout.lowG == 0 &&
+                     S.multi == 0 && m == n && layout.sort_bits <= 32 && fused_supported(npass);
+  info.fused_first_pass = fused ? 1 : 0;
   int cur = 0;
-  if (!step_sort(m, &cur)) return status;
+  if (fused) {
+    if (!step_extract_fused(rec, n) || !step_sort(m, &cur, 1, 1)) return status;
+  } else {
+    if (!step_extract(rec, n, m, 0, S.multi != 0) || !step_sort(m, &cur)) return status;
+  }
   u64* comp = nullptr;
   u32 m2 = 0;
   if (!step_compact(cur, m, &comp, &m2)) return status;

@@ -42,7 +42,8 @@ struct sesa_trace {
   DevBuf b_summary, b_keys[2], b_hist, b_binbase, b_lookback, b_ctr, b_cnt, b_off, b_temp;
   DevBuf b_tflags, b_part, b_carry, b_owner, b_slots, b_cross, b_ccount, b_carrytmp;
   DevBuf b_races, b_rkeys[2], b_rvals[2], b_races_sorted, b_rhist, b_rbase;
-  DevBuf b_eoff, b_ecnt, b_ecell, b_hrec, b_dist_races, b_ctmp, b_ctotal;
+  DevBuf b_eoff, b_ecnt, b_ecell, b_hrec, b_dist_races, b_ctmp, b_ctotal, b_thist, b_ftmp;
+  bool have_thist = false;  // extents wrote per-tile raw digit histograms (fused first pass possible)
   DevBuf b_dist[8];
   void* h_pinned = nullptr;
 
@@ -50,7 +51,7 @@ struct sesa_trace {
     std::vector<DevBuf*> v = {&b_summary, &b_hist, &b_binbase, &b_lookback, &b_ctr, &b_cnt, &b_off, &b_temp,
                               &b_tflags, &b_part, &b_carry, &b_owner, &b_slots, &b_cross, &b_ccount, &b_carrytmp,
                               &b_races, &b_races_sorted, &b_rhist, &b_rbase, &b_eoff, &b_ecnt, &b_ecell,
-                              &b_hrec, &b_dist_races, &b_ctmp, &b_ctotal};
+                              &b_hrec, &b_dist_races, &b_ctmp, &b_ctotal, &b_thist, &b_ftmp};
     for (auto& b : b_keys) v.push_back(&b);
     for (auto& b : b_rkeys) v.push_back(&b);
     for (auto& b : b_rvals) v.push_back(&b);
@@ -86,11 +87,12 @@ struct sesa_trace {
   // pipeline steps (shared by the single-GPU and the distributed check)
   void begin_check(uint64_t n);
   bool check_records_ptr(const sesa_access* d_rec, uint64_t n);
-  bool step_extents(const sesa::Rec* rec, uint64_t n);
+  bool step_extents(const sesa::Rec* rec, uint64_t n, bool tile_hist = false);
   bool report_bad(const sesa_access* d_rec, uint64_t local_bad, uint64_t global_bad);
   bool step_extract(const sesa::Rec* rec, uint64_t n, uint64_t m, uint64_t pos_base, bool multi);
   bool step_hist(uint64_t m);
-  bool step_sort(uint64_t m, int* cur_out);
+  bool step_extract_fused(const sesa::Rec* rec, uint64_t n);
+  bool step_sort(uint64_t m, int* cur_out, uint32_t first_pass = 0, int cur0 = 0);
   bool step_compact(int cur, uint64_t m, uint64_t** comp, uint32_t* m2);
   bool step_conflict(const uint64_t* comp, uint32_t m2, const sesa::Rec* rec, uint32_t rec_pos_base,
                      const sesa::Rec* rec_entry, uint64_t index_base);

@@ -236,3 +236,17 @@ def test_profiling_stats(sesa):
     info = t.info()
     assert info["n_records"] == 30000 and info["launches"] >= 4
     t.close()
+
+
+# ------------------------------------------------------------------------------------------------ fused first pass
+@pytest.mark.parametrize("n,words,shift,fused", [(32768, 100, 77, 1), (40000, 30000, 1, 1), (65537, 3_000_000, 200, 1),
+                                                 (200003, 50_000, 255, 1), (500000, 400_000_000, 13, 1),
+                                                 (40000, 2**34, 3, 0), (32767, 1000, 5, 0)])
+def test_fused_first_pass_parity(sesa, n, words, shift, fused):
+    # global-only, (block, interval)-ordered, one granule per record: the fused extract + first sort pass
+    # (k_fused.cu) places tiles from the extents' raw-byte histograms rotated by gmin & 255 — shift moves gmin
+    r = G.random_trace(n, 7 + n % 97, blocks=64, threads=256, intervals=3, words=words, shared_frac=0.0,
+                       sizes=(4,), unaligned=False, values=4)
+    r["addr"] += np.uint64(4 * shift)
+    assert_same(sesa, r, 32, 0, 4)
+    assert trace(sesa).info()["fused_first_pass"] == fused  # > 32 sort bits or < 32768 records: separate extract
