@@ -209,9 +209,33 @@ sesa_status sesa_trace_set_profiling(sesa_trace *t, int enable);
 sesa_status sesa_trace_info(const sesa_trace *t, sesa_check_info *out);
 sesa_status sesa_trace_kernel_stats(const sesa_trace *t, sesa_kernel_stat *out, uint32_t cap, uint32_t *n_out);
 
+/* ---- Out-of-bound check (Table IV "OOB" P:467, the histo_final OOB of Fig. 9).
+ * A memory region is an allocation {base, size} of one space (the paper's "size of the memory region the
+ * pointer ... refers to").  With regions registered for a space, a valid record of that space is OUT OF
+ * BOUND iff no registered region R of its space contains all its bytes: R.base <= addr and
+ * addr + size <= R.base + R.size.  Spaces without registered regions are not checked.  The check runs inside
+ * the validation pass of every sesa_race_check (no extra pass over the records); it does not change the race
+ * list.  The witness is canonical: the lowest (index_base-adjusted) record index among the OOB records. */
+typedef struct {
+  uint64_t base;  /* first byte (SHARED: offset in the block's window; GLOBAL: device byte address)          */
+  uint64_t size;  /* bytes, >= 1; base + size must not wrap                                                 */
+  uint32_t space; /* SESA_SPACE_*                                                                          */
+  uint32_t reserved; /* zero                                                                               */
+} sesa_region;
 
+/* Register n (<= 1024) regions (host array, copied); n == 0 clears them.  EINVAL on space > 1, size 0,
+ * wrap-around, reserved != 0, or two regions of one space that overlap. */
+sesa_status sesa_trace_set_regions(sesa_trace *t, const sesa_region *regions, uint32_t n);
 
+typedef struct {
+  uint64_t n_oob;       /* OOB records in the last check                                                   */
+  uint64_t first_index; /* lowest OOB record index (index_base-adjusted); UINT64_MAX if none                */
+  sesa_access first;    /* that record (zero if none)                                                       */
+} sesa_oob_report;
 
+/* The OOB report of the last successful check (ESTATE before one).  Distributed handles: every rank holds the
+ * report merged over all ranks (each rank checks its own shard against its own registered regions). */
+sesa_status sesa_oob_get(const sesa_trace *t, sesa_oob_report *out);
 
 void sesa_trace_destroy(sesa_trace *t); /* NULL-safe; frees all device scratch */
 const char *sesa_status_str(sesa_status s);

@@ -11,6 +11,7 @@ Functions
   pair_kind(rec_a, rec_b, warp_size, lockstep) -> 0 | 1 (RW) | 2 (WW)
   validate(records) -> None or lowest bad index
   expand(flows) -> records  (canonical schedule order)
+  oob(records, regions, index_base=0) -> (count, first_index or None)   out-of-bound check (NEXT-1)
 """
 from __future__ import annotations
 
@@ -147,3 +148,28 @@ def race_tuples(races: np.ndarray):
     """Races as plain tuples (for readable comparisons in tests)."""
     return [(int(x["space"]), int(x["block"]), int(x["interval"]), int(x["addr"]), int(x["kind"]),
              int(x["first"]), int(x["second"])) for x in races]
+
+
+def oob(records: np.ndarray, regions: np.ndarray, index_base: int = 0):
+    """Out-of-bound records, by the definition in include/sesa.h (sesa_region; Table IV "OOB" P:467, Fig. 9
+    P:569-571): a valid record of a space with registered regions is OOB iff NO region of its space contains all
+    its bytes (base <= addr and addr + size <= base + size).  Spaces without regions are not checked.  Plain
+    definition: every record against every region of its space (no search structure).  Returns
+    (count, lowest index_base-adjusted OOB index or None)."""
+    r = np.asarray(records)
+    addr = r["addr"].astype(np.uint64)
+    end = addr + r["size"].astype(np.uint64)  # one past the last byte (records do not wrap: validated)
+    bad = np.zeros(len(r), bool)
+    for sp in (0, 1):
+        regs = regions[regions["space"] == sp]
+        if len(regs) == 0:
+            continue
+        sel = r["space"] == sp
+        inside = np.zeros(len(r), bool)
+        for g in regs:  # each region in turn: the definition, record by record
+            b, e = np.uint64(g["base"]), np.uint64(g["base"]) + np.uint64(g["size"])
+            inside |= sel & (addr >= b) & (end <= e)
+        bad |= sel & ~inside
+    idx = np.nonzero(bad)[0]
+    return int(len(idx)), (int(idx[0]) + index_base if len(idx) else None)
+

@@ -266,7 +266,15 @@ struct Summary {
   unsigned int bmin[2], bmax[2], imin[2], imax[2];
   unsigned int unsorted;         // some record's (block, interval) < its predecessor's
   unsigned int pad;
+  unsigned long long oob_count;  // valid records outside every registered region of their space (NEXT-1)
+  unsigned long long oob_first;  // lowest such record index (~0 = none)
 };
+
+// one registered memory region (include/sesa.h sesa_region), bytes [base, end)
+struct Region {
+  u64 base, end;
+};
+constexpr int MAX_REGIONS = 1024;
 
 // ---- kernel launchers (implemented in the .cu files) -------------------------------------------------------
 struct Launch {

@@ -309,6 +309,35 @@ static sesa_status dist_check(std::vector<sesa_trace*>& ts, std::vector<RankIO>&
     }
     return SESA_EINVAL;
   }
+  // OOB report (NEXT-1): every rank contributes (count, global first index, that record); all ranks merge
+  {
+    struct OobPart {
+      u64 count, first;
+      sesa_access rec;
+    };
+    std::vector<OobPart> parts(W);
+    for (int r = 0; r < R; r++) {
+      OobPart op;
+      memset(&op, 0, sizeof op);
+      const Summary& h = ts[r]->h_summary;
+      op.count = h.oob_count;
+      op.first = h.oob_count ? io[r].index_base + h.oob_first : ~0ull;
+      if (h.oob_count) cudaMemcpy(&op.rec, io[r].rec + h.oob_first, 32, cudaMemcpyDeviceToHost);
+      if (ex) {
+        if (!ex->allgather(ts[0], &op, parts.data(), sizeof op)) return ts[0]->status;
+      } else {
+        parts[r] = op;
+      }
+    }
+    sesa_oob_report rep;
+    memset(&rep, 0, sizeof rep);
+    rep.first_index = ~0ull;
+    for (int p = 0; p < W; p++) {
+      rep.n_oob += parts[p].count;
+      if (parts[p].count && parts[p].first < rep.first_index) rep.first_index = parts[p].first, rep.first = parts[p].rec;
+    }
+    for (int r = 0; r < R; r++) ts[r]->oob = rep, ts[r]->have_oob = true;
+  }
   for (int p = 1; p < W; p++) {
     const Summary& q = sums[p];
     S.entries += q.entries, S.multi += q.multi, S.unsorted |= q.unsorted;

@@ -71,16 +71,23 @@ struct SpaceAcc2 {
 // tile histograms of the first sort digit ((g - gmin) & 255 is a rotation of g & 255), which lets the fused
 // extract + first sort pass place every tile without a look-back (k_fused.cu).
 template <int U>
+// With regions (nreg > 0; sorted by (space, base), non-overlapping, space s in [rs[s], rs[s+1])), every valid
+// record of a space with regions is also checked for containment (OOB, NEXT-1): binary search for the last
+// region starting at or below addr, then addr + size <= end.
 __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ rec, u32 n, u32 log2G, u32 rw,
-                                                       Summary* __restrict__ out, u32* __restrict__ tile_hist) {
+                                                       Summary* __restrict__ out, u32* __restrict__ tile_hist,
+                                                       const Region* __restrict__ regs, uint3 rs) {
   __shared__ u32 s_th[8][RADIX];
+  extern __shared__ Region s_reg[];  // [rs.z]
+  for (u32 i = threadIdx.x; i < rs.z; i += 256) s_reg[i] = regs[i];
+  if (rs.z) __syncthreads();
   constexpr int THREADS = 256;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const u32 gw = (blockIdx.x * THREADS + threadIdx.x) >> 5;
   const u64 start64 = (u64)gw * rw;
   const u32 start = (u32)min(start64, (u64)n), end = (u32)min((u64)n, start64 + rw);
   const u32 gmask = (1u << log2G) - 1u;
-  u32 bad = ~0u, extra = 0, multi = 0, unsorted = 0;
+  u32 bad = ~0u, extra = 0, multi = 0, unsorted = 0, oobc = 0, oobf = ~0u;
   SpaceAcc2 A0, A1;
   A0.init();
   A1.init();
@@ -128,6 +135,23 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
       allg = allg && (!ok[u] || sp == SP_GLOBAL);
       alls = alls && (!ok[u] || sp == SP_SHARED);
     }
+    if (rs.z) {  // OOB: containment in a registered region of the record's space
+#pragma unroll
+      for (int u = 0; u < U; u++) {
+        if (!ok[u]) continue;
+        const u32 sp = (b[u].w >> 16) & 0xFFu;
+        int lo = sp ? (int)rs.x : 0, hi = sp ? (int)rs.z : (int)rs.x;
+        if (lo >= hi) continue;  // no regions registered for this space: not checked
+        const u64 addr = ((u64)a[u].y << 32) | a[u].x;
+        const u64 last = addr + (u64)(b[u].w & 0xFFFFu) - 1ull;
+        while (hi - lo > 1) {
+          const int mid = (lo + hi) >> 1;
+          if (s_reg[mid].base <= addr) lo = mid;
+          else hi = mid;
+        }
+        if (!(s_reg[lo].base <= addr && last < s_reg[lo].end)) oobc++, oobf = min(oobf, r0 + u * 32 + lane);
+      }
+    }
     // one space decision per batch (traces are mostly single-space)
     const bool bg = __all_sync(~0u, allg), bs = !bg && __all_sync(~0u, alls);
 #pragma unroll
@@ -152,6 +176,12 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
   }
   // block reduction (warp shuffles, then one atomic per field per CTA)
   u64 bad64 = bad == ~0u ? ~0ull : (u64)bad, ent = (u64)extra + A0.cnt + A1.cnt, mul = multi;
+  if (rs.z) {
+    u64 oc = oobc, of = oobf == ~0u ? ~0ull : (u64)oobf;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) oc += __shfl_xor_sync(~0u, oc, o), of = min(of, __shfl_xor_sync(~0u, of, o));
+    if (lane == 0 && oc) atomicAdd(&out->oob_count, (unsigned long long)oc), atomicMin(&out->oob_first, (unsigned long long)of);
+  }
   SpaceAcc S0 = A0.to_acc(log2G), S1 = A1.to_acc(log2G);
   __shared__ SpaceAcc sa[THREADS / 32][2];
   __shared__ u64 s64[THREADS / 32][3];
@@ -213,7 +243,8 @@ static int ring_grid(const void* kern, int threads, size_t smem, size_t smem_max
   return sms * (per > 0 ? per : 1);
 }
 
-void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, u32* tile_hist, int grid, cudaStream_t st) {
+void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, u32* tile_hist, const Region* regs, u32 nreg,
+                    u32 nreg_shared, int grid, cudaStream_t st) {
   // extents2: contiguous warp ranges, one full wave of resident warps (the round-1 grid-stride kernel took
   // 7.7 ms on C5: 132 instructions per record, 64-bit index math and local-memory accumulators; this one 4.6 ms)
   static int sms = 0, per = 0;
@@ -223,13 +254,16 @@ void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, u32* tile_
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, extents2_kernel<4>, 256, 0);
     per = std::max(per, 1);
+    cudaFuncSetAttribute(extents2_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)(MAX_REGIONS * sizeof(Region)));
   }
   const u64 warps = (u64)sms * per * 8;
   const u64 gran = tile_hist ? FUSED_TILE : 128;  // warp ranges: whole tiles when tile histograms are wanted
   u64 rw = (n + warps - 1) / warps;
   rw = std::max<u64>(gran, (rw + gran - 1) / gran * gran);
   const u64 nw = (n + rw - 1) / rw;
-  extents2_kernel<4><<<(unsigned)((nw + 7) / 8), 256, 0, st>>>(rec, (u32)n, log2G, (u32)rw, d_sum, tile_hist);
+  extents2_kernel<4><<<(unsigned)((nw + 7) / 8), 256, nreg * sizeof(Region), st>>>(
+      rec, (u32)n, log2G, (u32)rw, d_sum, tile_hist, regs, make_uint3(nreg_shared, 0u, nreg));
   (void)grid;
 }
 

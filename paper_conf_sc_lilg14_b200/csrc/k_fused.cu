@@ -96,7 +96,6 @@ struct FusedArgs {
   const u32* toff;  // [T][RADIX] output offset of each tile's digit run
   u64* kout;
   u32* hist;        // [npass][RADIX] global digit histograms (rows 1.. are accumulated here)
-  u32 nohist;       // timing experiment only (SESA_FUSED_NOHIST): skip the later-digit histograms
 };
 
 // Persistent CTAs, software-pipelined in registers: right after a tile's digit counts (when its addresses have
@@ -191,11 +190,9 @@ __global__ void __launch_bounds__(FUSED_THREADS, FUSED_MINB) fused_extract_pass0
       const u64 key = keys_s[j];
       const u32 d = (u32)((key >> A.pos_bits) & (RADIX - 1));
       __stcs(A.kout + (globu[d] + j), key);
-      if (!A.nohist) {
 #pragma unroll
-        for (int p = 1; p < NP; p++)
-          atomicAdd(&hrest[(p - 1) * RADIX + (u32)((key >> (A.pos_bits + p * RADIX_BITS)) & (RADIX - 1))], 1u);
-      }
+      for (int p = 1; p < NP; p++)
+        atomicAdd(&hrest[(p - 1) * RADIX + (u32)((key >> (A.pos_bits + p * RADIX_BITS)) & (RADIX - 1))], 1u);
     }
     __syncthreads();  // shared memory is reused by the next tile
     tile = next;
@@ -254,7 +251,6 @@ void launch_fused_extract_pass0(const Rec* rec, u64 n, const KeyLayout& L, u32 n
   A.toff = O;
   A.kout = kout;
   A.hist = hist;
-  A.nohist = getenv("SESA_FUSED_NOHIST") ? 1u : 0u;
   const u32 g = std::min<u32>(T, (u32)grid);
   switch (npass) {
     case 1: fused_extract_pass0_kernel<1><<<g, FUSED_THREADS, sm, st>>>(A); break;

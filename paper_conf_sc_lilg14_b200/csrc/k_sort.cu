@@ -262,39 +262,6 @@ __global__ void __launch_bounds__(THREADS, MINB) onesweep_kernel(const u64* __re
 // only needed by the final coalesced write-out.  LATE_LB = walk the look-back after ranking (predecessors have
 // had the ranking time to publish their inclusive prefixes) instead of before.
 // ------------------------------------------------------------------------------------------------------------
-// Look-back sequencer (LBW == 0 variants): instead of every tile walking back over its predecessors' aggregates
-// (measured: ~2.8 us per tile, 15-30 predecessors deep, and longer with wider walks), one resident CTA turns the
-// published tile aggregates into inclusive prefixes in tile order — thread d owns digit d and keeps the running
-// prefix in a register, 32 tiles per L2 round trip — and each tile only polls its own status word.
-__device__ __noinline__ void lb_sequencer(u64* __restrict__ lb, u32 ntiles, u32 epoch) {
-  constexpr int K = 32;
-  const u32 d = threadIdx.x;
-  if (d >= RADIX) return;
-  u64 prefix = 0;
-  u32 j = 0;
-  while (j < ntiles) {
-    u64 w[K];
-#pragma unroll
-    for (int q = 0; q < K; q++) w[q] = j + q < ntiles ? ld_relaxed(lb + (u64)(j + q) * RADIX + d) : 0ull;
-    u32 c = 0;
-    bool stop = false;
-#pragma unroll
-    for (int q = 0; q < K; q++) {
-      if (stop || j + q >= ntiles) continue;
-      const u32 e = (u32)((w[q] >> 54) & 0xFF);
-      if (e != epoch || (w[q] & (3ull << 62)) == 0) {
-        stop = true;
-        continue;
-      }
-      prefix += w[q] & LB_VAL;
-      st_relaxed(lb + (u64)(j + q) * RADIX + d, lb_pack(LB_PREFIX, epoch, prefix));
-      c++;
-    }
-    j += c;
-    if (c == 0) __nanosleep(64);
-  }
-}
-
 template <int THREADS, int ITEMS, int LBW, bool FULL, bool LATE_LB, int S, bool BAL, bool TMA>
 __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64* __restrict__ kout, u32 m, u32 shift,
                                                const u64* __restrict__ bin_base, u64* __restrict__ lookback,
@@ -370,27 +337,13 @@ __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64*
     for (int w = 0; w < WARPS * S; w++) whist[w * RADIX + tid] += bs;
   }
   auto look_back = [&]() {
-    if (LBW == 0) {  // the sequencer publishes this tile's inclusive prefix: poll our own word
-      if (tid < RADIX) {
-        u64 w;
-        int spins = 0;
-        while (true) {
-          w = ld_relaxed(lookback + (u64)tile * RADIX + tid);
-          if ((u32)((w >> 54) & 0xFF) == epoch && (w & (3ull << 62)) == LB_PREFIX) break;
-          __nanosleep(++spins < 4 ? 32 : 128);
-        }
-        if (prof && tid == 0) prof[7] = (u64)spins;
-        globu[tid] = (u32)(bin_base[tid] + ((w & LB_VAL) - tot)) - bs;
-      }
-      return;
-    }
     if (tid < RADIX) {
       u64 excl = 0;
       if (tile > 0) {
         long long p = (long long)tile - 1;
         int spins = 0;
         while (true) {
-          constexpr int LW = LBW > 0 ? LBW : 1;
+          constexpr int LW = LBW;
           u64 w[LW];
 #pragma unroll
           for (int q = 0; q < LW; q++) w[q] = p - q >= 0 ? ld_relaxed(lookback + (u64)(p - q) * RADIX + tid) : 0ull;
@@ -488,11 +441,7 @@ __global__ void __launch_bounds__(THREADS, MINB) onesweep2_kernel(const u64* __r
   if (!BAL)
     for (int i = tid; i < WARPS * S * (RADIX + 1); i += THREADS) wmask[i] = 0;
   __syncthreads();
-  if (LBW == 0 && s_tile == 0) {  // the first CTA to run is the look-back sequencer (it is resident by definition)
-    lb_sequencer(lookback, (m + TILE - 1) / TILE, epoch);
-    return;
-  }
-  const u32 tile = s_tile - (LBW == 0 ? 1u : 0u);
+  const u32 tile = s_tile;
   unsigned long long* prof = g_prof ? g_prof + (u64)tile * 8 : nullptr;
   if (prof && tid == 0) prof[0] = gtime();
   if ((u64)(tile + 1) * TILE <= m)
@@ -518,7 +467,7 @@ static void launch_os2(const u64* kin, u64* kout, u32 m, u32 shift, const u64* b
     cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     set = true;
   }
-  const u32 tiles = (u32)((m + THREADS * ITEMS - 1) / (THREADS * ITEMS)) + (LBW == 0 ? 1u : 0u);
+  const u32 tiles = (u32)((m + THREADS * ITEMS - 1) / (THREADS * ITEMS));
   kern<<<tiles, THREADS, sm, st>>>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch);
 }
 
@@ -529,11 +478,14 @@ static size_t onesweep_smem() {
          (WARPS + 1) * 4 + (size_t)WARPS * (RADIX + 1) * 4;
 }
 
-// SESA_SORT_CFG selects the onesweep variant (all measured on C5, 1 B200; DESIGN.md §6 has the table):
+// SESA_SORT_CFG selects the onesweep variant (all measured on C5, 1 B200; DESIGN.md §9 has the numbers):
 //   0 / 1   onesweep (ranks kept in registers, look-back before ranking), 256 x 16 / 256 x 24 keys
-//   13..16  onesweep2, 256 x 24: early / late look-back at 2 CTAs/SM (13/14), 3 CTAs/SM (15/16)
-//   19 / 20 onesweep2, 256 x 32, early / late look-back (20 = default: fastest)
+//   15      onesweep2 256 x 24 at 3 CTAs/SM;  20: onesweep2 256 x 32, register loads, look-back after ranking
 //   21      as 20 with 16 predecessors per look-back round trip;  26: two rank streams;  31: ballot peers
+//   33      as 20 with the tile loaded by TMA bulk copies (default: fastest);  34: 33 with the early look-back
+//   35      as 33 with 512 x 16 tiles
+// Measured and removed: a look-back sequencer CTA, a dedicated look-back warp, cluster-level (DSMEM) look-back,
+// 256 x 40/48 tiles — each slower.
 int sort_cfg() {
   static int v = -1;
   if (v < 0) {
@@ -545,12 +497,9 @@ int sort_cfg() {
 
 u32 sort_tile_keys() {
   switch (sort_cfg()) {
-    case 1: case 13: case 14: case 15: case 16: return 256 * 24;
-    case 19: case 20: case 21: case 22: case 23: case 24: case 25: case 26: case 27: case 31: return 256 * 32;
-    case 28: case 29: case 35: return 512 * 16;
-    case 33: case 34: return 256 * 32;
-    case 30: return 512 * 12;
-    case 32: return 384 * 24;
+    case 1: case 15: return 256 * 24;
+    case 20: case 21: case 26: case 31: case 33: case 34: return 256 * 32;
+    case 35: return 512 * 16;
     default: return 256 * 16;
   }
 }
@@ -595,25 +544,12 @@ static void launch_os_cfg(const u64* kin, u64* kout, const u32* vin, u32* vout, 
                           const u64* bin_base, u64* lookback, u32* tile_ctr, u32 epoch, cudaStream_t st) {
   switch (sort_cfg()) {
     case 1: launch_os<256, 24, 2, VALS, MATCH>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 13: launch_os2<256, 24, 2, 4, false>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 14: launch_os2<256, 24, 2, 4, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
     case 15: launch_os2<256, 24, 3, 4, false>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 16: launch_os2<256, 24, 3, 4, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 19: launch_os2<256, 32, 2, 4, false>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
     case 20: launch_os2<256, 32, 2, 4, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
     case 21: launch_os2<256, 32, 2, 16, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 22: launch_os2<256, 32, 2, 32, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 23: launch_os2<256, 32, 2, 8, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 24: launch_os2<256, 32, 2, 16, false>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
     case 33: launch_os2<256, 32, 2, 4, true, 1, false, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
     case 34: launch_os2<256, 32, 2, 4, false, 1, false, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
     case 35: launch_os2<512, 16, 2, 4, true, 1, false, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 28: launch_os2<512, 16, 2, 4, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 29: launch_os2<512, 16, 2, 4, false>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 30: launch_os2<512, 12, 3, 4, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 32: launch_os2<384, 24, 2, 4, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 25: launch_os2<256, 32, 2, 0, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 27: launch_os2<256, 32, 2, 0, false>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
     case 26: launch_os2<256, 32, 2, 4, true, 2>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
     case 31: launch_os2<256, 32, 2, 4, true, 1, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
     default: launch_os<256, 16, 3, VALS, MATCH>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st);

@@ -21,7 +21,9 @@ constexpr int CT_TILE = CT_THREADS * CT_ITEMS;
 
 // k_extract.cu
 // tile_hist (optional, [ceil(n / FUSED_TILE)][RADIX]): per-tile histograms of (addr >> log2G) & 255 (k_fused.cu)
-void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, u32* tile_hist, int grid, cudaStream_t st);
+// regs (optional, device, nreg <= MAX_REGIONS): sorted by (space, base), the first nreg_shared are SHARED
+void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, u32* tile_hist, const Region* regs, u32 nreg,
+                    u32 nreg_shared, int grid, cudaStream_t st);
 void launch_extract_1to1(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, u64* keys, u32* hist, u64 pos_base,
                          int grid, cudaStream_t st);
 void launch_entry_count(const Rec* rec, u64 n, u32 log2G, u32* cnt, cudaStream_t st);

@@ -170,6 +170,7 @@ bool sesa_trace::make_layout(const Summary& S, u64 n) {
 
 void sesa_trace::begin_check(u64 n) {
   status = SESA_OK;
+  have_oob = false;
   err.clear();
   have_result = false;
   n_races = 0;
@@ -211,6 +212,7 @@ bool sesa_trace::step_extents(const Rec* rec, u64 n, bool tile_hist) {
   Summary init;
   memset(&init, 0, sizeof init);
   init.bad_index = ~0ull;
+  init.oob_first = ~0ull;
   init.gmin[0] = init.gmin[1] = ~0ull;
   init.bmin[0] = init.bmin[1] = init.imin[0] = init.imin[1] = ~0u;
   h_summary = init;
@@ -219,10 +221,19 @@ bool sesa_trace::step_extents(const Rec* rec, u64 n, bool tile_hist) {
     return false;
   const int grid_stream = (int)std::min<u64>((n + 255) / 256, (u64)num_sms * 8);
   LAUNCH("extents", 32.0 * n, launch_extents(rec, n, log2G, (Summary*)b_summary.p,
-                                             have_thist ? (u32*)b_thist.p : nullptr, grid_stream, stream));
+                                             have_thist ? (u32*)b_thist.p : nullptr, (const Region*)b_regions.p,
+                                             n_regions, n_regions_shared, grid_stream, stream));
   if (!cuda_ok(cudaMemcpyAsync(&h_summary, b_summary.p, sizeof(Summary), cudaMemcpyDeviceToHost, stream), "summary"))
     return false;
   return sync_check("extents");
+}
+
+void sesa_trace::set_oob(const sesa_access* d_rec, u64 count, u64 local_first, u64 index_base) {
+  memset(&oob, 0, sizeof oob);
+  oob.n_oob = count;
+  oob.first_index = count ? index_base + local_first : ~0ull;
+  if (count) cudaMemcpy(&oob.first, d_rec + local_first, sizeof(sesa_access), cudaMemcpyDeviceToHost);
+  have_oob = true;
 }
 
 bool sesa_trace::report_bad(const sesa_access* d_rec, u64 local_bad, u64 global_bad) {
@@ -461,6 +472,7 @@ bool sesa_trace::step_race_sort(u32 nr, const RaceOut* races, u64* rkeys0, u32* 
 sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_base) {
   begin_check(n);
   if (n == 0) {
+    set_oob(d_rec, 0, 0, index_base);
     have_result = true;
     collect_prof();
     return SESA_OK;
@@ -470,6 +482,7 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
   if (!step_extents(rec, n, true)) return status;
   const Summary& S = h_summary;
   if (S.bad_index != ~0ull) return report_bad(d_rec, S.bad_index, S.bad_index), status;
+  set_oob(d_rec, S.oob_count, S.oob_first, index_base);
   const u64 m = S.entries;
   info.n_entries = m;
   info.sorted_input = !S.unsorted;
@@ -693,6 +706,45 @@ sesa_status sesa_trace_set_profiling(sesa_trace* t, int enable) {
 sesa_status sesa_trace_info(const sesa_trace* t, sesa_check_info* out) {
   if (!t || !out) return SESA_EINVAL;
   *out = t->info;
+  return SESA_OK;
+}
+
+sesa_status sesa_trace_set_regions(sesa_trace* t, const sesa_region* regions, uint32_t n) {
+  if (!t || (n && !regions)) return SESA_EINVAL;
+  if (n > (uint32_t)MAX_REGIONS) return t->fail(SESA_EINVAL, "%u regions > %d", n, MAX_REGIONS), SESA_EINVAL;
+  std::vector<sesa_region> v(regions, regions + n);
+  for (uint32_t i = 0; i < n; i++) {
+    const sesa_region& r = v[i];
+    if (r.space > 1 || r.size == 0 || r.reserved != 0 || r.base + r.size < r.base)
+      return t->fail(SESA_EINVAL, "region %u invalid (space=%u size=%llu)", i, r.space, (unsigned long long)r.size),
+             SESA_EINVAL;
+  }
+  std::sort(v.begin(), v.end(), [](const sesa_region& a, const sesa_region& b) {
+    return a.space != b.space ? a.space < b.space : a.base < b.base;
+  });
+  uint32_t nsh = 0;
+  for (uint32_t i = 0; i < n; i++) {
+    if (v[i].space == SP_SHARED) nsh++;
+    if (i && v[i].space == v[i - 1].space && v[i - 1].base + v[i - 1].size > v[i].base)
+      return t->fail(SESA_EINVAL, "regions overlap (space %u, base 0x%llx)", v[i].space,
+                     (unsigned long long)v[i].base), SESA_EINVAL;
+  }
+  std::vector<Region> dev(n);
+  for (uint32_t i = 0; i < n; i++) dev[i].base = v[i].base, dev[i].end = v[i].base + v[i].size;
+  if (n) {
+    if (!t->grow(t->b_regions, n * sizeof(Region), "regions")) return t->status;
+    if (!t->cuda_ok(cudaMemcpy(t->b_regions.p, dev.data(), n * sizeof(Region), cudaMemcpyHostToDevice), "regions"))
+      return t->status;
+  }
+  t->n_regions = n;
+  t->n_regions_shared = nsh;
+  return SESA_OK;
+}
+
+sesa_status sesa_oob_get(const sesa_trace* t, sesa_oob_report* out) {
+  if (!t || !out) return SESA_EINVAL;
+  if (!t->have_result || !t->have_oob) return SESA_ESTATE;
+  *out = t->oob;
   return SESA_OK;
 }
 

@@ -44,6 +44,11 @@ struct sesa_trace {
   DevBuf b_races, b_rkeys[2], b_rvals[2], b_races_sorted, b_rhist, b_rbase;
   DevBuf b_eoff, b_ecnt, b_ecell, b_hrec, b_dist_races, b_ctmp, b_ctotal, b_thist, b_ftmp;
   bool have_thist = false;  // extents wrote per-tile raw digit histograms (fused first pass possible)
+  // out-of-bound check (NEXT-1): registered regions (sorted by space, base) and the last report
+  DevBuf b_regions;
+  uint32_t n_regions = 0, n_regions_shared = 0;
+  sesa_oob_report oob{};
+  bool have_oob = false;
   DevBuf b_dist[8];
   void* h_pinned = nullptr;
 
@@ -51,7 +56,7 @@ struct sesa_trace {
     std::vector<DevBuf*> v = {&b_summary, &b_hist, &b_binbase, &b_lookback, &b_ctr, &b_cnt, &b_off, &b_temp,
                               &b_tflags, &b_part, &b_carry, &b_owner, &b_slots, &b_cross, &b_ccount, &b_carrytmp,
                               &b_races, &b_races_sorted, &b_rhist, &b_rbase, &b_eoff, &b_ecnt, &b_ecell,
-                              &b_hrec, &b_dist_races, &b_ctmp, &b_ctotal, &b_thist, &b_ftmp};
+                              &b_hrec, &b_dist_races, &b_ctmp, &b_ctotal, &b_thist, &b_ftmp, &b_regions};
     for (auto& b : b_keys) v.push_back(&b);
     for (auto& b : b_rkeys) v.push_back(&b);
     for (auto& b : b_rvals) v.push_back(&b);
@@ -89,6 +94,7 @@ struct sesa_trace {
   bool check_records_ptr(const sesa_access* d_rec, uint64_t n);
   bool step_extents(const sesa::Rec* rec, uint64_t n, bool tile_hist = false);
   bool report_bad(const sesa_access* d_rec, uint64_t local_bad, uint64_t global_bad);
+  void set_oob(const sesa_access* d_rec, uint64_t count, uint64_t local_first, uint64_t index_base);
   bool step_extract(const sesa::Rec* rec, uint64_t n, uint64_t m, uint64_t pos_base, bool multi);
   bool step_hist(uint64_t m);
   bool step_extract_fused(const sesa::Rec* rec, uint64_t n);

@@ -34,6 +34,13 @@ FLOW_DTYPE = np.dtype(
      ("size", "<u2"), ("space", "u1"), ("rw", "u1"), ("flags", "<u4")], align=True)
 
 
+REGION_DTYPE = np.dtype([("base", "<u8"), ("size", "<u8"), ("space", "<u4"), ("reserved", "<u4")], align=True)
+
+
+class sesa_oob_report(ctypes.Structure):
+    _fields_ = [("n_oob", ctypes.c_uint64), ("first_index", ctypes.c_uint64), ("first", ctypes.c_uint8 * 32)]
+
+
 class sesa_config(ctypes.Structure):
     _fields_ = [("warp_size", ctypes.c_uint32), ("lockstep", ctypes.c_uint32), ("granularity", ctypes.c_uint32),
                 ("flags", ctypes.c_uint32)]
@@ -56,7 +63,7 @@ class sesa_check_info(ctypes.Structure):
 EXPORTS = ["sesa_trace_create", "sesa_trace_create_dist", "sesa_nccl_unique_id", "sesa_race_check",
            "sesa_race_check_host", "sesa_races_get", "sesa_races_device", "sesa_expand", "sesa_trace_set_profiling",
            "sesa_trace_info", "sesa_trace_kernel_stats", "sesa_trace_destroy", "sesa_status_str", "sesa_last_error",
-           "sesa_abi_version", "sesa_race_check_loopback"]
+           "sesa_abi_version", "sesa_race_check_loopback", "sesa_trace_set_regions", "sesa_oob_get"]
 
 _lib = None
 
@@ -197,6 +204,23 @@ class Trace:
         if st not in (SESA_OK, SESA_ETRUNC) or (st == SESA_ETRUNC and d_out is not None):
             self._raise(st, "sesa_expand")
         return n.value
+
+    def set_regions(self, regions: np.ndarray):
+        """Register memory regions (REGION_DTYPE array: base, size, space) for the out-of-bound check."""
+        a = np.ascontiguousarray(regions, dtype=REGION_DTYPE)
+        st = self.lib.sesa_trace_set_regions(self.h, ctypes.c_void_p(a.ctypes.data if len(a) else 0),
+                                             ctypes.c_uint32(len(a)))
+        if st != SESA_OK:
+            self._raise(st, "sesa_trace_set_regions")
+
+    def oob(self) -> dict:
+        """The last check's OOB report: n_oob, first_index (2**64-1 if none), first (record, ACCESS_DTYPE)."""
+        r = sesa_oob_report()
+        st = self.lib.sesa_oob_get(self.h, ctypes.byref(r))
+        if st != SESA_OK:
+            self._raise(st, "sesa_oob_get")
+        return dict(n_oob=r.n_oob, first_index=r.first_index,
+                    first=np.frombuffer(bytes(r.first), ACCESS_DTYPE)[0])
 
     def set_profiling(self, on: bool = True):
         self.lib.sesa_trace_set_profiling(self.h, 1 if on else 0)

@@ -41,6 +41,8 @@ def test_struct_layouts_match_generators_and_oracle():
     assert S.RACE_DTYPE == sesagen.RACE_DTYPE == O.RACE_DTYPE
     assert S.FLOW_DTYPE == sesagen.FLOW_DTYPE == O.FLOW_DTYPE
     assert ctypes.sizeof(S.sesa_config) == 16
+    assert S.REGION_DTYPE.itemsize == 24 and ctypes.sizeof(S.sesa_oob_report) == 48
+    assert S.REGION_DTYPE == sesagen.f6_regions().dtype
 
 
 def test_bad_config_rejected_before_device():
@@ -57,6 +59,8 @@ def test_null_handle_calls():
     n = ctypes.c_uint64()
     assert lib.sesa_races_get(None, None, 0, ctypes.byref(n)) == S.SESA_EINVAL
     assert lib.sesa_race_check(None, None, 0, 0, None) == S.SESA_EINVAL
+    assert lib.sesa_trace_set_regions(None, None, 0) == S.SESA_EINVAL
+    assert lib.sesa_oob_get(None, None) == S.SESA_EINVAL
     lib.sesa_trace_destroy(None)  # NULL-safe
     assert lib.sesa_last_error(None) == b""
 

@@ -250,3 +250,58 @@ def test_fused_first_pass_parity(sesa, n, words, shift, fused):
     r["addr"] += np.uint64(4 * shift)
     assert_same(sesa, r, 32, 0, 4)
     assert trace(sesa).info()["fused_first_pass"] == fused  # > 32 sort bits or < 32768 records: separate extract
+
+
+# ------------------------------------------------------------------------------------------------ OOB (NEXT-1)
+def _oob_check(S, recs, regions, base=0):
+    t = S.Trace(32, 0, 4)
+    t.set_regions(regions)
+    t.check(S.to_device(recs), len(recs), index_base=base)
+    got = t.oob()
+    t.close()
+    cnt, first = O.oob(recs, regions, index_base=base)
+    assert got["n_oob"] == cnt
+    assert got["first_index"] == (first if first is not None else 2**64 - 1)
+    if first is not None:
+        assert got["first"].tobytes() == recs[first - base].tobytes()
+    return got
+
+
+def test_f6_histo_final_oob(sesa):
+    got = _oob_check(sesa, G.f6_histo_final(), G.f6_regions())
+    assert got["n_oob"] == 12288 and (int(got["first"]["block"]), int(got["first"]["thread"])) == (18, 0)
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_oob_random_regions(sesa, seed):
+    rng = np.random.default_rng(seed)
+    r = G.random_trace([5000, 70000, 200003, 33][seed], 40 + seed, words=3000, blocks=9, threads=200)
+    # non-overlapping random regions over both spaces' word ranges (shared from 0, global from 2^40)
+    regs = []
+    for sp, base in ((0, 0), (1, 0x10000000000)):
+        cuts = np.sort(rng.choice(np.arange(1, 12000), size=2 * (5 + seed), replace=False))
+        for a, b in cuts.reshape(-1, 2):
+            regs.append((base + int(a), int(b - a), sp))
+    reg = np.zeros(len(regs), G.f6_regions().dtype)
+    for i, (b, z, sp) in enumerate(regs):
+        reg[i]["base"], reg[i]["size"], reg[i]["space"] = b, z, sp
+    _oob_check(sesa, r, reg, base=seed * 7)
+    _oob_check(sesa, r, reg[reg["space"] == 1])  # only global checked
+
+
+def test_oob_region_validation(sesa):
+    t = sesa.Trace(32, 0, 4)
+    reg = np.zeros(2, sesa.REGION_DTYPE)
+    reg["base"], reg["size"], reg["space"] = [0, 10], [16, 4], 1  # [0,16) and [10,14) overlap
+    with pytest.raises(sesa.SesaError):
+        t.set_regions(reg)
+    reg["size"] = [10, 0]
+    with pytest.raises(sesa.SesaError):
+        t.set_regions(reg)
+    reg["size"], reg["space"] = [10, 4], [1, 2]
+    with pytest.raises(sesa.SesaError):
+        t.set_regions(reg)
+    reg["space"] = 1
+    t.set_regions(reg)  # adjacent, fine
+    t.set_regions(reg[:0])  # clears
+    t.close()

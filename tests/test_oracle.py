@@ -362,3 +362,48 @@ def test_bad_config():
 
 def test_empty():
     assert len(O.check(np.zeros(0, G.REC_DTYPE))) == 0
+
+
+# ------------------------------------------------------------------------------------------------ OOB (NEXT-1)
+def _region(base, size, space=G.GLOBAL):
+    r = np.zeros(1, G.f6_regions().dtype)
+    r["base"], r["size"], r["space"] = base, size, space
+    return r
+
+
+def test_f6_histo_final_oob_closed_form():
+    # Fig. 9 / P:569-571: iteration i = t_lin + 47 * 42 * 512 reads bytes [8i, 8i + 8) of an 8,159,232-byte region
+    # -> out of bound iff 8 i + 8 > 8,159,232 <=> t_lin >= 9216 (only k = 47); 42 * 512 - 9216 = 12,288 records
+    recs = G.f6_histo_final()
+    assert len(recs) == 42 * 512 * 48
+    count, first = O.oob(recs, G.f6_regions())
+    assert count == 42 * 512 - 9216 == 12288
+    # lowest index: block 18, thread 0, k = 47 (canonical order block, thread, k)
+    assert first == 18 * 512 * 48 + 47
+    r = recs[first]
+    assert (int(r["block"]), int(r["thread"]), int(r["addr"]) - G.F6_HISTO) == (18, 0, 8 * (9216 + 47 * 21504))
+    # the paper's witness bid = <24,0,0>, tid = <0,0,0> is an OOB access of iteration 47
+    pw = 24 * 512 * 48 + 47
+    addr = int(recs[pw]["addr"]) - G.F6_HISTO
+    assert addr + 8 > G.F6_REGION and (int(recs[pw]["block"]), int(recs[pw]["thread"])) == (24, 0)
+    # one iteration fewer: nothing is out of bound
+    assert O.oob(G.f6_histo_final(iters=47), G.f6_regions()) == (0, None)
+
+
+def test_oob_boundaries_and_scope():
+    recs = np.zeros(5, O.REC_DTYPE)
+    recs["space"] = [G.GLOBAL, G.GLOBAL, G.GLOBAL, G.SHARED, G.GLOBAL]
+    recs["addr"] = [100, 196, 197, 0, 99]
+    recs["size"] = [4, 4, 4, 8, 1]
+    reg = _region(100, 100)  # bytes [100, 200)
+    # [100,104) in, [196,200) in (last byte 199), [197,201) out, shared not checked (no shared regions), 99 out
+    assert O.oob(recs, reg) == (2, 2)
+    assert O.oob(recs, reg, index_base=1000) == (2, 1002)
+    # a shared region makes the shared record checked: [0, 8) in [0, 8) -> in; [0, 7) -> out
+    both = np.concatenate([reg, _region(0, 8, G.SHARED)])
+    assert O.oob(recs, both) == (2, 2)
+    assert O.oob(recs, np.concatenate([reg, _region(0, 7, G.SHARED)])) == (3, 2)
+    # a record spanning two ADJACENT regions is not inside one allocation -> out of bound
+    two = np.concatenate([_region(100, 98), _region(198, 2)])
+    assert O.oob(recs[1:2], two) == (1, 0)
+    assert O.oob(recs, np.zeros(0, reg.dtype)) == (0, None)
