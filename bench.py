@@ -341,7 +341,7 @@ def main():
                            if n_total * 32 > 1e9 else "inputs smaller than L2 (latency-bound config)",
                            "sort_bits": info["sort_bits"], "sort_passes": info["sort_passes"],
                            "races": n_races, "crossing_tiles": info["crossing_tiles"],
-                           "entries_at_shared_locations": info["n_multi"]},
+                           "entries_at_multi_entry_locations": info["n_multi"], "fused_first_pass": bool(info["fused_first_pass"])},
                 "gpu_launches": launches, "roofline": roof,
                 "honesty": {"record_bytes_per_step": n_total * 32, "achieved_gbs_vs_32B_per_record":
                             n_total * 32 / (ms / args.steps / 1e3) / 1e9,

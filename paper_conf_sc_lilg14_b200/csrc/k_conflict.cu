@@ -550,12 +550,18 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
   }
 
   if (MODE == 1) {
+    // does the tile hold a sub-run head / tail anywhere? (block-wide votes over each thread's items)
+    bool my_sh = false, my_st = false;
+#pragma unroll
+    for (int q = 0; q < CT_ITEMS; q++) {
+      const u32 j = tid * CT_ITEMS + q;
+      if (j < cnt) my_sh |= (s.fl[j] & FL_SH) != 0, my_st |= (s.fl[j] & FL_ST) != 0;
+    }
+    const bool sh = __syncthreads_or(my_sh), st = __syncthreads_or(my_st);
     if (tid == 0) {
       u8 tf = 0;
       if (lhead >= 0) tf |= TF_GH;
       if (ftail < (int)cnt) tf |= TF_GT;
-      bool sh = false, st = false;
-      for (u32 j = 0; j < cnt; j++) sh |= (s.fl[j] & FL_SH) != 0, st |= (s.fl[j] & FL_ST) != 0;
       if (sh) tf |= TF_SH;
       if (st) tf |= TF_ST;
       if (cin) tf |= TF_CIN;
