@@ -9,6 +9,7 @@ they match the C structs' sizes.
 Functions
   check(records, index_base=0, warp_size=32, lockstep=0, granularity=4, method="grouped") -> races
   pair_kind(rec_a, rec_b, warp_size, lockstep) -> 0 | 1 (RW) | 2 (WW)
+  benign_pair(rec_a, rec_b) -> 0 | 1   (benign W/W pair: kind 3 with check(..., benign=True), NEXT-4)
   validate(records) -> None or lowest bad index
   expand(flows) -> records  (canonical schedule order)
   oob(records, regions, index_base=0) -> (count, first_index or None)   out-of-bound check (NEXT-1)
@@ -59,10 +60,12 @@ def _load():
         P, U64, U32 = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32
         for name in ("oracle_check_brute", "oracle_check_grouped"):
             f = getattr(lib, name)
-            f.argtypes = [P, U64, U64, U32, U32, U32, P, U64, ctypes.POINTER(U64)]
+            f.argtypes = [P, U64, U64, U32, U32, U32, U32, P, U64, ctypes.POINTER(U64)]
             f.restype = ctypes.c_int
         lib.oracle_pair_kind.argtypes = [P, P, U32, U32]
         lib.oracle_pair_kind.restype = ctypes.c_int
+        lib.oracle_benign_pair.argtypes = [P, P]
+        lib.oracle_benign_pair.restype = ctypes.c_int
         lib.oracle_validate.argtypes = [P, U64, ctypes.POINTER(U64)]
         lib.oracle_validate.restype = ctypes.c_int
         lib.oracle_expand.argtypes = [P, U64, P, U64]
@@ -90,8 +93,9 @@ def _as_recs(records) -> np.ndarray:
 
 
 def check(records, index_base: int = 0, warp_size: int = 32, lockstep: int = 0, granularity: int = 4,
-          method: str = "grouped") -> np.ndarray:
-    """Canonical race list (sorted by (space, block, interval, addr, kind)) of ``records``."""
+          method: str = "grouped", benign: bool = False) -> np.ndarray:
+    """Canonical race list (sorted by (space, block, interval, addr, kind)) of ``records``; with ``benign`` also
+    one kind-3 record per location holding a benign W/W pair (config flags bit 0, oracle_benign_pair)."""
     lib = _load()
     r = _as_recs(records)
     fn = lib.oracle_check_brute if method == "brute" else lib.oracle_check_grouped
@@ -100,7 +104,7 @@ def check(records, index_base: int = 0, warp_size: int = 32, lockstep: int = 0, 
         out = np.zeros(cap, RACE_DTYPE)
         nout = ctypes.c_uint64(0)
         rc = fn(r.ctypes.data if len(r) else None, len(r), index_base, warp_size, lockstep, granularity,
-                out.ctypes.data, cap, ctypes.byref(nout))
+                1 if benign else 0, out.ctypes.data, cap, ctypes.byref(nout))
         if rc == 7:
             cap = int(nout.value)
             continue
@@ -120,6 +124,13 @@ def pair_kind(a, b, warp_size: int = 32, lockstep: int = 0) -> int:
     ra = _as_recs(np.asarray(a).reshape(1))
     rb = _as_recs(np.asarray(b).reshape(1))
     return int(lib.oracle_pair_kind(ra.ctypes.data, rb.ctypes.data, warp_size, lockstep))
+
+
+def benign_pair(a, b) -> int:
+    lib = _load()
+    ra = _as_recs(np.asarray(a).reshape(1))
+    rb = _as_recs(np.asarray(b).reshape(1))
+    return int(lib.oracle_benign_pair(ra.ctypes.data, rb.ctypes.data))
 
 
 def validate(records):

@@ -20,6 +20,7 @@
  *   oracle_check_grouped — group entries by location (qsort), per location decide "has a partner of kind K"
  *                          by COUNTING partners (inclusion-exclusion over sorted tuples), then witness
  *                          x = min flagged index, y = min s with P(x, s) of kind K.  O(n log n).
+ * With flag F_BENIGN both also report benign W/W pairs as a third kind (oracle_benign_pair).
  * They agree on every input (tests/test_oracle.py); the GPU path uses neither method (it uses per-run
  * min/max summaries), so agreement of the GPU with this oracle is not circular.
  *
@@ -59,7 +60,8 @@ typedef struct {
 
 enum { SH = 0, GL = 1 };            /* memory sorts: shared / global */
 enum { RD = 0, WR = 1, AT = 2 };    /* load, store, atomic intrinsic */
-enum { K_RW = 1, K_WW = 2 };        /* the WR and WW checks of P:79 */
+enum { K_RW = 1, K_WW = 2, K_WWB = 3 }; /* the WR and WW checks of P:79; K_WWB = a benign W/W pair */
+#define F_BENIGN 1u                 /* config flag: also report benign W/W pairs as kind K_WWB (NEXT-4) */
 #define NOBI 0xFFFFFFFFu            /* block/interval of a GLOBAL location (not part of λ) */
 
 /* ---- validity (the rules of include/sesa.h, independently restated) -------------------------------------
@@ -103,6 +105,19 @@ int oracle_pair_kind(const orec *r, const orec *s, uint32_t ws, uint32_t ls) {
   /* (6) benign W/W: two plain writes of the same value (Table IV "W/W (Benign)") */
   if (r->rw == WR && s->rw == WR && r->value_hash == s->value_hash) return 0;
   return kind;
+}
+
+/* ---- the benign W/W pair B(r, s) (reported only with F_BENIGN) --------------------------------------------
+ * Table IV reports "W/W (Benign)" verdicts (bfs, cutcp, spmv) and the conclusion "races later deemed to be
+ * benign": a write/write conflict that rule (6) above removes from the race set because both threads
+ * write the same value.  B(r, s) = both plain writes, equal value_hash, and every other condition of a W/W race:
+ * different threads (1) and unordered (4).  Rules (2), (3) hold for two plain writes; (5) exempts only pairs
+ * with a read.  Same precondition as oracle_pair_kind.                                                        */
+int oracle_benign_pair(const orec *r, const orec *s) {
+  if (r->rw != WR || s->rw != WR || r->value_hash != s->value_hash) return 0;
+  if (r->block == s->block && r->thread == s->thread) return 0;                      /* (1) */
+  if (r->space == GL && r->block == s->block && r->interval != s->interval) return 0; /* (4) */
+  return 1;
 }
 
 /* granule range of a record: [addr/G, (addr+size-1)/G]  (reading R1: overlap at granularity G) */
@@ -193,9 +208,9 @@ static int emit_sorted(cvec *c, uint32_t G, uint64_t base, orace *out, uint64_t 
 
 /* ---- checker 1: brute force over all pairs ---------------------------------------------------------------
  * return 0 ok, 1 invalid record (*nout = bad index), 2 bad config, 3 no memory, 7 truncated */
-int oracle_check_brute(const orec *r, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls, uint32_t G, orace *out,
-                       uint64_t cap, uint64_t *nout) {
-  if (!oracle_config_ok(ws, ls, G)) return 2;
+int oracle_check_brute(const orec *r, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls, uint32_t G,
+                       uint32_t flags, orace *out, uint64_t cap, uint64_t *nout) {
+  if (!oracle_config_ok(ws, ls, G) || (flags & ~F_BENIGN)) return 2;
   uint64_t bad;
   if (oracle_validate(r, n, &bad)) {
     *nout = bad;
@@ -214,6 +229,7 @@ int oracle_check_brute(const orec *r, uint64_t n, uint64_t base, uint32_t ws, ui
       uint64_t lo = ilo > jlo ? ilo : jlo, hi = ihi < jhi ? ihi : jhi;
       if (lo > hi) continue; /* no common granule */
       int kind = oracle_pair_kind(&r[i], &r[j], ws, ls);
+      if (!kind && (flags & F_BENIGN) && oracle_benign_pair(&r[i], &r[j])) kind = K_WWB;
       if (!kind) continue;
       for (uint64_t g = lo; g <= hi; g++) {
         cand x;
@@ -282,9 +298,10 @@ static uint64_t count_prefix(const tup *a, uint64_t k, const tup *q, int nf) {
  *          = (C[W,v] - C[W,v,b]) + (C[W,v,b,i] - C[W,v,b,i,t])
  * (same block, other interval is ordered for global memory and impossible for shared: never counted.)
  *   RW(r)  = r read:  Σ_{X∈{W,A}} OB(X) + (ls ? SW(X) : ST(X));  r write/atomic: OB(R) + (ls ? SW(R) : ST(R))
- *   WW(r)  = r write: OB(A)+ST(A) + OB(W)+ST(W) - EQ;  r atomic: OB(W)+ST(W);  r read: 0                   */
+ *   WW(r)  = r write: OB(A)+ST(A) + OB(W)+ST(W) - EQ;  r atomic: OB(W)+ST(W);  r read: 0
+ *   B(r)   = r write: EQ (its benign partners, oracle_benign_pair);  otherwise 0                              */
 static int group_flags(const orec *r, const entry *e, uint64_t k, uint32_t ws, uint32_t ls, uint8_t *flag_rw,
-                       uint8_t *flag_ww) {
+                       uint8_t *flag_ww, uint8_t *flag_b) {
   tup *A = (tup *)malloc(k * sizeof(tup)); /* (type, block, interval, thread) */
   tup *B = (tup *)malloc(k * sizeof(tup)); /* (type, block, interval, warp)   */
   tup *V = (tup *)malloc(k * sizeof(tup)); /* (type, value, block, interval, thread) */
@@ -319,7 +336,7 @@ static int group_flags(const orec *r, const entry *e, uint64_t k, uint32_t ws, u
       ST[X] = cXbi - cXbit;
       SW[X] = cXbi - cXbiw;
     }
-    uint64_t rw = 0, ww = 0;
+    uint64_t rw = 0, ww = 0, eq = 0;
     if (x->rw == RD) {
       rw = OB[WR] + (ls ? SW[WR] : ST[WR]) + OB[AT] + (ls ? SW[AT] : ST[AT]);
     } else {
@@ -330,21 +347,22 @@ static int group_flags(const orec *r, const entry *e, uint64_t k, uint32_t ws, u
       q.f[0] = WR; q.f[1] = x->value_hash; q.f[2] = x->block; q.f[3] = x->interval; q.f[4] = x->thread;
       uint64_t cv = count_prefix(V, k, &q, 2), cvb = count_prefix(V, k, &q, 3);
       uint64_t cvbi = count_prefix(V, k, &q, 4), cvbit = count_prefix(V, k, &q, 5);
-      uint64_t eq = (cv - cvb) + (cvbi - cvbit);
+      eq = (cv - cvb) + (cvbi - cvbit);
       ww = OB[AT] + ST[AT] + OB[WR] + ST[WR] - eq;
     } else if (x->rw == AT) {
       ww = OB[WR] + ST[WR];
     }
     flag_rw[a] = rw > 0;
     flag_ww[a] = ww > 0;
+    flag_b[a] = eq > 0;
   }
   free(A); free(B); free(V);
   return 0;
 }
 
-int oracle_check_grouped(const orec *r, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls, uint32_t G, orace *out,
-                         uint64_t cap, uint64_t *nout) {
-  if (!oracle_config_ok(ws, ls, G)) return 2;
+int oracle_check_grouped(const orec *r, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls, uint32_t G,
+                         uint32_t flags, orace *out, uint64_t cap, uint64_t *nout) {
+  if (!oracle_config_ok(ws, ls, G) || (flags & ~F_BENIGN)) return 2;
   uint64_t bad;
   if (oracle_validate(r, n, &bad)) {
     *nout = bad;
@@ -372,7 +390,7 @@ int oracle_check_grouped(const orec *r, uint64_t n, uint64_t base, uint32_t ws, 
   qsort(e, m, sizeof(entry), entry_cmp);
   cvec c = {0, 0, 0};
   int rc = 0;
-  uint8_t *frw = NULL, *fww = NULL;
+  uint8_t *frw = NULL, *fww = NULL, *fb = NULL;
   uint64_t fcap = 0;
   for (uint64_t a = 0; a < m && rc == 0;) {
     uint64_t b = a + 1;
@@ -380,15 +398,16 @@ int oracle_check_grouped(const orec *r, uint64_t n, uint64_t base, uint32_t ws, 
     uint64_t k = b - a; /* group [a, b): every entry at one λ, ascending record index */
     if (k >= 2) {
       if (k > fcap) {
-        free(frw); free(fww);
-        frw = (uint8_t *)malloc(k); fww = (uint8_t *)malloc(k);
+        free(frw); free(fww); free(fb);
+        frw = (uint8_t *)malloc(k); fww = (uint8_t *)malloc(k); fb = (uint8_t *)malloc(k);
         fcap = k;
-        if (!frw || !fww) { rc = 3; break; }
+        if (!frw || !fww || !fb) { rc = 3; break; }
       }
-      rc = group_flags(r, &e[a], k, ws, ls, frw, fww);
+      rc = group_flags(r, &e[a], k, ws, ls, frw, fww, fb);
       if (rc) break;
-      for (int K = K_RW; K <= K_WW; K++) {
-        const uint8_t *fl = K == K_RW ? frw : fww;
+      const int kmax = (flags & F_BENIGN) ? K_WWB : K_WW;
+      for (int K = K_RW; K <= kmax; K++) {
+        const uint8_t *fl = K == K_RW ? frw : K == K_WW ? fww : fb;
         uint64_t xa = UINT64_MAX; /* x = min flagged record index (entries are index-ascending) */
         for (uint64_t q = 0; q < k; q++)
           if (fl[q]) { xa = q; break; }
@@ -397,7 +416,8 @@ int oracle_check_grouped(const orec *r, uint64_t n, uint64_t base, uint32_t ws, 
         uint64_t y = UINT64_MAX; /* y = min partner of x of kind K */
         for (uint64_t q = 0; q < k; q++) {
           if (q == xa) continue;
-          if (oracle_pair_kind(x, &r[e[a + q].idx], ws, ls) == K) {
+          const orec *sq = &r[e[a + q].idx];
+          if (K == K_WWB ? oracle_benign_pair(x, sq) : oracle_pair_kind(x, sq, ws, ls) == K) {
             y = e[a + q].idx;
             break;
           }
@@ -413,7 +433,7 @@ int oracle_check_grouped(const orec *r, uint64_t n, uint64_t base, uint32_t ws, 
     }
     a = b;
   }
-  free(frw); free(fww); free(e);
+  free(frw); free(fww); free(fb); free(e);
   if (rc) {
     free(c.v);
     return rc;

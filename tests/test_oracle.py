@@ -407,3 +407,76 @@ def test_oob_boundaries_and_scope():
     two = np.concatenate([_region(100, 98), _region(198, 2)])
     assert O.oob(recs[1:2], two) == (1, 0)
     assert O.oob(recs, np.zeros(0, reg.dtype)) == (0, None)
+
+
+# ------------------------------------------------------------------------------------------------ benign W/W (NEXT-4)
+WWB = 3
+
+
+@pytest.mark.parametrize("method", ["brute", "grouped"])
+def test_f1_equal_values_benign_closed_form(method):
+    """race() of Fig. 2 with every thread writing the same value: the second interval's writes
+    v[t >> 2] = ... by the odd threads t = 4k+1, 4k+3 (k = 0..15) are W/W pairs of one value — filtered from the
+    race set (72 races, reading R18) and, with benign reporting on, reported as 16 kind-3 records, each witnessed
+    by its two writers (record 128 + t: interval 0 holds 2 x 64 records, interval 1 one per thread)."""
+    r = G.f1_race(distinct=False)
+    plain = O.check(r, method=method)
+    rep = O.check(r, method=method, benign=True)
+    assert len(plain) == 72 and len(rep) == 88
+    assert tuples(rep[rep["kind"] != WWB]) == tuples(plain)
+    exp = [(SH, 0, 1, 4 * k, WWB, 128 + 4 * k + 1, 128 + 4 * k + 3) for k in range(16)]
+    assert tuples(rep[rep["kind"] == WWB]) == exp
+    # distinct values: every such pair is a real W/W race (kind 2), none is benign
+    d = G.f1_race(distinct=True)
+    assert O.check(d, method=method, benign=True).tobytes() == O.check(d, method=method).tobytes()
+
+
+def test_benign_pair_rules():
+    # rows: (addr, value_hash, block, thread, interval, size, space, rw)
+    rows = [(0x30, 9, 0, 0, 0, 4, GL, 1), (0x30, 9, 1, 0, 0, 4, GL, 1),      # same value, other block: benign
+            (0x40, 9, 0, 0, 0, 4, GL, 1), (0x40, 8, 1, 0, 0, 4, GL, 1),      # other value: a real WW
+            (0x50, 9, 0, 0, 0, 4, GL, 1), (0x50, 9, 0, 0, 0, 4, GL, 1),      # same thread: never (P:287)
+            (0x60, 9, 0, 0, 0, 4, GL, 1), (0x60, 9, 0, 1, 1, 4, GL, 1),      # same block, other interval: ordered
+            (0x70, 9, 0, 0, 0, 4, GL, 1), (0x70, 9, 1, 1, 1, 4, GL, 1),      # other block: unordered -> benign
+            (0x80, 9, 0, 0, 0, 4, GL, 2), (0x80, 9, 1, 0, 0, 4, GL, 1),      # W-A: a real WW, never benign
+            (0x90, 9, 0, 0, 0, 4, GL, 0), (0x90, 9, 1, 0, 0, 4, GL, 1)]      # R-W: RW
+    rec = G.recs(rows)
+    got = tuples(O.check(rec, benign=True))
+    assert got == [(GL, NOBI, NOBI, 0x30, WWB, 0, 1), (GL, NOBI, NOBI, 0x40, WW, 2, 3),
+                   (GL, NOBI, NOBI, 0x70, WWB, 8, 9), (GL, NOBI, NOBI, 0x80, WW, 10, 11),
+                   (GL, NOBI, NOBI, 0x90, RW, 12, 13)]
+    assert O.benign_pair(rec[0], rec[1]) == 1 and O.benign_pair(rec[10], rec[11]) == 0
+    # lockstep exempts only pairs with a read: an intra-warp benign pair stays benign
+    assert tuples(O.check(rec[:2], benign=True, lockstep=1)) == [(GL, NOBI, NOBI, 0x30, WWB, 0, 1)]
+
+
+@pytest.mark.parametrize("cfg", CONFIGS)
+def test_benign_brute_equals_grouped_random(cfg):
+    for seed in range(40):
+        n = 1 + (seed * 11) % 120
+        r = G.random_trace(n, seed + 500, threads=6 + seed % 20, values=2, write_frac=0.6, atomic_frac=0.1,
+                           sort=seed % 3 != 0)
+        kw = dict(warp_size=cfg["ws"], lockstep=cfg["ls"], granularity=cfg["G"], benign=True)
+        a = O.check(r, method="brute", **kw)
+        b = O.check(r, method="grouped", **kw)
+        assert a.tobytes() == b.tobytes(), (cfg, seed)
+        # reporting adds kind-3 records and changes nothing else
+        base = O.check(r, warp_size=cfg["ws"], lockstep=cfg["ls"], granularity=cfg["G"])
+        assert a[a["kind"] != WWB].tobytes() == base.tobytes()
+        for x in a[a["kind"] == WWB]:
+            assert O.benign_pair(r[int(x["first"])], r[int(x["second"])]) == 1
+
+
+def test_bfs_shape_is_benign_ww():
+    """Table IV reports the Lonestar BFS kernel as "W/W (Benign)": every thread that relaxes a node
+    writes the same level, so its write/write conflicts are all benign.  The C4 recipe at 2^10 nodes: with
+    benign reporting the trace holds benign W/W records (at `changed` and at dist[] entries written by several
+    frontier threads) and no real W/W race."""
+    from sesagen import configs as GC
+    c4 = GC.C4(log2n=10)
+    r = c4.host()
+    got = O.check(r, lockstep=1, benign=True)
+    kinds = set(got["kind"].tolist())
+    assert WW not in kinds and WWB in kinds
+    changed = int(c4.cfg().changed_base)
+    assert any(int(x["addr"]) == changed and int(x["kind"]) == WWB for x in got)
