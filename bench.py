@@ -216,6 +216,8 @@ def main():
     ap.add_argument("--ref-records", type=int, default=1 << 23)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--benign", action="store_true",
+                    help="also report benign W/W locations (flags bit 0, kind 3; single GPU)")
     ap.add_argument("--force-dist", action="store_true",
                     help="use the NCCL distributed handle even with one rank (exercises the N>1 code path)")
     args = ap.parse_args()
@@ -242,7 +244,7 @@ def main():
         dist.broadcast_object_list(obj, src=0)
         trace = S.Trace(c["ws"], c["ls"], 4, dist=(rank, world, obj[0]))
     else:
-        trace = S.Trace(c["ws"], c["ls"], 4)
+        trace = S.Trace(c["ws"], c["ls"], 4, benign=args.benign)
 
     recs, n_local, base, n_total = make_records(args.config, args.records, rank, world)
     torch.cuda.synchronize()
@@ -341,7 +343,8 @@ def main():
                            if n_total * 32 > 1e9 else "inputs smaller than L2 (latency-bound config)",
                            "sort_bits": info["sort_bits"], "sort_passes": info["sort_passes"],
                            "races": n_races, "crossing_tiles": info["crossing_tiles"],
-                           "entries_at_multi_entry_locations": info["n_multi"], "fused_first_pass": bool(info["fused_first_pass"])},
+                           "entries_at_multi_entry_locations": info["n_multi"], "fused_first_pass": bool(info["fused_first_pass"]),
+                           "report_benign": bool(args.benign)},
                 "gpu_launches": launches, "roofline": roof,
                 "honesty": {"record_bytes_per_step": n_total * 32, "achieved_gbs_vs_32B_per_record":
                             n_total * 32 / (ms / args.steps / 1e3) / 1e9,

@@ -64,15 +64,24 @@ typedef enum {
 enum { SESA_SPACE_SHARED = 0, SESA_SPACE_GLOBAL = 1 };
 /* access kinds: load -> READ, store -> WRITE (Fig. 3); any atomic RMW intrinsic -> ATOMIC */
 enum { SESA_READ = 0, SESA_WRITE = 1, SESA_ATOMIC = 2 };
-/* race kinds ("WW (Write-Write)" and "WR" checks) */
-enum { SESA_RACE_RW = 1, SESA_RACE_WW = 2 };
+/* race kinds ("WW (Write-Write)" and "WR" checks).  SESA_RACE_WW_BENIGN is reported only with
+ * SESA_FLAG_REPORT_BENIGN (Table IV "W/W (Benign)" verdicts; "races later deemed to
+ * be benign"): a location holding a benign pair = two plain WRITEs with equal value_hash that satisfy
+ * rules (1) and (4) above (rules (2), (3) hold for two plain writes; (5) exempts only pairs with a READ).  One
+ * record per such location, witnessed by the lexicographically smallest benign pair; rule (6) still keeps
+ * these pairs out of SESA_RACE_WW, so a location may carry both a WW and a WW_BENIGN record. */
+enum { SESA_RACE_RW = 1, SESA_RACE_WW = 2, SESA_RACE_WW_BENIGN = 3 };
+/* sesa_config.flags bits */
+enum { SESA_FLAG_REPORT_BENIGN = 1 };
 
 typedef struct {
   uint32_t warp_size;   /* >= 1.  32 = CUDA warp ("groups of 32 consecutively numbered threads");
                            1 = no warp semantics.  warp(r) = r.thread / warp_size              */
   uint32_t lockstep;    /* 0 | 1.  1 = exempt intra-warp pairs with a READ (R6-R8)    */
   uint32_t granularity; /* power of two in [1, 4096]: bytes per comparison unit; 1 = exact byte overlap */
-  uint32_t flags;       /* must be 0 in ABI v1                                                          */
+  uint32_t flags;       /* SESA_FLAG_* bits; others must be 0.  SESA_FLAG_REPORT_BENIGN: also report benign
+                           W/W locations (kind SESA_RACE_WW_BENIGN); single-GPU handles only
+                           (sesa_trace_create_dist / sesa_race_check_loopback return SESA_EINVAL)          */
 } sesa_config;
 
 /* One concrete access: the paper's race-state entry `c ? r|w(a)` of one thread.
@@ -158,7 +167,7 @@ typedef struct {
 } sesa_check_info;
 
 /* Create a single-GPU handle on the current CUDA device.  cfg is validated (EINVAL on warp_size 0,
- * lockstep > 1, granularity not a power of 2 or > 4096, flags != 0).  *out = NULL on error. */
+ * lockstep > 1, granularity not a power of 2 or > 4096, unknown flags bits).  *out = NULL on error. */
 sesa_status sesa_trace_create(const sesa_config *cfg, sesa_trace **out);
 
 /* Collective: create a handle that is rank `rank` of `world` (one process per GPU).  nccl_unique_id is the

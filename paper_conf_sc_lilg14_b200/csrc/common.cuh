@@ -24,7 +24,7 @@ namespace sesa {
 
 enum { SP_SHARED = 0, SP_GLOBAL = 1 };
 enum { RW_READ = 0, RW_WRITE = 1, RW_ATOMIC = 2 };
-enum { KIND_RW = 1, KIND_WW = 2 };
+enum { KIND_RW = 1, KIND_WW = 2, KIND_WWB = 3 };  // KIND_WWB: benign W/W (reported with flags bit 0)
 static constexpr u32 NOBI = 0xFFFFFFFFu;
 
 // Device-side view of one 32-byte access record (layout of sesa_access, include/sesa.h).

@@ -529,6 +529,7 @@ sesa_status sesa_trace_create_dist(const sesa_config* cfg, int rank, int world, 
   if (!out) return SESA_EINVAL;
   *out = nullptr;
   if (!uid || world < 1 || world > 8 || rank < 0 || rank >= world) return SESA_EINVAL;
+  if (cfg && (cfg->flags & SESA_FLAG_REPORT_BENIGN)) return SESA_EINVAL;  // benign reporting: single GPU in v1
   sesa_trace* t = nullptr;
   sesa_status s = sesa_trace_create(cfg, &t);
   if (s != SESA_OK) return s;
@@ -554,6 +555,7 @@ sesa_status sesa_race_check_loopback(const sesa_config* cfg, const sesa_access* 
                                      int world, uint64_t index_base, void* stream, sesa_trace** out) {
   if (!out || !offs || world < 1 || world > 8) return SESA_EINVAL;
   *out = nullptr;
+  if (cfg && (cfg->flags & SESA_FLAG_REPORT_BENIGN)) return SESA_EINVAL;  // benign reporting: single GPU in v1
   std::vector<sesa_trace*> ts(world, nullptr);
   for (int r = 0; r < world; r++) {
     sesa_status s = sesa_trace_create(cfg, &ts[r]);

@@ -509,7 +509,7 @@ __device__ void emit_race(const ConflictArgs& a, u64 head_hi, u32 kind, u32 x, u
 #pragma unroll
   for (int i = 0; i < 6; i++) r.reserved[i] = 0;
   a.races[idx] = r;
-  a.race_keys[idx] = (group_of_hi(L, head_hi) << 1) | (kind - 1);
+  a.race_keys[idx] = (group_of_hi(L, head_hi) << 2) | (kind - 1);  // 2 kind bits: RW, WW, benign WW
   a.race_vals[idx] = idx;
 }
 
@@ -942,7 +942,7 @@ __global__ void race_rekey_kernel(const RaceOut* __restrict__ r, u64 n, KeyLayou
   // global races carry block = interval = NOBI: use the layout minima so the (masked) low fields stay zero
   const bool glob = x.space == SP_GLOBAL;
   const u64 hi = key_hi_of(L, x.space, glob ? L.bminG : x.block, glob ? L.iminG : x.interval, x.addr >> L.log2G);
-  keys[i] = (group_of_hi(L, hi) << 1) | (u64)(x.kind - 1);
+  keys[i] = (group_of_hi(L, hi) << 2) | (u64)(x.kind - 1);
   vals[i] = (u32)i;
 }
 
@@ -958,6 +958,143 @@ __global__ void permute_races_kernel(const RaceOut* __restrict__ in, const u32* 
 
 void launch_permute_races(const RaceOut* in, const u32* order, RaceOut* out, u32 nr, cudaStream_t st) {
   if (nr) permute_races_kernel<<<(nr + 255) / 256, 256, 0, st>>>(in, order, out, nr);
+}
+
+
+// ------------------------------------------------------------------------------------------------ benign W/W
+// SURVEY §8f NEXT-4 (Table IV "W/W (Benign)" P:467): with SESA_FLAG_REPORT_BENIGN every location holding a
+// benign pair — two plain writes of one value by different threads, unordered — gets one kind-3 record.  "Exists
+// a plain write with another identity AND the same value" is not a min/max summary query, so the plain writes
+// of multi-entry locations are regrouped by (location, value) (sort by value, then stable by location ordinal)
+// and become a DERIVED trace: one plain write per entry, location = its (location, value) run, distinct values.
+// A W/W race of the derived trace (the ordinary pipeline, rule (6) never fires) is exactly a benign pair of the
+// original, and because a run lists its entries in original position order the derived witness maps to the
+// original lexicographic minimum; the minimum over a location's runs is taken with one atomicMin per race.
+
+// head flag (first entry of a location run) and plain-write flag of every compacted entry
+__global__ void benign_mark_kernel(const u64* __restrict__ comp, u32 m2, KeyLayout L, const Rec* __restrict__ rec,
+                                   u32* __restrict__ head, u32* __restrict__ wflag) {
+  const u32 j = blockIdx.x * blockDim.x + threadIdx.x;
+  if (j >= m2) return;
+  const u64 k = comp[j];
+  head[j] = (j == 0 || group_of_hi(L, k >> L.pos_bits) != group_of_hi(L, comp[j - 1] >> L.pos_bits)) ? 1u : 0u;
+  wflag[j] = rec[pos_of(L, k)].rw == RW_WRITE ? 1u : 0u;  // rw byte of the record (byte 31)
+}
+
+// plain writes -> (value, entry) pairs at their exclusive write rank; location ordinal of every entry
+__global__ void benign_gather_kernel(const u64* __restrict__ comp, u32 m2, KeyLayout L, const Rec* __restrict__ rec,
+                                     const u32* __restrict__ head, const u32* __restrict__ hscan,
+                                     const u32* __restrict__ wflag, const u32* __restrict__ wscan,
+                                     u32* __restrict__ gid, u64* __restrict__ vkey, u32* __restrict__ vidx) {
+  const u32 j = blockIdx.x * blockDim.x + threadIdx.x;
+  if (j >= m2) return;
+  gid[j] = hscan[j] + head[j] - 1;
+  if (wflag[j]) {
+    vkey[wscan[j]] = rec[pos_of(L, comp[j])].vh;
+    vidx[wscan[j]] = j;
+  }
+}
+
+// sort keys of the plain-write list (entry vidx[i]): 0 = original position, 1 = value hash, 2 = location ordinal
+__global__ void benign_keys_kernel(const u64* __restrict__ comp, KeyLayout L, const Rec* __restrict__ rec,
+                                   const u32* __restrict__ vidx, u32 m3, const u32* __restrict__ gid, int what,
+                                   u64* __restrict__ keys) {
+  const u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= m3) return;
+  const u32 j = vidx[i];
+  keys[i] = what == 2 ? (u64)gid[j] : what == 0 ? (u64)pos_of(L, comp[j]) : rec[pos_of(L, comp[j])].vh;
+}
+
+// run heads of the (location, value) order
+__global__ void benign_runs_kernel(const u64* __restrict__ comp, KeyLayout L, const Rec* __restrict__ rec,
+                                   const u32* __restrict__ gid, const u32* __restrict__ order, u32 m3,
+                                   u32* __restrict__ rhead) {
+  const u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= m3) return;
+  const u32 j = order[i];
+  bool h = i == 0;
+  if (!h) {
+    const u32 jp = order[i - 1];
+    h = gid[jp] != gid[j] || rec[pos_of(L, comp[jp])].vh != rec[pos_of(L, comp[j])].vh;
+  }
+  rhead[i] = h ? 1u : 0u;
+}
+
+// derived trace: record i = plain write of entry order[i] at location (its space, block, interval, run id) with
+// granularity 1 and the distinct value i + 1; dpos[i] = original position, dj[i] = entry
+__global__ void benign_derive_kernel(const u64* __restrict__ comp, KeyLayout L, const Rec* __restrict__ rec,
+                                     const u32* __restrict__ order, const u32* __restrict__ rhead,
+                                     const u32* __restrict__ rscan, u32 m3, Rec* __restrict__ out,
+                                     u32* __restrict__ dpos, u32* __restrict__ dj) {
+  const u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= m3) return;
+  const u32 j = order[i];
+  const u32 p = pos_of(L, comp[j]);
+  const Rec r = load_rec(rec + p);
+  Rec d = r;
+  d.addr = rscan[i] + rhead[i] - 1;
+  d.vh = (u64)i + 1;
+  d.size = 1;
+  d.rw = RW_WRITE;
+  out[i] = d;
+  dpos[i] = p;
+  dj[i] = j;
+}
+
+// child W/W races -> per location the lexicographic minimum (first << 32 | second) of original positions
+__global__ void benign_min_kernel(const RaceOut* __restrict__ cr, u32 nc, const u32* __restrict__ dpos,
+                                  const u32* __restrict__ dj, const u32* __restrict__ gid,
+                                  unsigned long long* __restrict__ slot) {
+  const u32 c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= nc) return;
+  const RaceOut x = cr[c];
+  const unsigned long long v = ((unsigned long long)dpos[x.first] << 32) | dpos[x.second];
+  atomicMin(&slot[gid[dj[x.first]]], v);
+}
+
+__global__ void benign_emit_kernel(ConflictArgs a, const RaceOut* __restrict__ cr, u32 nc,
+                                   const u32* __restrict__ dpos, const u32* __restrict__ dj,
+                                   const u32* __restrict__ gid, const unsigned long long* __restrict__ slot) {
+  const u32 c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= nc) return;
+  const RaceOut x = cr[c];
+  const u32 j = dj[x.first];
+  const unsigned long long v = ((unsigned long long)dpos[x.first] << 32) | dpos[x.second];
+  if (slot[gid[j]] != v) return;  // pairs are unique per location: exactly one child race wins
+  const u64 k = a.keys[j];
+  const Rec r = load_rec(a.rec + pos_of(a.L, k));
+  emit_race(a, k >> a.L.pos_bits, KIND_WWB, dpos[x.first], dpos[x.second], r.block, r.interval);
+}
+
+void launch_benign_mark(const u64* comp, u32 m2, const KeyLayout& L, const Rec* rec, u32* head, u32* wflag,
+                        cudaStream_t st) {
+  if (m2) benign_mark_kernel<<<(m2 + 255) / 256, 256, 0, st>>>(comp, m2, L, rec, head, wflag);
+}
+void launch_benign_gather(const u64* comp, u32 m2, const KeyLayout& L, const Rec* rec, const u32* head,
+                          const u32* hscan, const u32* wflag, const u32* wscan, u32* gid, u64* vkey, u32* vidx,
+                          cudaStream_t st) {
+  if (m2)
+    benign_gather_kernel<<<(m2 + 255) / 256, 256, 0, st>>>(comp, m2, L, rec, head, hscan, wflag, wscan, gid, vkey,
+                                                           vidx);
+}
+void launch_benign_keys(const u64* comp, const KeyLayout& L, const Rec* rec, const u32* vidx, u32 m3, const u32* gid,
+                        int what, u64* keys, cudaStream_t st) {
+  if (m3) benign_keys_kernel<<<(m3 + 255) / 256, 256, 0, st>>>(comp, L, rec, vidx, m3, gid, what, keys);
+}
+void launch_benign_runs(const u64* comp, const KeyLayout& L, const Rec* rec, const u32* gid, const u32* order,
+                        u32 m3, u32* rhead, cudaStream_t st) {
+  if (m3) benign_runs_kernel<<<(m3 + 255) / 256, 256, 0, st>>>(comp, L, rec, gid, order, m3, rhead);
+}
+void launch_benign_derive(const u64* comp, const KeyLayout& L, const Rec* rec, const u32* order, const u32* rhead,
+                          const u32* rscan, u32 m3, Rec* out, u32* dpos, u32* dj, cudaStream_t st) {
+  if (m3)
+    benign_derive_kernel<<<(m3 + 255) / 256, 256, 0, st>>>(comp, L, rec, order, rhead, rscan, m3, out, dpos, dj);
+}
+void launch_benign_min_emit(const ConflictArgs& a, const RaceOut* cr, u32 nc, const u32* dpos, const u32* dj,
+                            const u32* gid, unsigned long long* slot, cudaStream_t st) {
+  if (!nc) return;
+  benign_min_kernel<<<(nc + 255) / 256, 256, 0, st>>>(cr, nc, dpos, dj, gid, slot);
+  benign_emit_kernel<<<(nc + 255) / 256, 256, 0, st>>>(a, cr, nc, dpos, dj, gid, slot);
 }
 
 }  // namespace sesa

@@ -52,6 +52,19 @@ bool sesa_trace::grow(DevBuf& b, size_t bytes, const char* what) {
   return true;
 }
 
+bool sesa_trace::grow_keep(DevBuf& b, size_t bytes, size_t used, const char* what) {
+  if (b.cap >= bytes) return true;
+  void* p = nullptr;
+  const size_t want = std::max<size_t>(bytes, 256);
+  if (!cuda_ok(cudaMalloc(&p, want), what)) return false;
+  if (used && b.p && !cuda_ok(cudaMemcpyAsync(p, b.p, std::min(used, b.cap), cudaMemcpyDeviceToDevice, stream), what))
+    return false;
+  if (b.p) cudaFree(b.p);  // (synchronises: the copy has completed)
+  b.p = p;
+  b.cap = want;
+  return true;
+}
+
 void sesa_trace::free_all() {
   for (DevBuf* b : all_bufs())
     if (b->p) cudaFree(b->p), b->p = nullptr, b->cap = 0;
@@ -444,11 +457,163 @@ bool sesa_trace::step_conflict(const u64* comp, u32 m2, const Rec* rec, u32 rec_
   return fail(SESA_ECUDA, "race list did not fit after retries"), false;
 }
 
+// (u64 key, u32 value) pairs sorted stably by the low `bits` key bits (onesweep key/value passes, trivial
+// digits skipped); *which = 0 if the result is in (k0, v0), 1 if in (k1, v1)
+bool sesa_trace::sort_kv(u64* k0, u32* v0, u64* k1, u32* v1, u32 n, u32 bits, int* which) {
+  *which = 0;
+  const u32 npass = (bits + RADIX_BITS - 1) / RADIX_BITS;
+  if (n == 0 || npass == 0) return true;
+  const u32 tiles = sort_tiles(n);
+  if (!grow(b_rhist, (size_t)npass * RADIX * 4, "kv hist") || !grow(b_rbase, (size_t)npass * RADIX * 8, "kv base") ||
+      !grow(b_lookback, (size_t)tiles * RADIX * 8, "lookback") || !grow(b_ctr, 64 * 4, "counters"))
+    return false;
+  if (b_lookback.cap != lookback_cleared) {
+    cudaMemsetAsync(b_lookback.p, 0, b_lookback.cap, stream);
+    lookback_cleared = b_lookback.cap;
+    epoch = 0;
+  }
+  cudaMemsetAsync(b_rhist.p, 0, (size_t)npass * RADIX * 4, stream);
+  cudaMemsetAsync((u32*)b_ctr.p + 32, 0, 32 * 4, stream);
+  LAUNCH("kv_hist", 8.0 * n, launch_hist_keys(k0, n, npass, (u32*)b_rhist.p, stream));
+  LAUNCH("bin_base", 0.0, launch_bin_base((u32*)b_rhist.p, (u64*)b_rbase.p, npass, stream));
+  std::vector<u32> h((size_t)npass * RADIX);
+  if (!cuda_ok(cudaMemcpyAsync(h.data(), b_rhist.p, h.size() * 4, cudaMemcpyDeviceToHost, stream), "kv hist") ||
+      !sync_check("kv hist"))
+    return false;
+  u64* k[2] = {k0, k1};
+  u32* v[2] = {v0, v1};
+  int c = 0;
+  for (u32 p = 0; p < npass; p++) {
+    if (*std::max_element(h.data() + (size_t)p * RADIX, h.data() + (size_t)(p + 1) * RADIX) == n) continue;
+    if (++epoch >= 256) {
+      cudaMemsetAsync(b_lookback.p, 0, b_lookback.cap, stream);
+      epoch = 1;
+    }
+    LAUNCH("kv_sort", 24.0 * n,
+           launch_onesweep(k[c], k[c ^ 1], v[c], v[c ^ 1], n, p * RADIX_BITS, (u64*)b_rbase.p + (size_t)p * RADIX,
+                           (u64*)b_lookback.p, (u32*)b_ctr.p + 32 + p, epoch, stream));
+    c ^= 1;
+  }
+  *which = c;
+  return true;
+}
+
+// step 5b (flags bit 0): benign W/W records, appended to the unsorted race list
+// (k_conflict.cu "benign W/W" has the method).  n_races grows by the locations holding a benign pair.
+bool sesa_trace::step_benign(const u64* comp, u32 m2, const Rec* rec, u64 index_base) {
+  if (!(cfg.flags & SESA_FLAG_REPORT_BENIGN) || m2 < 2) return true;
+  const KeyLayout& L = layout;
+  if (!grow(b_bhead, (size_t)m2 * 4, "benign") || !grow(b_bhscan, (size_t)m2 * 4, "benign") ||
+      !grow(b_bwf, (size_t)m2 * 4, "benign") || !grow(b_bwscan, (size_t)m2 * 4, "benign") ||
+      !grow(b_bgid, (size_t)m2 * 4, "benign") || !grow(b_temp, scan_u32_temp_bytes(m2), "scan"))
+    return false;
+  LAUNCH("benign_mark", 16.0 * m2, launch_benign_mark(comp, m2, L, rec, (u32*)b_bhead.p, (u32*)b_bwf.p, stream));
+  LAUNCH("scan", 8.0 * m2, launch_scan_exclusive_u32((u32*)b_bhead.p, (u32*)b_bhscan.p, m2, b_temp.p, stream));
+  LAUNCH("scan", 8.0 * m2, launch_scan_exclusive_u32((u32*)b_bwf.p, (u32*)b_bwscan.p, m2, b_temp.p, stream));
+  u32 tail[4];
+  cudaMemcpyAsync(&tail[0], (u32*)b_bwscan.p + m2 - 1, 4, cudaMemcpyDeviceToHost, stream);
+  cudaMemcpyAsync(&tail[1], (u32*)b_bwf.p + m2 - 1, 4, cudaMemcpyDeviceToHost, stream);
+  cudaMemcpyAsync(&tail[2], (u32*)b_bhscan.p + m2 - 1, 4, cudaMemcpyDeviceToHost, stream);
+  cudaMemcpyAsync(&tail[3], (u32*)b_bhead.p + m2 - 1, 4, cudaMemcpyDeviceToHost, stream);
+  if (!sync_check("benign counts")) return false;
+  const u32 m3 = tail[0] + tail[1], ngroups = tail[2] + tail[3];
+  if (m3 < 2) return true;
+  if (!grow(b_bvk[0], (size_t)m3 * 8, "benign") || !grow(b_bvk[1], (size_t)m3 * 8, "benign") ||
+      !grow(b_bvi[0], (size_t)m3 * 4, "benign") || !grow(b_bvi[1], (size_t)m3 * 4, "benign") ||
+      !grow(b_brh, (size_t)m3 * 4, "benign") || !grow(b_brscan, (size_t)m3 * 4, "benign") ||
+      !grow(b_bder, (size_t)m3 * sizeof(Rec), "benign") || !grow(b_bdpos, (size_t)m3 * 4, "benign") ||
+      !grow(b_bdj, (size_t)m3 * 4, "benign") || !grow(b_bslot, (size_t)ngroups * 8, "benign") ||
+      !grow(b_temp, scan_u32_temp_bytes(m3), "scan"))
+    return false;
+  LAUNCH("benign_gather", 24.0 * m2,
+         launch_benign_gather(comp, m2, L, rec, (const u32*)b_bhead.p, (const u32*)b_bhscan.p, (const u32*)b_bwf.p,
+                              (const u32*)b_bwscan.p, (u32*)b_bgid.p, (u64*)b_bvk[0].p, (u32*)b_bvi[0].p, stream));
+  // stable LSD passes over the plain-write list -> (location, value, position) order.  Entries of a location
+  // are already position-ordered unless global keys carry (block, interval) below the granule (input not in
+  // (block, interval) order, lowG > 0): then a position sort comes first.
+  int w = 0;
+  if (L.lowG != 0) {
+    LAUNCH("benign_keys", 12.0 * m3,
+           launch_benign_keys(comp, L, rec, (const u32*)b_bvi[0].p, m3, (const u32*)b_bgid.p, 0, (u64*)b_bvk[0].p,
+                              stream));
+    if (!sort_kv((u64*)b_bvk[0].p, (u32*)b_bvi[0].p, (u64*)b_bvk[1].p, (u32*)b_bvi[1].p, m3, L.pos_bits, &w))
+      return false;
+    LAUNCH("benign_keys", 40.0 * m3,
+           launch_benign_keys(comp, L, rec, (const u32*)b_bvi[w].p, m3, (const u32*)b_bgid.p, 1, (u64*)b_bvk[w].p,
+                              stream));
+  }
+  int w1 = 0;
+  if (!sort_kv((u64*)b_bvk[w].p, (u32*)b_bvi[w].p, (u64*)b_bvk[w ^ 1].p, (u32*)b_bvi[w ^ 1].p, m3, 64, &w1))
+    return false;
+  w ^= w1;
+  LAUNCH("benign_keys", 12.0 * m3,
+         launch_benign_keys(comp, L, rec, (const u32*)b_bvi[w].p, m3, (const u32*)b_bgid.p, 2, (u64*)b_bvk[w].p,
+                            stream));
+  u32 gbits = 0;
+  while (gbits < 32 && (1ull << gbits) < ngroups) gbits++;
+  int w2 = 0;
+  if (!sort_kv((u64*)b_bvk[w].p, (u32*)b_bvi[w].p, (u64*)b_bvk[w ^ 1].p, (u32*)b_bvi[w ^ 1].p, m3, gbits, &w2))
+    return false;
+  const u32* order = (const u32*)(w2 ? b_bvi[w ^ 1].p : b_bvi[w].p);
+  LAUNCH("benign_runs", 24.0 * m3,
+         launch_benign_runs(comp, L, rec, (const u32*)b_bgid.p, order, m3, (u32*)b_brh.p, stream));
+  LAUNCH("scan", 8.0 * m3, launch_scan_exclusive_u32((u32*)b_brh.p, (u32*)b_brscan.p, m3, b_temp.p, stream));
+  LAUNCH("benign_derive", 80.0 * m3,
+         launch_benign_derive(comp, L, rec, order, (const u32*)b_brh.p, (const u32*)b_brscan.p, m3, (Rec*)b_bder.p,
+                              (u32*)b_bdpos.p, (u32*)b_bdj.p, stream));
+  if (!sync_check("benign derive")) return false;
+  // the derived trace: plain writes with distinct values at (location, value) runs, granularity 1
+  if (!child) {
+    sesa_config cc = cfg;
+    cc.granularity = 1;
+    cc.flags = 0;
+    if (sesa_trace_create(&cc, &child) != SESA_OK) return fail(SESA_ENOMEM, "benign child handle"), false;
+  }
+  child->stream = stream;
+  child->profiling = false;
+  const sesa_status cs = child->check_device((const sesa_access*)b_bder.p, m3, 0);
+  launches += child->launches;
+  if (cs != SESA_OK) return fail(cs, "benign derived check: %s", child->err.c_str()), false;
+  const u32 nc = (u32)child->n_races;
+  if (nc == 0) return true;
+  // append: keep the n_races records already emitted, grow for nc more
+  const u64 need = n_races + nc;
+  if (!grow_keep(b_races, need * sizeof(RaceOut), n_races * sizeof(RaceOut), "races") ||
+      !grow_keep(b_rkeys[0], need * 8, n_races * 8, "race keys") ||
+      !grow_keep(b_rvals[0], need * 4, n_races * 4, "race vals") || !grow(b_rkeys[1], need * 8, "race keys") ||
+      !grow(b_rvals[1], need * 4, "race vals") || !grow(b_ccount, 16, "ccount"))
+    return false;
+  const u32 nr0 = (u32)n_races;
+  cudaMemcpyAsync(b_ccount.p, &nr0, 4, cudaMemcpyHostToDevice, stream);
+  cudaMemsetAsync(b_bslot.p, 0xFF, (size_t)ngroups * 8, stream);
+  ConflictArgs A;
+  memset(&A, 0, sizeof A);
+  A.keys = comp;
+  A.m = m2;
+  A.rec = rec;
+  A.L = layout;
+  A.race_count = (u32*)b_ccount.p;
+  A.race_keys = (u64*)b_rkeys[0].p;
+  A.race_vals = (u32*)b_rvals[0].p;
+  A.races = (RaceOut*)b_races.p;
+  A.race_cap = (u32)need;
+  A.index_base = index_base;
+  LAUNCH("benign_emit", 0.0,
+         launch_benign_min_emit(A, (const RaceOut*)child->b_races_sorted.p, nc, (const u32*)b_bdpos.p,
+                                (const u32*)b_bdj.p, (const u32*)b_bgid.p, (unsigned long long*)b_bslot.p, stream));
+  u32 total = 0;
+  if (!cuda_ok(cudaMemcpyAsync(&total, b_ccount.p, 4, cudaMemcpyDeviceToHost, stream), "benign count") ||
+      !sync_check("benign emit"))
+    return false;
+  n_races = total;
+  return true;
+}
+
 // step 6: canonical order of nr races: sort (location key << 1 | kind, index), permute into `out`
 bool sesa_trace::step_race_sort(u32 nr, const RaceOut* races, u64* rkeys0, u32* rvals0, u64* rkeys1, u32* rvals1,
                                 RaceOut* out) {
   if (nr == 0) return true;
-  const u32 rbits = layout.sort_bits + 1;
+  const u32 rbits = layout.sort_bits + 2;  // race key = location << 2 | (kind - 1)
   const u32 rpass = (rbits + RADIX_BITS - 1) / RADIX_BITS;
   const u32 rtiles = sort_tiles(nr);
   if (!grow(b_rhist, (size_t)rpass * RADIX * 4, "race hist") || !grow(b_rbase, (size_t)rpass * RADIX * 8, "race base") ||
@@ -516,6 +681,7 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
   u32 m2 = 0;
   if (!step_compact(cur, m, &comp, &m2)) return status;
   if (!step_conflict(comp, m2, rec, 0, nullptr, index_base)) return status;
+  if (!step_benign(comp, m2, rec, index_base)) return status;
   const u32 nr = (u32)n_races;
   info.n_races = nr;
   if (!grow(b_races_sorted, (size_t)std::max(nr, 1u) * sizeof(RaceOut), "sorted races")) return status;
@@ -629,7 +795,7 @@ const char* sesa_status_str(sesa_status s) {
 static sesa_status check_cfg(const sesa_config* c) {
   if (!c) return SESA_EINVAL;
   if (c->warp_size < 1 || c->lockstep > 1 || c->granularity < 1 || c->granularity > 4096 ||
-      (c->granularity & (c->granularity - 1)) || c->flags != 0)
+      (c->granularity & (c->granularity - 1)) || (c->flags & ~(uint32_t)SESA_FLAG_REPORT_BENIGN) != 0)
     return SESA_EINVAL;
   return SESA_OK;
 }
@@ -769,6 +935,7 @@ sesa_status sesa_trace_kernel_stats(const sesa_trace* t, sesa_kernel_stat* out, 
 void sesa_trace_destroy(sesa_trace* t) {
   if (!t) return;
   t->destroy_dist();
+  if (t->child) sesa_trace_destroy(t->child), t->child = nullptr;
   t->free_all();
   delete t;
 }

@@ -46,6 +46,10 @@ struct sesa_trace {
   bool have_thist = false;  // extents wrote per-tile raw digit histograms (fused first pass possible)
   // out-of-bound check (NEXT-1): registered regions (sorted by space, base) and the last report
   DevBuf b_regions;
+  // benign W/W reporting (flags bit 0): regrouped plain writes and the derived trace checked by `child`
+  DevBuf b_bhead, b_bhscan, b_bwf, b_bwscan, b_bgid, b_bvk[2], b_bvi[2], b_brh, b_brscan, b_bder, b_bdpos, b_bdj,
+      b_bslot, b_btmp;
+  sesa_trace* child = nullptr;
   uint32_t n_regions = 0, n_regions_shared = 0;
   sesa_oob_report oob{};
   bool have_oob = false;
@@ -56,7 +60,9 @@ struct sesa_trace {
     std::vector<DevBuf*> v = {&b_summary, &b_hist, &b_binbase, &b_lookback, &b_ctr, &b_cnt, &b_off, &b_temp,
                               &b_tflags, &b_part, &b_carry, &b_owner, &b_slots, &b_cross, &b_ccount, &b_carrytmp,
                               &b_races, &b_races_sorted, &b_rhist, &b_rbase, &b_eoff, &b_ecnt, &b_ecell,
-                              &b_hrec, &b_dist_races, &b_ctmp, &b_ctotal, &b_thist, &b_ftmp, &b_regions};
+                              &b_hrec, &b_dist_races, &b_ctmp, &b_ctotal, &b_thist, &b_ftmp, &b_regions,
+                              &b_bhead, &b_bhscan, &b_bwf, &b_bwscan, &b_bgid, &b_bvk[0], &b_bvk[1], &b_bvi[0],
+                              &b_bvi[1], &b_brh, &b_brscan, &b_bder, &b_bdpos, &b_bdj, &b_bslot, &b_btmp};
     for (auto& b : b_keys) v.push_back(&b);
     for (auto& b : b_rkeys) v.push_back(&b);
     for (auto& b : b_rvals) v.push_back(&b);
@@ -81,6 +87,7 @@ struct sesa_trace {
   void fail(sesa_status s, const char* fmt, ...);
   bool cuda_ok(cudaError_t e, const char* what);
   bool grow(DevBuf& b, size_t bytes, const char* what);
+  bool grow_keep(DevBuf& b, size_t bytes, size_t used, const char* what);  // preserves the first `used` bytes
   bool sync_check(const char* what);
   void free_all();
   void launch_begin(const char* name);
@@ -102,6 +109,8 @@ struct sesa_trace {
   bool step_compact(int cur, uint64_t m, uint64_t** comp, uint32_t* m2);
   bool step_conflict(const uint64_t* comp, uint32_t m2, const sesa::Rec* rec, uint32_t rec_pos_base,
                      const sesa::Rec* rec_entry, uint64_t index_base);
+  bool sort_kv(uint64_t* k0, uint32_t* v0, uint64_t* k1, uint32_t* v1, uint32_t n, uint32_t bits, int* which);
+  bool step_benign(const uint64_t* comp, uint32_t m2, const sesa::Rec* rec, uint64_t index_base);
   bool step_race_sort(uint32_t nr, const sesa::RaceOut* races, uint64_t* rk0, uint32_t* rv0, uint64_t* rk1,
                       uint32_t* rv1, sesa::RaceOut* out);
   sesa_status expand(const sesa_flow* d_flows, uint64_t nf, sesa_access* d_out, uint64_t cap, uint64_t* n_out);

@@ -17,7 +17,8 @@ LIB_PATH = os.path.join(_PKG, "libsesa.so")
 SESA_OK, SESA_EINVAL, SESA_ERANGE, SESA_ENOMEM, SESA_ECUDA, SESA_ENCCL, SESA_ESTATE, SESA_ETRUNC = range(8)
 SESA_SPACE_SHARED, SESA_SPACE_GLOBAL = 0, 1
 SESA_READ, SESA_WRITE, SESA_ATOMIC = 0, 1, 2
-SESA_RACE_RW, SESA_RACE_WW = 1, 2
+SESA_RACE_RW, SESA_RACE_WW, SESA_RACE_WW_BENIGN = 1, 2, 3
+SESA_FLAG_REPORT_BENIGN = 1
 
 # numpy views of the ABI structs (declared here from include/sesa.h)
 ACCESS_DTYPE = np.dtype(
@@ -123,9 +124,11 @@ def _stream_ptr(stream):
 class Trace:
     """One sesa_trace handle (single GPU, or one rank of a distributed check)."""
 
-    def __init__(self, warp_size: int = 32, lockstep: int = 0, granularity: int = 4, *, dist=None):
+    def __init__(self, warp_size: int = 32, lockstep: int = 0, granularity: int = 4, *, dist=None,
+                 benign: bool = False):
         lib = load()
-        self.cfg = sesa_config(warp_size, lockstep, granularity, 0)
+        # flags bit 0 = SESA_FLAG_REPORT_BENIGN: also report benign W/W locations as kind 3 (single GPU)
+        self.cfg = sesa_config(warp_size, lockstep, granularity, 1 if benign else 0)
         h = ctypes.c_void_p()
         if dist is None:
             st = lib.sesa_trace_create(ctypes.byref(self.cfg), ctypes.byref(h))

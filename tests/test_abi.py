@@ -48,7 +48,7 @@ def test_struct_layouts_match_generators_and_oracle():
 def test_bad_config_rejected_before_device():
     lib = S.load()
     h = ctypes.c_void_p()
-    for cfg in ((0, 0, 4, 0), (32, 2, 4, 0), (32, 0, 3, 0), (32, 0, 8192, 0), (32, 0, 4, 1)):
+    for cfg in ((0, 0, 4, 0), (32, 2, 4, 0), (32, 0, 3, 0), (32, 0, 8192, 0), (32, 0, 4, 2), (32, 0, 4, 0x80)):
         c = S.sesa_config(*cfg)
         assert lib.sesa_trace_create(ctypes.byref(c), ctypes.byref(h)) == S.SESA_EINVAL
         assert not h.value

@@ -252,6 +252,70 @@ def test_fused_first_pass_parity(sesa, n, words, shift, fused):
     assert trace(sesa).info()["fused_first_pass"] == fused  # > 32 sort bits or < 32768 records: separate extract
 
 
+# ------------------------------------------------------------------------------------------------ benign W/W (NEXT-4)
+_btraces = {}
+
+
+def assert_same_benign(S, recs, ws=32, ls=0, G_=4, base=0, method="grouped"):
+    key = (ws, ls, G_)
+    if key not in _btraces:
+        _btraces[key] = S.Trace(ws, ls, G_, benign=True)
+    t = _btraces[key]
+    t.check(S.to_device(recs), len(recs), index_base=base)
+    torch.cuda.synchronize()
+    got = t.races()
+    exp = O.check(recs, index_base=base, warp_size=ws, lockstep=ls, granularity=G_, method=method, benign=True)
+    if got.tobytes() != exp.tobytes():
+        e, g = set(O.race_tuples(exp)), set(O.race_tuples(got))
+        raise AssertionError(f"{len(exp)} expected, {len(got)} got; missing {sorted(e - g)[:5]} extra {sorted(g - e)[:5]}")
+    return got
+
+
+def test_benign_f1_equal_values(sesa):
+    got = assert_same_benign(sesa, G.f1_race(distinct=False), method="brute")
+    assert (got["kind"] == 3).sum() == 16
+
+
+@pytest.mark.parametrize("cfg", CONFIGS)
+def test_benign_random_small(sesa, cfg):
+    ws, ls, G_ = cfg
+    for seed in range(25):
+        n = 2 + (seed * 41) % 500
+        r = G.random_trace(n, 300 + seed, threads=8 + seed % 40, values=2, write_frac=0.6, atomic_frac=0.1,
+                           sort=seed % 4 != 0, words=6 + seed % 30)
+        assert_same_benign(sesa, r, ws, ls, G_, base=seed * 77)
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_benign_medium_and_hot(sesa, seed):
+    # many tiles, hot locations crossing conflict tiles, few values: benign pairs everywhere
+    n = [30000, 70001, 120000, 9000][seed]
+    r = G.random_trace(n, 900 + seed, blocks=30, threads=256, intervals=3, words=[2000, 40, 7, 300][seed],
+                       values=[3, 2, 4, 1][seed], write_frac=0.5, sort=seed != 2)
+    assert_same_benign(sesa, r, 32, seed % 2, 4)
+
+
+@pytest.mark.parametrize("sort", [True, False])
+def test_benign_global_only(sesa, sort):
+    # one space: with unordered input the global keys carry (block, interval) and runs are not position-ordered
+    r = G.random_trace(40000, 77 + sort, blocks=50, threads=128, intervals=4, words=900, values=2, write_frac=0.5,
+                       shared_frac=0.0, sort=sort)
+    assert_same_benign(sesa, r, 32, 0, 4)
+
+
+def test_benign_bfs_shape(sesa):
+    # Table IV: the BFS kernel's W/W conflicts are benign — C4 recipe at 2^12 nodes, lockstep
+    from sesagen import configs as GC
+    r = GC.C4(log2n=12).host()
+    got = assert_same_benign(sesa, r, 32, 1, 4)
+    assert 2 not in set(got["kind"].tolist()) and 3 in set(got["kind"].tolist())
+
+
+def test_benign_flag_rejected_when_distributed(sesa):
+    with pytest.raises(sesa.SesaError):
+        sesa.Trace(32, 0, 4, dist=(0, 1, bytes(128)), benign=True)
+
+
 # ------------------------------------------------------------------------------------------------ OOB (NEXT-1)
 def _oob_check(S, recs, regions, base=0):
     t = S.Trace(32, 0, 4)
