@@ -335,6 +335,46 @@ struct TileSmem {
 
 __device__ __forceinline__ u32 pos_of(const KeyLayout& L, u64 key) { return (u32)(key & lowmask(L.pos_bits)); }
 
+// Tile windows.  Tiles step by CT_NOM entries; a tile also takes the rest of its last location run when that run
+// ends within CT_EXT entries past the nominal end (and the next tile skips those entries), so that the short
+// runs straddling a boundary — nearly every boundary in C2/C4, whose locations hold ~17 entries — are completed
+// inside one tile instead of going through the crossing-run carries (modes 2/3).  Windows partition the entries:
+// window(t) = [t*CT_NOM + skip(t*CT_NOM), (t+1)*CT_NOM + skip((t+1)*CT_NOM)) clipped to [0, m), <= CT_TILE long.
+constexpr u32 CT_EXT = 256, CT_NOM = CT_TILE - CT_EXT;
+
+// skip(b): entries from b on that belong to a run owned by the tile before boundary b (run head >= b - CT_NOM,
+// i.e. inside that tile) and ending by b + CT_EXT; 0 if b starts a run or the run is long.  All threads call it.
+__device__ u32 window_skip(const ConflictArgs& a, u64 b) {
+  __shared__ u32 s_first;
+  const KeyLayout& L = a.L;
+  if (b == 0 || b >= a.m) return 0;
+  const u64 g = group_of_hi(L, a.keys[b - 1] >> L.pos_bits);
+  if (group_of_hi(L, a.keys[b] >> L.pos_bits) != g) return 0;  // b heads a run
+  if (b >= (u64)CT_NOM + 1 && group_of_hi(L, a.keys[b - CT_NOM - 1] >> L.pos_bits) == g) return 0;  // long run
+  if (threadIdx.x == 0) s_first = ~0u;
+  __syncthreads();
+  const u32 t = threadIdx.x;  // entries b + 1 .. b + CT_EXT: the first one outside the run
+  if (t < CT_EXT) {
+    const u64 i = b + 1 + t;
+    if (i >= a.m || group_of_hi(L, a.keys[i] >> L.pos_bits) != g) atomicMin(&s_first, t + 1);
+  }
+  __syncthreads();
+  const u32 r = s_first;
+  __syncthreads();
+  return r;  // ~0u (> CT_EXT): the run is long
+}
+
+// window of tile t -> (tb, cnt); cnt = 0 for a tile whose entries all went to its predecessor
+__device__ __forceinline__ void tile_window(const ConflictArgs& a, u32 tile, u64* tb, u32* cnt) {
+  const u64 b0 = (u64)tile * CT_NOM, b1 = b0 + CT_NOM;
+  u32 s0 = window_skip(a, b0), s1 = window_skip(a, b1);
+  if (s0 > CT_EXT) s0 = 0;
+  if (s1 > CT_EXT) s1 = 0;
+  const u64 lo = min((u64)a.m, b0 + s0), hi = min((u64)a.m, b1 + s1);
+  *tb = lo;
+  *cnt = (u32)(hi - lo);
+}
+
 // the record of entry e (sorted/compacted entry index) with key `key`: by position in the caller's record array
 // (single GPU), or entry-aligned records fetched from the owner ranks (distributed check)
 __device__ __forceinline__ Rec rec_at(const ConflictArgs& a, u64 e, u64 key) {
@@ -364,7 +404,9 @@ __device__ bool tile_load(const ConflictArgs& a, TileSmem& s, u64 tb, u32 cnt) {
 #pragma unroll
   for (int q = 0; q < CT_ITEMS; q++) {
     const int j = j0 + q;
-    u8 f = FL_GH | FL_GT;
+    // items past the window's end carry no boundary flags: they are transparent to the segmented scans, so
+    // the backward carry of a run crossing out of a short window reaches its last real item (cnt - 1)
+    u8 f = j < (int)cnt ? (FL_GH | FL_GT) : 0;
     if (j < (int)cnt) {
       const u64 g = group_of_hi(L, s.key[j + 1] >> L.pos_bits);
       const bool sp = (j > 0 || tb > 0) && group_of_hi(L, s.key[j] >> L.pos_bits) == g;
@@ -406,7 +448,7 @@ __device__ bool tile_load(const ConflictArgs& a, TileSmem& s, u64 tb, u32 cnt) {
       const bool sh = (f & FL_GH) || s.blk[j] != s.blk[j + 1] || s.ivl[j] != s.ivl[j + 1];
       const bool st = (f & FL_GT) || s.blk[j + 2] != s.blk[j + 1] || s.ivl[j + 2] != s.ivl[j + 1];
       f |= (sh ? FL_SH : 0) | (st ? FL_ST : 0);
-    } else {
+    } else if (j < (int)cnt) {
       f |= FL_SH | FL_ST;
     }
     s.fl[j] = f;
@@ -520,12 +562,13 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
   const u32 tile = MODE == 1 ? blockIdx.x : a.cross_list[blockIdx.x];
-  const u64 tb = (u64)tile * CT_TILE;
-  const u32 cnt = (u32)min((u64)CT_TILE, (u64)a.m - tb);
+  u64 tb;
+  u32 cnt;
+  tile_window(a, tile, &tb, &cnt);
   const KeyLayout& L = a.L;
   const int tid = threadIdx.x;
 
-  if (!tile_load(a, s, tb, cnt)) {
+  if (cnt == 0 || !tile_load(a, s, tb, cnt)) {
     if (MODE == 1 && tid == 0) a.tile_flags[tile] = TF_GH | TF_GT | TF_SH | TF_ST;
     return;
   }
@@ -682,11 +725,12 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_y_kernel(ConflictArgs a) 
   extern __shared__ __align__(16) unsigned char smem_raw[];
   TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
   const u32 tile = a.cross_list[blockIdx.x];
-  const u64 tb = (u64)tile * CT_TILE;
-  const u32 cnt = (u32)min((u64)CT_TILE, (u64)a.m - tb);
+  u64 tb;
+  u32 cnt;
+  tile_window(a, tile, &tb, &cnt);
   const KeyLayout& L = a.L;
   const int tid = threadIdx.x;
-  if (!tile_load(a, s, tb, cnt)) return;
+  if (cnt == 0 || !tile_load(a, s, tb, cnt)) return;
   const bool cin = !(s.fl[0] & FL_GH), cout = !(s.fl[cnt - 1] & FL_GT);
   const int ftail = s.first_gtail, lhead = s.last_ghead;
   __shared__ F5 s_x[2][2];
@@ -752,7 +796,7 @@ __global__ void cross_emit_kernel(ConflictArgs a, u32 ncross) {
                 sl.hinterval);
 }
 
-u32 conflict_tiles(u64 m) { return (u32)((m + CT_TILE - 1) / CT_TILE); }
+u32 conflict_tiles(u64 m) { return (u32)((m + CT_NOM - 1) / CT_NOM); }
 
 template <int MODE, class A>
 static void launch_ck(const ConflictArgs& a, u32 nblocks, cudaStream_t st) {
