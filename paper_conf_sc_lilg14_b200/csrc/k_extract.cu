@@ -74,9 +74,12 @@ template <int U>
 // With regions (nreg > 0; sorted by (space, base), non-overlapping, space s in [rs[s], rs[s+1])), every valid
 // record of a space with regions is also checked for containment (OOB, NEXT-1): binary search for the last
 // region starting at or below addr, then addr + size <= end.
+// With gout != null the granule index addr >> log2G of every record is also written (8 bytes per record,
+// coalesced): the fused pass then reads 8 bytes per record instead of the record's 32-byte sector.
 __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ rec, u32 n, u32 log2G, u32 rw,
                                                        Summary* __restrict__ out, u32* __restrict__ tile_hist,
-                                                       const Region* __restrict__ regs, uint3 rs) {
+                                                       const Region* __restrict__ regs, uint3 rs,
+                                                       u64* __restrict__ gout) {
   __shared__ u32 s_th[8][RADIX];
   extern __shared__ Region s_reg[];  // [rs.z]
   for (u32 i = threadIdx.x; i < rs.z; i += 256) s_reg[i] = regs[i];
@@ -164,6 +167,7 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
         else A0.add(addr, last, b[u].x, b[u].z);
         if (tile_hist) atomicAdd(&th[(u32)(addr >> log2G) & (RADIX - 1)], 1u);
       }
+      if (gout && r0 + u * 32 + lane < tend) __stcs(gout + r0 + u * 32 + lane, addr >> log2G);
     }
   }
   if (tile_hist) {
@@ -244,7 +248,7 @@ static int ring_grid(const void* kern, int threads, size_t smem, size_t smem_max
 }
 
 void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, u32* tile_hist, const Region* regs, u32 nreg,
-                    u32 nreg_shared, int grid, cudaStream_t st) {
+                    u32 nreg_shared, int grid, cudaStream_t st, u64* gout) {
   // extents2: contiguous warp ranges, one full wave of resident warps (the round-1 grid-stride kernel took
   // 7.7 ms on C5: 132 instructions per record, 64-bit index math and local-memory accumulators; this one 4.6 ms)
   static int sms = 0, per = 0;
@@ -263,7 +267,7 @@ void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, u32* tile_
   rw = std::max<u64>(gran, (rw + gran - 1) / gran * gran);
   const u64 nw = (n + rw - 1) / rw;
   extents2_kernel<4><<<(unsigned)((nw + 7) / 8), 256, nreg * sizeof(Region), st>>>(
-      rec, (u32)n, log2G, (u32)rw, d_sum, tile_hist, regs, make_uint3(nreg_shared, 0u, nreg));
+      rec, (u32)n, log2G, (u32)rw, d_sum, tile_hist, regs, make_uint3(nreg_shared, 0u, nreg), gout);
   (void)grid;
 }
 

@@ -90,7 +90,7 @@ size_t fused_temp_bytes(u64 n) {
 
 // ---- the fused kernel -------------------------------------------------------------------------------------------
 struct FusedArgs {
-  const Rec* rec;
+  const u64* gran;  // granule index of every record (written by the extents pass)
   u32 n, log2G, pos_bits, npass;
   u64 gmin;
   const u32* toff;  // [T][RADIX] output offset of each tile's digit run
@@ -119,14 +119,14 @@ __global__ void __launch_bounds__(FUSED_THREADS, FUSED_MINB) fused_extract_pass0
   u32* wh = whist + warp * RADIX;
   u32* wm = wmask + warp * (RADIX + 1);
   const unsigned lt = lanemask_lt();
-  // (0) addresses of a tile's records: one 32-byte sector per record, the 8-byte address word is all the key needs
+  // (0) granule indices of a tile's records (8 bytes per record, coalesced), written by the extents pass
   u64 a[ITEMS];
   auto issue = [&](u32 t) {
     const u32 wb = t * TILE + warp * 32 * ITEMS + lane;
-    const u64* ap = reinterpret_cast<const u64*>(A.rec) + 4 * (u64)wb;  // record stride: 4 words
+    const u64* gp = A.gran + wb;
 #pragma unroll
     for (int i = 0; i < ITEMS; i++)
-      if (wb + i * 32 < A.n) a[i] = __ldcs(ap + i * 128);
+      if (wb + i * 32 < A.n) a[i] = __ldcs(gp + i * 32);
   };
   u32 tile = blockIdx.x;
   if (tile < T) issue(tile);
@@ -138,7 +138,7 @@ __global__ void __launch_bounds__(FUSED_THREADS, FUSED_MINB) fused_extract_pass0
     // record index, known from (tile, warp, item, lane)
     u32 kh[ITEMS];
 #pragma unroll
-    for (int i = 0; i < ITEMS; i++) kh[i] = i < nv ? (u32)((a[i] >> A.log2G) - A.gmin) : 0u;
+    for (int i = 0; i < ITEMS; i++) kh[i] = i < nv ? (u32)(a[i] - A.gmin) : 0u;
     auto digit = [&](int i) -> u32 { return i < nv ? (kh[i] & (RADIX - 1)) : (u32)RADIX; };
     for (u32 i = tid; i < WARPS * RADIX; i += THREADS) whist[i] = 0;
     __syncthreads();
@@ -223,7 +223,7 @@ void launch_tile_offsets(u64 n, const KeyLayout& L, const u32* tile_hist, void* 
 }
 
 // temp: holds the tile offsets (launch_tile_offsets); hist: [npass][RADIX] zeroed (rows >= 1 filled)
-void launch_fused_extract_pass0(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, void* temp, u64* kout,
+void launch_fused_extract_pass0(const u64* gran, u64 n, const KeyLayout& L, u32 npass, void* temp, u64* kout,
                                 u32* hist, cudaStream_t st) {
   if (!n) return;
   const u32 T = (u32)((n + FUSED_TILE - 1) / FUSED_TILE);
@@ -242,7 +242,7 @@ void launch_fused_extract_pass0(const Rec* rec, u64 n, const KeyLayout& L, u32 n
   }
   const size_t sm = fused_smem(npass);
   FusedArgs A;
-  A.rec = rec;
+  A.gran = gran;
   A.n = (u32)n;
   A.log2G = L.log2G;
   A.pos_bits = L.pos_bits;
