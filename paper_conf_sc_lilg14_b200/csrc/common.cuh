@@ -268,6 +268,9 @@ struct Summary {
   unsigned int pad;
   unsigned long long oob_count;  // valid records outside every registered region of their space (NEXT-1)
   unsigned long long oob_first;  // lowest such record index (~0 = none)
+  // with tile histograms (fused-pass candidates): histograms of the raw granule bytes 1..3, (g >> 8b) & 255 —
+  // the later sort digits once gmin is aligned down to a multiple of 2^(8 (npass - 1)) (sesa_api.cu)
+  unsigned int bhist[3][256];
 };
 
 // one registered memory region (include/sesa.h sesa_region), bytes [base, end)

@@ -81,9 +81,12 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
                                                        const Region* __restrict__ regs, uint3 rs,
                                                        u64* __restrict__ gout) {
   __shared__ u32 s_th[8][RADIX];
+  __shared__ u32 s_hb[3][RADIX];  // raw granule bytes 1..3 (with tile_hist)
   extern __shared__ Region s_reg[];  // [rs.z]
   for (u32 i = threadIdx.x; i < rs.z; i += 256) s_reg[i] = regs[i];
-  if (rs.z) __syncthreads();
+  if (tile_hist)
+    for (u32 i = threadIdx.x; i < 3 * RADIX; i += 256) (&s_hb[0][0])[i] = 0;
+  if (rs.z || tile_hist) __syncthreads();
   constexpr int THREADS = 256;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const u32 gw = (blockIdx.x * THREADS + threadIdx.x) >> 5;
@@ -165,7 +168,13 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
       if (ok[u]) {
         if (glob) A1.add(addr, last, b[u].x, b[u].z);
         else A0.add(addr, last, b[u].x, b[u].z);
-        if (tile_hist) atomicAdd(&th[(u32)(addr >> log2G) & (RADIX - 1)], 1u);
+        if (tile_hist) {
+          const u64 g = addr >> log2G;
+          atomicAdd(&th[(u32)g & (RADIX - 1)], 1u);
+          atomicAdd(&s_hb[0][(u32)(g >> 8) & (RADIX - 1)], 1u);
+          atomicAdd(&s_hb[1][(u32)(g >> 16) & (RADIX - 1)], 1u);
+          atomicAdd(&s_hb[2][(u32)(g >> 24) & (RADIX - 1)], 1u);
+        }
       }
       if (gout && r0 + u * 32 + lane < tend) __stcs(gout + r0 + u * 32 + lane, addr >> log2G);
     }
@@ -185,6 +194,13 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) oc += __shfl_xor_sync(~0u, oc, o), of = min(of, __shfl_xor_sync(~0u, of, o));
     if (lane == 0 && oc) atomicAdd(&out->oob_count, (unsigned long long)oc), atomicMin(&out->oob_first, (unsigned long long)of);
+  }
+  if (tile_hist) {
+    __syncthreads();
+    for (u32 i = threadIdx.x; i < 3 * RADIX; i += 256) {
+      const u32 v = (&s_hb[0][0])[i];
+      if (v) atomicAdd(&(&out->bhist[0][0])[i], v);
+    }
   }
   SpaceAcc S0 = A0.to_acc(log2G), S1 = A1.to_acc(log2G);
   __shared__ SpaceAcc sa[THREADS / 32][2];

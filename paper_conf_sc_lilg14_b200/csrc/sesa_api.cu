@@ -306,11 +306,21 @@ bool sesa_trace::step_extract_fused(const Rec* rec, u64 n) {
       !grow(b_ftmp, fused_temp_bytes(n), "fused temp"))
     return false;
   cudaMemsetAsync(b_hist.p, 0, (size_t)npass * RADIX * 4, stream);
+  if (hist_from_extents) {  // digit p >= 1 = raw granule byte p; the top digit rotated by byte p of gmin
+    std::vector<u32> rows((size_t)(npass - 1) * RADIX);
+    for (u32 p = 1; p < npass; p++) {
+      const u32 r = p == npass - 1 ? (u32)(L.gminG >> (RADIX_BITS * p)) & (RADIX - 1) : 0u;
+      for (u32 d = 0; d < (u32)RADIX; d++) rows[(size_t)(p - 1) * RADIX + d] = h_summary.bhist[p - 1][(d + r) & (RADIX - 1)];
+    }
+    if (!cuda_ok(cudaMemcpyAsync((u32*)b_hist.p + RADIX, rows.data(), rows.size() * 4, cudaMemcpyHostToDevice, stream),
+                 "hist rows"))
+      return false;
+  }
   LAUNCH("tile_offsets", 2.0 * RADIX * 4 * ((n + FUSED_TILE - 1) / FUSED_TILE),
          launch_tile_offsets(n, L, (const u32*)b_thist.p, b_ftmp.p, stream));
   LAUNCH("extract_pass0", 16.0 * n,
-         launch_fused_extract_pass0((const u64*)b_keys[0].p, n, L, npass, b_ftmp.p, (u64*)b_keys[1].p, (u32*)b_hist.p,
-                                    stream));
+         launch_fused_extract_pass0((const u64*)b_keys[0].p, n, L, hist_from_extents ? 1u : npass, b_ftmp.p,
+                                    (u64*)b_keys[1].p, (u32*)b_hist.p, stream));
   return true;
 }
 
@@ -675,6 +685,22 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
   const bool fused = have_thist && !layout.both && layout.single_space == SP_GLOBAL && layout.lowG == 0 &&
                      S.multi == 0 && m == n && layout.sort_bits <= 32 && fused_supported(npass);
   info.fused_first_pass = fused ? 1 : 0;
+  // Fused path: align gmin down to a multiple of 2^(8 (npass - 1)).  Then every later sort digit of
+  // key_hi = g - gmin is a raw granule byte (the top one rotated by a constant), whose histograms the extents
+  // pass already took — the fused pass needs no histogram atomics.  Only if the aligned span needs no extra pass.
+  hist_from_extents = false;
+  if (fused && npass > 1) {
+    const u32 D = RADIX_BITS * (npass - 1);
+    const u64 G0 = S.gmin[1] & ~((1ull << D) - 1ull);
+    const u32 nb = bits_of(S.gmax[1] - G0);
+    if ((nb + RADIX_BITS - 1) / RADIX_BITS == npass && nb + layout.pos_bits <= 64) {
+      layout.gminG = G0;
+      layout.gbG = nb;
+      layout.sort_bits = nb;
+      info.sort_bits = nb;
+      hist_from_extents = true;
+    }
+  }
   int cur = 0;
   if (fused) {
     if (!step_extract_fused(rec, n) || !step_sort(m, &cur, 1, 1)) return status;

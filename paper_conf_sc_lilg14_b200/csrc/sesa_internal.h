@@ -43,7 +43,8 @@ struct sesa_trace {
   DevBuf b_tflags, b_part, b_carry, b_owner, b_slots, b_cross, b_ccount, b_carrytmp;
   DevBuf b_races, b_rkeys[2], b_rvals[2], b_races_sorted, b_rhist, b_rbase;
   DevBuf b_eoff, b_ecnt, b_ecell, b_hrec, b_dist_races, b_ctmp, b_ctotal, b_thist, b_ftmp;
-  bool have_thist = false;  // extents wrote per-tile raw digit histograms (fused first pass possible)
+  bool have_thist = false;
+  bool hist_from_extents = false;  // fused path: later-digit histograms from the extents' raw granule bytes  // extents wrote per-tile raw digit histograms (fused first pass possible)
   // out-of-bound check (NEXT-1): registered regions (sorted by space, base) and the last report
   DevBuf b_regions;
   // benign W/W reporting (flags bit 0): regrouped plain writes and the derived trace checked by `child`

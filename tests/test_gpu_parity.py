@@ -241,10 +241,13 @@ def test_profiling_stats(sesa):
 # ------------------------------------------------------------------------------------------------ fused first pass
 @pytest.mark.parametrize("n,words,shift,fused", [(32768, 100, 77, 1), (40000, 30000, 1, 1), (65537, 3_000_000, 200, 1),
                                                  (200003, 50_000, 255, 1), (500000, 400_000_000, 13, 1),
+                                                 (70000, 65_500, 255, 1), (70000, 65_000, 255, 1),
                                                  (40000, 2**34, 3, 0), (32767, 1000, 5, 0)])
 def test_fused_first_pass_parity(sesa, n, words, shift, fused):
     # global-only, (block, interval)-ordered, one granule per record: the fused extract + first sort pass
-    # (k_fused.cu) places tiles from the extents' raw-byte histograms rotated by gmin & 255 — shift moves gmin
+    # (k_fused.cu) places tiles from the extents' raw-byte histograms rotated by gmin & 255 — shift moves gmin.
+    # The later digits' histograms come from the extents' raw granule bytes once gmin is aligned down to
+    # 2^(8 (npass - 1)) unless the aligned span needs an extra pass (65,500 words at gmin byte 255: fallback).
     r = G.random_trace(n, 7 + n % 97, blocks=64, threads=256, intervals=3, words=words, shared_frac=0.0,
                        sizes=(4,), unaligned=False, values=4)
     r["addr"] += np.uint64(4 * shift)
