@@ -555,6 +555,20 @@ __device__ void emit_race(const ConflictArgs& a, u64 head_hi, u32 kind, u32 x, u
   a.race_vals[idx] = idx;
 }
 
+// A location whose whole summary shows no possible pair of either kind: no RW (no read, or no write/atomic) and
+// no WW (no write, or no atomic and every write of one value — benign).  C4's `changed` run (60 M same-valued
+// writes) is one; its middle tiles skip the crossing modes entirely.
+__device__ __forceinline__ bool cannot_race(const AggC& g) {
+  const bool noR = g.mn[RW_READ] > g.mx[RW_READ], noW = g.mn[RW_WRITE] > g.mx[RW_WRITE];
+  const bool noA = g.mn[RW_ATOMIC] > g.mx[RW_ATOMIC];
+  return (noR || (noW && noA)) && (noW || (noA && g.vlo == g.vhi));
+}
+__device__ __forceinline__ bool cannot_race(const Agg& g) {
+  const bool noR = g.mn[RW_READ] > g.mx[RW_READ], noW = g.mn[RW_WRITE] > g.mx[RW_WRITE];
+  const bool noA = g.mn[RW_ATOMIC] > g.mx[RW_ATOMIC];
+  return (noR || (noW && noA)) && (noW || (noA && g.v1 == g.v2));
+}
+
 // ------------------------------------------------------------------------------------------------ mode 1 / 2
 template <int MODE, class A>
 __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
@@ -562,6 +576,24 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
   const u32 tile = MODE == 1 ? blockIdx.x : a.cross_list[blockIdx.x];
+  if (MODE == 2) {
+    // a tile inside one location run (crossing in and out, no run head): its flags only matter if the run's
+    // whole summary (carry in + this piece + carry out) allows a race
+    __shared__ int s_skip;
+    if (threadIdx.x == 0) {
+      const u8 tf = a.tile_flags[tile];
+      bool skip = false;
+      if ((tf & TF_CIN) && (tf & TF_COUT) && !(tf & TF_GH)) {
+        typedef typename OpOf<A>::type Op;
+        const A* c = reinterpret_cast<const Q*>(a.carry)[tile].a;
+        const A* pp = reinterpret_cast<const Q*>(a.part)[tile].a;
+        skip = cannot_race(Op()(Op()(c[0], pp[0]), c[1]));
+      }
+      s_skip = skip;
+    }
+    __syncthreads();
+    if (s_skip) return;
+  }
   u64 tb;
   u32 cnt;
   tile_window(a, tile, &tb, &cnt);
@@ -725,6 +757,25 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_y_kernel(ConflictArgs a) 
   extern __shared__ __align__(16) unsigned char smem_raw[];
   TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
   const u32 tile = a.cross_list[blockIdx.x];
+  {
+    // nothing to do unless a crossing run this tile takes part in has a witness x
+    __shared__ int s_any;
+    if (threadIdx.x == 0) {
+      const u8 tf = a.tile_flags[tile];
+      bool any = false;
+      if (tf & TF_CIN) {
+        const Slot& sl = a.slots[a.owner[tile]];
+        any |= sl.x[0] != ~0ull || sl.x[1] != ~0ull;
+      }
+      if ((tf & TF_COUT) && (tf & TF_GH)) {
+        const Slot& sl = a.slots[tile];
+        any |= sl.x[0] != ~0ull || sl.x[1] != ~0ull;
+      }
+      s_any = any;
+    }
+    __syncthreads();
+    if (!s_any) return;
+  }
   u64 tb;
   u32 cnt;
   tile_window(a, tile, &tb, &cnt);

@@ -238,6 +238,33 @@ def test_profiling_stats(sesa):
     t.close()
 
 
+@pytest.mark.parametrize("tail", ["none", "atomic", "other_value", "read"])
+def test_long_write_run_skip(sesa, tail):
+    # a C4-`changed`-like run of 60k same-valued writes crossing ~30 conflict tiles: its middle tiles skip the
+    # crossing modes when the whole run cannot race; one atomic, other value or read at its end must still be found
+    n = 60000
+    r = np.zeros(n, G.REC_DTYPE)
+    r["block"] = np.arange(n) // 256
+    r["thread"] = np.arange(n) % 256
+    r["space"] = 1
+    r["size"] = 4
+    r["addr"] = 0x9000
+    r["rw"] = 1
+    r["value_hash"] = 5
+    if tail == "atomic":
+        r["rw"][-1] = 2
+    elif tail == "other_value":
+        r["value_hash"][-1] = 6
+    elif tail == "read":
+        r["rw"][-1] = 0
+    extra = G.random_trace(5000, 17, blocks=300, threads=256, intervals=1, words=50, shared_frac=0.0, sizes=(4,),
+                           unaligned=False)
+    extra["block"] = np.sort(extra["block"]) + 300
+    recs = np.concatenate([r, extra])
+    got = assert_same(sesa, recs, 32, 0, 4)
+    assert (len([x for x in O.race_tuples(got) if x[3] == 0x9000]) == 0) == (tail == "none")
+
+
 # ------------------------------------------------------------------------------------------------ fused first pass
 @pytest.mark.parametrize("n,words,shift,fused", [(32768, 100, 77, 1), (40000, 30000, 1, 1), (65537, 3_000_000, 200, 1),
                                                  (200003, 50_000, 255, 1), (500000, 400_000_000, 13, 1),
