@@ -7,7 +7,7 @@ namespace sesa {
 constexpr int RADIX_BITS = 8;  // onesweep digit width (8-bit digits, 256 bins per pass)
 constexpr int RADIX = 1 << RADIX_BITS;
 // fused key extract + first sort pass (k_fused.cu): tiles of 256 threads x 32 records
-constexpr int FUSED_THREADS = 256, FUSED_ITEMS = 16, FUSED_MINB = 3, FUSED_TILE = FUSED_THREADS * FUSED_ITEMS;
+constexpr int FUSED_THREADS = 256, FUSED_ITEMS = 24, FUSED_MINB = 2, FUSED_TILE = FUSED_THREADS * FUSED_ITEMS;
 
 // onesweep tile: 256 threads x 16 keys (warp-striped); one lookback word per (tile, bin)
 constexpr int SORT_THREADS = 256;
