@@ -12,7 +12,8 @@
 // flag_K(e) = partner of kind K exists; witness x_K = min flagged position of the group, y_K = min position s
 // with P(x_K, s) of kind K (lexicographic minimum, reading R12).
 //
-// A CTA owns a tile of 2048 sorted entries.  Summaries are computed with a per-thread fold over its 8 entries
+// A CTA owns a window of up to CT_TILE = 1536 sorted entries (below).  Summaries are computed with a per-thread fold
+// over its CT_ITEMS = 6 entries
 // plus block-wide segmented scans of the per-thread folds (warp shuffles), forward and backward, so each entry
 // receives the total of its segment without storing per-entry summaries.  Runs that cross a tile boundary
 // (hot locations: C3 bins, C4 `changed`) are completed in three extra steps:
