@@ -559,16 +559,20 @@ __device__ void emit_race(const ConflictArgs& a, u64 head_hi, u32 kind, u32 x, u
 // A location whose whole summary shows no possible pair of either kind: no RW (no read, or no write/atomic) and
 // no WW (no write, or no atomic and every write of one value — benign).  C4's `changed` run (60 M same-valued
 // writes) is one; its middle tiles skip the crossing modes entirely.
-__device__ __forceinline__ bool cannot_race(const AggC& g) {
+// no_rw / no_ww: the summary of a whole run rules out every pair of that kind
+__device__ __forceinline__ void cannot_race(const AggC& g, bool* no_rw, bool* no_ww) {
   const bool noR = g.mn[RW_READ] > g.mx[RW_READ], noW = g.mn[RW_WRITE] > g.mx[RW_WRITE];
   const bool noA = g.mn[RW_ATOMIC] > g.mx[RW_ATOMIC];
-  return (noR || (noW && noA)) && (noW || (noA && g.vlo == g.vhi));
+  *no_rw = noR || (noW && noA);
+  *no_ww = noW || (noA && g.vlo == g.vhi);
 }
-__device__ __forceinline__ bool cannot_race(const Agg& g) {
+__device__ __forceinline__ void cannot_race(const Agg& g, bool* no_rw, bool* no_ww) {
   const bool noR = g.mn[RW_READ] > g.mx[RW_READ], noW = g.mn[RW_WRITE] > g.mx[RW_WRITE];
   const bool noA = g.mn[RW_ATOMIC] > g.mx[RW_ATOMIC];
-  return (noR || (noW && noA)) && (noW || (noA && g.v1 == g.v2));
+  *no_rw = noR || (noW && noA);
+  *no_ww = noW || (noA && g.v1 == g.v2);
 }
+__device__ __forceinline__ u64 ld_volatile(const u64* p) { return *reinterpret_cast<const volatile u64*>(p); }
 
 // ------------------------------------------------------------------------------------------------ mode 1 / 2
 template <int MODE, class A>
@@ -578,17 +582,36 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
   TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
   const u32 tile = MODE == 1 ? blockIdx.x : a.cross_list[blockIdx.x];
   if (MODE == 2) {
-    // a tile inside one location run (crossing in and out, no run head): its flags only matter if the run's
-    // whole summary (carry in + this piece + carry out) allows a race
+    // A crossing piece matters for a kind K only if its run's whole summary allows a K pair and — for the
+    // piece a run crosses IN with (its head lies in an earlier tile), in position-ordered runs (lowG == 0) — no
+    // entry before this tile is flagged K yet: x_K is a minimum position.  A tile whose pieces all cannot lower
+    // any x is skipped (C4's `changed`, the far tiles of C3's hot bins, the second tile of a crossing dist[v]).
     __shared__ int s_skip;
     if (threadIdx.x == 0) {
+      typedef typename OpOf<A>::type Op;
       const u8 tf = a.tile_flags[tile];
-      bool skip = false;
-      if ((tf & TF_CIN) && (tf & TF_COUT) && !(tf & TF_GH)) {
-        typedef typename OpOf<A>::type Op;
-        const A* c = reinterpret_cast<const Q*>(a.carry)[tile].a;
-        const A* pp = reinterpret_cast<const Q*>(a.part)[tile].a;
-        skip = cannot_race(Op()(Op()(c[0], pp[0]), c[1]));
+      const A* c = reinterpret_cast<const Q*>(a.carry)[tile].a;    // [grp In, grp Out, ...]
+      const A* pp = reinterpret_cast<const Q*>(a.part)[tile].a;    // [grp P, grp S, ...]
+      const bool middle = (tf & TF_CIN) && (tf & TF_COUT) && !(tf & TF_GH);
+      bool skip = true;
+      if (tf & TF_CIN) {  // piece A: the run crossing in (the whole tile if middle)
+        bool done[2];
+        const A run = middle ? Op()(Op()(c[0], pp[0]), c[1]) : Op()(c[0], pp[0]);
+        cannot_race(run, &done[0], &done[1]);
+        if (a.L.lowG == 0) {  // the window starts at the nominal start: the run crossing there is long
+          const u64 first = pos_of(a.L, a.keys[(u64)tile * CT_NOM]);
+          const Slot* sl = &a.slots[a.owner[tile]];
+          for (int k = 0; k < 2; k++) {
+            const u64 x = ld_volatile(&sl->x[k]);
+            done[k] = done[k] || (x != ~0ull && (x >> 32) < first);
+          }
+        }
+        skip = skip && done[0] && done[1];
+      }
+      if ((tf & TF_COUT) && (tf & TF_GH)) {  // piece B: a run starting here and crossing out
+        bool done[2];
+        cannot_race(Op()(pp[1], c[1]), &done[0], &done[1]);
+        skip = skip && done[0] && done[1];
       }
       s_skip = skip;
     }
@@ -766,7 +789,17 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_y_kernel(ConflictArgs a) 
       bool any = false;
       if (tf & TF_CIN) {
         const Slot& sl = a.slots[a.owner[tile]];
-        any |= sl.x[0] != ~0ull || sl.x[1] != ~0ull;
+        if (a.L.lowG == 0) {
+          // the run crossing in, position-ordered: y_K (a minimum position) cannot come from here if a partner
+          // before this tile is known
+          const u64 first = pos_of(a.L, a.keys[(u64)tile * CT_NOM]);
+          for (int k = 0; k < 2; k++) {
+            const u64 y = ld_volatile(&sl.y[k]);
+            any |= sl.x[k] != ~0ull && !(y != ~0ull && (y >> 32) < first);
+          }
+        } else {
+          any |= sl.x[0] != ~0ull || sl.x[1] != ~0ull;
+        }
       }
       if ((tf & TF_COUT) && (tf & TF_GH)) {
         const Slot& sl = a.slots[tile];
