@@ -679,12 +679,14 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
         a.slots[tile] = sl;
       }
     }
-    // no flagged entry in the tile (every internal group is race-free, e.g. all of C2): nothing to emit here
+    // no flagged entry in a group internal to the tile (every internal group race-free, e.g. all of C2; or only
+    // crossing pieces, e.g. the middle tiles of C3's hot bins — modes 2/3 own those): nothing to emit here
     bool my_res = false;
 #pragma unroll
     for (int q = 0; q < CT_ITEMS; q++) {
-      const u32 j = tid * CT_ITEMS + q;
-      if (j < cnt) my_res |= s.res[j] != 0 && (s.fl[j] & FL_INT);
+      const int j = tid * CT_ITEMS + q;
+      if (j < (int)cnt && !(cin && j <= ftail) && !(cout && j >= lhead))
+        my_res |= s.res[j] != 0 && (s.fl[j] & FL_INT);
     }
     if (!__syncthreads_or(my_res)) return;
     // x per group: min flagged (position << 11 | item) per kind; every entry then tests P(x, entry)
