@@ -640,6 +640,57 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
     if (!(s.fl[cnt - 1] & FL_ST)) co[1] = c[3];
   }
   __shared__ A s_part[4];
+  if (MODE == 1 && cin && cout && s.last_ghead < 0) {
+    // a window inside one crossing run: mode 1 only owes the carries their pieces (the run-level summary and the
+    // first / last sub-run pieces) — plain block reductions; modes 2/3 decide its entries
+    typedef typename OpOf<A>::type Op;
+    __shared__ int s_fst, s_lsh;
+    if (tid == 0) s_fst = (int)cnt - 1, s_lsh = 0;
+    __syncthreads();
+    bool sh = false, st = false;
+#pragma unroll
+    for (int q = 0; q < CT_ITEMS; q++) {
+      const int j = tid * CT_ITEMS + q;
+      if (j >= (int)cnt) continue;
+      if (s.fl[j] & FL_ST) atomicMin(&s_fst, j), st = true;
+      if (s.fl[j] & FL_SH) atomicMax(&s_lsh, j), sh = true;
+    }
+    const bool any_sh = __syncthreads_or(sh), any_st = __syncthreads_or(st);
+    const int fst = s_fst, lsh = s_lsh;
+    const A E = agg_empty_t<A>();
+    A g = E, p = E, q2 = E;
+#pragma unroll
+    for (int q = 0; q < CT_ITEMS; q++) {
+      const int j = tid * CT_ITEMS + q;
+      if (j >= (int)cnt) continue;
+      g = Op()(g, agg_item_t<A>(s.rw[j], s.blk[j + 1], s.vh[j]));
+      const A it = agg_item_t<A>(s.rw[j], s.thr[j], s.vh[j]);
+      if (j <= fst) p = Op()(p, it);
+      if (j >= lsh) q2 = Op()(q2, it);
+    }
+    A* wv = scan_scratch<A>(s);  // [WARPS]
+    const A red[3] = {g, p, q2};
+    for (int r = 0; r < 3; r++) {
+      A v = red[r];
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) v = Op()(v, shfl(v, o, true));
+      if ((tid & 31) == 0) wv[tid >> 5] = v;
+      __syncthreads();
+      if (tid == 0) {
+        A t = wv[0];
+        for (int w = 1; w < CT_THREADS / 32; w++) t = Op()(t, wv[w]);
+        if (r == 0) s_part[0] = s_part[1] = t;
+        else s_part[r + 1] = t;
+      }
+      __syncthreads();
+    }
+    if (tid == 0) {
+      a.tile_flags[tile] = (any_sh ? TF_SH : 0) | (any_st ? TF_ST : 0) | TF_CIN | TF_COUT;
+      for (int i = 0; i < 4; i++) reinterpret_cast<Q*>(a.part)[tile].a[i] = s_part[i];
+      a.cross_list[atomicAdd(a.cross_count, 1u)] = tile;
+    }
+    return;
+  }
   tile_flags<A>(a, s, cnt, ci, co, MODE == 1 ? s_part : nullptr);
   const int ftail = s.first_gtail, lhead = s.last_ghead;
   if (s.unknown) {  // a benign query the cheap summary cannot decide: the host reruns with exact summaries
