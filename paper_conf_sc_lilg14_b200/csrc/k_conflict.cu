@@ -474,28 +474,53 @@ __device__ __forceinline__ AggC* scan_scratch<AggC>(TileSmem& s) { return s.wvc;
 
 template <class A>
 __device__ void tile_flags(const ConflictArgs& a, TileSmem& s, u32 cnt, const A cin[2], const A cout[2],
-                           A* part /* [4] or null */) {
+                           A* part /* [4] or null */, bool one_group = false) {
   typedef typename OpOf<A>::type Op;
   const u32 ws = a.ws, ls = a.ls;
   const A E = agg_empty_t<A>();
   // group level (identity = block): "another block" queries -> s.gq (bit3: benign query yes, bit4: unknown)
-  tile_allreduce<A>(
-      s.fl, FL_GH, FL_GT,
-      [&](int j) { return (s.fl[j] & FL_INT) ? agg_item_t<A>(s.rw[j], s.blk[j + 1], s.vh[j]) : E; }, Op(), E, cin[0],
-      cout[0],
-      [&](int j, const A& R) {
-        if (part && j == 0) part[0] = R;
-        if (part && j == (int)cnt - 1) part[1] = R;
-        if (!(s.fl[j] & FL_INT)) return;
-        const u32 b = s.blk[j + 1];
-        u8 g = (ex_id(R, RW_READ, b) ? 1 : 0) | (ex_id(R, RW_WRITE, b) ? 2 : 0) | (ex_id(R, RW_ATOMIC, b) ? 4 : 0);
-        if (s.rw[j] == RW_WRITE) {
-          const int q = wval3(R, b, s.vh[j]);
-          g |= q == 1 ? 8 : q == 2 ? 16 : 0;
-        }
-        s.gq[j] = g;
-      },
-      scan_scratch<A>(s), s.wf);
+  auto gitem = [&](int j) { return (s.fl[j] & FL_INT) ? agg_item_t<A>(s.rw[j], s.blk[j + 1], s.vh[j]) : E; };
+  auto gcb = [&](int j, const A& R) {
+    if (part && j == 0) part[0] = R;
+    if (part && j == (int)cnt - 1) part[1] = R;
+    if (!(s.fl[j] & FL_INT)) return;
+    const u32 b = s.blk[j + 1];
+    u8 g = (ex_id(R, RW_READ, b) ? 1 : 0) | (ex_id(R, RW_WRITE, b) ? 2 : 0) | (ex_id(R, RW_ATOMIC, b) ? 4 : 0);
+    if (s.rw[j] == RW_WRITE) {
+      const int q = wval3(R, b, s.vh[j]);
+      g |= q == 1 ? 8 : q == 2 ? 16 : 0;
+    }
+    s.gq[j] = g;
+  };
+  if (one_group) {
+    // the window is one piece of one run: its summary is carry in + a plain block reduction + carry out
+    A v = E;
+#pragma unroll
+    for (int q = 0; q < CT_ITEMS; q++) {
+      const int j = threadIdx.x * CT_ITEMS + q;
+      if (j < (int)cnt) v = Op()(v, gitem(j));
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v = Op()(v, shfl(v, o, true));
+    A* wv = scan_scratch<A>(s);
+    __shared__ A s_run;
+    if ((threadIdx.x & 31) == 0) wv[threadIdx.x >> 5] = v;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      A t = cin[0];
+      for (int w = 0; w < CT_THREADS / 32; w++) t = Op()(t, wv[w]);
+      s_run = Op()(t, cout[0]);
+    }
+    __syncthreads();
+    const A R = s_run;
+#pragma unroll
+    for (int q = 0; q < CT_ITEMS; q++) {
+      const int j = threadIdx.x * CT_ITEMS + q;
+      if (j < (int)cnt) gcb(j, R);
+    }
+  } else {
+    tile_allreduce<A>(s.fl, FL_GH, FL_GT, gitem, Op(), E, cin[0], cout[0], gcb, scan_scratch<A>(s), s.wf);
+  }
   __syncthreads();
   // sub-run level (identity = thread): same block and interval
   tile_allreduce<A>(
@@ -691,7 +716,7 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
     }
     return;
   }
-  tile_flags<A>(a, s, cnt, ci, co, MODE == 1 ? s_part : nullptr);
+  tile_flags<A>(a, s, cnt, ci, co, MODE == 1 ? s_part : nullptr, MODE == 2 && cin && cout && s.last_ghead < 0);
   const int ftail = s.first_gtail, lhead = s.last_ghead;
   if (s.unknown) {  // a benign query the cheap summary cannot decide: the host reruns with exact summaries
     if (tid == 0) atomicOr(a.need_exact, 1u);
