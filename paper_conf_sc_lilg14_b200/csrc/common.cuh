@@ -97,6 +97,20 @@ __device__ __forceinline__ u64 granule_of_hi(const KeyLayout& L, u64 hi) {
   return ((hi >> L.lowG) & lowmask(L.gbG)) + L.gminG;
 }
 
+// Lanes holding the same digit (stable peers) without __match_any_sync: MATCH runs on the slow ADU pipe on
+// sm_100 (ncu: 65-96% ADU busy), ballots run on the ALU pipe.  NB = digit bits to compare.
+template <int NB>
+__device__ __forceinline__ unsigned peers_of(u32 d) {
+  unsigned p = ~0u;
+#pragma unroll
+  for (int b = 0; b < NB; b++) {
+    const bool bit = (d >> b) & 1u;
+    const unsigned m = __ballot_sync(~0u, bit);
+    p &= bit ? m : ~m;
+  }
+  return p;
+}
+
 __device__ __forceinline__ unsigned lanemask_lt() {
   unsigned m;
   asm volatile("mov.u32 %0, %%lanemask_lt;" : "=r"(m));

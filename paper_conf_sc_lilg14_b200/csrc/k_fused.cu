@@ -169,15 +169,19 @@ __global__ void __launch_bounds__(FUSED_THREADS, FUSED_MINB) fused_extract_pass0
     // (3) stable warp ranking (peer masks by shared-memory atomicOr), each key stored into its tile slot
 #pragma unroll
     for (int i = 0; i < ITEMS; i++) {
+      // every 4th item's peer set by ballots (ALU pipe) instead of shared-memory masks (LSU pipe, the binding one)
+      const bool bal = (i & 3) == 0;
       const u32 d = digit(i);
-      atomicOr(&wm[d], 1u << lane);
-      __syncwarp();
-      const unsigned peers = wm[d];
+      if (!bal) {
+        atomicOr(&wm[d], 1u << lane);
+        __syncwarp();
+      }
+      const unsigned peers = bal ? peers_of<RADIX_BITS + 1>(d) : wm[d];
       const u32 c = wh[d];
       __syncwarp();
       if (d < RADIX) keys_s[c + __popc(peers & lt)] = ((u64)kh[i] << A.pos_bits) | (u64)(wbase + i * 32);
       if (lane == 31 - __clz(peers)) {
-        wm[d] = 0;
+        if (!bal) wm[d] = 0;
         if (d < RADIX) wh[d] = c + __popc(peers);
       }
       __syncwarp();

@@ -38,19 +38,6 @@ __device__ __forceinline__ u64 ld_relaxed(const u64* p) {
   return v;
 }
 
-// Lanes holding the same digit (stable peers) without __match_any_sync: MATCH runs on the slow ADU pipe on
-// sm_100 (ncu: 65-96% ADU busy), ballots run on the ALU pipe.  NB = digit bits to compare.
-template <int NB>
-__device__ __forceinline__ unsigned peers_of(u32 d) {
-  unsigned p = ~0u;
-#pragma unroll
-  for (int b = 0; b < NB; b++) {
-    const bool bit = (d >> b) & 1u;
-    const unsigned m = __ballot_sync(~0u, bit);
-    p &= bit ? m : ~m;
-  }
-  return p;
-}
 
 // global exclusive prefix of each pass's digit histogram -> bin_base[pass][digit]
 __global__ void bin_base_kernel(const u32* __restrict__ hist, u64* __restrict__ base) {
@@ -262,7 +249,7 @@ __global__ void __launch_bounds__(THREADS, MINB) onesweep_kernel(const u64* __re
 // only needed by the final coalesced write-out.  LATE_LB = walk the look-back after ranking (predecessors have
 // had the ranking time to publish their inclusive prefixes) instead of before.
 // ------------------------------------------------------------------------------------------------------------
-template <int THREADS, int ITEMS, int LBW, bool FULL, bool LATE_LB, int S, bool BAL, int TMA>
+template <int THREADS, int ITEMS, int LBW, bool FULL, bool LATE_LB, int S, bool BAL, int TMA, int MIX = 0>
 __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64* __restrict__ kout, u32 m, u32 shift,
                                                const u64* __restrict__ bin_base, u64* __restrict__ lookback,
                                                u32 epoch, u32 tile, unsigned char* smem, unsigned long long* prof,
@@ -380,20 +367,25 @@ __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64*
   const unsigned lt = lanemask_lt();
 #pragma unroll
   for (int i = 0; i < IPS; i++) {
+    // peer sets: shared-memory masks (LSU), ballots per digit bit (BAL, ALU) or, with MIX, odd items by ballots
+    // (MIX 1) or by MATCH (MIX 2, ADU) so that two pipes share the work
+    const bool bal = BAL || (MIX == 1 && (i & 1)) || (MIX == 3 && i % 3 == 0) || (MIX == 4 && i % 4 == 0) ||
+                     (MIX == 5 && i % 4 != 0);
+    const bool mat = MIX == 2 && (i & 1);
+    const bool msk = !bal && !mat;
     u32 d[S];
 #pragma unroll
     for (int q = 0; q < S; q++) {
       d[q] = digit(q * IPS + i);
-      if (!BAL) atomicOr(&wm[q * (RADIX + 1) + d[q]], 1u << lane);
+      if (msk) atomicOr(&wm[q * (RADIX + 1) + d[q]], 1u << lane);
     }
-    if (!BAL) __syncwarp();
+    if (msk) __syncwarp();
     unsigned peers[S];
     u32 c[S];
 #pragma unroll
     for (int q = 0; q < S; q++) {
-      // BAL: the peer set from one ballot per digit bit (ALU pipe, no shared-memory traffic)
-      peers[q] = BAL ? (FULL ? peers_of<RADIX_BITS>(d[q]) : peers_of<RADIX_BITS + 1>(d[q]))
-                     : wm[q * (RADIX + 1) + d[q]];
+      peers[q] = bal ? (FULL ? peers_of<RADIX_BITS>(d[q]) : peers_of<RADIX_BITS + 1>(d[q]))
+                     : mat ? __match_any_sync(~0u, d[q]) : wm[q * (RADIX + 1) + d[q]];
       c[q] = wh[q * RADIX + d[q]];
     }
     __syncwarp();
@@ -402,7 +394,7 @@ __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64*
       const bool leader = lane == 31 - __clz(peers[q]);
       if (FULL || d[q] < RADIX) keys_s[c[q] + __popc(peers[q] & lt)] = k[q * IPS + i];
       if (leader) {
-        if (!BAL) wm[q * (RADIX + 1) + d[q]] = 0;
+        if (msk) wm[q * (RADIX + 1) + d[q]] = 0;
         if (FULL || d[q] < RADIX) wh[q * RADIX + d[q]] = c[q] + __popc(peers[q]);
       }
     }
@@ -426,7 +418,7 @@ __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64*
   }
 }
 
-template <int THREADS, int ITEMS, int MINB, int LBW, bool LATE_LB, int S, bool BAL, int TMA>
+template <int THREADS, int ITEMS, int MINB, int LBW, bool LATE_LB, int S, bool BAL, int TMA, int MIX = 0>
 __global__ void __launch_bounds__(THREADS, MINB) onesweep2_kernel(const u64* __restrict__ kin, u64* __restrict__ kout,
                                                                   u32 m, u32 shift, const u64* __restrict__ bin_base,
                                                                   u64* __restrict__ lookback,
@@ -462,9 +454,9 @@ __global__ void __launch_bounds__(THREADS, MINB) onesweep2_kernel(const u64* __r
   unsigned long long* prof = g_prof ? g_prof + (u64)tile * 8 : nullptr;
   if (prof && tid == 0) prof[0] = gtime();
   if ((u64)(tile + 1) * TILE <= m)
-    onesweep2_tile<THREADS, ITEMS, LBW, true, LATE_LB, S, BAL, TMA>(kin, kout, m, shift, bin_base, lookback, epoch, tile, smem, prof, &ebar);
+    onesweep2_tile<THREADS, ITEMS, LBW, true, LATE_LB, S, BAL, TMA, MIX>(kin, kout, m, shift, bin_base, lookback, epoch, tile, smem, prof, &ebar);
   else
-    onesweep2_tile<THREADS, ITEMS, LBW, false, LATE_LB, S, BAL, TMA>(kin, kout, m, shift, bin_base, lookback, epoch, tile, smem, prof, &ebar);
+    onesweep2_tile<THREADS, ITEMS, LBW, false, LATE_LB, S, BAL, TMA, MIX>(kin, kout, m, shift, bin_base, lookback, epoch, tile, smem, prof, &ebar);
 }
 
 template <int THREADS, int ITEMS, int S, bool BAL>
@@ -474,10 +466,11 @@ static size_t onesweep2_smem() {
          (BAL ? 0 : (size_t)WARPS * S * (RADIX + 1) * 4);
 }
 
-template <int THREADS, int ITEMS, int MINB, int LBW, bool LATE_LB, int S = 1, bool BAL = false, int TMA = 0>
+template <int THREADS, int ITEMS, int MINB, int LBW, bool LATE_LB, int S = 1, bool BAL = false, int TMA = 0,
+          int MIX = 0>
 static void launch_os2(const u64* kin, u64* kout, u32 m, u32 shift, const u64* bin_base, u64* lookback,
                        u32* tile_ctr, u32 epoch, cudaStream_t st) {
-  auto kern = onesweep2_kernel<THREADS, ITEMS, MINB, LBW, LATE_LB, S, BAL, TMA>;
+  auto kern = onesweep2_kernel<THREADS, ITEMS, MINB, LBW, LATE_LB, S, BAL, TMA, MIX>;
   const size_t sm = onesweep2_smem<THREADS, ITEMS, S, BAL>();
   static bool set = false;
   if (!set) {
@@ -502,14 +495,17 @@ static size_t onesweep_smem() {
 //   33      as 20 with the tile loaded by TMA bulk copies;  34: 33 with the early look-back
 //   35      as 33 with 512 x 16 tiles
 //   36      as 33 with the bulk copies issued in the kernel prologue, right after the tile id, before the counter
-//           arrays are cleared (default: 4.88 vs 4.98 ms per 1e9-key pass)
+//           arrays are cleared (4.88 vs 4.98 ms per 1e9-key pass)
+//   41-45   as 36 with some items' peer sets by ballots (ALU pipe) instead of shared-memory masks (LSU pipe, the
+//           binding one): 41 every 2nd item 4.79, 43 every 3rd 4.81-4.93, 44 every 4th 4.78 (default),
+//           45 three of four 4.85;  42: every 2nd item by MATCH (ADU pipe) 5.70 ms
 // Measured and removed: a look-back sequencer CTA, a dedicated look-back warp, cluster-level (DSMEM) look-back,
 // 256 x 40/48 tiles — each slower.
 int sort_cfg() {
   static int v = -1;
   if (v < 0) {
     const char* e = getenv("SESA_SORT_CFG");
-    v = e ? atoi(e) : 36;
+    v = e ? atoi(e) : 44;
   }
   return v;
 }
@@ -517,7 +513,7 @@ int sort_cfg() {
 u32 sort_tile_keys() {
   switch (sort_cfg()) {
     case 1: case 15: return 256 * 24;
-    case 20: case 21: case 26: case 31: case 33: case 34: case 36: return 256 * 32;
+    case 20: case 21: case 26: case 31: case 33: case 34: case 36: case 41: case 42: case 43: case 44: case 45: return 256 * 32;
     case 35: return 512 * 16;
     default: return 256 * 16;
   }
@@ -570,6 +566,11 @@ static void launch_os_cfg(const u64* kin, u64* kout, const u32* vin, u32* vout, 
     case 34: launch_os2<256, 32, 2, 4, false, 1, false, 1>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
     case 35: launch_os2<512, 16, 2, 4, true, 1, false, 1>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
     case 36: launch_os2<256, 32, 2, 4, true, 1, false, 2>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 41: launch_os2<256, 32, 2, 4, true, 1, false, 2, 1>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 42: launch_os2<256, 32, 2, 4, true, 1, false, 2, 2>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 43: launch_os2<256, 32, 2, 4, true, 1, false, 2, 3>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 44: launch_os2<256, 32, 2, 4, true, 1, false, 2, 4>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
+    case 45: launch_os2<256, 32, 2, 4, true, 1, false, 2, 5>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
     case 26: launch_os2<256, 32, 2, 4, true, 2>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
     case 31: launch_os2<256, 32, 2, 4, true, 1, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
     default: launch_os<256, 16, 3, VALS, MATCH>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
