@@ -74,12 +74,13 @@ template <int U>
 // With regions (nreg > 0; sorted by (space, base), non-overlapping, space s in [rs[s], rs[s+1])), every valid
 // record of a space with regions is also checked for containment (OOB, NEXT-1): binary search for the last
 // region starting at or below addr, then addr + size <= end.
-// With gout != null the granule index addr >> log2G of every record is also written (8 bytes per record,
+// With gout != null the low 32 bits of the granule index addr >> log2G of every record are also written (4 bytes
+// per record,
 // coalesced): the fused pass then reads 8 bytes per record instead of the record's 32-byte sector.
 __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ rec, u32 n, u32 log2G, u32 rw,
                                                        Summary* __restrict__ out, u32* __restrict__ tile_hist,
                                                        const Region* __restrict__ regs, uint3 rs,
-                                                       u64* __restrict__ gout) {
+                                                       u32* __restrict__ gout) {
   __shared__ u32 s_th[8][RADIX];
   __shared__ u32 s_hb[3][RADIX];  // raw granule bytes 1..3 (with tile_hist)
   extern __shared__ Region s_reg[];  // [rs.z]
@@ -176,7 +177,7 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
           atomicAdd(&s_hb[2][(u32)(g >> 24) & (RADIX - 1)], 1u);
         }
       }
-      if (gout && r0 + u * 32 + lane < tend) __stcs(gout + r0 + u * 32 + lane, addr >> log2G);
+      if (gout && r0 + u * 32 + lane < tend) __stcs(gout + r0 + u * 32 + lane, (u32)(addr >> log2G));
     }
   }
   if (tile_hist) {
@@ -264,7 +265,7 @@ static int ring_grid(const void* kern, int threads, size_t smem, size_t smem_max
 }
 
 void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, u32* tile_hist, const Region* regs, u32 nreg,
-                    u32 nreg_shared, int grid, cudaStream_t st, u64* gout) {
+                    u32 nreg_shared, int grid, cudaStream_t st, u32* gout) {
   // extents2: contiguous warp ranges, one full wave of resident warps (the round-1 grid-stride kernel took
   // 7.7 ms on C5: 132 instructions per record, 64-bit index math and local-memory accumulators; this one 4.6 ms)
   static int sms = 0, per = 0;

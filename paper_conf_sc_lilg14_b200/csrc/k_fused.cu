@@ -90,7 +90,7 @@ size_t fused_temp_bytes(u64 n) {
 
 // ---- the fused kernel -------------------------------------------------------------------------------------------
 struct FusedArgs {
-  const u64* gran;  // granule index of every record (written by the extents pass)
+  const u32* gran;  // low 32 bits of every record's granule index (written by the extents pass)
   u32 n, log2G, pos_bits, npass;
   u64 gmin;
   const u32* toff;  // [T][RADIX] output offset of each tile's digit run
@@ -119,11 +119,12 @@ __global__ void __launch_bounds__(FUSED_THREADS, FUSED_MINB) fused_extract_pass0
   u32* wh = whist + warp * RADIX;
   u32* wm = wmask + warp * (RADIX + 1);
   const unsigned lt = lanemask_lt();
-  // (0) granule indices of a tile's records (8 bytes per record, coalesced), written by the extents pass
-  u64 a[ITEMS];
+  // (0) granule indices of a tile's records (low 32 bits: 4 bytes per record, coalesced), from the extents pass;
+  //     on this path the span is < 2^32, so key_hi = g - gmin = (low32(g) - low32(gmin)) mod 2^32
+  u32 a[ITEMS];
   auto issue = [&](u32 t) {
     const u32 wb = t * TILE + warp * 32 * ITEMS + lane;
-    const u64* gp = A.gran + wb;
+    const u32* gp = A.gran + wb;
 #pragma unroll
     for (int i = 0; i < ITEMS; i++)
       if (wb + i * 32 < A.n) a[i] = __ldcs(gp + i * 32);
@@ -138,7 +139,7 @@ __global__ void __launch_bounds__(FUSED_THREADS, FUSED_MINB) fused_extract_pass0
     // record index, known from (tile, warp, item, lane)
     u32 kh[ITEMS];
 #pragma unroll
-    for (int i = 0; i < ITEMS; i++) kh[i] = i < nv ? (u32)(a[i] - A.gmin) : 0u;
+    for (int i = 0; i < ITEMS; i++) kh[i] = i < nv ? a[i] - (u32)A.gmin : 0u;
     auto digit = [&](int i) -> u32 { return i < nv ? (kh[i] & (RADIX - 1)) : (u32)RADIX; };
     for (u32 i = tid; i < WARPS * RADIX; i += THREADS) whist[i] = 0;
     __syncthreads();
@@ -227,7 +228,7 @@ void launch_tile_offsets(u64 n, const KeyLayout& L, const u32* tile_hist, void* 
 }
 
 // temp: holds the tile offsets (launch_tile_offsets); hist: [npass][RADIX] zeroed (rows >= 1 filled)
-void launch_fused_extract_pass0(const u64* gran, u64 n, const KeyLayout& L, u32 npass, void* temp, u64* kout,
+void launch_fused_extract_pass0(const u32* gran, u64 n, const KeyLayout& L, u32 npass, void* temp, u64* kout,
                                 u32* hist, cudaStream_t st) {
   if (!n) return;
   const u32 T = (u32)((n + FUSED_TILE - 1) / FUSED_TILE);

@@ -23,9 +23,9 @@ constexpr int CT_TILE = CT_THREADS * CT_ITEMS;
 // k_extract.cu
 // tile_hist (optional, [ceil(n / FUSED_TILE)][RADIX]): per-tile histograms of (addr >> log2G) & 255 (k_fused.cu)
 // regs (optional, device, nreg <= MAX_REGIONS): sorted by (space, base), the first nreg_shared are SHARED
-// gout (optional, n x u64): granule index addr >> log2G of every record (input of the fused pass)
+// gout (optional, n x u32): low 32 bits of the granule index addr >> log2G of every record (fused-pass input)
 void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, u32* tile_hist, const Region* regs, u32 nreg,
-                    u32 nreg_shared, int grid, cudaStream_t st, u64* gout = nullptr);
+                    u32 nreg_shared, int grid, cudaStream_t st, u32* gout = nullptr);
 void launch_extract_1to1(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, u64* keys, u32* hist, u64 pos_base,
                          int grid, cudaStream_t st);
 void launch_entry_count(const Rec* rec, u64 n, u32 log2G, u32* cnt, cudaStream_t st);
@@ -38,7 +38,7 @@ bool fused_supported(u32 npass);
 size_t fused_temp_bytes(u64 n);
 void launch_tile_offsets(u64 n, const KeyLayout& L, const u32* tile_hist, void* temp, cudaStream_t st);
 // gran: the extents pass's granule indices (gout); rec is not read
-void launch_fused_extract_pass0(const u64* gran, u64 n, const KeyLayout& L, u32 npass, void* temp, u64* kout,
+void launch_fused_extract_pass0(const u32* gran, u64 n, const KeyLayout& L, u32 npass, void* temp, u64* kout,
                                 u32* hist, cudaStream_t st);
 
 // k_util.cu

@@ -246,10 +246,10 @@ bool sesa_trace::step_extents(const Rec* rec, u64 n, bool tile_hist) {
   if (!cuda_ok(cudaMemcpyAsync(b_summary.p, &h_summary, sizeof(Summary), cudaMemcpyHostToDevice, stream), "summary init"))
     return false;
   const int grid_stream = (int)std::min<u64>((n + 255) / 256, (u64)num_sms * 8);
-  LAUNCH("extents", (have_thist ? 40.0 : 32.0) * n, launch_extents(rec, n, log2G, (Summary*)b_summary.p,
+  LAUNCH("extents", (have_thist ? 36.0 : 32.0) * n, launch_extents(rec, n, log2G, (Summary*)b_summary.p,
                                              have_thist ? (u32*)b_thist.p : nullptr, (const Region*)b_regions.p,
                                              n_regions, n_regions_shared, grid_stream, stream,
-                                             have_thist ? (u64*)b_keys[0].p : nullptr));
+                                             have_thist ? (u32*)b_keys[0].p : nullptr));
   if (!cuda_ok(cudaMemcpyAsync(&h_summary, b_summary.p, sizeof(Summary), cudaMemcpyDeviceToHost, stream), "summary"))
     return false;
   return sync_check("extents");
@@ -318,8 +318,8 @@ bool sesa_trace::step_extract_fused(const Rec* rec, u64 n) {
   }
   LAUNCH("tile_offsets", 2.0 * RADIX * 4 * ((n + FUSED_TILE - 1) / FUSED_TILE),
          launch_tile_offsets(n, L, (const u32*)b_thist.p, b_ftmp.p, stream));
-  LAUNCH("extract_pass0", 16.0 * n,
-         launch_fused_extract_pass0((const u64*)b_keys[0].p, n, L, hist_from_extents ? 1u : npass, b_ftmp.p,
+  LAUNCH("extract_pass0", 12.0 * n,
+         launch_fused_extract_pass0((const u32*)b_keys[0].p, n, L, hist_from_extents ? 1u : npass, b_ftmp.p,
                                     (u64*)b_keys[1].p, (u32*)b_hist.p, stream));
   return true;
 }
