@@ -492,7 +492,47 @@ __device__ void tile_flags(const ConflictArgs& a, TileSmem& s, u32 cnt, const A 
     }
     s.gq[j] = g;
   };
-  if (one_group) {
+  // a shared location fixes its block, so "another block" never holds for shared entries: a tile of shared
+  // locations only (e.g. most of C2) skips the run-level scan
+  bool my_g = false;
+#pragma unroll
+  for (int q = 0; q < CT_ITEMS; q++) {
+    const int j = threadIdx.x * CT_ITEMS + q;
+    if (j < (int)cnt && (s.fl[j] & FL_INT)) my_g |= space_of_hi(a.L, s.key[j + 1] >> a.L.pos_bits) == SP_GLOBAL;
+  }
+  if (!__syncthreads_or(my_g)) {
+#pragma unroll
+    for (int q = 0; q < CT_ITEMS; q++) {
+      const int j = threadIdx.x * CT_ITEMS + q;
+      if (j < (int)cnt) s.gq[j] = 0;
+    }
+    if (part) {
+      // the carries (and the crossing-mode skips) still need the first / last run pieces: two masked reductions
+      const int ft = s.first_gtail, lh = s.last_ghead;
+      A p0 = E, p1 = E;
+#pragma unroll
+      for (int q = 0; q < CT_ITEMS; q++) {
+        const int j = threadIdx.x * CT_ITEMS + q;
+        if (j >= (int)cnt) continue;
+        const A it = gitem(j);
+        if (j <= ft) p0 = Op()(p0, it);
+        if (j >= lh) p1 = Op()(p1, it);
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) p0 = Op()(p0, shfl(p0, o, true)), p1 = Op()(p1, shfl(p1, o, true));
+      A* wv = scan_scratch<A>(s);
+      for (int r = 0; r < 2; r++) {
+        if ((threadIdx.x & 31) == 0) wv[threadIdx.x >> 5] = r ? p1 : p0;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+          A t = wv[0];
+          for (int w = 1; w < CT_THREADS / 32; w++) t = Op()(t, wv[w]);
+          part[r] = t;
+        }
+        __syncthreads();
+      }
+    }
+  } else if (one_group) {
     // the window is one piece of one run: its summary is carry in + a plain block reduction + carry out
     A v = E;
 #pragma unroll
