@@ -659,7 +659,7 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
       const A* pp = reinterpret_cast<const Q*>(a.part)[tile].a;    // [grp P, grp S, ...]
       const bool middle = (tf & TF_CIN) && (tf & TF_COUT) && !(tf & TF_GH);
       bool skip = true;
-      if (tf & TF_CIN) {  // piece A: the run crossing in (the whole tile if middle)
+      if ((tf & TF_CIN) && a.phase != 1) {  // piece A: the run crossing in (the whole tile if middle)
         bool done[2];
         const A run = middle ? Op()(Op()(c[0], pp[0]), c[1]) : Op()(c[0], pp[0]);
         cannot_race(run, &done[0], &done[1]);
@@ -673,7 +673,7 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
         }
         skip = skip && done[0] && done[1];
       }
-      if ((tf & TF_COUT) && (tf & TF_GH)) {  // piece B: a run starting here and crossing out
+      if ((tf & TF_COUT) && (tf & TF_GH) && a.phase != 2) {  // piece B: a run starting here and crossing out
         bool done[2];
         cannot_race(Op()(pp[1], c[1]), &done[0], &done[1]);
         skip = skip && done[0] && done[1];
@@ -877,7 +877,7 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
     // (position, entry index): the witness is the min POSITION (with an unsorted-input layout, entries of a run
     // are ordered by (block, interval) first); the entry index locates its record in mode 3
     const unsigned long long p = ((unsigned long long)pos_of(L, s.key[j + 1]) << 32) | (u32)(tb + j);
-    const bool A = cin && j <= ftail, B = cout && j >= lhead;
+    const bool A = cin && j <= ftail && a.phase != 1, B = cout && j >= lhead && a.phase != 2;
     if (A) {
       if (s.res[j] & 1) atomicMin(&s_min[0], p);
       if (s.res[j] & 2) atomicMin(&s_min[1], p);
@@ -913,7 +913,7 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_y_kernel(ConflictArgs a) 
     if (threadIdx.x == 0) {
       const u8 tf = a.tile_flags[tile];
       bool any = false;
-      if (tf & TF_CIN) {
+      if ((tf & TF_CIN) && a.phase != 1) {
         const Slot& sl = a.slots[a.owner[tile]];
         if (a.L.lowG == 0) {
           // the run crossing in, position-ordered: y_K (a minimum position) cannot come from here if a partner
@@ -927,7 +927,7 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_y_kernel(ConflictArgs a) 
           any |= sl.x[0] != ~0ull || sl.x[1] != ~0ull;
         }
       }
-      if ((tf & TF_COUT) && (tf & TF_GH)) {
+      if ((tf & TF_COUT) && (tf & TF_GH) && a.phase != 2) {
         const Slot& sl = a.slots[tile];
         any |= sl.x[0] != ~0ull || sl.x[1] != ~0ull;
       }
@@ -949,8 +949,8 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_y_kernel(ConflictArgs a) 
   __shared__ unsigned long long s_min[2][2];
   __shared__ u32 s_owner[2];
   if (tid == 0) {
-    s_owner[0] = cin ? a.owner[tile] : ~0u;
-    s_owner[1] = (cout && lhead >= 0 && !(cin && lhead <= ftail)) ? tile : ~0u;
+    s_owner[0] = cin && a.phase != 1 ? a.owner[tile] : ~0u;
+    s_owner[1] = (cout && lhead >= 0 && !(cin && lhead <= ftail)) && a.phase != 2 ? tile : ~0u;
   }
   __syncthreads();
   if (tid < 4) {

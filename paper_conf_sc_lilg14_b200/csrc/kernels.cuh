@@ -103,6 +103,7 @@ struct ConflictArgs {
   u32* owner;             // per tile: tile index holding the head of the group that crosses into this tile
   struct Slot* slots;     // per owner tile
   u64 index_base;
+  u32 phase;  // modes 2/3: 0 = every crossing piece, 1 = pieces starting a run (crossing out), 2 = the rest
 };
 
 struct RaceOut {  // == sesa_race (40 bytes)

@@ -448,13 +448,22 @@ bool sesa_trace::step_conflict(const u64* comp, u32 m2, const Rec* rec, u32 rec_
       info.crossing_tiles = cc[1];
       if (cc[1]) {
         LAUNCH("carry", 0.0, launch_carry(exact, A, ctiles, b_carrytmp.p, stream));
+        // pieces that start a run first (with position-ordered runs they hold its lowest positions, so the
+        // witnesses they find let the other pieces skip), then the rest
+        A.phase = 1;
+        LAUNCH("conflict_cross", 0.0, launch_conflict(2, exact, A, cc[1], stream));
+        A.phase = 2;
         LAUNCH("conflict_cross", 0.0, launch_conflict(2, exact, A, cc[1], stream));
         if (!exact) {
           if (!cuda_ok(cudaMemcpyAsync(cc, b_ccount.p, 12, cudaMemcpyDeviceToHost, stream), "counts")) return false;
           if (!sync_check("crossing")) return false;
           if (cc[2]) continue;
         }
+        A.phase = 1;
         LAUNCH("conflict_y", 0.0, launch_conflict(3, exact, A, cc[1], stream));
+        A.phase = 2;
+        LAUNCH("conflict_y", 0.0, launch_conflict(3, exact, A, cc[1], stream));
+        A.phase = 0;
         LAUNCH("cross_emit", 0.0, launch_cross_emit(A, cc[1], stream));
         if (!cuda_ok(cudaMemcpyAsync(cc, b_ccount.p, 12, cudaMemcpyDeviceToHost, stream), "counts")) return false;
         if (!sync_check("crossing")) return false;
