@@ -25,7 +25,12 @@
 // 2e5 of C5's 1e9 entries — cost 8 bytes of key traffic.
 #include "kernels.cuh"
 
+#ifndef CT_UNROLL
+#define CT_UNROLL 1
+#endif
+
 namespace sesa {
+constexpr int kCtUnroll = CT_UNROLL;
 
 // ------------------------------------------------------------------------------------------------ summaries
 __device__ __forceinline__ Agg agg_empty() {
@@ -261,14 +266,15 @@ __device__ __forceinline__ void tile_allreduce(const u8* fl, u8 hbit, u8 tbit, I
   // per-thread folds: F = from the last head to the end, B = from the start to the first tail
   T F = ident, B = ident;
   bool ff = false, bf = false;
-#pragma unroll
+  // loops kept rolled (CT_UNROLL): the kernels are instruction-cache bound when every item is inlined
+#pragma unroll kCtUnroll
   for (int q = 0; q < CT_ITEMS; q++) {
     const int j = j0 + q;
     const T it = item(j);
     if (fl[j] & hbit) F = it, ff = true;
     else F = op(F, it);
   }
-#pragma unroll
+#pragma unroll kCtUnroll
   for (int q = CT_ITEMS - 1; q >= 0; q--) {
     const int j = j0 + q;
     const T it = item(j);
@@ -402,7 +408,7 @@ __device__ bool tile_load(const ConflictArgs& a, TileSmem& s, u64 tb, u32 cnt) {
   __syncthreads();
   const int j0 = tid * CT_ITEMS;
   bool any = false;
-#pragma unroll
+#pragma unroll kCtUnroll
   for (int q = 0; q < CT_ITEMS; q++) {
     const int j = j0 + q;
     // items past the window's end carry no boundary flags: they are transparent to the segmented scans, so
@@ -441,7 +447,7 @@ __device__ bool tile_load(const ConflictArgs& a, TileSmem& s, u64 tb, u32 cnt) {
   }
   __syncthreads();
   // sub-runs: a new (block, interval) inside a group (contiguous: input order is (block, interval) order)
-#pragma unroll
+#pragma unroll kCtUnroll
   for (int q = 0; q < CT_ITEMS; q++) {
     const int j = j0 + q;
     u8 f = s.fl[j];
@@ -495,13 +501,13 @@ __device__ void tile_flags(const ConflictArgs& a, TileSmem& s, u32 cnt, const A 
   // a shared location fixes its block, so "another block" never holds for shared entries: a tile of shared
   // locations only (e.g. most of C2) skips the run-level scan
   bool my_g = false;
-#pragma unroll
+#pragma unroll kCtUnroll
   for (int q = 0; q < CT_ITEMS; q++) {
     const int j = threadIdx.x * CT_ITEMS + q;
     if (j < (int)cnt && (s.fl[j] & FL_INT)) my_g |= space_of_hi(a.L, s.key[j + 1] >> a.L.pos_bits) == SP_GLOBAL;
   }
   if (!__syncthreads_or(my_g)) {
-#pragma unroll
+#pragma unroll kCtUnroll
     for (int q = 0; q < CT_ITEMS; q++) {
       const int j = threadIdx.x * CT_ITEMS + q;
       if (j < (int)cnt) s.gq[j] = 0;
@@ -510,7 +516,7 @@ __device__ void tile_flags(const ConflictArgs& a, TileSmem& s, u32 cnt, const A 
       // the carries (and the crossing-mode skips) still need the first / last run pieces: two masked reductions
       const int ft = s.first_gtail, lh = s.last_ghead;
       A p0 = E, p1 = E;
-#pragma unroll
+#pragma unroll kCtUnroll
       for (int q = 0; q < CT_ITEMS; q++) {
         const int j = threadIdx.x * CT_ITEMS + q;
         if (j >= (int)cnt) continue;
@@ -535,7 +541,7 @@ __device__ void tile_flags(const ConflictArgs& a, TileSmem& s, u32 cnt, const A 
   } else if (one_group) {
     // the window is one piece of one run: its summary is carry in + a plain block reduction + carry out
     A v = E;
-#pragma unroll
+#pragma unroll kCtUnroll
     for (int q = 0; q < CT_ITEMS; q++) {
       const int j = threadIdx.x * CT_ITEMS + q;
       if (j < (int)cnt) v = Op()(v, gitem(j));
@@ -553,7 +559,7 @@ __device__ void tile_flags(const ConflictArgs& a, TileSmem& s, u32 cnt, const A 
     }
     __syncthreads();
     const A R = s_run;
-#pragma unroll
+#pragma unroll kCtUnroll
     for (int q = 0; q < CT_ITEMS; q++) {
       const int j = threadIdx.x * CT_ITEMS + q;
       if (j < (int)cnt) gcb(j, R);
@@ -713,7 +719,7 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
     if (tid == 0) s_fst = (int)cnt - 1, s_lsh = 0;
     __syncthreads();
     bool sh = false, st = false;
-#pragma unroll
+#pragma unroll kCtUnroll
     for (int q = 0; q < CT_ITEMS; q++) {
       const int j = tid * CT_ITEMS + q;
       if (j >= (int)cnt) continue;
@@ -724,7 +730,7 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
     const int fst = s_fst, lsh = s_lsh;
     const A E = agg_empty_t<A>();
     A g = E, p = E, q2 = E;
-#pragma unroll
+#pragma unroll kCtUnroll
     for (int q = 0; q < CT_ITEMS; q++) {
       const int j = tid * CT_ITEMS + q;
       if (j >= (int)cnt) continue;
@@ -767,7 +773,7 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
   if (MODE == 1) {
     // does the tile hold a sub-run head / tail anywhere? (block-wide votes over each thread's items)
     bool my_sh = false, my_st = false;
-#pragma unroll
+#pragma unroll kCtUnroll
     for (int q = 0; q < CT_ITEMS; q++) {
       const u32 j = tid * CT_ITEMS + q;
       if (j < cnt) my_sh |= (s.fl[j] & FL_SH) != 0, my_st |= (s.fl[j] & FL_ST) != 0;
@@ -798,7 +804,7 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
     // no flagged entry in a group internal to the tile (every internal group race-free, e.g. all of C2; or only
     // crossing pieces, e.g. the middle tiles of C3's hot bins — modes 2/3 own those): nothing to emit here
     bool my_res = false;
-#pragma unroll
+#pragma unroll kCtUnroll
     for (int q = 0; q < CT_ITEMS; q++) {
       const int j = tid * CT_ITEMS + q;
       if (j < (int)cnt && !(cin && j <= ftail) && !(cout && j >= lhead))
@@ -870,7 +876,7 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
   if (tid < 4) s_min[tid] = ~0ull;
   __syncthreads();
   const int j0 = tid * CT_ITEMS;
-#pragma unroll
+#pragma unroll kCtUnroll
   for (int q = 0; q < CT_ITEMS; q++) {
     const int j = j0 + q;
     if (j >= (int)cnt || !(s.fl[j] & FL_INT)) continue;
