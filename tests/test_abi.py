@@ -75,3 +75,23 @@ def test_no_cpu_fallback_without_device():
     assert lib.sesa_trace_create(ctypes.byref(c), ctypes.byref(h)) == S.SESA_ECUDA
     with pytest.raises(S.SesaError):
         S.Trace()
+
+
+def test_product_path_independent_of_oracle():
+    """The product (package + CUDA sources + generators) never names the oracle, and the oracle never names the
+    product: the two share no code (task rule ③)."""
+    pkg = os.path.join(ROOT, "paper_conf_sc_lilg14_b200")
+    product = [os.path.join(d, f) for d, _, fs in os.walk(pkg) for f in fs
+               if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp"))]
+    product += [os.path.join(ROOT, "include", f) for f in os.listdir(os.path.join(ROOT, "include"))]
+    assert len(product) > 10
+    for path in product:
+        text = open(path).read()
+        assert not re.search(r"^\s*(from|import)\s+oracle\b|#include\s*[<\"][^>\"]*oracle|sesa_oracle|oracle/_build",
+                             text, flags=re.M), path
+    odir = os.path.join(ROOT, "oracle")
+    for f in os.listdir(odir):
+        if f.endswith((".py", ".c", ".h")):
+            text = open(os.path.join(odir, f)).read()
+            assert not re.search(r"^\s*(from|import)\s+paper_conf_sc_lilg14_b200|#include\s*[<\"]sesa|libsesa\.so",
+                                 text, flags=re.M), f
