@@ -109,6 +109,17 @@ def test_random_medium_spans_tiles(sesa, seed):
     assert_same(sesa, r, 32, seed % 2, 4)
 
 
+@pytest.mark.parametrize("G_", [1, 64, 4096])
+def test_wide_accesses_extreme_granularity(sesa, G_):
+    # accesses of up to 300 bytes at G = 1 span up to 300 granules each (multi-granule extraction, entries >>
+    # records, runs crossing conflict tiles); at G = 4096 the whole shared window is one granule per block
+    for seed in range(3):
+        r = G.random_trace(3000 + 4111 * seed, 500 + seed, blocks=5, threads=200, intervals=3, words=900,
+                           sizes=(1, 3, 8, 64, 300), values=4, sort=seed != 1)
+        for ws, ls in ((32, 0), (32, 1), (4, 1)):
+            assert_same(sesa, r, ws, ls, G_, base=7 * seed)
+
+
 @pytest.mark.parametrize("words", [1, 3, 40, 700])
 def test_hot_locations_cross_tiles(sesa, words):
     # few words -> location runs of thousands of entries: runs and sub-runs cross conflict-tile boundaries

@@ -480,3 +480,16 @@ def test_bfs_shape_is_benign_ww():
     assert WW not in kinds and WWB in kinds
     changed = int(c4.cfg().changed_base)
     assert any(int(x["addr"]) == changed and int(x["kind"]) == WWB for x in got)
+
+
+@pytest.mark.parametrize("G_", [1, 64, 4096])
+def test_grouped_equals_brute_wide_accesses(G_):
+    """Multi-granule accesses: the grouped oracle agrees with the O(n^2) pair definition (include/sesa.h rules)."""
+    import sesagen as G
+    for seed in range(4):
+        r = G.random_trace(300, 900 + seed, blocks=3, threads=40, intervals=2, words=200,
+                           sizes=(1, 3, 8, 64, 300), values=3, sort=seed % 2 == 0)
+        for ws, ls in ((32, 0), (4, 1)):
+            a = O.check(r, warp_size=ws, lockstep=ls, granularity=G_, method="grouped")
+            b = O.check(r, warp_size=ws, lockstep=ls, granularity=G_, method="brute")
+            assert a.tobytes() == b.tobytes()
