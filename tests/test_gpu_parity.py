@@ -120,6 +120,13 @@ def test_wide_accesses_extreme_granularity(sesa, G_):
             assert_same(sesa, r, ws, ls, G_, base=7 * seed)
 
 
+def test_large_index_base(sesa):
+    # witnesses are u64 record indices offset by index_base (include/sesa.h): a base past 2^32 and 2^40
+    r = G.random_trace(5000, 77, blocks=4, threads=128, intervals=2, words=300)
+    for base in ((1 << 32) - 17, (1 << 40) + 3):
+        assert_same(sesa, r, 32, 0, 4, base=base)
+
+
 @pytest.mark.parametrize("words", [1, 3, 40, 700])
 def test_hot_locations_cross_tiles(sesa, words):
     # few words -> location runs of thousands of entries: runs and sub-runs cross conflict-tile boundaries
