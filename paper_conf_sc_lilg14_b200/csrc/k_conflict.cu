@@ -647,7 +647,8 @@ __device__ __forceinline__ u64 ld_volatile(const u64* p) { return *reinterpret_c
 
 // ------------------------------------------------------------------------------------------------ mode 1 / 2
 template <int MODE, class A>
-__global__ void __launch_bounds__(CT_THREADS) conflict_kernel(ConflictArgs a) {
+// mode 1 at 3 CTAs/SM (the shared-memory limit): up to 80 registers, no spills; mode 2 at 2 (128 registers)
+__global__ void __launch_bounds__(CT_THREADS, MODE == 1 ? 3 : 2) conflict_kernel(ConflictArgs a) {
   typedef typename QuadOf<A>::type Q;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
