@@ -16,7 +16,7 @@ constexpr int SORT_TILE = SORT_THREADS * SORT_ITEMS;
 
 // conflict tile: 256 threads x 6 entries (blocked; 1536-entry capacity, 3 CTAs/SM — measured against 4, 5, 7, 8:
 // C2 3.01 -> 2.62, C3 18.4 -> 16.1, C4 65.1 -> 55.7 ms from 8; 7 re-measured on the final tree: C3 7.76 -> 9.37,
-// C4 41.0 -> 45.3 ms, 2 CTAs/SM)
+// C4 41.0 -> 45.3 ms, 2 CTAs/SM; 5 with mode 1 at 4 CTAs/SM / 64 registers: C3 7.76 -> 8.91, C4 41.0 -> 44.5 ms)
 constexpr int CT_THREADS = 256;
 constexpr int CT_ITEMS = 6;
 constexpr int CT_TILE = CT_THREADS * CT_ITEMS;
