@@ -7,7 +7,8 @@ header for the rule-by-rule citations) with ctypes.  It shares no code with the 
 they match the C structs' sizes.
 
 Functions
-  check(records, index_base=0, warp_size=32, lockstep=0, granularity=4, method="grouped") -> races
+  check(records, index_base=0, warp_size=32, lockstep=0, granularity=4, method="grouped", threads=None) -> races
+      method = "brute" | "grouped" | "partitioned" (T threads, locations split by hash; same bytes as "grouped")
   pair_kind(rec_a, rec_b, warp_size, lockstep) -> 0 | 1 (RW) | 2 (WW)
   benign_pair(rec_a, rec_b) -> 0 | 1   (benign W/W pair: kind 3 with check(..., benign=True), NEXT-4)
   validate(records) -> None or lowest bad index
@@ -48,7 +49,7 @@ def build(force: bool = False) -> str:
     os.makedirs(os.path.dirname(_SO), exist_ok=True)
     if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
         tmp = _SO + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-Wall", "-o", tmp, _SRC])
+        subprocess.check_call(["gcc", "-O2", "-std=gnu11", "-fPIC", "-shared", "-pthread", "-Wall", "-o", tmp, _SRC])
         os.replace(tmp, _SO)
     return _SO
 
@@ -62,6 +63,8 @@ def _load():
             f = getattr(lib, name)
             f.argtypes = [P, U64, U64, U32, U32, U32, U32, P, U64, ctypes.POINTER(U64)]
             f.restype = ctypes.c_int
+        lib.oracle_check_partitioned.argtypes = [P, U64, U64, U32, U32, U32, U32, U32, P, U64, ctypes.POINTER(U64)]
+        lib.oracle_check_partitioned.restype = ctypes.c_int
         lib.oracle_pair_kind.argtypes = [P, P, U32, U32]
         lib.oracle_pair_kind.restype = ctypes.c_int
         lib.oracle_benign_pair.argtypes = [P, P]
@@ -92,19 +95,33 @@ def _as_recs(records) -> np.ndarray:
     return r
 
 
+def nthreads() -> int:
+    """Host threads the partitioned checker uses by default (the cores this process may run on)."""
+    try:
+        return max(1, len(os.sched_getaffinity(0)))
+    except AttributeError:  # pragma: no cover
+        return max(1, os.cpu_count() or 1)
+
+
 def check(records, index_base: int = 0, warp_size: int = 32, lockstep: int = 0, granularity: int = 4,
-          method: str = "grouped", benign: bool = False) -> np.ndarray:
+          method: str = "grouped", benign: bool = False, threads: int | None = None) -> np.ndarray:
     """Canonical race list (sorted by (space, block, interval, addr, kind)) of ``records``; with ``benign`` also
-    one kind-3 record per location holding a benign W/W pair (config flags bit 0, oracle_benign_pair)."""
+    one kind-3 record per location holding a benign W/W pair (config flags bit 0, oracle_benign_pair).
+    method: "brute" (all pairs), "grouped" (1 thread), "partitioned" (``threads`` threads, default nthreads())."""
     lib = _load()
     r = _as_recs(records)
-    fn = lib.oracle_check_brute if method == "brute" else lib.oracle_check_grouped
+    T = nthreads() if threads is None else int(threads)
     cap = 1024
     while True:
         out = np.zeros(cap, RACE_DTYPE)
         nout = ctypes.c_uint64(0)
-        rc = fn(r.ctypes.data if len(r) else None, len(r), index_base, warp_size, lockstep, granularity,
-                1 if benign else 0, out.ctypes.data, cap, ctypes.byref(nout))
+        args = (r.ctypes.data if len(r) else None, len(r), index_base, warp_size, lockstep, granularity,
+                1 if benign else 0)
+        if method == "partitioned":
+            rc = lib.oracle_check_partitioned(*args, T, out.ctypes.data, cap, ctypes.byref(nout))
+        else:
+            fn = lib.oracle_check_brute if method == "brute" else lib.oracle_check_grouped
+            rc = fn(*args, out.ctypes.data, cap, ctypes.byref(nout))
         if rc == 7:
             cap = int(nout.value)
             continue

@@ -20,13 +20,17 @@
  *   oracle_check_grouped — group entries by location (qsort), per location decide "has a partner of kind K"
  *                          by COUNTING partners (inclusion-exclusion over sorted tuples), then witness
  *                          x = min flagged index, y = min s with P(x, s) of kind K.  O(n log n).
- * With flag F_BENIGN both also report benign W/W pairs as a third kind (oracle_benign_pair).
+ *   oracle_check_partitioned — checker 2 on T threads: locations partitioned by a hash of λ mod T (a race is a
+ *                          property of one location, c.1), each thread runs the unchanged group algorithm on its
+ *                          partition; byte-identical output (SURVEY §8c.3 "T-thread mode"; full-size parity).
+ * With flag F_BENIGN all three also report benign W/W pairs as a third kind (oracle_benign_pair).
  * They agree on every input (tests/test_oracle.py); the GPU path uses neither method (it uses per-run
  * min/max summaries), so agreement of the GPU with this oracle is not circular.
  *
  * Also: oracle_validate (the record validity rules of include/sesa.h, re-stated) and oracle_expand (the
  * parametric-flow instantiation "replace i by j", §IV-A).
  */
+#include <pthread.h>
 #include <stdint.h>
 #include <stdlib.h>
 #include <string.h>
@@ -266,13 +270,15 @@ static int entry_cmp(const void *pa, const void *pb) {
 typedef struct {
   uint64_t f[6];
 } tup;
-static int g_nf; /* number of fields compared by tup_cmp (qsort has no context argument) */
 static int tup_cmp_n(const tup *a, const tup *b, int nf) {
   for (int k = 0; k < nf; k++)
     if (a->f[k] != b->f[k]) return a->f[k] < b->f[k] ? -1 : 1;
   return 0;
 }
-static int tup_cmp(const void *pa, const void *pb) { return tup_cmp_n((const tup *)pa, (const tup *)pb, g_nf); }
+/* qsort has no context argument: one comparator per field count (no global state, so worker threads of
+ * oracle_check_partitioned can sort concurrently) */
+static int tup_cmp4(const void *pa, const void *pb) { return tup_cmp_n((const tup *)pa, (const tup *)pb, 4); }
+static int tup_cmp5(const void *pa, const void *pb) { return tup_cmp_n((const tup *)pa, (const tup *)pb, 5); }
 
 /* number of tuples in sorted array a[0..k) whose first nf fields equal q's */
 static uint64_t count_prefix(const tup *a, uint64_t k, const tup *q, int nf) {
@@ -300,29 +306,26 @@ static uint64_t count_prefix(const tup *a, uint64_t k, const tup *q, int nf) {
  *   RW(r)  = r read:  Σ_{X∈{W,A}} OB(X) + (ls ? SW(X) : ST(X));  r write/atomic: OB(R) + (ls ? SW(R) : ST(R))
  *   WW(r)  = r write: OB(A)+ST(A) + OB(W)+ST(W) - EQ;  r atomic: OB(W)+ST(W);  r read: 0
  *   B(r)   = r write: EQ (its benign partners, oracle_benign_pair);  otherwise 0                              */
-static int group_flags(const orec *r, const entry *e, uint64_t k, uint32_t ws, uint32_t ls, uint8_t *flag_rw,
-                       uint8_t *flag_ww, uint8_t *flag_b) {
-  tup *A = (tup *)malloc(k * sizeof(tup)); /* (type, block, interval, thread) */
-  tup *B = (tup *)malloc(k * sizeof(tup)); /* (type, block, interval, warp)   */
-  tup *V = (tup *)malloc(k * sizeof(tup)); /* (type, value, block, interval, thread) */
-  if (!A || !B || !V) {
-    free(A); free(B); free(V);
-    return 3;
-  }
-  for (uint64_t a = 0; a < k; a++) {
-    const orec *x = &r[e[a].idx];
-    memset(&A[a], 0, sizeof(tup));
-    memset(&B[a], 0, sizeof(tup));
-    memset(&V[a], 0, sizeof(tup));
-    A[a].f[0] = x->rw; A[a].f[1] = x->block; A[a].f[2] = x->interval; A[a].f[3] = x->thread;
-    B[a].f[0] = x->rw; B[a].f[1] = x->block; B[a].f[2] = x->interval; B[a].f[3] = x->thread / ws;
-    V[a].f[0] = x->rw; V[a].f[1] = x->value_hash; V[a].f[2] = x->block; V[a].f[3] = x->interval;
-    V[a].f[4] = x->thread;
-  }
-  g_nf = 4; qsort(A, k, sizeof(tup), tup_cmp);
-  g_nf = 4; qsort(B, k, sizeof(tup), tup_cmp);
-  g_nf = 5; qsort(V, k, sizeof(tup), tup_cmp);
-  for (uint64_t a = 0; a < k; a++) {
+typedef struct {
+  const orec *r;
+  const entry *e;
+  uint64_t k;
+  uint32_t ws, ls;
+  tup *A, *B, *V;
+  uint8_t *flag_rw, *flag_ww, *flag_b;
+  uint64_t a0, a1; /* entries this worker flags */
+  tup *sort_arr;   /* sort worker: the array and its field count */
+  int sort_nf;
+} gjob;
+
+/* the counts and flags of entries [a0, a1) of one group (A, B, V sorted) */
+static void flags_range(const gjob *g) {
+  const orec *r = g->r;
+  const entry *e = g->e;
+  const uint64_t k = g->k;
+  const uint32_t ws = g->ws, ls = g->ls;
+  const tup *A = g->A, *B = g->B, *V = g->V;
+  for (uint64_t a = g->a0; a < g->a1; a++) {
     const orec *x = &r[e[a].idx];
     uint64_t OB[3], ST[3], SW[3];
     for (int X = 0; X < 3; X++) {
@@ -352,43 +355,94 @@ static int group_flags(const orec *r, const entry *e, uint64_t k, uint32_t ws, u
     } else if (x->rw == AT) {
       ww = OB[WR] + ST[WR];
     }
-    flag_rw[a] = rw > 0;
-    flag_ww[a] = ww > 0;
-    flag_b[a] = eq > 0;
+    g->flag_rw[a] = rw > 0;
+    g->flag_ww[a] = ww > 0;
+    g->flag_b[a] = eq > 0;
+  }
+}
+
+static void *flags_worker(void *arg) {
+  flags_range((const gjob *)arg);
+  return NULL;
+}
+static void *sort_worker(void *arg) {
+  gjob *g = (gjob *)arg;
+  qsort(g->sort_arr, g->k, sizeof(tup), g->sort_nf == 5 ? tup_cmp5 : tup_cmp4);
+  return NULL;
+}
+
+/* Groups this large are sorted and counted by `par` threads (the arithmetic is unchanged: the three sorts
+ * are independent and every entry's counts only read the sorted arrays). */
+#define GROUP_PAR_MIN (1u << 20)
+
+static int group_flags(const orec *r, const entry *e, uint64_t k, uint32_t ws, uint32_t ls, uint8_t *flag_rw,
+                       uint8_t *flag_ww, uint8_t *flag_b, uint32_t par) {
+  tup *A = (tup *)malloc(k * sizeof(tup)); /* (type, block, interval, thread) */
+  tup *B = (tup *)malloc(k * sizeof(tup)); /* (type, block, interval, warp)   */
+  tup *V = (tup *)malloc(k * sizeof(tup)); /* (type, value, block, interval, thread) */
+  if (!A || !B || !V) {
+    free(A); free(B); free(V);
+    return 3;
+  }
+  for (uint64_t a = 0; a < k; a++) {
+    const orec *x = &r[e[a].idx];
+    memset(&A[a], 0, sizeof(tup));
+    memset(&B[a], 0, sizeof(tup));
+    memset(&V[a], 0, sizeof(tup));
+    A[a].f[0] = x->rw; A[a].f[1] = x->block; A[a].f[2] = x->interval; A[a].f[3] = x->thread;
+    B[a].f[0] = x->rw; B[a].f[1] = x->block; B[a].f[2] = x->interval; B[a].f[3] = x->thread / ws;
+    V[a].f[0] = x->rw; V[a].f[1] = x->value_hash; V[a].f[2] = x->block; V[a].f[3] = x->interval;
+    V[a].f[4] = x->thread;
+  }
+  gjob g;
+  memset(&g, 0, sizeof g);
+  g.r = r; g.e = e; g.k = k; g.ws = ws; g.ls = ls; g.A = A; g.B = B; g.V = V;
+  g.flag_rw = flag_rw; g.flag_ww = flag_ww; g.flag_b = flag_b;
+  if (par <= 1 || k < GROUP_PAR_MIN) {
+    qsort(A, k, sizeof(tup), tup_cmp4);
+    qsort(B, k, sizeof(tup), tup_cmp4);
+    qsort(V, k, sizeof(tup), tup_cmp5);
+    g.a0 = 0; g.a1 = k;
+    flags_range(&g);
+  } else {
+    gjob s[3];
+    pthread_t th[64];
+    tup *arr[3] = {A, B, V};
+    for (int q = 0; q < 3; q++) {
+      s[q] = g;
+      s[q].sort_arr = arr[q];
+      s[q].sort_nf = q == 2 ? 5 : 4;
+    }
+    int ok[3];
+    for (int q = 1; q < 3; q++) ok[q] = pthread_create(&th[q], NULL, sort_worker, &s[q]) == 0;
+    sort_worker(&s[0]);
+    for (int q = 1; q < 3; q++) {
+      if (ok[q]) pthread_join(th[q], NULL);
+      else sort_worker(&s[q]);
+    }
+    const uint32_t P = par > 64 ? 64 : par;
+    gjob w[64];
+    for (uint32_t t = 0; t < P; t++) {
+      w[t] = g;
+      w[t].a0 = k * t / P;
+      w[t].a1 = k * (t + 1) / P;
+    }
+    int okw[64];
+    for (uint32_t t = 1; t < P; t++) okw[t] = pthread_create(&th[t], NULL, flags_worker, &w[t]) == 0;
+    flags_range(&w[0]);
+    for (uint32_t t = 1; t < P; t++) {
+      if (okw[t]) pthread_join(th[t], NULL);
+      else flags_range(&w[t]);
+    }
   }
   free(A); free(B); free(V);
   return 0;
 }
 
-int oracle_check_grouped(const orec *r, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls, uint32_t G,
-                         uint32_t flags, orace *out, uint64_t cap, uint64_t *nout) {
-  if (!oracle_config_ok(ws, ls, G) || (flags & ~F_BENIGN)) return 2;
-  uint64_t bad;
-  if (oracle_validate(r, n, &bad)) {
-    *nout = bad;
-    return 1;
-  }
-  /* entries = (record, granule) pairs */
-  uint64_t m = 0;
-  for (uint64_t i = 0; i < n; i++) {
-    uint64_t lo, hi;
-    granules(&r[i], G, &lo, &hi);
-    m += hi - lo + 1;
-  }
-  entry *e = (entry *)malloc((m ? m : 1) * sizeof(entry));
-  if (!e) return 3;
-  uint64_t p = 0;
-  for (uint64_t i = 0; i < n; i++) {
-    uint64_t lo, hi;
-    granules(&r[i], G, &lo, &hi);
-    for (uint64_t g = lo; g <= hi; g++) {
-      e[p].L = loc_of(&r[i], g);
-      e[p].idx = i;
-      p++;
-    }
-  }
-  qsort(e, m, sizeof(entry), entry_cmp);
-  cvec c = {0, 0, 0};
+/* Entries e[0..m) sorted by (λ, record index): per group (all entries at one λ) flags by counting, then the
+ * canonical witness per kind; candidates are appended to *c.  Returns 0, 3 (no memory) or 9 (counting bug). */
+static int process_groups(const orec *r, const entry *e, uint64_t m, uint32_t ws, uint32_t ls, uint32_t flags,
+                          uint32_t par, cvec *c) {
   int rc = 0;
   uint8_t *frw = NULL, *fww = NULL, *fb = NULL;
   uint64_t fcap = 0;
@@ -403,7 +457,7 @@ int oracle_check_grouped(const orec *r, uint64_t n, uint64_t base, uint32_t ws, 
         fcap = k;
         if (!frw || !fww || !fb) { rc = 3; break; }
       }
-      rc = group_flags(r, &e[a], k, ws, ls, frw, fww, fb);
+      rc = group_flags(r, &e[a], k, ws, ls, frw, fww, fb, par);
       if (rc) break;
       const int kmax = (flags & F_BENIGN) ? K_WWB : K_WW;
       for (int K = K_RW; K <= kmax; K++) {
@@ -428,12 +482,143 @@ int oracle_check_grouped(const orec *r, uint64_t n, uint64_t base, uint32_t ws, 
         cd.kind = (uint32_t)K;
         cd.i = e[a + xa].idx < y ? e[a + xa].idx : y;
         cd.j = e[a + xa].idx < y ? y : e[a + xa].idx;
-        if (cpush(&c, cd)) { rc = 3; break; }
+        if (cpush(c, cd)) { rc = 3; break; }
       }
     }
     a = b;
   }
-  free(frw); free(fww); free(fb); free(e);
+  free(frw); free(fww); free(fb);
+  return rc;
+}
+
+/* hash of a location λ (splitmix64 finaliser, the same mix as oracle_expand's value hash) */
+static uint64_t mix(uint64_t x);
+static uint64_t loc_hash(const loc *L) {
+  return mix(mix(mix(((uint64_t)L->space << 32) ^ L->block) ^ L->interval) ^ L->g);
+}
+
+/* Entries of the records whose location hash falls in partition `part` of `nparts` (nparts == 1: every entry),
+ * sorted by (λ, record index); *m_out = count.  NULL on no memory (*m_out = UINT64_MAX). */
+static entry *collect_entries(const orec *r, uint64_t n, uint32_t G, uint32_t part, uint32_t nparts,
+                              uint64_t *m_out) {
+  uint64_t m = 0;
+  for (uint64_t i = 0; i < n; i++) {
+    uint64_t lo, hi;
+    granules(&r[i], G, &lo, &hi);
+    for (uint64_t g = lo; g <= hi; g++) {
+      if (nparts > 1) {
+        loc L = loc_of(&r[i], g);
+        if (loc_hash(&L) % nparts != part) continue;
+      }
+      m++;
+    }
+  }
+  entry *e = (entry *)malloc((m ? m : 1) * sizeof(entry));
+  if (!e) {
+    *m_out = UINT64_MAX;
+    return NULL;
+  }
+  uint64_t p = 0;
+  for (uint64_t i = 0; i < n; i++) {
+    uint64_t lo, hi;
+    granules(&r[i], G, &lo, &hi);
+    for (uint64_t g = lo; g <= hi; g++) {
+      loc L = loc_of(&r[i], g);
+      if (nparts > 1 && loc_hash(&L) % nparts != part) continue;
+      e[p].L = L;
+      e[p].idx = i;
+      p++;
+    }
+  }
+  qsort(e, m, sizeof(entry), entry_cmp);
+  *m_out = m;
+  return e;
+}
+
+int oracle_check_grouped(const orec *r, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls, uint32_t G,
+                         uint32_t flags, orace *out, uint64_t cap, uint64_t *nout) {
+  if (!oracle_config_ok(ws, ls, G) || (flags & ~F_BENIGN)) return 2;
+  uint64_t bad;
+  if (oracle_validate(r, n, &bad)) {
+    *nout = bad;
+    return 1;
+  }
+  /* entries = (record, granule) pairs, grouped by location */
+  uint64_t m = 0;
+  entry *e = collect_entries(r, n, G, 0, 1, &m);
+  if (!e) return 3;
+  cvec c = {0, 0, 0};
+  int rc = process_groups(r, e, m, ws, ls, flags, 1, &c);
+  free(e);
+  if (rc) {
+    free(c.v);
+    return rc;
+  }
+  rc = emit_sorted(&c, G, base, out, cap, nout);
+  free(c.v);
+  return rc;
+}
+
+/* ---- checker 2, T threads: the locations are partitioned by loc_hash mod T (SURVEY §8c.3 "T-thread mode").
+ * A race is a property of one location (c.1), so every group lands whole in one partition and each thread
+ * runs the unchanged group algorithm on its partition; the candidate lists are concatenated and emitted in
+ * the canonical order.  The result is byte-identical to oracle_check_grouped (tests/test_oracle.py).       */
+typedef struct {
+  const orec *r;
+  uint64_t n;
+  uint32_t ws, ls, G, flags, part, nparts;
+  cvec c;
+  int rc;
+} pjob;
+
+static void *pworker(void *arg) {
+  pjob *j = (pjob *)arg;
+  uint64_t m = 0;
+  entry *e = collect_entries(j->r, j->n, j->G, j->part, j->nparts, &m);
+  if (!e) {
+    j->rc = 3;
+    return NULL;
+  }
+  j->rc = process_groups(j->r, e, m, j->ws, j->ls, j->flags, j->nparts, &j->c);
+  free(e);
+  return NULL;
+}
+
+int oracle_check_partitioned(const orec *r, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls, uint32_t G,
+                             uint32_t flags, uint32_t T, orace *out, uint64_t cap, uint64_t *nout) {
+  if (!oracle_config_ok(ws, ls, G) || (flags & ~F_BENIGN)) return 2;
+  if (T < 1) T = 1;
+  if (T > 1024) T = 1024;
+  uint64_t bad;
+  if (oracle_validate(r, n, &bad)) {
+    *nout = bad;
+    return 1;
+  }
+  pjob *jobs = (pjob *)calloc(T, sizeof(pjob));
+  pthread_t *th = (pthread_t *)calloc(T, sizeof(pthread_t));
+  if (!jobs || !th) {
+    free(jobs); free(th);
+    return 3;
+  }
+  for (uint32_t t = 0; t < T; t++) {
+    jobs[t].r = r; jobs[t].n = n; jobs[t].ws = ws; jobs[t].ls = ls; jobs[t].G = G; jobs[t].flags = flags;
+    jobs[t].part = t; jobs[t].nparts = T;
+  }
+  for (uint32_t t = 1; t < T; t++)
+    if (pthread_create(&th[t], NULL, pworker, &jobs[t]) != 0) jobs[t].rc = -1;
+  pworker(&jobs[0]);
+  int rc = jobs[0].rc;
+  for (uint32_t t = 1; t < T; t++) {
+    if (jobs[t].rc == -1) { pworker(&jobs[t]); } /* thread creation failed: run it here */
+    else pthread_join(th[t], NULL);
+    if (jobs[t].rc && !rc) rc = jobs[t].rc;
+  }
+  cvec c = {0, 0, 0};
+  for (uint32_t t = 0; t < T && !rc; t++)
+    for (uint64_t q = 0; q < jobs[t].c.n && !rc; q++)
+      if (cpush(&c, jobs[t].c.v[q])) rc = 3;
+  for (uint32_t t = 0; t < T; t++) free(jobs[t].c.v);
+  free(jobs); free(th);
   if (rc) {
     free(c.v);
     return rc;

@@ -35,6 +35,15 @@ class C4Cfg(ctypes.Structure):
                 ("row_base", ctypes.c_uint64), ("col_base", ctypes.c_uint64), ("changed_base", ctypes.c_uint64)]
 
 
+class RndCfg(ctypes.Structure):
+    _fields_ = [("seed", ctypes.c_uint64), ("n", ctypes.c_uint64), ("blocks", ctypes.c_uint32),
+                ("threads", ctypes.c_uint32), ("intervals", ctypes.c_uint32), ("words", ctypes.c_uint32),
+                ("shared_pm", ctypes.c_uint32), ("atomic_pm", ctypes.c_uint32), ("write_pm", ctypes.c_uint32),
+                ("values", ctypes.c_uint32), ("nsizes", ctypes.c_uint32), ("sorted", ctypes.c_uint32),
+                ("unaligned", ctypes.c_uint32), ("pad", ctypes.c_uint32), ("sizes", ctypes.c_uint16 * 4),
+                ("gbase", ctypes.c_uint64)]
+
+
 _host = _dev = None
 
 
@@ -51,6 +60,8 @@ def _hostlib():
         _host.gen_c4_layout_host.argtypes = [P, P, P, P]
         _host.gen_c4_layout_host.restype = U64
         _host.gen_c4_host.argtypes = [P, P, P, P, P]
+        _host.gen_random_host.argtypes = [P, U64, U64, P]
+        assert _host.gen_sizeof_rndcfg() == ctypes.sizeof(RndCfg)
         assert _host.gen_sizeof_c3cfg() == ctypes.sizeof(C3Cfg)
         assert _host.gen_sizeof_c4cfg() == ctypes.sizeof(C4Cfg)
         assert _host.gen_sizeof_c5cfg() == ctypes.sizeof(C5Cfg)
@@ -251,3 +262,22 @@ class C4:
                                     ctypes.c_void_p(rows.data_ptr()), ctypes.c_void_p(off.data_ptr()),
                                     ctypes.c_void_p(out.data_ptr()), s) == 0
         return out, n
+
+
+# ---------------------------------------------------------------------------------------------------- random
+def rnd_cfg(n: int, seed: int, *, blocks: int = 3, threads: int = 70, intervals: int = 3, words: int = 24,
+            shared_frac: float = 0.5, sizes=(1, 2, 4, 8), atomic_frac: float = 0.15, write_frac: float = 0.35,
+            values: int = 3, sort: bool = True, unaligned: bool = True) -> RndCfg:
+    sz = (ctypes.c_uint16 * 4)(*(list(sizes) + [1] * (4 - len(sizes))))
+    return RndCfg(SEED_BASE + 0x100 + seed, n, blocks, threads, intervals, words, int(round(shared_frac * 1000)),
+                  int(round(atomic_frac * 1000)), int(round(write_frac * 1000)), values, len(sizes), int(sort),
+                  int(unaligned), 0, sz, 0x10000000000)
+
+
+def rnd_host(n: int, seed: int, **kw) -> np.ndarray:
+    """Counter-based random trace (gen_common.h rnd_record): a C twin of sesagen.random_trace for large sweeps."""
+    c = rnd_cfg(n, seed, **kw)
+    out = np.zeros(n, REC_DTYPE)
+    if n:
+        _hostlib().gen_random_host(ctypes.byref(c), 0, n, out.ctypes.data)
+    return out

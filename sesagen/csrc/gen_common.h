@@ -192,4 +192,43 @@ GEN_HD void c4_write(const c4cfg *c, const uint64_t *dcdf, uint64_t v, uint64_t 
     }
   }
 }
+/* ------------------------------------------------------------------------------------------------ random
+ * Random traces for property sweeps (oracle self-consistency, GPU parity).  Record i is a pure function of
+ * (cfg, i): block / interval either from the position (sorted = 1: (block, interval) ascending, the canonical
+ * schedule of P:257) or hashed; thread, space, access kind, size, word (+ in-word offset) and value from
+ * independent hashes.  Dense collisions come from a small `words`.  No race-check arithmetic. */
+typedef struct {
+  uint64_t seed, n;
+  uint32_t blocks, threads, intervals, words;
+  uint32_t shared_pm, atomic_pm, write_pm; /* per mille */
+  uint32_t values;                         /* value hashes in [0, values) */
+  uint32_t nsizes, sorted, unaligned, pad;
+  uint16_t sizes[4];
+  uint64_t gbase;                          /* global addresses: gbase + 4 * word + offset */
+} rndcfg;
+
+GEN_HD void rnd_record(const rndcfg *c, uint64_t i, grec *r) {
+  const uint64_t h = gmix(c->seed ^ gmix(i));
+  const uint64_t h1 = gmix(h + 1), h2 = gmix(h + 2), h3 = gmix(h + 3), h4 = gmix(h + 4), h5 = gmix(h + 5),
+                 h6 = gmix(h + 6), h7 = gmix(h + 7);
+  uint32_t b, iv;
+  if (c->sorted) {
+    const uint64_t cells = (uint64_t)c->blocks * c->intervals;
+    const uint64_t bi = c->n ? (uint64_t)(((unsigned __int128)i * cells) / c->n) : 0;
+    b = (uint32_t)(bi / c->intervals);
+    iv = (uint32_t)(bi % c->intervals);
+  } else {
+    b = (uint32_t)(h1 % c->blocks);
+    iv = (uint32_t)((h1 >> 32) % c->intervals);
+  }
+  const uint32_t t = (uint32_t)(h2 % c->threads);
+  const uint8_t sp = (h3 % 1000) < c->shared_pm ? G_SHARED : G_GLOBAL;
+  const uint32_t u = (uint32_t)(h4 % 1000);
+  const uint8_t rw = u < c->atomic_pm ? G_A : u < c->atomic_pm + c->write_pm ? G_W : G_R;
+  const uint16_t sz = c->sizes[h5 % c->nsizes];
+  const uint64_t w = h6 % c->words, off = c->unaligned ? (h6 >> 40) % 4 : 0;
+  const uint64_t addr = sp == G_GLOBAL ? c->gbase + 4 * w + off : 4 * w + off;
+  gset(r, addr, h7 % c->values, b, t, iv, sz, sp, rw);
+}
+
 #endif

@@ -51,6 +51,12 @@ void gen_c4_host(const c4cfg *c, const uint64_t *dcdf, const uint64_t *rows, con
   }
 }
 
+/* records [lo, hi) of a random trace */
+void gen_random_host(const rndcfg *c, uint64_t lo, uint64_t hi, grec *out) {
+  for (uint64_t i = lo; i < hi; i++) rnd_record(c, i, &out[i - lo]);
+}
+
+uint64_t gen_sizeof_rndcfg(void) { return sizeof(rndcfg); }
 uint64_t gen_sizeof_c3cfg(void) { return sizeof(c3cfg); }
 uint64_t gen_sizeof_c4cfg(void) { return sizeof(c4cfg); }
 uint64_t gen_sizeof_c5cfg(void) { return sizeof(c5cfg); }

@@ -1,10 +1,10 @@
 """Parity at BASELINE.json's full sizes, in the launch configuration bench.py times.
 
-C5 (1e9 records) is compared in full with its construction truth; C2 (18.3 M) must be race-free; C3 (101.4 M) and
-C4 (412 M) are checked on SAMPLED locations: the oracle gets every record touching a sampled location (taken from
-the host generator, which produces the same bytes as the device generator — tests/test_generators.py), and the
-GPU's races at those locations must equal the oracle's exactly (witnesses included).  Races are a property of one
-location, so this is exact for the sample.  Plus whole-trace invariants.
+Every config is compared IN FULL: C5 (1e9 records) with its construction truth (itself pinned to the oracle at
+reduced size, tests/test_oracle.py); C2 (18.3 M, and its one-barrier-removed mutant), C3 (101.4 M) and C4 (412 M,
+with and without benign reporting) with the T-thread oracle (oracle_check_partitioned) run on the same bytes copied
+back from the device — every race record, witnesses included (byte equality of the sorted race arrays).  Plus
+whole-trace invariants.
 """
 import numpy as np
 import pytest
@@ -24,45 +24,36 @@ def S():
     return sesa
 
 
-def sampled_parity(S, dev_recs, n, host_recs, ws, ls, nsample=64, seed=0, benign=False):
+def full_parity(S, dev_recs, n, ws, ls, benign=False, lockstep_subset=False):
+    """The GPU race list of the whole trace against the T-thread oracle (oracle_check_partitioned, byte-identical
+    to the 1-thread grouped checker) on the SAME bytes, copied back from the device: every race, every witness."""
     t = S.Trace(ws, ls, 4, benign=benign)
     t.check(dev_recs, n)
     got = t.races()
     t.close()
-    assert len(host_recs) == n
-    rng = np.random.default_rng(seed)
-    gran = host_recs["addr"] // 4
-    # sample: locations the GPU reported + random accessed locations (all global in C3/C4)
-    pick = set((got["addr"][rng.choice(len(got), min(nsample, len(got)), replace=False)] // 4).tolist()) if len(got) else set()
-    pick |= set(gran[rng.integers(0, n, nsample)].tolist())
-    pick = np.array(sorted(pick), dtype=np.uint64)
-    sel = np.flatnonzero(np.isin(gran, pick))
-    exp = O.check(host_recs[sel], warp_size=ws, lockstep=ls, benign=benign)
-    exp["first"] = sel[exp["first"].astype(np.int64)]
-    exp["second"] = sel[exp["second"].astype(np.int64)]
-    got_s = got[np.isin(got["addr"] // 4, pick)]
-    assert got_s.tobytes() == exp.tobytes(), (len(got_s), len(exp))
-    return got, len(pick), len(sel)
+    host = dev_recs.cpu().numpy().view(G.REC_DTYPE)
+    assert len(host) == n
+    exp = O.check(host, warp_size=ws, lockstep=ls, benign=benign, method="partitioned")
+    assert len(got) == len(exp), (len(got), len(exp))
+    assert got.tobytes() == exp.tobytes()
+    return got, host
 
 
-def test_c3_full_size_sampled(S):
+def test_c3_full_size_parity(S):
     cfg = C.C3()
     dev, n = cfg.device()
-    host = cfg.host()
-    got, npick, nsel = sampled_parity(S, dev, n, host, 32, 0)
     assert n == 101447621
+    got, host = full_parity(S, dev, n, 32, 0)
     # invariants: atomics never race with each other -> every race is RW at a bin (a guard read vs an atomic)
     assert set(got["kind"].tolist()) <= {1}
-    bins_lo = cfg.cfg().bins_base
-    assert (got["addr"] >= bins_lo).all()
-    print(f"C3: {len(got)} races; {npick} sampled locations ({nsel} records) equal to the oracle")
+    assert (got["addr"] >= cfg.cfg().bins_base).all()
+    print(f"C3: {len(got)} races equal to the oracle's over all {n} records")
 
 
-def test_c4_full_size_sampled(S):
+def test_c4_full_size_parity(S):
     cfg = C.C4()
     dev, n = cfg.device()
-    host = cfg.host()
-    got, npick, nsel = sampled_parity(S, dev, n, host, 32, 1)
+    got, host = full_parity(S, dev, n, 32, 1)
     # invariants: all writes at one location carry the same value -> no WW; races only on dist[]
     assert set(got["kind"].tolist()) == {1}
     c = cfg.cfg()
@@ -74,21 +65,20 @@ def test_c4_full_size_sampled(S):
     t.close()
     key = lambda r: set(zip(r["addr"].tolist(), r["kind"].tolist()))  # noqa: E731
     assert key(got) <= key(nols)
-    print(f"C4: {len(got)} races ({len(nols)} without lockstep); {npick} sampled locations ({nsel} records) ok")
+    print(f"C4: {len(got)} races ({len(nols)} without lockstep) equal to the oracle's over all {n} records")
 
 
-def test_c4_full_size_benign(S):
+def test_c4_full_size_benign_parity(S):
     """Table IV reports the BFS kernel as "W/W (Benign)": with benign reporting the full-size C4 trace
     gets kind-3 records (at `changed` and at dist[] entries written by several frontier threads) and still no
-    kind-2 race; sampled locations equal the oracle's, witnesses included."""
+    kind-2 race; the whole list equals the oracle's, witnesses included."""
     cfg = C.C4()
     dev, n = cfg.device()
-    host = cfg.host()
-    got, npick, nsel = sampled_parity(S, dev, n, host, 32, 1, benign=True)
+    got, host = full_parity(S, dev, n, 32, 1, benign=True)
     kinds = set(got["kind"].tolist())
     assert kinds == {1, 3}
     assert int(cfg.cfg().changed_base) in set(got["addr"][got["kind"] == 3].tolist())
-    print(f"C4 benign: {(got['kind'] == 3).sum()} benign locations; {npick} sampled ({nsel} records) ok")
+    print(f"C4 benign: {(got['kind'] == 3).sum()} benign locations; full list equal to the oracle's")
 
 
 def test_c5_full_size_truth(S):
@@ -109,14 +99,11 @@ def test_c2_full_size_race_free_and_mutant(S):
         t.expand(d_fl, len(fl), out, n)
         nr = t.check(out, n)
         assert (nr > 0) == expect_races
-        if expect_races:  # parity for the mutant on the shared locations of two blocks (all their records)
-            host = O.expand(fl)
-            got = t.races()
+        host = O.expand(fl)  # the oracle's own expansion of the same descriptors
+        assert out.cpu().numpy().tobytes() == host.tobytes()  # the whole expansion, byte for byte
+        got = t.races()
+        exp = O.check(host, method="partitioned")  # the whole race list of the expanded trace
+        assert got.tobytes() == exp.tobytes()
+        if expect_races:
             assert set(got["space"].tolist()) == {0}  # only the shared tiles lose their barrier
-            blocks = (0, 63)
-            sel = np.flatnonzero((host["space"] == 0) & np.isin(host["block"], blocks))
-            exp = O.check(host[sel])
-            exp["first"] = sel[exp["first"].astype(np.int64)]
-            exp["second"] = sel[exp["second"].astype(np.int64)]
-            assert got[np.isin(got["block"], blocks)].tobytes() == exp.tobytes()
     t.close()

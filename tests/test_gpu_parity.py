@@ -177,11 +177,9 @@ def test_c2_full_expand_and_race_free(sesa):
     assert n == 18300928
     out = torch.empty(n * 32, dtype=torch.uint8, device="cuda")
     t.expand(d_fl, len(fl), out, n)
-    # sampled parity of the expansion at full size (oracle expands the same descriptors)
+    # the whole expansion at full size, byte for byte (the oracle expands the same descriptors)
     exp = O.expand(fl)
-    got = out.cpu().numpy().view(G.REC_DTYPE)
-    idx = np.random.default_rng(0).integers(0, n, 200000)
-    assert got[idx].tobytes() == exp[idx].tobytes()
+    assert out.cpu().numpy().tobytes() == exp.tobytes()
     assert t.check(out, n) == 0  # race-free by construction (double buffering, one barrier per k-tile)
 
 

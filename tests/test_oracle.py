@@ -493,3 +493,29 @@ def test_grouped_equals_brute_wide_accesses(G_):
             a = O.check(r, warp_size=ws, lockstep=ls, granularity=G_, method="grouped")
             b = O.check(r, warp_size=ws, lockstep=ls, granularity=G_, method="brute")
             assert a.tobytes() == b.tobytes()
+
+
+# ------------------------------------------------------------------------------------------------ T-thread mode
+@pytest.mark.parametrize("cfg", CONFIGS)
+def test_partitioned_equals_grouped(cfg):
+    """oracle_check_partitioned (SURVEY §8c.3 T-thread mode: locations split by hash) is byte-identical to the
+    1-thread grouped checker, for any thread count."""
+    for seed in range(12):
+        n = 200 + seed * 900
+        r = G.random_trace(n, 3000 + seed, threads=12 + 9 * seed, blocks=1 + seed % 5, words=8 + 40 * seed,
+                           sort=seed % 3 != 0)
+        a = O.check(r, warp_size=cfg["ws"], lockstep=cfg["ls"], granularity=cfg["G"], method="grouped")
+        b = O.check(r, warp_size=cfg["ws"], lockstep=cfg["ls"], granularity=cfg["G"], method="partitioned",
+                    threads=1 + seed % 6)
+        assert a.tobytes() == b.tobytes(), (cfg, seed)
+
+
+@pytest.mark.parametrize("benign", [False, True])
+def test_partitioned_hot_location_parallel_path(benign):
+    """A location with >= 2^20 entries takes the multi-threaded sort/count path of group_flags; same result."""
+    from sesagen import configs as C
+    r = C.rnd_host(1_200_000, 77, blocks=3, threads=256, intervals=2, words=3, shared_frac=0.0, sizes=(4,),
+                   values=40, unaligned=False)
+    a = O.check(r, warp_size=32, lockstep=1, benign=benign, method="grouped")
+    b = O.check(r, warp_size=32, lockstep=1, benign=benign, method="partitioned", threads=4)
+    assert len(a) > 0 and a.tobytes() == b.tobytes()
