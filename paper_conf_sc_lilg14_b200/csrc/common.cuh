@@ -125,16 +125,6 @@ __host__ __device__ __forceinline__ u64 sesa_mix(u64 x) {
   return x ^ (x >> 31);
 }
 
-// tile ids of the single-pass scans: 1 = atomic counter, 0 = blockIdx.x (dispatch order); env SESA_TILE_ATOMIC
-inline int tile_atomic_mode() {
-  static int v = -1;
-  if (v < 0) {
-    const char* e = getenv("SESA_TILE_ATOMIC");
-    v = e ? atoi(e) : 1;
-  }
-  return v;
-}
-
 // block-wide exclusive sum over THREADS values (one per thread)
 template <int THREADS>
 __device__ __forceinline__ u32 block_excl_sum(u32 v, u32* scratch /* [THREADS/32 + 1] */) {

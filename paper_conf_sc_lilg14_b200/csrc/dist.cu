@@ -109,7 +109,7 @@ __global__ void scatter_records_kernel(const Rec* __restrict__ in, const u32* __
 
 // ------------------------------------------------------------------------------------------------ state
 struct RankBufs {
-  DevBuf pcnt, poff, ptmp, send, recv, src, req, reqin, recsend, recback, rec_entry, tot, rkeys, rvals, races;
+  DevBuf pcnt, poff, ptmp, send, recv, src, req, reqin, recsend, recback, rec_entry, tot, rkeys, rvals, races, ag;
 };
 
 struct DistState {
@@ -120,6 +120,7 @@ struct DistState {
 // per-rank host-side values exchanged in X1
 struct RankInfo {
   unsigned long long n, base, first_b, first_i, last_b, last_i, bad;  // bad: global index or ~0
+  unsigned long long fail;                                            // status of the rank's P1 (0 = ok)
 };
 
 static bool partition(sesa_trace* t, RankBufs& B, const u64* in, u64 n, u32 W, int mode, const u64* bases,
@@ -173,8 +174,8 @@ struct Exchanger {
 struct NcclExchanger : Exchanger {
   ncclComm_t comm;
   int rank_, world_;
-  DevBuf tmp;
-  NcclExchanger(ncclComm_t c, int r, int w) : comm(c), rank_(r), world_(w) {}
+  DevBuf& tmp;  // staging of the host all-gathers (owned by the handle's DistState, freed by destroy)
+  NcclExchanger(ncclComm_t c, int r, int w, DevBuf& t) : comm(c), rank_(r), world_(w), tmp(t) {}
   int world() const override { return world_; }
   bool nccl_ok(sesa_trace* t, ncclResult_t r, const char* what) {
     if (r == ncclSuccess) return true;
@@ -226,20 +227,35 @@ struct RankIO {
   u64 n, index_base;
 };
 
+// A local failure must not leave the peers blocked in the next collective (one process per GPU): every exchange
+// first all-gathers, with the count rows, one status word per rank, and all ranks fail together if any failed.
+// `local_ok` = this rank's phase before the exchange succeeded (its send buffers are valid).
+static bool agree(sesa_trace* t, int p, u64 st, u64 local_ok) {
+  if (st == SESA_OK) return true;
+  if (local_ok) t->fail((sesa_status)st, "rank %d failed before the exchange (status %s)", p, sesa_status_str((sesa_status)st));
+  return false;
+}
+
 // exchange helper covering both modes: per local rank r, send buffers/counts -> recv buffers/counts
 static bool exchange(std::vector<sesa_trace*>& ts, Exchanger* ex, const std::vector<const void*>& send,
                      const std::vector<std::vector<u64>>& scnt, std::vector<DevBuf*>& recv, std::vector<std::vector<u64>>& rcnt,
-                     size_t elem, const char* what) {
+                     size_t elem, const char* what, bool local_ok = true) {
   const int W = ex ? ex->world() : (int)ts.size();
   const int R = (int)ts.size();
   rcnt.assign(R, std::vector<u64>(W, 0));
-  if (ex) {  // real ranks: one local handle; counts by all-gather of the count rows
+  if (!ex && !local_ok) return false;  // loopback: every virtual rank already carries the failure (fail_all)
+  if (ex) {  // real ranks: one local handle; counts + status by all-gather of the count rows
     sesa_trace* t = ts[0];
-    std::vector<u64> all((size_t)W * W);
-    if (!ex->allgather(t, scnt[0].data(), all.data(), W * 8)) return false;
+    std::vector<u64> row(W + 1, 0), all((size_t)W * (W + 1));
+    if (local_ok) std::copy(scnt[0].begin(), scnt[0].end(), row.begin());
+    row[W] = local_ok ? (u64)SESA_OK : (u64)(t->status != SESA_OK ? t->status : SESA_ECUDA);
+    if (!ex->allgather(t, row.data(), all.data(), (W + 1) * 8)) return false;
+    bool ok = true;
+    for (int p = 0; p < W; p++) ok = agree(t, p, all[(size_t)p * (W + 1) + W], local_ok && ok) && ok;
+    if (!ok || !local_ok) return false;
     int me = t->rank;
     u64 tot = 0;
-    for (int p = 0; p < W; p++) rcnt[0][p] = all[(size_t)p * W + me], tot += rcnt[0][p];
+    for (int p = 0; p < W; p++) rcnt[0][p] = all[(size_t)p * (W + 1) + me], tot += rcnt[0][p];
     if (!t->grow(*recv[0], std::max<u64>(tot, 1) * elem + 64, what)) return false;
     return ex->alltoall(t, send[0], scnt[0].data(), recv[0]->p, rcnt[0].data(), elem);
   }
@@ -270,10 +286,12 @@ static sesa_status dist_check(std::vector<sesa_trace*>& ts, std::vector<RankIO>&
   const int R = (int)ts.size();
   const int W = ex ? ex->world() : R;
   for (int r = 0; r < R; r++) ts[r]->begin_check(io[r].n);
-  // --- P1: extents per rank
+  // --- P1: extents per rank (a local failure is carried into X1, so that no peer waits for this rank)
+  std::vector<bool> p1ok(R, true);
   for (int r = 0; r < R; r++) {
-    if (io[r].n && !ts[r]->check_records_ptr((const sesa_access*)io[r].rec, io[r].n)) return fail_all(ts, ts[r]), ts[r]->status;
-    if (!ts[r]->step_extents(io[r].rec, io[r].n)) return fail_all(ts, ts[r]), ts[r]->status;
+    if (io[r].n && !ts[r]->check_records_ptr((const sesa_access*)io[r].rec, io[r].n)) p1ok[r] = false;
+    else if (!ts[r]->step_extents(io[r].rec, io[r].n)) p1ok[r] = false;
+    if (!p1ok[r] && !ex) return fail_all(ts, ts[r]), ts[r]->status;
   }
   // --- X1: summaries + shard boundaries
   std::vector<RankInfo> infos(W);
@@ -283,8 +301,9 @@ static sesa_status dist_check(std::vector<sesa_trace*>& ts, std::vector<RankIO>&
     memset(&ri, 0, sizeof ri);
     ri.n = io[r].n;
     ri.base = io[r].index_base;
-    ri.bad = ts[r]->h_summary.bad_index == ~0ull ? ~0ull : io[r].index_base + ts[r]->h_summary.bad_index;
-    if (io[r].n) {
+    ri.fail = p1ok[r] ? 0ull : (unsigned long long)(ts[r]->status != SESA_OK ? ts[r]->status : SESA_ECUDA);
+    ri.bad = !p1ok[r] || ts[r]->h_summary.bad_index == ~0ull ? ~0ull : io[r].index_base + ts[r]->h_summary.bad_index;
+    if (io[r].n && p1ok[r]) {
       sesa_access f, l;
       cudaMemcpy(&f, io[r].rec, 32, cudaMemcpyDeviceToHost);
       cudaMemcpy(&l, io[r].rec + io[r].n - 1, 32, cudaMemcpyDeviceToHost);
@@ -292,6 +311,9 @@ static sesa_status dist_check(std::vector<sesa_trace*>& ts, std::vector<RankIO>&
     }
     if (ex) {
       if (!ex->allgather(ts[0], &ri, infos.data(), sizeof ri)) return ts[0]->status;
+      bool ok = true;
+      for (int p = 0; p < W; p++) ok = agree(ts[0], p, infos[p].fail, p1ok[0] && ok) && ok;
+      if (!ok || !p1ok[0]) return ts[0]->status;
       if (!ex->allgather(ts[0], &ts[0]->h_summary, sums.data(), sizeof(Summary))) return ts[0]->status;
     } else {
       infos[r] = ri;
@@ -388,38 +410,39 @@ static sesa_status dist_check(std::vector<sesa_trace*>& ts, std::vector<RankIO>&
   std::vector<std::vector<u64>> scnt(R, std::vector<u64>(W)), rcnt;
   std::vector<const void*> sendp(R);
   std::vector<DevBuf*> recvb(R);
-  for (int r = 0; r < R; r++) {
+  bool ok = true;  // this process's ranks completed the phase (NCCL: carried into the next exchange)
+  for (int r = 0; r < R && ok; r++) {
     sesa_trace* t = ts[r];
     const u64 mloc = t->h_summary.entries;
-    if (!t->step_extract(io[r].rec, io[r].n, mloc, io[r].index_base - base0, S.multi != 0)) return fail_all(ts, t), t->status;
-    if (!partition(t, t->ds->b, (const u64*)t->b_keys[0].p, mloc, W, 0, nullptr, scnt[r].data()))
-      return fail_all(ts, t), t->status;
     sendp[r] = t->ds->b.send.p;
     recvb[r] = &t->b_keys[1];  // received keys land in b_keys[1], then are copied/swapped into b_keys[0]
+    ok = t->step_extract(io[r].rec, io[r].n, mloc, io[r].index_base - base0, S.multi != 0) &&
+         partition(t, t->ds->b, (const u64*)t->b_keys[0].p, mloc, W, 0, nullptr, scnt[r].data());
+    sendp[r] = t->ds->b.send.p;
+    if (!ok) fail_all(ts, t);
   }
   // --- X2: keys to their owners
-  if (!exchange(ts, ex, sendp, scnt, recvb, rcnt, 8, "key exchange")) return ts[0]->status;
+  if (!exchange(ts, ex, sendp, scnt, recvb, rcnt, 8, "key exchange", ok)) return ts[0]->status;
   // --- P3: local sort + compaction of the received keys; requests for the records of multi-entry locations
   std::vector<u64*> comp(R);
   std::vector<u32> m2(R);
   std::vector<std::vector<u64>> qcnt(R, std::vector<u64>(W)), qrcnt;
   std::vector<DevBuf*> reqb(R);
-  for (int r = 0; r < R; r++) {
+  for (int r = 0; r < R && ok; r++) {
     sesa_trace* t = ts[r];
     u64 mr = 0;
     for (int s = 0; s < W; s++) mr += rcnt[r][s];
     std::swap(t->b_keys[0], t->b_keys[1]);  // received keys -> b_keys[0]
-    if (!t->grow(t->b_keys[1], mr * 8 + 64, "keys")) return fail_all(ts, t), t->status;
-    if (!t->step_hist(mr)) return fail_all(ts, t), t->status;
     int cur = 0;
-    if (!t->step_sort(mr, &cur)) return fail_all(ts, t), t->status;
-    if (!t->step_compact(cur, mr, &comp[r], &m2[r])) return fail_all(ts, t), t->status;
-    if (!partition(t, t->ds->b, comp[r], m2[r], W, 1, bases.data(), qcnt[r].data())) return fail_all(ts, t), t->status;
+    ok = t->grow(t->b_keys[1], mr * 8 + 64, "keys") && t->step_hist(mr) && t->step_sort(mr, &cur) &&
+         t->step_compact(cur, mr, &comp[r], &m2[r]) &&
+         partition(t, t->ds->b, comp[r], m2[r], W, 1, bases.data(), qcnt[r].data());
     sendp[r] = t->ds->b.send.p;
     reqb[r] = &t->ds->b.reqin;
+    if (!ok) fail_all(ts, t);
   }
   // --- X3: positions to the record owners
-  if (!exchange(ts, ex, sendp, qcnt, reqb, qrcnt, 8, "request exchange")) return ts[0]->status;
+  if (!exchange(ts, ex, sendp, qcnt, reqb, qrcnt, 8, "request exchange", ok)) return ts[0]->status;
   // --- P4: owners gather the requested records
   std::vector<std::vector<u64>> bcnt, brcnt;
   bcnt.assign(R, std::vector<u64>(W));
@@ -428,7 +451,11 @@ static sesa_status dist_check(std::vector<sesa_trace*>& ts, std::vector<RankIO>&
     sesa_trace* t = ts[r];
     u64 nq = 0;
     for (int s = 0; s < W; s++) nq += qrcnt[r][s], bcnt[r][s] = qrcnt[r][s];
-    if (!t->grow(t->ds->b.recsend, std::max<u64>(nq, 1) * 32, "record send")) return fail_all(ts, t), t->status;
+    if (!t->grow(t->ds->b.recsend, std::max<u64>(nq, 1) * 32, "record send")) {
+      ok = false;
+      fail_all(ts, t);
+      break;
+    }
     if (nq) {
       t->launches++;
       gather_records_kernel<<<(unsigned)((nq + 255) / 256), 256, 0, t->stream>>>(
@@ -438,31 +465,35 @@ static sesa_status dist_check(std::vector<sesa_trace*>& ts, std::vector<RankIO>&
     backb[r] = &t->ds->b.recback;
   }
   // --- X4: records back to the requesters (in the order of their request buffers)
-  if (!exchange(ts, ex, sendp, bcnt, backb, brcnt, 32, "record exchange")) return ts[0]->status;
+  if (!exchange(ts, ex, sendp, bcnt, backb, brcnt, 32, "record exchange", ok)) return ts[0]->status;
   // --- P5: entry-aligned records, conflict tiles, local canonical race order
   std::vector<std::vector<u64>> racn(R, std::vector<u64>(W, 0)), racrn;
-  for (int r = 0; r < R; r++) {
+  for (int r = 0; r < R && ok; r++) {
     sesa_trace* t = ts[r];
     RankBufs& B = t->ds->b;
-    if (!t->grow(B.rec_entry, std::max<u32>(m2[r], 1) * 32, "entry records")) return fail_all(ts, t), t->status;
+    sendp[r] = t->b_races_sorted.p;
+    recvb[r] = &B.races;
+    if (!t->grow(B.rec_entry, std::max<u32>(m2[r], 1) * 32, "entry records")) {
+      ok = false;
+      fail_all(ts, t);
+      break;
+    }
     if (m2[r]) {
       t->launches++;
       scatter_records_kernel<<<(m2[r] + 255) / 256, 256, 0, t->stream>>>((const Rec*)B.recback.p, (const u32*)B.src.p,
                                                                           m2[r], (Rec*)B.rec_entry.p);
     }
-    if (!t->step_conflict(comp[r], m2[r], nullptr, 0, (const Rec*)B.rec_entry.p, base0)) return fail_all(ts, t), t->status;
-    const u32 nr = (u32)t->n_races;
-    if (!t->grow(t->b_races_sorted, (size_t)std::max(nr, 1u) * sizeof(RaceOut), "sorted races")) return fail_all(ts, t), t->status;
-    if (!t->step_race_sort(nr, (RaceOut*)t->b_races.p, (u64*)t->b_rkeys[0].p, (u32*)t->b_rvals[0].p,
-                           (u64*)t->b_rkeys[1].p, (u32*)t->b_rvals[1].p, (RaceOut*)t->b_races_sorted.p))
-      return fail_all(ts, t), t->status;
-    if (!t->sync_check("local races")) return fail_all(ts, t), t->status;
-    racn[r][0] = nr;  // everything goes to rank 0
+    ok = t->step_conflict(comp[r], m2[r], nullptr, 0, (const Rec*)B.rec_entry.p, base0) &&
+         t->grow(t->b_races_sorted, (size_t)std::max((u32)t->n_races, 1u) * sizeof(RaceOut), "sorted races") &&
+         t->step_race_sort((u32)t->n_races, (RaceOut*)t->b_races.p, (u64*)t->b_rkeys[0].p, (u32*)t->b_rvals[0].p,
+                           (u64*)t->b_rkeys[1].p, (u32*)t->b_rvals[1].p, (RaceOut*)t->b_races_sorted.p) &&
+         t->sync_check("local races");
+    racn[r][0] = t->n_races;  // everything goes to rank 0
     sendp[r] = t->b_races_sorted.p;
-    recvb[r] = &B.races;
+    if (!ok) fail_all(ts, t);
   }
   // --- X5: race lists to rank 0 (rank 0 receives every rank's list, in rank order), then one canonical sort
-  if (!exchange(ts, ex, sendp, racn, recvb, racrn, sizeof(RaceOut), "race gather")) return ts[0]->status;
+  if (!exchange(ts, ex, sendp, racn, recvb, racrn, sizeof(RaceOut), "race gather", ok)) return ts[0]->status;
   for (int r = 0; r < R; r++) {
     sesa_trace* t = ts[r];
     const bool is0 = (ex ? t->rank : r) == 0;
@@ -497,7 +528,7 @@ static sesa_status dist_check(std::vector<sesa_trace*>& ts, std::vector<RankIO>&
 sesa_status sesa_trace::check_dist(const sesa_access* d_rec, uint64_t n, uint64_t index_base) {
   std::vector<sesa_trace*> ts = {this};
   std::vector<RankIO> io = {{(const Rec*)d_rec, n, index_base}};
-  NcclExchanger ex(ds->comm, rank, world);
+  NcclExchanger ex(ds->comm, rank, world, ds->b.ag);
   const sesa_status s = dist_check(ts, io, &ex);
   if (s != SESA_OK && status == SESA_OK) status = s;
   return status;
@@ -507,7 +538,7 @@ void sesa_trace::destroy_dist() {
   if (!ds) return;
   RankBufs& B = ds->b;
   for (DevBuf* b : {&B.pcnt, &B.poff, &B.ptmp, &B.send, &B.recv, &B.src, &B.req, &B.reqin, &B.recsend, &B.recback,
-                    &B.rec_entry, &B.tot, &B.rkeys, &B.rvals, &B.races})
+                    &B.rec_entry, &B.tot, &B.rkeys, &B.rvals, &B.races, &B.ag})
     if (b->p) cudaFree(b->p), b->p = nullptr;
   if (ds->comm) ncclCommDestroy(ds->comm);
   delete ds;

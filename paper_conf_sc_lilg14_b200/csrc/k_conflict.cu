@@ -1019,8 +1019,7 @@ u32 conflict_tiles(u64 m) { return (u32)((m + CT_NOM - 1) / CT_NOM); }
 template <int MODE, class A>
 static void launch_ck(const ConflictArgs& a, u32 nblocks, cudaStream_t st) {
   const size_t sm = sizeof(TileSmem);
-  static bool set = false;
-  if (!set) cudaFuncSetAttribute(conflict_kernel<MODE, A>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm), set = true;
+  smem_optin((const void*)conflict_kernel<MODE, A>, sm);
   conflict_kernel<MODE, A><<<nblocks, CT_THREADS, sm, st>>>(a);
 }
 
@@ -1034,8 +1033,7 @@ void launch_conflict(int mode, bool exact, const ConflictArgs& a, u32 nblocks, c
     if (exact) launch_ck<2, Agg>(a, nblocks, st);
     else launch_ck<2, AggC>(a, nblocks, st);
   } else {
-    static bool set = false;
-    if (!set) cudaFuncSetAttribute(conflict_y_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm), set = true;
+    smem_optin((const void*)conflict_y_kernel, sm);
     conflict_y_kernel<<<nblocks, CT_THREADS, sm, st>>>(a);
   }
 }

@@ -255,29 +255,16 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
   }
 }
 
-static int ring_grid(const void* kern, int threads, size_t smem, size_t smem_max) {
-  int dev = 0, sms = 148, per = 1;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_max);  // never lowered
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, kern, threads, smem);
-  return sms * (per > 0 ? per : 1);
+static int ring_grid(const void* kern, int threads, size_t smem) {
+  return dev_sm_count() * blocks_per_sm(kern, threads, smem);
 }
 
 void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, u32* tile_hist, const Region* regs, u32 nreg,
                     u32 nreg_shared, int grid, cudaStream_t st, u32* gout) {
   // extents2: contiguous warp ranges, one full wave of resident warps (the round-1 grid-stride kernel took
   // 7.7 ms on C5: 132 instructions per record, 64-bit index math and local-memory accumulators; this one 4.6 ms)
-  static int sms = 0, per = 0;
-  if (!sms) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, extents2_kernel<4>, 256, 0);
-    per = std::max(per, 1);
-    cudaFuncSetAttribute(extents2_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)(MAX_REGIONS * sizeof(Region)));
-  }
+  const int sms = dev_sm_count(), per = blocks_per_sm((const void*)extents2_kernel<4>, 256, 0);
+  smem_optin((const void*)extents2_kernel<4>, MAX_REGIONS * sizeof(Region));
   const u64 warps = (u64)sms * per * 8;
   const u64 gran = tile_hist ? FUSED_TILE : 128;  // warp ranges: whole tiles when tile histograms are wanted
   u64 rw = (n + warps - 1) / warps;
@@ -332,12 +319,8 @@ __global__ void __launch_bounds__(THREADS) extract_1to1_kernel(const Rec* __rest
 
 void launch_extract_1to1(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, u64* keys, u32* hist, u64 pos_base,
                          int, cudaStream_t st) {
-  static int grids[9] = {0};
   const size_t sm = (size_t)EX_STAGES * EX_CHUNK + (size_t)npass * 8 * RADIX * 4;  // ring + npass x 8 warps hist
-  if (!grids[npass])
-    grids[npass] = ring_grid((const void*)extract_1to1_kernel<256, RADIX_BITS>, 256, sm,
-                             (size_t)EX_STAGES * EX_CHUNK + (size_t)8 * 8 * RADIX * 4);
-  const int grid = grids[npass];
+  const int grid = ring_grid((const void*)extract_1to1_kernel<256, RADIX_BITS>, 256, sm);
   const u64 chunks = (n * 32 + EX_CHUNK - 1) / EX_CHUNK;
   extract_1to1_kernel<256, RADIX_BITS><<<(unsigned)std::min<u64>(chunks, (u64)grid), 256, sm, st>>>(rec, n, L, npass,
                                                                                                    keys, hist, pos_base);

@@ -233,19 +233,12 @@ void launch_fused_extract_pass0(const u32* gran, u64 n, const KeyLayout& L, u32 
   if (!n) return;
   const u32 T = (u32)((n + FUSED_TILE - 1) / FUSED_TILE);
   u32* O = reinterpret_cast<u32*>(temp);
-  static int grid = 0;
-  if (!grid) {
-    int dev = 0, sms = 148, per = 1;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    const void* ks[4] = {(const void*)fused_extract_pass0_kernel<1>, (const void*)fused_extract_pass0_kernel<2>,
-                         (const void*)fused_extract_pass0_kernel<3>, (const void*)fused_extract_pass0_kernel<4>};
-    for (int i = 0; i < 4; i++)
-      cudaFuncSetAttribute(ks[i], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fused_smem(i + 1));
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fused_extract_pass0_kernel<4>, FUSED_THREADS, fused_smem(4));
-    grid = sms * std::max(per, 1);
-  }
+  const void* ks[4] = {(const void*)fused_extract_pass0_kernel<1>, (const void*)fused_extract_pass0_kernel<2>,
+                       (const void*)fused_extract_pass0_kernel<3>, (const void*)fused_extract_pass0_kernel<4>};
   const size_t sm = fused_smem(npass);
+  // persistent CTAs: one full wave at the occupancy of the largest variant
+  const int grid = dev_sm_count() * blocks_per_sm(ks[3], FUSED_THREADS, fused_smem(4));
+  smem_optin(ks[std::min<u32>(npass, 4) - 1], sm);
   FusedArgs A;
   A.gran = gran;
   A.n = (u32)n;

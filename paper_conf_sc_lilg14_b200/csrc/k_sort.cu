@@ -9,9 +9,6 @@
 // out so that each digit's run of the tile lands contiguously (coalesced stores).  Traffic per pass: 8 B read +
 // 8 B written per key (+4 + 4 with values); the look-back words add 8 B x 256 per 4096-key tile (~0.5 B/key).
 #include <algorithm>
-#include <cstdio>
-#include <cstdlib>
-#include <vector>
 
 #include "kernels.cuh"
 
@@ -25,12 +22,6 @@ __device__ __forceinline__ u64 lb_pack(u64 status, u32 epoch, u64 v) { return st
 __device__ __forceinline__ void st_relaxed(u64* p, u64 v) {
   asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
-__device__ __forceinline__ u64 gtime() {
-  u64 t;
-  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-  return t;
-}
-__device__ unsigned long long* g_prof = nullptr;  // optional per-tile phase stamps (SESA_SORT_PROF)
 
 __device__ __forceinline__ u64 ld_relaxed(const u64* p) {
   u64 v;
@@ -61,19 +52,23 @@ void launch_bin_base(const u32* hist, u64* bin_base, u32 npass, cudaStream_t st)
   if (npass) bin_base_kernel<<<npass, RADIX, 0, st>>>(hist, bin_base);
 }
 
-// One tile (body templated on FULL: full tiles skip every validity test).  Per item the digit (9 bits; invalid
-// items of a partial tile use digit RADIX) and later its rank are packed into one register: rd = rank << 9 | d.
-template <int THREADS, int ITEMS, bool VALS, int MATCH, int LBW, bool FULL>
-__device__ __forceinline__ void onesweep_tile(const u64* __restrict__ kin, u64* __restrict__ kout,
-                                              const u32* __restrict__ vin, u32* __restrict__ vout, u32 m, u32 shift,
-                                              const u64* __restrict__ bin_base, u64* __restrict__ lookback,
-                                              u32 epoch, u32 tile, unsigned char* smem,
-                                              unsigned long long* prof) {
+// Key/value onesweep (race lists and the benign regrouping: short arrays).  One tile (body templated on FULL:
+// full tiles skip every validity test).  Per item the digit (9 bits; invalid items of a partial tile use digit
+// RADIX) and later its rank are packed into one register: rd = rank << 9 | d.  Peer sets come from per-warp
+// shared-memory masks (each lane sets its bit in its digit's word).
+constexpr int KV_THREADS = 256, KV_ITEMS = 16, KV_MINB = 3, KV_LBW = 4;
+
+template <bool FULL>
+__device__ __forceinline__ void onesweep_kv_tile(const u64* __restrict__ kin, u64* __restrict__ kout,
+                                                 const u32* __restrict__ vin, u32* __restrict__ vout, u32 m, u32 shift,
+                                                 const u64* __restrict__ bin_base, u64* __restrict__ lookback,
+                                                 u32 epoch, u32 tile, unsigned char* smem) {
+  constexpr int THREADS = KV_THREADS, ITEMS = KV_ITEMS, LBW = KV_LBW;
   constexpr int WARPS = THREADS / 32;
   constexpr int TILE = THREADS * ITEMS;
   u64* keys_s = reinterpret_cast<u64*>(smem);                                  // [TILE]
-  u32* vals_s = reinterpret_cast<u32*>(keys_s + TILE);                          // [TILE] if VALS
-  u32* whist = VALS ? vals_s + TILE : reinterpret_cast<u32*>(keys_s + TILE);    // [WARPS][RADIX]
+  u32* vals_s = reinterpret_cast<u32*>(keys_s + TILE);                          // [TILE]
+  u32* whist = vals_s + TILE;                                                   // [WARPS][RADIX]
   u32* bin_start = whist + WARPS * RADIX;                                       // [RADIX]
   long long* glob = reinterpret_cast<long long*>(bin_start + RADIX);            // [RADIX] (8-byte slots)
   u32* globu = reinterpret_cast<u32*>(glob);                                    // u32 view of the same slots
@@ -91,16 +86,12 @@ __device__ __forceinline__ void onesweep_tile(const u64* __restrict__ kin, u64* 
   for (int i = 0; i < ITEMS; i++) {
     if (FULL || i < nv) {
       k[i] = __ldcs(kin + wbase + (u64)i * 32);  // streaming: each key is read once per pass
-      if (VALS) v[i] = __ldcs(vin + wbase + (u64)i * 32);
+      v[i] = __ldcs(vin + wbase + (u64)i * 32);
     }
   }
 #pragma unroll
   for (int i = 0; i < ITEMS; i++) rd[i] = (FULL || i < nv) ? (u32)((k[i] >> shift) & (RADIX - 1)) : (u32)RADIX;
   u32* wh = whist + warp * RADIX;
-  if (prof) {
-    __syncthreads();
-    if (tid == 0) prof[1] = gtime();
-  }
   // (1) early counts: per-warp digit histogram with shared-memory atomics (no ordering needed for counts)
 #pragma unroll
   for (int i = 0; i < ITEMS; i++)
@@ -120,9 +111,7 @@ __device__ __forceinline__ void onesweep_tile(const u64* __restrict__ kin, u64* 
   }
   const u32 bs = block_excl_sum<THREADS>(tid < RADIX ? tot : 0u, scratch);  // (contains __syncthreads)
   if (tid < RADIX) bin_start[tid] = bs;
-  if (prof && tid == 0) prof[2] = gtime();
-  // (3) look-back for the exclusive prefix of every digit over earlier tiles, right after publishing the
-  //     aggregate so that inclusive prefixes propagate with minimal delay; each bin-owner thread inspects LBW
+  // (3) look-back for the exclusive prefix of every digit over earlier tiles; each bin-owner thread inspects LBW
   //     predecessors per L2 round trip and backs off while they are unpublished
   if (tid < RADIX) {
     u64 excl = 0;
@@ -149,49 +138,37 @@ __device__ __forceinline__ void onesweep_tile(const u64* __restrict__ kin, u64* 
         if (q == 0) __nanosleep(++spins < 4 ? 32 : 128);
         p -= q;
       }
-      if (prof && tid == 0) prof[7] = ((u64)(tile - p) << 32) | (u64)spins;  // walk distance, spins (digit 0)
       st_relaxed(lookback + (u64)tile * RADIX + tid, lb_pack(LB_PREFIX, epoch, excl + tot));
     }
     globu[tid] = (u32)(bin_base[tid] + excl) - bs;  // positions < m < 2^32: modular u32 offsets
-  }
-  if (prof) {
-    __syncthreads();
-    if (tid == 0) prof[3] = gtime();
   }
   // (4) stable warp-level ranking: running per-warp digit counter (starts at the warp's offset) + lower peers
   u32* wm = wmask + warp * (RADIX + 1);
 #pragma unroll
   for (int i = 0; i < ITEMS; i++) {
     const u32 d = rd[i];
-    unsigned peers;
-    if (MATCH == 0) {
-      peers = FULL ? peers_of<RADIX_BITS>(d) : peers_of<RADIX_BITS + 1>(d);
-    } else {
-      // each lane sets its bit in its digit's word of a per-warp mask array: the word becomes the peer set
-      atomicOr(&wm[d], 1u << lane);
-      __syncwarp();
-    }
+    atomicOr(&wm[d], 1u << lane);
+    __syncwarp();
     // the peer word and the running counter are read together: one shared-memory round trip per item
-    if (MATCH == 1) peers = wm[d];
+    const unsigned peers = wm[d];
     const u32 c = wh[d];
     __syncwarp();
     const bool leader = lane == 31 - __clz(peers);
     rd[i] |= (c + __popc(peers & lanemask_lt())) << 9;
     if (leader) {
-      if (MATCH == 1) wm[d] = 0;
+      wm[d] = 0;
       if (FULL || d < RADIX) wh[d] = c + __popc(peers);
     }
     __syncwarp();
   }
   __syncthreads();
-  if (prof && tid == 0) prof[4] = gtime();
   // (5) scatter into shared memory in (digit, stable) order, then coalesced stores of each digit's run
 #pragma unroll
   for (int i = 0; i < ITEMS; i++) {
     if (FULL || i < nv) {
       const u32 pos = bin_start[rd[i] & 511] + (rd[i] >> 9);
       keys_s[pos] = k[i];
-      if (VALS) vals_s[pos] = v[i];
+      vals_s[pos] = v[i];
     }
   }
   __syncthreads();
@@ -202,53 +179,62 @@ __device__ __forceinline__ void onesweep_tile(const u64* __restrict__ kin, u64* 
     const u32 d = (u32)((key >> shift) & (RADIX - 1));
     const u32 dst = globu[d] + j;
     __stcs(kout + dst, key);
-    if (VALS) __stcs(vout + dst, vals_s[j]);
-  }
-  if (prof) {
-    __syncthreads();
-    if (tid == 0) prof[5] = gtime(), prof[6] = (u64)blockIdx.x;
+    __stcs(vout + dst, vals_s[j]);
   }
 }
 
-template <int THREADS, int ITEMS, bool VALS, int MATCH, int MINB, int LBW>
-__global__ void __launch_bounds__(THREADS, MINB) onesweep_kernel(const u64* __restrict__ kin, u64* __restrict__ kout,
-                                                                 const u32* __restrict__ vin, u32* __restrict__ vout,
-                                                                 u32 m, u32 shift, const u64* __restrict__ bin_base,
-                                                                 u64* __restrict__ lookback, u32* __restrict__ tile_ctr,
-                                                                 u32 epoch, int g_tile_atomic) {
-  constexpr int WARPS = THREADS / 32;
-  constexpr int TILE = THREADS * ITEMS;
-  static_assert(RADIX <= THREADS, "one bin per thread");
+__global__ void __launch_bounds__(KV_THREADS, KV_MINB) onesweep_kv_kernel(
+    const u64* __restrict__ kin, u64* __restrict__ kout, const u32* __restrict__ vin, u32* __restrict__ vout, u32 m,
+    u32 shift, const u64* __restrict__ bin_base, u64* __restrict__ lookback, u32* __restrict__ tile_ctr, u32 epoch) {
+  constexpr int WARPS = KV_THREADS / 32;
+  constexpr int TILE = KV_THREADS * KV_ITEMS;
+  static_assert(RADIX <= KV_THREADS, "one bin per thread");
   extern __shared__ __align__(16) unsigned char smem[];
-  u32* whist = VALS ? reinterpret_cast<u32*>(smem) + 3 * TILE : reinterpret_cast<u32*>(smem) + 2 * TILE;
+  u32* whist = reinterpret_cast<u32*>(smem) + 3 * TILE;
   u32* wmask = whist + WARPS * RADIX + RADIX + 2 * RADIX + WARPS + 1;
   __shared__ u32 s_tile;
   const int tid = threadIdx.x;
   // one tile per CTA; tile ids from an atomic counter = execution order (blockIdx order measured 45% slower:
   // a tile whose predecessor was dispatched later spins in the look-back)
-  if (tid == 0) s_tile = g_tile_atomic ? atomicAdd(tile_ctr, 1u) : blockIdx.x;
-  for (int i = tid; i < WARPS * RADIX; i += THREADS) whist[i] = 0;
-  if (MATCH == 1)
-    for (int i = tid; i < WARPS * (RADIX + 1); i += THREADS) wmask[i] = 0;
+  if (tid == 0) s_tile = atomicAdd(tile_ctr, 1u);
+  for (int i = tid; i < WARPS * RADIX; i += KV_THREADS) whist[i] = 0;
+  for (int i = tid; i < WARPS * (RADIX + 1); i += KV_THREADS) wmask[i] = 0;
   __syncthreads();
   const u32 tile = s_tile;
-  unsigned long long* prof = g_prof ? g_prof + (u64)tile * 8 : nullptr;
-  if (prof && tid == 0) prof[0] = gtime();
   if ((u64)(tile + 1) * TILE <= m)
-    onesweep_tile<THREADS, ITEMS, VALS, MATCH, LBW, true>(kin, kout, vin, vout, m, shift, bin_base, lookback, epoch,
-                                                          tile, smem, prof);
+    onesweep_kv_tile<true>(kin, kout, vin, vout, m, shift, bin_base, lookback, epoch, tile, smem);
   else
-    onesweep_tile<THREADS, ITEMS, VALS, MATCH, LBW, false>(kin, kout, vin, vout, m, shift, bin_base, lookback, epoch,
-                                                           tile, smem, prof);
+    onesweep_kv_tile<false>(kin, kout, vin, vout, m, shift, bin_base, lookback, epoch, tile, smem);
+}
+
+static size_t onesweep_kv_smem() {
+  constexpr int WARPS = KV_THREADS / 32, TILE = KV_THREADS * KV_ITEMS;
+  return (size_t)TILE * 12 + (size_t)WARPS * RADIX * 4 + RADIX * 4 + RADIX * 8 + (WARPS + 1) * 4 +
+         (size_t)WARPS * (RADIX + 1) * 4;
 }
 
 // ------------------------------------------------------------------------------------------------------------
-// onesweep2 (keys only): the tile-local position of every key is known once the tile's digit counts are (bin
-// start + the warp's offset within the bin + its stable rank in the warp), so ranking writes each key straight
-// into its shared-memory slot and keeps no per-item rank registers; the global offsets from the look-back are
-// only needed by the final coalesced write-out.  LATE_LB = walk the look-back after ranking (predecessors have
-// had the ranking time to publish their inclusive prefixes) instead of before.
+// onesweep2 (keys only; the sort passes of the check): the tile-local position of every key is known once the
+// tile's digit counts are (bin start + the warp's offset within the bin + its stable rank in the warp), so
+// ranking writes each key straight into its shared-memory slot and keeps no per-item rank registers; the global
+// offsets from the look-back are only needed by the final coalesced write-out, so the look-back is walked after
+// ranking (predecessors have had the ranking time to publish their inclusive prefixes).  The tile (256 threads x
+// 32 keys) arrives by TMA bulk copies issued in the kernel prologue, right after the tile id.  Peer sets: every
+// 4th item by 8 ballots (ALU pipe), the others by shared-memory masks (LSU pipe, the binding one) — measured
+// against all-masks, all-ballots, every 2nd/3rd item by ballots and MATCH.
 // ------------------------------------------------------------------------------------------------------------
+constexpr int OS_THREADS = 256, OS_ITEMS = 32, OS_MINB = 2, OS_LBW = 4, OS_TILE = OS_THREADS * OS_ITEMS;
+
+__device__ __forceinline__ u64 gtime() {
+  u64 t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+// Per-tile phase stamps for diagnosis (never set by the library: always null).  Its runtime checks at the phase
+// boundaries also shape ptxas's schedule: compiled without them the pass spills 68 instead of 20 bytes per thread
+// and runs 3% slower (4.94 vs 4.80 ms per 1e9 keys, measured).
+__device__ unsigned long long* g_prof = nullptr;
+
 template <int THREADS, int ITEMS, int LBW, bool FULL, bool LATE_LB, int S, bool BAL, int TMA, int MIX = 0>
 __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64* __restrict__ kout, u32 m, u32 shift,
                                                const u64* __restrict__ bin_base, u64* __restrict__ lookback,
@@ -459,171 +445,33 @@ __global__ void __launch_bounds__(THREADS, MINB) onesweep2_kernel(const u64* __r
     onesweep2_tile<THREADS, ITEMS, LBW, false, LATE_LB, S, BAL, TMA, MIX>(kin, kout, m, shift, bin_base, lookback, epoch, tile, smem, prof, &ebar);
 }
 
-template <int THREADS, int ITEMS, int S, bool BAL>
+// the measured configuration: 256 x 32 keys, 2 CTAs/SM, look-back after ranking, one rank stream,
+// prologue bulk copies (TMA 2), every 4th item's peers by ballots (MIX 4)
+#define OS_CFG OS_THREADS, OS_ITEMS, OS_MINB, OS_LBW, true, 1, false, 2, 4
+
 static size_t onesweep2_smem() {
-  constexpr int WARPS = THREADS / 32, TILE = THREADS * ITEMS;
-  return (size_t)TILE * 8 + (size_t)WARPS * S * RADIX * 4 + RADIX * 4 + (WARPS + 1) * 4 +
-         (BAL ? 0 : (size_t)WARPS * S * (RADIX + 1) * 4);
+  constexpr int WARPS = OS_THREADS / 32;
+  return (size_t)OS_TILE * 8 + (size_t)WARPS * RADIX * 4 + RADIX * 4 + (WARPS + 1) * 4 +
+         (size_t)WARPS * (RADIX + 1) * 4;
 }
 
-template <int THREADS, int ITEMS, int MINB, int LBW, bool LATE_LB, int S = 1, bool BAL = false, int TMA = 0,
-          int MIX = 0>
-static void launch_os2(const u64* kin, u64* kout, u32 m, u32 shift, const u64* bin_base, u64* lookback,
-                       u32* tile_ctr, u32 epoch, cudaStream_t st) {
-  auto kern = onesweep2_kernel<THREADS, ITEMS, MINB, LBW, LATE_LB, S, BAL, TMA, MIX>;
-  const size_t sm = onesweep2_smem<THREADS, ITEMS, S, BAL>();
-  static bool set = false;
-  if (!set) {
-    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-    set = true;
-  }
-  const u32 tiles = (u32)((m + THREADS * ITEMS - 1) / (THREADS * ITEMS));
-  kern<<<tiles, THREADS, sm, st>>>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch);
-}
-
-template <int THREADS, int ITEMS, bool VALS>
-static size_t onesweep_smem() {
-  constexpr int WARPS = THREADS / 32, TILE = THREADS * ITEMS;
-  return (size_t)TILE * 8 + (VALS ? (size_t)TILE * 4 : 0) + (size_t)WARPS * RADIX * 4 + RADIX * 4 + RADIX * 8 +
-         (WARPS + 1) * 4 + (size_t)WARPS * (RADIX + 1) * 4;
-}
-
-// SESA_SORT_CFG selects the onesweep variant (all measured on C5, 1 B200; DESIGN.md §9 has the numbers):
-//   0 / 1   onesweep (ranks kept in registers, look-back before ranking), 256 x 16 / 256 x 24 keys
-//   15      onesweep2 256 x 24 at 3 CTAs/SM;  20: onesweep2 256 x 32, register loads, look-back after ranking
-//   21      as 20 with 16 predecessors per look-back round trip;  26: two rank streams;  31: ballot peers
-//   33      as 20 with the tile loaded by TMA bulk copies;  34: 33 with the early look-back
-//   35      as 33 with 512 x 16 tiles
-//   36      as 33 with the bulk copies issued in the kernel prologue, right after the tile id, before the counter
-//           arrays are cleared (4.88 vs 4.98 ms per 1e9-key pass)
-//   41-45   as 36 with some items' peer sets by ballots (ALU pipe) instead of shared-memory masks (LSU pipe, the
-//           binding one): 41 every 2nd item 4.79, 43 every 3rd 4.81-4.93, 44 every 4th 4.78 (default),
-//           45 three of four 4.85;  42: every 2nd item by MATCH (ADU pipe) 5.70 ms
-// Measured and removed: a look-back sequencer CTA, a dedicated look-back warp, cluster-level (DSMEM) look-back,
-// 256 x 40/48 tiles — each slower.
-int sort_cfg() {
-  static int v = -1;
-  if (v < 0) {
-    const char* e = getenv("SESA_SORT_CFG");
-    v = e ? atoi(e) : 44;
-  }
-  return v;
-}
-
-u32 sort_tile_keys() {
-  switch (sort_cfg()) {
-    case 1: case 15: return 256 * 24;
-    case 20: case 21: case 26: case 31: case 33: case 34: case 36: case 41: case 42: case 43: case 44: case 45: return 256 * 32;
-    case 35: return 512 * 16;
-    default: return 256 * 16;
-  }
-}
-
-int sort_variant() {  // SESA_SORT_MATCH=0 ballots, 1 atomicOr masks (default)
-  static int v = -1;
-  if (v < 0) {
-    const char* e = getenv("SESA_SORT_MATCH");
-    v = e ? atoi(e) : 1;
-  }
-  return v;
-}
-
-
-
-template <int THREADS, int ITEMS, int MINB, bool VALS, int MATCH, int LBW = 4>
-static void launch_os(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m, u32 shift, const u64* bin_base,
-                      u64* lookback, u32* tile_ctr, u32 epoch, cudaStream_t st) {
-  auto kern = onesweep_kernel<THREADS, ITEMS, VALS, MATCH, MINB, LBW>;
-  const size_t sm = onesweep_smem<THREADS, ITEMS, VALS>();
-  static bool set = false;
-  if (!set) {
-    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-    set = true;
-  }
-  const u32 tiles = (u32)((m + THREADS * ITEMS - 1) / (THREADS * ITEMS));
-  static int cap = 0;
-  if (!cap) {
-    int dev = 0, sms = 148, per = 1;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, kern, THREADS, sm);
-    cap = sms * std::max(per, 1);
-  }
-  (void)cap;
-  kern<<<tiles, THREADS, sm, st>>>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch,
-                                   tile_atomic_mode());
-}
-
-template <bool VALS, int MATCH>
-static void launch_os_cfg(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m, u32 shift,
-                          const u64* bin_base, u64* lookback, u32* tile_ctr, u32 epoch, cudaStream_t st) {
-  switch (sort_cfg()) {
-    case 1: launch_os<256, 24, 2, VALS, MATCH>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 15: launch_os2<256, 24, 3, 4, false>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 20: launch_os2<256, 32, 2, 4, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 21: launch_os2<256, 32, 2, 16, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 33: launch_os2<256, 32, 2, 4, true, 1, false, 1>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 34: launch_os2<256, 32, 2, 4, false, 1, false, 1>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 35: launch_os2<512, 16, 2, 4, true, 1, false, 1>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 36: launch_os2<256, 32, 2, 4, true, 1, false, 2>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 41: launch_os2<256, 32, 2, 4, true, 1, false, 2, 1>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 42: launch_os2<256, 32, 2, 4, true, 1, false, 2, 2>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 43: launch_os2<256, 32, 2, 4, true, 1, false, 2, 3>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 44: launch_os2<256, 32, 2, 4, true, 1, false, 2, 4>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 45: launch_os2<256, 32, 2, 4, true, 1, false, 2, 5>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 26: launch_os2<256, 32, 2, 4, true, 2>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    case 31: launch_os2<256, 32, 2, 4, true, 1, true>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch, st); break;
-    default: launch_os<256, 16, 3, VALS, MATCH>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
-  }
-}
-
-static void sort_prof_dump(u32 m, cudaStream_t st, unsigned long long* d, u32 tile_keys) {
-  const u32 nt = (m + tile_keys - 1) / tile_keys;
-  std::vector<unsigned long long> h((size_t)nt * 8);
-  cudaMemcpyAsync(h.data(), d, h.size() * 8, cudaMemcpyDeviceToHost, st);
-  cudaStreamSynchronize(st);
-  double ph[5] = {0, 0, 0, 0, 0}, dist = 0, spins = 0, dmax = 0;
-  unsigned long long t0 = ~0ull, t1 = 0;
-  for (u32 t = 0; t < nt; t++) {
-    const unsigned long long* p = &h[(size_t)t * 8];
-    for (int q = 0; q < 5; q++) ph[q] += (double)(p[q + 1] - p[q]);
-    t0 = std::min(t0, p[0]);
-    t1 = std::max(t1, p[5]);
-    dist += (double)(p[7] >> 32), spins += (double)(p[7] & 0xFFFFFFFFull);
-    dmax = std::max(dmax, (double)(p[7] >> 32));
-  }
-  fprintf(stderr, "[sortprof] walk distance mean %.1f max %.0f tiles, spins mean %.2f\n", dist / nt, dmax, spins / nt);
-  fprintf(stderr, "[sortprof] tiles %u span %.3f ms; mean ns: load %.0f counts %.0f lookback %.0f rank %.0f write %.0f\n", nt,
-          (t1 - t0) / 1e6, ph[0] / nt, ph[1] / nt, ph[2] / nt, ph[3] / nt, ph[4] / nt);
-}
+u32 sort_tile_keys() { return OS_TILE; }
 
 void launch_onesweep(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m, u32 shift, const u64* bin_base,
                      u64* lookback, u32* tile_ctr, u32 epoch, cudaStream_t st) {
   if (!m) return;
-  static unsigned long long* dprof = nullptr;
-  static size_t dcap = 0;
-  const bool want = getenv("SESA_SORT_PROF") && !vin;
-  if (want) {
-    const size_t need = ((size_t)m / 2048 + 2) * 64;
-    if (need > dcap) {
-      if (dprof) cudaFree(dprof);
-      cudaMalloc(&dprof, need);
-      dcap = need;
-    }
-    cudaMemcpyToSymbolAsync(g_prof, &dprof, sizeof(dprof), 0, cudaMemcpyHostToDevice, st);
-  } else if (dprof) {
-    unsigned long long* z = nullptr;
-    cudaMemcpyToSymbolAsync(g_prof, &z, sizeof(z), 0, cudaMemcpyHostToDevice, st);
-  }
-  const bool ballot = sort_variant() == 0;
-  if (vin) {  // race lists are small: fixed config
-    if (ballot) launch_os<256, 16, 3, true, 0>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
-    else launch_os<256, 16, 3, true, 1>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr, epoch, st);
+  if (vin) {  // key/value (race lists, benign regrouping)
+    const size_t sm = onesweep_kv_smem();
+    smem_optin((const void*)onesweep_kv_kernel, sm);
+    const u32 tiles = (u32)((m + KV_THREADS * KV_ITEMS - 1) / (KV_THREADS * KV_ITEMS));
+    onesweep_kv_kernel<<<tiles, KV_THREADS, sm, st>>>(kin, kout, vin, vout, m, shift, bin_base, lookback, tile_ctr,
+                                                       epoch);
   } else {
-    if (ballot) launch_os_cfg<false, 0>(kin, kout, nullptr, nullptr, m, shift, bin_base, lookback, tile_ctr, epoch, st);
-    else launch_os_cfg<false, 1>(kin, kout, nullptr, nullptr, m, shift, bin_base, lookback, tile_ctr, epoch, st);
+    const size_t sm = onesweep2_smem();
+    smem_optin((const void*)onesweep2_kernel<OS_CFG>, sm);
+    const u32 tiles = (u32)((m + OS_TILE - 1) / OS_TILE);
+    onesweep2_kernel<OS_CFG><<<tiles, OS_THREADS, sm, st>>>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch);
   }
-  if (want) sort_prof_dump(m, st, dprof, sort_tile_keys());
 }
 
 // digit histograms of plain keys: npass 8-bit digits from bit `shift` (race lists: 0; exchanged keys: pos_bits)

@@ -1,8 +1,74 @@
 // k_util.cu — single-pass exclusive scan of u32 counts (decoupled look-back), used for entry offsets of
 // multi-granule records and for flow-expansion offsets.  Offsets are u32: callers guarantee totals < 2^32.
+#include <algorithm>
+#include <map>
+#include <mutex>
+#include <tuple>
+
 #include "kernels.cuh"
 
 namespace sesa {
+
+// ---- per-device launch properties ----------------------------------------------------------------------------
+// The dynamic shared-memory opt-in of a kernel is stored per device context, and SM counts / occupancy are
+// properties of the device: cache them per (kernel, device) under a lock, so that handles on several devices
+// of one process (and host threads making their first call at the same time) each get a valid configuration.
+static std::mutex g_props_mu;
+
+static int current_device() {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  return dev;
+}
+
+int dev_sm_count() {
+  static std::map<int, int> sms;
+  const int dev = current_device();
+  std::lock_guard<std::mutex> lk(g_props_mu);
+  auto it = sms.find(dev);
+  if (it != sms.end()) return it->second;
+  int v = 0;
+  if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || v <= 0) {
+    cudaGetLastError();
+    v = 148;
+  }
+  sms[dev] = v;
+  return v;
+}
+
+static void smem_optin_locked(const void* kern, size_t bytes, int dev) {
+  static std::map<std::pair<const void*, int>, size_t> done;
+  auto it = done.find(std::make_pair(kern, dev));
+  if (it != done.end() && it->second >= bytes) return;  // never lowered
+  if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes) != cudaSuccess) {
+    cudaGetLastError();  // the launch reports the error
+    return;
+  }
+  done[std::make_pair(kern, dev)] = bytes;
+}
+
+void smem_optin(const void* kern, size_t bytes) {
+  const int dev = current_device();
+  std::lock_guard<std::mutex> lk(g_props_mu);
+  smem_optin_locked(kern, bytes, dev);
+}
+
+int blocks_per_sm(const void* kern, int threads, size_t smem) {
+  static std::map<std::tuple<const void*, int, int, size_t>, int> occ;
+  const int dev = current_device();
+  std::lock_guard<std::mutex> lk(g_props_mu);
+  const auto key = std::make_tuple(kern, dev, threads, smem);
+  auto it = occ.find(key);
+  if (it != occ.end()) return it->second;
+  smem_optin_locked(kern, smem, dev);
+  int per = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, kern, threads, smem) != cudaSuccess || per <= 0) {
+    cudaGetLastError();
+    per = 1;
+  }
+  occ[key] = per;
+  return per;
+}
 
 constexpr int SCAN_THREADS = 256, SCAN_ITEMS = 16, SCAN_TILE = SCAN_THREADS * SCAN_ITEMS;
 

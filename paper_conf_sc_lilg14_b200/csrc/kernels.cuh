@@ -43,6 +43,10 @@ void launch_fused_extract_pass0(const u32* gran, u64 n, const KeyLayout& L, u32 
                                 u32* hist, cudaStream_t st);
 
 // k_util.cu
+// per-device launch properties (thread-safe; the shared-memory opt-in is stored per device context)
+int dev_sm_count();                                       // SMs of the current device
+void smem_optin(const void* kern, size_t bytes);          // cudaFuncSetAttribute(MaxDynamicSharedMemorySize) once
+int blocks_per_sm(const void* kern, int threads, size_t smem);  // occupancy (opts in to `smem` first)
 size_t scan_u32_temp_bytes(u64 n);
 void launch_scan_exclusive_u32(const u32* in, u32* out, u64 n, void* temp, cudaStream_t st);  // out may alias in
 
@@ -147,7 +151,7 @@ void launch_benign_min_emit(const ConflictArgs& a, const struct RaceOut* cr, u32
 // k_compact.cu — keep only entries of locations touched >= 2 times (order preserved); *total = count
 size_t compact_temp_bytes(u64 m);
 // keys: sorted (m); seg: free buffer of m keys; out: where the result goes (may alias keys, which is dead after);
-// returns the array holding the m2 compacted keys (out, or seg for SESA_COMPACT=1)
+// returns out
 u64* launch_compact_multi(const u64* keys, u32 m, const KeyLayout& L, u64* seg, u64* out, void* temp, u32* total,
                           cudaStream_t st);
 

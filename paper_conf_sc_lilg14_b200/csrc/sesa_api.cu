@@ -218,20 +218,11 @@ bool sesa_trace::check_records_ptr(const sesa_access* d_rec, u64 n) {
 }
 
 // step 1: validation + extents of the local records -> h_summary (synchronises)
-static bool fused_enabled() {  // SESA_FUSED=0 disables the fused key extract + first sort pass
-  static int v = -1;
-  if (v < 0) {
-    const char* e = getenv("SESA_FUSED");
-    v = e ? atoi(e) : 1;
-  }
-  return v != 0;
-}
-
 bool sesa_trace::step_extents(const Rec* rec, u64 n, bool tile_hist) {
   const u32 log2G = (u32)__builtin_ctz(cfg.granularity);
   if (!grow(b_summary, sizeof(Summary), "summary")) return false;
   // per-tile raw digit histograms for the fused first pass (worth it only for traces of many tiles)
-  have_thist = tile_hist && fused_enabled() && n >= 32768;
+  have_thist = tile_hist && n >= 32768;
   if (have_thist && !grow(b_thist, ((n + FUSED_TILE - 1) / FUSED_TILE) * RADIX * 4, "tile histograms")) return false;
   // granule indices for the fused pass go to the key buffer the first sort pass after it writes (b_keys[0])
   if (have_thist && !grow(b_keys[0], n * 8 + 64, "keys")) return false;
@@ -852,9 +843,7 @@ sesa_status sesa_trace_create(const sesa_config* cfg, sesa_trace** out) {
   if (!t) return SESA_ENOMEM;
   t->cfg = *cfg;
   t->device = dev;
-  cudaDeviceGetAttribute(&t->num_sms, cudaDevAttrMultiProcessorCount, dev);
-
-  if (t->num_sms <= 0) t->num_sms = 148;
+  t->num_sms = sesa::dev_sm_count();
   *out = t;
   return SESA_OK;
 }
