@@ -163,7 +163,8 @@ typedef struct {
   uint32_t crossing_tiles;  /* conflict tiles with a location run crossing a tile boundary          */
   uint32_t n_stats;         /* valid entries of sesa_trace_kernel_stats                             */
   uint32_t fused_first_pass;/* key extract and the first sort pass ran as one kernel   */
-  uint32_t reserved;
+  uint32_t bucket_path;     /* the sort ran only over the two high digits and each chunk of 2^15 granules was
+                               resolved by a shared-memory bitmap ("bucket path")             */
 } sesa_check_info;
 
 /* Create a single-GPU handle on the current CUDA device.  cfg is validated (EINVAL on warp_size 0,

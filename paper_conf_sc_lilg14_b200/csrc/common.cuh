@@ -273,9 +273,15 @@ struct Summary {
   unsigned long long oob_count;  // valid records outside every registered region of their space (NEXT-1)
   unsigned long long oob_first;  // lowest such record index (~0 = none)
   // with tile histograms (fused-pass candidates): histograms of the raw granule bytes 1..3, (g >> 8b) & 255 —
-  // the later sort digits once gmin is aligned down to a multiple of 2^(8 (npass - 1)) (sesa_api.cu)
-  unsigned int bhist[3][256];
+  // the later sort digits once gmin is aligned down to a multiple of 2^(8 (npass - 1)) (sesa_api.cu); row 3:
+  // (g >> (HYB_LO + 8)) & 255, the second global digit of the bucket path (k_bucket.cu)
+  unsigned int bhist[4][256];
 };
+
+// bucket path (k_bucket.cu): the two global sort digits are key bits [HYB_LO, HYB_LO + 16); the bits below are
+// resolved per chunk of 2^HYB_CHUNK granules by a shared-memory bitmap and a shared-memory sort of the survivors
+constexpr unsigned HYB_LO = 14;
+constexpr unsigned HYB_CHUNK = 15;  // >= HYB_LO: a chunk = 2^15 granules (4 KB bitmaps; ~250 KB of C5 keys)
 
 // one registered memory region (include/sesa.h sesa_region), bytes [base, end)
 struct Region {

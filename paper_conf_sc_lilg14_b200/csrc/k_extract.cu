@@ -77,16 +77,20 @@ template <int U>
 // With gout != null the low 32 bits of the granule index addr >> log2G of every record are also written (4 bytes
 // per record,
 // coalesced): the fused pass then reads 8 bytes per record instead of the record's 32-byte sector.
+// With tile_hist2 != null (large traces: candidates for the bucket path, k_bucket.cu) each warp also writes the
+// per-tile histograms of the raw digit (g >> HYB_LO) & 255, and the CTA the histogram of (g >> (HYB_LO + 8)) & 255
+// (bhist[3]): the two global digits of the bucket path.
 __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ rec, u32 n, u32 log2G, u32 rw,
                                                        Summary* __restrict__ out, u32* __restrict__ tile_hist,
                                                        const Region* __restrict__ regs, uint3 rs,
-                                                       u32* __restrict__ gout) {
+                                                       u32* __restrict__ gout, u32* __restrict__ tile_hist2) {
   __shared__ u32 s_th[8][RADIX];
-  __shared__ u32 s_hb[3][RADIX];  // raw granule bytes 1..3 (with tile_hist)
+  __shared__ u32 s_th2[8][RADIX];
+  __shared__ u32 s_hb[4][RADIX];  // raw granule bytes 1..3 (with tile_hist), bits 22..29 (with tile_hist2)
   extern __shared__ Region s_reg[];  // [rs.z]
   for (u32 i = threadIdx.x; i < rs.z; i += 256) s_reg[i] = regs[i];
   if (tile_hist)
-    for (u32 i = threadIdx.x; i < 3 * RADIX; i += 256) (&s_hb[0][0])[i] = 0;
+    for (u32 i = threadIdx.x; i < 4 * RADIX; i += 256) (&s_hb[0][0])[i] = 0;
   if (rs.z || tile_hist) __syncthreads();
   constexpr int THREADS = 256;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -105,12 +109,16 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
     prev_bi = ((u64)p.x << 32) | p.z;
   }
   u32* th = s_th[warp];
+  u32* th2 = s_th2[warp];
   const u32 seg = tile_hist ? (u32)FUSED_TILE : rw;  // records between histogram flushes
   for (u32 t0 = start; t0 < end; t0 += seg) {
   const u32 tend = min(end, t0 + seg);
   if (tile_hist) {
 #pragma unroll
     for (int q = 0; q < RADIX / 32; q++) th[q * 32 + lane] = 0;
+    if (tile_hist2)
+#pragma unroll
+      for (int q = 0; q < RADIX / 32; q++) th2[q * 32 + lane] = 0;
     __syncwarp();
   }
   for (u32 r0 = t0; r0 < tend; r0 += 32 * U) {
@@ -175,6 +183,10 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
           atomicAdd(&s_hb[0][(u32)(g >> 8) & (RADIX - 1)], 1u);
           atomicAdd(&s_hb[1][(u32)(g >> 16) & (RADIX - 1)], 1u);
           atomicAdd(&s_hb[2][(u32)(g >> 24) & (RADIX - 1)], 1u);
+          if (tile_hist2) {
+            atomicAdd(&th2[(u32)(g >> HYB_LO) & (RADIX - 1)], 1u);
+            atomicAdd(&s_hb[3][(u32)(g >> (HYB_LO + RADIX_BITS)) & (RADIX - 1)], 1u);
+          }
         }
       }
       if (gout && r0 + u * 32 + lane < tend) __stcs(gout + r0 + u * 32 + lane, (u32)(addr >> log2G));
@@ -185,6 +197,11 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
     u32* dst = tile_hist + (u64)(t0 / FUSED_TILE) * RADIX;
 #pragma unroll
     for (int q = 0; q < RADIX / 32; q++) dst[q * 32 + lane] = th[q * 32 + lane];
+    if (tile_hist2) {
+      u32* dst2 = tile_hist2 + (u64)(t0 / FUSED_TILE) * RADIX;
+#pragma unroll
+      for (int q = 0; q < RADIX / 32; q++) dst2[q * 32 + lane] = th2[q * 32 + lane];
+    }
     __syncwarp();
   }
   }
@@ -198,7 +215,7 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
   }
   if (tile_hist) {
     __syncthreads();
-    for (u32 i = threadIdx.x; i < 3 * RADIX; i += 256) {
+    for (u32 i = threadIdx.x; i < (tile_hist2 ? 4u : 3u) * RADIX; i += 256) {
       const u32 v = (&s_hb[0][0])[i];
       if (v) atomicAdd(&(&out->bhist[0][0])[i], v);
     }
@@ -260,7 +277,7 @@ static int ring_grid(const void* kern, int threads, size_t smem) {
 }
 
 void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, u32* tile_hist, const Region* regs, u32 nreg,
-                    u32 nreg_shared, int grid, cudaStream_t st, u32* gout) {
+                    u32 nreg_shared, int grid, cudaStream_t st, u32* gout, u32* tile_hist2) {
   // extents2: contiguous warp ranges, one full wave of resident warps (the round-1 grid-stride kernel took
   // 7.7 ms on C5: 132 instructions per record, 64-bit index math and local-memory accumulators; this one 4.6 ms)
   const int sms = dev_sm_count(), per = blocks_per_sm((const void*)extents2_kernel<4>, 256, 0);
@@ -271,7 +288,8 @@ void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, u32* tile_
   rw = std::max<u64>(gran, (rw + gran - 1) / gran * gran);
   const u64 nw = (n + rw - 1) / rw;
   extents2_kernel<4><<<(unsigned)((nw + 7) / 8), 256, nreg * sizeof(Region), st>>>(
-      rec, (u32)n, log2G, (u32)rw, d_sum, tile_hist, regs, make_uint3(nreg_shared, 0u, nreg), gout);
+      rec, (u32)n, log2G, (u32)rw, d_sum, tile_hist, regs, make_uint3(nreg_shared, 0u, nreg), gout,
+      tile_hist ? tile_hist2 : nullptr);
   (void)grid;
 }
 

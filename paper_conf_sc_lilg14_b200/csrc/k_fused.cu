@@ -92,6 +92,7 @@ size_t fused_temp_bytes(u64 n) {
 struct FusedArgs {
   const u32* gran;  // low 32 bits of every record's granule index (written by the extents pass)
   u32 n, log2G, pos_bits, npass;
+  u32 dsh;          // the pass's digit is key_hi bits [dsh, dsh + 8): 0, or HYB_LO on the bucket path
   u64 gmin;
   const u32* toff;  // [T][RADIX] output offset of each tile's digit run
   u64* kout;
@@ -140,7 +141,7 @@ __global__ void __launch_bounds__(FUSED_THREADS, FUSED_MINB) fused_extract_pass0
     u32 kh[ITEMS];
 #pragma unroll
     for (int i = 0; i < ITEMS; i++) kh[i] = i < nv ? a[i] - (u32)A.gmin : 0u;
-    auto digit = [&](int i) -> u32 { return i < nv ? (kh[i] & (RADIX - 1)) : (u32)RADIX; };
+    auto digit = [&](int i) -> u32 { return i < nv ? ((kh[i] >> A.dsh) & (RADIX - 1)) : (u32)RADIX; };
     for (u32 i = tid; i < WARPS * RADIX; i += THREADS) whist[i] = 0;
     __syncthreads();
     // (1) per-warp counts of digit 0
@@ -193,7 +194,7 @@ __global__ void __launch_bounds__(FUSED_THREADS, FUSED_MINB) fused_extract_pass0
 #pragma unroll 4
     for (u32 j = tid; j < tcount; j += THREADS) {
       const u64 key = keys_s[j];
-      const u32 d = (u32)((key >> A.pos_bits) & (RADIX - 1));
+      const u32 d = (u32)((key >> (A.pos_bits + A.dsh)) & (RADIX - 1));
       __stcs(A.kout + (globu[d] + j), key);
 #pragma unroll
       for (int p = 1; p < NP; p++)
@@ -215,13 +216,13 @@ static size_t fused_smem(u32 npass) {
 bool fused_supported(u32 npass) { return npass >= 1 && npass <= 4; }  // sort_bits <= 32 on this path
 
 // tile offsets O[t][d] into temp (fused_temp_bytes(n)) from the extents' raw per-tile histograms
-void launch_tile_offsets(u64 n, const KeyLayout& L, const u32* tile_hist, void* temp, cudaStream_t st) {
+void launch_tile_offsets(u64 n, const KeyLayout& L, const u32* tile_hist, void* temp, cudaStream_t st, u32 dsh) {
   if (!n) return;
   const u32 T = (u32)((n + FUSED_TILE - 1) / FUSED_TILE);
   u32* O = reinterpret_cast<u32*>(temp);
   u32* P = reinterpret_cast<u32*>(reinterpret_cast<char*>(temp) + ((u64)T * RADIX * 4 + 255) / 256 * 256);
   const u32 C = std::min<u32>(T, 1024), tpc = (T + C - 1) / C, Cu = (T + tpc - 1) / tpc;
-  const u32 r0 = (u32)(L.gminG & (RADIX - 1));
+  const u32 r0 = (u32)((L.gminG >> dsh) & (RADIX - 1));
   tile_col_reduce_kernel<<<Cu, RADIX, 0, st>>>(tile_hist, T, tpc, P);
   tile_col_scan_kernel<<<1, RADIX, 0, st>>>(P, Cu, r0);
   tile_col_down_kernel<<<Cu, RADIX, 0, st>>>(tile_hist, T, tpc, P, r0, O);
@@ -229,7 +230,7 @@ void launch_tile_offsets(u64 n, const KeyLayout& L, const u32* tile_hist, void* 
 
 // temp: holds the tile offsets (launch_tile_offsets); hist: [npass][RADIX] zeroed (rows >= 1 filled)
 void launch_fused_extract_pass0(const u32* gran, u64 n, const KeyLayout& L, u32 npass, void* temp, u64* kout,
-                                u32* hist, cudaStream_t st) {
+                                u32* hist, cudaStream_t st, u32 dsh) {
   if (!n) return;
   const u32 T = (u32)((n + FUSED_TILE - 1) / FUSED_TILE);
   u32* O = reinterpret_cast<u32*>(temp);
@@ -245,6 +246,7 @@ void launch_fused_extract_pass0(const u32* gran, u64 n, const KeyLayout& L, u32 
   A.log2G = L.log2G;
   A.pos_bits = L.pos_bits;
   A.npass = npass;
+  A.dsh = dsh;
   A.gmin = L.gminG;
   A.toff = O;
   A.kout = kout;

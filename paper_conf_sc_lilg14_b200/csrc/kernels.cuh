@@ -25,8 +25,9 @@ constexpr int CT_TILE = CT_THREADS * CT_ITEMS;
 // tile_hist (optional, [ceil(n / FUSED_TILE)][RADIX]): per-tile histograms of (addr >> log2G) & 255 (k_fused.cu)
 // regs (optional, device, nreg <= MAX_REGIONS): sorted by (space, base), the first nreg_shared are SHARED
 // gout (optional, n x u32): low 32 bits of the granule index addr >> log2G of every record (fused-pass input)
+// tile_hist2 (optional, needs tile_hist): per-tile histograms of (addr >> log2G >> HYB_LO) & 255 (k_bucket.cu)
 void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, u32* tile_hist, const Region* regs, u32 nreg,
-                    u32 nreg_shared, int grid, cudaStream_t st, u32* gout = nullptr);
+                    u32 nreg_shared, int grid, cudaStream_t st, u32* gout = nullptr, u32* tile_hist2 = nullptr);
 void launch_extract_1to1(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, u64* keys, u32* hist, u64 pos_base,
                          int grid, cudaStream_t st);
 void launch_entry_count(const Rec* rec, u64 n, u32 log2G, u32* cnt, cudaStream_t st);
@@ -37,10 +38,21 @@ void launch_extract_multi(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, 
 // input, one granule per record); tile_hist from launch_extents
 bool fused_supported(u32 npass);
 size_t fused_temp_bytes(u64 n);
-void launch_tile_offsets(u64 n, const KeyLayout& L, const u32* tile_hist, void* temp, cudaStream_t st);
+// dsh: the digit is key_hi bits [dsh, dsh + 8) (tile_hist then holds the raw (g >> dsh) & 255 histograms and gmin
+// is a multiple of 2^dsh)
+void launch_tile_offsets(u64 n, const KeyLayout& L, const u32* tile_hist, void* temp, cudaStream_t st, u32 dsh = 0);
 // gran: the extents pass's granule indices (gout); rec is not read
 void launch_fused_extract_pass0(const u32* gran, u64 n, const KeyLayout& L, u32 npass, void* temp, u64* kout,
-                                u32* hist, cudaStream_t st);
+                                u32* hist, cudaStream_t st, u32 dsh = 0);
+
+constexpr uint64_t BUCKET_MIN_N = 1ull << 24;  // traces of fewer records keep the full sort
+// k_bucket.cu — bucket path of the sort + compaction (keys sorted by key_hi >> HYB_LO only)
+size_t bucket_temp_bytes(u32 nchunks);
+// sample of the chunk sizes from the extents' granule array: *h_max (host, after a sync) = largest sampled count
+u32 bucket_sample_max(const u32* gran, u32 n, u32 gmin_lo, u32 nchunks, void* temp, cudaStream_t st, u32* h_max,
+                      u32* samples);
+u32 launch_bucket_compact(u64* keys, u64* stage, u32 m, u32 pos_bits, u32 nchunks, void* temp, u32* total,
+                          cudaStream_t st);
 
 // k_util.cu
 // per-device launch properties (thread-safe; the shared-memory opt-in is stored per device context)

@@ -224,6 +224,9 @@ bool sesa_trace::step_extents(const Rec* rec, u64 n, bool tile_hist) {
   // per-tile raw digit histograms for the fused first pass (worth it only for traces of many tiles)
   have_thist = tile_hist && n >= 32768;
   if (have_thist && !grow(b_thist, ((n + FUSED_TILE - 1) / FUSED_TILE) * RADIX * 4, "tile histograms")) return false;
+  // large traces: also the tile histograms of the bucket path's first digit (k_bucket.cu)
+  have_thist2 = have_thist && n >= BUCKET_MIN_N;
+  if (have_thist2 && !grow(b_thist2, ((n + FUSED_TILE - 1) / FUSED_TILE) * RADIX * 4, "tile histograms")) return false;
   // granule indices for the fused pass go to the key buffer the first sort pass after it writes (b_keys[0])
   if (have_thist && !grow(b_keys[0], n * 8 + 64, "keys")) return false;
   Summary init;
@@ -240,7 +243,8 @@ bool sesa_trace::step_extents(const Rec* rec, u64 n, bool tile_hist) {
   LAUNCH("extents", (have_thist ? 36.0 : 32.0) * n, launch_extents(rec, n, log2G, (Summary*)b_summary.p,
                                              have_thist ? (u32*)b_thist.p : nullptr, (const Region*)b_regions.p,
                                              n_regions, n_regions_shared, grid_stream, stream,
-                                             have_thist ? (u32*)b_keys[0].p : nullptr));
+                                             have_thist ? (u32*)b_keys[0].p : nullptr,
+                                             have_thist2 ? (u32*)b_thist2.p : nullptr));
   if (!cuda_ok(cudaMemcpyAsync(&h_summary, b_summary.p, sizeof(Summary), cudaMemcpyDeviceToHost, stream), "summary"))
     return false;
   return sync_check("extents");
@@ -312,6 +316,84 @@ bool sesa_trace::step_extract_fused(const Rec* rec, u64 n) {
   LAUNCH("extract_pass0", 12.0 * n,
          launch_fused_extract_pass0((const u32*)b_keys[0].p, n, L, hist_from_extents ? 1u : npass, b_ftmp.p,
                                     (u64*)b_keys[1].p, (u32*)b_hist.p, stream));
+  return true;
+}
+
+// ---- bucket path (k_bucket.cu): decide, then fused pass on key_hi bits [14, 22), one onesweep pass on [22, 30),
+// per-chunk bitmap filter + sort of the survivors.  Chosen when the granules spread evenly: a sample of the
+// granule array must show no chunk of 2^HYB_CHUNK granules much above the mean (C5); hot regions (C3's bins,
+// C4's dist[]) keep the full sort, where almost every entry survives anyway.
+bool sesa_trace::bucket_choose(u64 n, u64* gmin_aligned, u32* nbits, u32* nchunks) {
+  const Summary& S = h_summary;
+  const u32 D = HYB_LO + RADIX_BITS;  // gmin aligned to 2^22: both global digits are raw granule bytes, rotated
+  const u64 G0 = S.gmin[1] & ~((1ull << D) - 1ull);
+  const u32 nb = bits_of(S.gmax[1] - G0);
+  if (nb <= D || nb > HYB_LO + 2 * RADIX_BITS || nb + layout.pos_bits > 64) return false;
+  const u32 nc = (u32)(((S.gmax[1] - G0) >> HYB_CHUNK) + 1);
+  if (!grow(b_btmp2, bucket_temp_bytes(nc), "bucket temp")) return false;
+  u32 hmax = 0, samples = 0;
+  LAUNCH("bucket_sample", 4.0 * (n >> 8), launches += bucket_sample_max((const u32*)b_keys[0].p, (u32)n, (u32)G0, nc,
+                                                                        b_btmp2.p, stream, &hmax, &samples) - 1);
+  if (!sync_check("bucket sample")) return false;
+  const double est_max = (double)hmax * (double)n / (double)std::max(1u, samples), mean = (double)n / nc;
+  if (est_max > 4.0 * mean + 2048.0 || est_max > (double)(1u << 20)) return false;
+  *gmin_aligned = G0;
+  *nbits = nb;
+  *nchunks = nc;
+  return true;
+}
+
+bool sesa_trace::step_bucket(u64 n, u32 nchunks, u64** comp, u32* m2) {
+  const KeyLayout& L = layout;
+  if (!grow(b_keys[1], n * 8 + 64, "keys") || !grow(b_hist, 2 * RADIX * 4, "hist") ||
+      !grow(b_binbase, 2 * RADIX * 8, "binbase") || !grow(b_ftmp, fused_temp_bytes(n), "fused temp") ||
+      !grow(b_ctotal, 16, "compact count"))
+    return false;
+  // digit B (key_hi bits [22, 30)) = raw granule bits [22, 30) rotated by those of gmin: its histogram is the
+  // extents' row 3
+  std::vector<u32> row(RADIX);
+  const u32 r = (u32)(L.gminG >> (HYB_LO + RADIX_BITS)) & (RADIX - 1);
+  for (u32 d = 0; d < (u32)RADIX; d++) row[d] = h_summary.bhist[3][(d + r) & (RADIX - 1)];
+  if (!cuda_ok(cudaMemcpyAsync((u32*)b_hist.p + RADIX, row.data(), RADIX * 4, cudaMemcpyHostToDevice, stream), "hist"))
+    return false;
+  cudaMemsetAsync(b_hist.p, 0, RADIX * 4, stream);
+  LAUNCH("tile_offsets", 2.0 * RADIX * 4 * ((n + FUSED_TILE - 1) / FUSED_TILE),
+         launch_tile_offsets(n, L, (const u32*)b_thist2.p, b_ftmp.p, stream, HYB_LO));
+  LAUNCH("extract_pass0", 12.0 * n,
+         launch_fused_extract_pass0((const u32*)b_keys[0].p, n, L, 1, b_ftmp.p, (u64*)b_keys[1].p, (u32*)b_hist.p,
+                                    stream, HYB_LO));
+  int cur = 1;
+  u32 passes = 1;
+  if (*std::max_element(row.begin(), row.end()) != n) {  // digit B not trivial
+    LAUNCH("bin_base", 0.0, launch_bin_base((u32*)b_hist.p, (u64*)b_binbase.p, 2, stream));
+    const u32 stiles = sort_tiles(n);
+    if (!grow(b_lookback, (size_t)stiles * RADIX * 8, "lookback") || !grow(b_ctr, 64 * 4, "counters")) return false;
+    if (b_lookback.cap != lookback_cleared) {
+      cudaMemsetAsync(b_lookback.p, 0, b_lookback.cap, stream);
+      lookback_cleared = b_lookback.cap;
+      epoch = 0;
+    }
+    cudaMemsetAsync(b_ctr.p, 0, 64 * 4, stream);
+    if (++epoch >= 256) {
+      cudaMemsetAsync(b_lookback.p, 0, b_lookback.cap, stream);
+      epoch = 1;
+    }
+    LAUNCH("onesweep_pass", 16.0 * n,
+           launch_onesweep((u64*)b_keys[1].p, (u64*)b_keys[0].p, nullptr, nullptr, (u32)n,
+                           L.pos_bits + HYB_LO + RADIX_BITS, (u64*)b_binbase.p + RADIX, (u64*)b_lookback.p,
+                           (u32*)b_ctr.p, epoch, stream));
+    cur = 0;
+    passes++;
+  }
+  info.sort_passes = passes;
+  // per-chunk bitmap filter + sort of the survivors; result (sorted, compacted) back in b_keys[cur]
+  LAUNCH("bucket", 8.0 * n,
+         launches += launch_bucket_compact((u64*)b_keys[cur].p, (u64*)b_keys[cur ^ 1].p, (u32)n, L.pos_bits, nchunks,
+                                           b_btmp2.p, (u32*)b_ctotal.p, stream) - 1);
+  *comp = (u64*)b_keys[cur].p;
+  if (!cuda_ok(cudaMemcpyAsync(m2, b_ctotal.p, 4, cudaMemcpyDeviceToHost, stream), "bucket count")) return false;
+  if (!sync_check("bucket")) return false;
+  info.n_multi = *m2;
   return true;
 }
 
@@ -685,6 +767,21 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
   const bool fused = have_thist && !layout.both && layout.single_space == SP_GLOBAL && layout.lowG == 0 &&
                      S.multi == 0 && m == n && layout.sort_bits <= 32 && fused_supported(npass);
   info.fused_first_pass = fused ? 1 : 0;
+  // bucket path: large traces whose granules spread evenly (k_bucket.cu)
+  u64 hyb_g0 = 0;
+  u32 hyb_nb = 0, hyb_nc = 0;
+  if (fused && have_thist2 && bucket_choose(n, &hyb_g0, &hyb_nb, &hyb_nc)) {
+    layout.gminG = hyb_g0;
+    layout.gbG = hyb_nb;
+    layout.sort_bits = hyb_nb;
+    info.sort_bits = hyb_nb;
+    info.bucket_path = 1;
+    u64* comp = nullptr;
+    u32 m2 = 0;
+    if (!step_bucket(n, hyb_nc, &comp, &m2)) return status;
+    return finish_check(comp, m2, rec, index_base);
+  }
+  if (status != SESA_OK) return status;
   // Fused path: align gmin down to a multiple of 2^(8 (npass - 1)).  Then every later sort digit of
   // key_hi = g - gmin is a raw granule byte (the top one rotated by a constant), whose histograms the extents
   // pass already took — the fused pass needs no histogram atomics.  Only if the aligned span needs no extra pass.
@@ -710,6 +807,11 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
   u64* comp = nullptr;
   u32 m2 = 0;
   if (!step_compact(cur, m, &comp, &m2)) return status;
+  return finish_check(comp, m2, rec, index_base);
+}
+
+// steps 5-6 (shared by the sort + compaction and the bucket paths): conflict tiles, benign regrouping, race sort
+sesa_status sesa_trace::finish_check(const u64* comp, u32 m2, const Rec* rec, u64 index_base) {
   if (!step_conflict(comp, m2, rec, 0, nullptr, index_base)) return status;
   if (!step_benign(comp, m2, rec, index_base)) return status;
   const u32 nr = (u32)n_races;

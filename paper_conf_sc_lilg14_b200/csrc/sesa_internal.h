@@ -42,7 +42,8 @@ struct sesa_trace {
   DevBuf b_summary, b_keys[2], b_hist, b_binbase, b_lookback, b_ctr, b_cnt, b_off, b_temp;
   DevBuf b_tflags, b_part, b_carry, b_owner, b_slots, b_cross, b_ccount, b_carrytmp;
   DevBuf b_races, b_rkeys[2], b_rvals[2], b_races_sorted, b_rhist, b_rbase;
-  DevBuf b_eoff, b_ecnt, b_ecell, b_hrec, b_dist_races, b_ctmp, b_ctotal, b_thist, b_ftmp;
+  DevBuf b_eoff, b_ecnt, b_ecell, b_hrec, b_dist_races, b_ctmp, b_ctotal, b_thist, b_ftmp, b_thist2, b_btmp2;
+  bool have_thist2 = false;  // extents also wrote the per-tile histograms of the bucket path's first digit
   bool have_thist = false;
   bool hist_from_extents = false;  // fused path: later-digit histograms from the extents' raw granule bytes  // extents wrote per-tile raw digit histograms (fused first pass possible)
   // out-of-bound check (NEXT-1): registered regions (sorted by space, base) and the last report
@@ -61,7 +62,7 @@ struct sesa_trace {
     std::vector<DevBuf*> v = {&b_summary, &b_hist, &b_binbase, &b_lookback, &b_ctr, &b_cnt, &b_off, &b_temp,
                               &b_tflags, &b_part, &b_carry, &b_owner, &b_slots, &b_cross, &b_ccount, &b_carrytmp,
                               &b_races, &b_races_sorted, &b_rhist, &b_rbase, &b_eoff, &b_ecnt, &b_ecell,
-                              &b_hrec, &b_dist_races, &b_ctmp, &b_ctotal, &b_thist, &b_ftmp, &b_regions,
+                              &b_hrec, &b_dist_races, &b_ctmp, &b_ctotal, &b_thist, &b_ftmp, &b_thist2, &b_btmp2, &b_regions,
                               &b_bhead, &b_bhscan, &b_bwf, &b_bwscan, &b_bgid, &b_bvk[0], &b_bvk[1], &b_bvi[0],
                               &b_bvi[1], &b_brh, &b_brscan, &b_bder, &b_bdpos, &b_bdj, &b_bslot, &b_btmp};
     for (auto& b : b_keys) v.push_back(&b);
@@ -97,6 +98,7 @@ struct sesa_trace {
   void collect_prof();
   bool make_layout(const sesa::Summary& S, uint64_t n);
   sesa_status check_device(const sesa_access* d_rec, uint64_t n, uint64_t index_base);
+  sesa_status finish_check(const uint64_t* comp, uint32_t m2, const sesa::Rec* rec, uint64_t index_base);
   // pipeline steps (shared by the single-GPU and the distributed check)
   void begin_check(uint64_t n);
   bool check_records_ptr(const sesa_access* d_rec, uint64_t n);
@@ -106,6 +108,8 @@ struct sesa_trace {
   bool step_extract(const sesa::Rec* rec, uint64_t n, uint64_t m, uint64_t pos_base, bool multi);
   bool step_hist(uint64_t m);
   bool step_extract_fused(const sesa::Rec* rec, uint64_t n);
+  bool bucket_choose(uint64_t n, uint64_t* gmin_aligned, uint32_t* nbits, uint32_t* nchunks);
+  bool step_bucket(uint64_t n, uint32_t nchunks, uint64_t** comp, uint32_t* m2);
   bool step_sort(uint64_t m, int* cur_out, uint32_t first_pass = 0, int cur0 = 0);
   bool step_compact(int cur, uint64_t m, uint64_t** comp, uint32_t* m2);
   bool step_conflict(const uint64_t* comp, uint32_t m2, const sesa::Rec* rec, uint32_t rec_pos_base,

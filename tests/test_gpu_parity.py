@@ -415,3 +415,53 @@ def test_oob_region_validation(sesa):
     t.set_regions(reg)  # adjacent, fine
     t.set_regions(reg[:0])  # clears
     t.close()
+
+
+# ------------------------------------------------------------------------------------------------ bucket path
+# Large single-space traces with evenly spread granules take the bucket path (k_bucket.cu: two high-digit sort
+# passes, per-chunk shared-memory bitmaps, survivors sorted per chunk); it must give the oracle's list exactly,
+# through the bitonic (few survivors per chunk) and the overflow (> 4096 survivors per chunk) sorts.
+@pytest.mark.slow
+@pytest.mark.parametrize("words_log2,ls,benign", [(28, 0, False), (26, 1, False), (25, 0, True), (27, 1, True)])
+def test_bucket_path_random(sesa, words_log2, ls, benign):
+    from sesagen import configs as C
+    n = 20_000_000
+    r = C.rnd_host(n, 40 + words_log2, blocks=4096, threads=512, intervals=3, words=1 << words_log2,
+                   shared_frac=0.0, sizes=(4,), unaligned=False, values=3, atomic_frac=0.05, write_frac=0.35)
+    t = sesa.Trace(32, ls, 4, benign=benign)
+    t.check(sesa.to_device(r), n)
+    assert t.info()["bucket_path"] == 1
+    got = t.races()
+    t.close()
+    exp = O.check(r, warp_size=32, lockstep=ls, benign=benign, method="partitioned")
+    assert len(got) == len(exp) and got.tobytes() == exp.tobytes()
+
+
+@pytest.mark.slow
+def test_bucket_path_c5_reduced(sesa):
+    """C5's recipe at 2^24 + 12345 records: the bucket path's race list equals the construction truth and the
+    oracle's."""
+    from sesagen import configs as C
+    n = (1 << 24) + 12345
+    dev = C.c5_device(n)
+    t = sesa.Trace(32, 0, 4)
+    t.check(dev, n)
+    assert t.info()["bucket_path"] == 1
+    got = t.races()
+    t.close()
+    assert got.tobytes() == C.c5_truth(n).tobytes()
+    host = dev.cpu().numpy().view(G.REC_DTYPE)
+    assert got.tobytes() == O.check(host, method="partitioned").tobytes()
+
+
+@pytest.mark.slow
+def test_hot_traces_keep_the_full_sort(sesa):
+    """The sample test sends traces with a hot granule region to the full sort (C3-shaped: Zipf bins)."""
+    from sesagen import configs as C
+    cfg = C.C3(blocks=384)
+    dev, n = cfg.device()
+    assert n >= 1 << 24
+    t = sesa.Trace(32, 0, 4)
+    t.check(dev, n)
+    assert t.info()["bucket_path"] == 0
+    t.close()
