@@ -281,7 +281,7 @@ struct Summary {
 // bucket path (k_bucket.cu): the two global sort digits are key bits [HYB_LO, HYB_LO + 16); the bits below are
 // resolved per chunk of 2^HYB_CHUNK granules by a shared-memory bitmap and a shared-memory sort of the survivors
 constexpr unsigned HYB_LO = 14;
-constexpr unsigned HYB_CHUNK = 15;  // >= HYB_LO: a chunk = 2^15 granules (4 KB bitmaps; ~250 KB of C5 keys)
+constexpr unsigned HYB_CHUNK = 15;  // >= HYB_LO: a chunk = 2^15 granules (4 KB bitmaps; ~30 K C5 keys)
 
 // one registered memory region (include/sesa.h sesa_region), bytes [base, end)
 struct Region {

@@ -11,7 +11,8 @@
 //            word: a bit already set marks the granule "touched >= 2 times" in a second bitmap)
 //   sweep 2  stream the keys again (an L2 hit: chunks are ~250 KB) and keep those at marked granules, in order
 //   sort     the survivors by their full 64-bit key (granule, then record position) — a bitonic sort in shared
-//            memory, or, beyond its capacity, a stable two-pass radix sort of the chunk's range in global memory
+//            memory, or, beyond its capacity (2048), a stable two-pass radix sort of the chunk's range in global
+//            memory
 // Output: the chunk's survivors, sorted, at the chunk's own offset of the other key buffer, plus a count; a scan
 // of the counts and a gather concatenate them — exactly the array the full sort + compaction produce.
 //
@@ -23,7 +24,12 @@
 
 namespace sesa {
 
-constexpr int BK_THREADS = 256, BK_WORDS = (1 << HYB_CHUNK) / 32, BK_CAPC = 4096, BK_U = 4;
+// Measured on C5 (bucket kernels per 1e9 keys): chunks of 2^15 granules with 8 keys in flight per thread and the
+// next round's loads issued before the current round is processed: 2.28 ms; 4 in flight 2.37 (2.51 without the
+// prefetch); chunks of 2^14: 2.39; 2^16: 3.21; sweep 2 from 16-bit granule offsets kept in shared memory instead
+// of re-reading the keys (an L2 hit): 3.35 (the smem footprint halves the CTAs per SM).
+constexpr int BK_THREADS = 256, BK_WORDS = (1 << HYB_CHUNK) / 32, BK_CAPC = 2048, BK_U = 8;
+constexpr size_t BK_DSMEM = (size_t)BK_CAPC * 8;  // dynamic: the survivors
 
 // ---- chunk boundaries: bounds[c] = first position whose key is >= c << (HYB_CHUNK + pos_bits) (warp per c) ----
 __global__ void bucket_bounds_kernel(const u64* __restrict__ keys, u32 m, u32 nchunks, u32 shift,
@@ -86,7 +92,8 @@ __device__ __forceinline__ void bitonic_smem(u64* a, u32 k, u32 kp) {
 
 __global__ void __launch_bounds__(BK_THREADS) bucket_local_kernel(BucketArgs A) {
   __shared__ u32 seen[BK_WORDS], dup[BK_WORDS];
-  __shared__ __align__(16) u64 cand[BK_CAPC];
+  extern __shared__ __align__(16) unsigned char bk_dyn[];
+  u64* cand = reinterpret_cast<u64*>(bk_dyn);  // [BK_CAPC] survivors
   __shared__ u32 s_chunk, s_w[BK_THREADS / 32 + 1];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const u32 gmask = (1u << HYB_CHUNK) - 1u;
@@ -98,34 +105,41 @@ __global__ void __launch_bounds__(BK_THREADS) bucket_local_kernel(BucketArgs A) 
     const u32 c = s_chunk;
     if (c >= A.nchunks) return;
     const u32 s = A.bounds[c], e = A.bounds[c + 1];
-    // sweep 1: granule bitmap; a second touch marks the granule
-    for (u32 b0 = s; b0 < e; b0 += BK_THREADS * BK_U) {
-      u64 k[BK_U];
+    // sweep 1: the chunk's keys (BK_U in flight per thread, the next round's loads issued before this round is
+    // processed; kept in L2 for sweep 2): granule bitmap, a second touch marks the granule
+    u64 k[BK_U];
+    auto load = [&](u64* dst, u32 b0) {
 #pragma unroll
       for (int u = 0; u < BK_U; u++) {
         const u32 i = b0 + u * BK_THREADS + tid;
-        k[u] = i < e ? __ldcg(A.keys + i) : 0ull;
+        dst[u] = i < e ? __ldcg(A.keys + i) : 0ull;
       }
+    };
+    load(k, s);
+    for (u32 b0 = s; b0 < e; b0 += BK_THREADS * BK_U) {
+      u64 kn[BK_U];
+      load(kn, b0 + BK_THREADS * BK_U);  // next round in flight while this one is processed
 #pragma unroll
       for (int u = 0; u < BK_U; u++) {
-        if (b0 + u * BK_THREADS + tid >= e) continue;
+        const u32 i = b0 + u * BK_THREADS + tid;
+        if (i >= e) continue;
         const u32 g = (u32)(k[u] >> A.pos_bits) & gmask, bit = 1u << (g & 31);
         if (atomicOr(&seen[g >> 5], bit) & bit) atomicOr(&dup[g >> 5], bit);
       }
+#pragma unroll
+      for (int u = 0; u < BK_U; u++) k[u] = kn[u];
     }
     __syncthreads();
-    // sweep 2: survivors in order (element order = position), into shared memory while they fit, else straight
-    // to the chunk's staging range
+    // sweep 2: survivors in order (element order = position); their full keys are read back (few on this path)
     u32 k_total = 0;  // survivors so far (uniform)
     for (u32 b0 = s; b0 < e; b0 += BK_THREADS * BK_U) {
-      u64 k[BK_U];
       bool keep[BK_U];
       bool any = false;
 #pragma unroll
       for (int u = 0; u < BK_U; u++) {
         const u32 i = b0 + u * BK_THREADS + tid;
-        k[u] = i < e ? __ldcs(A.keys + i) : 0ull;
-        const u32 g = (u32)(k[u] >> A.pos_bits) & gmask;
+        u32 g = 0;
+        if (i < e) g = (u32)(__ldcs(A.keys + i) >> A.pos_bits) & gmask;
         keep[u] = i < e && ((dup[g >> 5] >> (g & 31)) & 1u);
         any |= keep[u];
       }
@@ -142,9 +156,11 @@ __global__ void __launch_bounds__(BK_THREADS) bucket_local_kernel(BucketArgs A) 
           row += x;
         }
         if (keep[u]) {
+          const u32 i = b0 + u * BK_THREADS + tid;
+          const u64 key = __ldcg(A.keys + i);
           const u32 j = k_total + before + __popc(bal & lt);
-          if (j < BK_CAPC) cand[j] = k[u];
-          A.stage[s + j] = k[u];  // (also staged: the overflow path reads the survivors from here)
+          if (j < BK_CAPC) cand[j] = key;
+          A.stage[s + j] = key;  // (also staged: the overflow path reads the survivors from here)
         }
         k_total += row;
         __syncthreads();
@@ -300,9 +316,9 @@ u32 launch_bucket_compact(u64* keys, u64* stage, u32 m, u32 pos_bits, u32 nchunk
   A.over = over;
   A.nchunks = nchunks;
   A.pos_bits = pos_bits;
-  const int per = blocks_per_sm((const void*)bucket_local_kernel, BK_THREADS, 0);
+  const int per = blocks_per_sm((const void*)bucket_local_kernel, BK_THREADS, BK_DSMEM);
   const u32 grid = std::min<u32>(nchunks, (u32)(dev_sm_count() * per));
-  bucket_local_kernel<<<grid, BK_THREADS, 0, st>>>(A);
+  bucket_local_kernel<<<grid, BK_THREADS, BK_DSMEM, st>>>(A);
   // overflow chunks (rare on this path; their count is on the device): a small grid walks the list
   bucket_overflow_kernel<<<dev_sm_count(), BK_THREADS, 0, st>>>(A);
   launch_scan_exclusive_u32(cnt, off, nchunks, stemp, st);
