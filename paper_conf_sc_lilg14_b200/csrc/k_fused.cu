@@ -102,7 +102,9 @@ struct FusedArgs {
 // Persistent CTAs, software-pipelined in registers: right after a tile's digit counts (when its addresses have
 // become 32-bit key parts), the CTA issues the loads of its NEXT tile's addresses into the freed registers, so
 // they are in flight during the ranking and write-out of the current tile — the CTA's HBM reads never pause.
-template <int NP>
+// UNST (the bucket path, which needs no stable order within a digit): the count atomic's return value is the
+// key's rank within its (warp, digit) group, and the ranking loop is skipped.
+template <int NP, bool UNST = false>
 __global__ void __launch_bounds__(FUSED_THREADS, FUSED_MINB) fused_extract_pass0_kernel(FusedArgs A) {
   constexpr int THREADS = FUSED_THREADS, ITEMS = FUSED_ITEMS, WARPS = THREADS / 32, TILE = FUSED_TILE;
   extern __shared__ __align__(16) unsigned char smem[];
@@ -144,10 +146,17 @@ __global__ void __launch_bounds__(FUSED_THREADS, FUSED_MINB) fused_extract_pass0
     auto digit = [&](int i) -> u32 { return i < nv ? ((kh[i] >> A.dsh) & (RADIX - 1)) : (u32)RADIX; };
     for (u32 i = tid; i < WARPS * RADIX; i += THREADS) whist[i] = 0;
     __syncthreads();
-    // (1) per-warp counts of digit 0
+    // (1) per-warp counts of the digit (UNST: with the ranks)
+    u32 rk[UNST ? (ITEMS + 1) / 2 : 1];
+    if (UNST)
+#pragma unroll
+      for (int i = 0; i < (ITEMS + 1) / 2; i++) rk[i] = 0;
 #pragma unroll
     for (int i = 0; i < ITEMS; i++)
-      if (i < nv) atomicAdd(&wh[digit(i)], 1u);
+      if (i < nv) {
+        const u32 r = atomicAdd(&wh[digit(i)], 1u);
+        if (UNST) rk[i / 2] |= r << (16 * (i & 1));
+      }
     __syncthreads();
     // (2) tile-local bases = bin start + warp offset; global write offsets from the precomputed table
     u32 tot = 0;
@@ -168,6 +177,15 @@ __global__ void __launch_bounds__(FUSED_THREADS, FUSED_MINB) fused_extract_pass0
     __syncthreads();
     const u32 next = tile + gridDim.x;
     if (next < T) issue(next);  // prefetch: in flight during ranking and write-out
+    if (UNST) {
+      // (3') each key straight to its slot: (warp, digit) base + its count-atomic rank
+#pragma unroll
+      for (int i = 0; i < ITEMS; i++) {
+        const u32 d = digit(i);
+        if (d < RADIX)
+          keys_s[wh[d] + ((rk[i / 2] >> (16 * (i & 1))) & 0xFFFFu)] = ((u64)kh[i] << A.pos_bits) | (u64)(wbase + i * 32);
+      }
+    } else {
     // (3) stable warp ranking (peer masks by shared-memory atomicOr), each key stored into its tile slot
 #pragma unroll
     for (int i = 0; i < ITEMS; i++) {
@@ -188,6 +206,7 @@ __global__ void __launch_bounds__(FUSED_THREADS, FUSED_MINB) fused_extract_pass0
       }
       __syncwarp();
     }
+        }
     __syncthreads();
     // (4) coalesced write-out of each digit run, and the CTA histograms of the later digits
     const u32 tcount = min((u32)TILE, A.n - tbase);
@@ -230,7 +249,7 @@ void launch_tile_offsets(u64 n, const KeyLayout& L, const u32* tile_hist, void* 
 
 // temp: holds the tile offsets (launch_tile_offsets); hist: [npass][RADIX] zeroed (rows >= 1 filled)
 void launch_fused_extract_pass0(const u32* gran, u64 n, const KeyLayout& L, u32 npass, void* temp, u64* kout,
-                                u32* hist, cudaStream_t st, u32 dsh) {
+                                u32* hist, cudaStream_t st, u32 dsh, bool unstable) {
   if (!n) return;
   const u32 T = (u32)((n + FUSED_TILE - 1) / FUSED_TILE);
   u32* O = reinterpret_cast<u32*>(temp);
@@ -252,6 +271,11 @@ void launch_fused_extract_pass0(const u32* gran, u64 n, const KeyLayout& L, u32 
   A.kout = kout;
   A.hist = hist;
   const u32 g = std::min<u32>(T, (u32)grid);
+  if (unstable) {  // the bucket path: one digit, no later-digit histograms
+    smem_optin((const void*)fused_extract_pass0_kernel<1, true>, sm);
+    fused_extract_pass0_kernel<1, true><<<g, FUSED_THREADS, sm, st>>>(A);
+    return;
+  }
   switch (npass) {
     case 1: fused_extract_pass0_kernel<1><<<g, FUSED_THREADS, sm, st>>>(A); break;
     case 2: fused_extract_pass0_kernel<2><<<g, FUSED_THREADS, sm, st>>>(A); break;

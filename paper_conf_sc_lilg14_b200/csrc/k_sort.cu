@@ -235,7 +235,8 @@ __device__ __forceinline__ u64 gtime() {
 // and runs 3% slower (4.94 vs 4.80 ms per 1e9 keys, measured).
 __device__ unsigned long long* g_prof = nullptr;
 
-template <int THREADS, int ITEMS, int LBW, bool FULL, bool LATE_LB, int S, bool BAL, int TMA, int MIX = 0>
+template <int THREADS, int ITEMS, int LBW, bool FULL, bool LATE_LB, int S, bool BAL, int TMA, int MIX = 0,
+          bool UNST = false>
 __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64* __restrict__ kout, u32 m, u32 shift,
                                                const u64* __restrict__ bin_base, u64* __restrict__ lookback,
                                                u32 epoch, u32 tile, unsigned char* smem, unsigned long long* prof,
@@ -291,10 +292,18 @@ __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64*
     __syncthreads();
     if (tid == 0) prof[1] = gtime();
   }
-  // (1) per-(warp, stream) digit counts
+  // (1) per-(warp, stream) digit counts.  UNST (the bucket path's partition passes, which need no stable order):
+  //     the count atomic's return value is the key's rank within its (warp, digit) group — no ranking loop
+  u32 rk[UNST ? (ITEMS + 1) / 2 : 1];
+  if (UNST)
+#pragma unroll
+    for (int i = 0; i < (ITEMS + 1) / 2; i++) rk[i] = 0;
 #pragma unroll
   for (int i = 0; i < ITEMS; i++)
-    if (FULL || i < nv) atomicAdd(&wh[(i / IPS) * RADIX + digit(i)], 1u);
+    if (FULL || i < nv) {
+      const u32 r = atomicAdd(&wh[(i / IPS) * RADIX + digit(i)], 1u);
+      if (UNST) rk[i / 2] |= r << (16 * (i & 1));
+    }
   __syncthreads();
   // (2) tile totals -> publish the aggregate; per-(warp, stream, digit) tile-local base = bin start + offset
   u32 tot = 0;
@@ -348,6 +357,14 @@ __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64*
   if (!LATE_LB) look_back();
   __syncthreads();
   if (prof && tid == 0) prof[2] = gtime();
+  if (UNST) {
+    // (3') each key straight to its slot: (warp, digit) base + its count-atomic rank
+#pragma unroll
+    for (int i = 0; i < ITEMS; i++) {
+      const u32 d = digit(i);
+      if (FULL || d < RADIX) keys_s[wh[d] + ((rk[i / 2] >> (16 * (i & 1))) & 0xFFFFu)] = k[i];
+    }
+  } else {
   // (3) stable warp ranking, each key stored straight into its tile-local slot
   u32* wm = wmask + warp * S * (RADIX + 1);
   const unsigned lt = lanemask_lt();
@@ -386,6 +403,7 @@ __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64*
     }
     __syncwarp();
   }
+  }
   if (prof && tid == 0) prof[3] = gtime();
   if (LATE_LB) look_back();
   __syncthreads();
@@ -404,7 +422,8 @@ __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64*
   }
 }
 
-template <int THREADS, int ITEMS, int MINB, int LBW, bool LATE_LB, int S, bool BAL, int TMA, int MIX = 0>
+template <int THREADS, int ITEMS, int MINB, int LBW, bool LATE_LB, int S, bool BAL, int TMA, int MIX = 0,
+          bool UNST = false>
 __global__ void __launch_bounds__(THREADS, MINB) onesweep2_kernel(const u64* __restrict__ kin, u64* __restrict__ kout,
                                                                   u32 m, u32 shift, const u64* __restrict__ bin_base,
                                                                   u64* __restrict__ lookback,
@@ -433,21 +452,28 @@ __global__ void __launch_bounds__(THREADS, MINB) onesweep2_kernel(const u64* __r
     }
   }
   for (int i = tid; i < WARPS * S * RADIX; i += THREADS) whist[i] = 0;
-  if (!BAL)
+  if (!BAL && !UNST)
     for (int i = tid; i < WARPS * S * (RADIX + 1); i += THREADS) wmask[i] = 0;
   __syncthreads();
   const u32 tile = s_tile;
   unsigned long long* prof = g_prof ? g_prof + (u64)tile * 8 : nullptr;
   if (prof && tid == 0) prof[0] = gtime();
   if ((u64)(tile + 1) * TILE <= m)
-    onesweep2_tile<THREADS, ITEMS, LBW, true, LATE_LB, S, BAL, TMA, MIX>(kin, kout, m, shift, bin_base, lookback, epoch, tile, smem, prof, &ebar);
+    onesweep2_tile<THREADS, ITEMS, LBW, true, LATE_LB, S, BAL, TMA, MIX, UNST>(kin, kout, m, shift, bin_base, lookback,
+                                                                             epoch, tile, smem, prof, &ebar);
   else
-    onesweep2_tile<THREADS, ITEMS, LBW, false, LATE_LB, S, BAL, TMA, MIX>(kin, kout, m, shift, bin_base, lookback, epoch, tile, smem, prof, &ebar);
+    onesweep2_tile<THREADS, ITEMS, LBW, false, LATE_LB, S, BAL, TMA, MIX, UNST>(kin, kout, m, shift, bin_base, lookback,
+                                                                              epoch, tile, smem, prof, &ebar);
 }
 
 // the measured configuration: 256 x 32 keys, 2 CTAs/SM, look-back after ranking, one rank stream,
 // prologue bulk copies (TMA 2), every 4th item's peers by ballots (MIX 4)
 #define OS_CFG OS_THREADS, OS_ITEMS, OS_MINB, OS_LBW, true, 1, false, 2, 4
+// the bucket path's partition pass (no stable order needed)
+// (measured on C5, per 1e9 keys: 256 x 32 at 2 CTAs/SM 4.09 ms; 256 x 24 at 3: 4.21; 256 x 20 at 3: 4.36;
+// 512 x 16 at 2: 4.44; 256 x 16 at 4: 4.69)
+constexpr int PT_THREADS = 256, PT_ITEMS = 32, PT_MINB = 2;
+#define OS_UCFG PT_THREADS, PT_ITEMS, PT_MINB, OS_LBW, true, 1, false, 2, 4, true
 
 static size_t onesweep2_smem() {
   constexpr int WARPS = OS_THREADS / 32;
@@ -456,6 +482,17 @@ static size_t onesweep2_smem() {
 }
 
 u32 sort_tile_keys() { return OS_TILE; }
+
+// unstable partition pass (the bucket path: chunk order only, survivors are sorted per chunk afterwards)
+void launch_partition_pass(const u64* kin, u64* kout, u32 m, u32 shift, const u64* bin_base, u64* lookback,
+                           u32* tile_ctr, u32 epoch, cudaStream_t st) {
+  if (!m) return;
+  constexpr int WARPS = PT_THREADS / 32, TILE = PT_THREADS * PT_ITEMS;
+  const size_t sm = (size_t)TILE * 8 + (size_t)WARPS * RADIX * 4 + RADIX * 4 + (WARPS + 1) * 4;
+  smem_optin((const void*)onesweep2_kernel<OS_UCFG>, sm);
+  const u32 tiles = (u32)((m + TILE - 1) / TILE);
+  onesweep2_kernel<OS_UCFG><<<tiles, PT_THREADS, sm, st>>>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch);
+}
 
 void launch_onesweep(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m, u32 shift, const u64* bin_base,
                      u64* lookback, u32* tile_ctr, u32 epoch, cudaStream_t st) {

@@ -42,8 +42,9 @@ size_t fused_temp_bytes(u64 n);
 // is a multiple of 2^dsh)
 void launch_tile_offsets(u64 n, const KeyLayout& L, const u32* tile_hist, void* temp, cudaStream_t st, u32 dsh = 0);
 // gran: the extents pass's granule indices (gout); rec is not read
+// unstable: no stable order within a digit (the bucket path); npass must be 1
 void launch_fused_extract_pass0(const u32* gran, u64 n, const KeyLayout& L, u32 npass, void* temp, u64* kout,
-                                u32* hist, cudaStream_t st, u32 dsh = 0);
+                                u32* hist, cudaStream_t st, u32 dsh = 0, bool unstable = false);
 
 constexpr uint64_t BUCKET_MIN_N = 1ull << 24;  // traces of fewer records keep the full sort
 // k_bucket.cu — bucket path of the sort + compaction (keys sorted by key_hi >> HYB_LO only)
@@ -68,6 +69,9 @@ void launch_bin_base(const u32* hist, u64* bin_base, u32 npass, cudaStream_t st)
 void launch_onesweep(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m, u32 shift, const u64* bin_base,
                      u64* lookback, u32* tile_ctr, u32 epoch, cudaStream_t st);
 u32 sort_tile_keys();
+// the same pass without the stable order (the bucket path): counting atomics give the ranks
+void launch_partition_pass(const u64* kin, u64* kout, u32 m, u32 shift, const u64* bin_base, u64* lookback,
+                           u32* tile_ctr, u32 epoch, cudaStream_t st);
 inline u32 sort_tiles(u64 m) { return (u32)((m + 2047) / 2048); }  // upper bound (smallest tile: 2048 keys)
 // race-list keys: (race key, index) -> histograms for npass digits starting at bit 0
 void launch_hist_keys(const u64* keys, u32 m, u32 npass, u32* hist, cudaStream_t st);

@@ -361,7 +361,7 @@ bool sesa_trace::step_bucket(u64 n, u32 nchunks, u64** comp, u32* m2) {
          launch_tile_offsets(n, L, (const u32*)b_thist2.p, b_ftmp.p, stream, HYB_LO));
   LAUNCH("extract_pass0", 12.0 * n,
          launch_fused_extract_pass0((const u32*)b_keys[0].p, n, L, 1, b_ftmp.p, (u64*)b_keys[1].p, (u32*)b_hist.p,
-                                    stream, HYB_LO));
+                                    stream, HYB_LO, true));
   int cur = 1;
   u32 passes = 1;
   if (*std::max_element(row.begin(), row.end()) != n) {  // digit B not trivial
@@ -378,10 +378,9 @@ bool sesa_trace::step_bucket(u64 n, u32 nchunks, u64** comp, u32* m2) {
       cudaMemsetAsync(b_lookback.p, 0, b_lookback.cap, stream);
       epoch = 1;
     }
-    LAUNCH("onesweep_pass", 16.0 * n,
-           launch_onesweep((u64*)b_keys[1].p, (u64*)b_keys[0].p, nullptr, nullptr, (u32)n,
-                           L.pos_bits + HYB_LO + RADIX_BITS, (u64*)b_binbase.p + RADIX, (u64*)b_lookback.p,
-                           (u32*)b_ctr.p, epoch, stream));
+    LAUNCH("partition_pass", 16.0 * n,
+           launch_partition_pass((u64*)b_keys[1].p, (u64*)b_keys[0].p, (u32)n, L.pos_bits + HYB_LO + RADIX_BITS,
+                                 (u64*)b_binbase.p + RADIX, (u64*)b_lookback.p, (u32*)b_ctr.p, epoch, stream));
     cur = 0;
     passes++;
   }
