@@ -158,6 +158,26 @@ def measured_peak_hbm():
     return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
+def host_info():
+    """CPU model, cores this process may use, RAM (the oracle's hardware, stated beside its numbers)."""
+    model = "unknown"
+    try:
+        for line in subprocess.run(["lscpu"], capture_output=True, text=True).stdout.splitlines():
+            if line.startswith("Model name:"):
+                model = line.split(":", 1)[1].strip()
+    except FileNotFoundError:
+        pass
+    ram = None
+    try:
+        for line in open("/proc/meminfo"):
+            if line.startswith("MemTotal:"):
+                ram = round(int(line.split()[1]) / 2**20, 1)
+    except OSError:
+        pass
+    from oracle import oracle as O
+    return {"cpu": model, "cores": O.nthreads(), "ram_gib": ram}
+
+
 def ncu_traffic(cfg: str, kernel: str):
     """DRAM bytes per launch of `kernel` from the committed ncu --set full summary, if one exists."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -167,15 +187,27 @@ def ncu_traffic(cfg: str, kernel: str):
     return d.get(cfg, {}).get(kernel)
 
 
-def run_cpu_baseline(cfg: str, budget_records: int):
+def run_cpu_baseline(cfg: str, budget_records: int, runs: int = 3):
+    """The oracle as it stands on the host's cores: the T-thread location-partitioned checker at T = every core
+    this process may use (the line's value) and at T = 1, each the median of `runs` runs (the paper averages three
+    runs), on a bounded sample of the same recipe."""
     from oracle import oracle as O
     recs, sample = host_sample(cfg, budget_records)
     c = CONFIGS[cfg]
-    t0 = time.perf_counter()
-    O.check(recs, warp_size=c["ws"], lockstep=c["ls"], granularity=4)
-    dt = time.perf_counter() - t0
-    return {"value": len(recs) / dt / 1e9, "unit": "Grec/s", "cores": 1, "kind": "oracle",
-            "sample": f"{sample}: {len(recs)} records in {dt:.2f} s (oracle_check_grouped, 1 thread)"}
+    hi = host_info()
+    med = {}
+    for T in (1, hi["cores"]):
+        ts = []
+        for _ in range(runs):
+            t0 = time.perf_counter()
+            O.check(recs, warp_size=c["ws"], lockstep=c["ls"], granularity=4, method="partitioned", threads=T)
+            ts.append(time.perf_counter() - t0)
+        med[T] = statistics.median(ts)
+    T = hi["cores"]
+    return {"value": len(recs) / med[T] / 1e9, "unit": "Grec/s", "cores": T, "kind": "oracle",
+            "value_1_thread": len(recs) / med[1] / 1e9, "runs": runs, "host": hi,
+            "sample": f"{sample}: {len(recs)} records; median of {runs} runs {med[T]:.2f} s at {T} threads, "
+                      f"{med[1]:.2f} s at 1 thread (oracle_check_partitioned)"}
 
 
 def reference_arm(args, rank, world):
@@ -186,12 +218,13 @@ def reference_arm(args, rank, world):
     c = CONFIGS[args.config]
     budget = args.ref_records
     recs, sample = host_sample(args.config, budget)
+    hi = host_info()
     for _ in range(args.warmup):
-        O.check(recs[: min(len(recs), 100000)], warp_size=c["ws"], lockstep=c["ls"])
+        O.check(recs[: min(len(recs), 100000)], warp_size=c["ws"], lockstep=c["ls"], method="partitioned")
     times = []
     for _ in range(args.steps):
         t0 = time.perf_counter()
-        O.check(recs, warp_size=c["ws"], lockstep=c["ls"], granularity=4)
+        O.check(recs, warp_size=c["ws"], lockstep=c["ls"], granularity=4, method="partitioned", threads=hi["cores"])
         times.append(time.perf_counter() - t0)
     tot = sum(times)
     value = len(recs) * args.steps / tot / 1e9
@@ -199,7 +232,8 @@ def reference_arm(args, rank, world):
             "warmup": args.warmup, "ms_per_step": 1000 * tot / args.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
             "config": {"workload": c["workload"], "sample": sample}, "impl": "reference",
-            "cpu_baseline": {"value": value, "unit": "Grec/s", "cores": 1, "kind": "oracle", "sample": sample},
+            "cpu_baseline": {"value": value, "unit": "Grec/s", "cores": hi["cores"], "kind": "oracle",
+                             "sample": f"{sample} (oracle_check_partitioned, {hi['cores']} threads)", "host": hi},
             "e2e": {"value": value, "unit": "Grec/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -213,7 +247,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--records", type=int, default=None, help="override the C5 record count")
     ap.add_argument("--cpu-records", type=int, default=1 << 24)
-    ap.add_argument("--ref-records", type=int, default=1 << 23)
+    ap.add_argument("--ref-records", type=int, default=1 << 24)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--benign", action="store_true",
@@ -222,6 +256,15 @@ def main():
                     help="use the NCCL distributed handle even with one rank (exercises the N>1 code path)")
     args = ap.parse_args()
 
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        # not launched by torchrun: start one process per GPU ourselves (same command, under torch.distributed.run)
+        import socket
+        with socket.socket() as so:
+            so.bind(("127.0.0.1", 0))
+            port = so.getsockname()[1]
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+        sys.exit(subprocess.call(cmd))
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
@@ -296,41 +339,63 @@ def main():
         check = bool(got.tobytes() == exp.tobytes())
         log(f"[bench] C5 races {len(got)} (expected {len(exp)}), identical to construction truth: {check}")
 
-    # roofline of the dominant kernel (the onesweep pass): algorithmic bytes / CUDA-event time per launch
+    # roofline of the dominant kernel (most device time in the step): algorithmic bytes / CUDA-event time per launch
     peak, peak_src = measured_peak_hbm()
-    dom = max(kstats, key=lambda k: kstats[k]["ms"]) if kstats else None
+    ours = {k: v for k, v in kstats.items() if k != "alltoall"}
+    dom = max(ours, key=lambda k: ours[k]["ms"]) if ours else None
     roof = None
-    if "onesweep_pass" in kstats and kstats["onesweep_pass"]["launches"]:
-        o = kstats["onesweep_pass"]
+    if dom and ours[dom]["launches"] and ours[dom]["ms"] > 0:
+        o = ours[dom]
         ach = o["bytes"] / (o["ms"] / 1e3) / 1e9
-        trf = ncu_traffic(args.config, "onesweep_pass")
-        roof = {"bound": "hbm", "kernel": "onesweep_pass", "achieved": ach, "peak": peak, "unit": "GB/s",
+        trf = ncu_traffic(args.config, dom)
+        roof = {"bound": "hbm", "kernel": dom, "achieved": ach, "peak": peak, "unit": "GB/s",
                 "frac": ach / peak, "traffic": trf, "bytes_per_launch": o["bytes"] / o["launches"],
                 "ms_per_launch": o["ms"] / o["launches"], "peak_source": peak_src,
-                "share_of_step": o["ms"] / max(1e-9, sum(v["ms"] for v in kstats.values()))}
+                "share_of_step": o["ms"] / max(1e-9, sum(v["ms"] for v in ours.values()))}
     step_bytes = sum(v["bytes"] for v in kstats.values()) / max(1, args.steps)
 
     # end-to-end through the public API with host buffers (H2D of the records + D2H of the race list each step)
+    # end to end through the public API (sesa_race_check_host: every rank's shard from pinned host memory, H2D inside
+    # the call, race list D2H on rank 0), max over ranks
     e2e = None
-    if not args.no_e2e and rank == 0 and world == 1:
+    if not args.no_e2e:
         pinned = torch.empty(n_local * 32, dtype=torch.uint8, pin_memory=True)
         pinned.copy_(recs)
         torch.cuda.synchronize()
         e_steps = max(1, min(args.steps, 3))
-        trace.check_host_ptr(pinned.data_ptr(), n_local)  # warm-up
-        trace.races()
+        trace.check_host_ptr(pinned.data_ptr(), n_local, index_base=base)  # warm-up
+        if rank == 0:
+            trace.races()
+        if pg:
+            pg.barrier()
         t0 = time.perf_counter()
+        nrr = 0
         for _ in range(e_steps):
             trace.check_host_ptr(pinned.data_ptr(), n_local, index_base=base)
-            rr = trace.races()
+            if rank == 0:
+                nrr = len(trace.races())
         dt = time.perf_counter() - t0
-        e2e = {"value": n_total * e_steps / dt / 1e9, "unit": "Grec/s", "h2d_bytes_per_step": n_local * 32,
-               "d2h_bytes_per_step": int(len(rr) * 40), "steps": e_steps}
+        if pg:
+            tt = torch.tensor([dt], device="cuda")
+            pg.all_reduce(tt, op=pg.ReduceOp.MAX)
+            dt = float(tt.item())
+        e2e = {"value": n_total * e_steps / dt / 1e9, "unit": "Grec/s", "h2d_bytes_per_step": n_total * 32,
+               "d2h_bytes_per_step": int(nrr * 40), "steps": e_steps}
         del pinned
+
+    # NVLink: all-to-all bytes this rank sent to other ranks / all-to-all time, against 900 GB/s per direction
+    nvlink = None
+    if world > 1 and "alltoall" in kstats and kstats["alltoall"]["ms"] > 0:
+        a = kstats["alltoall"]
+        gbs = a["bytes"] / (a["ms"] / 1e3) / 1e9
+        nvlink = {"sent_bytes_per_step": a["bytes"] / args.steps, "ms_per_step": a["ms"] / args.steps, "achieved": gbs,
+                  "peak": 900.0, "unit": "GB/s", "frac": gbs / 900.0, "rank": rank}
 
     cpu = None
     if not args.no_cpu and rank == 0 and world == 1:
         cpu = run_cpu_baseline(args.config, args.cpu_records)
+    if world > 1 and not args.no_cpu and rank == 0:
+        cpu = {"skipped": "cpu_baseline is timed on rank 0 at N = 1 only"}
 
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": "Grec/s", "n_gpus": world, "steps": args.steps,
@@ -344,6 +409,7 @@ def main():
                            "sort_bits": info["sort_bits"], "sort_passes": info["sort_passes"],
                            "races": n_races, "crossing_tiles": info["crossing_tiles"],
                            "entries_at_multi_entry_locations": info["n_multi"], "fused_first_pass": bool(info["fused_first_pass"]),
+                           "bucket_path": bool(info["bucket_path"]),
                            "report_benign": bool(args.benign)},
                 "gpu_launches": launches, "roofline": roof,
                 "honesty": {"record_bytes_per_step": n_total * 32, "achieved_gbs_vs_32B_per_record":
@@ -354,7 +420,7 @@ def main():
                 "kernels": {k: dict(launches=v["launches"], ms_per_step=v["ms"] / args.steps,
                                     gbs=(v["bytes"] / (v["ms"] / 1e3) / 1e9) if v["ms"] > 0 else None)
                             for k, v in sorted(kstats.items(), key=lambda kv: -kv[1]["ms"])},
-                "dominant_kernel": dom, "e2e": e2e, "cpu_baseline": cpu, "clocks": clk.summary(),
+                "dominant_kernel": dom, "e2e": e2e, "cpu_baseline": cpu, "clocks": clk.summary(), "nvlink": nvlink,
                 "full_size_check": check}
         print(json.dumps(line), flush=True)
     trace.close()

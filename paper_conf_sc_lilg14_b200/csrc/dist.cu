@@ -257,7 +257,13 @@ static bool exchange(std::vector<sesa_trace*>& ts, Exchanger* ex, const std::vec
     u64 tot = 0;
     for (int p = 0; p < W; p++) rcnt[0][p] = all[(size_t)p * (W + 1) + me], tot += rcnt[0][p];
     if (!t->grow(*recv[0], std::max<u64>(tot, 1) * elem + 64, what)) return false;
-    return ex->alltoall(t, send[0], scnt[0].data(), recv[0]->p, rcnt[0].data(), elem);
+    u64 sent = 0;  // bytes that cross NVLink (to other ranks)
+    for (int p = 0; p < W; p++)
+      if (p != me) sent += scnt[0][p] * elem;
+    t->launch_begin("alltoall");
+    const bool ok2 = ex->alltoall(t, send[0], scnt[0].data(), recv[0]->p, rcnt[0].data(), elem);
+    t->launch_end((double)sent);
+    return ok2;
   }
   // loopback: rank r receives from every s, in source order
   if (getenv("SESA_SYNC_DEBUG"))

@@ -31,3 +31,17 @@ def test_reference_arm_silent_on_other_ranks():
     r = _run({"RANK": "1", "WORLD_SIZE": "2", "LOCAL_RANK": "1"}, "--steps", "1", "--warmup", "1",
              "--ref-records", "100000")
     assert r.returncode == 0 and r.stdout.strip() == ""
+
+
+def test_gpus_flag_self_launches_one_process_per_gpu():
+    """`bench.py --gpus 2` outside torchrun starts torch.distributed.run with 2 ranks itself; rank 0 alone prints
+    (shown here with the CPU reference arm, which needs no GPU)."""
+    env = {k: v for k, v in os.environ.items() if k not in ("RANK", "WORLD_SIZE", "LOCAL_RANK")}
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--gpus", "2",
+                        "--steps", "1", "--warmup", "1", "--ref-records", "100000"],
+                       capture_output=True, text=True, env=env, cwd=ROOT, timeout=300)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [l for l in r.stdout.splitlines() if l.strip().startswith("{")]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["impl"] == "reference" and d["n_gpus"] == 2
