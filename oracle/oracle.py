@@ -33,7 +33,7 @@ REC_DTYPE = np.dtype(
      ("size", "<u2"), ("space", "u1"), ("rw", "u1")], align=True)
 RACE_DTYPE = np.dtype(
     [("addr", "<u8"), ("first", "<u8"), ("second", "<u8"), ("block", "<u4"), ("interval", "<u4"),
-     ("space", "u1"), ("kind", "u1"), ("reserved", "u1", (6,))], align=True)
+     ("space", "u1"), ("kind", "u1"), ("reserved", "u1", (2,)), ("epoch", "<u4")], align=True)
 FLOW_DTYPE = np.dtype(
     [("base", "<u8"), ("bstride", "<i8"), ("tstride", "<i8"), ("istride", "<i8"), ("value_seed", "<u8"),
      ("block_lo", "<u4"), ("block_hi", "<u4"), ("nthreads", "<u4"), ("interval", "<u4"),
@@ -65,6 +65,13 @@ def _load():
             f.restype = ctypes.c_int
         lib.oracle_check_partitioned.argtypes = [P, U64, U64, U32, U32, U32, U32, U32, P, U64, ctypes.POINTER(U64)]
         lib.oracle_check_partitioned.restype = ctypes.c_int
+        for name in ("oracle_check_brute_ep", "oracle_check_grouped_ep"):
+            f = getattr(lib, name)
+            f.argtypes = [P, P, U64, U64, U32, U32, U32, U32, P, U64, ctypes.POINTER(U64)]
+            f.restype = ctypes.c_int
+        lib.oracle_check_partitioned_ep.argtypes = [P, P, U64, U64, U32, U32, U32, U32, U32, P, U64,
+                                                    ctypes.POINTER(U64)]
+        lib.oracle_check_partitioned_ep.restype = ctypes.c_int
         lib.oracle_pair_kind.argtypes = [P, P, U32, U32]
         lib.oracle_pair_kind.restype = ctypes.c_int
         lib.oracle_benign_pair.argtypes = [P, P]
@@ -104,24 +111,38 @@ def nthreads() -> int:
 
 
 def check(records, index_base: int = 0, warp_size: int = 32, lockstep: int = 0, granularity: int = 4,
-          method: str = "grouped", benign: bool = False, threads: int | None = None) -> np.ndarray:
-    """Canonical race list (sorted by (space, block, interval, addr, kind)) of ``records``; with ``benign`` also
-    one kind-3 record per location holding a benign W/W pair (config flags bit 0, oracle_benign_pair).
-    method: "brute" (all pairs), "grouped" (1 thread), "partitioned" (``threads`` threads, default nthreads())."""
+          method: str = "grouped", benign: bool = False, threads: int | None = None, launches=None) -> np.ndarray:
+    """Canonical race list (sorted by (epoch, space, block, interval, addr, kind)) of ``records``; with ``benign``
+    also one kind-3 record per location holding a benign W/W pair (config flags bit 0, oracle_benign_pair).
+    method: "brute" (all pairs), "grouped" (1 thread), "partitioned" (``threads`` threads, default nthreads()).
+    launches: multi-launch trace (NEXT-4): offsets [0, o1, ..., n] — records [o_e, o_{e+1}) ran in kernel launch
+    e; accesses of different launches are ordered and never race (the race's `epoch` field names its launch)."""
     lib = _load()
     r = _as_recs(records)
     T = nthreads() if threads is None else int(threads)
+    ep = None
+    if launches is not None:
+        offs = np.asarray(launches, dtype=np.int64)
+        assert offs[0] == 0 and offs[-1] == len(r) and (np.diff(offs) >= 0).all()
+        ep = np.repeat(np.arange(len(offs) - 1, dtype=np.uint32), np.diff(offs))
     cap = 1024
     while True:
         out = np.zeros(cap, RACE_DTYPE)
         nout = ctypes.c_uint64(0)
-        args = (r.ctypes.data if len(r) else None, len(r), index_base, warp_size, lockstep, granularity,
-                1 if benign else 0)
-        if method == "partitioned":
-            rc = lib.oracle_check_partitioned(*args, T, out.ctypes.data, cap, ctypes.byref(nout))
+        rp = r.ctypes.data if len(r) else None
+        args = (len(r), index_base, warp_size, lockstep, granularity, 1 if benign else 0)
+        if ep is not None:
+            epp = ep.ctypes.data if len(ep) else None
+            if method == "partitioned":
+                rc = lib.oracle_check_partitioned_ep(rp, epp, *args, T, out.ctypes.data, cap, ctypes.byref(nout))
+            else:
+                fn = lib.oracle_check_brute_ep if method == "brute" else lib.oracle_check_grouped_ep
+                rc = fn(rp, epp, *args, out.ctypes.data, cap, ctypes.byref(nout))
+        elif method == "partitioned":
+            rc = lib.oracle_check_partitioned(rp, *args, T, out.ctypes.data, cap, ctypes.byref(nout))
         else:
             fn = lib.oracle_check_brute if method == "brute" else lib.oracle_check_grouped
-            rc = fn(*args, out.ctypes.data, cap, ctypes.byref(nout))
+            rc = fn(rp, *args, out.ctypes.data, cap, ctypes.byref(nout))
         if rc == 7:
             cap = int(nout.value)
             continue

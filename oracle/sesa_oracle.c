@@ -47,7 +47,8 @@ typedef struct {
   uint64_t addr, first, second;
   uint32_t block, interval;
   uint8_t space, kind;
-  uint8_t reserved[6];
+  uint8_t reserved[2];
+  uint32_t epoch; /* kernel launch of the location (multi-launch traces, NEXT-4); 0 for one launch */
 } orace;
 
 typedef struct {
@@ -130,14 +131,18 @@ static void granules(const orec *r, uint32_t G, uint64_t *lo, uint64_t *hi) {
   *hi = (r->addr + (uint64_t)(r->size - 1)) / G;
 }
 
-/* λ of record r at granule g: (SHARED, block, interval, g) or (GLOBAL, -, -, g) */
+/* λ of record r at granule g: (SHARED, block, interval, g) or (GLOBAL, -, -, g), in kernel launch `epoch`.
+ * Multi-launch traces (reading R23): the launches of one trace run one after the
+ * other (each kernel completes before the next starts on the stream), so accesses of different launches are
+ * ordered — like accesses separated by a barrier — and never race: the launch is part of λ. */
 typedef struct {
-  uint32_t space, block, interval;
+  uint32_t epoch, space, block, interval;
   uint64_t g;
 } loc;
 
-static loc loc_of(const orec *r, uint64_t g) {
+static loc loc_of(const orec *r, uint64_t g, uint32_t epoch) {
   loc L;
+  L.epoch = epoch;
   L.space = r->space;
   L.block = r->space == SH ? r->block : NOBI;
   L.interval = r->space == SH ? r->interval : NOBI;
@@ -146,6 +151,7 @@ static loc loc_of(const orec *r, uint64_t g) {
 }
 
 static int loc_cmp(const loc *a, const loc *b) {
+  if (a->epoch != b->epoch) return a->epoch < b->epoch ? -1 : 1;
   if (a->space != b->space) return a->space < b->space ? -1 : 1;
   if (a->block != b->block) return a->block < b->block ? -1 : 1;
   if (a->interval != b->interval) return a->interval < b->interval ? -1 : 1;
@@ -203,6 +209,7 @@ static int emit_sorted(cvec *c, uint32_t G, uint64_t base, orace *out, uint64_t 
       o->interval = c->v[a].L.interval;
       o->space = (uint8_t)c->v[a].L.space;
       o->kind = (uint8_t)c->v[a].kind;
+      o->epoch = c->v[a].L.epoch;
     }
     k++;
   }
@@ -212,8 +219,10 @@ static int emit_sorted(cvec *c, uint32_t G, uint64_t base, orace *out, uint64_t 
 
 /* ---- checker 1: brute force over all pairs ---------------------------------------------------------------
  * return 0 ok, 1 invalid record (*nout = bad index), 2 bad config, 3 no memory, 7 truncated */
-int oracle_check_brute(const orec *r, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls, uint32_t G,
-                       uint32_t flags, orace *out, uint64_t cap, uint64_t *nout) {
+/* epoch: per-record kernel launch (NULL: one launch) */
+#define EP(i) (epoch ? epoch[i] : 0u)
+int oracle_check_brute_ep(const orec *r, const uint32_t *epoch, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls,
+                          uint32_t G, uint32_t flags, orace *out, uint64_t cap, uint64_t *nout) {
   if (!oracle_config_ok(ws, ls, G) || (flags & ~F_BENIGN)) return 2;
   uint64_t bad;
   if (oracle_validate(r, n, &bad)) {
@@ -225,6 +234,7 @@ int oracle_check_brute(const orec *r, uint64_t n, uint64_t base, uint32_t ws, ui
     uint64_t ilo, ihi;
     granules(&r[i], G, &ilo, &ihi);
     for (uint64_t j = i + 1; j < n; j++) {
+      if (EP(i) != EP(j)) continue; /* different launches are ordered (reading R23) */
       if (r[i].space != r[j].space) continue;
       /* shared memory is per block and λ includes the interval */
       if (r[i].space == SH && (r[i].block != r[j].block || r[i].interval != r[j].interval)) continue;
@@ -237,7 +247,7 @@ int oracle_check_brute(const orec *r, uint64_t n, uint64_t base, uint32_t ws, ui
       if (!kind) continue;
       for (uint64_t g = lo; g <= hi; g++) {
         cand x;
-        x.L = loc_of(&r[i], g);
+        x.L = loc_of(&r[i], g, EP(i));
         x.kind = (uint32_t)kind;
         x.i = i;
         x.j = j;
@@ -251,6 +261,11 @@ int oracle_check_brute(const orec *r, uint64_t n, uint64_t base, uint32_t ws, ui
   int rc = emit_sorted(&c, G, base, out, cap, nout);
   free(c.v);
   return rc;
+}
+
+int oracle_check_brute(const orec *r, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls, uint32_t G,
+                       uint32_t flags, orace *out, uint64_t cap, uint64_t *nout) {
+  return oracle_check_brute_ep(r, NULL, n, base, ws, ls, G, flags, out, cap, nout);
 }
 
 /* ---- checker 2: group by location, count partners --------------------------------------------------------- */
@@ -494,20 +509,20 @@ static int process_groups(const orec *r, const entry *e, uint64_t m, uint32_t ws
 /* hash of a location λ (splitmix64 finaliser, the same mix as oracle_expand's value hash) */
 static uint64_t mix(uint64_t x);
 static uint64_t loc_hash(const loc *L) {
-  return mix(mix(mix(((uint64_t)L->space << 32) ^ L->block) ^ L->interval) ^ L->g);
+  return mix(mix(mix(mix(((uint64_t)L->space << 32) ^ L->block) ^ L->interval) ^ L->g) ^ L->epoch);
 }
 
 /* Entries of the records whose location hash falls in partition `part` of `nparts` (nparts == 1: every entry),
  * sorted by (λ, record index); *m_out = count.  NULL on no memory (*m_out = UINT64_MAX). */
-static entry *collect_entries(const orec *r, uint64_t n, uint32_t G, uint32_t part, uint32_t nparts,
-                              uint64_t *m_out) {
+static entry *collect_entries(const orec *r, const uint32_t *epoch, uint64_t n, uint32_t G, uint32_t part,
+                              uint32_t nparts, uint64_t *m_out) {
   uint64_t m = 0;
   for (uint64_t i = 0; i < n; i++) {
     uint64_t lo, hi;
     granules(&r[i], G, &lo, &hi);
     for (uint64_t g = lo; g <= hi; g++) {
       if (nparts > 1) {
-        loc L = loc_of(&r[i], g);
+        loc L = loc_of(&r[i], g, EP(i));
         if (loc_hash(&L) % nparts != part) continue;
       }
       m++;
@@ -523,7 +538,7 @@ static entry *collect_entries(const orec *r, uint64_t n, uint32_t G, uint32_t pa
     uint64_t lo, hi;
     granules(&r[i], G, &lo, &hi);
     for (uint64_t g = lo; g <= hi; g++) {
-      loc L = loc_of(&r[i], g);
+      loc L = loc_of(&r[i], g, EP(i));
       if (nparts > 1 && loc_hash(&L) % nparts != part) continue;
       e[p].L = L;
       e[p].idx = i;
@@ -535,8 +550,8 @@ static entry *collect_entries(const orec *r, uint64_t n, uint32_t G, uint32_t pa
   return e;
 }
 
-int oracle_check_grouped(const orec *r, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls, uint32_t G,
-                         uint32_t flags, orace *out, uint64_t cap, uint64_t *nout) {
+int oracle_check_grouped_ep(const orec *r, const uint32_t *epoch, uint64_t n, uint64_t base, uint32_t ws,
+                            uint32_t ls, uint32_t G, uint32_t flags, orace *out, uint64_t cap, uint64_t *nout) {
   if (!oracle_config_ok(ws, ls, G) || (flags & ~F_BENIGN)) return 2;
   uint64_t bad;
   if (oracle_validate(r, n, &bad)) {
@@ -545,7 +560,7 @@ int oracle_check_grouped(const orec *r, uint64_t n, uint64_t base, uint32_t ws, 
   }
   /* entries = (record, granule) pairs, grouped by location */
   uint64_t m = 0;
-  entry *e = collect_entries(r, n, G, 0, 1, &m);
+  entry *e = collect_entries(r, epoch, n, G, 0, 1, &m);
   if (!e) return 3;
   cvec c = {0, 0, 0};
   int rc = process_groups(r, e, m, ws, ls, flags, 1, &c);
@@ -559,12 +574,18 @@ int oracle_check_grouped(const orec *r, uint64_t n, uint64_t base, uint32_t ws, 
   return rc;
 }
 
+int oracle_check_grouped(const orec *r, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls, uint32_t G,
+                         uint32_t flags, orace *out, uint64_t cap, uint64_t *nout) {
+  return oracle_check_grouped_ep(r, NULL, n, base, ws, ls, G, flags, out, cap, nout);
+}
+
 /* ---- checker 2, T threads: the locations are partitioned by loc_hash mod T (SURVEY §8c.3 "T-thread mode").
  * A race is a property of one location (c.1), so every group lands whole in one partition and each thread
  * runs the unchanged group algorithm on its partition; the candidate lists are concatenated and emitted in
  * the canonical order.  The result is byte-identical to oracle_check_grouped (tests/test_oracle.py).       */
 typedef struct {
   const orec *r;
+  const uint32_t *epoch;
   uint64_t n;
   uint32_t ws, ls, G, flags, part, nparts;
   cvec c;
@@ -574,7 +595,7 @@ typedef struct {
 static void *pworker(void *arg) {
   pjob *j = (pjob *)arg;
   uint64_t m = 0;
-  entry *e = collect_entries(j->r, j->n, j->G, j->part, j->nparts, &m);
+  entry *e = collect_entries(j->r, j->epoch, j->n, j->G, j->part, j->nparts, &m);
   if (!e) {
     j->rc = 3;
     return NULL;
@@ -584,8 +605,9 @@ static void *pworker(void *arg) {
   return NULL;
 }
 
-int oracle_check_partitioned(const orec *r, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls, uint32_t G,
-                             uint32_t flags, uint32_t T, orace *out, uint64_t cap, uint64_t *nout) {
+int oracle_check_partitioned_ep(const orec *r, const uint32_t *epoch, uint64_t n, uint64_t base, uint32_t ws,
+                                uint32_t ls, uint32_t G, uint32_t flags, uint32_t T, orace *out, uint64_t cap,
+                                uint64_t *nout) {
   if (!oracle_config_ok(ws, ls, G) || (flags & ~F_BENIGN)) return 2;
   if (T < 1) T = 1;
   if (T > 1024) T = 1024;
@@ -601,7 +623,7 @@ int oracle_check_partitioned(const orec *r, uint64_t n, uint64_t base, uint32_t 
     return 3;
   }
   for (uint32_t t = 0; t < T; t++) {
-    jobs[t].r = r; jobs[t].n = n; jobs[t].ws = ws; jobs[t].ls = ls; jobs[t].G = G; jobs[t].flags = flags;
+    jobs[t].r = r; jobs[t].epoch = epoch; jobs[t].n = n; jobs[t].ws = ws; jobs[t].ls = ls; jobs[t].G = G; jobs[t].flags = flags;
     jobs[t].part = t; jobs[t].nparts = T;
   }
   for (uint32_t t = 1; t < T; t++)
@@ -626,6 +648,11 @@ int oracle_check_partitioned(const orec *r, uint64_t n, uint64_t base, uint32_t 
   rc = emit_sorted(&c, G, base, out, cap, nout);
   free(c.v);
   return rc;
+}
+
+int oracle_check_partitioned(const orec *r, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls, uint32_t G,
+                             uint32_t flags, uint32_t T, orace *out, uint64_t cap, uint64_t *nout) {
+  return oracle_check_partitioned_ep(r, NULL, n, base, ws, ls, G, flags, T, out, cap, nout);
 }
 
 /* ---- parametric flow instantiation (replace thread id i by j in the race history) ---------- */

@@ -6,7 +6,7 @@ REC_DTYPE = np.dtype(
      ("size", "<u2"), ("space", "u1"), ("rw", "u1")], align=True)
 RACE_DTYPE = np.dtype(
     [("addr", "<u8"), ("first", "<u8"), ("second", "<u8"), ("block", "<u4"), ("interval", "<u4"),
-     ("space", "u1"), ("kind", "u1"), ("reserved", "u1", (6,))], align=True)
+     ("space", "u1"), ("kind", "u1"), ("reserved", "u1", (2,)), ("epoch", "<u4")], align=True)
 FLOW_DTYPE = np.dtype(
     [("base", "<u8"), ("bstride", "<i8"), ("tstride", "<i8"), ("istride", "<i8"), ("value_seed", "<u8"),
      ("block_lo", "<u4"), ("block_hi", "<u4"), ("nthreads", "<u4"), ("interval", "<u4"),

@@ -8,7 +8,8 @@
  * Traces come from the seeded counter-based generator of sesagen (gen_common.h rnd_record); per trace the
  * structure parameters (blocks, threads, intervals, words, spaces, sizes, atomics/writes, values, order) and the
  * config (warp size, lockstep, granularity, benign reporting) are drawn from the trace seed, so that dense
- * collisions, partial overlaps, mixed sizes, all access kinds and every ordering rule are exercised.
+ * collisions, partial overlaps, mixed sizes, all access kinds and every ordering rule are exercised.  Every fifth
+ * trace is a multi-launch trace (NEXT-4) with per-record launch ids (the *_ep checkers).
  *
  *   oracle_sweep <first_seed> <count>      -> prints "traces=... racy=... races=..." and exits 0, or 1 on the
  *                                             first disagreement (printing the seed and config).           */
@@ -23,7 +24,8 @@ typedef struct {
   uint64_t addr, first, second;
   uint32_t block, interval;
   uint8_t space, kind;
-  uint8_t reserved[6];
+  uint8_t reserved[2];
+  uint32_t epoch;
 } race_t;
 
 int oracle_check_brute(const void *r, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls, uint32_t G,
@@ -32,6 +34,13 @@ int oracle_check_grouped(const void *r, uint64_t n, uint64_t base, uint32_t ws, 
                          uint32_t flags, race_t *out, uint64_t cap, uint64_t *nout);
 int oracle_check_partitioned(const void *r, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls, uint32_t G,
                              uint32_t flags, uint32_t T, race_t *out, uint64_t cap, uint64_t *nout);
+int oracle_check_brute_ep(const void *r, const uint32_t *ep, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls,
+                          uint32_t G, uint32_t flags, race_t *out, uint64_t cap, uint64_t *nout);
+int oracle_check_grouped_ep(const void *r, const uint32_t *ep, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls,
+                            uint32_t G, uint32_t flags, race_t *out, uint64_t cap, uint64_t *nout);
+int oracle_check_partitioned_ep(const void *r, const uint32_t *ep, uint64_t n, uint64_t base, uint32_t ws,
+                                uint32_t ls, uint32_t G, uint32_t flags, uint32_t T, race_t *out, uint64_t cap,
+                                uint64_t *nout);
 
 #define CAP 200000
 
@@ -44,6 +53,7 @@ int main(int argc, char **argv) {
   static const uint16_t SZ[][4] = {{4, 4, 4, 4}, {1, 2, 4, 8}, {1, 1, 2, 2}, {4, 8, 16, 3}, {8, 8, 1, 4}};
   race_t *a = malloc(CAP * sizeof(race_t)), *b = malloc(CAP * sizeof(race_t)), *c = malloc(CAP * sizeof(race_t));
   grec *recs = malloc(4096 * sizeof(grec));
+  uint32_t *ep = malloc(4096 * sizeof(uint32_t));
   uint64_t racy = 0, total = 0, kinds[4] = {0, 0, 0, 0};
   for (uint64_t s = s0; s < s0 + cnt; s++) {
     const uint64_t h = gmix(0xC0FFEE00ull ^ s);
@@ -70,9 +80,19 @@ int main(int argc, char **argv) {
     const uint32_t T = 1 + (uint32_t)(s % 4);
     const uint64_t base = (gmix(h + 15) % 5 == 0) ? (1ull << 33) : 0;
     uint64_t na = 0, nb = 0, nc = 0;
-    int ra = oracle_check_brute(recs, R.n, base, WS[k], LS[k], GR[k], flags, a, CAP, &na);
-    int rb = oracle_check_grouped(recs, R.n, base, WS[k], LS[k], GR[k], flags, b, CAP, &nb);
-    int rc = oracle_check_partitioned(recs, R.n, base, WS[k], LS[k], GR[k], flags, T, c, CAP, &nc);
+    int ra, rb, rc;
+    if (s % 5 == 4) { /* multi-launch trace (NEXT-4): per-record launch ids, non-decreasing or arbitrary */
+      const uint32_t E = 1 + (uint32_t)(gmix(h + 16) % 4);
+      for (uint64_t i = 0; i < R.n; i++)
+        ep[i] = (gmix(h + 17) & 1) ? (uint32_t)((i * E) / R.n) : (uint32_t)(gmix(h ^ (i + 99)) % E);
+      ra = oracle_check_brute_ep(recs, ep, R.n, base, WS[k], LS[k], GR[k], flags, a, CAP, &na);
+      rb = oracle_check_grouped_ep(recs, ep, R.n, base, WS[k], LS[k], GR[k], flags, b, CAP, &nb);
+      rc = oracle_check_partitioned_ep(recs, ep, R.n, base, WS[k], LS[k], GR[k], flags, T, c, CAP, &nc);
+    } else {
+      ra = oracle_check_brute(recs, R.n, base, WS[k], LS[k], GR[k], flags, a, CAP, &na);
+      rb = oracle_check_grouped(recs, R.n, base, WS[k], LS[k], GR[k], flags, b, CAP, &nb);
+      rc = oracle_check_partitioned(recs, R.n, base, WS[k], LS[k], GR[k], flags, T, c, CAP, &nc);
+    }
     if (ra || rb || rc || na != nb || na != nc || memcmp(a, b, na * sizeof(race_t)) ||
         memcmp(a, c, na * sizeof(race_t))) {
       printf("MISMATCH seed=%llu n=%llu ws=%u ls=%u G=%u flags=%u T=%u rc=%d/%d/%d races=%llu/%llu/%llu\n",
@@ -87,6 +107,6 @@ int main(int argc, char **argv) {
   printf("traces=%llu racy=%llu races=%llu rw=%llu ww=%llu benign=%llu\n", (unsigned long long)cnt,
          (unsigned long long)racy, (unsigned long long)total, (unsigned long long)kinds[1],
          (unsigned long long)kinds[2], (unsigned long long)kinds[3]);
-  free(a); free(b); free(c); free(recs);
+  free(a); free(b); free(c); free(recs); free(ep);
   return 0;
 }

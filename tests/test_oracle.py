@@ -519,3 +519,52 @@ def test_partitioned_hot_location_parallel_path(benign):
     a = O.check(r, warp_size=32, lockstep=1, benign=benign, method="grouped")
     b = O.check(r, warp_size=32, lockstep=1, benign=benign, method="partitioned", threads=4)
     assert len(a) > 0 and a.tobytes() == b.tobytes()
+
+
+# ------------------------------------------------------------------------------------------------ launches (NEXT-4)
+def test_launch_boundary_orders_accesses():
+    """Reading R23: the launches of one trace run one after another on the stream, so a write in launch 0 and a
+    read of the same word in launch 1 never race, while the same two records in ONE launch (same interval, other
+    threads) do.  Closed form: launch 0 = v[k] written by thread k, launch 1 = v[k] read by thread k + 1."""
+    B = 64
+    r = np.zeros(2 * B, G.REC_DTYPE)
+    r["size"] = 4
+    r["space"] = 0
+    r["addr"][:B] = 4 * np.arange(B)
+    r["thread"][:B] = np.arange(B)
+    r["rw"][:B] = 1
+    r["value_hash"][:B] = np.arange(B) + 1
+    r["addr"][B:] = 4 * np.arange(B)
+    r["thread"][B:] = (np.arange(B) + 1) % B
+    r["rw"][B:] = 0
+    one = O.check(r)
+    assert len(one) == B and set(one["kind"].tolist()) == {RW}
+    for method in ("brute", "grouped", "partitioned"):
+        assert len(O.check(r, launches=[0, B, 2 * B], method=method)) == 0
+    # within each launch the slices are race-free on their own, too
+    assert len(O.check(r[:B])) == 0 and len(O.check(r[B:])) == 0
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_launches_decompose_per_launch(seed):
+    """A multi-launch check is the union of the per-launch checks, each with its records' global indices and its
+    launch number in `epoch` (a consequence of λ including the launch; independent index arithmetic here)."""
+    rng = np.random.default_rng(seed)
+    n = 400 + 50 * seed
+    r = G.random_trace(n, 7000 + seed, threads=30, words=20)
+    cuts = np.sort(rng.integers(0, n, 3))
+    offs = [0, *cuts.tolist(), n]
+    got = O.check(r, launches=offs, warp_size=4, lockstep=seed % 2, benign=seed % 3 == 0)
+    parts = []
+    for e in range(len(offs) - 1):
+        p = O.check(r[offs[e]:offs[e + 1]], index_base=offs[e], warp_size=4, lockstep=seed % 2, benign=seed % 3 == 0)
+        p["epoch"] = e
+        parts.append(p)
+    exp = np.concatenate(parts)
+    assert got.tobytes() == exp.tobytes()
+    # and the F1 race() kernel launched twice: the same 88 races in each launch, indices shifted
+    f = G.f1_race()
+    two = O.check(np.concatenate([f, f]), launches=[0, len(f), 2 * len(f)])
+    a, b = two[two["epoch"] == 0], two[two["epoch"] == 1]
+    assert len(a) == len(b) == 88
+    assert (b["first"] - a["first"] == len(f)).all() and (b["second"] - a["second"] == len(f)).all()
