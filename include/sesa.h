@@ -26,7 +26,7 @@
  *   One race record per (λ, kind), witnessed by the lexicographically smallest (first, second) pair of
  *   record indices (first < second).  The paper's witnesses are "a solution" of the solver; this
  *   library fixes the canonical one so that results are reproducible (reading R12).
- *   Output order: (space, block, interval, addr, kind), SHARED < GLOBAL; a global race has
+ *   Output order: (epoch, space, block, interval, addr, kind), SHARED < GLOBAL; a global race has
  *   block = interval = 0xFFFFFFFF.
  *
  * Conventions
@@ -106,7 +106,8 @@ typedef struct {
                                minimum over all racing pairs at this (location, kind)                      */
   uint32_t block, interval; /* SHARED: the location's block and interval; GLOBAL: 0xFFFFFFFF, 0xFFFFFFFF  */
   uint8_t space, kind;      /* SESA_SPACE_*, SESA_RACE_*                                                   */
-  uint8_t reserved[6];      /* zero                                                                        */
+  uint8_t reserved[2];      /* zero                                                                        */
+  uint32_t epoch;           /* the kernel launch of the location (sesa_race_check_launches); else 0        */
 } sesa_race;
 
 /* Parametric access descriptor: one access of one parametric flow (§IV).  The paper instantiates
@@ -200,6 +201,18 @@ sesa_status sesa_race_check_loopback(const sesa_config *cfg, const sesa_access *
  * when h_records is pageable) inside the call.  This is the end-to-end entry point. */
 sesa_status sesa_race_check_host(sesa_trace *t, const sesa_access *h_records, uint64_t n, uint64_t index_base,
                                  void *cuda_stream);
+
+/* Multi-launch trace (Table IV's per-kernel verdicts P:467 come from programs that launch
+ * several kernels): records [launch_offsets[e], launch_offsets[e+1]) were made by kernel launch e, e < n_launches
+ * (launch_offsets: HOST array of n_launches + 1 entries, launch_offsets[0] = 0, non-decreasing,
+ * launch_offsets[n_launches] = n; else EINVAL).  The launches of one trace run one after another on the stream,
+ * so accesses of different launches are ordered — like accesses separated by a barrier — and never race
+ * (reading R23): the launch is part of the location, and each race record names it in `epoch`.
+ * Record i keeps its global index index_base + i.  The OOB report covers every launch.  Single-GPU handles only
+ * (EINVAL on distributed handles). */
+sesa_status sesa_race_check_launches(sesa_trace *t, const sesa_access *d_records, uint64_t n,
+                                     const uint64_t *launch_offsets, uint32_t n_launches, uint64_t index_base,
+                                     void *cuda_stream);
 
 /* Copy the last race list to host memory (caller-owned).  cap == 0: only *n_races is set.  cap < count:
  * copies cap races, sets *n_races = count, returns SESA_ETRUNC.  ESTATE when no successful check. */

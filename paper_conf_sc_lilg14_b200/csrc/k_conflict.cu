@@ -621,7 +621,8 @@ __device__ void emit_race(const ConflictArgs& a, u64 head_hi, u32 kind, u32 x, u
   r.space = (u8)sp;
   r.kind = (u8)kind;
 #pragma unroll
-  for (int i = 0; i < 6; i++) r.reserved[i] = 0;
+  r.reserved[0] = r.reserved[1] = 0;
+  r.epoch = 0;
   a.races[idx] = r;
   a.race_keys[idx] = (group_of_hi(L, head_hi) << 2) | (kind - 1);  // 2 kind bits: RW, WW, benign WW
   a.race_vals[idx] = idx;
@@ -1012,6 +1013,19 @@ __global__ void cross_emit_kernel(ConflictArgs a, u32 ncross) {
     if (sl.x[k] != ~0ull)  // (position << 32 | entry): report positions
       emit_race(a, sl.head_key >> a.L.pos_bits, (u32)(k + 1), (u32)(sl.x[k] >> 32), (u32)(sl.y[k] >> 32), sl.hblock,
                 sl.hinterval);
+}
+
+__global__ void races_set_epoch_kernel(const RaceOut* __restrict__ in, u32 nr, u32 e, RaceOut* __restrict__ out) {
+  const u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < nr) {
+    RaceOut r = in[i];
+    r.epoch = e;
+    out[i] = r;
+  }
+}
+
+void launch_races_set_epoch(const RaceOut* in, u32 nr, u32 e, RaceOut* out, cudaStream_t st) {
+  if (nr) races_set_epoch_kernel<<<(nr + 255) / 256, 256, 0, st>>>(in, nr, e, out);
 }
 
 u32 conflict_tiles(u64 m) { return (u32)((m + CT_NOM - 1) / CT_NOM); }

@@ -130,7 +130,8 @@ struct ConflictArgs {
 struct RaceOut {  // == sesa_race (40 bytes)
   u64 addr, first, second;
   u32 block, interval;
-  u8 space, kind, reserved[6];
+  u8 space, kind, reserved[2];
+  u32 epoch;  // kernel launch of the location (multi-launch checks); 0 otherwise
 };
 static_assert(sizeof(RaceOut) == 40, "race layout");
 
@@ -147,6 +148,8 @@ void launch_carry(bool exact, const ConflictArgs& a, u32 ntiles, void* temp, cud
 size_t carry_temp_bytes(u32 ntiles);
 void launch_cross_emit(const ConflictArgs& a, u32 ntiles, cudaStream_t st);
 void launch_permute_races(const RaceOut* in, const u32* order, RaceOut* out, u32 nr, cudaStream_t st);
+// out[i] = in[i] with epoch = e (appending one launch's race list to a multi-launch result)
+void launch_races_set_epoch(const RaceOut* in, u32 nr, u32 e, RaceOut* out, cudaStream_t st);
 void race_rekey_launch(const RaceOut* r, u64 n, const KeyLayout& L, u64* keys, u32* vals, cudaStream_t st);
 u32 conflict_tiles(u64 m);
 // benign W/W reporting (k_conflict.cu)

@@ -827,6 +827,57 @@ sesa_status sesa_trace::finish_check(const u64* comp, u32 m2, const Rec* rec, u6
   return SESA_OK;
 }
 
+// ------------------------------------------------------------------------------------------------ launches
+// Multi-launch trace (NEXT-4): the launch is part of every location, so the check is the union of the per-launch
+// checks; their canonical lists concatenated in launch order are the canonical list ordered by (epoch, ...).
+sesa_status sesa_trace::check_launches(const sesa_access* d_rec, u64 n, const u64* offs, u32 nl, u64 index_base) {
+  if (!offs || nl == 0) return begin_check(n), fail(SESA_EINVAL, "launch_offsets is NULL or n_launches is 0"), status;
+  if (offs[0] != 0 || offs[nl] != n)
+    return begin_check(n), fail(SESA_EINVAL, "launch_offsets must start at 0 and end at n"), status;
+  for (u32 e = 0; e < nl; e++)
+    if (offs[e + 1] < offs[e]) return begin_check(n), fail(SESA_EINVAL, "launch_offsets decrease at %u", e), status;
+  u64 total = 0, entries = 0, multi = 0, oob_n = 0, oob_first = ~0ull;
+  u32 kernels = 0;
+  sesa_access oob_rec;
+  memset(&oob_rec, 0, sizeof oob_rec);
+  for (u32 e = 0; e < nl; e++) {
+    const u64 ne = offs[e + 1] - offs[e];
+    const sesa_status st = check_device(ne ? d_rec + offs[e] : d_rec, ne, index_base + offs[e]);
+    if (st != SESA_OK) {
+      err = "launch " + std::to_string(e) + ": " + err;
+      return st;
+    }
+    entries += info.n_entries, multi += info.n_multi, kernels += launches;
+    if (oob.n_oob) {
+      if (oob.first_index < oob_first) oob_first = oob.first_index, oob_rec = oob.first;
+      oob_n += oob.n_oob;
+    }
+    const u32 nr = (u32)n_races;
+    if (nr) {
+      if (!grow_keep(b_lraces, (total + nr) * sizeof(RaceOut), total * sizeof(RaceOut), "launch races")) return status;
+      launches++;
+      launch_races_set_epoch((const RaceOut*)b_races_sorted.p, nr, e, (RaceOut*)b_lraces.p + total, stream);
+      total += nr;
+    }
+  }
+  if (!sync_check("launch races")) return status;
+  // the union becomes the handle's result
+  if (!grow(b_races_sorted, std::max<u64>(total, 1) * sizeof(RaceOut), "sorted races")) return status;
+  if (total && !cuda_ok(cudaMemcpyAsync(b_races_sorted.p, b_lraces.p, total * sizeof(RaceOut), cudaMemcpyDeviceToDevice,
+                                        stream), "launch races"))
+    return status;
+  if (!sync_check("launch races")) return status;
+  n_races = total;
+  info.n_records = n, info.n_entries = entries, info.n_multi = multi, info.n_races = total, info.launches = kernels;
+  memset(&oob, 0, sizeof oob);
+  oob.n_oob = oob_n;
+  oob.first_index = oob_n ? oob_first : ~0ull;
+  oob.first = oob_rec;
+  have_oob = true;
+  have_result = true;
+  return SESA_OK;
+}
+
 // ------------------------------------------------------------------------------------------------ expand
 sesa_status sesa_trace::expand(const sesa_flow* d_flows, u64 nf, sesa_access* d_out, u64 cap, u64* n_out) {
   status = SESA_OK;
@@ -970,6 +1021,15 @@ sesa_status sesa_race_check_host(sesa_trace* t, const sesa_access* h_records, ui
                   "records H2D"))
     return t->status;
   return sesa_race_check(t, (const sesa_access*)t->b_hrec.p, n, index_base, cuda_stream);
+}
+
+sesa_status sesa_race_check_launches(sesa_trace* t, const sesa_access* d_records, uint64_t n,
+                                     const uint64_t* launch_offsets, uint32_t n_launches, uint64_t index_base,
+                                     void* cuda_stream) {
+  if (!t) return SESA_EINVAL;
+  t->stream = (cudaStream_t)cuda_stream;
+  if (t->dist) return t->begin_check(n), t->fail(SESA_EINVAL, "multi-launch checks need a single-GPU handle"), SESA_EINVAL;
+  return t->check_launches(d_records, n, launch_offsets, n_launches, index_base);
 }
 
 sesa_status sesa_races_get(sesa_trace* t, sesa_race* host_out, uint64_t cap, uint64_t* n_races) {

@@ -43,6 +43,7 @@ struct sesa_trace {
   DevBuf b_tflags, b_part, b_carry, b_owner, b_slots, b_cross, b_ccount, b_carrytmp;
   DevBuf b_races, b_rkeys[2], b_rvals[2], b_races_sorted, b_rhist, b_rbase;
   DevBuf b_eoff, b_ecnt, b_ecell, b_hrec, b_dist_races, b_ctmp, b_ctotal, b_thist, b_ftmp, b_thist2, b_btmp2;
+  DevBuf b_lraces;  // multi-launch checks: the races of the launches checked so far
   bool have_thist2 = false;  // extents also wrote the per-tile histograms of the bucket path's first digit
   bool have_thist = false;
   bool hist_from_extents = false;  // fused path: later-digit histograms from the extents' raw granule bytes  // extents wrote per-tile raw digit histograms (fused first pass possible)
@@ -62,7 +63,7 @@ struct sesa_trace {
     std::vector<DevBuf*> v = {&b_summary, &b_hist, &b_binbase, &b_lookback, &b_ctr, &b_cnt, &b_off, &b_temp,
                               &b_tflags, &b_part, &b_carry, &b_owner, &b_slots, &b_cross, &b_ccount, &b_carrytmp,
                               &b_races, &b_races_sorted, &b_rhist, &b_rbase, &b_eoff, &b_ecnt, &b_ecell,
-                              &b_hrec, &b_dist_races, &b_ctmp, &b_ctotal, &b_thist, &b_ftmp, &b_thist2, &b_btmp2, &b_regions,
+                              &b_hrec, &b_dist_races, &b_ctmp, &b_ctotal, &b_thist, &b_ftmp, &b_thist2, &b_btmp2, &b_lraces, &b_regions,
                               &b_bhead, &b_bhscan, &b_bwf, &b_bwscan, &b_bgid, &b_bvk[0], &b_bvk[1], &b_bvi[0],
                               &b_bvi[1], &b_brh, &b_brscan, &b_bder, &b_bdpos, &b_bdj, &b_bslot, &b_btmp};
     for (auto& b : b_keys) v.push_back(&b);
@@ -98,6 +99,8 @@ struct sesa_trace {
   void collect_prof();
   bool make_layout(const sesa::Summary& S, uint64_t n);
   sesa_status check_device(const sesa_access* d_rec, uint64_t n, uint64_t index_base);
+  sesa_status check_launches(const sesa_access* d_rec, uint64_t n, const uint64_t* offs, uint32_t nl,
+                             uint64_t index_base);
   sesa_status finish_check(const uint64_t* comp, uint32_t m2, const sesa::Rec* rec, uint64_t index_base);
   // pipeline steps (shared by the single-GPU and the distributed check)
   void begin_check(uint64_t n);

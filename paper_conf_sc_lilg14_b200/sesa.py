@@ -26,7 +26,7 @@ ACCESS_DTYPE = np.dtype(
      ("size", "<u2"), ("space", "u1"), ("rw", "u1")], align=True)
 RACE_DTYPE = np.dtype(
     [("addr", "<u8"), ("first", "<u8"), ("second", "<u8"), ("block", "<u4"), ("interval", "<u4"),
-     ("space", "u1"), ("kind", "u1"), ("reserved", "u1", (6,))], align=True)
+     ("space", "u1"), ("kind", "u1"), ("reserved", "u1", (2,)), ("epoch", "<u4")], align=True)
 FLOW_DTYPE = np.dtype(
     [("base", "<u8"), ("bstride", "<i8"), ("tstride", "<i8"), ("istride", "<i8"), ("value_seed", "<u8"),
      ("block_lo", "<u4"), ("block_hi", "<u4"), ("nthreads", "<u4"), ("interval", "<u4"),
@@ -64,7 +64,8 @@ class sesa_check_info(ctypes.Structure):
 EXPORTS = ["sesa_trace_create", "sesa_trace_create_dist", "sesa_nccl_unique_id", "sesa_race_check",
            "sesa_race_check_host", "sesa_races_get", "sesa_races_device", "sesa_expand", "sesa_trace_set_profiling",
            "sesa_trace_info", "sesa_trace_kernel_stats", "sesa_trace_destroy", "sesa_status_str", "sesa_last_error",
-           "sesa_abi_version", "sesa_race_check_loopback", "sesa_trace_set_regions", "sesa_oob_get"]
+           "sesa_abi_version", "sesa_race_check_loopback", "sesa_trace_set_regions", "sesa_oob_get",
+           "sesa_race_check_launches"]
 
 _lib = None
 
@@ -84,6 +85,7 @@ def load() -> ctypes.CDLL:
     lib.sesa_nccl_unique_id.argtypes = [P]
     lib.sesa_race_check.argtypes = [P, P, U64, U64, P]
     lib.sesa_race_check_host.argtypes = [P, P, U64, U64, P]
+    lib.sesa_race_check_launches.argtypes = [P, P, U64, P, U32, U64, P]
     lib.sesa_race_check_loopback.argtypes = [ctypes.POINTER(sesa_config), P, P, I, U64, P, PP]
     lib.sesa_races_get.argtypes = [P, P, U64, ctypes.POINTER(U64)]
     lib.sesa_races_device.argtypes = [P, PP, ctypes.POINTER(U64)]
@@ -157,6 +159,16 @@ class Trace:
         st = self.lib.sesa_race_check(self.h, ctypes.c_void_p(ptr), count, index_base, _stream_ptr(stream))
         if st != SESA_OK:
             self._raise(st, "sesa_race_check")
+        return self.n_races()
+
+    def check_launches(self, d_records, n: int, launch_offsets, index_base: int = 0, stream=None) -> int:
+        """Multi-launch trace: records [launch_offsets[e], launch_offsets[e+1]) came from kernel launch e."""
+        ptr, count = _dev_ptr(d_records, n)
+        offs = np.ascontiguousarray(np.asarray(launch_offsets, dtype=np.uint64))
+        st = self.lib.sesa_race_check_launches(self.h, ctypes.c_void_p(ptr), count, ctypes.c_void_p(offs.ctypes.data),
+                                               len(offs) - 1, index_base, _stream_ptr(stream))
+        if st != SESA_OK:
+            self._raise(st, "sesa_race_check_launches")
         return self.n_races()
 
     def check_host(self, h_records: np.ndarray, index_base: int = 0, stream=None) -> int:

@@ -465,3 +465,40 @@ def test_hot_traces_keep_the_full_sort(sesa):
     t.check(dev, n)
     assert t.info()["bucket_path"] == 0
     t.close()
+
+
+# ------------------------------------------------------------------------------------------------ launches (NEXT-4)
+@pytest.mark.parametrize("seed", range(8))
+def test_launches_random(sesa, seed):
+    """sesa_race_check_launches == the oracle's multi-launch check (launch = part of the location, R23): random
+    traces cut into launches (empty ones included), benign reporting on some, one launch large enough to take the
+    fused first pass."""
+    rng = np.random.default_rng(500 + seed)
+    n = [3000, 50000, 120000, 700][seed % 4]
+    r = G.random_trace(n, 9000 + seed, threads=200, blocks=8, words=300 + 40 * seed, sort=seed % 3 != 0)
+    k = int(rng.integers(1, 6))
+    cuts = np.sort(rng.integers(0, n + 1, k - 1)) if k > 1 else np.array([], np.int64)
+    offs = [0, *cuts.tolist(), n]
+    if seed == 5:
+        offs = [0, 0, n // 2, n // 2, n]  # empty launches
+    ls, benign = seed % 2, seed % 3 == 1
+    t = sesa.Trace(32, ls, 4, benign=benign)
+    t.check_launches(sesa.to_device(r), n, offs, index_base=7 * seed)
+    got = t.races()
+    t.close()
+    exp = O.check(r, launches=offs, lockstep=ls, benign=benign, index_base=7 * seed)
+    assert got.tobytes() == exp.tobytes()
+
+
+def test_launches_f1_twice_and_validation(sesa):
+    f = G.f1_race()
+    two = np.concatenate([f, f])
+    t = sesa.Trace(32, 0, 4)
+    t.check_launches(sesa.to_device(two), len(two), [0, len(f), len(two)])
+    got = t.races()
+    assert len(got) == 176 and (got["epoch"] == 0).sum() == 88
+    assert got.tobytes() == O.check(two, launches=[0, len(f), len(two)]).tobytes()
+    for bad in ([0, 10], [1, len(two)], [0, 500, 400, len(two)]):
+        with pytest.raises(sesa.SesaError):
+            t.check_launches(sesa.to_device(two), len(two), bad)
+    t.close()
