@@ -80,8 +80,7 @@ typedef struct {
   uint32_t lockstep;    /* 0 | 1.  1 = exempt intra-warp pairs with a READ (R6-R8)    */
   uint32_t granularity; /* power of two in [1, 4096]: bytes per comparison unit; 1 = exact byte overlap */
   uint32_t flags;       /* SESA_FLAG_* bits; others must be 0.  SESA_FLAG_REPORT_BENIGN: also report benign
-                           W/W locations (kind SESA_RACE_WW_BENIGN); single-GPU handles only
-                           (sesa_trace_create_dist / sesa_race_check_loopback return SESA_EINVAL)          */
+                           W/W locations (kind SESA_RACE_WW_BENIGN), on single-GPU and distributed handles  */
 } sesa_config;
 
 /* One concrete access: the paper's race-state entry `c ? r|w(a)` of one thread.

@@ -490,6 +490,7 @@ static sesa_status dist_check(std::vector<sesa_trace*>& ts, std::vector<RankIO>&
                                                                           m2[r], (Rec*)B.rec_entry.p);
     }
     ok = t->step_conflict(comp[r], m2[r], nullptr, 0, (const Rec*)B.rec_entry.p, base0) &&
+         t->step_benign(comp[r], m2[r], nullptr, base0, (const Rec*)B.rec_entry.p) &&
          t->grow(t->b_races_sorted, (size_t)std::max((u32)t->n_races, 1u) * sizeof(RaceOut), "sorted races") &&
          t->step_race_sort((u32)t->n_races, (RaceOut*)t->b_races.p, (u64*)t->b_rkeys[0].p, (u32*)t->b_rvals[0].p,
                            (u64*)t->b_rkeys[1].p, (u32*)t->b_rvals[1].p, (RaceOut*)t->b_races_sorted.p) &&
@@ -566,7 +567,6 @@ sesa_status sesa_trace_create_dist(const sesa_config* cfg, int rank, int world, 
   if (!out) return SESA_EINVAL;
   *out = nullptr;
   if (!uid || world < 1 || world > 8 || rank < 0 || rank >= world) return SESA_EINVAL;
-  if (cfg && (cfg->flags & SESA_FLAG_REPORT_BENIGN)) return SESA_EINVAL;  // benign reporting: single GPU in v1
   sesa_trace* t = nullptr;
   sesa_status s = sesa_trace_create(cfg, &t);
   if (s != SESA_OK) return s;
@@ -592,7 +592,6 @@ sesa_status sesa_race_check_loopback(const sesa_config* cfg, const sesa_access* 
                                      int world, uint64_t index_base, void* stream, sesa_trace** out) {
   if (!out || !offs || world < 1 || world > 8) return SESA_EINVAL;
   *out = nullptr;
-  if (cfg && (cfg->flags & SESA_FLAG_REPORT_BENIGN)) return SESA_EINVAL;  // benign reporting: single GPU in v1
   std::vector<sesa_trace*> ts(world, nullptr);
   for (int r = 0; r < world; r++) {
     sesa_status s = sesa_trace_create(cfg, &ts[r]);

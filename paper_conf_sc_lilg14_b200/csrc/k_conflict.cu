@@ -1245,18 +1245,25 @@ void launch_permute_races(const RaceOut* in, const u32* order, RaceOut* out, u32
 // original, and because a run lists its entries in original position order the derived witness maps to the
 // original lexicographic minimum; the minimum over a location's runs is taken with one atomicMin per race.
 
+// The record of compacted entry j: by its position (single GPU), or entry-aligned (rec_entry: the distributed
+// check fetches the records of multi-entry locations from their owner ranks, dist.cu)
+__device__ __forceinline__ Rec benign_rec(const Rec* rec, const Rec* rec_entry, const KeyLayout& L, const u64* comp,
+                                          u32 j) {
+  return rec_entry ? load_rec(rec_entry + j) : load_rec(rec + pos_of(L, comp[j]));
+}
+
 // head flag (first entry of a location run) and plain-write flag of every compacted entry
-__global__ void benign_mark_kernel(const u64* __restrict__ comp, u32 m2, KeyLayout L, const Rec* __restrict__ rec,
+__global__ void benign_mark_kernel(const u64* __restrict__ comp, u32 m2, KeyLayout L, const Rec* __restrict__ rec, const Rec* __restrict__ rec_entry,
                                    u32* __restrict__ head, u32* __restrict__ wflag) {
   const u32 j = blockIdx.x * blockDim.x + threadIdx.x;
   if (j >= m2) return;
   const u64 k = comp[j];
   head[j] = (j == 0 || group_of_hi(L, k >> L.pos_bits) != group_of_hi(L, comp[j - 1] >> L.pos_bits)) ? 1u : 0u;
-  wflag[j] = rec[pos_of(L, k)].rw == RW_WRITE ? 1u : 0u;  // rw byte of the record (byte 31)
+  wflag[j] = benign_rec(rec, rec_entry, L, comp, j).rw == RW_WRITE ? 1u : 0u;
 }
 
 // plain writes -> (value, entry) pairs at their exclusive write rank; location ordinal of every entry
-__global__ void benign_gather_kernel(const u64* __restrict__ comp, u32 m2, KeyLayout L, const Rec* __restrict__ rec,
+__global__ void benign_gather_kernel(const u64* __restrict__ comp, u32 m2, KeyLayout L, const Rec* __restrict__ rec, const Rec* __restrict__ rec_entry,
                                      const u32* __restrict__ head, const u32* __restrict__ hscan,
                                      const u32* __restrict__ wflag, const u32* __restrict__ wscan,
                                      u32* __restrict__ gid, u64* __restrict__ vkey, u32* __restrict__ vidx) {
@@ -1264,23 +1271,23 @@ __global__ void benign_gather_kernel(const u64* __restrict__ comp, u32 m2, KeyLa
   if (j >= m2) return;
   gid[j] = hscan[j] + head[j] - 1;
   if (wflag[j]) {
-    vkey[wscan[j]] = rec[pos_of(L, comp[j])].vh;
+    vkey[wscan[j]] = benign_rec(rec, rec_entry, L, comp, j).vh;
     vidx[wscan[j]] = j;
   }
 }
 
 // sort keys of the plain-write list (entry vidx[i]): 0 = original position, 1 = value hash, 2 = location ordinal
-__global__ void benign_keys_kernel(const u64* __restrict__ comp, KeyLayout L, const Rec* __restrict__ rec,
+__global__ void benign_keys_kernel(const u64* __restrict__ comp, KeyLayout L, const Rec* __restrict__ rec, const Rec* __restrict__ rec_entry,
                                    const u32* __restrict__ vidx, u32 m3, const u32* __restrict__ gid, int what,
                                    u64* __restrict__ keys) {
   const u32 i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= m3) return;
   const u32 j = vidx[i];
-  keys[i] = what == 2 ? (u64)gid[j] : what == 0 ? (u64)pos_of(L, comp[j]) : rec[pos_of(L, comp[j])].vh;
+  keys[i] = what == 2 ? (u64)gid[j] : what == 0 ? (u64)pos_of(L, comp[j]) : benign_rec(rec, rec_entry, L, comp, j).vh;
 }
 
 // run heads of the (location, value) order
-__global__ void benign_runs_kernel(const u64* __restrict__ comp, KeyLayout L, const Rec* __restrict__ rec,
+__global__ void benign_runs_kernel(const u64* __restrict__ comp, KeyLayout L, const Rec* __restrict__ rec, const Rec* __restrict__ rec_entry,
                                    const u32* __restrict__ gid, const u32* __restrict__ order, u32 m3,
                                    u32* __restrict__ rhead) {
   const u32 i = blockIdx.x * blockDim.x + threadIdx.x;
@@ -1289,14 +1296,14 @@ __global__ void benign_runs_kernel(const u64* __restrict__ comp, KeyLayout L, co
   bool h = i == 0;
   if (!h) {
     const u32 jp = order[i - 1];
-    h = gid[jp] != gid[j] || rec[pos_of(L, comp[jp])].vh != rec[pos_of(L, comp[j])].vh;
+    h = gid[jp] != gid[j] || benign_rec(rec, rec_entry, L, comp, jp).vh != benign_rec(rec, rec_entry, L, comp, j).vh;
   }
   rhead[i] = h ? 1u : 0u;
 }
 
 // derived trace: record i = plain write of entry order[i] at location (its space, block, interval, run id) with
 // granularity 1 and the distinct value i + 1; dpos[i] = original position, dj[i] = entry
-__global__ void benign_derive_kernel(const u64* __restrict__ comp, KeyLayout L, const Rec* __restrict__ rec,
+__global__ void benign_derive_kernel(const u64* __restrict__ comp, KeyLayout L, const Rec* __restrict__ rec, const Rec* __restrict__ rec_entry,
                                      const u32* __restrict__ order, const u32* __restrict__ rhead,
                                      const u32* __restrict__ rscan, u32 m3, Rec* __restrict__ out,
                                      u32* __restrict__ dpos, u32* __restrict__ dj) {
@@ -1304,7 +1311,7 @@ __global__ void benign_derive_kernel(const u64* __restrict__ comp, KeyLayout L, 
   if (i >= m3) return;
   const u32 j = order[i];
   const u32 p = pos_of(L, comp[j]);
-  const Rec r = load_rec(rec + p);
+  const Rec r = benign_rec(rec, rec_entry, L, comp, j);
   Rec d = r;
   d.addr = rscan[i] + rhead[i] - 1;
   d.vh = (u64)i + 1;
@@ -1336,33 +1343,33 @@ __global__ void benign_emit_kernel(ConflictArgs a, const RaceOut* __restrict__ c
   const unsigned long long v = ((unsigned long long)dpos[x.first] << 32) | dpos[x.second];
   if (slot[gid[j]] != v) return;  // pairs are unique per location: exactly one child race wins
   const u64 k = a.keys[j];
-  const Rec r = load_rec(a.rec + pos_of(a.L, k));
+  const Rec r = benign_rec(a.rec, a.rec_entry, a.L, a.keys, j);
   emit_race(a, k >> a.L.pos_bits, KIND_WWB, dpos[x.first], dpos[x.second], r.block, r.interval);
 }
 
-void launch_benign_mark(const u64* comp, u32 m2, const KeyLayout& L, const Rec* rec, u32* head, u32* wflag,
+void launch_benign_mark(const u64* comp, u32 m2, const KeyLayout& L, const Rec* rec, const Rec* rec_entry, u32* head, u32* wflag,
                         cudaStream_t st) {
-  if (m2) benign_mark_kernel<<<(m2 + 255) / 256, 256, 0, st>>>(comp, m2, L, rec, head, wflag);
+  if (m2) benign_mark_kernel<<<(m2 + 255) / 256, 256, 0, st>>>(comp, m2, L, rec, rec_entry, head, wflag);
 }
-void launch_benign_gather(const u64* comp, u32 m2, const KeyLayout& L, const Rec* rec, const u32* head,
+void launch_benign_gather(const u64* comp, u32 m2, const KeyLayout& L, const Rec* rec, const Rec* rec_entry, const u32* head,
                           const u32* hscan, const u32* wflag, const u32* wscan, u32* gid, u64* vkey, u32* vidx,
                           cudaStream_t st) {
   if (m2)
-    benign_gather_kernel<<<(m2 + 255) / 256, 256, 0, st>>>(comp, m2, L, rec, head, hscan, wflag, wscan, gid, vkey,
+    benign_gather_kernel<<<(m2 + 255) / 256, 256, 0, st>>>(comp, m2, L, rec, rec_entry, head, hscan, wflag, wscan, gid, vkey,
                                                            vidx);
 }
-void launch_benign_keys(const u64* comp, const KeyLayout& L, const Rec* rec, const u32* vidx, u32 m3, const u32* gid,
+void launch_benign_keys(const u64* comp, const KeyLayout& L, const Rec* rec, const Rec* rec_entry, const u32* vidx, u32 m3, const u32* gid,
                         int what, u64* keys, cudaStream_t st) {
-  if (m3) benign_keys_kernel<<<(m3 + 255) / 256, 256, 0, st>>>(comp, L, rec, vidx, m3, gid, what, keys);
+  if (m3) benign_keys_kernel<<<(m3 + 255) / 256, 256, 0, st>>>(comp, L, rec, rec_entry, vidx, m3, gid, what, keys);
 }
-void launch_benign_runs(const u64* comp, const KeyLayout& L, const Rec* rec, const u32* gid, const u32* order,
+void launch_benign_runs(const u64* comp, const KeyLayout& L, const Rec* rec, const Rec* rec_entry, const u32* gid, const u32* order,
                         u32 m3, u32* rhead, cudaStream_t st) {
-  if (m3) benign_runs_kernel<<<(m3 + 255) / 256, 256, 0, st>>>(comp, L, rec, gid, order, m3, rhead);
+  if (m3) benign_runs_kernel<<<(m3 + 255) / 256, 256, 0, st>>>(comp, L, rec, rec_entry, gid, order, m3, rhead);
 }
-void launch_benign_derive(const u64* comp, const KeyLayout& L, const Rec* rec, const u32* order, const u32* rhead,
+void launch_benign_derive(const u64* comp, const KeyLayout& L, const Rec* rec, const Rec* rec_entry, const u32* order, const u32* rhead,
                           const u32* rscan, u32 m3, Rec* out, u32* dpos, u32* dj, cudaStream_t st) {
   if (m3)
-    benign_derive_kernel<<<(m3 + 255) / 256, 256, 0, st>>>(comp, L, rec, order, rhead, rscan, m3, out, dpos, dj);
+    benign_derive_kernel<<<(m3 + 255) / 256, 256, 0, st>>>(comp, L, rec, rec_entry, order, rhead, rscan, m3, out, dpos, dj);
 }
 void launch_benign_min_emit(const ConflictArgs& a, const RaceOut* cr, u32 nc, const u32* dpos, const u32* dj,
                             const u32* gid, unsigned long long* slot, cudaStream_t st) {

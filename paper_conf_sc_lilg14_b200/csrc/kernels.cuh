@@ -153,16 +153,16 @@ void launch_races_set_epoch(const RaceOut* in, u32 nr, u32 e, RaceOut* out, cuda
 void race_rekey_launch(const RaceOut* r, u64 n, const KeyLayout& L, u64* keys, u32* vals, cudaStream_t st);
 u32 conflict_tiles(u64 m);
 // benign W/W reporting (k_conflict.cu)
-void launch_benign_mark(const u64* comp, u32 m2, const KeyLayout& L, const Rec* rec, u32* head, u32* wflag,
+void launch_benign_mark(const u64* comp, u32 m2, const KeyLayout& L, const Rec* rec, const Rec* rec_entry, u32* head, u32* wflag,
                         cudaStream_t st);
-void launch_benign_gather(const u64* comp, u32 m2, const KeyLayout& L, const Rec* rec, const u32* head,
+void launch_benign_gather(const u64* comp, u32 m2, const KeyLayout& L, const Rec* rec, const Rec* rec_entry, const u32* head,
                           const u32* hscan, const u32* wflag, const u32* wscan, u32* gid, u64* vkey, u32* vidx,
                           cudaStream_t st);
-void launch_benign_keys(const u64* comp, const KeyLayout& L, const Rec* rec, const u32* vidx, u32 m3, const u32* gid,
+void launch_benign_keys(const u64* comp, const KeyLayout& L, const Rec* rec, const Rec* rec_entry, const u32* vidx, u32 m3, const u32* gid,
                         int what, u64* keys, cudaStream_t st);
-void launch_benign_runs(const u64* comp, const KeyLayout& L, const Rec* rec, const u32* gid, const u32* order,
+void launch_benign_runs(const u64* comp, const KeyLayout& L, const Rec* rec, const Rec* rec_entry, const u32* gid, const u32* order,
                         u32 m3, u32* rhead, cudaStream_t st);
-void launch_benign_derive(const u64* comp, const KeyLayout& L, const Rec* rec, const u32* order, const u32* rhead,
+void launch_benign_derive(const u64* comp, const KeyLayout& L, const Rec* rec, const Rec* rec_entry, const u32* order, const u32* rhead,
                           const u32* rscan, u32 m3, Rec* out, u32* dpos, u32* dj, cudaStream_t st);
 void launch_benign_min_emit(const ConflictArgs& a, const struct RaceOut* cr, u32 nc, const u32* dpos, const u32* dj,
                             const u32* gid, unsigned long long* slot, cudaStream_t st);

@@ -595,14 +595,14 @@ bool sesa_trace::sort_kv(u64* k0, u32* v0, u64* k1, u32* v1, u32 n, u32 bits, in
 
 // step 5b (flags bit 0): benign W/W records, appended to the unsorted race list
 // (k_conflict.cu "benign W/W" has the method).  n_races grows by the locations holding a benign pair.
-bool sesa_trace::step_benign(const u64* comp, u32 m2, const Rec* rec, u64 index_base) {
+bool sesa_trace::step_benign(const u64* comp, u32 m2, const Rec* rec, u64 index_base, const Rec* rec_entry) {
   if (!(cfg.flags & SESA_FLAG_REPORT_BENIGN) || m2 < 2) return true;
   const KeyLayout& L = layout;
   if (!grow(b_bhead, (size_t)m2 * 4, "benign") || !grow(b_bhscan, (size_t)m2 * 4, "benign") ||
       !grow(b_bwf, (size_t)m2 * 4, "benign") || !grow(b_bwscan, (size_t)m2 * 4, "benign") ||
       !grow(b_bgid, (size_t)m2 * 4, "benign") || !grow(b_temp, scan_u32_temp_bytes(m2), "scan"))
     return false;
-  LAUNCH("benign_mark", 16.0 * m2, launch_benign_mark(comp, m2, L, rec, (u32*)b_bhead.p, (u32*)b_bwf.p, stream));
+  LAUNCH("benign_mark", 16.0 * m2, launch_benign_mark(comp, m2, L, rec, rec_entry, (u32*)b_bhead.p, (u32*)b_bwf.p, stream));
   LAUNCH("scan", 8.0 * m2, launch_scan_exclusive_u32((u32*)b_bhead.p, (u32*)b_bhscan.p, m2, b_temp.p, stream));
   LAUNCH("scan", 8.0 * m2, launch_scan_exclusive_u32((u32*)b_bwf.p, (u32*)b_bwscan.p, m2, b_temp.p, stream));
   u32 tail[4];
@@ -621,7 +621,7 @@ bool sesa_trace::step_benign(const u64* comp, u32 m2, const Rec* rec, u64 index_
       !grow(b_temp, scan_u32_temp_bytes(m3), "scan"))
     return false;
   LAUNCH("benign_gather", 24.0 * m2,
-         launch_benign_gather(comp, m2, L, rec, (const u32*)b_bhead.p, (const u32*)b_bhscan.p, (const u32*)b_bwf.p,
+         launch_benign_gather(comp, m2, L, rec, rec_entry, (const u32*)b_bhead.p, (const u32*)b_bhscan.p, (const u32*)b_bwf.p,
                               (const u32*)b_bwscan.p, (u32*)b_bgid.p, (u64*)b_bvk[0].p, (u32*)b_bvi[0].p, stream));
   // stable LSD passes over the plain-write list -> (location, value, position) order.  Entries of a location
   // are already position-ordered unless global keys carry (block, interval) below the granule (input not in
@@ -629,12 +629,12 @@ bool sesa_trace::step_benign(const u64* comp, u32 m2, const Rec* rec, u64 index_
   int w = 0;
   if (L.lowG != 0) {
     LAUNCH("benign_keys", 12.0 * m3,
-           launch_benign_keys(comp, L, rec, (const u32*)b_bvi[0].p, m3, (const u32*)b_bgid.p, 0, (u64*)b_bvk[0].p,
+           launch_benign_keys(comp, L, rec, rec_entry, (const u32*)b_bvi[0].p, m3, (const u32*)b_bgid.p, 0, (u64*)b_bvk[0].p,
                               stream));
     if (!sort_kv((u64*)b_bvk[0].p, (u32*)b_bvi[0].p, (u64*)b_bvk[1].p, (u32*)b_bvi[1].p, m3, L.pos_bits, &w))
       return false;
     LAUNCH("benign_keys", 40.0 * m3,
-           launch_benign_keys(comp, L, rec, (const u32*)b_bvi[w].p, m3, (const u32*)b_bgid.p, 1, (u64*)b_bvk[w].p,
+           launch_benign_keys(comp, L, rec, rec_entry, (const u32*)b_bvi[w].p, m3, (const u32*)b_bgid.p, 1, (u64*)b_bvk[w].p,
                               stream));
   }
   int w1 = 0;
@@ -642,7 +642,7 @@ bool sesa_trace::step_benign(const u64* comp, u32 m2, const Rec* rec, u64 index_
     return false;
   w ^= w1;
   LAUNCH("benign_keys", 12.0 * m3,
-         launch_benign_keys(comp, L, rec, (const u32*)b_bvi[w].p, m3, (const u32*)b_bgid.p, 2, (u64*)b_bvk[w].p,
+         launch_benign_keys(comp, L, rec, rec_entry, (const u32*)b_bvi[w].p, m3, (const u32*)b_bgid.p, 2, (u64*)b_bvk[w].p,
                             stream));
   u32 gbits = 0;
   while (gbits < 32 && (1ull << gbits) < ngroups) gbits++;
@@ -651,10 +651,10 @@ bool sesa_trace::step_benign(const u64* comp, u32 m2, const Rec* rec, u64 index_
     return false;
   const u32* order = (const u32*)(w2 ? b_bvi[w ^ 1].p : b_bvi[w].p);
   LAUNCH("benign_runs", 24.0 * m3,
-         launch_benign_runs(comp, L, rec, (const u32*)b_bgid.p, order, m3, (u32*)b_brh.p, stream));
+         launch_benign_runs(comp, L, rec, rec_entry, (const u32*)b_bgid.p, order, m3, (u32*)b_brh.p, stream));
   LAUNCH("scan", 8.0 * m3, launch_scan_exclusive_u32((u32*)b_brh.p, (u32*)b_brscan.p, m3, b_temp.p, stream));
   LAUNCH("benign_derive", 80.0 * m3,
-         launch_benign_derive(comp, L, rec, order, (const u32*)b_brh.p, (const u32*)b_brscan.p, m3, (Rec*)b_bder.p,
+         launch_benign_derive(comp, L, rec, rec_entry, order, (const u32*)b_brh.p, (const u32*)b_brscan.p, m3, (Rec*)b_bder.p,
                               (u32*)b_bdpos.p, (u32*)b_bdj.p, stream));
   if (!sync_check("benign derive")) return false;
   // the derived trace: plain writes with distinct values at (location, value) runs, granularity 1
@@ -686,6 +686,7 @@ bool sesa_trace::step_benign(const u64* comp, u32 m2, const Rec* rec, u64 index_
   A.keys = comp;
   A.m = m2;
   A.rec = rec;
+  A.rec_entry = rec_entry;
   A.L = layout;
   A.race_count = (u32*)b_ccount.p;
   A.race_keys = (u64*)b_rkeys[0].p;

@@ -118,7 +118,8 @@ struct sesa_trace {
   bool step_conflict(const uint64_t* comp, uint32_t m2, const sesa::Rec* rec, uint32_t rec_pos_base,
                      const sesa::Rec* rec_entry, uint64_t index_base);
   bool sort_kv(uint64_t* k0, uint32_t* v0, uint64_t* k1, uint32_t* v1, uint32_t n, uint32_t bits, int* which);
-  bool step_benign(const uint64_t* comp, uint32_t m2, const sesa::Rec* rec, uint64_t index_base);
+  bool step_benign(const uint64_t* comp, uint32_t m2, const sesa::Rec* rec, uint64_t index_base,
+                   const sesa::Rec* rec_entry = nullptr);
   bool step_race_sort(uint32_t nr, const sesa::RaceOut* races, uint64_t* rk0, uint32_t* rv0, uint64_t* rk1,
                       uint32_t* rv1, sesa::RaceOut* out);
   sesa_status expand(const sesa_flow* d_flows, uint64_t nf, sesa_access* d_out, uint64_t cap, uint64_t* n_out);

@@ -129,7 +129,7 @@ class Trace:
     def __init__(self, warp_size: int = 32, lockstep: int = 0, granularity: int = 4, *, dist=None,
                  benign: bool = False):
         lib = load()
-        # flags bit 0 = SESA_FLAG_REPORT_BENIGN: also report benign W/W locations as kind 3 (single GPU)
+        # flags bit 0 = SESA_FLAG_REPORT_BENIGN: also report benign W/W locations as kind 3
         self.cfg = sesa_config(warp_size, lockstep, granularity, 1 if benign else 0)
         h = ctypes.c_void_p()
         if dist is None:
@@ -264,10 +264,11 @@ def _dev_ptr(x, n):
     return x.data_ptr(), (n if n is not None else nbytes // 32)
 
 
-def check_loopback(d_records, offs, warp_size=32, lockstep=0, granularity=4, index_base=0, stream=None):
+def check_loopback(d_records, offs, warp_size=32, lockstep=0, granularity=4, index_base=0, stream=None,
+                   benign=False):
     """Distributed check with len(offs)-1 virtual ranks on this GPU; returns the merged race array."""
     lib = load()
-    cfg = sesa_config(warp_size, lockstep, granularity, 0)
+    cfg = sesa_config(warp_size, lockstep, granularity, SESA_FLAG_REPORT_BENIGN if benign else 0)
     o = (ctypes.c_uint64 * len(offs))(*offs)
     h = ctypes.c_void_p()
     ptr, _ = _dev_ptr(d_records, offs[-1])

@@ -357,9 +357,17 @@ def test_benign_bfs_shape(sesa):
     assert 2 not in set(got["kind"].tolist()) and 3 in set(got["kind"].tolist())
 
 
-def test_benign_flag_rejected_when_distributed(sesa):
-    with pytest.raises(sesa.SesaError):
-        sesa.Trace(32, 0, 4, dist=(0, 1, bytes(128)), benign=True)
+def test_benign_flag_on_distributed_handles(sesa):
+    """Benign W/W reporting on the distributed path (records of multi-entry locations fetched from their owner
+    ranks): loopback with 1-5 virtual ranks == the single-GPU list == the oracle's."""
+    for W, seed in ((1, 0), (2, 1), (3, 2), (5, 3)):
+        r = G.random_trace(6000, 600 + seed, threads=80, words=150, values=2, write_frac=0.6, atomic_frac=0.1,
+                           sort=seed != 2)
+        exp = O.check(r, benign=True, lockstep=seed % 2)
+        assert (exp["kind"] == 3).any()
+        offs = [len(r) * k // W for k in range(W + 1)]
+        got = sesa.check_loopback(sesa.to_device(r), offs, lockstep=seed % 2, benign=True)
+        assert got.tobytes() == exp.tobytes()
 
 
 # ------------------------------------------------------------------------------------------------ OOB (NEXT-1)
