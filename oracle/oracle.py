@@ -41,6 +41,8 @@ FLOW_DTYPE = np.dtype(
      ("fkind", "<u4"), ("fc", "<u4"), ("fm", "<u4"), ("count", "<u4"),
      ("size", "<u2"), ("space", "u1"), ("rw", "u1"), ("flags", "<u4")], align=True)
 
+EXT_DTYPE = np.dtype([("pc", "<u4"), ("div", "<u4")])  # precise warp model extension (NEXT-3)
+
 _lib = None
 
 
@@ -72,6 +74,12 @@ def _load():
         lib.oracle_check_partitioned_ep.argtypes = [P, P, U64, U64, U32, U32, U32, U32, U32, P, U64,
                                                     ctypes.POINTER(U64)]
         lib.oracle_check_partitioned_ep.restype = ctypes.c_int
+        for name in ("oracle_check_warp_brute", "oracle_check_warp_grouped"):
+            f = getattr(lib, name)
+            f.argtypes = [P, P, U64, U64, U32, U32, U32, P, U64, ctypes.POINTER(U64)]
+            f.restype = ctypes.c_int
+        lib.oracle_pair_kind_warp.argtypes = [P, P, P, P, U32, U32]
+        lib.oracle_pair_kind_warp.restype = ctypes.c_int
         lib.oracle_pair_kind.argtypes = [P, P, U32, U32]
         lib.oracle_pair_kind.restype = ctypes.c_int
         lib.oracle_benign_pair.argtypes = [P, P]
@@ -143,6 +151,28 @@ def check(records, index_base: int = 0, warp_size: int = 32, lockstep: int = 0, 
         else:
             fn = lib.oracle_check_brute if method == "brute" else lib.oracle_check_grouped
             rc = fn(rp, *args, out.ctypes.data, cap, ctypes.byref(nout))
+        if rc == 7:
+            cap = int(nout.value)
+            continue
+        if rc != 0:
+            raise OracleError(rc, int(nout.value))
+        return out[: nout.value].copy()
+
+
+def check_warp(records, ext, index_base: int = 0, warp_size: int = 32, lockstep: int = 1, granularity: int = 4,
+               method: str = "grouped") -> np.ndarray:
+    """Precise warp model (NEXT-3, oracle_pair_kind_warp): ``ext`` holds one {pc, div} per record."""
+    lib = _load()
+    r = _as_recs(records)
+    e = np.ascontiguousarray(np.asarray(ext).view(EXT_DTYPE) if np.asarray(ext).dtype != EXT_DTYPE else ext)
+    assert len(e) == len(r)
+    fn = lib.oracle_check_warp_brute if method == "brute" else lib.oracle_check_warp_grouped
+    cap = 1024
+    while True:
+        out = np.zeros(cap, RACE_DTYPE)
+        nout = ctypes.c_uint64(0)
+        rc = fn(r.ctypes.data if len(r) else None, e.ctypes.data if len(e) else None, len(r), index_base, warp_size,
+                lockstep, granularity, out.ctypes.data, cap, ctypes.byref(nout))
         if rc == 7:
             cap = int(nout.value)
             continue

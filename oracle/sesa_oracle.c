@@ -24,6 +24,8 @@
  *                          property of one location, c.1), each thread runs the unchanged group algorithm on its
  *                          partition; byte-identical output (SURVEY §8c.3 "T-thread mode"; full-size parity).
  * With flag F_BENIGN all three also report benign W/W pairs as a third kind (oracle_benign_pair).
+ * Precise warp model (NEXT-3): oracle_pair_kind_warp + oracle_check_warp_brute / oracle_check_warp_grouped, on
+ * records with an instruction / divergence extension.
  * They agree on every input (tests/test_oracle.py); the GPU path uses neither method (it uses per-run
  * min/max summaries), so agreement of the GPU with this oracle is not circular.
  *
@@ -653,6 +655,123 @@ int oracle_check_partitioned_ep(const orec *r, const uint32_t *epoch, uint64_t n
 int oracle_check_partitioned(const orec *r, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls, uint32_t G,
                              uint32_t flags, uint32_t T, orace *out, uint64_t cap, uint64_t *nout) {
   return oracle_check_partitioned_ep(r, NULL, n, base, ws, ls, G, flags, T, out, cap, nout);
+}
+
+/* ---- precise warp model (reading R24) -------------------------------------------
+ * Each record carries an extension {pc, div}: pc = the static instruction that made the access; div = 0 when the
+ * thread's warp was convergent at that instruction, else (branch instance << 1 | side) of the divergent branch
+ * region containing it (innermost region).  P:281 (§IV-B): "threads within a warp are executed in a lock-step
+ * manner: two intra-warp threads can race only if they simultaneously write to the same shared variable at the
+ * same instruction.  In case of divergence, we execute the two sides sequentially ... the executor has to
+ * enumerate both orders"; P:87 (§II): the divergent read/write of race() is a race "no matter whether t1 and t2
+ * are within a warp".  So, with lockstep on, for two threads of one warp (same block, same interval):
+ *   - on the two sides of one divergent branch instance: both orders of the sides occur -> unordered, rules 1-4
+ *     and 6 decide as without lockstep ("both orders");
+ *   - otherwise lockstep orders them, except two writes at the same instruction (simultaneous): then a
+ *     W/W race (benign filter 6 still applies); every other intra-warp pair is exempt.
+ * With lockstep off the extension is ignored.  With every pc equal and every div 0 this is exactly rule (5) of
+ * oracle_pair_kind (intra-warp pairs with a read exempt, intra-warp writes kept).                            */
+typedef struct {
+  uint32_t pc, div;
+} oext;
+
+int oracle_pair_kind_warp(const orec *r, const orec *s, const oext *er, const oext *es, uint32_t ws, uint32_t ls) {
+  if (r->block == s->block && r->thread == s->thread) return 0;                        /* (1) */
+  if (r->rw == RD && s->rw == RD) return 0;                                            /* (2) */
+  if (r->rw == AT && s->rw == AT) return 0;                                            /* (3) */
+  if (r->space == GL && r->block == s->block && r->interval != s->interval) return 0;   /* (4) */
+  int kind = (r->rw == RD || s->rw == RD) ? K_RW : K_WW;
+  if (ls && r->block == s->block && r->interval == s->interval && r->thread / ws == s->thread / ws) {
+    const int divergent = er->div != 0 && es->div != 0 && (er->div >> 1) == (es->div >> 1) &&
+                          (er->div & 1) != (es->div & 1);
+    if (!divergent && (kind == K_RW || er->pc != es->pc)) return 0;                    /* (5') */
+  }
+  if (r->rw == WR && s->rw == WR && r->value_hash == s->value_hash) return 0;           /* (6) */
+  return kind;
+}
+
+/* brute force over all pairs (the definition); returns like oracle_check_brute (no benign flag) */
+int oracle_check_warp_brute(const orec *r, const oext *ext, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls,
+                            uint32_t G, orace *out, uint64_t cap, uint64_t *nout) {
+  if (!oracle_config_ok(ws, ls, G)) return 2;
+  uint64_t bad;
+  if (oracle_validate(r, n, &bad)) {
+    *nout = bad;
+    return 1;
+  }
+  cvec c = {0, 0, 0};
+  for (uint64_t i = 0; i < n; i++) {
+    uint64_t ilo, ihi;
+    granules(&r[i], G, &ilo, &ihi);
+    for (uint64_t j = i + 1; j < n; j++) {
+      if (r[i].space != r[j].space) continue;
+      if (r[i].space == SH && (r[i].block != r[j].block || r[i].interval != r[j].interval)) continue;
+      uint64_t jlo, jhi;
+      granules(&r[j], G, &jlo, &jhi);
+      uint64_t lo = ilo > jlo ? ilo : jlo, hi = ihi < jhi ? ihi : jhi;
+      if (lo > hi) continue;
+      const int kind = oracle_pair_kind_warp(&r[i], &r[j], &ext[i], &ext[j], ws, ls);
+      if (!kind) continue;
+      for (uint64_t g = lo; g <= hi; g++) {
+        cand x;
+        x.L = loc_of(&r[i], g, 0);
+        x.kind = (uint32_t)kind;
+        x.i = i;
+        x.j = j;
+        if (cpush(&c, x)) {
+          free(c.v);
+          return 3;
+        }
+      }
+    }
+  }
+  int rc = emit_sorted(&c, G, base, out, cap, nout);
+  free(c.v);
+  return rc;
+}
+
+/* grouped by location, then every pair of the group in lexicographic (i, j) order: the first racing pair of a
+ * kind is its witness (O(sum of group sizes squared); an independent organisation of the same definition) */
+int oracle_check_warp_grouped(const orec *r, const oext *ext, uint64_t n, uint64_t base, uint32_t ws, uint32_t ls,
+                              uint32_t G, orace *out, uint64_t cap, uint64_t *nout) {
+  if (!oracle_config_ok(ws, ls, G)) return 2;
+  uint64_t bad;
+  if (oracle_validate(r, n, &bad)) {
+    *nout = bad;
+    return 1;
+  }
+  uint64_t m = 0;
+  entry *e = collect_entries(r, NULL, n, G, 0, 1, &m);
+  if (!e) return 3;
+  cvec c = {0, 0, 0};
+  int rc = 0;
+  for (uint64_t a = 0; a < m && !rc;) {
+    uint64_t b = a + 1;
+    while (b < m && loc_cmp(&e[b].L, &e[a].L) == 0) b++;
+    int found[3] = {0, 0, 0};
+    for (uint64_t x = a; x < b && !(found[K_RW] && found[K_WW]) && !rc; x++)
+      for (uint64_t y = x + 1; y < b; y++) {
+        const uint64_t i = e[x].idx, j = e[y].idx;
+        const int kind = oracle_pair_kind_warp(&r[i], &r[j], &ext[i], &ext[j], ws, ls);
+        if (!kind || found[kind]) continue;
+        found[kind] = 1;
+        cand cd;
+        cd.L = e[a].L;
+        cd.kind = (uint32_t)kind;
+        cd.i = i;
+        cd.j = j;
+        if (cpush(&c, cd)) { rc = 3; break; }
+      }
+    a = b;
+  }
+  free(e);
+  if (rc) {
+    free(c.v);
+    return rc;
+  }
+  rc = emit_sorted(&c, G, base, out, cap, nout);
+  free(c.v);
+  return rc;
 }
 
 /* ---- parametric flow instantiation (replace thread id i by j in the race history) ---------- */

@@ -568,3 +568,70 @@ def test_launches_decompose_per_launch(seed):
     a, b = two[two["epoch"] == 0], two[two["epoch"] == 1]
     assert len(a) == len(b) == 88
     assert (b["first"] - a["first"] == len(f)).all() and (b["second"] - a["second"] == len(f)).all()
+
+
+# ------------------------------------------------------------------------------------------------ precise warps (NEXT-3)
+def test_f1_precise_warp_model():
+    """race() under the precise warp model (reading R24: P:281 + P:87).  Interval 0 (`v[t] = v[(t+1)%B]`) is
+    convergent: an intra-warp read (pc 0) precedes the other thread's write (pc 1) in lockstep, so only the two
+    inter-warp pairs race (v[0]: reader 63 / writer 0; v[32]: reader 31 / writer 32).  Interval 1 diverges in
+    every warp: the read side and the write side run in either order, so every RW pair races "no matter whether
+    t1 and t2 are within a warp", and the two writers of v[j] write at the same instruction: all of
+    interval 1 is as without lockstep.  26 races, from the hand-derived lockstep-0 set (f1_closed_form)."""
+    r, e = G.f1_race(), G.f1_race_ext()
+    full = f1_closed_form(ls=False)
+    exp = {x for x in full if x[2] == 1} | {x for x in full if x[2] == 0 and x[3] in (0, 4 * 32)}
+    assert len(exp) == 26
+    for method in ("brute", "grouped"):
+        got = set(tuples(O.check_warp(r, e, lockstep=1, method=method)))
+        assert got == exp, method
+    # lockstep off: the extension is ignored
+    assert O.check_warp(r, e, lockstep=0).tobytes() == O.check(r, lockstep=0).tobytes()
+
+
+def test_precise_warp_generic_example():
+    """Fig. 1's Generic example shape and P:281: two threads of one warp writing one word."""
+    def pair(div0, div1, pc0, pc1, v0=1, v1=2, t1=5, rw1=1):
+        r = np.zeros(2, G.REC_DTYPE)
+        r["size"], r["space"] = 4, 0
+        r["thread"] = [3, t1]
+        r["rw"] = [1, rw1]
+        r["value_hash"] = [v0, v1]
+        e = np.zeros(2, O.EXT_DTYPE)
+        e["pc"], e["div"] = [pc0, pc1], [div0, div1]
+        return [(int(x["kind"])) for x in O.check_warp(r, e, lockstep=1, method="brute")]
+    I = 7 << 1
+    assert pair(I | 0, I | 1, 10, 11) == [WW]        # the two sides of one branch: both orders occur (P:281)
+    assert pair(I | 0, I | 0, 10, 11) == []          # same side, two instructions: ordered by lockstep
+    assert pair(I | 0, I | 0, 10, 10) == [WW]        # same instruction: a simultaneous write (P:281)
+    assert pair(0, 0, 10, 10, v0=4, v1=4) == []      # ... of one value: benign (rule 6)
+    assert pair(I | 0, (I + 2) | 1, 10, 11) == []    # sides of two different branch instances: ordered
+    assert pair(I | 0, I | 1, 10, 11, rw1=0) == [RW]  # a read on the other side (P:87)
+    assert pair(0, 0, 10, 10, rw1=0) == []           # convergent read/write: ordered by lockstep
+    assert pair(0, 0, 10, 11, t1=40) == [WW]         # another warp: the plain rules
+
+
+def test_precise_warp_reduces_to_coarse_and_f4():
+    # one instruction and no divergence anywhere = rule (5) of the coarse model (intra-warp reads exempt,
+    # intra-warp writes kept)
+    for seed in range(20):
+        r = G.random_trace(150, 4000 + seed, threads=64, words=12)
+        z = np.zeros(len(r), O.EXT_DTYPE)
+        for ws in (32, 4):
+            assert O.check_warp(r, z, warp_size=ws).tobytes() == O.check(r, warp_size=ws, lockstep=1).tobytes()
+    # histo_prescan (Fig. 8): SUM(32)'s write of Avg[17] happens before SUM(16)'s divergent read in lockstep
+    f, fe = G.f4_histo_prescan(), G.f4_histo_prescan_ext()
+    assert len(O.check_warp(f, fe)) == 0
+    assert len(O.check_warp(f, fe, warp_size=1)) == 32  # warp size 1 (P:91): the real RW race of P:567
+
+
+@pytest.mark.parametrize("cfg", CONFIGS)
+def test_precise_warp_brute_equals_grouped(cfg):
+    for seed in range(40):
+        n = 1 + (seed * 13) % 120
+        r = G.random_trace(n, 5000 + seed, threads=8 + seed % 70, blocks=1 + seed % 3, words=6 + seed % 20,
+                           sort=seed % 3 != 0)
+        e = G.random_ext(n, seed, npc=1 + seed % 4, ninst=1 + seed % 3)
+        a = O.check_warp(r, e, warp_size=cfg["ws"], lockstep=cfg["ls"], granularity=cfg["G"], method="brute")
+        b = O.check_warp(r, e, warp_size=cfg["ws"], lockstep=cfg["ls"], granularity=cfg["G"], method="grouped")
+        assert a.tobytes() == b.tobytes(), (cfg, seed)
