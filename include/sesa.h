@@ -213,6 +213,28 @@ sesa_status sesa_race_check_launches(sesa_trace *t, const sesa_access *d_records
                                      const uint64_t *launch_offsets, uint32_t n_launches, uint64_t index_base,
                                      void *cuda_stream);
 
+/* Precise warp model.  P:281 (§IV-B): "two intra-warp threads can race only if they
+ * simultaneously write to the same shared variable at the same instruction.  In case of divergence, we execute
+ * the two sides sequentially ... [and] enumerate both orders"; P:87 (§II): a divergent read/write races "no matter
+ * whether t1 and t2 are within a warp".  Every record gets an extension: pc = the static instruction of the
+ * access; div = 0 if its warp was convergent there, else (branch instance << 1 | side) of the innermost divergent
+ * branch region containing it (instances numbered by the producer, unique per warp execution of a branch).
+ * With cfg.lockstep = 1, two records of different threads in one block, interval and warp race only if
+ *   (a) they lie on the two sides of one branch instance (same div >> 1, different div & 1, both != 0) — then by
+ *       rules (1)-(4) and (6) as without lockstep — or
+ *   (b) both write (plain or atomic, not both atomic) at the same pc — a W/W race, benign filter (6) applies;
+ * this replaces rule (5) (reading R24).  Pairs of different warps or blocks follow the ordinary rules.
+ * With every pc equal and every div 0 the model is rule (5).  lockstep = 0: d_ext is ignored.
+ * d_ext: DEVICE array of n sesa_access_ext (8 bytes each), borrowed like d_records.  Single-GPU handles, no
+ * SESA_FLAG_REPORT_BENIGN (EINVAL). */
+typedef struct {
+  uint32_t pc;   /* static instruction id                                                                     */
+  uint32_t div;  /* 0 = convergent; else (branch instance << 1) | side                                        */
+} sesa_access_ext;
+
+sesa_status sesa_race_check_warp(sesa_trace *t, const sesa_access *d_records, const sesa_access_ext *d_ext,
+                                 uint64_t n, uint64_t index_base, void *cuda_stream);
+
 /* Copy the last race list to host memory (caller-owned).  cap == 0: only *n_races is set.  cap < count:
  * copies cap races, sets *n_races = count, returns SESA_ETRUNC.  ESTATE when no successful check. */
 sesa_status sesa_races_get(sesa_trace *t, sesa_race *host_out, uint64_t cap, uint64_t *n_races);

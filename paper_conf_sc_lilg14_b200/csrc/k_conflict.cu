@@ -384,8 +384,11 @@ __device__ __forceinline__ void tile_window(const ConflictArgs& a, u32 tile, u64
 
 // the record of entry e (sorted/compacted entry index) with key `key`: by position in the caller's record array
 // (single GPU), or entry-aligned records fetched from the owner ranks (distributed check)
+// (tdiv > 1: the identity of a record is its warp thread / tdiv — the inter-warp half of the precise warp model)
 __device__ __forceinline__ Rec rec_at(const ConflictArgs& a, u64 e, u64 key) {
-  return a.rec_entry ? load_rec(a.rec_entry + e) : load_rec(a.rec + (pos_of(a.L, key) - a.rec_pos_base));
+  Rec r = a.rec_entry ? load_rec(a.rec_entry + e) : load_rec(a.rec + (pos_of(a.L, key) - a.rec_pos_base));
+  if (a.tdiv > 1) r.thread /= a.tdiv;
+  return r;
 }
 
 // Loads keys, computes group membership and gathers records.  Returns false if no entry of the tile has a
@@ -620,7 +623,6 @@ __device__ void emit_race(const ConflictArgs& a, u64 head_hi, u32 kind, u32 x, u
   r.interval = sp == SP_SHARED ? hi_ : NOBI;
   r.space = (u8)sp;
   r.kind = (u8)kind;
-#pragma unroll
   r.reserved[0] = r.reserved[1] = 0;
   r.epoch = 0;
   a.races[idx] = r;
@@ -1026,6 +1028,121 @@ __global__ void races_set_epoch_kernel(const RaceOut* __restrict__ in, u32 nr, u
 
 void launch_races_set_epoch(const RaceOut* in, u32 nr, u32 e, RaceOut* out, cudaStream_t st) {
   if (nr) races_set_epoch_kernel<<<(nr + 255) / 256, 256, 0, st>>>(in, nr, e, out);
+}
+
+// ------------------------------------------------------------------------------------------------ precise warps
+// SURVEY §8f NEXT-3 (reading R24).  With lockstep on, records extended with {pc, div}:
+// intra-warp pairs race only on the two sides of one divergent branch instance (any kind) or as two writes at
+// one instruction (W/W).  The per-location witness is the lexicographic minimum over the union of
+//   (A) the pairs of different warps (or blocks): the ordinary conflict tiles with identity = warp (tdiv = ws,
+//       lockstep off) — two records of one warp then look like one thread (rule 1) — and
+//   (B) the pairs inside one (location, block, interval, warp) group, checked pair by pair (such groups hold at
+//       most 32 threads' accesses): entries regrouped by a sort on (run ordinal, hash of (block, interval, warp)).
+// Both halves fold their pairs into one atomicMin slot per (run, kind) as (position << 32 | position).
+__device__ __forceinline__ u32 warp_hash(u32 b, u32 i, u32 w) {
+  return (u32)(sesa_mix(((u64)b << 32) ^ ((u64)i << 20) ^ (u64)w) >> 32);
+}
+
+// run heads and the (block, interval, warp) hash of every compacted entry
+__global__ void warp_key_kernel(const u64* __restrict__ comp, u32 m2, KeyLayout L, const Rec* __restrict__ rec,
+                                u32 ws, u32* __restrict__ head, u32* __restrict__ hkey) {
+  const u32 j = blockIdx.x * blockDim.x + threadIdx.x;
+  if (j >= m2) return;
+  const u64 k = comp[j];
+  head[j] = (j == 0 || group_of_hi(L, k >> L.pos_bits) != group_of_hi(L, comp[j - 1] >> L.pos_bits)) ? 1u : 0u;
+  const Rec r = load_rec(rec + pos_of(L, k));
+  hkey[j] = warp_hash(r.block, r.interval, r.thread / ws);
+}
+
+__global__ void warp_key2_kernel(const u32* __restrict__ head, const u32* __restrict__ hscan,
+                                 const u32* __restrict__ hkey, u32 m2, u64* __restrict__ key2, u32* __restrict__ val) {
+  const u32 j = blockIdx.x * blockDim.x + threadIdx.x;
+  if (j >= m2) return;
+  key2[j] = ((u64)(hscan[j] + head[j] - 1) << 32) | hkey[j];
+  val[j] = j;
+}
+
+// (B): thread p checks its entry against the later entries of its (run, hash) segment, pair by pair
+__global__ void warp_pairs_kernel(const u64* __restrict__ comp, KeyLayout L, const Rec* __restrict__ rec,
+                                  const uint2* __restrict__ ext, u32 ws, const u64* __restrict__ key2,
+                                  const u32* __restrict__ order, u32 m2, unsigned long long* __restrict__ slot) {
+  const u32 p = blockIdx.x * blockDim.x + threadIdx.x;
+  if (p >= m2) return;
+  const u64 kk = key2[p];
+  if (p + 1 >= m2 || key2[p + 1] != kk) return;
+  const u32 x = order[p], px = pos_of(L, comp[x]);
+  const Rec X = load_rec(rec + px);
+  const uint2 ex = ext[px];
+  const u32 gid = (u32)(kk >> 32);
+  for (u32 q = p + 1; q < m2 && key2[q] == kk; q++) {
+    const u32 py = pos_of(L, comp[order[q]]);
+    const Rec Y = load_rec(rec + py);
+    if (X.block != Y.block || X.interval != Y.interval || X.thread / ws != Y.thread / ws) continue;  // hash twin
+    if (X.thread == Y.thread) continue;                                                      // (1)
+    if (X.rw == RW_READ && Y.rw == RW_READ) continue;                                        // (2)
+    if (X.rw == RW_ATOMIC && Y.rw == RW_ATOMIC) continue;                                    // (3)
+    const u32 kind = (X.rw == RW_READ || Y.rw == RW_READ) ? KIND_RW : KIND_WW;
+    const uint2 ey = ext[py];
+    const bool divergent = ex.y != 0 && ey.y != 0 && (ex.y >> 1) == (ey.y >> 1) && ((ex.y ^ ey.y) & 1u);
+    if (!divergent && (kind == KIND_RW || ex.x != ey.x)) continue;                           // (5')
+    if (X.rw == RW_WRITE && Y.rw == RW_WRITE && X.vh == Y.vh) continue;                      // (6)
+    const u32 lo = min(px, py), hi = max(px, py);
+    atomicMin(&slot[2 * (u64)gid + kind - 1], ((unsigned long long)lo << 32) | hi);
+  }
+}
+
+// (A): the inter-warp races of the ordinary conflict tiles, folded into the slots of their runs
+__global__ void warp_fold_kernel(const u64* __restrict__ rkeys, const RaceOut* __restrict__ races, u32 nr,
+                                 const u64* __restrict__ comp, u32 m2, KeyLayout L, const u32* __restrict__ hscan,
+                                 u64 index_base, unsigned long long* __restrict__ slot) {
+  const u32 r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= nr) return;
+  const u64 hk = rkeys[r] >> 2;
+  const u32 kind = (u32)(rkeys[r] & 3) + 1;
+  u32 lo = 0, hi = m2;  // first entry of the run: lower bound of its group key
+  while (lo < hi) {
+    const u32 mid = (lo + hi) >> 1;
+    if (group_of_hi(L, comp[mid] >> L.pos_bits) < hk) lo = mid + 1;
+    else hi = mid;
+  }
+  const RaceOut x = races[r];
+  atomicMin(&slot[2 * (u64)hscan[lo] + kind - 1],
+            ((unsigned long long)(x.first - index_base) << 32) | (unsigned long long)(x.second - index_base));
+}
+
+__global__ void warp_emit_kernel(ConflictArgs a, const u32* __restrict__ head, const u32* __restrict__ hscan,
+                                 const unsigned long long* __restrict__ slot) {
+  const u32 j = blockIdx.x * blockDim.x + threadIdx.x;
+  if (j >= a.m || !head[j]) return;
+  const u32 gid = hscan[j];
+  const u64 k = a.keys[j];
+  for (u32 kind = KIND_RW; kind <= KIND_WW; kind++) {
+    const unsigned long long v = slot[2 * (u64)gid + kind - 1];
+    if (v == ~0ull) continue;
+    const Rec r = load_rec(a.rec + pos_of(a.L, k));
+    emit_race(a, k >> a.L.pos_bits, kind, (u32)(v >> 32), (u32)v, r.block, r.interval);
+  }
+}
+
+void launch_warp_keys(const u64* comp, u32 m2, const KeyLayout& L, const Rec* rec, u32 ws, u32* head, u32* hkey,
+                      cudaStream_t st) {
+  if (m2) warp_key_kernel<<<(m2 + 255) / 256, 256, 0, st>>>(comp, m2, L, rec, ws, head, hkey);
+}
+void launch_warp_key2(const u32* head, const u32* hscan, const u32* hkey, u32 m2, u64* key2, u32* val, cudaStream_t st) {
+  if (m2) warp_key2_kernel<<<(m2 + 255) / 256, 256, 0, st>>>(head, hscan, hkey, m2, key2, val);
+}
+void launch_warp_pairs(const u64* comp, const KeyLayout& L, const Rec* rec, const void* ext, u32 ws, const u64* key2,
+                       const u32* order, u32 m2, unsigned long long* slot, cudaStream_t st) {
+  if (m2)
+    warp_pairs_kernel<<<(m2 + 255) / 256, 256, 0, st>>>(comp, L, rec, (const uint2*)ext, ws, key2, order, m2, slot);
+}
+void launch_warp_fold(const u64* rkeys, const RaceOut* races, u32 nr, const u64* comp, u32 m2, const KeyLayout& L,
+                      const u32* hscan, u64 index_base, unsigned long long* slot, cudaStream_t st) {
+  if (nr) warp_fold_kernel<<<(nr + 255) / 256, 256, 0, st>>>(rkeys, races, nr, comp, m2, L, hscan, index_base, slot);
+}
+void launch_warp_emit(const ConflictArgs& a, const u32* head, const u32* hscan, const unsigned long long* slot,
+                      cudaStream_t st) {
+  if (a.m) warp_emit_kernel<<<(a.m + 255) / 256, 256, 0, st>>>(a, head, hscan, slot);
 }
 
 u32 conflict_tiles(u64 m) { return (u32)((m + CT_NOM - 1) / CT_NOM); }

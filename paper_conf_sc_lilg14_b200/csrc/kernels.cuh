@@ -125,6 +125,7 @@ struct ConflictArgs {
   struct Slot* slots;     // per owner tile
   u64 index_base;
   u32 phase;  // modes 2/3: 0 = every crossing piece, 1 = pieces starting a run (crossing out), 2 = the rest
+  u32 tdiv;   // > 1: a record's identity is thread / tdiv (precise warp model, inter-warp half)
 };
 
 struct RaceOut {  // == sesa_race (40 bytes)
@@ -166,6 +167,17 @@ void launch_benign_derive(const u64* comp, const KeyLayout& L, const Rec* rec, c
                           const u32* rscan, u32 m3, Rec* out, u32* dpos, u32* dj, cudaStream_t st);
 void launch_benign_min_emit(const ConflictArgs& a, const struct RaceOut* cr, u32 nc, const u32* dpos, const u32* dj,
                             const u32* gid, unsigned long long* slot, cudaStream_t st);
+
+// precise warp model (k_conflict.cu): slots [2 * runs] of (position << 32 | position) minima
+void launch_warp_keys(const u64* comp, u32 m2, const KeyLayout& L, const Rec* rec, u32 ws, u32* head, u32* hkey,
+                      cudaStream_t st);
+void launch_warp_key2(const u32* head, const u32* hscan, const u32* hkey, u32 m2, u64* key2, u32* val, cudaStream_t st);
+void launch_warp_pairs(const u64* comp, const KeyLayout& L, const Rec* rec, const void* ext, u32 ws, const u64* key2,
+                       const u32* order, u32 m2, unsigned long long* slot, cudaStream_t st);
+void launch_warp_fold(const u64* rkeys, const struct RaceOut* races, u32 nr, const u64* comp, u32 m2,
+                      const KeyLayout& L, const u32* hscan, u64 index_base, unsigned long long* slot, cudaStream_t st);
+void launch_warp_emit(const ConflictArgs& a, const u32* head, const u32* hscan, const unsigned long long* slot,
+                      cudaStream_t st);
 
 // k_compact.cu — keep only entries of locations touched >= 2 times (order preserved); *total = count
 size_t compact_temp_bytes(u64 m);

@@ -491,8 +491,9 @@ bool sesa_trace::step_conflict(const u64* comp, u32 m2, const Rec* rec, u32 rec_
     A.rec_entry = rec_entry;
     A.rec_pos_base = rec_pos_base;
     A.L = layout;
-    A.ws = cfg.warp_size;
-    A.ls = cfg.lockstep;
+    A.ws = conflict_tdiv > 1 ? 1u : cfg.warp_size;
+    A.ls = conflict_tdiv > 1 ? 0u : cfg.lockstep;
+    A.tdiv = conflict_tdiv;
     A.race_count = (u32*)b_ccount.p;
     A.cross_count = (u32*)b_ccount.p + 1;
     A.need_exact = (u32*)b_ccount.p + 2;
@@ -705,6 +706,75 @@ bool sesa_trace::step_benign(const u64* comp, u32 m2, const Rec* rec, u64 index_
   return true;
 }
 
+// step 5' (precise warp model; k_conflict.cu "precise warps" has the method): the
+// inter-warp half by the conflict tiles with identity = warp, the intra-warp half pair by pair inside each
+// (location, block, interval, warp) group, both folded into per-(run, kind) minimum slots, then emitted
+bool sesa_trace::step_warp_model(const u64* comp, u32 m2, const Rec* rec, u64 index_base) {
+  const u32 ws = cfg.warp_size;
+  // warp size 1: no two threads share a warp, the ordinary check is the model
+  conflict_tdiv = ws > 1 ? ws : 0;
+  const bool ok = step_conflict(comp, m2, rec, 0, nullptr, index_base);
+  conflict_tdiv = 0;
+  if (!ok || ws == 1 || m2 < 2) return ok;
+  const u32 nA = (u32)n_races;
+  const KeyLayout& L = layout;
+  if (!grow(b_bhead, (size_t)m2 * 4, "warp") || !grow(b_bhscan, (size_t)m2 * 4, "warp") ||
+      !grow(b_bwf, (size_t)m2 * 4, "warp") || !grow(b_bvk[0], (size_t)m2 * 8, "warp") ||
+      !grow(b_bvk[1], (size_t)m2 * 8, "warp") || !grow(b_bvi[0], (size_t)m2 * 4, "warp") ||
+      !grow(b_bvi[1], (size_t)m2 * 4, "warp") || !grow(b_temp, scan_u32_temp_bytes(m2), "scan"))
+    return false;
+  u32* head = (u32*)b_bhead.p;
+  u32* hscan = (u32*)b_bhscan.p;
+  LAUNCH("warp_keys", 40.0 * m2, launch_warp_keys(comp, m2, L, rec, ws, head, (u32*)b_bwf.p, stream));
+  LAUNCH("scan", 8.0 * m2, launch_scan_exclusive_u32(head, hscan, m2, b_temp.p, stream));
+  u32 tail[2];
+  cudaMemcpyAsync(&tail[0], hscan + m2 - 1, 4, cudaMemcpyDeviceToHost, stream);
+  cudaMemcpyAsync(&tail[1], head + m2 - 1, 4, cudaMemcpyDeviceToHost, stream);
+  if (!sync_check("warp runs")) return false;
+  const u32 ngroups = tail[0] + tail[1];
+  LAUNCH("warp_key2", 20.0 * m2,
+         launch_warp_key2(head, hscan, (const u32*)b_bwf.p, m2, (u64*)b_bvk[0].p, (u32*)b_bvi[0].p, stream));
+  u32 gbits = 0;
+  while (gbits < 32 && (1ull << gbits) < ngroups) gbits++;
+  int w = 0;
+  if (!sort_kv((u64*)b_bvk[0].p, (u32*)b_bvi[0].p, (u64*)b_bvk[1].p, (u32*)b_bvi[1].p, m2, 32 + gbits, &w)) return false;
+  if (!grow(b_bslot, (size_t)ngroups * 16, "warp slots")) return false;
+  unsigned long long* slot = (unsigned long long*)b_bslot.p;
+  cudaMemsetAsync(slot, 0xFF, (size_t)ngroups * 16, stream);
+  LAUNCH("warp_pairs", 0.0,
+         launch_warp_pairs(comp, L, rec, warp_ext, ws, (const u64*)b_bvk[w].p, (const u32*)b_bvi[w].p, m2, slot,
+                           stream));
+  LAUNCH("warp_fold", 0.0,
+         launch_warp_fold((const u64*)b_rkeys[0].p, (const RaceOut*)b_races.p, nA, comp, m2, L, hscan, index_base, slot,
+                          stream));
+  // re-emit every (run, kind) from its slot
+  const u64 need = 2ull * ngroups;
+  if (!grow(b_races, need * sizeof(RaceOut), "races") || !grow(b_rkeys[0], need * 8, "race keys") ||
+      !grow(b_rkeys[1], need * 8, "race keys") || !grow(b_rvals[0], need * 4, "race vals") ||
+      !grow(b_rvals[1], need * 4, "race vals") || !grow(b_ccount, 16, "ccount"))
+    return false;
+  cudaMemsetAsync(b_ccount.p, 0, 16, stream);
+  ConflictArgs A;
+  memset(&A, 0, sizeof A);
+  A.keys = comp;
+  A.m = m2;
+  A.rec = rec;
+  A.L = L;
+  A.race_count = (u32*)b_ccount.p;
+  A.race_keys = (u64*)b_rkeys[0].p;
+  A.race_vals = (u32*)b_rvals[0].p;
+  A.races = (RaceOut*)b_races.p;
+  A.race_cap = (u32)need;
+  A.index_base = index_base;
+  LAUNCH("warp_emit", 0.0, launch_warp_emit(A, head, hscan, slot, stream));
+  u32 total = 0;
+  if (!cuda_ok(cudaMemcpyAsync(&total, b_ccount.p, 4, cudaMemcpyDeviceToHost, stream), "warp count") ||
+      !sync_check("warp emit"))
+    return false;
+  n_races = total;
+  return true;
+}
+
 // step 6: canonical order of nr races: sort (location key << 1 | kind, index), permute into `out`
 bool sesa_trace::step_race_sort(u32 nr, const RaceOut* races, u64* rkeys0, u32* rvals0, u64* rkeys1, u32* rvals1,
                                 RaceOut* out) {
@@ -812,8 +882,12 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
 
 // steps 5-6 (shared by the sort + compaction and the bucket paths): conflict tiles, benign regrouping, race sort
 sesa_status sesa_trace::finish_check(const u64* comp, u32 m2, const Rec* rec, u64 index_base) {
-  if (!step_conflict(comp, m2, rec, 0, nullptr, index_base)) return status;
-  if (!step_benign(comp, m2, rec, index_base)) return status;
+  if (warp_ext && cfg.lockstep) {
+    if (!step_warp_model(comp, m2, rec, index_base)) return status;
+  } else {
+    if (!step_conflict(comp, m2, rec, 0, nullptr, index_base)) return status;
+    if (!step_benign(comp, m2, rec, index_base)) return status;
+  }
   const u32 nr = (u32)n_races;
   info.n_races = nr;
   if (!grow(b_races_sorted, (size_t)std::max(nr, 1u) * sizeof(RaceOut), "sorted races")) return status;
@@ -1031,6 +1105,21 @@ sesa_status sesa_race_check_launches(sesa_trace* t, const sesa_access* d_records
   t->stream = (cudaStream_t)cuda_stream;
   if (t->dist) return t->begin_check(n), t->fail(SESA_EINVAL, "multi-launch checks need a single-GPU handle"), SESA_EINVAL;
   return t->check_launches(d_records, n, launch_offsets, n_launches, index_base);
+}
+
+sesa_status sesa_race_check_warp(sesa_trace* t, const sesa_access* d_records, const sesa_access_ext* d_ext,
+                                 uint64_t n, uint64_t index_base, void* cuda_stream) {
+  if (!t) return SESA_EINVAL;
+  t->stream = (cudaStream_t)cuda_stream;
+  if (t->dist) return t->begin_check(n), t->fail(SESA_EINVAL, "the precise warp model needs a single-GPU handle"), SESA_EINVAL;
+  if (t->cfg.flags & SESA_FLAG_REPORT_BENIGN)
+    return t->begin_check(n), t->fail(SESA_EINVAL, "benign reporting is not defined for the precise warp model"),
+           SESA_EINVAL;
+  if (n && !d_ext) return t->begin_check(n), t->fail(SESA_EINVAL, "d_ext is NULL"), SESA_EINVAL;
+  t->warp_ext = d_ext;
+  const sesa_status st = t->check_device(d_records, n, index_base);
+  t->warp_ext = nullptr;
+  return st;
 }
 
 sesa_status sesa_races_get(sesa_trace* t, sesa_race* host_out, uint64_t cap, uint64_t* n_races) {

@@ -44,6 +44,8 @@ struct sesa_trace {
   DevBuf b_races, b_rkeys[2], b_rvals[2], b_races_sorted, b_rhist, b_rbase;
   DevBuf b_eoff, b_ecnt, b_ecell, b_hrec, b_dist_races, b_ctmp, b_ctotal, b_thist, b_ftmp, b_thist2, b_btmp2;
   DevBuf b_lraces;  // multi-launch checks: the races of the launches checked so far
+  const void* warp_ext = nullptr;  // precise warp model: the {pc, div} extension of the records being checked
+  uint32_t conflict_tdiv = 0;      // > 1: conflict tiles with identity = thread / tdiv, lockstep off
   bool have_thist2 = false;  // extents also wrote the per-tile histograms of the bucket path's first digit
   bool have_thist = false;
   bool hist_from_extents = false;  // fused path: later-digit histograms from the extents' raw granule bytes  // extents wrote per-tile raw digit histograms (fused first pass possible)
@@ -101,6 +103,7 @@ struct sesa_trace {
   sesa_status check_device(const sesa_access* d_rec, uint64_t n, uint64_t index_base);
   sesa_status check_launches(const sesa_access* d_rec, uint64_t n, const uint64_t* offs, uint32_t nl,
                              uint64_t index_base);
+  bool step_warp_model(const uint64_t* comp, uint32_t m2, const sesa::Rec* rec, uint64_t index_base);
   sesa_status finish_check(const uint64_t* comp, uint32_t m2, const sesa::Rec* rec, uint64_t index_base);
   // pipeline steps (shared by the single-GPU and the distributed check)
   void begin_check(uint64_t n);

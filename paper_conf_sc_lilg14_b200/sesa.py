@@ -65,7 +65,7 @@ EXPORTS = ["sesa_trace_create", "sesa_trace_create_dist", "sesa_nccl_unique_id",
            "sesa_race_check_host", "sesa_races_get", "sesa_races_device", "sesa_expand", "sesa_trace_set_profiling",
            "sesa_trace_info", "sesa_trace_kernel_stats", "sesa_trace_destroy", "sesa_status_str", "sesa_last_error",
            "sesa_abi_version", "sesa_race_check_loopback", "sesa_trace_set_regions", "sesa_oob_get",
-           "sesa_race_check_launches"]
+           "sesa_race_check_launches", "sesa_race_check_warp"]
 
 _lib = None
 
@@ -86,6 +86,7 @@ def load() -> ctypes.CDLL:
     lib.sesa_race_check.argtypes = [P, P, U64, U64, P]
     lib.sesa_race_check_host.argtypes = [P, P, U64, U64, P]
     lib.sesa_race_check_launches.argtypes = [P, P, U64, P, U32, U64, P]
+    lib.sesa_race_check_warp.argtypes = [P, P, P, U64, U64, P]
     lib.sesa_race_check_loopback.argtypes = [ctypes.POINTER(sesa_config), P, P, I, U64, P, PP]
     lib.sesa_races_get.argtypes = [P, P, U64, ctypes.POINTER(U64)]
     lib.sesa_races_device.argtypes = [P, PP, ctypes.POINTER(U64)]
@@ -169,6 +170,16 @@ class Trace:
                                                len(offs) - 1, index_base, _stream_ptr(stream))
         if st != SESA_OK:
             self._raise(st, "sesa_race_check_launches")
+        return self.n_races()
+
+    def check_warp(self, d_records, d_ext, n: int, index_base: int = 0, stream=None) -> int:
+        """Precise warp model (NEXT-3): d_ext = device array of n {pc, div} u32 pairs."""
+        ptr, count = _dev_ptr(d_records, n)
+        eptr = d_ext if isinstance(d_ext, int) else d_ext.data_ptr()
+        st = self.lib.sesa_race_check_warp(self.h, ctypes.c_void_p(ptr), ctypes.c_void_p(eptr), count, index_base,
+                                           _stream_ptr(stream))
+        if st != SESA_OK:
+            self._raise(st, "sesa_race_check_warp")
         return self.n_races()
 
     def check_host(self, h_records: np.ndarray, index_base: int = 0, stream=None) -> int:

@@ -510,3 +510,62 @@ def test_launches_f1_twice_and_validation(sesa):
         with pytest.raises(sesa.SesaError):
             t.check_launches(sesa.to_device(two), len(two), bad)
     t.close()
+
+
+# ------------------------------------------------------------------------------------------------ precise warps (NEXT-3)
+def _ext_dev(e):
+    return torch.from_numpy(np.ascontiguousarray(e).view(np.uint8).reshape(-1)).cuda()
+
+
+def test_precise_warp_f1_f4(sesa):
+    for r, e, ws in ((G.f1_race(), G.f1_race_ext(), 32), (G.f4_histo_prescan(), G.f4_histo_prescan_ext(), 32),
+                     (G.f4_histo_prescan(), G.f4_histo_prescan_ext(), 1)):
+        t = sesa.Trace(ws, 1, 4)
+        t.check_warp(sesa.to_device(r), _ext_dev(e), len(r))
+        assert t.races().tobytes() == O.check_warp(r, e, warp_size=ws).tobytes()
+        t.close()
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_precise_warp_random(sesa, seed):
+    """Random traces with random {pc, div}: sizes from one tile to many (hot locations cross tiles), shared and
+    global, warp sizes 32/4/3; equal to the oracle's precise-warp checker."""
+    n = [500, 4000, 30000, 120000, 2000][seed % 5]
+    ws = [32, 4, 3, 32, 8][seed % 5]
+    r = G.random_trace(n, 8800 + seed, threads=[64, 256, 700][seed % 3], blocks=1 + seed % 4,
+                       words=[5, 60, 2000][seed % 3], sort=seed % 4 != 3, values=3)
+    e = G.random_ext(n, seed, npc=1 + seed % 5, ninst=1 + seed % 3, div_frac=[0.0, 0.5, 1.0][seed % 3])
+    t = sesa.Trace(ws, 1, 4)
+    t.check_warp(sesa.to_device(r), _ext_dev(e), n, index_base=seed)
+    got = t.races()
+    t.close()
+    assert got.tobytes() == O.check_warp(r, e, warp_size=ws, index_base=seed).tobytes()
+
+
+def test_precise_warp_lockstep_off_and_validation(sesa):
+    r, e = G.f1_race(), G.f1_race_ext()
+    t = sesa.Trace(32, 0, 4)
+    t.check_warp(sesa.to_device(r), _ext_dev(e), len(r))
+    assert t.races().tobytes() == O.check(r).tobytes()  # extension ignored without lockstep
+    t.close()
+    t = sesa.Trace(32, 1, 4, benign=True)
+    with pytest.raises(sesa.SesaError):
+        t.check_warp(sesa.to_device(r), _ext_dev(e), len(r))
+    t.close()
+
+
+@pytest.mark.slow
+def test_precise_warp_large(sesa):
+    """2 M records, ~100 entries per location (runs cross many conflict tiles), global + shared, the fused path
+    not taken (mixed spaces): equal to the oracle."""
+    from sesagen import configs as C
+    n = 2_000_000
+    r = C.rnd_host(n, 4242, blocks=64, threads=512, intervals=4, words=20000, shared_frac=0.3, sizes=(4, 8),
+                   values=4, unaligned=False)
+    e = G.random_ext(n, 99, npc=6, ninst=4, div_frac=0.6)
+    t = sesa.Trace(32, 1, 4)
+    t.check_warp(sesa.to_device(r), _ext_dev(e), n)
+    got = t.races()
+    t.close()
+    exp = O.check_warp(r, e, warp_size=32)
+    assert len(exp) > 1000 and got.tobytes() == exp.tobytes()
