@@ -255,12 +255,15 @@ __global__ void bucket_total_kernel(const u32* off, const u32* cnt, u32 n, u32* 
 }
 
 // ---- sample of the chunk sizes: histogram of the chunks of every stride-th granule, and the maximum --------------
+// (warp-aggregated: lanes of one chunk add once — a hot chunk, C3's bins, would otherwise serialise the atomics)
 __global__ void bucket_sample_kernel(const u32* __restrict__ gran, u32 n, u32 stride, u32 gmin_lo, u32 nchunks,
                                      u32* __restrict__ hist) {
-  for (u64 i = (u64)(blockIdx.x * blockDim.x + threadIdx.x) * stride; i < n;
-       i += (u64)gridDim.x * blockDim.x * stride) {
-    const u32 c = (gran[i] - gmin_lo) >> HYB_CHUNK;
-    if (c < nchunks) atomicAdd(&hist[c], 1u);
+  const u64 step = (u64)gridDim.x * blockDim.x * stride;
+  for (u64 i0 = (u64)(blockIdx.x * blockDim.x + (threadIdx.x & ~31u)) * stride; i0 < n; i0 += step) {
+    const u64 i = i0 + (u64)(threadIdx.x & 31) * stride;
+    const u32 c = i < n ? (gran[i] - gmin_lo) >> HYB_CHUNK : ~0u;
+    const unsigned peers = __match_any_sync(~0u, c);
+    if (c < nchunks && (threadIdx.x & 31) == __ffs(peers) - 1) atomicAdd(&hist[c], (u32)__popc(peers));
   }
 }
 
@@ -278,10 +281,9 @@ size_t bucket_temp_bytes(u32 nchunks) {
 }
 
 u32 bucket_sample_max(const u32* gran, u32 n, u32 gmin_lo, u32 nchunks, void* temp, cudaStream_t st, u32* h_max,
-                      u32* samples) {
+                      u32* samples, u32 want) {
   u32* hist = reinterpret_cast<u32*>(temp);
   u32* mx = hist + nchunks;
-  const u32 want = 1u << 22;
   const u32 stride = std::max<u32>(1, n / want);
   *samples = (n + stride - 1) / stride;
   cudaMemsetAsync(temp, 0, ((size_t)nchunks + 1) * 4, st);

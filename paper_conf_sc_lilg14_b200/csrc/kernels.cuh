@@ -51,7 +51,7 @@ constexpr uint64_t BUCKET_MIN_N = 1ull << 24;  // traces of fewer records keep t
 size_t bucket_temp_bytes(u32 nchunks);
 // sample of the chunk sizes from the extents' granule array: *h_max (host, after a sync) = largest sampled count
 u32 bucket_sample_max(const u32* gran, u32 n, u32 gmin_lo, u32 nchunks, void* temp, cudaStream_t st, u32* h_max,
-                      u32* samples);
+                      u32* samples, u32 want);
 u32 launch_bucket_compact(u64* keys, u64* stage, u32 m, u32 pos_bits, u32 nchunks, void* temp, u32* total,
                           cudaStream_t st);
 

@@ -331,12 +331,17 @@ bool sesa_trace::bucket_choose(u64 n, u64* gmin_aligned, u32* nbits, u32* nchunk
   if (nb <= D || nb > HYB_LO + 2 * RADIX_BITS || nb + layout.pos_bits > 64) return false;
   const u32 nc = (u32)(((S.gmax[1] - G0) >> HYB_CHUNK) + 1);
   if (!grow(b_btmp2, bucket_temp_bytes(nc), "bucket temp")) return false;
-  u32 hmax = 0, samples = 0;
-  LAUNCH("bucket_sample", 4.0 * (n >> 8), launches += bucket_sample_max((const u32*)b_keys[0].p, (u32)n, (u32)G0, nc,
-                                                                        b_btmp2.p, stream, &hmax, &samples) - 1);
-  if (!sync_check("bucket sample")) return false;
-  const double est_max = (double)hmax * (double)n / (double)std::max(1u, samples), mean = (double)n / nc;
-  if (est_max > 4.0 * mean + 2048.0 || est_max > (double)(1u << 20)) return false;
+  // a 64 K sample first: a hot region (C3's bins, C4's `changed`) shows at once; then 4 M samples for the bound
+  const double mean = (double)n / nc;
+  for (u32 want : {1u << 16, 1u << 22}) {
+    u32 hmax = 0, samples = 0;
+    LAUNCH("bucket_sample", 4.0 * (double)want, launches += bucket_sample_max((const u32*)b_keys[0].p, (u32)n, (u32)G0, nc,
+                                                                             b_btmp2.p, stream, &hmax, &samples, want) - 1);
+    if (!sync_check("bucket sample")) return false;
+    const double est_max = (double)hmax * (double)n / (double)std::max(1u, samples);
+    if (want < (1u << 22) ? est_max > 32.0 * mean + 65536.0 : (est_max > 4.0 * mean + 2048.0 || est_max > (double)(1u << 20)))
+      return false;
+  }
   *gmin_aligned = G0;
   *nbits = nb;
   *nchunks = nc;

@@ -51,34 +51,36 @@ def test_c3_full_size_parity(S):
 
 
 def test_c4_full_size_parity(S):
+    """C4 (lockstep) in full, with and without benign reporting, against ONE oracle run with benign reporting (its
+    kinds 1-2 are the plain list: rule (6) keeps benign pairs out of them either way).  Table IV reports the BFS
+    kernel as "W/W (Benign)": kind-3 records appear (at `changed` and at dist[] entries written by several
+    frontier threads) and still no kind-2 race."""
     cfg = C.C4()
     dev, n = cfg.device()
-    got, host = full_parity(S, dev, n, 32, 1)
+    host = dev.cpu().numpy().view(G.REC_DTYPE)
+    exp = O.check(host, warp_size=32, lockstep=1, benign=True, method="partitioned")
+    for benign in (False, True):
+        t = S.Trace(32, 1, 4, benign=benign)
+        t.check(dev, n)
+        got = t.races()
+        t.close()
+        want = exp if benign else exp[exp["kind"] != 3]
+        assert len(got) == len(want) and got.tobytes() == want.tobytes()
+    assert set(exp["kind"].tolist()) == {1, 3}
+    assert int(cfg.cfg().changed_base) in set(exp["addr"][exp["kind"] == 3].tolist())
     # invariants: all writes at one location carry the same value -> no WW; races only on dist[]
-    assert set(got["kind"].tolist()) == {1}
+    rw = exp[exp["kind"] == 1]
     c = cfg.cfg()
-    assert ((got["addr"] >= c.dist_base) & (got["addr"] < c.dist_base + 4 * (1 << cfg.log2n))).all()
+    assert ((rw["addr"] >= c.dist_base) & (rw["addr"] < c.dist_base + 4 * (1 << cfg.log2n))).all()
     # lockstep only removes races
     t = S.Trace(32, 0, 4)
     t.check(dev, n)
     nols = t.races()
     t.close()
     key = lambda r: set(zip(r["addr"].tolist(), r["kind"].tolist()))  # noqa: E731
-    assert key(got) <= key(nols)
-    print(f"C4: {len(got)} races ({len(nols)} without lockstep) equal to the oracle's over all {n} records")
-
-
-def test_c4_full_size_benign_parity(S):
-    """Table IV reports the BFS kernel as "W/W (Benign)": with benign reporting the full-size C4 trace
-    gets kind-3 records (at `changed` and at dist[] entries written by several frontier threads) and still no
-    kind-2 race; the whole list equals the oracle's, witnesses included."""
-    cfg = C.C4()
-    dev, n = cfg.device()
-    got, host = full_parity(S, dev, n, 32, 1, benign=True)
-    kinds = set(got["kind"].tolist())
-    assert kinds == {1, 3}
-    assert int(cfg.cfg().changed_base) in set(got["addr"][got["kind"] == 3].tolist())
-    print(f"C4 benign: {(got['kind'] == 3).sum()} benign locations; full list equal to the oracle's")
+    assert key(rw) <= key(nols)
+    print(f"C4: {len(rw)} races ({len(nols)} without lockstep), {(exp['kind'] == 3).sum()} benign locations: "
+          f"equal to the oracle's over all {n} records")
 
 
 def test_c5_full_size_truth(S):
