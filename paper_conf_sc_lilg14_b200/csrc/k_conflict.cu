@@ -1185,6 +1185,7 @@ template <class A>
 struct CarryEl {
   A a;
   u32 owner;
+  u32 pad;  // explicit (always 0): stored with the struct, so global copies carry no uninitialised bytes
 };
 
 template <class A>
@@ -1193,6 +1194,7 @@ struct OpCarry {
     CarryEl<A> r;
     r.a = typename OpOf<A>::type()(x.a, y.a);
     r.owner = max(x.owner, y.owner);
+    r.pad = 0;
     return r;
   }
 };
@@ -1201,6 +1203,7 @@ __device__ __forceinline__ CarryEl<A> shfl(const CarryEl<A>& c, int o, bool down
   CarryEl<A> r;
   r.a = shfl(c.a, o, down);
   r.owner = shfl(c.owner, o, down);
+  r.pad = 0;
   return r;
 }
 
@@ -1211,6 +1214,7 @@ __device__ __forceinline__ void carry_element(const ConflictArgs& a, u32 j, u32 
   typedef typename QuadOf<A>::type Q;
   e.a = agg_empty_t<A>();
   e.owner = 0;
+  e.pad = 0;
   f = true;
   if (j >= ntiles) return;
   const u8 tf = a.tile_flags[j];
@@ -1241,7 +1245,7 @@ __global__ void __launch_bounds__(CARRY_T) carry_chunk_kernel(ConflictArgs a, u3
     CarryEl<A> e;
     carry_element<A>(a, j, ntiles, d, f, e);
     CarryEl<A> seed;
-    seed.a = agg_empty_t<A>(), seed.owner = 0;
+    seed.a = agg_empty_t<A>(), seed.owner = 0, seed.pad = 0;
     const bool rev = d & 1;
     CarryEl<A> inc = rev ? carry_block_scan<A, true>(f, e, seed, s_wv, s_wf)
                          : carry_block_scan<A, false>(f, e, seed, s_wv, s_wf);
@@ -1264,10 +1268,10 @@ __global__ void __launch_bounds__(CARRY_T) carry_top_kernel(u32 nchunks, CarryEl
   for (int d = 0; d < 4; d++) {
     CarryEl<A> e;
     bool f = true;
-    e.a = agg_empty_t<A>(), e.owner = 0;
+    e.a = agg_empty_t<A>(), e.owner = 0, e.pad = 0;
     if (c < nchunks) e = chunk_tot[c * 4 + d], f = chunk_f[c * 4 + d];
     CarryEl<A> seed;
-    seed.a = agg_empty_t<A>(), seed.owner = 0;
+    seed.a = agg_empty_t<A>(), seed.owner = 0, seed.pad = 0;
     CarryEl<A> ex =
         (d & 1) ? block_seg_excl<CarryEl<A>, OpCarry<A>, true, CARRY_T>(f, e, seed, OpCarry<A>(), s_wv, s_wf)
                 : block_seg_excl<CarryEl<A>, OpCarry<A>, false, CARRY_T>(f, e, seed, OpCarry<A>(), s_wv, s_wf);

@@ -29,7 +29,11 @@ __global__ void tile_col_reduce_kernel(const u32* __restrict__ H, u32 T, u32 tpc
 }
 
 // (2) one CTA: exclusive prefix over chunks per raw byte, plus the bin base of each digit (rotated order)
-__global__ void tile_col_scan_kernel(u32* __restrict__ P, u32 C, u32 r0) {
+// pad32 (the bucket path): every digit run is padded to a multiple of 32 slots with ~0 sentinels (written here,
+// into kout), so that no 32-key row of the next, unstable pass holds two digit values (k_bucket.cu); *mtot = the
+// padded length
+__global__ void tile_col_scan_kernel(u32* __restrict__ P, u32 C, u32 r0, u64* __restrict__ kout,
+                                     u32* __restrict__ mtot) {
   __shared__ u32 s_tot[RADIX], s_w[RADIX / 32 + 1];
   const u32 r = threadIdx.x, lane = r & 31, warp = r >> 5;
   u32 run = 0;
@@ -42,7 +46,8 @@ __global__ void tile_col_scan_kernel(u32* __restrict__ P, u32 C, u32 r0) {
       if (c0 + q < C) P[(u64)(c0 + q) * RADIX + r] = run, run += v[q];
   }
   const u32 d = (r - r0) & (RADIX - 1);
-  s_tot[d] = run;
+  const u32 real = run;
+  s_tot[d] = kout ? (run + 31u) & ~31u : run;
   __syncthreads();
   // exclusive scan over digits d (thread d holds s_tot[d])
   const u32 v = s_tot[r];
@@ -64,8 +69,11 @@ __global__ void tile_col_scan_kernel(u32* __restrict__ P, u32 C, u32 r0) {
   }
   __syncthreads();
   s_tot[r] = s_w[warp] + x - v;  // bin base of digit r
+  if (kout && r == RADIX - 1) *mtot = s_w[warp] + x;
   __syncthreads();
   const u32 base = s_tot[d];
+  if (kout)  // sentinels after the run's real keys
+    for (u32 q = base + real; q < ((base + real + 31u) & ~31u); q++) kout[q] = ~0ull;
   for (u32 c = 0; c < C; c++) P[(u64)c * RADIX + r] += base;
 }
 
@@ -197,7 +205,7 @@ __global__ void __launch_bounds__(FUSED_THREADS, FUSED_MINB) fused_extract_pass0
         __syncwarp();
       }
       const unsigned peers = bal ? peers_of<RADIX_BITS + 1>(d) : wm[d];
-      const u32 c = wh[d];
+      const u32 c = d < RADIX ? wh[d] : 0u;  // (invalid items: digit RADIX, no counter)
       __syncwarp();
       if (d < RADIX) keys_s[c + __popc(peers & lt)] = ((u64)kh[i] << A.pos_bits) | (u64)(wbase + i * 32);
       if (lane == 31 - __clz(peers)) {
@@ -235,7 +243,8 @@ static size_t fused_smem(u32 npass) {
 bool fused_supported(u32 npass) { return npass >= 1 && npass <= 4; }  // sort_bits <= 32 on this path
 
 // tile offsets O[t][d] into temp (fused_temp_bytes(n)) from the extents' raw per-tile histograms
-void launch_tile_offsets(u64 n, const KeyLayout& L, const u32* tile_hist, void* temp, cudaStream_t st, u32 dsh) {
+void launch_tile_offsets(u64 n, const KeyLayout& L, const u32* tile_hist, void* temp, cudaStream_t st, u32 dsh,
+                         u64* pad_kout, u32* mtot) {
   if (!n) return;
   const u32 T = (u32)((n + FUSED_TILE - 1) / FUSED_TILE);
   u32* O = reinterpret_cast<u32*>(temp);
@@ -243,7 +252,7 @@ void launch_tile_offsets(u64 n, const KeyLayout& L, const u32* tile_hist, void* 
   const u32 C = std::min<u32>(T, 1024), tpc = (T + C - 1) / C, Cu = (T + tpc - 1) / tpc;
   const u32 r0 = (u32)((L.gminG >> dsh) & (RADIX - 1));
   tile_col_reduce_kernel<<<Cu, RADIX, 0, st>>>(tile_hist, T, tpc, P);
-  tile_col_scan_kernel<<<1, RADIX, 0, st>>>(P, Cu, r0);
+  tile_col_scan_kernel<<<1, RADIX, 0, st>>>(P, Cu, r0, pad_kout, mtot);
   tile_col_down_kernel<<<Cu, RADIX, 0, st>>>(tile_hist, T, tpc, P, r0, O);
 }
 

@@ -151,7 +151,7 @@ __device__ __forceinline__ void onesweep_kv_tile(const u64* __restrict__ kin, u6
     __syncwarp();
     // the peer word and the running counter are read together: one shared-memory round trip per item
     const unsigned peers = wm[d];
-    const u32 c = wh[d];
+    const u32 c = (FULL || d < RADIX) ? wh[d] : 0u;  // (invalid items of a partial tile: digit RADIX, no counter)
     __syncwarp();
     const bool leader = lane == 31 - __clz(peers);
     rd[i] |= (c + __popc(peers & lanemask_lt())) << 9;
@@ -282,8 +282,13 @@ __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64*
     for (int i = 0; i < ITEMS; i++)
       if (FULL || i < nv) k[i] = __ldcs(kin + wbase + (u64)i * 32);
   }
+  // (UNST: the input's ~0 sentinels — padding of 32-aligned digit runs — are no keys)
+  //  UNST passes sort by the TOP digit (nothing above it), so a sentinel is the only key whose shifted value is
+  //  >= RADIX)
   auto digit = [&](int i) -> u32 {
-    return (FULL || i < nv) ? (u32)((k[i] >> shift) & (RADIX - 1)) : (u32)RADIX;
+    if (!(FULL || i < nv)) return (u32)RADIX;
+    if (UNST) { const u32 d9 = (u32)(k[i] >> shift) & (2 * RADIX - 1); return d9 < RADIX ? d9 : (u32)RADIX; }
+    return (u32)((k[i] >> shift) & (RADIX - 1));
   };
   // rank streams: items [s*IPS, (s+1)*IPS) of a warp form stream s (stable order = warp, stream, item, lane),
   // each with its own counters and peer masks, so that S items are ranked per shared-memory round trip
@@ -300,7 +305,7 @@ __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64*
     for (int i = 0; i < (ITEMS + 1) / 2; i++) rk[i] = 0;
 #pragma unroll
   for (int i = 0; i < ITEMS; i++)
-    if (FULL || i < nv) {
+    if ((FULL || i < nv) && (!UNST || digit(i) < RADIX)) {
       const u32 r = atomicAdd(&wh[(i / IPS) * RADIX + digit(i)], 1u);
       if (UNST) rk[i / 2] |= r << (16 * (i & 1));
     }
@@ -321,6 +326,8 @@ __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64*
 #pragma unroll
     for (int w = 0; w < WARPS * S; w++) whist[w * RADIX + tid] += bs;
   }
+  __shared__ u32 s_real;  // UNST: keys of the tile (sentinels excluded)
+  if (UNST && tid == RADIX - 1) s_real = bs + tot;
   auto look_back = [&]() {
     if (tid < RADIX) {
       u64 excl = 0;
@@ -362,7 +369,7 @@ __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64*
 #pragma unroll
     for (int i = 0; i < ITEMS; i++) {
       const u32 d = digit(i);
-      if (FULL || d < RADIX) keys_s[wh[d] + ((rk[i / 2] >> (16 * (i & 1))) & 0xFFFFu)] = k[i];
+      if (d < RADIX) keys_s[wh[d] + ((rk[i / 2] >> (16 * (i & 1))) & 0xFFFFu)] = k[i];
     }
   } else {
   // (3) stable warp ranking, each key stored straight into its tile-local slot
@@ -389,7 +396,7 @@ __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64*
     for (int q = 0; q < S; q++) {
       peers[q] = bal ? (FULL ? peers_of<RADIX_BITS>(d[q]) : peers_of<RADIX_BITS + 1>(d[q]))
                      : mat ? __match_any_sync(~0u, d[q]) : wm[q * (RADIX + 1) + d[q]];
-      c[q] = wh[q * RADIX + d[q]];
+      c[q] = (FULL || d[q] < RADIX) ? wh[q * RADIX + d[q]] : 0u;  // (invalid items: digit RADIX, no counter)
     }
     __syncwarp();
 #pragma unroll
@@ -409,12 +416,21 @@ __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64*
   __syncthreads();
   if (prof && tid == 0) prof[4] = gtime();
   // (4) coalesced write-out of each digit's run
-  const u32 tcount = FULL ? (u32)TILE : (u32)min((u64)TILE, (u64)m - tbase);
+  if (FULL && (!UNST || s_real == (u32)TILE)) {  // (the common case: a full tile without sentinels)
 #pragma unroll 4
-  for (u32 j = tid; j < tcount; j += THREADS) {
-    const u64 key = keys_s[j];
-    const u32 d = (u32)((key >> shift) & (RADIX - 1));
-    __stcs(kout + (globu[d] + j), key);
+    for (u32 j = tid; j < (u32)TILE; j += THREADS) {
+      const u64 key = keys_s[j];
+      const u32 d = (u32)((key >> shift) & (RADIX - 1));
+      __stcs(kout + (globu[d] + j), key);
+    }
+  } else {
+    const u32 tcount = UNST ? s_real : FULL ? (u32)TILE : (u32)min((u64)TILE, (u64)m - tbase);
+#pragma unroll 4
+    for (u32 j = tid; j < tcount; j += THREADS) {
+      const u64 key = keys_s[j];
+      const u32 d = (u32)((key >> shift) & (RADIX - 1));
+      __stcs(kout + (globu[d] + j), key);
+    }
   }
   if (prof) {
     __syncthreads();

@@ -40,7 +40,10 @@ bool fused_supported(u32 npass);
 size_t fused_temp_bytes(u64 n);
 // dsh: the digit is key_hi bits [dsh, dsh + 8) (tile_hist then holds the raw (g >> dsh) & 255 histograms and gmin
 // is a multiple of 2^dsh)
-void launch_tile_offsets(u64 n, const KeyLayout& L, const u32* tile_hist, void* temp, cudaStream_t st, u32 dsh = 0);
+// pad_kout (bucket path): pad every digit run of the output to a multiple of 32 with ~0 sentinels; *mtot (device)
+// = the padded length
+void launch_tile_offsets(u64 n, const KeyLayout& L, const u32* tile_hist, void* temp, cudaStream_t st, u32 dsh = 0,
+                         u64* pad_kout = nullptr, u32* mtot = nullptr);
 // gran: the extents pass's granule indices (gout); rec is not read
 // unstable: no stable order within a digit (the bucket path); npass must be 1
 void launch_fused_extract_pass0(const u32* gran, u64 n, const KeyLayout& L, u32 npass, void* temp, u64* kout,

@@ -350,7 +350,8 @@ bool sesa_trace::bucket_choose(u64 n, u64* gmin_aligned, u32* nbits, u32* nchunk
 
 bool sesa_trace::step_bucket(u64 n, u32 nchunks, u64** comp, u32* m2) {
   const KeyLayout& L = layout;
-  if (!grow(b_keys[1], n * 8 + 64, "keys") || !grow(b_hist, 2 * RADIX * 4, "hist") ||
+  // the fused pass's output carries up to 31 sentinels per digit run (32-aligned runs, below)
+  if (!grow(b_keys[1], (n + 32 * RADIX) * 8 + 64, "keys") || !grow(b_hist, 2 * RADIX * 4, "hist") ||
       !grow(b_binbase, 2 * RADIX * 8, "binbase") || !grow(b_ftmp, fused_temp_bytes(n), "fused temp") ||
       !grow(b_ctotal, 16, "compact count"))
     return false;
@@ -362,16 +363,25 @@ bool sesa_trace::step_bucket(u64 n, u32 nchunks, u64** comp, u32* m2) {
   if (!cuda_ok(cudaMemcpyAsync((u32*)b_hist.p + RADIX, row.data(), RADIX * 4, cudaMemcpyHostToDevice, stream), "hist"))
     return false;
   cudaMemsetAsync(b_hist.p, 0, RADIX * 4, stream);
+  // Both partition passes are unstable (k_bucket.cu).  The second keeps the first one's digit order only if no
+  // 32-key row of its input holds two first-digit values: the first pass pads every digit run to a multiple of
+  // 32 with ~0 sentinels, which the second pass skips.
+  const bool pass2 = *std::max_element(row.begin(), row.end()) != n;  // digit B not trivial
   LAUNCH("tile_offsets", 2.0 * RADIX * 4 * ((n + FUSED_TILE - 1) / FUSED_TILE),
-         launch_tile_offsets(n, L, (const u32*)b_thist2.p, b_ftmp.p, stream, HYB_LO));
+         launch_tile_offsets(n, L, (const u32*)b_thist2.p, b_ftmp.p, stream, HYB_LO,
+                             pass2 ? (u64*)b_keys[1].p : nullptr, (u32*)b_ctotal.p + 2));
+  u32 mpad = (u32)n;
+  if (pass2 && (!cuda_ok(cudaMemcpyAsync(&mpad, (u32*)b_ctotal.p + 2, 4, cudaMemcpyDeviceToHost, stream), "padded") ||
+                !sync_check("tile offsets")))
+    return false;
   LAUNCH("extract_pass0", 12.0 * n,
          launch_fused_extract_pass0((const u32*)b_keys[0].p, n, L, 1, b_ftmp.p, (u64*)b_keys[1].p, (u32*)b_hist.p,
                                     stream, HYB_LO, true));
   int cur = 1;
   u32 passes = 1;
-  if (*std::max_element(row.begin(), row.end()) != n) {  // digit B not trivial
+  if (pass2) {
     LAUNCH("bin_base", 0.0, launch_bin_base((u32*)b_hist.p, (u64*)b_binbase.p, 2, stream));
-    const u32 stiles = sort_tiles(n);
+    const u32 stiles = sort_tiles(mpad);
     if (!grow(b_lookback, (size_t)stiles * RADIX * 8, "lookback") || !grow(b_ctr, 64 * 4, "counters")) return false;
     if (b_lookback.cap != lookback_cleared) {
       cudaMemsetAsync(b_lookback.p, 0, b_lookback.cap, stream);
@@ -384,7 +394,7 @@ bool sesa_trace::step_bucket(u64 n, u32 nchunks, u64** comp, u32* m2) {
       epoch = 1;
     }
     LAUNCH("partition_pass", 16.0 * n,
-           launch_partition_pass((u64*)b_keys[1].p, (u64*)b_keys[0].p, (u32)n, L.pos_bits + HYB_LO + RADIX_BITS,
+           launch_partition_pass((u64*)b_keys[1].p, (u64*)b_keys[0].p, mpad, L.pos_bits + HYB_LO + RADIX_BITS,
                                  (u64*)b_binbase.p + RADIX, (u64*)b_lookback.p, (u32*)b_ctr.p, epoch, stream));
     cur = 0;
     passes++;
