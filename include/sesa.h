@@ -248,6 +248,25 @@ sesa_status sesa_races_device(sesa_trace *t, const sesa_race **d_races, uint64_t
 sesa_status sesa_expand(sesa_trace *t, const sesa_flow *d_flows, uint64_t n_flows, sesa_access *d_out, uint64_t cap,
                         uint64_t *n_out, void *cuda_stream);
 
+/* Descriptor-level check: the race list of the trace that sesa_expand(d_flows) describes —
+ * identical, witnesses included (indices in the canonical expansion order), to expanding and checking it — decided
+ * per pair of descriptors first.  The paper instantiates two flows' accesses at two symbolic threads t1 != t2 and
+ * asks a solver whether an address can coincide (§IV-A, §IV-B); here interval arithmetic on
+ * the address functions (base + bstride*block + tstride*f(t) + istride*k, f in {id, modadd, xor, shr, row2d})
+ * proves pairs race-free without instantiating any thread: disjoint granule ranges, read/read, atomic/atomic, no
+ * common block or interval where ordering requires one, and plain-write descriptors whose instances never share a
+ * granule (injective f, strides beyond size + G - 1).  Only descriptors left in some undecided pair are
+ * instantiated and checked.  d_flows: DEVICE array.  Synchronises the stream. */
+sesa_status sesa_race_check_flows(sesa_trace *t, const sesa_flow *d_flows, uint64_t n_flows, void *cuda_stream);
+
+typedef struct {
+  uint64_t n_flows;           /* descriptors given                                                         */
+  uint64_t n_flows_checked;   /* descriptors left in an undecided pair (instantiated)                      */
+  uint64_t n_records;         /* records the descriptors describe (the full expansion)                     */
+  uint64_t n_records_checked; /* records instantiated and checked                                          */
+} sesa_flow_check_info;
+sesa_status sesa_flow_check_get(const sesa_trace *t, sesa_flow_check_info *out);
+
 /* Profiling: when enabled, every kernel of a check is bracketed by CUDA events on the check's stream. */
 sesa_status sesa_trace_set_profiling(sesa_trace *t, int enable);
 sesa_status sesa_trace_info(const sesa_trace *t, sesa_check_info *out);

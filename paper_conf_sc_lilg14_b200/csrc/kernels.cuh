@@ -195,4 +195,14 @@ void launch_flow_count2(const void* flows, const u32* ivoff, const u32* idx, u32
 void launch_flow_write2(const void* flows, const u32* ivoff, const u32* idx, u32 niv, u32 bmin, u64 ncell, u32 tmax,
                         const u32* off, Rec* out, cudaStream_t st);
 
+// descriptor-level check (k_expand.cu)
+size_t flow_range_bytes(u32 nf);
+void launch_flow_ranges(const void* flows, u32 nf, u32 log2G, void* ranges, u32* keep, cudaStream_t st);
+void launch_flow_count_sel(const void* flows, const u32* ivoff, const u32* idx, u32 niv, u32 bmin, u64 ncell, u32 tmax,
+                           const u32* keep, u32* cnt_all, u32* cnt_kept, cudaStream_t st);
+void launch_flow_write_sel(const void* flows, const u32* ivoff, const u32* idx, u32 niv, u32 bmin, u64 ncell, u32 tmax,
+                           const u32* keep, const u32* off_all, const u32* off_kept, Rec* out, u32* orig,
+                           cudaStream_t st);
+void launch_race_remap(struct RaceOut* races, u32 nr, const u32* orig, cudaStream_t st);
+
 }  // namespace sesa

@@ -79,7 +79,7 @@ static unsigned kernels_of(const char* name) {
   static const struct {
     const char* n;
     unsigned k;
-  } tab[] = {{"tile_offsets", 3}, {"compact", 4}, {"carry", 3}, {"alltoall", 0}};  // alltoall: NCCL's kernels
+  } tab[] = {{"tile_offsets", 3}, {"compact", 4}, {"carry", 3}, {"alltoall", 0}, {"flow_pairs", 2}};  // alltoall: NCCL's kernels
   for (const auto& e : tab)
     if (!strcmp(e.n, name)) return e.k;
   return 1;
@@ -968,6 +968,103 @@ sesa_status sesa_trace::check_launches(const sesa_access* d_rec, u64 n, const u6
   return SESA_OK;
 }
 
+// ------------------------------------------------------------------------------------------------ flows (NEXT-2)
+sesa_status sesa_trace::check_flows(const sesa_flow* d_flows, u64 nf) {
+  begin_check(0);
+  memset(&flow_info, 0, sizeof flow_info);
+  flow_info.n_flows = nf;
+  if (nf && !d_flows) return fail(SESA_EINVAL, "d_flows is NULL"), status;
+  std::vector<sesa_flow> h(nf);
+  if (nf && !cuda_ok(cudaMemcpy(h.data(), d_flows, nf * sizeof(sesa_flow), cudaMemcpyDeviceToHost), "flows D2H"))
+    return status;
+  u32 bmin = ~0u, bmax = 0, tmax = 0;
+  std::vector<u32> ivs;
+  for (u64 d = 0; d < nf; d++) {
+    const sesa_flow& f = h[d];
+    if (f.fkind > 4 || (f.fkind == SESA_F_MODADD && f.fm == 0) || (f.fkind >= SESA_F_SHR && f.fc >= 32) ||
+        f.space > 1 || f.rw > 2 || f.size == 0)
+      return fail(SESA_EINVAL, "flow %llu invalid", (unsigned long long)d), status;
+    ivs.push_back(f.interval);
+    if (f.block_lo >= f.block_hi) continue;
+    bmin = std::min(bmin, f.block_lo);
+    bmax = std::max(bmax, f.block_hi);
+    tmax = std::max(tmax, f.nthreads);
+  }
+  if (nf == 0 || bmin >= bmax || tmax == 0) return check_device(nullptr, 0, 0);
+  std::sort(ivs.begin(), ivs.end());
+  ivs.erase(std::unique(ivs.begin(), ivs.end()), ivs.end());
+  const u32 niv = (u32)ivs.size();
+  std::vector<u32> ivoff(niv + 1, 0), idx;
+  for (u32 q = 0; q < niv; q++) {
+    for (u64 d = 0; d < nf; d++)
+      if (h[d].interval == ivs[q]) idx.push_back((u32)d);
+    ivoff[q + 1] = (u32)idx.size();
+  }
+  const u64 ncell = (u64)(bmax - bmin) * niv * tmax;
+  if (!grow(b_eoff, (niv + 1 + idx.size()) * 4, "flow csr") || !grow(b_franges, flow_range_bytes((u32)nf), "ranges") ||
+      !grow(b_fkeep, nf * 4, "keep") || !grow(b_ecnt, ncell * 4, "cell counts") || !grow(b_ecell, ncell * 4, "cells") ||
+      !grow(b_fcnt2, ncell * 4, "cell counts") || !grow(b_foff2, ncell * 4, "cells") ||
+      !grow(b_temp, scan_u32_temp_bytes(ncell), "scan"))
+    return status;
+  u32* d_ivoff = (u32*)b_eoff.p;
+  u32* d_idx = d_ivoff + niv + 1;
+  cudaMemcpyAsync(d_ivoff, ivoff.data(), ivoff.size() * 4, cudaMemcpyHostToDevice, stream);
+  cudaMemcpyAsync(d_idx, idx.data(), idx.size() * 4, cudaMemcpyHostToDevice, stream);
+  // (1) the descriptor-pair decisions
+  LAUNCH("flow_pairs", 0.0, launch_flow_ranges(d_flows, (u32)nf, (u32)__builtin_ctz(cfg.granularity), b_franges.p,
+                                               (u32*)b_fkeep.p, stream));
+  std::vector<u32> keep(nf);
+  if (!cuda_ok(cudaMemcpyAsync(keep.data(), b_fkeep.p, nf * 4, cudaMemcpyDeviceToHost, stream), "keep")) return status;
+  // (2) canonical offsets of the full expansion and of the undecided descriptors' instances
+  LAUNCH("flow_count", 8.0 * ncell,
+         launch_flow_count_sel(d_flows, d_ivoff, d_idx, niv, bmin, ncell, tmax, (const u32*)b_fkeep.p, (u32*)b_ecnt.p,
+                               (u32*)b_fcnt2.p, stream));
+  LAUNCH("scan", 8.0 * ncell, launch_scan_exclusive_u32((u32*)b_ecnt.p, (u32*)b_ecell.p, ncell, b_temp.p, stream));
+  LAUNCH("scan", 8.0 * ncell, launch_scan_exclusive_u32((u32*)b_fcnt2.p, (u32*)b_foff2.p, ncell, b_temp.p, stream));
+  u32 last[4];
+  cudaMemcpyAsync(&last[0], (u32*)b_ecell.p + ncell - 1, 4, cudaMemcpyDeviceToHost, stream);
+  cudaMemcpyAsync(&last[1], (u32*)b_ecnt.p + ncell - 1, 4, cudaMemcpyDeviceToHost, stream);
+  cudaMemcpyAsync(&last[2], (u32*)b_foff2.p + ncell - 1, 4, cudaMemcpyDeviceToHost, stream);
+  cudaMemcpyAsync(&last[3], (u32*)b_fcnt2.p + ncell - 1, 4, cudaMemcpyDeviceToHost, stream);
+  if (!sync_check("flow counts")) return status;
+  u64 bound = 0;  // the u32 scans wrap past 2^32: refuse before (sum of per-flow maxima)
+  for (u64 d = 0; d < nf; d++)
+    if (h[d].block_lo < h[d].block_hi)
+      bound += (u64)(h[d].block_hi - h[d].block_lo) * std::min<u64>(h[d].nthreads, h[d].phi > h[d].plo ? h[d].phi - h[d].plo : 0) * h[d].count;
+  if (bound >= (1ull << 31)) return fail(SESA_ERANGE, "the flows may describe >= 2^31 records"), status;
+  const u64 total = (u64)last[0] + last[1], kept = (u64)last[2] + last[3];
+  u64 nkept_flows = 0;
+  for (u64 d = 0; d < nf; d++) nkept_flows += keep[d] ? 1 : 0;
+  // (3) instantiate the undecided descriptors only, with their canonical indices; (4) check them
+  if (!grow(b_frec, std::max<u64>(kept, 1) * sizeof(Rec), "flow records") || !grow(b_forig, std::max<u64>(kept, 1) * 4, "orig"))
+    return status;
+  if (kept)
+    LAUNCH("flow_write", 36.0 * kept,
+           launch_flow_write_sel(d_flows, d_ivoff, d_idx, niv, bmin, ncell, tmax, (const u32*)b_fkeep.p,
+                                 (const u32*)b_ecell.p, (const u32*)b_foff2.p, (Rec*)b_frec.p, (u32*)b_forig.p, stream));
+  if (!sync_check("flow write")) return status;
+  const u32 k0 = launches;
+  const sesa_status st = check_device((const sesa_access*)b_frec.p, kept, 0);
+  if (st != SESA_OK) return st;
+  launches += k0;
+  if (n_races) {
+    launches++;
+    launch_race_remap((RaceOut*)b_races_sorted.p, (u32)n_races, (const u32*)b_forig.p, stream);
+  }
+  if (oob.n_oob) {
+    u32 o = 0;
+    cudaMemcpy(&o, (const u32*)b_forig.p + oob.first_index, 4, cudaMemcpyDeviceToHost);
+    oob.first_index = o;
+  }
+  if (!sync_check("race remap")) return status;
+  info.launches = launches;
+  info.n_records = total;
+  flow_info.n_flows_checked = nkept_flows;
+  flow_info.n_records = total;
+  flow_info.n_records_checked = kept;
+  return SESA_OK;
+}
+
 // ------------------------------------------------------------------------------------------------ expand
 sesa_status sesa_trace::expand(const sesa_flow* d_flows, u64 nf, sesa_access* d_out, u64 cap, u64* n_out) {
   status = SESA_OK;
@@ -1135,6 +1232,20 @@ sesa_status sesa_race_check_warp(sesa_trace* t, const sesa_access* d_records, co
   const sesa_status st = t->check_device(d_records, n, index_base);
   t->warp_ext = nullptr;
   return st;
+}
+
+sesa_status sesa_race_check_flows(sesa_trace* t, const sesa_flow* d_flows, uint64_t n_flows, void* cuda_stream) {
+  if (!t) return SESA_EINVAL;
+  t->stream = (cudaStream_t)cuda_stream;
+  if (t->dist) return t->begin_check(0), t->fail(SESA_EINVAL, "descriptor checks need a single-GPU handle"), SESA_EINVAL;
+  return t->check_flows(d_flows, n_flows);
+}
+
+sesa_status sesa_flow_check_get(const sesa_trace* t, sesa_flow_check_info* out) {
+  if (!t || !out) return SESA_EINVAL;
+  if (!t->have_result) return SESA_ESTATE;
+  *out = t->flow_info;
+  return SESA_OK;
 }
 
 sesa_status sesa_races_get(sesa_trace* t, sesa_race* host_out, uint64_t cap, uint64_t* n_races) {

@@ -44,6 +44,8 @@ struct sesa_trace {
   DevBuf b_races, b_rkeys[2], b_rvals[2], b_races_sorted, b_rhist, b_rbase;
   DevBuf b_eoff, b_ecnt, b_ecell, b_hrec, b_dist_races, b_ctmp, b_ctotal, b_thist, b_ftmp, b_thist2, b_btmp2;
   DevBuf b_lraces;  // multi-launch checks: the races of the launches checked so far
+  DevBuf b_franges, b_fkeep, b_fcnt2, b_foff2, b_frec, b_forig;  // descriptor-level check (NEXT-2)
+  sesa_flow_check_info flow_info{};
   const void* warp_ext = nullptr;  // precise warp model: the {pc, div} extension of the records being checked
   uint32_t conflict_tdiv = 0;      // > 1: conflict tiles with identity = thread / tdiv, lockstep off
   bool have_thist2 = false;  // extents also wrote the per-tile histograms of the bucket path's first digit
@@ -65,7 +67,8 @@ struct sesa_trace {
     std::vector<DevBuf*> v = {&b_summary, &b_hist, &b_binbase, &b_lookback, &b_ctr, &b_cnt, &b_off, &b_temp,
                               &b_tflags, &b_part, &b_carry, &b_owner, &b_slots, &b_cross, &b_ccount, &b_carrytmp,
                               &b_races, &b_races_sorted, &b_rhist, &b_rbase, &b_eoff, &b_ecnt, &b_ecell,
-                              &b_hrec, &b_dist_races, &b_ctmp, &b_ctotal, &b_thist, &b_ftmp, &b_thist2, &b_btmp2, &b_lraces, &b_regions,
+                              &b_hrec, &b_dist_races, &b_ctmp, &b_ctotal, &b_thist, &b_ftmp, &b_thist2, &b_btmp2, &b_lraces, &b_franges, &b_fkeep, &b_fcnt2,
+                              &b_foff2, &b_frec, &b_forig, &b_regions,
                               &b_bhead, &b_bhscan, &b_bwf, &b_bwscan, &b_bgid, &b_bvk[0], &b_bvk[1], &b_bvi[0],
                               &b_bvi[1], &b_brh, &b_brscan, &b_bder, &b_bdpos, &b_bdj, &b_bslot, &b_btmp};
     for (auto& b : b_keys) v.push_back(&b);
@@ -125,6 +128,7 @@ struct sesa_trace {
                    const sesa::Rec* rec_entry = nullptr);
   bool step_race_sort(uint32_t nr, const sesa::RaceOut* races, uint64_t* rk0, uint32_t* rv0, uint64_t* rk1,
                       uint32_t* rv1, sesa::RaceOut* out);
+  sesa_status check_flows(const sesa_flow* d_flows, uint64_t nf);
   sesa_status expand(const sesa_flow* d_flows, uint64_t nf, sesa_access* d_out, uint64_t cap, uint64_t* n_out);
   sesa_status check_dist(const sesa_access* d_rec, uint64_t n, uint64_t index_base);
   void destroy_dist();

@@ -52,6 +52,11 @@ class sesa_kernel_stat(ctypes.Structure):
                 ("bytes", ctypes.c_double)]
 
 
+class sesa_flow_check_info(ctypes.Structure):
+    _fields_ = [("n_flows", ctypes.c_uint64), ("n_flows_checked", ctypes.c_uint64), ("n_records", ctypes.c_uint64),
+                ("n_records_checked", ctypes.c_uint64)]
+
+
 class sesa_check_info(ctypes.Structure):
     _fields_ = [("n_records", ctypes.c_uint64), ("n_entries", ctypes.c_uint64), ("n_races", ctypes.c_uint64),
                 ("n_multi", ctypes.c_uint64), ("sort_bits", ctypes.c_uint32), ("pos_bits", ctypes.c_uint32), ("digit_bits", ctypes.c_uint32),
@@ -65,7 +70,7 @@ EXPORTS = ["sesa_trace_create", "sesa_trace_create_dist", "sesa_nccl_unique_id",
            "sesa_race_check_host", "sesa_races_get", "sesa_races_device", "sesa_expand", "sesa_trace_set_profiling",
            "sesa_trace_info", "sesa_trace_kernel_stats", "sesa_trace_destroy", "sesa_status_str", "sesa_last_error",
            "sesa_abi_version", "sesa_race_check_loopback", "sesa_trace_set_regions", "sesa_oob_get",
-           "sesa_race_check_launches", "sesa_race_check_warp"]
+           "sesa_race_check_launches", "sesa_race_check_warp", "sesa_race_check_flows", "sesa_flow_check_get"]
 
 _lib = None
 
@@ -87,6 +92,8 @@ def load() -> ctypes.CDLL:
     lib.sesa_race_check_host.argtypes = [P, P, U64, U64, P]
     lib.sesa_race_check_launches.argtypes = [P, P, U64, P, U32, U64, P]
     lib.sesa_race_check_warp.argtypes = [P, P, P, U64, U64, P]
+    lib.sesa_race_check_flows.argtypes = [P, P, U64, P]
+    lib.sesa_flow_check_get.argtypes = [P, ctypes.POINTER(sesa_flow_check_info)]
     lib.sesa_race_check_loopback.argtypes = [ctypes.POINTER(sesa_config), P, P, I, U64, P, PP]
     lib.sesa_races_get.argtypes = [P, P, U64, ctypes.POINTER(U64)]
     lib.sesa_races_device.argtypes = [P, PP, ctypes.POINTER(U64)]
@@ -181,6 +188,19 @@ class Trace:
         if st != SESA_OK:
             self._raise(st, "sesa_race_check_warp")
         return self.n_races()
+
+    def check_flows(self, d_flows, n_flows: int, stream=None) -> int:
+        """Descriptor-level check (NEXT-2): the race list of the expansion of n_flows device descriptors."""
+        ptr = d_flows if isinstance(d_flows, int) else d_flows.data_ptr()
+        st = self.lib.sesa_race_check_flows(self.h, ctypes.c_void_p(ptr), n_flows, _stream_ptr(stream))
+        if st != SESA_OK:
+            self._raise(st, "sesa_race_check_flows")
+        return self.n_races()
+
+    def flow_info(self) -> dict:
+        i = sesa_flow_check_info()
+        self.lib.sesa_flow_check_get(self.h, ctypes.byref(i))
+        return {k: getattr(i, k) for k, _ in sesa_flow_check_info._fields_}
 
     def check_host(self, h_records: np.ndarray, index_base: int = 0, stream=None) -> int:
         a = np.ascontiguousarray(h_records)

@@ -569,3 +569,41 @@ def test_precise_warp_large(sesa):
     t.close()
     exp = O.check_warp(r, e, warp_size=32)
     assert len(exp) > 1000 and got.tobytes() == exp.tobytes()
+
+
+# ------------------------------------------------------------------------------------------------ descriptors (NEXT-2)
+def _flows_dev(fl):
+    return torch.from_numpy(np.ascontiguousarray(fl).view(np.uint8).reshape(-1)).cuda()
+
+
+@pytest.mark.parametrize("name", ["f1", "f2", "f4", "f5", "c1", "c2", "c2m", "c2m7"])
+def test_flow_check_equals_expand_then_check(sesa, name):
+    """sesa_race_check_flows == expand-then-check (the oracle: oracle_expand + the checker) on the paper
+    fixtures, C1, the full C2 and its mutants; race-free descriptor pairs are decided without instantiation."""
+    fl = {"f1": G.f1_flows(), "f2": G.f2_flows(), "f4": G.f4_flows(), "f5": G.f5_flows(), "c1": G.c1_flows(),
+          "c2": G.c2_flows(), "c2m": G.c2_mutant_flows(drop_barrier=3, gx=2, gy=2, K=64),
+          "c2m7": G.c2_mutant_flows(drop_barrier=7)}[name]
+    t = sesa.Trace(32, 0, 4)
+    t.check_flows(_flows_dev(fl), len(fl))
+    got = t.races()
+    info = t.flow_info()
+    t.close()
+    exp = O.check(O.expand(fl), method="partitioned")
+    assert got.tobytes() == exp.tobytes()
+    assert info["n_records"] == len(O.expand(fl)) if name != "c2" else info["n_records"] == 18300928
+    if name == "c2":  # race-free by construction: decided arithmetically, nothing instantiated
+        assert info["n_records_checked"] == 0 and len(got) == 0
+    if name == "c2m7":  # only the descriptors of the merged intervals are instantiated
+        assert 0 < info["n_records_checked"] < info["n_records"] // 4
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_flow_check_random_descriptors(sesa, seed):
+    fl = G.random_flows(seed, nd=4 + seed % 12)
+    for ls, gran in ((0, 4), (1, 1), (1, 8)):
+        t = sesa.Trace(4 if seed % 2 else 32, ls, gran)
+        t.check_flows(_flows_dev(fl), len(fl))
+        got = t.races()
+        t.close()
+        exp = O.check(O.expand(fl), warp_size=4 if seed % 2 else 32, lockstep=ls, granularity=gran)
+        assert got.tobytes() == exp.tobytes(), (seed, ls, gran, len(got), len(exp))

@@ -183,7 +183,7 @@ def test_c1_truth_by_construction():
 
 
 # ------------------------------------------------------------------------------------------------ expansion
-@pytest.mark.parametrize("name", ["f1", "f1c", "f2", "f5", "c1"])
+@pytest.mark.parametrize("name", ["f1", "f1c", "f2", "f5", "c1", "f4"])
 def test_expand_matches_direct(name):
     direct, fl = {
         "f1": (G.f1_race(), G.f1_flows()),
@@ -191,6 +191,7 @@ def test_expand_matches_direct(name):
         "f2": (G.f2_reduction(), G.f2_flows()),
         "f5": (G.f5_binning(), G.f5_flows()),
         "c1": (G.c1(), G.c1_flows()),
+        "f4": (G.f4_histo_prescan(), G.f4_flows()),
     }[name]
     ex = O.expand(fl)
     assert len(ex) == len(direct)
