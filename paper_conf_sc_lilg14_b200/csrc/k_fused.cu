@@ -113,7 +113,7 @@ struct FusedArgs {
 // UNST (the bucket path, which needs no stable order within a digit): the count atomic's return value is the
 // key's rank within its (warp, digit) group, and the ranking loop is skipped.
 template <int NP, bool UNST = false>
-__global__ void __launch_bounds__(FUSED_THREADS, FUSED_MINB) fused_extract_pass0_kernel(FusedArgs A) {
+__global__ void __launch_bounds__(FUSED_THREADS, UNST ? FUSED_UMINB : FUSED_MINB) fused_extract_pass0_kernel(FusedArgs A) {
   constexpr int THREADS = FUSED_THREADS, ITEMS = FUSED_ITEMS, WARPS = THREADS / 32, TILE = FUSED_TILE;
   extern __shared__ __align__(16) unsigned char smem[];
   u64* keys_s = reinterpret_cast<u64*>(smem);              // [TILE]
@@ -266,7 +266,9 @@ void launch_fused_extract_pass0(const u32* gran, u64 n, const KeyLayout& L, u32 
                        (const void*)fused_extract_pass0_kernel<3>, (const void*)fused_extract_pass0_kernel<4>};
   const size_t sm = fused_smem(npass);
   // persistent CTAs: one full wave at the occupancy of the largest variant
-  const int grid = dev_sm_count() * blocks_per_sm(ks[3], FUSED_THREADS, fused_smem(4));
+  const int grid = dev_sm_count() * (unstable ? blocks_per_sm((const void*)fused_extract_pass0_kernel<1, true>,
+                                                               FUSED_THREADS, fused_smem(1))
+                                              : blocks_per_sm(ks[3], FUSED_THREADS, fused_smem(4)));
   smem_optin(ks[std::min<u32>(npass, 4) - 1], sm);
   FusedArgs A;
   A.gran = gran;
