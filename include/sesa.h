@@ -196,8 +196,10 @@ sesa_status sesa_race_check(sesa_trace *t, const sesa_access *d_records, uint64_
 sesa_status sesa_race_check_loopback(const sesa_config *cfg, const sesa_access *d_records, const uint64_t *offs,
                                      int world, uint64_t index_base, void *cuda_stream, sesa_trace **out);
 
-/* Same, for records in HOST memory: the library copies them to the device (chunked through pinned staging
- * when h_records is pageable) inside the call.  This is the end-to-end entry point. */
+/* Same, for records in HOST memory: the library copies them to the device inside the call — one DMA when
+ * h_records is page-locked (cudaHostAlloc / registered), else in 64 MiB chunks through two page-locked staging
+ * buffers (the host copy of a chunk overlaps the DMA of the previous one).  The device copy is owned by the
+ * handle (grow-only).  This is the end-to-end entry point. */
 sesa_status sesa_race_check_host(sesa_trace *t, const sesa_access *h_records, uint64_t n, uint64_t index_base,
                                  void *cuda_stream);
 

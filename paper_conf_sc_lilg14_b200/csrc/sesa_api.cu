@@ -1204,9 +1204,33 @@ sesa_status sesa_race_check_host(sesa_trace* t, const sesa_access* h_records, ui
   if (n == 0) return sesa_race_check(t, nullptr, 0, index_base, cuda_stream);
   if (!h_records) return t->fail(SESA_EINVAL, "h_records is NULL"), t->status;
   if (!t->grow(t->b_hrec, n * sizeof(sesa_access), "record copy")) return t->status;
-  if (!t->cuda_ok(cudaMemcpyAsync(t->b_hrec.p, h_records, n * sizeof(sesa_access), cudaMemcpyHostToDevice, t->stream),
-                  "records H2D"))
-    return t->status;
+  const size_t bytes = n * sizeof(sesa_access);
+  cudaPointerAttributes pa;
+  const bool pinned = cudaPointerGetAttributes(&pa, h_records) == cudaSuccess && pa.type == cudaMemoryTypeHost;
+  cudaGetLastError();
+  if (pinned) {  // page-locked: one DMA
+    if (!t->cuda_ok(cudaMemcpyAsync(t->b_hrec.p, h_records, bytes, cudaMemcpyHostToDevice, t->stream), "records H2D"))
+      return t->status;
+  } else {
+    // pageable: chunked through two page-locked staging buffers; the host copy of chunk i + 1 overlaps the DMA
+    // of chunk i
+    const size_t CH = 64ull << 20;
+    if (!t->h_pinned && !t->cuda_ok(cudaMallocHost(&t->h_pinned, 2 * CH), "pinned staging")) return t->status;
+    cudaEvent_t ev[2];
+    for (auto& e : ev) cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+    bool ok = true;
+    for (size_t off = 0, i = 0; off < bytes && ok; off += CH, i++) {
+      const size_t len = std::min(CH, bytes - off);
+      char* stage = (char*)t->h_pinned + (i & 1) * CH;
+      if (i >= 2) cudaEventSynchronize(ev[i & 1]);  // its previous DMA has finished
+      memcpy(stage, (const char*)h_records + off, len);
+      ok = t->cuda_ok(cudaMemcpyAsync((char*)t->b_hrec.p + off, stage, len, cudaMemcpyHostToDevice, t->stream),
+                      "records H2D") &&
+           t->cuda_ok(cudaEventRecord(ev[i & 1], t->stream), "records H2D");
+    }
+    for (auto& e : ev) cudaEventDestroy(e);  // (destroy after pending records complete is allowed)
+    if (!ok) return t->status;
+  }
   return sesa_race_check(t, (const sesa_access*)t->b_hrec.p, n, index_base, cuda_stream);
 }
 

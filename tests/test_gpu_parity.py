@@ -607,3 +607,20 @@ def test_flow_check_random_descriptors(sesa, seed):
         t.close()
         exp = O.check(O.expand(fl), warp_size=4 if seed % 2 else 32, lockstep=ls, granularity=gran)
         assert got.tobytes() == exp.tobytes(), (seed, ls, gran, len(got), len(exp))
+
+
+def test_host_entry_pageable_chunks_and_pinned(sesa):
+    """sesa_race_check_host: a pageable 96 MB array goes through the chunked pinned staging (two 64 MiB
+    buffers), a page-locked one by one DMA; both give the oracle's list."""
+    from sesagen import configs as C
+    n = 3_000_000
+    r = C.rnd_host(n, 31337, blocks=256, threads=512, intervals=2, words=1 << 22, shared_frac=0.0, sizes=(4,),
+                   unaligned=False, values=3)
+    exp = O.check(r, method="partitioned")
+    t = trace(sesa)
+    t.check_host(r)
+    assert t.races().tobytes() == exp.tobytes()
+    pinned = torch.from_numpy(r.view(np.uint8)).pin_memory()
+    t.check_host_ptr(pinned.data_ptr(), n)
+    assert t.races().tobytes() == exp.tobytes()
+    t.close()
