@@ -235,7 +235,10 @@ def reference_arm(args, rank, world):
             "cpu_baseline": {"value": value, "unit": "Grec/s", "cores": hi["cores"], "kind": "oracle",
                              "sample": f"{sample} (oracle_check_partitioned, {hi['cores']} threads)", "host": hi},
             "e2e": {"value": value, "unit": "Grec/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
-    print(json.dumps(line), flush=True)
+    print(json.dumps(line), file=JSON_OUT, flush=True)
+
+
+JSON_OUT = sys.stdout
 
 
 def main():
@@ -268,6 +271,12 @@ def main():
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # stdout carries exactly one JSON line: anything native libraries print to fd 1 (NCCL's version banner at
+    # communicator init, ...) goes to stderr instead
+    global JSON_OUT
+    JSON_OUT = os.fdopen(os.dup(1), "w")
+    sys.stdout.flush()
+    os.dup2(2, 1)
     if args.impl == "reference":
         reference_arm(args, rank, world)
         return
@@ -422,7 +431,7 @@ def main():
                             for k, v in sorted(kstats.items(), key=lambda kv: -kv[1]["ms"])},
                 "dominant_kernel": dom, "e2e": e2e, "cpu_baseline": cpu, "clocks": clk.summary(), "nvlink": nvlink,
                 "full_size_check": check}
-        print(json.dumps(line), flush=True)
+        print(json.dumps(line), file=JSON_OUT, flush=True)
     trace.close()
     if pg:
         pg.destroy_process_group()

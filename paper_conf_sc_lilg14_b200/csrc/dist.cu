@@ -145,13 +145,12 @@ static bool partition(sesa_trace* t, RankBufs& B, const u64* in, u64 n, u32 W, i
   a.out_src = mode == 1 ? (u32*)B.src.p : nullptr;
   if (n) {
     const unsigned grid = (unsigned)std::min<u64>((nch + 7) / 8, (u64)t->num_sms * 8);
-    t->launches += 3;
-    if (getenv("SESA_SYNC_DEBUG")) fprintf(stderr, "[sesa debug] partition n=%llu W=%u grid=%u nch=%llu\n",
-                                           (unsigned long long)n, W, grid, (unsigned long long)nch);
+    t->launch_begin("owner_partition");  // (3 kernels + the scan's one: kernels_of counts them)
     partition_kernel<false><<<grid, PT_THREADS, 0, t->stream>>>(a);
     launch_scan_exclusive_u32((u32*)B.pcnt.p, (u32*)B.poff.p, nch * W, B.ptmp.p, t->stream);
     partition_kernel<true><<<grid, PT_THREADS, 0, t->stream>>>(a);
     bucket_totals_kernel<<<1, 32, 0, t->stream>>>((u32*)B.pcnt.p, (u32*)B.poff.p, nch, W, (u64*)B.tot.p);
+    t->launch_end(24.0 * (double)n);
     if (!t->cuda_ok(cudaMemcpyAsync(out_tot, B.tot.p, W * 8, cudaMemcpyDeviceToHost, t->stream), "totals")) return false;
   } else {
     for (u32 i = 0; i < W; i++) out_tot[i] = 0;
@@ -440,8 +439,9 @@ static sesa_status dist_check(std::vector<sesa_trace*>& ts, std::vector<RankIO>&
     for (int s = 0; s < W; s++) mr += rcnt[r][s];
     std::swap(t->b_keys[0], t->b_keys[1]);  // received keys -> b_keys[0]
     int cur = 0;
-    ok = t->grow(t->b_keys[1], mr * 8 + 64, "keys") && t->step_hist(mr) && t->step_sort(mr, &cur) &&
-         t->step_compact(cur, mr, &comp[r], &m2[r]) &&
+    bool used = false;  // the bucket path on the received keys when their granules spread evenly (C5)
+    ok = t->grow(t->b_keys[1], mr * 8 + 64, "keys") && t->try_bucket_keys(mr, &comp[r], &m2[r], &used) &&
+         (used || (t->step_hist(mr) && t->step_sort(mr, &cur) && t->step_compact(cur, mr, &comp[r], &m2[r]))) &&
          partition(t, t->ds->b, comp[r], m2[r], W, 1, bases.data(), qcnt[r].data());
     sendp[r] = t->ds->b.send.p;
     reqb[r] = &t->ds->b.reqin;
@@ -533,6 +533,11 @@ static sesa_status dist_check(std::vector<sesa_trace*>& ts, std::vector<RankIO>&
 
 // ------------------------------------------------------------------------------------------------ handle glue
 sesa_status sesa_trace::check_dist(const sesa_access* d_rec, uint64_t n, uint64_t index_base) {
+  if (world == 1) {  // one rank owns every location: nothing to exchange, the single-GPU pipeline is the check
+    const sesa_status s = check_device(d_rec, n, index_base);
+    if (s == SESA_OK) std::swap(b_dist_races, b_races_sorted);  // rank 0's merged list lives in b_dist_races
+    return s;
+  }
   std::vector<sesa_trace*> ts = {this};
   std::vector<RankIO> io = {{(const Rec*)d_rec, n, index_base}};
   NcclExchanger ex(ds->comm, rank, world, ds->b.ag);

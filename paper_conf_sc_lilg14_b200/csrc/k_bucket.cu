@@ -267,12 +267,38 @@ __global__ void bucket_sample_kernel(const u32* __restrict__ gran, u32 n, u32 st
   }
 }
 
+// the same from a key array: chunk = key >> shift
+__global__ void bucket_sample_keys_kernel(const u64* __restrict__ keys, u32 m, u32 stride, u32 shift, u32 nchunks,
+                                          u32* __restrict__ hist) {
+  const u64 step = (u64)gridDim.x * blockDim.x * stride;
+  for (u64 i0 = (u64)(blockIdx.x * blockDim.x + (threadIdx.x & ~31u)) * stride; i0 < m; i0 += step) {
+    const u64 i = i0 + (u64)(threadIdx.x & 31) * stride;
+    const u32 c = i < m ? (u32)min(keys[i] >> shift, (u64)~0u) : ~0u;
+    const unsigned peers = __match_any_sync(~0u, c);
+    if (c < nchunks && (threadIdx.x & 31) == __ffs(peers) - 1) atomicAdd(&hist[c], (u32)__popc(peers));
+  }
+}
+
 __global__ void bucket_sample_max_kernel(const u32* __restrict__ hist, u32 nchunks, u32* __restrict__ out) {
   u32 mx = 0;
   for (u32 c = blockIdx.x * blockDim.x + threadIdx.x; c < nchunks; c += gridDim.x * blockDim.x) mx = max(mx, hist[c]);
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) mx = max(mx, __shfl_xor_sync(~0u, mx, o));
   if ((threadIdx.x & 31) == 0) atomicMax(out, mx);
+}
+
+u32 bucket_sample_keys_max(const u64* keys, u32 m, u32 shift, u32 nchunks, void* temp, cudaStream_t st, u32* h_max,
+                           u32* samples, u32 want) {
+  u32* hist = reinterpret_cast<u32*>(temp);
+  u32* mx = hist + nchunks;
+  const u32 stride = std::max<u32>(1, m / want);
+  *samples = (m + stride - 1) / stride;
+  cudaMemsetAsync(temp, 0, ((size_t)nchunks + 1) * 4, st);
+  const u32 grid = (u32)std::min<u64>(((u64)*samples + 255) / 256, (u64)dev_sm_count() * 8);
+  bucket_sample_keys_kernel<<<grid, 256, 0, st>>>(keys, m, stride, shift, nchunks, hist);
+  bucket_sample_max_kernel<<<std::min<u32>((nchunks + 255) / 256, 1024u), 256, 0, st>>>(hist, nchunks, mx);
+  cudaMemcpyAsync(h_max, mx, 4, cudaMemcpyDeviceToHost, st);
+  return 2;
 }
 
 size_t bucket_temp_bytes(u32 nchunks) {

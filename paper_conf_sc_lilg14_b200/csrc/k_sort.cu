@@ -236,7 +236,7 @@ __device__ __forceinline__ u64 gtime() {
 __device__ unsigned long long* g_prof = nullptr;
 
 template <int THREADS, int ITEMS, int LBW, bool FULL, bool LATE_LB, int S, bool BAL, int TMA, int MIX = 0,
-          bool UNST = false>
+          int UNST = 0>
 __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64* __restrict__ kout, u32 m, u32 shift,
                                                const u64* __restrict__ bin_base, u64* __restrict__ lookback,
                                                u32 epoch, u32 tile, unsigned char* smem, unsigned long long* prof,
@@ -282,12 +282,12 @@ __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64*
     for (int i = 0; i < ITEMS; i++)
       if (FULL || i < nv) k[i] = __ldcs(kin + wbase + (u64)i * 32);
   }
-  // (UNST: the input's ~0 sentinels — padding of 32-aligned digit runs — are no keys)
-  //  UNST passes sort by the TOP digit (nothing above it), so a sentinel is the only key whose shifted value is
-  //  >= RADIX)
+  // (UNST = 0: stable pass; 1: unstable pass on the TOP digit whose input carries ~0 sentinels — padding of
+  //  32-aligned digit runs: nothing lies above the top digit, so a sentinel is the only key whose shifted value is
+  //  >= RADIX; 2: unstable pass on any digit, no sentinels)
   auto digit = [&](int i) -> u32 {
     if (!(FULL || i < nv)) return (u32)RADIX;
-    if (UNST) { const u32 d9 = (u32)(k[i] >> shift) & (2 * RADIX - 1); return d9 < RADIX ? d9 : (u32)RADIX; }
+    if (UNST == 1) { const u32 d9 = (u32)(k[i] >> shift) & (2 * RADIX - 1); return d9 < RADIX ? d9 : (u32)RADIX; }
     return (u32)((k[i] >> shift) & (RADIX - 1));
   };
   // rank streams: items [s*IPS, (s+1)*IPS) of a warp form stream s (stable order = warp, stream, item, lane),
@@ -439,7 +439,7 @@ __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64*
 }
 
 template <int THREADS, int ITEMS, int MINB, int LBW, bool LATE_LB, int S, bool BAL, int TMA, int MIX = 0,
-          bool UNST = false>
+          int UNST = 0>
 __global__ void __launch_bounds__(THREADS, MINB) onesweep2_kernel(const u64* __restrict__ kin, u64* __restrict__ kout,
                                                                   u32 m, u32 shift, const u64* __restrict__ bin_base,
                                                                   u64* __restrict__ lookback,
@@ -485,11 +485,13 @@ __global__ void __launch_bounds__(THREADS, MINB) onesweep2_kernel(const u64* __r
 // the measured configuration: 256 x 32 keys, 2 CTAs/SM, look-back after ranking, one rank stream,
 // prologue bulk copies (TMA 2), every 4th item's peers by ballots (MIX 4)
 #define OS_CFG OS_THREADS, OS_ITEMS, OS_MINB, OS_LBW, true, 1, false, 2, 4
-// the bucket path's partition pass (no stable order needed)
+// the bucket path's partition passes (no stable order needed): on the top digit with sentinels (1), on a lower
+// digit of a key array (2)
 // (measured on C5, per 1e9 keys: 256 x 32 at 2 CTAs/SM 4.09 ms; 256 x 24 at 3: 4.21; 256 x 20 at 3: 4.36;
 // 512 x 16 at 2: 4.44; 256 x 16 at 4: 4.69)
 constexpr int PT_THREADS = 256, PT_ITEMS = 32, PT_MINB = 2;
-#define OS_UCFG PT_THREADS, PT_ITEMS, PT_MINB, OS_LBW, true, 1, false, 2, 4, true
+#define OS_UCFG PT_THREADS, PT_ITEMS, PT_MINB, OS_LBW, true, 1, false, 2, 4, 1
+#define OS_UCFG2 PT_THREADS, PT_ITEMS, PT_MINB, OS_LBW, true, 1, false, 2, 4, 2
 
 static size_t onesweep2_smem() {
   constexpr int WARPS = OS_THREADS / 32;
@@ -499,15 +501,47 @@ static size_t onesweep2_smem() {
 
 u32 sort_tile_keys() { return OS_TILE; }
 
-// unstable partition pass (the bucket path: chunk order only, survivors are sorted per chunk afterwards)
+// unstable partition pass (the bucket path: chunk order only, survivors are sorted per chunk afterwards);
+// top = the pass's digit is the key's top digit and its input may hold ~0 sentinels
 void launch_partition_pass(const u64* kin, u64* kout, u32 m, u32 shift, const u64* bin_base, u64* lookback,
-                           u32* tile_ctr, u32 epoch, cudaStream_t st) {
+                           u32* tile_ctr, u32 epoch, cudaStream_t st, bool top) {
   if (!m) return;
   constexpr int WARPS = PT_THREADS / 32, TILE = PT_THREADS * PT_ITEMS;
   const size_t sm = (size_t)TILE * 8 + (size_t)WARPS * RADIX * 4 + RADIX * 4 + (WARPS + 1) * 4;
-  smem_optin((const void*)onesweep2_kernel<OS_UCFG>, sm);
   const u32 tiles = (u32)((m + TILE - 1) / TILE);
-  onesweep2_kernel<OS_UCFG><<<tiles, PT_THREADS, sm, st>>>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch);
+  if (top) {
+    smem_optin((const void*)onesweep2_kernel<OS_UCFG>, sm);
+    onesweep2_kernel<OS_UCFG><<<tiles, PT_THREADS, sm, st>>>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch);
+  } else {
+    smem_optin((const void*)onesweep2_kernel<OS_UCFG2>, sm);
+    onesweep2_kernel<OS_UCFG2><<<tiles, PT_THREADS, sm, st>>>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch);
+  }
+}
+
+// bin bases of a digit histogram with every run padded to a multiple of 32 (the bucket path's first pass on a key
+// array); the pad slots of kout get ~0 sentinels; *mpad = padded length
+__global__ void padded_bin_base_kernel(const u32* __restrict__ hist, u64* __restrict__ base, u64* __restrict__ kout,
+                                       u32* __restrict__ mpad) {
+  __shared__ u32 s[RADIX];
+  const u32 d = threadIdx.x, c = hist[d];
+  s[d] = (c + 31u) & ~31u;
+  __syncthreads();
+  if (d == 0) {
+    u32 acc = 0;
+    for (int i = 0; i < RADIX; i++) {
+      const u32 v = s[i];
+      s[i] = acc;
+      acc += v;
+    }
+    *mpad = acc;
+  }
+  __syncthreads();
+  base[d] = s[d];
+  for (u32 q = s[d] + c; q < s[d] + ((c + 31u) & ~31u); q++) kout[q] = ~0ull;
+}
+
+void launch_padded_bin_base(const u32* hist, u64* base, u64* kout, u32* mpad, cudaStream_t st) {
+  padded_bin_base_kernel<<<1, RADIX, 0, st>>>(hist, base, kout, mpad);
 }
 
 void launch_onesweep(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m, u32 shift, const u64* bin_base,

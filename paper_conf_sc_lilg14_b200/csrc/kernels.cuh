@@ -58,6 +58,8 @@ size_t bucket_temp_bytes(u32 nchunks);
 // sample of the chunk sizes from the extents' granule array: *h_max (host, after a sync) = largest sampled count
 u32 bucket_sample_max(const u32* gran, u32 n, u32 gmin_lo, u32 nchunks, void* temp, cudaStream_t st, u32* h_max,
                       u32* samples, u32 want);
+u32 bucket_sample_keys_max(const u64* keys, u32 m, u32 shift, u32 nchunks, void* temp, cudaStream_t st, u32* h_max,
+                           u32* samples, u32 want);
 u32 launch_bucket_compact(u64* keys, u64* stage, u32 m, u32 pos_bits, u32 nchunks, void* temp, u32* total,
                           cudaStream_t st);
 
@@ -77,7 +79,9 @@ void launch_onesweep(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m
 u32 sort_tile_keys();
 // the same pass without the stable order (the bucket path): counting atomics give the ranks
 void launch_partition_pass(const u64* kin, u64* kout, u32 m, u32 shift, const u64* bin_base, u64* lookback,
-                           u32* tile_ctr, u32 epoch, cudaStream_t st);
+                           u32* tile_ctr, u32 epoch, cudaStream_t st, bool top = true);
+// padded (32-aligned runs) bin bases of one digit histogram; sentinels into kout's pad slots; *mpad (device)
+void launch_padded_bin_base(const u32* hist, u64* base, u64* kout, u32* mpad, cudaStream_t st);
 inline u32 sort_tiles(u64 m) { return (u32)((m + 2047) / 2048); }  // upper bound (smallest tile: 2048 keys)
 // race-list keys: (race key, index) -> histograms for npass digits starting at bit 0
 void launch_hist_keys(const u64* keys, u32 m, u32 npass, u32* hist, cudaStream_t st);

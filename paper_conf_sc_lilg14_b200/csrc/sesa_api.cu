@@ -79,7 +79,8 @@ static unsigned kernels_of(const char* name) {
   static const struct {
     const char* n;
     unsigned k;
-  } tab[] = {{"tile_offsets", 3}, {"compact", 4}, {"carry", 3}, {"alltoall", 0}, {"flow_pairs", 2}};  // alltoall: NCCL's kernels
+  } tab[] = {{"tile_offsets", 3}, {"compact", 4}, {"carry", 3}, {"alltoall", 0}, {"flow_pairs", 2},
+                 {"owner_partition", 4}};  // alltoall: NCCL's kernels
   for (const auto& e : tab)
     if (!strcmp(e.n, name)) return e.k;
   return 1;
@@ -408,6 +409,84 @@ bool sesa_trace::step_bucket(u64 n, u32 nchunks, u64** comp, u32* m2) {
   if (!cuda_ok(cudaMemcpyAsync(m2, b_ctotal.p, 4, cudaMemcpyDeviceToHost, stream), "bucket count")) return false;
   if (!sync_check("bucket")) return false;
   info.n_multi = *m2;
+  return true;
+}
+
+// Bucket path on a key array (b_keys[0], m keys of the current layout) — the distributed check's received keys,
+// or a single-GPU trace the fused first pass does not cover: an unstable pass on key_hi bits [14, 22) into
+// 32-aligned runs (padded bin bases, sentinels), one on [22, 30), the chunk bitmaps.  *used = false (and true
+// returned) when the trace is not eligible: the caller sorts in full.
+bool sesa_trace::try_bucket_keys(u64 m, u64** comp, u32* m2, bool* used) {
+  *used = false;
+  const KeyLayout& L = layout;
+  if (m < BUCKET_MIN_N || L.both || (L.single_space == SP_GLOBAL && L.lowG) || L.sort_bits <= HYB_LO + RADIX_BITS ||
+      L.sort_bits > HYB_LO + 2 * RADIX_BITS || m >= (1ull << 31))
+    return true;
+  const u32 nc = (u32)((((1ull << L.sort_bits) - 1) >> HYB_CHUNK) + 1);
+  if (!grow(b_btmp2, bucket_temp_bytes(nc), "bucket temp")) return false;
+  const double mean = (double)m / nc;
+  for (u32 want : {1u << 16, 1u << 22}) {
+    u32 hmax = 0, samples = 0;
+    LAUNCH("bucket_sample", 8.0 * (double)want,
+           launches += bucket_sample_keys_max((const u64*)b_keys[0].p, (u32)m, L.pos_bits + HYB_CHUNK, nc, b_btmp2.p,
+                                              stream, &hmax, &samples, want) - 1);
+    if (!sync_check("bucket sample")) return false;
+    const double est_max = (double)hmax * (double)m / (double)std::max(1u, samples);
+    if (want < (1u << 22) ? est_max > 32.0 * mean + 65536.0 : (est_max > 4.0 * mean + 2048.0 || est_max > (double)(1u << 20)))
+      return true;
+  }
+  info.bucket_path = 1;
+  if (!grow(b_keys[1], (m + 32 * RADIX) * 8 + 64, "keys") || !grow(b_hist, 2 * RADIX * 4, "hist") ||
+      !grow(b_binbase, 2 * RADIX * 8, "binbase") || !grow(b_ctotal, 16, "bucket count"))
+    return false;
+  cudaMemsetAsync(b_hist.p, 0, 2 * RADIX * 4, stream);
+  LAUNCH("hist", 8.0 * m, launch_hist_keys_shift((const u64*)b_keys[0].p, (u32)m, 2, L.pos_bits + HYB_LO,
+                                                 (u32*)b_hist.p, stream));
+  std::vector<u32> rowB(RADIX);
+  if (!cuda_ok(cudaMemcpyAsync(rowB.data(), (u32*)b_hist.p + RADIX, RADIX * 4, cudaMemcpyDeviceToHost, stream), "hist") ||
+      !sync_check("bucket hist"))
+    return false;
+  const bool pass2 = *std::max_element(rowB.begin(), rowB.end()) != m;
+  u32 mpad = (u32)m;
+  if (pass2) {  // 32-aligned digit runs (sentinels in the pad slots) for the second, unstable pass
+    LAUNCH("bin_base", 0.0, launch_padded_bin_base((const u32*)b_hist.p, (u64*)b_binbase.p, (u64*)b_keys[1].p,
+                                                   (u32*)b_ctotal.p + 2, stream));
+    LAUNCH("bin_base", 0.0, launch_bin_base((const u32*)b_hist.p + RADIX, (u64*)b_binbase.p + RADIX, 1, stream));
+    if (!cuda_ok(cudaMemcpyAsync(&mpad, (u32*)b_ctotal.p + 2, 4, cudaMemcpyDeviceToHost, stream), "padded") ||
+        !sync_check("padded bins"))
+      return false;
+  } else {
+    LAUNCH("bin_base", 0.0, launch_bin_base((const u32*)b_hist.p, (u64*)b_binbase.p, 1, stream));
+  }
+  const u32 stiles = sort_tiles(std::max<u64>(mpad, m));
+  if (!grow(b_lookback, (size_t)stiles * RADIX * 8, "lookback") || !grow(b_ctr, 64 * 4, "counters")) return false;
+  if (b_lookback.cap != lookback_cleared) {
+    cudaMemsetAsync(b_lookback.p, 0, b_lookback.cap, stream);
+    lookback_cleared = b_lookback.cap;
+    epoch = 0;
+  }
+  cudaMemsetAsync(b_ctr.p, 0, 64 * 4, stream);
+  for (int pass = 0; pass < (pass2 ? 2 : 1); pass++) {
+    if (++epoch >= 256) {
+      cudaMemsetAsync(b_lookback.p, 0, b_lookback.cap, stream);
+      epoch = 1;
+    }
+    LAUNCH("partition_pass", 16.0 * m,
+           launch_partition_pass((u64*)b_keys[pass].p, (u64*)b_keys[pass ^ 1].p, pass ? mpad : (u32)m,
+                                 L.pos_bits + HYB_LO + pass * RADIX_BITS, (u64*)b_binbase.p + pass * RADIX,
+                                 (u64*)b_lookback.p, (u32*)b_ctr.p + pass, epoch, stream, pass == 1));
+  }
+  info.sort_passes = pass2 ? 2 : 1;
+  const int cur = pass2 ? 0 : 1;
+  LAUNCH("bucket", 8.0 * m,
+         launches += launch_bucket_compact((u64*)b_keys[cur].p, (u64*)b_keys[cur ^ 1].p, (u32)m, L.pos_bits, nc,
+                                           b_btmp2.p, (u32*)b_ctotal.p, stream) - 1);
+  *comp = (u64*)b_keys[cur].p;
+  if (!cuda_ok(cudaMemcpyAsync(m2, b_ctotal.p, 4, cudaMemcpyDeviceToHost, stream), "bucket count") ||
+      !sync_check("bucket"))
+    return false;
+  info.n_multi = *m2;
+  *used = true;
   return true;
 }
 
@@ -887,7 +966,13 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
   if (fused) {
     if (!step_extract_fused(rec, n) || !step_sort(m, &cur, 1, 1)) return status;
   } else {
-    if (!step_extract(rec, n, m, 0, S.multi != 0) || !step_sort(m, &cur)) return status;
+    if (!step_extract(rec, n, m, 0, S.multi != 0)) return status;
+    bool used = false;
+    u64* bcomp = nullptr;
+    u32 bm2 = 0;
+    if (!try_bucket_keys(m, &bcomp, &bm2, &used)) return status;
+    if (used) return finish_check(bcomp, bm2, rec, index_base);
+    if (!step_sort(m, &cur)) return status;
   }
   u64* comp = nullptr;
   u32 m2 = 0;

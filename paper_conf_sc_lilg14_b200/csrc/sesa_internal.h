@@ -119,6 +119,7 @@ struct sesa_trace {
   bool step_extract_fused(const sesa::Rec* rec, uint64_t n);
   bool bucket_choose(uint64_t n, uint64_t* gmin_aligned, uint32_t* nbits, uint32_t* nchunks);
   bool step_bucket(uint64_t n, uint32_t nchunks, uint64_t** comp, uint32_t* m2);
+  bool try_bucket_keys(uint64_t m, uint64_t** comp, uint32_t* m2, bool* used);
   bool step_sort(uint64_t m, int* cur_out, uint32_t first_pass = 0, int cur0 = 0);
   bool step_compact(int cur, uint64_t m, uint64_t** comp, uint32_t* m2);
   bool step_conflict(const uint64_t* comp, uint32_t m2, const sesa::Rec* rec, uint32_t rec_pos_base,

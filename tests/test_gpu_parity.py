@@ -624,3 +624,20 @@ def test_host_entry_pageable_chunks_and_pinned(sesa):
     t.check_host_ptr(pinned.data_ptr(), n)
     assert t.races().tobytes() == exp.tobytes()
     t.close()
+
+
+@pytest.mark.slow
+def test_bucket_path_on_key_arrays(sesa):
+    """The bucket path from a key array (no fused first pass): multi-granule records (8-byte accesses at G = 4)
+    over an evenly spread region, 17 M records; equal to the oracle."""
+    from sesagen import configs as C
+    n = (1 << 24) + 4321
+    r = C.rnd_host(n, 777, blocks=4096, threads=512, intervals=2, words=1 << 26, shared_frac=0.0, sizes=(4, 8),
+                   unaligned=False, values=3)
+    t = sesa.Trace(32, 0, 4)
+    t.check(sesa.to_device(r), n)
+    info = t.info()
+    got = t.races()
+    t.close()
+    assert info["bucket_path"] == 1 and info["fused_first_pass"] == 0
+    assert got.tobytes() == O.check(r, method="partitioned").tobytes()
