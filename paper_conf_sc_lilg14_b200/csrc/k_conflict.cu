@@ -648,6 +648,274 @@ __device__ __forceinline__ void cannot_race(const Agg& g, bool* no_rw, bool* no_
 }
 __device__ __forceinline__ u64 ld_volatile(const u64* p) { return *reinterpret_cast<const volatile u64*>(p); }
 
+// ------------------------------------------------------------------------------------------------ internal groups
+// Mode 1 fast path for the groups that lie wholly inside the window.  The witness of (λ, K) needs only x_K (the
+// lowest flagged position) and y_K (the lowest partner of x_K), not every entry's flag: per group, one exact
+// summary G with identity = block decides "a partner in another block" for any entry in O(1); a partner in the
+// entry's own (block, interval) sub-run is found pair by pair (sub-runs are short: the tile takes the scan path
+// if an internal sub-run exceeds SR_MAX entries).  With position-ordered runs (lowG == 0) the x and y searches
+// stop at the first hit — usually within the first few entries.  Groups of up to GR_SEQ entries: one thread each;
+// longer groups: one warp each (lane-strided summary + butterfly merge, 32 candidates per step, ballots).
+constexpr int GR_SEQ = 16;
+constexpr int SR_MAX = 64;
+
+__device__ __forceinline__ Agg shfl_x(const Agg& a, int o) {
+  Agg r;
+#pragma unroll
+  for (int x = 0; x < 3; x++) r.mn[x] = __shfl_xor_sync(~0u, a.mn[x], o), r.mx[x] = __shfl_xor_sync(~0u, a.mx[x], o);
+  r.i1 = __shfl_xor_sync(~0u, a.i1, o), r.i2 = __shfl_xor_sync(~0u, a.i2, o);
+  r.v1 = __shfl_xor_sync(~0u, a.v1, o), r.v1b = __shfl_xor_sync(~0u, a.v1b, o);
+  r.v2 = __shfl_xor_sync(~0u, a.v2, o), r.v2b = __shfl_xor_sync(~0u, a.v2b, o);
+  return r;
+}
+
+// a partner of e in another block (G: the group's exact summary, identity = block): RW / WW
+__device__ __forceinline__ void flags_other_block(const Agg& G, const F5& e, bool* rwf, bool* wwf) {
+  const u32 b = e.block;
+  if (e.rw == RW_READ) {
+    *rwf = ex_id(G, RW_WRITE, b) || ex_id(G, RW_ATOMIC, b);
+    *wwf = false;
+  } else {
+    *rwf = ex_id(G, RW_READ, b);
+    *wwf = e.rw == RW_WRITE ? (ex_id(G, RW_ATOMIC, b) || ex_wval(G, b, e.vh)) : ex_id(G, RW_WRITE, b);
+  }
+}
+
+// a partner of item j in its sub-run [sh, st] (same block and interval): rules 1-6 pair by pair
+__device__ __forceinline__ void flags_subrun(const TileSmem& s, int j, int sh, int st, const F5& me, u32 ws, u32 ls,
+                                             bool* f0, bool* f1) {
+  for (int q = sh; q <= st && !(*f0 && *f1); q++) {
+    if (q == j) continue;
+    const u32 k = pair_kind(me, fields(s, q), ws, ls);
+    *f0 = *f0 || k == KIND_RW;
+    *f1 = *f1 || k == KIND_WW;
+  }
+}
+
+__device__ __forceinline__ void emit_group(const ConflictArgs& a, const TileSmem& s, int t, u32 kind, u32 x, u32 y) {
+  emit_race(a, s.key[t + 1] >> a.L.pos_bits, kind, x, y, s.blk[t + 1], s.ivl[t + 1]);
+}
+
+// one thread: group [h, t] (>= 2 entries, all gathered)
+__device__ void group_thread(const ConflictArgs& a, const TileSmem& s, int h, int t) {
+  const KeyLayout& L = a.L;
+  Agg G = agg_empty();
+  for (int j = h; j <= t; j++) G = agg_merge(G, agg_item(s.rw[j], s.blk[j + 1], s.vh[j]));
+  bool no0, no1;
+  cannot_race(G, &no0, &no1);
+  if (no0 && no1) return;
+  const bool ordered = L.lowG == 0;
+  bool need0 = !no0, need1 = !no1;
+  u32 xp0 = ~0u, xp1 = ~0u;
+  int xj0 = -1, xj1 = -1, sh = h, st = h;
+  for (int j = h; j <= t && (need0 || need1); j++) {
+    if (s.fl[j] & FL_SH) {
+      sh = st = j;
+      while (!(s.fl[st] & FL_ST)) st++;
+    }
+    const F5 me = fields(s, j);
+    bool f0, f1;
+    flags_other_block(G, me, &f0, &f1);
+    f0 = f0 && need0, f1 = f1 && need1;
+    if (st > sh && (need0 != f0 || need1 != f1)) {
+      flags_subrun(s, j, sh, st, me, a.ws, a.ls, &f0, &f1);
+      f0 = f0 && need0, f1 = f1 && need1;
+    }
+    const u32 p = pos_of(L, s.key[j + 1]);
+    if (f0 && p < xp0) xp0 = p, xj0 = j, need0 = !ordered;
+    if (f1 && p < xp1) xp1 = p, xj1 = j, need1 = !ordered;
+  }
+#pragma unroll 1
+  for (int k = 0; k < 2; k++) {
+    const int xj = k ? xj1 : xj0;
+    if (xj < 0) continue;
+    const F5 X = fields(s, xj);
+    u32 y = ~0u;
+    for (int q = h; q <= t; q++) {
+      if (pair_kind(X, fields(s, q), a.ws, a.ls) != (u32)(k + 1)) continue;
+      y = min(y, pos_of(L, s.key[q + 1]));
+      if (ordered) break;
+    }
+    emit_group(a, s, t, (u32)(k + 1), k ? xp1 : xp0, y);
+  }
+}
+
+// one warp: group [h, t]
+__device__ void group_warp(const ConflictArgs& a, const TileSmem& s, int h, int t) {
+  const KeyLayout& L = a.L;
+  const int lane = threadIdx.x & 31;
+  Agg G = agg_empty();
+  for (int j = h + lane; j <= t; j += 32) G = agg_merge(G, agg_item(s.rw[j], s.blk[j + 1], s.vh[j]));
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) G = agg_merge(G, shfl_x(G, o));
+  bool no0, no1;
+  cannot_race(G, &no0, &no1);
+  if (no0 && no1) return;
+  const bool ordered = L.lowG == 0;
+  bool need0 = !no0, need1 = !no1;
+  u32 xp[2] = {~0u, ~0u};
+  int xj[2] = {-1, -1};
+  for (int c = h; c <= t && (need0 || need1); c += 32) {
+    const int j = c + lane;
+    bool f0 = false, f1 = false;
+    u32 p = ~0u;
+    if (j <= t) {
+      const F5 me = fields(s, j);
+      flags_other_block(G, me, &f0, &f1);
+      f0 = f0 && need0, f1 = f1 && need1;
+      if (need0 != f0 || need1 != f1) {
+        const u8 fj = s.fl[j];
+        if (!((fj & FL_SH) && (fj & FL_ST))) {
+          int sh = j, st = j;
+          while (!(s.fl[sh] & FL_SH)) sh--;
+          while (!(s.fl[st] & FL_ST)) st++;
+          flags_subrun(s, j, sh, st, me, a.ws, a.ls, &f0, &f1);
+          f0 = f0 && need0, f1 = f1 && need1;
+        }
+      }
+      p = pos_of(L, s.key[j + 1]);
+    }
+#pragma unroll
+    for (int k = 0; k < 2; k++) {
+      const bool f = k ? f1 : f0;
+      const u32 m = __reduce_min_sync(~0u, f ? p : ~0u);
+      if (m < xp[k]) {
+        xp[k] = m;
+        xj[k] = c + __ffs(__ballot_sync(~0u, f && p == m)) - 1;
+        if (ordered) (k ? need1 : need0) = false;
+      }
+    }
+  }
+#pragma unroll
+  for (int k = 0; k < 2; k++) {
+    if (xj[k] < 0) continue;
+    const F5 X = fields(s, xj[k]);
+    u32 y = ~0u;
+    for (int c = h; c <= t; c += 32) {
+      const int j = c + lane;
+      const bool hit = j <= t && pair_kind(X, fields(s, j), a.ws, a.ls) == (u32)(k + 1);
+      y = min(y, __reduce_min_sync(~0u, hit ? pos_of(L, s.key[j + 1]) : ~0u));
+      if (ordered && y != ~0u) break;
+    }
+    if (lane == 0) emit_group(a, s, t, (u32)(k + 1), xp[k], y);
+  }
+}
+
+// exclusive block-wide sum of v (CT_THREADS threads); *total = the sum over the block
+__device__ __forceinline__ u32 block_excl_sum(u32 v, u32* s_w, u32* total) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  u32 x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const u32 y = __shfl_up_sync(~0u, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) s_w[warp] = x;
+  __syncthreads();
+  u32 off = 0, tot = 0;
+#pragma unroll
+  for (int w = 0; w < CT_THREADS / 32; w++) {
+    const u32 sw = s_w[w];
+    off += w < warp ? sw : 0u;
+    tot += sw;
+  }
+  __syncthreads();
+  *total = tot;
+  return off + x - v;
+}
+
+// Does an internal group of the tile (entries [lo, hi)) hold a sub-run longer than SR_MAX?  (all threads call)
+__device__ __forceinline__ bool long_subrun(const TileSmem& s, int lo, int hi) {
+  bool lsr = false;
+#pragma unroll kCtUnroll
+  for (int q = 0; q < CT_ITEMS; q++) {
+    const int j = threadIdx.x * CT_ITEMS + q;
+    const u8 f = s.fl[j];
+    if (j < lo || j >= hi || !(f & FL_INT) || !(f & FL_SH) || (f & FL_ST)) continue;
+    int e = j + 1;
+    while (!(s.fl[e] & FL_ST) && e - j < SR_MAX) e++;
+    lsr = lsr || !(s.fl[e] & FL_ST);
+  }
+  return __syncthreads_or(lsr) != 0;
+}
+
+// races of the internal groups (entries [lo, hi)): group list by a block scan, then threads / warps
+__device__ void internal_groups(const ConflictArgs& a, TileSmem& s, int lo, int hi) {
+  __shared__ u32 s_w[CT_THREADS / 32];
+  unsigned short* gh = reinterpret_cast<unsigned short*>(&s.xy[0][0]);
+  unsigned short* gt = gh + CT_TILE / 2 + 8;
+  u32 nh = 0, nt = 0;
+#pragma unroll kCtUnroll
+  for (int q = 0; q < CT_ITEMS; q++) {
+    const int j = threadIdx.x * CT_ITEMS + q;
+    const u8 f = s.fl[j];
+    if (j < lo || j >= hi || !(f & FL_INT)) continue;
+    nh += (f & FL_GH) ? 1u : 0u;
+    nt += (f & FL_GT) ? 1u : 0u;
+  }
+  u32 tot;
+  const u32 ex = block_excl_sum(nh | (nt << 16), s_w, &tot);
+  u32 oh = ex & 0xFFFFu, ot = ex >> 16;
+#pragma unroll kCtUnroll
+  for (int q = 0; q < CT_ITEMS; q++) {
+    const int j = threadIdx.x * CT_ITEMS + q;
+    const u8 f = s.fl[j];
+    if (j < lo || j >= hi || !(f & FL_INT)) continue;
+    if (f & FL_GH) gh[oh++] = (unsigned short)j;
+    if (f & FL_GT) gt[ot++] = (unsigned short)j;
+  }
+  __syncthreads();
+  const int ng = (int)(tot & 0xFFFFu);
+  for (int g = threadIdx.x; g < ng; g += CT_THREADS)
+    if (gt[g] - gh[g] < GR_SEQ) group_thread(a, s, gh[g], gt[g]);
+  for (int g = threadIdx.x >> 5; g < ng; g += CT_THREADS / 32)
+    if (gt[g] - gh[g] >= GR_SEQ) group_warp(a, s, gh[g], gt[g]);
+}
+
+// the tile-edge pieces for the carries without the segmented scans: part[0] / part[1] = run-level summaries of
+// [0, first run tail] / [last run head, cnt), part[2] / part[3] = sub-run-level ones of [0, first sub-run tail] /
+// [last sub-run head, cnt) — what tile_flags hands the carries
+template <class A>
+__device__ void tile_parts(const TileSmem& s, u32 cnt, A* part) {
+  typedef typename OpOf<A>::type Op;
+  __shared__ int s_fst, s_lsh;
+  __shared__ A s_red[2][CT_THREADS / 32];
+  if (threadIdx.x == 0) s_fst = (int)cnt - 1, s_lsh = 0;
+  __syncthreads();
+#pragma unroll kCtUnroll
+  for (int q = 0; q < CT_ITEMS; q++) {
+    const int j = threadIdx.x * CT_ITEMS + q;
+    if (j >= (int)cnt) continue;
+    if (s.fl[j] & FL_ST) atomicMin(&s_fst, j);
+    if (s.fl[j] & FL_SH) atomicMax(&s_lsh, j);
+  }
+  __syncthreads();
+  const int ft = s.first_gtail, lh = s.last_ghead, fst = s_fst, lsh = s_lsh;
+  const A E = agg_empty_t<A>();
+#pragma unroll 1
+  for (int r = 0; r < 2; r++) {
+    A p0 = E, p1 = E;
+#pragma unroll kCtUnroll
+    for (int q = 0; q < CT_ITEMS; q++) {
+      const int j = threadIdx.x * CT_ITEMS + q;
+      if (j >= (int)cnt || !(s.fl[j] & FL_INT)) continue;
+      const A it = agg_item_t<A>(s.rw[j], r ? s.thr[j] : s.blk[j + 1], s.vh[j]);
+      if (j <= (r ? fst : ft)) p0 = Op()(p0, it);
+      if (j >= (r ? lsh : lh)) p1 = Op()(p1, it);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) p0 = Op()(p0, shfl(p0, o, true)), p1 = Op()(p1, shfl(p1, o, true));
+    if ((threadIdx.x & 31) == 0) s_red[0][threadIdx.x >> 5] = p0, s_red[1][threadIdx.x >> 5] = p1;
+    __syncthreads();
+    if (threadIdx.x < 2) {
+      A t = s_red[threadIdx.x][0];
+      for (int w = 1; w < CT_THREADS / 32; w++) t = Op()(t, s_red[threadIdx.x][w]);
+      part[2 * r + threadIdx.x] = t;
+    }
+    __syncthreads();
+  }
+}
+
 // ------------------------------------------------------------------------------------------------ mode 1 / 2
 template <int MODE, class A>
 // mode 1 at 3 CTAs/SM (the shared-memory limit): up to 80 registers, no spills; mode 2 at 2 (128 registers)
@@ -766,7 +1034,15 @@ __global__ void __launch_bounds__(CT_THREADS, MODE == 1 ? 3 : 2) conflict_kernel
     }
     return;
   }
-  tile_flags<A>(a, s, cnt, ci, co, MODE == 1 ? s_part : nullptr, MODE == 2 && cin && cout && s.last_ghead < 0);
+  // mode 1: the groups wholly inside the window [ilo, ihi) take the fast path (internal_groups) unless one of
+  // their sub-runs is long; the crossing pieces only owe the carries their edge summaries (tile_parts)
+  const int ilo = cin ? s.first_gtail + 1 : 0, ihi = cout ? s.last_ghead : (int)cnt;
+  const bool fast = MODE == 1 && !long_subrun(s, ilo, ihi);
+  if (fast) {
+    if (cin || cout) tile_parts<A>(s, cnt, s_part);
+  } else {
+    tile_flags<A>(a, s, cnt, ci, co, MODE == 1 ? s_part : nullptr, MODE == 2 && cin && cout && s.last_ghead < 0);
+  }
   const int ftail = s.first_gtail, lhead = s.last_ghead;
   if (s.unknown) {  // a benign query the cheap summary cannot decide: the host reruns with exact summaries
     if (tid == 0) atomicOr(a.need_exact, 1u);
@@ -804,6 +1080,10 @@ __global__ void __launch_bounds__(CT_THREADS, MODE == 1 ? 3 : 2) conflict_kernel
         sl.hinterval = s.ivl[lhead + 1];
         a.slots[tile] = sl;
       }
+    }
+    if (fast) {
+      internal_groups(a, s, ilo, ihi);
+      return;
     }
     // no flagged entry in a group internal to the tile (every internal group race-free, e.g. all of C2; or only
     // crossing pieces, e.g. the middle tiles of C3's hot bins — modes 2/3 own those): nothing to emit here
