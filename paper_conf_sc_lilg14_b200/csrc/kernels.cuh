@@ -136,6 +136,7 @@ struct ConflictArgs {
   u64 index_base;
   u32 phase;  // modes 2/3: 0 = every crossing piece, 1 = pieces starting a run (crossing out), 2 = the rest
   u32 tdiv;   // > 1: a record's identity is thread / tdiv (precise warp model, inter-warp half)
+  const u32* tstart;  // [tiles + 1]: first entry of every tile window (launch_tile_starts)
 };
 
 struct RaceOut {  // == sesa_race (40 bytes)
@@ -163,6 +164,7 @@ void launch_permute_races(const RaceOut* in, const u32* order, RaceOut* out, u32
 void launch_races_set_epoch(const RaceOut* in, u32 nr, u32 e, RaceOut* out, cudaStream_t st);
 void race_rekey_launch(const RaceOut* r, u64 n, const KeyLayout& L, u64* keys, u32* vals, cudaStream_t st);
 u32 conflict_tiles(u64 m);
+void launch_tile_starts(const ConflictArgs& a, u32 ntiles, u32* tstart, cudaStream_t st);
 // benign W/W reporting (k_conflict.cu)
 void launch_benign_mark(const u64* comp, u32 m2, const KeyLayout& L, const Rec* rec, const Rec* rec_entry, u32* head, u32* wflag,
                         cudaStream_t st);

@@ -575,7 +575,8 @@ bool sesa_trace::step_conflict(const u64* comp, u32 m2, const Rec* rec, u32 rec_
         !grow(b_ccount, 16, "ccount") || !grow(b_races, (size_t)race_cap * sizeof(RaceOut), "races") ||
         !grow(b_rkeys[0], (size_t)race_cap * 8, "race keys") || !grow(b_rkeys[1], (size_t)race_cap * 8, "race keys") ||
         !grow(b_rvals[0], (size_t)race_cap * 4, "race vals") || !grow(b_rvals[1], (size_t)race_cap * 4, "race vals") ||
-        !grow(b_carrytmp, carry_temp_bytes(ctiles), "carry temp"))
+        !grow(b_carrytmp, carry_temp_bytes(ctiles), "carry temp") ||
+        !grow(b_tstart, ((size_t)ctiles + 1) * 4, "tile starts"))
       return false;
     ConflictArgs A;
     memset(&A, 0, sizeof A);
@@ -602,6 +603,8 @@ bool sesa_trace::step_conflict(const u64* comp, u32 m2, const Rec* rec, u32 rec_
     A.owner = (u32*)b_owner.p;
     A.slots = (Slot*)b_slots.p;
     A.index_base = index_base;
+    A.tstart = (const u32*)b_tstart.p;
+    LAUNCH("tile_starts", 8.0 * m2, launch_tile_starts(A, ctiles, (u32*)b_tstart.p, stream));
     // cheap summaries first; a benign query they cannot decide (>= 2 writers with >= 2 values at one location)
     // makes the whole check rerun with the exact summaries (mode 1 and, for crossing runs, mode 2 can detect it)
     u32 cc[3] = {0, 0, 0};
