@@ -416,9 +416,11 @@ __device__ __forceinline__ Rec rec_at(const ConflictArgs& a, u64 e, u64 key) {
   return r;
 }
 
-// Loads keys and gathers records (every entry of a compacted array has a partner candidate somewhere, so the
-// record loads go out with the key loads instead of after the membership flags), computes group membership.
-// Returns false if no entry of the tile has a partner candidate (all singletons).
+// Loads keys and group flags; with GATHER (mode 1) also every record — every entry of a compacted array has a
+// partner candidate somewhere, so the record loads go out with the key loads — and the sub-run flags.  Modes 2/3
+// gather only their crossing pieces afterwards (tile_gather).  Returns false if no entry of the tile has a
+// partner candidate (all singletons).
+template <bool GATHER>
 __device__ bool tile_load(const ConflictArgs& a, TileSmem& s, u64 tb, u32 cnt) {
   const KeyLayout& L = a.L;
   const int tid = threadIdx.x;
@@ -432,27 +434,33 @@ __device__ bool tile_load(const ConflictArgs& a, TileSmem& s, u64 tb, u32 cnt) {
 #pragma unroll
   for (int h = 0; h < CT_ITEMS; h += HALF) {
     Rec r[HALF];
+    if (GATHER) {
 #pragma unroll
-    for (int q = 0; q < HALF; q++)
-      if ((h + q) * CT_THREADS + tid < (int)cnt) r[q] = rec_at(a, tb + (h + q) * CT_THREADS + tid, k[h + q]);
+      for (int q = 0; q < HALF; q++)
+        if ((h + q) * CT_THREADS + tid < (int)cnt) r[q] = rec_at(a, tb + (h + q) * CT_THREADS + tid, k[h + q]);
+    }
 #pragma unroll
     for (int q = 0; q < HALF; q++) {
       const u32 j = (h + q) * CT_THREADS + tid;
       if (j >= cnt) continue;
       s.key[j + 1] = k[h + q];
-      s.blk[j + 1] = r[q].block;
-      s.ivl[j + 1] = r[q].interval;
-      s.thr[j] = r[q].thread;
-      s.rw[j] = r[q].rw;
-      s.vh[j] = r[q].vh;
+      if (GATHER) {
+        s.blk[j + 1] = r[q].block;
+        s.ivl[j + 1] = r[q].interval;
+        s.thr[j] = r[q].thread;
+        s.rw[j] = r[q].rw;
+        s.vh[j] = r[q].vh;
+      }
     }
   }
-  if (tid == 0) {  // the entries just outside the window: key and (block, interval)
+  if (tid == 0) {  // the entries just outside the window: key (and (block, interval))
     s.key[0] = 0ull;
     if (tb > 0) {
-      const u64 k = a.keys[tb - 1];
-      const Rec r = rec_at(a, tb - 1, k);
-      s.key[0] = k, s.blk[0] = r.block, s.ivl[0] = r.interval;
+      s.key[0] = a.keys[tb - 1];
+      if (GATHER) {
+        const Rec r = rec_at(a, tb - 1, s.key[0]);
+        s.blk[0] = r.block, s.ivl[0] = r.interval;
+      }
     }
     s.any = 0;
     s.first_gtail = CT_TILE;
@@ -461,9 +469,11 @@ __device__ bool tile_load(const ConflictArgs& a, TileSmem& s, u64 tb, u32 cnt) {
   if (tid == CT_THREADS - 1) {
     s.key[cnt + 1] = 0ull;
     if (tb + cnt < a.m) {
-      const u64 k = a.keys[tb + cnt];
-      const Rec r = rec_at(a, tb + cnt, k);
-      s.key[cnt + 1] = k, s.blk[cnt + 1] = r.block, s.ivl[cnt + 1] = r.interval;
+      s.key[cnt + 1] = a.keys[tb + cnt];
+      if (GATHER) {
+        const Rec r = rec_at(a, tb + cnt, s.key[cnt + 1]);
+        s.blk[cnt + 1] = r.block, s.ivl[cnt + 1] = r.interval;
+      }
     }
   }
   __syncthreads();
@@ -481,30 +491,77 @@ __device__ bool tile_load(const ConflictArgs& a, TileSmem& s, u64 tb, u32 cnt) {
       const bool sn = (j + 1 < (int)cnt || tb + cnt < a.m) && group_of_hi(L, s.key[j + 2] >> L.pos_bits) == g;
       f = (sp ? 0 : FL_GH) | (sn ? 0 : FL_GT) | ((sp || sn) ? FL_INT : 0);
       any |= sp || sn;
+      if (f & FL_GT) atomicMin(&s.first_gtail, j);
+      if (f & FL_GH) atomicMax(&s.last_ghead, j);
     }
     s.fl[j] = f;
   }
   if (!__syncthreads_or(any)) return false;
-  // sub-runs: a new (block, interval) inside a group (contiguous: input order is (block, interval) order)
+  if (GATHER) {
+    // sub-runs: a new (block, interval) inside a group (contiguous: input order is (block, interval) order)
 #pragma unroll kCtUnroll
-  for (int q = 0; q < CT_ITEMS; q++) {
-    const int j = j0 + q;
+    for (int q = 0; q < CT_ITEMS; q++) {
+      const int j = j0 + q;
+      u8 f = s.fl[j];
+      if (f & FL_INT) {
+        const bool sh = (f & FL_GH) || s.blk[j] != s.blk[j + 1] || s.ivl[j] != s.ivl[j + 1];
+        const bool st = (f & FL_GT) || s.blk[j + 2] != s.blk[j + 1] || s.ivl[j + 2] != s.ivl[j + 1];
+        f |= (sh ? FL_SH : 0) | (st ? FL_ST : 0);
+      } else if (j < (int)cnt) {
+        f |= FL_SH | FL_ST;
+      }
+      s.fl[j] = f;
+    }
+    __syncthreads();
+  }
+  return true;
+}
+
+// Modes 2/3: records and sub-run flags of the entries [lo, hi) (whole crossing pieces: a piece starting at 0
+// needs the (block, interval) of the entry before the window, one ending at cnt that of the entry after it).
+// All threads call.
+__device__ void tile_gather(const ConflictArgs& a, TileSmem& s, u64 tb, u32 cnt, int lo, int hi) {
+  const int tid = threadIdx.x;
+  constexpr int B = 3;
+  for (int j0 = lo; j0 < hi; j0 += B * CT_THREADS) {
+    Rec r[B];
+#pragma unroll
+    for (int q = 0; q < B; q++) {
+      const int j = j0 + q * CT_THREADS + tid;
+      if (j < hi) r[q] = rec_at(a, tb + j, s.key[j + 1]);
+    }
+#pragma unroll
+    for (int q = 0; q < B; q++) {
+      const int j = j0 + q * CT_THREADS + tid;
+      if (j >= hi) continue;
+      s.blk[j + 1] = r[q].block;
+      s.ivl[j + 1] = r[q].interval;
+      s.thr[j] = r[q].thread;
+      s.rw[j] = r[q].rw;
+      s.vh[j] = r[q].vh;
+    }
+  }
+  if (lo == 0 && tid == 0 && tb > 0) {
+    const Rec r = rec_at(a, tb - 1, s.key[0]);
+    s.blk[0] = r.block, s.ivl[0] = r.interval;
+  }
+  if (hi == (int)cnt && tid == CT_THREADS - 1 && tb + cnt < a.m) {
+    const Rec r = rec_at(a, tb + cnt, s.key[cnt + 1]);
+    s.blk[cnt + 1] = r.block, s.ivl[cnt + 1] = r.interval;
+  }
+  __syncthreads();
+  for (int j = lo + tid; j < hi; j += CT_THREADS) {
     u8 f = s.fl[j];
     if (f & FL_INT) {
       const bool sh = (f & FL_GH) || s.blk[j] != s.blk[j + 1] || s.ivl[j] != s.ivl[j + 1];
       const bool st = (f & FL_GT) || s.blk[j + 2] != s.blk[j + 1] || s.ivl[j + 2] != s.ivl[j + 1];
       f |= (sh ? FL_SH : 0) | (st ? FL_ST : 0);
-    } else if (j < (int)cnt) {
+    } else {
       f |= FL_SH | FL_ST;
     }
     s.fl[j] = f;
-    if (j < (int)cnt) {
-      if (f & FL_GT) atomicMin(&s.first_gtail, j);
-      if (f & FL_GH) atomicMax(&s.last_ghead, j);
-    }
   }
   __syncthreads();
-  return true;
 }
 
 // group- and sub-run-level summaries -> s.res[j] = bit0 RW partner, bit1 WW partner.  In mode 1 also returns
@@ -952,6 +1009,134 @@ __device__ void tile_parts(const TileSmem& s, u32 cnt, A* part) {
   }
 }
 
+// ------------------------------------------------------------------------------------------------ mode 2 fast
+// Mode 2 without the segmented scans: a crossing piece only needs its lowest flagged position per kind (x into
+// the owner's slot), and an entry's flag follows from the run summary R (carries + the piece's part, identity =
+// block: "a partner in another block"), the summary S of its sub-run if that sub-run continues across the
+// window's edge (carries + part, identity = thread), or pair by pair inside a sub-run within the window.  Only
+// the pieces' records are gathered; with position-ordered runs the search stops at the first chunk that flags.
+// Returns false (nothing done) when an inner sub-run is longer than SR_MAX: the caller takes the scan path.
+template <class A>
+__device__ bool cross_pieces_fast(const ConflictArgs& a, TileSmem& s, u32 tile, u64 tb, u32 cnt, bool cin,
+                                  bool cout, const u8 (*need)[2]) {
+  typedef typename OpOf<A>::type Op;
+  typedef typename QuadOf<A>::type Q;
+  const int tid = threadIdx.x;
+  const int ftail = s.first_gtail, lhead = s.last_ghead;
+  const bool pa = cin && a.phase != 1 && (need[0][0] || need[0][1]);
+  const bool pb = cout && lhead >= 0 && a.phase != 2 && (need[1][0] || need[1][1]);
+  const int aend = min(ftail, (int)cnt - 1);
+  if (pa) tile_gather(a, s, tb, cnt, 0, aend + 1);
+  if (pb) tile_gather(a, s, tb, cnt, lhead, (int)cnt);
+  __shared__ int s_fst, s_lsh, s_long;
+  __shared__ A s_R[2], s_S[2];
+  __shared__ unsigned long long s_min[4];
+  if (tid == 0) s_fst = (int)cnt - 1, s_lsh = 0, s_long = 0;
+  if (tid < 4) s_min[tid] = ~0ull;
+  __syncthreads();
+  auto in_piece = [&](int j) { return (pa && j <= aend) || (pb && j >= lhead && j < (int)cnt); };
+  // the edge sub-runs: the first one of piece A (if it continues in from the previous window) and the last one
+  // of the piece that ends the window (B, or A when the window lies inside one run) if it continues out
+  const bool middle = cin && cout && lhead < 0;
+  const bool lastp = pb || (pa && middle);  // the window's last entry belongs to a processed piece
+  const int llo = pb ? lhead : 0;
+  for (int j = tid; j < (int)cnt; j += CT_THREADS) {
+    if (pa && j <= aend && (s.fl[j] & FL_ST)) atomicMin(&s_fst, j);
+    if (lastp && j >= llo && (s.fl[j] & FL_SH)) atomicMax(&s_lsh, j);
+  }
+  __syncthreads();
+  const int fst = s_fst, lsh = s_lsh;
+  const bool cinS = pa && !(s.fl[0] & FL_SH), coutS = lastp && !(s.fl[cnt - 1] & FL_ST);
+  // inner sub-runs (not continuing across an edge) longer than SR_MAX: the scan path
+  for (int j = tid; j < (int)cnt; j += CT_THREADS) {
+    if (!in_piece(j) || !(s.fl[j] & FL_SH) || (s.fl[j] & FL_ST) || (coutS && j == lsh)) continue;
+    int e = j + 1;
+    while (e < (int)cnt - 1 && !(s.fl[e] & FL_ST) && e - j < SR_MAX) e++;
+    if (!(s.fl[e] & FL_ST)) s_long = 1;
+  }
+  if (tid == 0) {
+    const A* c = reinterpret_cast<const Q*>(a.carry)[tile].a;  // [grp In, grp Out, sub In, sub Out]
+    const A* pp = reinterpret_cast<const Q*>(a.part)[tile].a;  // [grp P, grp S, sub P, sub S]
+    const A E = agg_empty_t<A>();
+    s_R[0] = middle ? Op()(Op()(c[0], pp[0]), c[1]) : Op()(c[0], pp[0]);
+    s_R[1] = Op()(pp[1], c[1]);
+    s_S[0] = Op()(Op()(c[2], pp[2]), (fst == (int)cnt - 1 && coutS) ? c[3] : E);
+    s_S[1] = Op()(Op()((lsh == 0 && cinS) ? c[2] : E, pp[3]), c[3]);
+  }
+  if (__syncthreads_or(s_long)) return false;
+  const bool ordered = a.L.lowG == 0;
+  const u32 ws = a.ws, ls = a.ls;
+#pragma unroll 1
+  for (int P = 0; P < 2; P++) {
+    if (!(P ? pb : pa)) continue;
+    const int lo = P ? lhead : 0, hi = P ? (int)cnt - 1 : aend;
+    bool n0 = need[P][0], n1 = need[P][1];
+    for (int c0 = lo; c0 <= hi && (n0 || n1); c0 += CT_THREADS) {
+      const int j = c0 + tid;
+      bool f0 = false, f1 = false, unk = false;
+      if (j <= hi && (s.fl[j] & FL_INT)) {
+        const F5 me = fields(s, j);
+        const A& R = s_R[P];
+        const u32 b = me.block, t = me.thread;
+        int qg = 0, qs = 0;
+        if (me.rw == RW_READ) {
+          f0 = ex_id(R, RW_WRITE, b) || ex_id(R, RW_ATOMIC, b);
+        } else {
+          f0 = ex_id(R, RW_READ, b);
+          if (me.rw == RW_WRITE) qg = wval3(R, b, me.vh), f1 = ex_id(R, RW_ATOMIC, b) || qg == 1;
+          else f1 = ex_id(R, RW_WRITE, b);
+        }
+        const bool inF = cinS && j <= fst, inL = coutS && j >= lsh;
+        if (inF || inL) {
+          const A& S = s_S[inF ? 0 : 1];
+          const u32 w = t / ws;
+          if (me.rw == RW_READ) {
+            f0 = f0 || (ls ? (ex_warp(S, RW_WRITE, w, ws) || ex_warp(S, RW_ATOMIC, w, ws))
+                           : (ex_id(S, RW_WRITE, t) || ex_id(S, RW_ATOMIC, t)));
+          } else {
+            f0 = f0 || (ls ? ex_warp(S, RW_READ, w, ws) : ex_id(S, RW_READ, t));
+            if (me.rw == RW_WRITE) qs = wval3(S, t, me.vh), f1 = f1 || ex_id(S, RW_ATOMIC, t) || qs == 1;
+            else f1 = f1 || ex_id(S, RW_WRITE, t);
+          }
+        } else if ((n0 && !f0) || (n1 && !f1)) {
+          const u8 fj = s.fl[j];
+          if (!((fj & FL_SH) && (fj & FL_ST))) {
+            int sh = j, st = j;
+            while (!(s.fl[sh] & FL_SH)) sh--;
+            while (!(s.fl[st] & FL_ST)) st++;
+            flags_subrun(s, j, sh, st, me, ws, ls, &f0, &f1);
+          }
+        }
+        f0 = f0 && n0, f1 = f1 && n1;
+        unk = n1 && !f1 && (qg == 2 || qs == 2);
+      }
+      if (__syncthreads_or(unk)) {  // a benign query the cheap summary cannot decide: the host reruns exactly
+        if (tid == 0) atomicOr(a.need_exact, 1u);
+        return true;
+      }
+      const unsigned long long p = ((unsigned long long)pos_of(a.L, s.key[j + 1]) << 32) | (u32)(tb + j);
+      if (f0) atomicMin(&s_min[2 * P], p);
+      if (f1) atomicMin(&s_min[2 * P + 1], p);
+      __syncthreads();
+      if (ordered) n0 = n0 && s_min[2 * P] == ~0ull, n1 = n1 && s_min[2 * P + 1] == ~0ull;
+      __syncthreads();
+    }
+  }
+  if (tid == 0) {
+    if (pa) {
+      Slot* sl = &a.slots[a.owner[tile]];
+      if (s_min[0] != ~0ull) atomicMin((unsigned long long*)&sl->x[0], s_min[0]);
+      if (s_min[1] != ~0ull) atomicMin((unsigned long long*)&sl->x[1], s_min[1]);
+    }
+    if (pb) {
+      Slot* sl = &a.slots[tile];
+      if (s_min[2] != ~0ull) atomicMin((unsigned long long*)&sl->x[0], s_min[2]);
+      if (s_min[3] != ~0ull) atomicMin((unsigned long long*)&sl->x[1], s_min[3]);
+    }
+  }
+  return true;
+}
+
 // ------------------------------------------------------------------------------------------------ mode 1 / 2
 template <int MODE, class A>
 // mode 1 at 3 CTAs/SM (the shared-memory limit): up to 80 registers, no spills; mode 2 at 2 (128 registers)
@@ -960,6 +1145,7 @@ __global__ void __launch_bounds__(CT_THREADS, MODE == 1 ? 3 : 2) conflict_kernel
   extern __shared__ __align__(16) unsigned char smem_raw[];
   TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
   const u32 tile = MODE == 1 ? blockIdx.x : a.cross_list[blockIdx.x];
+  __shared__ u8 s_need[2][2];  // mode 2: piece (A = crossing in, B = crossing out) x kind (RW, WW) can lower x
   if (MODE == 2) {
     // A crossing piece matters for a kind K only if its run's whole summary allows a K pair and — for the
     // piece a run crosses IN with (its head lies in an earlier tile), in position-ordered runs (lowG == 0) — no
@@ -968,6 +1154,7 @@ __global__ void __launch_bounds__(CT_THREADS, MODE == 1 ? 3 : 2) conflict_kernel
     __shared__ int s_skip;
     if (threadIdx.x == 0) {
       typedef typename OpOf<A>::type Op;
+      s_need[0][0] = s_need[0][1] = s_need[1][0] = s_need[1][1] = 0;
       const u8 tf = a.tile_flags[tile];
       const A* c = reinterpret_cast<const Q*>(a.carry)[tile].a;    // [grp In, grp Out, ...]
       const A* pp = reinterpret_cast<const Q*>(a.part)[tile].a;    // [grp P, grp S, ...]
@@ -986,11 +1173,13 @@ __global__ void __launch_bounds__(CT_THREADS, MODE == 1 ? 3 : 2) conflict_kernel
           }
         }
         skip = skip && done[0] && done[1];
+        s_need[0][0] = !done[0], s_need[0][1] = !done[1];
       }
       if ((tf & TF_COUT) && (tf & TF_GH) && a.phase != 2) {  // piece B: a run starting here and crossing out
         bool done[2];
         cannot_race(Op()(pp[1], c[1]), &done[0], &done[1]);
         skip = skip && done[0] && done[1];
+        s_need[1][0] = !done[0], s_need[1][1] = !done[1];
       }
       s_skip = skip;
     }
@@ -1003,7 +1192,7 @@ __global__ void __launch_bounds__(CT_THREADS, MODE == 1 ? 3 : 2) conflict_kernel
   const KeyLayout& L = a.L;
   const int tid = threadIdx.x;
 
-  if (cnt == 0 || !tile_load(a, s, tb, cnt)) {
+  if (cnt == 0 || !tile_load<MODE == 1>(a, s, tb, cnt)) {
     if (MODE == 1 && tid == 0) a.tile_flags[tile] = TF_GH | TF_GT | TF_SH | TF_ST;
     return;
   }
@@ -1011,6 +1200,10 @@ __global__ void __launch_bounds__(CT_THREADS, MODE == 1 ? 3 : 2) conflict_kernel
   A ci[2], co[2];
   ci[0] = ci[1] = co[0] = co[1] = agg_empty_t<A>();
   if (tid == 0) s.unknown = 0;
+  if (MODE == 2) {
+    if (cross_pieces_fast<A>(a, s, tile, tb, cnt, cin, cout, s_need)) return;
+    tile_gather(a, s, tb, cnt, 0, (int)cnt);  // the scan path: every record
+  }
   if (MODE == 2) {
     const A* c = reinterpret_cast<const Q*>(a.carry)[tile].a;  // [grp In, grp Out, sub In, sub Out]
     if (cin) ci[0] = c[0];
@@ -1267,7 +1460,7 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_y_kernel(ConflictArgs a) 
   tile_window(a, tile, &tb, &cnt);
   const KeyLayout& L = a.L;
   const int tid = threadIdx.x;
-  if (cnt == 0 || !tile_load(a, s, tb, cnt)) return;
+  if (cnt == 0 || !tile_load<false>(a, s, tb, cnt)) return;
   const bool cin = !(s.fl[0] & FL_GH), cout = !(s.fl[cnt - 1] & FL_GT);
   const int ftail = s.first_gtail, lhead = s.last_ghead;
   __shared__ F5 s_x[2][2];
@@ -1296,12 +1489,15 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_y_kernel(ConflictArgs a) 
     }
   }
   __syncthreads();
+  // records of the pieces only
+  if (s_owner[0] != ~0u && (s_has[0][0] || s_has[0][1])) tile_gather(a, s, tb, cnt, 0, min(ftail, (int)cnt - 1) + 1);
+  if (s_owner[1] != ~0u && (s_has[1][0] || s_has[1][1])) tile_gather(a, s, tb, cnt, lhead, (int)cnt);
   const int j0 = tid * CT_ITEMS;
 #pragma unroll
   for (int q = 0; q < CT_ITEMS; q++) {
     const int j = j0 + q;
     if (j >= (int)cnt || !(s.fl[j] & FL_INT)) continue;
-    const bool A = cin && j <= ftail, B = cout && j >= lhead && s_owner[1] != ~0u;
+    const bool A = cin && j <= ftail && s_owner[0] != ~0u, B = cout && j >= lhead && s_owner[1] != ~0u;
     const int g = A ? 0 : (B ? 1 : -1);
     if (g < 0) continue;
     const F5 me = fields(s, j);
