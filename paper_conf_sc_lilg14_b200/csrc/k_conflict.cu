@@ -43,9 +43,11 @@ __device__ __forceinline__ Agg agg_empty() {
   return r;
 }
 
+// (per-type fields set by selects: an index by the runtime access type would put the summary in local memory)
 __device__ __forceinline__ Agg agg_item(u32 rw, u32 id, u64 vh) {
   Agg r = agg_empty();
-  r.mn[rw] = r.mx[rw] = id;
+#pragma unroll
+  for (int x = 0; x < 3; x++) r.mn[x] = rw == (u32)x ? id : ~0u, r.mx[x] = rw == (u32)x ? id : 0u;
   if (rw == RW_WRITE) {
     r.v1 = r.v2 = vh;
     r.i1 = r.i2 = id;
@@ -140,7 +142,8 @@ __device__ __forceinline__ Agg agg_item_t<Agg>(u32 rw, u32 id, u64 vh) { return 
 template <>
 __device__ __forceinline__ AggC agg_item_t<AggC>(u32 rw, u32 id, u64 vh) {
   AggC r = agg_empty_t<AggC>();
-  r.mn[rw] = r.mx[rw] = id;
+#pragma unroll
+  for (int x = 0; x < 3; x++) r.mn[x] = rw == (u32)x ? id : ~0u, r.mx[x] = rw == (u32)x ? id : 0u;
   if (rw == RW_WRITE) r.vlo = r.vhi = vh;
   return r;
 }
