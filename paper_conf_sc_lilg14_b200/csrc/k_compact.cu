@@ -114,7 +114,7 @@ __global__ void compact_gather_kernel(const u64* __restrict__ seg, u32 rw, u32 n
 static u32 compact_warps(u64 m, u32* rw_out) {
   // resident warps of one full wave on this device (both variants: the smaller occupancy)
   const int a = blocks_per_sm((const void*)compact_seg_kernel<12, true>, 256, 0);
-  const int b = blocks_per_sm((const void*)compact_seg_kernel<12, false>, 256, 0);
+  const int b = blocks_per_sm((const void*)compact_seg_kernel<8, false>, 256, 0);
   const u64 target = (u64)dev_sm_count() * 8 * (u64)std::max(1, std::min(a, b));
   u64 rw = (m + target - 1) / target;
   rw = std::max<u64>(256, (rw + 255) / 256 * 256);
@@ -152,7 +152,7 @@ u64* launch_compact_multi(const u64* keys, u32 m, const KeyLayout& L, u64* seg, 
     R.mask_s = ~((sh_shared >= 64) ? ~0ull : ((1ull << sh_shared) - 1ull));
     R.mask_g = ~((sh_global >= 64) ? ~0ull : ((1ull << sh_global) - 1ull));
     R.mask_fixed = L.single_space == SP_GLOBAL ? R.mask_g : R.mask_s;
-    compact_seg_kernel<12, false><<<grid, 256, 0, st>>>(keys, m, R, rw, seg, cnt);
+    compact_seg_kernel<8, false><<<grid, 256, 0, st>>>(keys, m, R, rw, seg, cnt);
   }
   launch_scan_exclusive_u32(cnt, off, nw, stemp, st);
   compact_gather_kernel<<<grid, 256, 0, st>>>(seg, rw, nw, cnt, off, out);

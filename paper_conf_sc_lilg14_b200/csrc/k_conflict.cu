@@ -1141,51 +1141,88 @@ __device__ bool cross_pieces_fast(const ConflictArgs& a, TileSmem& s, u32 tile, 
 }
 
 // ------------------------------------------------------------------------------------------------ mode 1 / 2
-template <int MODE, class A>
-// mode 1 at 3 CTAs/SM (the shared-memory limit): up to 80 registers, no spills; mode 2 at 2 (128 registers)
-__global__ void __launch_bounds__(CT_THREADS, MODE == 1 ? 3 : 2) conflict_kernel(ConflictArgs a) {
+// Mode 2: which crossing pieces of a tile can still lower a witness x.  A crossing piece matters for a kind K
+// only if its run's whole summary allows a K pair and — for the piece a run crosses IN with (its head lies in an
+// earlier tile), in position-ordered runs (lowG == 0) — no entry before this tile is flagged K yet: x_K is a
+// minimum position.  need[piece][kind] (piece 0 = crossing in, 1 = crossing out); returns true if nothing is
+// needed (C4's `changed`, the far tiles of C3's hot bins, the second tile of a crossing dist[v]).
+template <class A>
+__device__ bool mode2_skip(const ConflictArgs& a, u32 tile, u8 need[2][2]) {
+  typedef typename OpOf<A>::type Op;
   typedef typename QuadOf<A>::type Q;
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
-  const u32 tile = MODE == 1 ? blockIdx.x : a.cross_list[blockIdx.x];
+  need[0][0] = need[0][1] = need[1][0] = need[1][1] = 0;
+  const u8 tf = a.tile_flags[tile];
+  const A* c = reinterpret_cast<const Q*>(a.carry)[tile].a;    // [grp In, grp Out, ...]
+  const A* pp = reinterpret_cast<const Q*>(a.part)[tile].a;    // [grp P, grp S, ...]
+  const bool middle = (tf & TF_CIN) && (tf & TF_COUT) && !(tf & TF_GH);
+  bool skip = true;
+  if ((tf & TF_CIN) && a.phase != 1) {  // piece A: the run crossing in (the whole tile if middle)
+    bool done[2];
+    const A run = middle ? Op()(Op()(c[0], pp[0]), c[1]) : Op()(c[0], pp[0]);
+    cannot_race(run, &done[0], &done[1]);
+    if (a.L.lowG == 0) {  // the window starts at the nominal start: the run crossing there is long
+      const u64 first = pos_of(a.L, a.keys[(u64)tile * CT_NOM]);
+      const Slot* sl = &a.slots[a.owner[tile]];
+      for (int k = 0; k < 2; k++) {
+        const u64 x = ld_volatile(&sl->x[k]);
+        done[k] = done[k] || (x != ~0ull && (x >> 32) < first);
+      }
+    }
+    skip = skip && done[0] && done[1];
+    need[0][0] = !done[0], need[0][1] = !done[1];
+  }
+  if ((tf & TF_COUT) && (tf & TF_GH) && a.phase != 2) {  // piece B: a run starting here and crossing out
+    bool done[2];
+    cannot_race(Op()(pp[1], c[1]), &done[0], &done[1]);
+    skip = skip && done[0] && done[1];
+    need[1][0] = !done[0], need[1][1] = !done[1];
+  }
+  return skip;
+}
+
+// Mode 3: does a crossing run this tile takes part in have a witness x (and, position-ordered, no partner y
+// before this tile yet)?
+__device__ bool mode3_any(const ConflictArgs& a, u32 tile) {
+  const u8 tf = a.tile_flags[tile];
+  bool any = false;
+  if ((tf & TF_CIN) && a.phase != 1) {
+    const Slot& sl = a.slots[a.owner[tile]];
+    if (a.L.lowG == 0) {
+      const u64 first = pos_of(a.L, a.keys[(u64)tile * CT_NOM]);
+      for (int k = 0; k < 2; k++) {
+        const u64 y = ld_volatile(&sl.y[k]);
+        any |= sl.x[k] != ~0ull && !(y != ~0ull && (y >> 32) < first);
+      }
+    } else {
+      any |= sl.x[0] != ~0ull || sl.x[1] != ~0ull;
+    }
+  }
+  if ((tf & TF_COUT) && (tf & TF_GH) && a.phase != 2) {
+    const Slot& sl = a.slots[tile];
+    any |= sl.x[0] != ~0ull || sl.x[1] != ~0ull;
+  }
+  return any;
+}
+
+// Modes 2/3 run persistent CTAs over a worklist of the crossing tiles that still have work (one thread per
+// crossing tile decides): skipped tiles cost no CTA launch (C4: 133 K crossing tiles, most skipped in phase 2).
+template <class A>
+__global__ void cross_filter_kernel(ConflictArgs a, u32 ncross, int mode) {
+  const u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= ncross) return;
+  const u32 tile = a.cross_list[i];
+  u8 need[2][2];
+  const bool keep = mode == 2 ? !mode2_skip<A>(a, tile, need) : mode3_any(a, tile);
+  if (keep) a.work[atomicAdd(a.work_count, 1u)] = tile;
+}
+
+template <int MODE, class A>
+__device__ void conflict_tile(const ConflictArgs& a, TileSmem& s, u32 tile) {
+  typedef typename QuadOf<A>::type Q;
   __shared__ u8 s_need[2][2];  // mode 2: piece (A = crossing in, B = crossing out) x kind (RW, WW) can lower x
   if (MODE == 2) {
-    // A crossing piece matters for a kind K only if its run's whole summary allows a K pair and — for the
-    // piece a run crosses IN with (its head lies in an earlier tile), in position-ordered runs (lowG == 0) — no
-    // entry before this tile is flagged K yet: x_K is a minimum position.  A tile whose pieces all cannot lower
-    // any x is skipped (C4's `changed`, the far tiles of C3's hot bins, the second tile of a crossing dist[v]).
     __shared__ int s_skip;
-    if (threadIdx.x == 0) {
-      typedef typename OpOf<A>::type Op;
-      s_need[0][0] = s_need[0][1] = s_need[1][0] = s_need[1][1] = 0;
-      const u8 tf = a.tile_flags[tile];
-      const A* c = reinterpret_cast<const Q*>(a.carry)[tile].a;    // [grp In, grp Out, ...]
-      const A* pp = reinterpret_cast<const Q*>(a.part)[tile].a;    // [grp P, grp S, ...]
-      const bool middle = (tf & TF_CIN) && (tf & TF_COUT) && !(tf & TF_GH);
-      bool skip = true;
-      if ((tf & TF_CIN) && a.phase != 1) {  // piece A: the run crossing in (the whole tile if middle)
-        bool done[2];
-        const A run = middle ? Op()(Op()(c[0], pp[0]), c[1]) : Op()(c[0], pp[0]);
-        cannot_race(run, &done[0], &done[1]);
-        if (a.L.lowG == 0) {  // the window starts at the nominal start: the run crossing there is long
-          const u64 first = pos_of(a.L, a.keys[(u64)tile * CT_NOM]);
-          const Slot* sl = &a.slots[a.owner[tile]];
-          for (int k = 0; k < 2; k++) {
-            const u64 x = ld_volatile(&sl->x[k]);
-            done[k] = done[k] || (x != ~0ull && (x >> 32) < first);
-          }
-        }
-        skip = skip && done[0] && done[1];
-        s_need[0][0] = !done[0], s_need[0][1] = !done[1];
-      }
-      if ((tf & TF_COUT) && (tf & TF_GH) && a.phase != 2) {  // piece B: a run starting here and crossing out
-        bool done[2];
-        cannot_race(Op()(pp[1], c[1]), &done[0], &done[1]);
-        skip = skip && done[0] && done[1];
-        s_need[1][0] = !done[0], s_need[1][1] = !done[1];
-      }
-      s_skip = skip;
-    }
+    if (threadIdx.x == 0) s_skip = mode2_skip<A>(a, tile, s_need);
     __syncthreads();
     if (s_skip) return;
   }
@@ -1424,37 +1461,29 @@ __global__ void __launch_bounds__(CT_THREADS, MODE == 1 ? 3 : 2) conflict_kernel
   }
 }
 
-// ------------------------------------------------------------------------------------------------ mode 3: y
-__global__ void __launch_bounds__(CT_THREADS) conflict_y_kernel(ConflictArgs a) {
+template <int MODE, class A>
+// mode 1 at 3 CTAs/SM (the shared-memory limit): up to 80 registers, no spills; mode 2 at 2 (128 registers)
+__global__ void __launch_bounds__(CT_THREADS, MODE == 1 ? 3 : 2) conflict_kernel(ConflictArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
-  const u32 tile = a.cross_list[blockIdx.x];
-  {
-    // nothing to do unless a crossing run this tile takes part in has a witness x
-    __shared__ int s_any;
-    if (threadIdx.x == 0) {
-      const u8 tf = a.tile_flags[tile];
-      bool any = false;
-      if ((tf & TF_CIN) && a.phase != 1) {
-        const Slot& sl = a.slots[a.owner[tile]];
-        if (a.L.lowG == 0) {
-          // the run crossing in, position-ordered: y_K (a minimum position) cannot come from here if a partner
-          // before this tile is known
-          const u64 first = pos_of(a.L, a.keys[(u64)tile * CT_NOM]);
-          for (int k = 0; k < 2; k++) {
-            const u64 y = ld_volatile(&sl.y[k]);
-            any |= sl.x[k] != ~0ull && !(y != ~0ull && (y >> 32) < first);
-          }
-        } else {
-          any |= sl.x[0] != ~0ull || sl.x[1] != ~0ull;
-        }
-      }
-      if ((tf & TF_COUT) && (tf & TF_GH) && a.phase != 2) {
-        const Slot& sl = a.slots[tile];
-        any |= sl.x[0] != ~0ull || sl.x[1] != ~0ull;
-      }
-      s_any = any;
+  if (MODE == 1) {
+    conflict_tile<MODE, A>(a, s, blockIdx.x);
+  } else {
+    const u32 nw = *a.work_count;
+    for (u32 w = blockIdx.x; w < nw; w += gridDim.x) {
+      conflict_tile<MODE, A>(a, s, a.work[w]);
+      __syncthreads();
     }
+  }
+}
+
+// ------------------------------------------------------------------------------------------------ mode 3: y
+__device__ void y_tile(const ConflictArgs& a, TileSmem& s, u32 tile) {
+  {
+    // nothing to do unless a crossing run this tile takes part in has a witness x (re-checked: other tiles of
+    // the phase may have lowered y since the worklist was made)
+    __shared__ int s_any;
+    if (threadIdx.x == 0) s_any = mode3_any(a, tile);
     __syncthreads();
     if (!s_any) return;
   }
@@ -1513,6 +1542,16 @@ __global__ void __launch_bounds__(CT_THREADS) conflict_y_kernel(ConflictArgs a) 
     const int g = tid >> 1, k = tid & 1;
     if (s_owner[g] != ~0u && s_min[g][k] != ~0ull)
       atomicMin((unsigned long long*)&a.slots[s_owner[g]].y[k], s_min[g][k]);
+  }
+}
+
+__global__ void __launch_bounds__(CT_THREADS) conflict_y_kernel(ConflictArgs a) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
+  const u32 nw = *a.work_count;
+  for (u32 w = blockIdx.x; w < nw; w += gridDim.x) {
+    y_tile(a, s, a.work[w]);
+    __syncthreads();
   }
 }
 
@@ -1669,19 +1708,26 @@ static void launch_ck(const ConflictArgs& a, u32 nblocks, cudaStream_t st) {
   conflict_kernel<MODE, A><<<nblocks, CT_THREADS, sm, st>>>(a);
 }
 
+// modes 2/3: nblocks = crossing tiles; a filter kernel makes the worklist, persistent CTAs (one full wave) take it
 void launch_conflict(int mode, bool exact, const ConflictArgs& a, u32 nblocks, cudaStream_t st) {
   if (!nblocks) return;
   const size_t sm = sizeof(TileSmem);
   if (mode == 1) {
     if (exact) launch_ck<1, Agg>(a, nblocks, st);
     else launch_ck<1, AggC>(a, nblocks, st);
-  } else if (mode == 2) {
-    if (exact) launch_ck<2, Agg>(a, nblocks, st);
-    else launch_ck<2, AggC>(a, nblocks, st);
-  } else {
-    smem_optin((const void*)conflict_y_kernel, sm);
-    conflict_y_kernel<<<nblocks, CT_THREADS, sm, st>>>(a);
+    return;
   }
+  cudaMemsetAsync(a.work_count, 0, 4, st);
+  if (exact) cross_filter_kernel<Agg><<<(nblocks + 255) / 256, 256, 0, st>>>(a, nblocks, mode);
+  else cross_filter_kernel<AggC><<<(nblocks + 255) / 256, 256, 0, st>>>(a, nblocks, mode);
+  const void* k = mode == 3 ? (const void*)conflict_y_kernel
+                            : exact ? (const void*)conflict_kernel<2, Agg> : (const void*)conflict_kernel<2, AggC>;
+  smem_optin(k, sm);
+  const u32 wave = (u32)(dev_sm_count() * std::max(1, blocks_per_sm(k, CT_THREADS, sm)));
+  const u32 grid = std::min(nblocks, wave);
+  if (mode == 3) conflict_y_kernel<<<grid, CT_THREADS, sm, st>>>(a);
+  else if (exact) conflict_kernel<2, Agg><<<grid, CT_THREADS, sm, st>>>(a);
+  else conflict_kernel<2, AggC><<<grid, CT_THREADS, sm, st>>>(a);
 }
 
 void launch_cross_emit(const ConflictArgs& a, u32 ncross, cudaStream_t st) {

@@ -137,6 +137,8 @@ struct ConflictArgs {
   u32 phase;  // modes 2/3: 0 = every crossing piece, 1 = pieces starting a run (crossing out), 2 = the rest
   u32 tdiv;   // > 1: a record's identity is thread / tdiv (precise warp model, inter-warp half)
   const u32* tstart;  // [tiles + 1]: first entry of every tile window (launch_tile_starts)
+  u32* work;          // modes 2/3: crossing tiles with work (cross_filter_kernel), count in *work_count
+  u32* work_count;
 };
 
 struct RaceOut {  // == sesa_race (40 bytes)

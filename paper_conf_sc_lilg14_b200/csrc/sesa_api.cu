@@ -80,7 +80,7 @@ static unsigned kernels_of(const char* name) {
     const char* n;
     unsigned k;
   } tab[] = {{"tile_offsets", 3}, {"compact", 4}, {"carry", 3}, {"alltoall", 0}, {"flow_pairs", 2},
-                 {"owner_partition", 4}};  // alltoall: NCCL's kernels
+                 {"owner_partition", 4}, {"conflict_cross", 2}, {"conflict_y", 2}};  // alltoall: NCCL's kernels
   for (const auto& e : tab)
     if (!strcmp(e.n, name)) return e.k;
   return 1;
@@ -576,7 +576,7 @@ bool sesa_trace::step_conflict(const u64* comp, u32 m2, const Rec* rec, u32 rec_
         !grow(b_rkeys[0], (size_t)race_cap * 8, "race keys") || !grow(b_rkeys[1], (size_t)race_cap * 8, "race keys") ||
         !grow(b_rvals[0], (size_t)race_cap * 4, "race vals") || !grow(b_rvals[1], (size_t)race_cap * 4, "race vals") ||
         !grow(b_carrytmp, carry_temp_bytes(ctiles), "carry temp") ||
-        !grow(b_tstart, ((size_t)ctiles + 1) * 4, "tile starts"))
+        !grow(b_tstart, ((size_t)ctiles + 1) * 4, "tile starts") || !grow(b_work, (size_t)ctiles * 4, "worklist"))
       return false;
     ConflictArgs A;
     memset(&A, 0, sizeof A);
@@ -604,6 +604,8 @@ bool sesa_trace::step_conflict(const u64* comp, u32 m2, const Rec* rec, u32 rec_
     A.slots = (Slot*)b_slots.p;
     A.index_base = index_base;
     A.tstart = (const u32*)b_tstart.p;
+    A.work = (u32*)b_work.p;
+    A.work_count = (u32*)b_ccount.p + 3;
     LAUNCH("tile_starts", 8.0 * m2, launch_tile_starts(A, ctiles, (u32*)b_tstart.p, stream));
     // cheap summaries first; a benign query they cannot decide (>= 2 writers with >= 2 values at one location)
     // makes the whole check rerun with the exact summaries (mode 1 and, for crossing runs, mode 2 can detect it)

@@ -40,7 +40,7 @@ struct sesa_trace {
 
   // device buffers (grow-only, freed by destroy)
   DevBuf b_summary, b_keys[2], b_hist, b_binbase, b_lookback, b_ctr, b_cnt, b_off, b_temp;
-  DevBuf b_tflags, b_part, b_carry, b_owner, b_slots, b_cross, b_ccount, b_carrytmp, b_tstart;
+  DevBuf b_tflags, b_part, b_carry, b_owner, b_slots, b_cross, b_ccount, b_carrytmp, b_tstart, b_work;
   DevBuf b_races, b_rkeys[2], b_rvals[2], b_races_sorted, b_rhist, b_rbase;
   DevBuf b_eoff, b_ecnt, b_ecell, b_hrec, b_dist_races, b_ctmp, b_ctotal, b_thist, b_ftmp, b_thist2, b_btmp2;
   DevBuf b_lraces;  // multi-launch checks: the races of the launches checked so far
@@ -65,7 +65,7 @@ struct sesa_trace {
 
   std::vector<DevBuf*> all_bufs() {
     std::vector<DevBuf*> v = {&b_summary, &b_hist, &b_binbase, &b_lookback, &b_ctr, &b_cnt, &b_off, &b_temp,
-                              &b_tflags, &b_part, &b_carry, &b_owner, &b_slots, &b_cross, &b_ccount, &b_carrytmp, &b_tstart,
+                              &b_tflags, &b_part, &b_carry, &b_owner, &b_slots, &b_cross, &b_ccount, &b_carrytmp, &b_tstart, &b_work,
                               &b_races, &b_races_sorted, &b_rhist, &b_rbase, &b_eoff, &b_ecnt, &b_ecell,
                               &b_hrec, &b_dist_races, &b_ctmp, &b_ctotal, &b_thist, &b_ftmp, &b_thist2, &b_btmp2, &b_lraces, &b_franges, &b_fkeep, &b_fcnt2,
                               &b_foff2, &b_frec, &b_forig, &b_regions,
