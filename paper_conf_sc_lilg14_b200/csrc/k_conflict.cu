@@ -1031,10 +1031,10 @@ __device__ bool cross_pieces_fast(const ConflictArgs& a, TileSmem& s, u32 tile, 
   const int aend = min(ftail, (int)cnt - 1);
   if (pa) tile_gather(a, s, tb, cnt, 0, aend + 1);
   if (pb) tile_gather(a, s, tb, cnt, lhead, (int)cnt);
-  __shared__ int s_fst, s_lsh, s_long;
+  __shared__ int s_fst, s_lsh;
   __shared__ A s_R[2], s_S[2];
   __shared__ unsigned long long s_min[4];
-  if (tid == 0) s_fst = (int)cnt - 1, s_lsh = 0, s_long = 0;
+  if (tid == 0) s_fst = (int)cnt - 1, s_lsh = 0;
   if (tid < 4) s_min[tid] = ~0ull;
   __syncthreads();
   auto in_piece = [&](int j) { return (pa && j <= aend) || (pb && j >= lhead && j < (int)cnt); };
@@ -1051,22 +1051,23 @@ __device__ bool cross_pieces_fast(const ConflictArgs& a, TileSmem& s, u32 tile, 
   const int fst = s_fst, lsh = s_lsh;
   const bool cinS = pa && !(s.fl[0] & FL_SH), coutS = lastp && !(s.fl[cnt - 1] & FL_ST);
   // inner sub-runs (not continuing across an edge) longer than SR_MAX: the scan path
+  bool lng = false;
   for (int j = tid; j < (int)cnt; j += CT_THREADS) {
     if (!in_piece(j) || !(s.fl[j] & FL_SH) || (s.fl[j] & FL_ST) || (coutS && j == lsh)) continue;
     int e = j + 1;
     while (e < (int)cnt - 1 && !(s.fl[e] & FL_ST) && e - j < SR_MAX) e++;
-    if (!(s.fl[e] & FL_ST)) s_long = 1;
+    lng = lng || !(s.fl[e] & FL_ST);
   }
   if (tid == 0) {
     const A* c = reinterpret_cast<const Q*>(a.carry)[tile].a;  // [grp In, grp Out, sub In, sub Out]
     const A* pp = reinterpret_cast<const Q*>(a.part)[tile].a;  // [grp P, grp S, sub P, sub S]
-    const A E = agg_empty_t<A>();
-    s_R[0] = middle ? Op()(Op()(c[0], pp[0]), c[1]) : Op()(c[0], pp[0]);
-    s_R[1] = Op()(pp[1], c[1]);
-    s_S[0] = Op()(Op()(c[2], pp[2]), (fst == (int)cnt - 1 && coutS) ? c[3] : E);
-    s_S[1] = Op()(Op()((lsh == 0 && cinS) ? c[2] : E, pp[3]), c[3]);
+    const A E = agg_empty_t<A>();  // (only the summaries a piece uses: the others are not written this check)
+    if (pa) s_R[0] = middle ? Op()(Op()(c[0], pp[0]), c[1]) : Op()(c[0], pp[0]);
+    if (pb) s_R[1] = Op()(pp[1], c[1]);
+    if (cinS) s_S[0] = Op()(Op()(c[2], pp[2]), (fst == (int)cnt - 1 && coutS) ? c[3] : E);
+    if (coutS) s_S[1] = Op()(Op()((lsh == 0 && cinS) ? c[2] : E, pp[3]), c[3]);
   }
-  if (__syncthreads_or(s_long)) return false;
+  if (__syncthreads_or(lng)) return false;
   const bool ordered = a.L.lowG == 0;
   const u32 ws = a.ws, ls = a.ls;
 #pragma unroll 1

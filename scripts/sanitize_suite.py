@@ -45,6 +45,14 @@ def main():
             t.check(S.to_device(r), n)
             same(t.races(), O.check(r, lockstep=seed % 2, benign=benign), f"random {seed} benign={benign}")
             t.close()
+    # many blocks, medium locations (C4-like): groups of ~100-1000 entries inside and across tile windows with
+    # short sub-runs (mode 1 per-group path, thread and warp groups; mode 2 pieces with edge sub-runs)
+    for ls, words in ((0, 2000), (1, 300)):
+        r = G.random_trace(200000, 21 + ls, threads=32, blocks=2000, words=words, sort=True)
+        t = S.Trace(32, ls, 4)
+        t.check(S.to_device(r), len(r))
+        same(t.races(), O.check(r, lockstep=ls), f"medium groups ls={ls} words={words}")
+        t.close()
     r = G.random_trace(5000, 5, threads=64, words=300, sizes=(1, 6, 16))
     t = S.Trace(32, 0, 1)
     t.check(S.to_device(r), len(r))
