@@ -399,7 +399,7 @@ __device__ __forceinline__ void tile_window(const ConflictArgs& a, u32 tile, u64
 // with the early gather and this load (vs 11.3 with L1-allocating 256-bit loads).
 __device__ __forceinline__ Rec load_rec_gather(const Rec* p) {
   u32 w[8];
-  asm("ld.global.cg.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+  asm("ld.global.cg.L2::64B.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
       : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]), "=r"(w[6]), "=r"(w[7])
       : "l"(p));
   Rec r;
