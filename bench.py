@@ -23,6 +23,7 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "access records race-checked/sec (Grec/s) at 1/2/4/8 B200; % HBM roofline"
+RANDOM_GATHER_GPS = 36.85e9  # 266 M random 32-byte gathers from a 12.5 GB array in 7.22 ms (profiles/r2_gather_mb.txt)
 CONFIGS = {
     "c1": dict(workload="C1 tree reduction 1x64 threads, 6 intervals, 959 records, 1 injected WW", ws=32, ls=0),
     "c2": dict(workload="C2 Parboil-sgemm-shaped 64 blocks x 256 threads, 32 intervals, 18,300,928 records",
@@ -361,6 +362,13 @@ def main():
                 "frac": ach / peak, "traffic": trf, "bytes_per_launch": o["bytes"] / o["launches"],
                 "ms_per_launch": o["ms"] / o["launches"], "peak_source": peak_src,
                 "share_of_step": o["ms"] / max(1e-9, sum(v["ms"] for v in ours.values()))}
+        if dom == "conflict":
+            # the conflict kernel's real bound: one random 32-byte record gather per compacted entry (40 algorithmic
+            # bytes = 8 key + 32 record); B200's random-gather rate measured by scripts/gather_mb.cu (DESIGN 5.5)
+            g = o["bytes"] / 40.0 / (o["ms"] / 1e3)
+            roof["random_gather"] = {"achieved": g / 1e9, "peak": RANDOM_GATHER_GPS / 1e9, "unit": "G gathers/s",
+                                     "frac": g / RANDOM_GATHER_GPS,
+                                     "peak_source": "measured, scripts/gather_mb.cu (profiles/r2_gather_mb.txt)"}
     step_bytes = sum(v["bytes"] for v in kstats.values()) / max(1, args.steps)
 
     # end-to-end through the public API with host buffers (H2D of the records + D2H of the race list each step)
