@@ -32,11 +32,17 @@ namespace sesa {
 // Stable partition of u64 items into W <= 8 buckets.  Warp chunks of 512 items (16 coalesced rows); per-chunk
 // bucket counts -> one exclusive scan over the bucket-major count matrix -> writes.  MODE 0: item = sort key,
 // bucket = mix64(location run key) mod W.  MODE 1: item = key of a compacted entry, emitted as its global
-// position, bucket = owner rank of that position (bases[W+1]); the entry index is written alongside.
+// position, bucket = owner rank of that position (bases[W+1]); the entry index is written alongside.  MODE 2 =
+// MODE 0 with the key formed on the fly from the extents pass's 32-bit granule array (one-granule global records,
+// key_hi = g - gmin < 2^32): the key extraction pass (a second 32-byte read per record) is gone, and both
+// partition sweeps read 4 instead of 8 bytes per record.
 constexpr int PT_ROWS = 16, PT_CHUNK = 32 * PT_ROWS, PT_THREADS = 256;
 
 struct PartArgs {
   const u64* in;
+  const u32* gran;  // MODE 2: granule low halves
+  u32 gmin_lo;      // MODE 2: low 32 bits of the layout's gminG
+  u64 pos_base;     // MODE 2: global position of item 0
   u64 n;
   u32 W;
   int mode;
@@ -48,42 +54,105 @@ struct PartArgs {
   u32* out_src;
 };
 
+// MODE 2 owner: a 32-bit mix of key_hi scaled to [0, W) (one layout for every rank; MODE 0 is never mixed in)
+__device__ __forceinline__ u32 owner32(u32 h, u32 W) {
+  h ^= h >> 16, h *= 0x85EBCA6Bu, h ^= h >> 13, h *= 0xC2B2AE35u, h ^= h >> 16;
+  return __umulhi(h, W);
+}
+
 __device__ __forceinline__ u32 part_bucket(const PartArgs& a, u64 item) {
-  if (a.mode == 0) return (u32)(sesa_mix(group_of_hi(a.L, item >> a.L.pos_bits)) % a.W);
+  // owner = the high half of a 64-bit hash of the location scaled to [0, W) (multiply-shift: a 64-bit modulo by a
+  // runtime W is a ~100-instruction emulated division and made both partition sweeps ALU-bound)
+  if (a.mode != 1) return (u32)(((sesa_mix(group_of_hi(a.L, item >> a.L.pos_bits)) >> 32) * a.W) >> 32);
   const u64 pos = item & lowmask(a.L.pos_bits);
   u32 r = 0;
   while (r + 1 < a.W && pos >= a.bases[r + 1]) r++;
   return r;
 }
 
-template <bool WRITE>
+template <bool WRITE, int MODE>
 __global__ void __launch_bounds__(PT_THREADS) partition_kernel(PartArgs a) {
+  // Per row of 32 items a warp multi-split: three ballots of the bucket bits give every lane the mask of its
+  // bucket peers (rank = peers before it) and lane d the count of bucket d; lane d keeps bucket d's running
+  // offset (a per-bucket ballot loop cost ~100 thread instructions per item).  MODE 0/2 writes: the chunk is
+  // staged per bucket in shared memory (chunk-local bases from the count sweep) and leaves in coalesced runs.
+  constexpr bool STAGE = WRITE && MODE != 1;
+  __shared__ u64 stage[STAGE ? PT_THREADS / 32 : 1][STAGE ? PT_CHUNK : 1];
   const int lane = threadIdx.x & 31;
+  const unsigned lt = lanemask_lt();
   const u64 nch = (a.n + PT_CHUNK - 1) / PT_CHUNK;
   const u64 gw = ((u64)blockIdx.x * PT_THREADS + threadIdx.x) >> 5, nw = ((u64)gridDim.x * PT_THREADS) >> 5;
+  u64* st = stage[STAGE ? (threadIdx.x >> 5) : 0];
+  const bool own = lane < (int)a.W;  // lane d owns bucket d
   for (u64 c = gw; c < nch; c += nw) {
-    u32 run[8];
+    // lane d: global offset of bucket d's part of this chunk (write) and its chunk-local staging base
+    const u32 mycnt = STAGE && own ? a.cnt[(u64)lane * nch + c] : 0u;
+    u32 lbase = mycnt;  // exclusive prefix over the buckets (lanes) of the chunk counts
 #pragma unroll
-    for (int d = 0; d < 8; d++) run[d] = (WRITE && d < (int)a.W) ? a.off[(u64)d * nch + c] : 0u;
+    for (int o = 1; o < 8; o <<= 1) {
+      const u32 y = __shfl_up_sync(~0u, lbase, o);
+      if (lane >= o) lbase += y;
+    }
+    lbase -= mycnt;
+    const u32 goff = WRITE && own ? a.off[(u64)lane * nch + c] : 0u;
+    u32 run = STAGE ? lbase : goff;  // lane d: next slot of bucket d (staging or global)
+    const u32 total = __shfl_sync(~0u, lbase + mycnt, 7);
+    // every row of the chunk in flight first (the sweep was latency-bound one row at a time)
+    u64 items[PT_ROWS];
+#pragma unroll
+    for (int r = 0; r < PT_ROWS; r++) {
+      const u64 i = c * PT_CHUNK + (u64)r * 32 + lane;
+      if (MODE == 2) {  // key_hi in the low half until the bucket is known
+        items[r] = i >= a.n ? 0ull : (u64)(__ldg(a.gran + i) - a.gmin_lo);
+      } else {
+        items[r] = i >= a.n ? 0ull : __ldg(a.in + i);
+      }
+    }
+#pragma unroll
     for (int r = 0; r < PT_ROWS; r++) {
       const u64 i = c * PT_CHUNK + (u64)r * 32 + lane;
       const bool valid = i < a.n;
-      const u64 item = valid ? a.in[i] : 0ull;
-      const u32 b = valid ? part_bucket(a, item) : 99u;
-#pragma unroll
-      for (int d = 0; d < 8; d++) {
-        if (d >= (int)a.W) break;
-        const unsigned m = __ballot_sync(~0u, b == (u32)d);
-        if (WRITE && b == (u32)d) {
-          const u32 o = run[d] + __popc(m & lanemask_lt());
-          a.out[o] = a.mode == 0 ? item : (item & lowmask(a.L.pos_bits));
-          if (a.out_src) a.out_src[o] = (u32)i;
+      u64 item = items[r];
+      u32 b = 0;
+      if (valid) {
+        if (MODE == 2) {
+          b = owner32((u32)item, a.W);
+          item = (item << a.L.pos_bits) | (a.pos_base + i);
+        } else {
+          b = part_bucket(a, item);
         }
-        run[d] += __popc(m);
       }
+      const unsigned vm = __ballot_sync(~0u, valid), m0 = __ballot_sync(~0u, b & 1u),
+                     m1 = __ballot_sync(~0u, b & 2u), m2 = __ballot_sync(~0u, b & 4u);
+      const unsigned peers = vm & ((b & 1u) ? m0 : ~m0) & ((b & 2u) ? m1 : ~m1) & ((b & 4u) ? m2 : ~m2);
+      const u32 d = (u32)lane;  // the bucket this lane counts
+      const unsigned dm = vm & ((d & 1u) ? m0 : ~m0) & ((d & 2u) ? m1 : ~m1) & ((d & 4u) ? m2 : ~m2);
+      const u32 slot = __shfl_sync(~0u, run, (int)b) + __popc(peers & lt);
+      if (valid && WRITE) {
+        if (STAGE) {
+          st[slot] = item;
+        } else {
+          a.out[slot] = MODE != 1 ? item : (item & lowmask(a.L.pos_bits));
+          if (a.out_src) a.out_src[slot] = (u32)i;
+        }
+      }
+      if (own) run += __popc(dm);
     }
-    if (!WRITE && lane == 0)
-      for (int d = 0; d < (int)a.W; d++) a.cnt[(u64)d * nch + c] = run[d];
+    if (STAGE) {
+      u32 LB[8], GO[8];
+#pragma unroll
+      for (int q = 0; q < 8; q++) LB[q] = __shfl_sync(~0u, lbase, q), GO[q] = __shfl_sync(~0u, goff, q);
+      __syncwarp();
+      for (u32 j = lane; j < total; j += 32) {  // bucket of slot j: the last one whose base is <= j
+        u32 dst = 0;
+#pragma unroll
+        for (int q = 0; q < 8; q++)
+          if (q < (int)a.W && j >= LB[q]) dst = GO[q] + (j - LB[q]);
+        a.out[dst] = st[j];
+      }
+      __syncwarp();
+    }
+    if (!WRITE && own) a.cnt[(u64)lane * nch + c] = run;
   }
 }
 
@@ -109,7 +178,7 @@ __global__ void scatter_records_kernel(const Rec* __restrict__ in, const u32* __
 
 // ------------------------------------------------------------------------------------------------ state
 struct RankBufs {
-  DevBuf pcnt, poff, ptmp, send, recv, src, req, reqin, recsend, recback, rec_entry, tot, rkeys, rvals, races, ag;
+  DevBuf pcnt, poff, ptmp, send, recv, src, req, reqin, recsend, recback, rec_entry, tot, rkeys, rvals, races, ag, gran;
 };
 
 struct DistState {
@@ -124,10 +193,13 @@ struct RankInfo {
 };
 
 static bool partition(sesa_trace* t, RankBufs& B, const u64* in, u64 n, u32 W, int mode, const u64* bases,
-                      u64* out_tot /*[W]*/) {
+                      u64* out_tot /*[W]*/, const u32* gran = nullptr, u64 pos_base = 0) {
   PartArgs a;
   memset(&a, 0, sizeof a);
   a.in = in;
+  a.gran = gran;
+  a.gmin_lo = (u32)t->layout.gminG;
+  a.pos_base = pos_base;
   a.n = n;
   a.W = W;
   a.mode = mode;
@@ -146,9 +218,17 @@ static bool partition(sesa_trace* t, RankBufs& B, const u64* in, u64 n, u32 W, i
   if (n) {
     const unsigned grid = (unsigned)std::min<u64>((nch + 7) / 8, (u64)t->num_sms * 8);
     t->launch_begin("owner_partition");  // (3 kernels + the scan's one: kernels_of counts them)
-    partition_kernel<false><<<grid, PT_THREADS, 0, t->stream>>>(a);
+    auto sweep = [&](bool write) {
+      if (mode == 2) write ? partition_kernel<true, 2><<<grid, PT_THREADS, 0, t->stream>>>(a)
+                           : partition_kernel<false, 2><<<grid, PT_THREADS, 0, t->stream>>>(a);
+      else if (mode == 1) write ? partition_kernel<true, 1><<<grid, PT_THREADS, 0, t->stream>>>(a)
+                                : partition_kernel<false, 1><<<grid, PT_THREADS, 0, t->stream>>>(a);
+      else write ? partition_kernel<true, 0><<<grid, PT_THREADS, 0, t->stream>>>(a)
+                 : partition_kernel<false, 0><<<grid, PT_THREADS, 0, t->stream>>>(a);
+    };
+    sweep(false);
     launch_scan_exclusive_u32((u32*)B.pcnt.p, (u32*)B.poff.p, nch * W, B.ptmp.p, t->stream);
-    partition_kernel<true><<<grid, PT_THREADS, 0, t->stream>>>(a);
+    sweep(true);
     bucket_totals_kernel<<<1, 32, 0, t->stream>>>((u32*)B.pcnt.p, (u32*)B.poff.p, nch, W, (u64*)B.tot.p);
     t->launch_end(24.0 * (double)n);
     if (!t->cuda_ok(cudaMemcpyAsync(out_tot, B.tot.p, W * 8, cudaMemcpyDeviceToHost, t->stream), "totals")) return false;
@@ -295,7 +375,10 @@ static sesa_status dist_check(std::vector<sesa_trace*>& ts, std::vector<RankIO>&
   std::vector<bool> p1ok(R, true);
   for (int r = 0; r < R; r++) {
     if (io[r].n && !ts[r]->check_records_ptr((const sesa_access*)io[r].rec, io[r].n)) p1ok[r] = false;
-    else if (!ts[r]->step_extents(io[r].rec, io[r].n)) p1ok[r] = false;
+    // (+ the 32-bit granule array: the owner partition forms the keys from it when the global layout allows)
+    else if (!ts[r]->grow(ts[r]->ds->b.gran, std::max<u64>(io[r].n, 1) * 4, "granules") ||
+             !ts[r]->step_extents(io[r].rec, io[r].n, false, (u32*)ts[r]->ds->b.gran.p))
+      p1ok[r] = false;
     if (!p1ok[r] && !ex) return fail_all(ts, ts[r]), ts[r]->status;
   }
   // --- X1: summaries + shard boundaries
@@ -421,8 +504,14 @@ static sesa_status dist_check(std::vector<sesa_trace*>& ts, std::vector<RankIO>&
     const u64 mloc = t->h_summary.entries;
     sendp[r] = t->ds->b.send.p;
     recvb[r] = &t->b_keys[1];  // received keys land in b_keys[1], then are copied/swapped into b_keys[0]
-    ok = t->step_extract(io[r].rec, io[r].n, mloc, io[r].index_base - base0, S.multi != 0) &&
-         partition(t, t->ds->b, (const u64*)t->b_keys[0].p, mloc, W, 0, nullptr, scnt[r].data());
+    const KeyLayout& L = t->layout;
+    const bool fused = S.multi == 0 && !L.both && L.single_space == SP_GLOBAL && L.lowG == 0 && L.sort_bits <= 32;
+    if (fused)  // keys formed from the granule array inside the partition sweeps
+      ok = partition(t, t->ds->b, nullptr, mloc, W, 2, nullptr, scnt[r].data(), (const u32*)t->ds->b.gran.p,
+                     io[r].index_base - base0);
+    else
+      ok = t->step_extract(io[r].rec, io[r].n, mloc, io[r].index_base - base0, S.multi != 0) &&
+           partition(t, t->ds->b, (const u64*)t->b_keys[0].p, mloc, W, 0, nullptr, scnt[r].data());
     sendp[r] = t->ds->b.send.p;
     if (!ok) fail_all(ts, t);
   }
@@ -550,7 +639,7 @@ void sesa_trace::destroy_dist() {
   if (!ds) return;
   RankBufs& B = ds->b;
   for (DevBuf* b : {&B.pcnt, &B.poff, &B.ptmp, &B.send, &B.recv, &B.src, &B.req, &B.reqin, &B.recsend, &B.recback,
-                    &B.rec_entry, &B.tot, &B.rkeys, &B.rvals, &B.races, &B.ag})
+                    &B.rec_entry, &B.tot, &B.rkeys, &B.rvals, &B.races, &B.ag, &B.gran})
     if (b->p) cudaFree(b->p), b->p = nullptr;
   if (ds->comm) ncclCommDestroy(ds->comm);
   delete ds;

@@ -219,7 +219,7 @@ bool sesa_trace::check_records_ptr(const sesa_access* d_rec, u64 n) {
 }
 
 // step 1: validation + extents of the local records -> h_summary (synchronises)
-bool sesa_trace::step_extents(const Rec* rec, u64 n, bool tile_hist) {
+bool sesa_trace::step_extents(const Rec* rec, u64 n, bool tile_hist, u32* gran_out) {
   const u32 log2G = (u32)__builtin_ctz(cfg.granularity);
   if (!grow(b_summary, sizeof(Summary), "summary")) return false;
   // per-tile raw digit histograms for the fused first pass (worth it only for traces of many tiles)
@@ -241,10 +241,11 @@ bool sesa_trace::step_extents(const Rec* rec, u64 n, bool tile_hist) {
   if (!cuda_ok(cudaMemcpyAsync(b_summary.p, &h_summary, sizeof(Summary), cudaMemcpyHostToDevice, stream), "summary init"))
     return false;
   const int grid_stream = (int)std::min<u64>((n + 255) / 256, (u64)num_sms * 8);
-  LAUNCH("extents", (have_thist ? 36.0 : 32.0) * n, launch_extents(rec, n, log2G, (Summary*)b_summary.p,
+  // the 32-bit granule array: for the fused first pass (b_keys[0]) or the caller's (distributed owner partition)
+  u32* gout = have_thist ? (u32*)b_keys[0].p : gran_out;
+  LAUNCH("extents", (gout ? 36.0 : 32.0) * n, launch_extents(rec, n, log2G, (Summary*)b_summary.p,
                                              have_thist ? (u32*)b_thist.p : nullptr, (const Region*)b_regions.p,
-                                             n_regions, n_regions_shared, grid_stream, stream,
-                                             have_thist ? (u32*)b_keys[0].p : nullptr,
+                                             n_regions, n_regions_shared, grid_stream, stream, gout,
                                              have_thist2 ? (u32*)b_thist2.p : nullptr));
   if (!cuda_ok(cudaMemcpyAsync(&h_summary, b_summary.p, sizeof(Summary), cudaMemcpyDeviceToHost, stream), "summary"))
     return false;

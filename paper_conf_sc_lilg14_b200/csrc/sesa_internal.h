@@ -111,7 +111,7 @@ struct sesa_trace {
   // pipeline steps (shared by the single-GPU and the distributed check)
   void begin_check(uint64_t n);
   bool check_records_ptr(const sesa_access* d_rec, uint64_t n);
-  bool step_extents(const sesa::Rec* rec, uint64_t n, bool tile_hist = false);
+  bool step_extents(const sesa::Rec* rec, uint64_t n, bool tile_hist = false, uint32_t* gran_out = nullptr);
   bool report_bad(const sesa_access* d_rec, uint64_t local_bad, uint64_t global_bad);
   void set_oob(const sesa_access* d_rec, uint64_t count, uint64_t local_first, uint64_t index_base);
   bool step_extract(const sesa::Rec* rec, uint64_t n, uint64_t m, uint64_t pos_base, bool multi);
