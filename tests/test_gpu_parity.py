@@ -641,3 +641,39 @@ def test_bucket_path_on_key_arrays(sesa):
     t.close()
     assert info["bucket_path"] == 1 and info["fused_first_pass"] == 0
     assert got.tobytes() == O.check(r, method="partitioned").tobytes()
+
+
+# ------------------------------------------------------------------------------------- conflict fast paths (round 2)
+# Mode 1 decides groups wholly inside a tile window group by group (one thread per group of <= 16 entries, one warp
+# per longer group; partners in other blocks from the group summary, inside the (block, interval) sub-run pair by
+# pair); a window with an inner sub-run > 64 entries keeps the segmented scans; mode 2 decides crossing pieces from
+# carried summaries (edge sub-runs) or pair by pair.  These traces aim at each branch and at their boundaries.
+@pytest.mark.parametrize("threads,words,sort", [(32, 4000, True), (32, 400, True), (2, 3000, True), (512, 60, True),
+                                                (32, 4000, False), (512, 60, False)])
+def test_conflict_group_paths(sesa, threads, words, sort):
+    # many blocks x few threads: short sub-runs, groups of ~10-1000 entries inside and across windows;
+    # 512 threads over 60 words: sub-runs longer than 64 (scan path); unsorted input: runs ordered by
+    # (block, interval) first (lowG > 0: the x / y searches cannot stop early)
+    r = G.random_trace(120000, 4242 + threads + words, blocks=3000 if threads < 512 else 4, threads=threads,
+                       intervals=2, words=words, shared_frac=0.0, sort=sort, values=2)
+    for ls in (0, 1):
+        assert_same(sesa, r, 32, ls, 4)
+
+
+@pytest.mark.parametrize("glen", [2, 15, 16, 17, 31, 32, 33, 64, 65, 1535, 1536, 1537, 4000])
+def test_conflict_group_length_boundaries(sesa, glen):
+    # one location per group of exactly glen entries (thread / warp group boundary at 16, warp chunks of 32,
+    # tile window 1536): reads by many threads, one write in the middle by another block, another location after
+    rng = np.random.default_rng(glen)
+    n = glen * 7
+    r = np.zeros(n, G.REC_DTYPE)
+    r["space"] = G.GLOBAL
+    r["size"] = 4
+    r["block"] = np.arange(n) // 7
+    r["thread"] = rng.integers(0, 64, n)
+    r["interval"] = 0
+    r["addr"] = 0x10000000000 + 4 * (np.arange(n) % 7)
+    r["rw"] = np.where(rng.random(n) < 0.1, G.WRITE, G.READ)
+    r["value_hash"] = rng.integers(0, 2, n)
+    for ls in (0, 1):
+        assert_same(sesa, r, 32, ls, 4)
