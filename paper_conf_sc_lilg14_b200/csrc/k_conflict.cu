@@ -489,9 +489,9 @@ __device__ bool tile_load(const ConflictArgs& a, TileSmem& s, u64 tb, u32 cnt) {
     // the backward carry of a run crossing out of a short window reaches its last real item (cnt - 1)
     u8 f = j < (int)cnt ? (FL_GH | FL_GT) : 0;
     if (j < (int)cnt) {
-      const u64 g = group_of_hi(L, s.key[j + 1] >> L.pos_bits);
-      const bool sp = (j > 0 || tb > 0) && group_of_hi(L, s.key[j] >> L.pos_bits) == g;
-      const bool sn = (j + 1 < (int)cnt || tb + cnt < a.m) && group_of_hi(L, s.key[j + 2] >> L.pos_bits) == g;
+      const u64 kj = s.key[j + 1];
+      const bool sp = (j > 0 || tb > 0) && same_group(L, s.key[j], kj);
+      const bool sn = (j + 1 < (int)cnt || tb + cnt < a.m) && same_group(L, kj, s.key[j + 2]);
       f = (sp ? 0 : FL_GH) | (sn ? 0 : FL_GT) | ((sp || sn) ? FL_INT : 0);
       any |= sp || sn;
       if (f & FL_GT) atomicMin(&s.first_gtail, j);
@@ -765,15 +765,33 @@ __device__ __forceinline__ Agg shfl_x(const Agg& a, int o) {
   return r;
 }
 
-// a partner of e in another block (G: the group's exact summary, identity = block): RW / WW
-__device__ __forceinline__ void flags_other_block(const Agg& G, const F5& e, bool* rwf, bool* wwf) {
+__device__ __forceinline__ AggC shfl_x(const AggC& a, int o) {
+  AggC r;
+#pragma unroll
+  for (int x = 0; x < 3; x++) r.mn[x] = __shfl_xor_sync(~0u, a.mn[x], o), r.mx[x] = __shfl_xor_sync(~0u, a.mx[x], o);
+  r.vlo = __shfl_xor_sync(~0u, a.vlo, o), r.vhi = __shfl_xor_sync(~0u, a.vhi, o);
+  return r;
+}
+
+// The group summary is built cheap first (per type min/max identity, min/max write value): it decides "a plain
+// write of another identity with another value" (false) whenever all plain writes share one value or come from one
+// identity; only otherwise is the exact summary built.
+__device__ __forceinline__ bool cheap_decides(const AggC& G) {
+  return G.vlo == G.vhi || !(G.mn[RW_WRITE] < G.mx[RW_WRITE]);
+}
+__device__ __forceinline__ bool wval_other(const Agg& G, u32 b, u64 v) { return ex_wval(G, b, v); }
+__device__ __forceinline__ bool wval_other(const AggC&, u32, u64) { return false; }  // (cheap_decides holds)
+
+// a partner of e in another block (G: the group's summary, identity = block): RW / WW
+template <class S>
+__device__ __forceinline__ void flags_other_block(const S& G, const F5& e, bool* rwf, bool* wwf) {
   const u32 b = e.block;
   if (e.rw == RW_READ) {
     *rwf = ex_id(G, RW_WRITE, b) || ex_id(G, RW_ATOMIC, b);
     *wwf = false;
   } else {
     *rwf = ex_id(G, RW_READ, b);
-    *wwf = e.rw == RW_WRITE ? (ex_id(G, RW_ATOMIC, b) || ex_wval(G, b, e.vh)) : ex_id(G, RW_WRITE, b);
+    *wwf = e.rw == RW_WRITE ? (ex_id(G, RW_ATOMIC, b) || wval_other(G, b, e.vh)) : ex_id(G, RW_WRITE, b);
   }
 }
 
@@ -792,11 +810,10 @@ __device__ __forceinline__ void emit_group(const ConflictArgs& a, const TileSmem
   emit_race(a, s.key[t + 1] >> a.L.pos_bits, kind, x, y, s.blk[t + 1], s.ivl[t + 1]);
 }
 
-// one thread: group [h, t] (>= 2 entries, all gathered)
-__device__ void group_thread(const ConflictArgs& a, const TileSmem& s, int h, int t) {
+// one thread: group [h, t] (>= 2 entries, all gathered), given its summary G
+template <class S>
+__device__ void group_thread_search(const ConflictArgs& a, const TileSmem& s, int h, int t, const S& G) {
   const KeyLayout& L = a.L;
-  Agg G = agg_empty();
-  for (int j = h; j <= t; j++) G = agg_merge(G, agg_item(s.rw[j], s.blk[j + 1], s.vh[j]));
   bool no0, no1;
   cannot_race(G, &no0, &no1);
   if (no0 && no1) return;
@@ -836,14 +853,23 @@ __device__ void group_thread(const ConflictArgs& a, const TileSmem& s, int h, in
   }
 }
 
-// one warp: group [h, t]
-__device__ void group_warp(const ConflictArgs& a, const TileSmem& s, int h, int t) {
+__device__ void group_thread(const ConflictArgs& a, const TileSmem& s, int h, int t) {
+  AggC C = agg_empty_t<AggC>();
+  for (int j = h; j <= t; j++) C = OpAggC()(C, agg_item_t<AggC>(s.rw[j], s.blk[j + 1], s.vh[j]));
+  if (cheap_decides(C)) {
+    group_thread_search(a, s, h, t, C);
+  } else {
+    Agg G = agg_empty();
+    for (int j = h; j <= t; j++) G = agg_merge(G, agg_item(s.rw[j], s.blk[j + 1], s.vh[j]));
+    group_thread_search(a, s, h, t, G);
+  }
+}
+
+// one warp: group [h, t], given its summary G (in every lane)
+template <class S>
+__device__ void group_warp_search(const ConflictArgs& a, const TileSmem& s, int h, int t, const S& G) {
   const KeyLayout& L = a.L;
   const int lane = threadIdx.x & 31;
-  Agg G = agg_empty();
-  for (int j = h + lane; j <= t; j += 32) G = agg_merge(G, agg_item(s.rw[j], s.blk[j + 1], s.vh[j]));
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) G = agg_merge(G, shfl_x(G, o));
   bool no0, no1;
   cannot_race(G, &no0, &no1);
   if (no0 && no1) return;
@@ -894,6 +920,23 @@ __device__ void group_warp(const ConflictArgs& a, const TileSmem& s, int h, int 
       if (ordered && y != ~0u) break;
     }
     if (lane == 0) emit_group(a, s, t, (u32)(k + 1), xp[k], y);
+  }
+}
+
+__device__ void group_warp(const ConflictArgs& a, const TileSmem& s, int h, int t) {
+  const int lane = threadIdx.x & 31;
+  AggC C = agg_empty_t<AggC>();
+  for (int j = h + lane; j <= t; j += 32) C = OpAggC()(C, agg_item_t<AggC>(s.rw[j], s.blk[j + 1], s.vh[j]));
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) C = OpAggC()(C, shfl_x(C, o));
+  if (cheap_decides(C)) {  // (warp-uniform: every lane holds the whole summary)
+    group_warp_search(a, s, h, t, C);
+  } else {
+    Agg G = agg_empty();
+    for (int j = h + lane; j <= t; j += 32) G = agg_merge(G, agg_item(s.rw[j], s.blk[j + 1], s.vh[j]));
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) G = agg_merge(G, shfl_x(G, o));
+    group_warp_search(a, s, h, t, G);
   }
 }
 

@@ -1,39 +1,32 @@
-"""Summarise an ncu --metrics launch list (csv log): per-kernel launches, device time, DRAM bytes, and share.
-usage: python scripts/launch_summary.py gpurun_out/launches_*.csv"""
+"""Summarise an ncu launch list (gpu__time_duration.sum [+ dram bytes]) of `bench.py`: the LAST step (from the
+last extents launch on), time per kernel family and its share of the step.  Cold-cache and serialised per launch:
+compare shares, not absolute times, with the bench line."""
 import csv
 import sys
+from collections import OrderedDict, defaultdict
 
-
-def summarise(path):
-    lines = [l for l in open(path) if not l.startswith("==")]
-    rows = list(csv.reader(lines))
-    h = rows[0]
-    name, mn, mv, idc = h.index("Kernel Name"), h.index("Metric Name"), h.index("Metric Value"), h.index("ID")
-    mu = h.index("Metric Unit")
-    scale = {"nsecond": 1.0, "usecond": 1e3, "msecond": 1e6, "second": 1e9, "byte": 1.0, "Kbyte": 1e3, "Mbyte": 1e6,
-             "Gbyte": 1e9}
-    per = {}
-    for r in rows[1:]:
-        if len(r) <= mv:
-            continue
-        per.setdefault((r[idc], r[name].split("(")[0].replace("void ", "")[:48]), {})[r[mn]] = \
-            float(r[mv].replace(",", "")) * scale.get(r[mu], 1.0)
-    tot = {}
-    for (_, k), m in per.items():
-        t = tot.setdefault(k, [0, 0.0, 0.0, 0.0])
-        t[0] += 1
-        t[1] += m.get("gpu__time_duration.sum", 0)  # ns
-        t[2] += m.get("dram__bytes_read.sum", 0)
-        t[3] += m.get("dram__bytes_write.sum", 0)
-    alltime = sum(t[1] for t in tot.values())
-    out = []
-    for k, t in sorted(tot.items(), key=lambda x: -x[1][1]):
-        out.append(f"{k:50s} {t[0]:4d} launches {t[1] / 1e6:9.3f} ms {100 * t[1] / alltime:5.1f}%  "
-                   f"dram rd {t[2] / 1e9:7.2f} GB wr {t[3] / 1e9:7.2f} GB")
-    return out
-
-
-if __name__ == "__main__":
-    for p in sys.argv[1:]:
-        print("==", p)
-        print("\n".join(summarise(p)))
+rows = list(csv.reader(open(sys.argv[1])))
+h, L = None, OrderedDict()
+for r in rows:
+    if r and r[0] == "ID":
+        h = r
+        continue
+    if h and len(r) == len(h):
+        d = dict(zip(h, r))
+        e = L.setdefault(d["ID"], {"name": d["Kernel Name"].split("(")[0].replace("void ", "")})
+        e[d["Metric Name"]] = float(d["Metric Value"].replace(",", ""))
+ls = list(L.values())
+last = max(i for i, x in enumerate(ls) if "extents2" in x["name"])
+step = ls[last:]
+agg = defaultdict(lambda: [0, 0.0, 0.0, 0.0])
+for x in step:
+    k = x["name"][:60]
+    agg[k][0] += 1
+    agg[k][1] += x.get("gpu__time_duration.sum", 0) / 1e6
+    agg[k][2] += x.get("dram__bytes_read.sum", 0) / 1e9
+    agg[k][3] += x.get("dram__bytes_write.sum", 0) / 1e9
+tot = sum(v[1] for v in agg.values())
+print(f"{sys.argv[1]}: last step, {len(step)} launches, {tot:.2f} ms of kernel time (ncu, serialised)")
+print(f"{'kernel':62s} {'n':>3s} {'ms':>8s} {'share':>6s} {'DRAM R GB':>10s} {'W GB':>7s}")
+for k, v in sorted(agg.items(), key=lambda x: -x[1][1]):
+    print(f"{k:62s} {v[0]:3d} {v[1]:8.3f} {v[1] / tot:6.3f} {v[2]:10.3f} {v[3]:7.3f}")

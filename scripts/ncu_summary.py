@@ -1,37 +1,34 @@
-"""Summarise ncu reports: python scripts/ncu_summary.py gpurun_out/prof_*.ncu-rep"""
+"""Key metrics of every kernel in an ncu --set full report (for profiles/): duration, DRAM bytes, instructions,
+occupancy, registers, the top warp-stall reasons."""
 import csv
 import io
 import subprocess
 import sys
 
-KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
-        "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "sm__throughput.avg.pct_of_peak_sustained_elapsed",
-        "sm__warps_active.avg.pct_of_peak_sustained_active", "launch__registers_per_thread", "launch__grid_size",
-        "launch__occupancy_limit_registers", "launch__occupancy_limit_shared_mem", "smsp__inst_executed.sum"]
+for rep in sys.argv[1:]:
+    raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    r = list(csv.reader(io.StringIO(raw)))
+    h, units = r[0], dict(zip(r[0], r[1]))
+    scale = {"ns": 1e-6, "us": 1e-3, "usecond": 1e-3, "msecond": 1.0, "ms": 1.0, "nsecond": 1e-6, "second": 1e3,
+             "byte": 1e-9, "Kbyte": 1e-6, "Mbyte": 1e-3, "Gbyte": 1.0, "Tbyte": 1e3}
+    print(f"== {rep}")
+    for row in r[2:]:
+        d = dict(zip(h, row))
 
-
-def summary(path, extra=False):
-    out = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
-    rows = list(csv.reader(io.StringIO(out)))
-    if len(rows) < 3:
-        return {}
-    h, units, v = rows[0], rows[1], rows[2]
-    d = {k: f"{v[h.index(k)]} {units[h.index(k)]}".strip() for k in KEYS if k in h}
-    d["kernel"] = v[h.index("Kernel Name")] if "Kernel Name" in h else "?"
-    if extra:
-        for i, name in enumerate(h):
-            if ("pipe" in name and "inst_executed" in name and name.endswith("avg.pct_of_peak_sustained_active")) or \
-                    (name.startswith("smsp__average_warps_issue_stalled") and name.endswith("per_issue_active.ratio")):
-                try:
-                    if float(v[i]) > 0.5:
-                        d[name] = v[i]
-                except ValueError:
-                    pass
-    return d
-
-
-if __name__ == "__main__":
-    for p in sys.argv[1:]:
-        print("==", p)
-        for k, val in summary(p, extra=True).items():
-            print(f"  {k}: {val}")
+        def f(k, norm=False):  # norm: ms for times, GB for bytes
+            try:
+                v = float(d.get(k, "nan").replace(",", ""))
+            except ValueError:
+                return float("nan")
+            return v * scale.get(units.get(k, ""), 1.0) if norm else v
+        print(f"  {d['Kernel Name'][:70]}")
+        print(f"    duration {f('gpu__time_duration.sum', True):.3f} ms | DRAM read {f('dram__bytes_read.sum', True):.2f} GB"
+              f" write {f('dram__bytes_write.sum', True):.2f} GB | warp instructions {f('smsp__inst_executed.sum') / 1e6:.0f} M"
+              f" | regs {f('launch__registers_per_thread'):.0f} | warps active {f('sm__warps_active.avg.pct_of_peak_sustained_active'):.1f}%"
+              f" | issue active {f('smsp__issue_active.avg.pct_of_peak_sustained_active'):.1f}%"
+              f" | L2 tex read sectors {f('lts__t_sectors_srcunit_tex_op_read.sum') / 1e6:.0f} M")
+        st = {k.replace("smsp__pcsamp_warps_issue_stalled_", ""): f(k) for k in h
+              if k.startswith("smsp__pcsamp_warps_issue_stalled") and not k.endswith("not_issued")}
+        tot = sum(v for v in st.values() if v == v)
+        top = sorted(((v, k) for k, v in st.items() if v == v), reverse=True)[:5]
+        print("    stalls: " + ", ".join(f"{k} {v / tot:.0%}" for v, k in top))

@@ -28,7 +28,7 @@ _traces = {}
 
 def trace(S, ws=32, ls=0, G_=4):
     key = (ws, ls, G_)
-    if key not in _traces:
+    if key not in _traces or not _traces[key].h:  # (a test may have closed the shared handle)
         _traces[key] = S.Trace(ws, ls, G_)
     return _traces[key]
 
