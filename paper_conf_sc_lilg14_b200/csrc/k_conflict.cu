@@ -1181,6 +1181,29 @@ __device__ bool cross_pieces_fast(const ConflictArgs& a, TileSmem& s, u32 tile, 
       if (s_min[3] != ~0ull) atomicMin((unsigned long long*)&sl->x[1], s_min[3]);
     }
   }
+  // Position-ordered runs: piece B is the run's first entries, so an x found there is final, and so is the lowest
+  // partner y found there (any other entry lies later) — search it now, while the records are in shared memory;
+  // mode 3 then skips the run (mode3_any).
+  if (ordered && pb) {
+    __shared__ unsigned long long s_y[2];
+    __shared__ F5 s_X[2];
+    if (tid < 2) {
+      s_y[tid] = ~0ull;
+      if (s_min[2 + tid] != ~0ull) s_X[tid] = fields(s, (int)((u32)s_min[2 + tid] - (u32)tb));
+    }
+    __syncthreads();
+#pragma unroll 1
+    for (int k = 0; k < 2; k++) {
+      if (s_min[2 + k] == ~0ull) continue;
+      for (int c0 = lhead; c0 < (int)cnt; c0 += CT_THREADS) {
+        const int j = c0 + tid;
+        const bool hit = j < (int)cnt && (s.fl[j] & FL_INT) && pair_kind(s_X[k], fields(s, j), ws, ls) == (u32)(k + 1);
+        if (hit) atomicMin(&s_y[k], ((unsigned long long)pos_of(a.L, s.key[j + 1]) << 32) | (u32)(tb + j));
+        if (__syncthreads_or(hit)) break;
+      }
+    }
+    if (tid < 2 && s_y[tid] != ~0ull) atomicMin((unsigned long long*)&a.slots[tile].y[tid], s_y[tid]);
+  }
   return true;
 }
 
@@ -1241,9 +1264,9 @@ __device__ bool mode3_any(const ConflictArgs& a, u32 tile) {
       any |= sl.x[0] != ~0ull || sl.x[1] != ~0ull;
     }
   }
-  if ((tf & TF_COUT) && (tf & TF_GH) && a.phase != 2) {
+  if ((tf & TF_COUT) && (tf & TF_GH) && a.phase != 2) {  // (position-ordered: mode 2 found y with x in this piece)
     const Slot& sl = a.slots[tile];
-    any |= sl.x[0] != ~0ull || sl.x[1] != ~0ull;
+    for (int k = 0; k < 2; k++) any |= sl.x[k] != ~0ull && !(a.L.lowG == 0 && sl.y[k] != ~0ull);
   }
   return any;
 }
