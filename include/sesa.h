@@ -156,7 +156,8 @@ typedef struct {
 
 typedef struct {
   uint64_t n_records, n_entries, n_races;
-  uint64_t n_multi;         /* entries at locations touched >= 2 times (the only ones that can race) */
+  uint64_t n_multi;         /* entries at locations touched >= 2 times (the only ones that can race) — with
+                               wbit_filter, minus (most) entries of locations that no entry writes   */
   uint32_t sort_bits, pos_bits, digit_bits, sort_passes; /* key layout chosen by the extents pass   */
   uint32_t sorted_input;    /* records were (block, interval)-ordered                               */
   uint32_t launches;        /* kernels launched by the last check (all families)                    */
@@ -165,6 +166,8 @@ typedef struct {
   uint32_t fused_first_pass;/* key extract and the first sort pass ran as one kernel   */
   uint32_t bucket_path;     /* the sort ran only over the two high digits and each chunk of 2^15 granules was
                                resolved by a shared-memory bitmap ("bucket path")             */
+  uint32_t wbit_filter;     /* the compaction also dropped read-only locations (a write bit in the sort key,
+                               DESIGN.md §5.6; chosen by a sample of the sorted keys)                        */
 } sesa_check_info;
 
 /* Create a single-GPU handle on the current CUDA device.  cfg is validated (EINVAL on warp_size 0,

@@ -60,6 +60,11 @@ struct KeyLayout {
   u32 bminS, iminS, gbS, ibS, bbS;
   u64 gminG;
   u32 bminG, iminG, gbG, ibG, bbG, lowG;
+  // wbit = 1 (sort + compaction path): the key carries one more bit below the position, set when the entry's
+  // record writes (plain WRITE or ATOMIC): key = key_hi << (pos_bits + 1) | pos << 1 | w.  The order inside a
+  // location run is still by position; compaction uses the bit to drop read-only runs (no race: P:43 needs a
+  // write) and strips it, so every later stage sees the plain layout.
+  u32 wbit;
 };
 
 __device__ __forceinline__ u64 lowmask(u32 b) { return b >= 64 ? ~0ull : ((1ull << b) - 1ull); }

@@ -77,13 +77,16 @@ template <int U>
 // With gout != null the low 32 bits of the granule index addr >> log2G of every record are also written (4 bytes
 // per record,
 // coalesced): the fused pass then reads 8 bytes per record instead of the record's 32-byte sector.
+// With wout != null (and tile_hist) bit (i & 31) of wout[i >> 5] is set iff record i writes (WRITE or ATOMIC):
+// the fused pass puts it into the key (KeyLayout::wbit).
 // With tile_hist2 != null (large traces: candidates for the bucket path, k_bucket.cu) each warp also writes the
 // per-tile histograms of the raw digit (g >> HYB_LO) & 255, and the CTA the histogram of (g >> (HYB_LO + 8)) & 255
 // (bhist[3]): the two global digits of the bucket path.
 __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ rec, u32 n, u32 log2G, u32 rw,
                                                        Summary* __restrict__ out, u32* __restrict__ tile_hist,
                                                        const Region* __restrict__ regs, uint3 rs,
-                                                       u32* __restrict__ gout, u32* __restrict__ tile_hist2) {
+                                                       u32* __restrict__ gout, u32* __restrict__ tile_hist2,
+                                                       u32* __restrict__ wout) {
   __shared__ u32 s_th[8][RADIX];
   __shared__ u32 s_th2[8][RADIX];
   __shared__ u32 s_hb[4][RADIX];  // raw granule bytes 1..3 (with tile_hist), bits 22..29 (with tile_hist2)
@@ -111,6 +114,7 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
   u32* th = s_th[warp];
   u32* th2 = s_th2[warp];
   const u32 seg = tile_hist ? (u32)FUSED_TILE : rw;  // records between histogram flushes
+  u32 wacc = 0;  // write bits of row (32 * group + lane) (wout)
   for (u32 t0 = start; t0 < end; t0 += seg) {
   const u32 tend = min(end, t0 + seg);
   if (tile_hist) {
@@ -190,6 +194,17 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
         }
       }
       if (gout && r0 + u * 32 + lane < tend) __stcs(gout + r0 + u * 32 + lane, (u32)(addr >> log2G));
+    }
+    if (wout) {  // one bit per record: it writes.  Rows of 32 records are 32-aligned (warp ranges are whole
+                 // tiles of 6 x 32 rows); lane j collects row j of each group of 32 rows, written as one 128-B line
+#pragma unroll
+      for (int u = 0; u < U; u++) {
+        const unsigned wm = __ballot_sync(~0u, ok[u] && (b[u].w >> 24) != RW_READ);
+        if (((((r0 + u * 32) >> 5) & 31u) == (u32)lane) && r0 + u * 32 < tend) wacc = wm;
+      }
+      const u32 lastR = (min(r0 + 32 * U, tend) - 1) >> 5, g0 = lastR & ~31u;
+      if ((lastR & 31u) == 31u || r0 + 32 * U >= tend)
+        if (g0 + lane <= lastR) wout[g0 + lane] = wacc;
     }
   }
   if (tile_hist) {
@@ -277,7 +292,7 @@ static int ring_grid(const void* kern, int threads, size_t smem) {
 }
 
 void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, u32* tile_hist, const Region* regs, u32 nreg,
-                    u32 nreg_shared, int grid, cudaStream_t st, u32* gout, u32* tile_hist2) {
+                    u32 nreg_shared, int grid, cudaStream_t st, u32* gout, u32* tile_hist2, u32* wout) {
   // extents2: contiguous warp ranges, one full wave of resident warps (the round-1 grid-stride kernel took
   // 7.7 ms on C5: 132 instructions per record, 64-bit index math and local-memory accumulators; this one 4.6 ms)
   const int sms = dev_sm_count(), per = blocks_per_sm((const void*)extents2_kernel<4>, 256, 0);
@@ -289,7 +304,7 @@ void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, u32* tile_
   const u64 nw = (n + rw - 1) / rw;
   extents2_kernel<4><<<(unsigned)((nw + 7) / 8), 256, nreg * sizeof(Region), st>>>(
       rec, (u32)n, log2G, (u32)rw, d_sum, tile_hist, regs, make_uint3(nreg_shared, 0u, nreg), gout,
-      tile_hist ? tile_hist2 : nullptr);
+      tile_hist ? tile_hist2 : nullptr, tile_hist ? wout : nullptr);
   (void)grid;
 }
 

@@ -105,6 +105,8 @@ struct FusedArgs {
   const u32* toff;  // [T][RADIX] output offset of each tile's digit run
   u64* kout;
   u32* hist;        // [npass][RADIX] global digit histograms (rows 1.. are accumulated here)
+  const u32* wbits; // with wbit: bit (i & 31) of wbits[i >> 5] = record i writes (extents pass)
+  u32 wbit;         // 1: key = key_hi << pos_bits | pos << 1 | w (pos_bits here includes the bit)
 };
 
 // Persistent CTAs, software-pipelined in registers: right after a tile's digit counts (when its addresses have
@@ -133,12 +135,14 @@ __global__ void __launch_bounds__(FUSED_THREADS, UNST ? FUSED_UMINB : FUSED_MINB
   // (0) granule indices of a tile's records (low 32 bits: 4 bytes per record, coalesced), from the extents pass;
   //     on this path the span is < 2^32, so key_hi = g - gmin = (low32(g) - low32(gmin)) mod 2^32
   u32 a[ITEMS];
+  u32 wq = 0;  // with wbit: lane i < ITEMS holds the write bits of the warp's row i (32 records)
   auto issue = [&](u32 t) {
     const u32 wb = t * TILE + warp * 32 * ITEMS + lane;
     const u32* gp = A.gran + wb;
 #pragma unroll
     for (int i = 0; i < ITEMS; i++)
       if (wb + i * 32 < A.n) a[i] = __ldcs(gp + i * 32);
+    if (!UNST && A.wbit && lane < ITEMS && wb - lane + lane * 32 < A.n) wq = __ldcs(A.wbits + ((wb - lane) >> 5) + lane);
   };
   u32 tile = blockIdx.x;
   if (tile < T) issue(tile);
@@ -151,6 +155,13 @@ __global__ void __launch_bounds__(FUSED_THREADS, UNST ? FUSED_UMINB : FUSED_MINB
     u32 kh[ITEMS];
 #pragma unroll
     for (int i = 0; i < ITEMS; i++) kh[i] = i < nv ? a[i] - (u32)A.gmin : 0u;
+    const u32 wcur = wq;  // (the prefetch below overwrites wq)
+    // the low part of item i's key: its position (and, with wbit, its write bit below it)
+    auto low = [&](int i) -> u64 {
+      const u64 pos = (u64)(wbase + i * 32);
+      if (UNST || !A.wbit) return pos;
+      return (pos << 1) | (u64)((__shfl_sync(~0u, wcur, i) >> lane) & 1u);
+    };
     auto digit = [&](int i) -> u32 { return i < nv ? ((kh[i] >> A.dsh) & (RADIX - 1)) : (u32)RADIX; };
     for (u32 i = tid; i < WARPS * RADIX; i += THREADS) whist[i] = 0;
     __syncthreads();
@@ -191,7 +202,7 @@ __global__ void __launch_bounds__(FUSED_THREADS, UNST ? FUSED_UMINB : FUSED_MINB
       for (int i = 0; i < ITEMS; i++) {
         const u32 d = digit(i);
         if (d < RADIX)
-          keys_s[wh[d] + ((rk[i / 2] >> (16 * (i & 1))) & 0xFFFFu)] = ((u64)kh[i] << A.pos_bits) | (u64)(wbase + i * 32);
+          keys_s[wh[d] + ((rk[i / 2] >> (16 * (i & 1))) & 0xFFFFu)] = ((u64)kh[i] << A.pos_bits) | low(i);
       }
     } else {
     // (3) stable warp ranking (peer masks by shared-memory atomicOr), each key stored into its tile slot
@@ -200,6 +211,7 @@ __global__ void __launch_bounds__(FUSED_THREADS, UNST ? FUSED_UMINB : FUSED_MINB
       // every 4th item's peer set by ballots (ALU pipe) instead of shared-memory masks (LSU pipe, the binding one)
       const bool bal = (i & 3) == 0;
       const u32 d = digit(i);
+      const u64 lo = low(i);  // (warp-wide shuffle: before any lane diverges)
       if (!bal) {
         atomicOr(&wm[d], 1u << lane);
         __syncwarp();
@@ -207,7 +219,7 @@ __global__ void __launch_bounds__(FUSED_THREADS, UNST ? FUSED_UMINB : FUSED_MINB
       const unsigned peers = bal ? peers_of<RADIX_BITS + 1>(d) : wm[d];
       const u32 c = d < RADIX ? wh[d] : 0u;  // (invalid items: digit RADIX, no counter)
       __syncwarp();
-      if (d < RADIX) keys_s[c + __popc(peers & lt)] = ((u64)kh[i] << A.pos_bits) | (u64)(wbase + i * 32);
+      if (d < RADIX) keys_s[c + __popc(peers & lt)] = ((u64)kh[i] << A.pos_bits) | lo;
       if (lane == 31 - __clz(peers)) {
         if (!bal) wm[d] = 0;
         if (d < RADIX) wh[d] = c + __popc(peers);
@@ -258,7 +270,7 @@ void launch_tile_offsets(u64 n, const KeyLayout& L, const u32* tile_hist, void* 
 
 // temp: holds the tile offsets (launch_tile_offsets); hist: [npass][RADIX] zeroed (rows >= 1 filled)
 void launch_fused_extract_pass0(const u32* gran, u64 n, const KeyLayout& L, u32 npass, void* temp, u64* kout,
-                                u32* hist, cudaStream_t st, u32 dsh, bool unstable) {
+                                u32* hist, cudaStream_t st, u32 dsh, bool unstable, const u32* wbits) {
   if (!n) return;
   const u32 T = (u32)((n + FUSED_TILE - 1) / FUSED_TILE);
   u32* O = reinterpret_cast<u32*>(temp);
@@ -274,7 +286,9 @@ void launch_fused_extract_pass0(const u32* gran, u64 n, const KeyLayout& L, u32 
   A.gran = gran;
   A.n = (u32)n;
   A.log2G = L.log2G;
-  A.pos_bits = L.pos_bits;
+  A.wbit = unstable ? 0u : L.wbit;
+  A.wbits = wbits;
+  A.pos_bits = L.pos_bits + A.wbit;
   A.npass = npass;
   A.dsh = dsh;
   A.gmin = L.gminG;

@@ -29,8 +29,10 @@ constexpr int CT_TILE = CT_THREADS * CT_ITEMS;
 // regs (optional, device, nreg <= MAX_REGIONS): sorted by (space, base), the first nreg_shared are SHARED
 // gout (optional, n x u32): low 32 bits of the granule index addr >> log2G of every record (fused-pass input)
 // tile_hist2 (optional, needs tile_hist): per-tile histograms of (addr >> log2G >> HYB_LO) & 255 (k_bucket.cu)
+// wout (optional, needs tile_hist, ceil(n / 32) x u32): bit i & 31 of wout[i >> 5] = record i writes (KeyLayout::wbit)
 void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, u32* tile_hist, const Region* regs, u32 nreg,
-                    u32 nreg_shared, int grid, cudaStream_t st, u32* gout = nullptr, u32* tile_hist2 = nullptr);
+                    u32 nreg_shared, int grid, cudaStream_t st, u32* gout = nullptr, u32* tile_hist2 = nullptr,
+                    u32* wout = nullptr);
 void launch_extract_1to1(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, u64* keys, u32* hist, u64 pos_base,
                          int grid, cudaStream_t st);
 void launch_entry_count(const Rec* rec, u64 n, u32 log2G, u32* cnt, cudaStream_t st);
@@ -50,7 +52,8 @@ void launch_tile_offsets(u64 n, const KeyLayout& L, const u32* tile_hist, void* 
 // gran: the extents pass's granule indices (gout); rec is not read
 // unstable: no stable order within a digit (the bucket path); npass must be 1
 void launch_fused_extract_pass0(const u32* gran, u64 n, const KeyLayout& L, u32 npass, void* temp, u64* kout,
-                                u32* hist, cudaStream_t st, u32 dsh = 0, bool unstable = false);
+                                u32* hist, cudaStream_t st, u32 dsh = 0, bool unstable = false,
+                                const u32* wbits = nullptr);  // wbits: extents' wout, needed when L.wbit
 
 constexpr uint64_t BUCKET_MIN_N = 1ull << 24;  // traces of fewer records keep the full sort
 // k_bucket.cu — bucket path of the sort + compaction (keys sorted by key_hi >> HYB_LO only)
@@ -197,8 +200,12 @@ void launch_warp_emit(const ConflictArgs& a, const u32* head, const u32* hscan, 
 size_t compact_temp_bytes(u64 m);
 // keys: sorted (m); seg: free buffer of m keys; out: where the result goes (may alias keys, which is dead after);
 // returns out
+// filter (needs L.wbit): also drop read-only locations (compact_seg_w_kernel); with L.wbit the output is always
+// the plain layout (the bit stripped)
 u64* launch_compact_multi(const u64* keys, u32 m, const KeyLayout& L, u64* seg, u64* out, void* temp, u32* total,
-                          cudaStream_t st);
+                          cudaStream_t st, bool filter = false);
+// sample whether the write-bit filter pays on these sorted keys (one sync); temp: >= 16 bytes of device memory
+bool compact_filter_pays(const u64* keys, u32 m, const KeyLayout& L, void* temp, cudaStream_t st);
 
 // k_expand.cu — cells (block, interval slot, thread); descriptors of slot q are idx[ivoff[q] .. ivoff[q+1])
 void launch_flow_count2(const void* flows, const u32* ivoff, const u32* idx, u32 niv, u32 bmin, u64 ncell, u32 tmax,

@@ -230,6 +230,8 @@ bool sesa_trace::step_extents(const Rec* rec, u64 n, bool tile_hist, u32* gran_o
   if (have_thist2 && !grow(b_thist2, ((n + FUSED_TILE - 1) / FUSED_TILE) * RADIX * 4, "tile histograms")) return false;
   // granule indices for the fused pass go to the key buffer the first sort pass after it writes (b_keys[0])
   if (have_thist && !grow(b_keys[0], n * 8 + 64, "keys")) return false;
+  // and the per-record write bits the fused pass puts into the keys (KeyLayout::wbit)
+  if (have_thist && !grow(b_wbits, (n + 31) / 32 * 4, "write bits")) return false;
   Summary init;
   memset(&init, 0, sizeof init);
   init.bad_index = ~0ull;
@@ -246,7 +248,8 @@ bool sesa_trace::step_extents(const Rec* rec, u64 n, bool tile_hist, u32* gran_o
   LAUNCH("extents", (gout ? 36.0 : 32.0) * n, launch_extents(rec, n, log2G, (Summary*)b_summary.p,
                                              have_thist ? (u32*)b_thist.p : nullptr, (const Region*)b_regions.p,
                                              n_regions, n_regions_shared, grid_stream, stream, gout,
-                                             have_thist2 ? (u32*)b_thist2.p : nullptr));
+                                             have_thist2 ? (u32*)b_thist2.p : nullptr,
+                                             have_thist ? (u32*)b_wbits.p : nullptr));
   if (!cuda_ok(cudaMemcpyAsync(&h_summary, b_summary.p, sizeof(Summary), cudaMemcpyDeviceToHost, stream), "summary"))
     return false;
   return sync_check("extents");
@@ -317,7 +320,7 @@ bool sesa_trace::step_extract_fused(const Rec* rec, u64 n) {
          launch_tile_offsets(n, L, (const u32*)b_thist.p, b_ftmp.p, stream));
   LAUNCH("extract_pass0", 12.0 * n,
          launch_fused_extract_pass0((const u32*)b_keys[0].p, n, L, hist_from_extents ? 1u : npass, b_ftmp.p,
-                                    (u64*)b_keys[1].p, (u32*)b_hist.p, stream));
+                                    (u64*)b_keys[1].p, (u32*)b_hist.p, stream, 0, false, (const u32*)b_wbits.p));
   return true;
 }
 
@@ -535,7 +538,7 @@ bool sesa_trace::step_sort(u64 m, int* cur_out, u32 first_pass, int cur0) {
     }
     LAUNCH("onesweep_pass", 16.0 * m,
            launch_onesweep((u64*)b_keys[cur].p, (u64*)b_keys[cur ^ 1].p, nullptr, nullptr, (u32)m,
-                           L.pos_bits + p * RADIX_BITS, (u64*)b_binbase.p + (size_t)p * RADIX, (u64*)b_lookback.p,
+                           L.pos_bits + L.wbit + p * RADIX_BITS, (u64*)b_binbase.p + (size_t)p * RADIX, (u64*)b_lookback.p,
                            (u32*)b_ctr.p + passes_run, epoch, stream));
     cur ^= 1;
     passes_run++;
@@ -552,9 +555,14 @@ bool sesa_trace::step_compact(int cur, u64 m, u64** comp, u32* m2) {
   *m2 = 0;
   if (m == 0) return true;
   if (!grow(b_ctmp, compact_temp_bytes(m), "compact temp") || !grow(b_ctotal, 16, "compact count")) return false;
+  // with the write bit: drop read-only locations too, if a sample of the sorted keys says it pays
+  bool filter = false;
+  if (layout.wbit) LAUNCH("compact_sample", 8.0 * 32 * 16384,
+                          filter = compact_filter_pays((const u64*)b_keys[cur].p, (u32)m, layout, b_ctotal.p, stream));
+  info.wbit_filter = filter ? 1 : 0;
   LAUNCH("compact", 8.0 * m, *comp = launch_compact_multi((const u64*)b_keys[cur].p, (u32)m, layout,
                                                           (u64*)b_keys[cur ^ 1].p, (u64*)b_keys[cur].p, b_ctmp.p,
-                                                          (u32*)b_ctotal.p, stream));
+                                                          (u32*)b_ctotal.p, stream, filter));
   if (!cuda_ok(cudaMemcpyAsync(m2, b_ctotal.p, 4, cudaMemcpyDeviceToHost, stream), "compact count")) return false;
   if (!sync_check("compact")) return false;
   info.n_multi = *m2;
@@ -970,6 +978,10 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
   }
   int cur = 0;
   if (fused) {
+    // the write bit below the position (KeyLayout::wbit): compaction drops read-only locations
+#ifndef SESA_NO_WBIT
+    layout.wbit = layout.sort_bits + layout.pos_bits + 1 <= 64 ? 1u : 0u;
+#endif
     if (!step_extract_fused(rec, n) || !step_sort(m, &cur, 1, 1)) return status;
   } else {
     if (!step_extract(rec, n, m, 0, S.multi != 0)) return status;

@@ -43,6 +43,7 @@ struct sesa_trace {
   DevBuf b_tflags, b_part, b_carry, b_owner, b_slots, b_cross, b_ccount, b_carrytmp, b_tstart, b_work;
   DevBuf b_races, b_rkeys[2], b_rvals[2], b_races_sorted, b_rhist, b_rbase;
   DevBuf b_eoff, b_ecnt, b_ecell, b_hrec, b_dist_races, b_ctmp, b_ctotal, b_thist, b_ftmp, b_thist2, b_btmp2;
+  DevBuf b_wbits;   // per-record write bits from the extents pass (KeyLayout::wbit)
   DevBuf b_lraces;  // multi-launch checks: the races of the launches checked so far
   DevBuf b_franges, b_fkeep, b_fcnt2, b_foff2, b_frec, b_forig;  // descriptor-level check (NEXT-2)
   sesa_flow_check_info flow_info{};

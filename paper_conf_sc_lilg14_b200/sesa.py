@@ -62,7 +62,8 @@ class sesa_check_info(ctypes.Structure):
                 ("n_multi", ctypes.c_uint64), ("sort_bits", ctypes.c_uint32), ("pos_bits", ctypes.c_uint32), ("digit_bits", ctypes.c_uint32),
                 ("sort_passes", ctypes.c_uint32), ("sorted_input", ctypes.c_uint32), ("launches", ctypes.c_uint32),
                 ("crossing_tiles", ctypes.c_uint32), ("n_stats", ctypes.c_uint32),
-                ("fused_first_pass", ctypes.c_uint32), ("bucket_path", ctypes.c_uint32)]
+                ("fused_first_pass", ctypes.c_uint32), ("bucket_path", ctypes.c_uint32),
+                ("wbit_filter", ctypes.c_uint32)]
 
 
 # every symbol include/sesa.h declares (tests assert the library exports all of them)
