@@ -49,6 +49,10 @@ struct SpaceAcc2 {
   u32 cnt, bmin, bmax, imin, imax;
   u64 amin, amax;
   __device__ __forceinline__ void init() { cnt = 0, amin = ~0ull, amax = 0, bmin = ~0u, bmax = 0, imin = ~0u, imax = 0; }
+  __device__ __forceinline__ void add_a(u64 a, u64 last) {  // address extents only
+    cnt++;
+    amin = min(amin, a), amax = max(amax, last);
+  }
   __device__ __forceinline__ void add(u64 a, u64 last, u32 b, u32 i) {
     cnt++;
     amin = min(amin, a), amax = max(amax, last);
@@ -70,6 +74,63 @@ struct SpaceAcc2 {
 // tile, the histogram of the raw low granule byte (addr >> log2G) & 255: once the extents fix gmin, these are the
 // tile histograms of the first sort digit ((g - gmin) & 255 is a rotation of g & 255), which lets the fused
 // extract + first sort pass place every tile without a look-back (k_fused.cu).
+// block reduction of one CTA's extents (warp shuffles, then one atomic per field per CTA) into the Summary
+template <int THREADS>
+__device__ __forceinline__ void flush_summary(u64 bad64, u64 ent, u64 mul, u32 unsorted, const SpaceAcc2& A0,
+                                              const SpaceAcc2& A1, u32 log2G, Summary* __restrict__ out) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  SpaceAcc S0 = A0.to_acc(log2G), S1 = A1.to_acc(log2G);
+  __shared__ SpaceAcc sa[THREADS / 32][2];
+  __shared__ u64 s64[THREADS / 32][3];
+  __shared__ u32 s_uns[THREADS / 32];
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    bad64 = min(bad64, __shfl_xor_sync(~0u, bad64, o));
+    ent += __shfl_xor_sync(~0u, ent, o);
+    mul += __shfl_xor_sync(~0u, mul, o);
+    unsorted |= __shfl_xor_sync(~0u, unsorted, o);
+  }
+  S0.warp_reduce();
+  S1.warp_reduce();
+  if (lane == 0) {
+    s64[warp][0] = bad64, s64[warp][1] = ent, s64[warp][2] = mul;
+    sa[warp][0] = S0, sa[warp][1] = S1;
+    s_uns[warp] = unsorted;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    for (int w = 1; w < THREADS / 32; w++) {
+      s64[0][0] = min(s64[0][0], s64[w][0]);
+      s64[0][1] += s64[w][1];
+      s64[0][2] += s64[w][2];
+      s_uns[0] |= s_uns[w];
+      for (int x = 0; x < 2; x++) {
+        SpaceAcc& d = sa[0][x];
+        const SpaceAcc& e = sa[w][x];
+        d.cnt += e.cnt;
+        d.gmin = min(d.gmin, e.gmin), d.gmax = max(d.gmax, e.gmax);
+        d.bmin = min(d.bmin, e.bmin), d.bmax = max(d.bmax, e.bmax);
+        d.imin = min(d.imin, e.imin), d.imax = max(d.imax, e.imax);
+      }
+    }
+    if (s64[0][0] != ~0ull) atomicMin(&out->bad_index, (unsigned long long)s64[0][0]);
+    if (s64[0][1]) atomicAdd(&out->entries, (unsigned long long)s64[0][1]);
+    if (s64[0][2]) atomicAdd(&out->multi, (unsigned long long)s64[0][2]);
+    for (int x = 0; x < 2; x++) {
+      const SpaceAcc& d = sa[0][x];
+      if (!d.cnt) continue;
+      atomicAdd(&out->count[x], (unsigned long long)d.cnt);
+      atomicMin(&out->gmin[x], (unsigned long long)d.gmin);
+      atomicMax(&out->gmax[x], (unsigned long long)d.gmax);
+      atomicMin(&out->bmin[x], d.bmin);
+      atomicMax(&out->bmax[x], d.bmax);
+      atomicMin(&out->imin[x], d.imin);
+      atomicMax(&out->imax[x], d.imax);
+    }
+    if (s_uns[0]) atomicOr(&out->unsorted, 1u);
+  }
+}
+
 template <int U>
 // With regions (nreg > 0; sorted by (space, base), non-overlapping, space s in [rs[s], rs[s+1])), every valid
 // record of a space with regions is also checked for containment (OOB, NEXT-1): binary search for the last
@@ -235,56 +296,257 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
       if (v) atomicAdd(&(&out->bhist[0][0])[i], v);
     }
   }
-  SpaceAcc S0 = A0.to_acc(log2G), S1 = A1.to_acc(log2G);
-  __shared__ SpaceAcc sa[THREADS / 32][2];
-  __shared__ u64 s64[THREADS / 32][3];
-  __shared__ u32 s_uns[THREADS / 32];
+  flush_summary<THREADS>(bad64, ent, mul, unsorted, A0, A1, log2G, out);
+}
+
+// ------------------------------------------------------------------------------------------------------------
+// Extents fused with the bucket path's first partition (k_bucket.cu; C5-like traces, chosen by a sample of the
+// records before any pass).  The bucket path's first digit is key_hi bits [HYB_LO, HYB_LO + 8) with gmin aligned
+// down to 2^(HYB_LO + 16), i.e. the RAW granule bits [14, 22): known while the records stream by, before gmin
+// is.  So one pass validates, reduces the extents and writes every record's key into the region of its digit —
+// keys carry the raw low 30 granule bits (key_hi = g - G0 follows modulo 2^30 once G0 is known; the second
+// partition pass rebases them) — instead of an extents pass writing a 4-byte granule array that a fused pass
+// reads back (C5: 36 + 12 GB -> 40 GB of traffic).  Order inside a region does not matter on the bucket path
+// (each chunk's survivors are sorted by full key), so a CTA takes slots of region d in windows of XP_WIN
+// reserved by one global atomic, and a tile's keys, grouped by digit in shared memory, leave in coalesced runs.
+// Window remainders are filled with ~0 sentinels, which the second pass skips.  A region that would pass its
+// capacity sets *overflow (the host then runs the ordinary path: the result never depends on this pass's
+// speculation).  Per tile of XP_TILE records: (1) load the next tile's records into registers (in flight during
+// the rest), (2) validate + extents + count atomics (rank = return value), (3) digit bases + windows (thread d),
+// (4) keys into shared memory by digit, (5) coalesced write-out.
+// ------------------------------------------------------------------------------------------------------------
+#ifndef XP_THREADS_
+#define XP_THREADS_ 512
+#endif
+#ifndef XP_ROWS_
+#define XP_ROWS_ 4
+#endif
+#ifndef XP_STAGES_
+#define XP_STAGES_ 3
+#endif
+constexpr int XP_THREADS = XP_THREADS_, XP_ROWS = XP_ROWS_, XP_TILE = XP_THREADS * XP_ROWS, XP_STAGES = XP_STAGES_;
+#ifndef XP_WIN_
+#define XP_WIN_ 256
+#endif
+constexpr u32 XP_WIN = XP_WIN_;
+constexpr size_t XP_SMEM = (size_t)XP_STAGES * XP_TILE * 32;  // the record ring (dynamic shared memory)
+
+// The tiles' records arrive by TMA bulk copies into a ring of XP_STAGES tiles (192 KB in flight per SM without
+// registers: one CTA of 512 threads per SM would otherwise hold one tile in flight and stall on every barrier).
+__global__ void __launch_bounds__(XP_THREADS, 1) extents_part_kernel(XPArgs A) {
+  constexpr int THREADS = XP_THREADS, U = XP_ROWS;
+  extern __shared__ __align__(128) unsigned char xp_ring[];
+  __shared__ u64 bars[XP_STAGES];
+  __shared__ u64 stage[XP_TILE];
+  __shared__ u32 s_cnt[RADIX], s_base[RADIX], s_hb[RADIX];
+  __shared__ uint4 s_wo[RADIX];  // per digit: {d1, split, d2, -} (write-out deltas)
+  __shared__ u32 s_tot;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  for (int i = tid; i < RADIX; i += THREADS) s_cnt[i] = 0, s_hb[i] = 0;
+  u32 wpos = 0, wend = 0;  // thread d < RADIX: its CTA's current window of region d
+  u32 nstart = 0;          // and the next one, reserved ahead
+  bool nvalid = false;
+  const u32 n = A.n, log2G = A.log2G, gmask = (1u << log2G) - 1u;
+  const uint4* q = reinterpret_cast<const uint4*>(A.rec);
+  u32 bad = ~0u, extra = 0, multi = 0, unsorted = 0;
+  SpaceAcc2 A0, A1;
+  A0.init();
+  A1.init();
+  BulkRing<XP_STAGES> ring(xp_ring, bars, XP_TILE * 32);
+  ring.start(A.rec, (u64)n * 32);  // (contains __syncthreads)
+  for (u64 j = 0; ring.next(j); j++) {
+    const u32 tile = (u32)ring.chunk_index(j);
+    const u32 tb = tile * XP_TILE, r0 = tb + warp * 32 * U;
+    // the (block, interval) before the warp's first row: in the ring, or (warp 0) the previous tile's last record
+    uint4 pv = make_uint4(0, 0, 0, 0);
+    if (warp == 0 && tb > 0) pv = __ldg(q + 2 * (u64)(tb - 1) + 1);
+    const uint4* R = reinterpret_cast<const uint4*>(ring.wait(j));
+    if (warp > 0) pv = R[2 * (warp * 32 * U - 1) + 1];
+    u64 prev_bi = ((u64)pv.x << 32) | pv.z;
+    u64 key[U];
+    u32 rk[U];
 #pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    bad64 = min(bad64, __shfl_xor_sync(~0u, bad64, o));
-    ent += __shfl_xor_sync(~0u, ent, o);
-    mul += __shfl_xor_sync(~0u, mul, o);
-    unsorted |= __shfl_xor_sync(~0u, unsorted, o);
-  }
-  S0.warp_reduce();
-  S1.warp_reduce();
-  if (lane == 0) {
-    s64[warp][0] = bad64, s64[warp][1] = ent, s64[warp][2] = mul;
-    sa[warp][0] = S0, sa[warp][1] = S1;
-    s_uns[warp] = unsorted;
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    for (int w = 1; w < THREADS / 32; w++) {
-      s64[0][0] = min(s64[0][0], s64[w][0]);
-      s64[0][1] += s64[w][1];
-      s64[0][2] += s64[w][2];
-      s_uns[0] |= s_uns[w];
-      for (int x = 0; x < 2; x++) {
-        SpaceAcc& d = sa[0][x];
-        const SpaceAcc& e = sa[w][x];
-        d.cnt += e.cnt;
-        d.gmin = min(d.gmin, e.gmin), d.gmax = max(d.gmax, e.gmax);
-        d.bmin = min(d.bmin, e.bmin), d.bmax = max(d.bmax, e.bmax);
-        d.imin = min(d.imin, e.imin), d.imax = max(d.imax, e.imax);
+    for (int u = 0; u < U; u++) {
+      const u32 i = r0 + u * 32 + lane, li = warp * 32 * U + u * 32 + lane;
+      const bool in = i < n;
+      const uint4 ca = in ? R[2 * li] : make_uint4(0, 0, 0, 0), cb = in ? R[2 * li + 1] : make_uint4(0, 0, 0, 0);
+      const u64 bi = ((u64)cb.x << 32) | cb.z;
+      const u64 up = __shfl_up_sync(~0u, bi, 1);
+      const u64 pbi = lane ? up : prev_bi;
+      prev_bi = __shfl_sync(~0u, bi, 31);
+      const u32 size = cb.w & 0xFFFFu, sp = (cb.w >> 16) & 0xFFu, rwv = cb.w >> 24;
+      const u64 addr = ((u64)ca.y << 32) | ca.x;
+      const bool ok = in && sp <= 1u && rwv <= 2u && size >= 1u && addr + (u64)size - 1ull >= addr;
+      bad = (in && !ok) ? min(bad, i) : bad;
+      const u32 e = ((ca.x & gmask) + size - 1u) >> log2G;
+      extra += ok ? e : 0u;
+      multi += (ok && e != 0u) ? 1u : 0u;
+      unsorted |= (ok && i > 0 && bi < pbi) ? 1u : 0u;
+      const u64 last = addr + (u64)size - 1ull;
+      // (block / interval extents are not kept: the fused path needs them only for unsorted or shared traces,
+      // which go back to the ordinary path)
+      if (ok) {
+        if (sp == SP_GLOBAL) A1.add_a(addr, last);
+        else A0.cnt++;
+      }
+      const u64 g = addr >> log2G;
+      key[u] = ((g & ((1ull << 30) - 1ull)) << A.pos_bits) | (u64)i;
+      rk[u] = ~0u;
+      if (ok) {
+        atomicAdd(&s_hb[(u32)(g >> (HYB_LO + RADIX_BITS)) & (RADIX - 1)], 1u);
+        rk[u] = atomicAdd(&s_cnt[(u32)(g >> HYB_LO) & (RADIX - 1)], 1u);
       }
     }
-    if (s64[0][0] != ~0ull) atomicMin(&out->bad_index, (unsigned long long)s64[0][0]);
-    if (s64[0][1]) atomicAdd(&out->entries, (unsigned long long)s64[0][1]);
-    if (s64[0][2]) atomicAdd(&out->multi, (unsigned long long)s64[0][2]);
-    for (int x = 0; x < 2; x++) {
-      const SpaceAcc& d = sa[0][x];
-      if (!d.cnt) continue;
-      atomicAdd(&out->count[x], (unsigned long long)d.cnt);
-      atomicMin(&out->gmin[x], (unsigned long long)d.gmin);
-      atomicMax(&out->gmax[x], (unsigned long long)d.gmax);
-      atomicMin(&out->bmin[x], d.bmin);
-      atomicMax(&out->bmax[x], d.bmax);
-      atomicMin(&out->imin[x], d.imin);
-      atomicMax(&out->imax[x], d.imax);
+    ring.release(j);  // (contains __syncthreads: the slot is refilled with tile j + XP_STAGES)
+    // Thread d < RADIX (warps 0-7): the digit's stage base — the counts of the warps before it by one warp
+    // reduction each (redux), its own warp by a shuffle scan: no block scan, one barrier less — and this tile's
+    // slots in the CTA's windows.  The next window is reserved ahead (its atomic's result is first needed a tile
+    // or more later, so its latency is off the critical path); a run longer than a window reserves at once.
+    if (tid < RADIX) {
+      u32 before = 0;
+#pragma unroll
+      for (int w2 = 0; w2 < RADIX / 32 - 1; w2++)  // (independent loads and reductions: no dependent chain)
+        before += __reduce_add_sync(~0u, w2 < warp ? s_cnt[w2 * 32 + lane] : 0u);
+      const u32 c = s_cnt[tid];
+      u32 x = c;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const u32 y = __shfl_up_sync(~0u, x, o);
+        if (lane >= o) x += y;
+      }
+      const u32 base = before + x - c;
+      s_base[tid] = base;
+      if (tid == RADIX - 1) s_tot = before + x;
+      const u32 avail = wend - wpos, seg1 = min(c, avail);
+      // stage slot jj of this digit -> window slot jj + d1 (jj < split) or jj + d2 (modular u32 deltas)
+      uint4 wo = make_uint4(wpos - base, base + seg1, 0u, 0u);
+      wpos += seg1;
+      if (c > seg1) {
+        const u32 rest = c - seg1;
+        u32 st, res;
+        if (nvalid && rest <= XP_WIN) {
+          st = nstart, res = XP_WIN, nvalid = false;
+        } else {
+          res = max(XP_WIN, (rest + 31u) & ~31u);
+          st = atomicAdd(&A.gfill[tid], res);
+        }
+        if ((u64)st + res > A.cap) atomicOr(A.overflow, 1u);
+        wo.z = st - (base + seg1);
+        wpos = st + rest;
+        wend = st + res;
+      }
+      s_wo[tid] = wo;
+      if (!nvalid && wend - wpos < XP_WIN / 2) nstart = atomicAdd(&A.gfill[tid], XP_WIN), nvalid = true;
     }
-    if (s_uns[0]) atomicOr(&out->unsorted, 1u);
+    __syncthreads();
+    if (tid < RADIX) s_cnt[tid] = 0;  // (every count was read before the barrier)
+#pragma unroll
+    for (int u = 0; u < U; u++)
+      if (rk[u] != ~0u) stage[s_base[(u32)(key[u] >> (A.pos_bits + HYB_LO)) & (RADIX - 1)] + rk[u]] = key[u];
+    __syncthreads();
+    // coalesced runs: stage slot jj of digit d goes to its window slot
+    const u32 tot = s_tot;
+    for (u32 jj = tid; jj < tot; jj += THREADS) {
+      const u64 k = stage[jj];
+      const uint4 wo = s_wo[(u32)(k >> (A.pos_bits + HYB_LO)) & (RADIX - 1)];
+      const u32 dst = jj + (jj < wo.y ? wo.x : wo.z), d = (u32)(k >> (A.pos_bits + HYB_LO)) & (RADIX - 1);
+      // (plain stores: a run's partial edge sectors wait in L2 for the CTA's next run of the digit; streaming
+      // stores evicted them half-written)
+      if (dst < A.cap) A.kout[(u64)d * A.cap + dst] = k;
+    }
+    // (the next tile's first barrier, in ring.release, orders these reads of the tables before they change)
   }
+  // window remainders (and a reserved next window) -> sentinels
+  if (tid < RADIX) {
+    for (u32 jj = wpos; jj < wend && jj < A.cap; jj++) A.kout[(u64)tid * A.cap + jj] = ~0ull;
+    if (nvalid) {
+      if ((u64)nstart + XP_WIN > A.cap) atomicOr(A.overflow, 1u);
+      for (u32 jj = nstart; jj < nstart + XP_WIN && jj < A.cap; jj++) A.kout[(u64)tid * A.cap + jj] = ~0ull;
+    }
+  }
+  __syncthreads();
+  for (int i = tid; i < RADIX; i += THREADS)
+    if (s_hb[i]) atomicAdd(&A.out->bhist[3][i], s_hb[i]);
+  const u64 bad64 = bad == ~0u ? ~0ull : (u64)bad, ent = (u64)extra + A0.cnt + A1.cnt;
+  flush_summary<THREADS>(bad64, ent, (u64)multi, unsorted, A0, A1, log2G, A.out);
+}
+
+void launch_extents_part(const XPArgs& A, cudaStream_t st) {
+  const u32 T = (A.n + XP_TILE - 1) / XP_TILE;
+  const u32 grid = std::min<u32>(T, (u32)dev_sm_count());
+  smem_optin((const void*)extents_part_kernel, XP_SMEM);
+  extents_part_kernel<<<grid, XP_THREADS, XP_SMEM, st>>>(A);
+}
+
+u64 extents_part_cap(u64 n) {
+  // per region: the mean, 1/8 more, a window per CTA and a tile of slack, in whole 32-key rows
+  const u64 mean = (n + RADIX - 1) / RADIX;
+  return ((mean + mean / 8 + (u64)XP_WIN * (u64)dev_sm_count() + XP_TILE) + 31) & ~31ull;
+}
+
+// ---- record sample predicting the fused path (before any pass) -----------------------------------------------
+// every stride-th record: flags bit 0 = a sampled record is invalid, shared, spans two granules or sits below
+// its predecessor in (block, interval) order; min / max granule; histogram of the absolute chunk index g >> 15
+// modulo 2^15 (G0 is a multiple of 2^15, so these are the bucket path's chunks; folding can only raise the max)
+__global__ void presample_kernel(const Rec* __restrict__ rec, u32 n, u32 stride, u32 log2G, u32* __restrict__ hist,
+                                 unsigned long long* __restrict__ ext /* [0] flags, [1] gmin, [2] gmax */) {
+  const u64 step = (u64)gridDim.x * blockDim.x * stride;
+  u64 gmn = ~0ull, gmx = 0;
+  u32 flags = 0;
+  for (u64 i0 = (u64)(blockIdx.x * blockDim.x + (threadIdx.x & ~31u)) * stride; i0 < n; i0 += step) {
+    const u64 i = i0 + (u64)(threadIdx.x & 31) * stride;
+    u32 c = ~0u;
+    if (i < n) {
+      const Rec r = load_rec(rec + i);
+      const u64 g = r.addr >> log2G, gl = (r.addr + (u64)r.size - 1ull) >> log2G;
+      const bool ok = r.space == SP_GLOBAL && r.rw <= 2 && r.size >= 1 && r.addr + (u64)r.size - 1ull >= r.addr && g == gl;
+      if (!ok) flags |= 1u;
+      if (i > 0) {
+        const Rec p = load_rec(rec + i - 1);
+        if (((u64)r.block << 32 | r.interval) < ((u64)p.block << 32 | p.interval)) flags |= 1u;
+      }
+      gmn = min(gmn, g), gmx = max(gmx, g);
+      c = (u32)(g >> HYB_CHUNK) & ((1u << 15) - 1u);
+    }
+    const unsigned peers = __match_any_sync(~0u, c);
+    if (c != ~0u && (threadIdx.x & 31) == __ffs(peers) - 1) atomicAdd(&hist[c], (u32)__popc(peers));
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    flags |= __shfl_xor_sync(~0u, flags, o);
+    gmn = min(gmn, __shfl_xor_sync(~0u, gmn, o));
+    gmx = max(gmx, __shfl_xor_sync(~0u, gmx, o));
+  }
+  if ((threadIdx.x & 31) == 0) {
+    if (flags) atomicOr(&ext[0], (unsigned long long)flags);
+    atomicMin(&ext[1], gmn);
+    atomicMax(&ext[2], gmx);
+  }
+}
+
+__global__ void presample_max_kernel(const u32* __restrict__ hist, unsigned long long* __restrict__ ext) {
+  u32 mx = 0;
+  for (u32 c = blockIdx.x * blockDim.x + threadIdx.x; c < (1u << 15); c += gridDim.x * blockDim.x) mx = max(mx, hist[c]);
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) mx = max(mx, __shfl_xor_sync(~0u, mx, o));
+  if ((threadIdx.x & 31) == 0) atomicMax(&ext[3], (unsigned long long)mx);
+}
+
+// temp: >= presample_temp_bytes(); h_ext (host, valid after a sync): flags, gmin, gmax, max chunk count; *samples
+size_t presample_temp_bytes() { return (1u << 15) * 4 + 64; }
+void launch_presample(const Rec* rec, u32 n, u32 log2G, u32 want, void* temp, unsigned long long* h_ext,
+                      u32* samples, cudaStream_t st) {
+  u32* hist = reinterpret_cast<u32*>(temp);
+  unsigned long long* ext = reinterpret_cast<unsigned long long*>(hist + (1u << 15));
+  const u32 stride = std::max<u32>(1, n / want);
+  *samples = (n + stride - 1) / stride;
+  cudaMemsetAsync(hist, 0, (1u << 15) * 4 + 32, st);
+  const unsigned long long init[4] = {0ull, ~0ull, 0ull, 0ull};
+  cudaMemcpyAsync(ext, init, 32, cudaMemcpyHostToDevice, st);
+  const u32 grid = (u32)std::min<u64>(((u64)*samples + 255) / 256, (u64)dev_sm_count() * 8);
+  presample_kernel<<<grid, 256, 0, st>>>(rec, n, stride, log2G, hist, ext);
+  presample_max_kernel<<<32, 256, 0, st>>>(hist, ext);
+  cudaMemcpyAsync(h_ext, ext, 32, cudaMemcpyDeviceToHost, st);
 }
 
 static int ring_grid(const void* kern, int threads, size_t smem) {

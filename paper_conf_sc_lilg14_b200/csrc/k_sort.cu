@@ -235,12 +235,23 @@ __device__ __forceinline__ u64 gtime() {
 // and runs 3% slower (4.94 vs 4.80 ms per 1e9 keys, measured).
 __device__ unsigned long long* g_prof = nullptr;
 
+// UNST == 3 (the second partition pass after the fused extents + first partition, k_extract.cu): the input is
+// RADIX regions of cap keys, region r holding fill[r] keys (sentinel-padded); tiles never straddle regions
+// (tile t of region r: tprefix[r] <= t < tprefix[r + 1]), and each key is rebased on load from raw low-30 granule
+// bits to key_hi = (raw - g0) mod 2^30 (sentinels stay ~0)
+struct MapArgs {
+  const u32* tprefix;  // [RADIX + 1]
+  const u32* fill;     // [RADIX]
+  u64 cap;
+  u32 pos_bits, g0;    // rebase: pos_bits of the layout, low 30 bits of G0
+};
+
 template <int THREADS, int ITEMS, int LBW, bool FULL, bool LATE_LB, int S, bool BAL, int TMA, int MIX = 0,
           int UNST = 0>
 __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64* __restrict__ kout, u32 m, u32 shift,
                                                const u64* __restrict__ bin_base, u64* __restrict__ lookback,
                                                u32 epoch, u32 tile, unsigned char* smem, unsigned long long* prof,
-                                               u64* ebar) {
+                                               u64* ebar, const MapArgs& mp) {
   constexpr int WARPS = THREADS / 32;
   constexpr int TILE = THREADS * ITEMS;
   constexpr int IPS = ITEMS / S;  // items per rank stream
@@ -276,6 +287,13 @@ __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64*
 #pragma unroll
     for (int i = 0; i < ITEMS; i++)
       if (FULL || i < nv) k[i] = keys_s[warp * 32 * ITEMS + i * 32 + lane];
+    if (UNST == 3) {
+      const u64 pm = (1ull << mp.pos_bits) - 1ull;
+#pragma unroll
+      for (int i = 0; i < ITEMS; i++)
+        if ((FULL || i < nv) && k[i] != ~0ull)
+          k[i] = ((((k[i] >> mp.pos_bits) - (u64)mp.g0) & ((1ull << 30) - 1ull)) << mp.pos_bits) | (k[i] & pm);
+    }
     __syncthreads();
   } else {
 #pragma unroll
@@ -287,7 +305,7 @@ __device__ __forceinline__ void onesweep2_tile(const u64* __restrict__ kin, u64*
   //  >= RADIX; 2: unstable pass on any digit, no sentinels)
   auto digit = [&](int i) -> u32 {
     if (!(FULL || i < nv)) return (u32)RADIX;
-    if (UNST == 1) { const u32 d9 = (u32)(k[i] >> shift) & (2 * RADIX - 1); return d9 < RADIX ? d9 : (u32)RADIX; }
+    if (UNST == 1 || UNST == 3) { const u32 d9 = (u32)(k[i] >> shift) & (2 * RADIX - 1); return d9 < RADIX ? d9 : (u32)RADIX; }
     return (u32)((k[i] >> shift) & (RADIX - 1));
   };
   // rank streams: items [s*IPS, (s+1)*IPS) of a warp form stream s (stable order = warp, stream, item, lane),
@@ -443,22 +461,42 @@ template <int THREADS, int ITEMS, int MINB, int LBW, bool LATE_LB, int S, bool B
 __global__ void __launch_bounds__(THREADS, MINB) onesweep2_kernel(const u64* __restrict__ kin, u64* __restrict__ kout,
                                                                   u32 m, u32 shift, const u64* __restrict__ bin_base,
                                                                   u64* __restrict__ lookback,
-                                                                  u32* __restrict__ tile_ctr, u32 epoch) {
+                                                                  u32* __restrict__ tile_ctr, u32 epoch,
+                                                                  MapArgs mp) {
   constexpr int WARPS = THREADS / 32;
   constexpr int TILE = THREADS * ITEMS;
   static_assert(RADIX <= THREADS, "one bin per thread");
   extern __shared__ __align__(16) unsigned char smem[];
   u32* whist = reinterpret_cast<u32*>(smem) + 2 * TILE;
   u32* wmask = whist + WARPS * S * RADIX + RADIX + WARPS + 1;
-  __shared__ u32 s_tile;
-  __shared__ u64 ebar;
+  __shared__ u32 s_tile, s_mcnt;
+  __shared__ u64 ebar, s_msrc;
+  __shared__ u32 s_tp[UNST == 3 ? RADIX + 1 : 1], s_fill[UNST == 3 ? RADIX : 1];
   const int tid = threadIdx.x;
+  if (UNST == 3) {  // the region map, loaded while thread 0's tile-counter atomic is in flight
+    if (tid <= RADIX) s_tp[tid] = mp.tprefix[tid];
+    if (tid < RADIX) s_fill[tid] = mp.fill[tid];
+    if (tid == 0) s_tile = atomicAdd(tile_ctr, 1u);
+    __syncthreads();
+  }
   if (tid == 0) {
-    const u32 t = atomicAdd(tile_ctr, 1u);
+    const u32 t = UNST == 3 ? s_tile : atomicAdd(tile_ctr, 1u);
     s_tile = t;
+    u64 tb = (u64)t * TILE;
+    u32 cnt = (u32)min((u64)TILE, (u64)m - tb);
+    if (UNST == 3) {  // region of tile t (binary search of the tile prefix), its keys' offset and count
+      u32 lo = 0, hi = RADIX;  // tprefix[lo] <= t < tprefix[hi]
+      while (hi - lo > 1) {
+        const u32 mid = (lo + hi) >> 1;
+        if (s_tp[mid] <= t) lo = mid;
+        else hi = mid;
+      }
+      const u32 o = (t - s_tp[lo]) * TILE;
+      tb = (u64)lo * mp.cap + o;
+      cnt = min((u32)TILE, s_fill[lo] - o);
+      s_msrc = tb, s_mcnt = cnt;
+    }
     if (TMA == 2) {  // start the tile's bulk copies before the counter arrays are cleared
-      const u64 tb = (u64)t * TILE;
-      const u32 cnt = (u32)min((u64)TILE, (u64)m - tb);
       const u32 bytes = (cnt * 8 + 15) & ~15u;  // key buffers carry >= 16 bytes of slack
       mbar_init(&ebar, 1);
       fence_mbar_init();
@@ -474,12 +512,16 @@ __global__ void __launch_bounds__(THREADS, MINB) onesweep2_kernel(const u64* __r
   const u32 tile = s_tile;
   unsigned long long* prof = g_prof ? g_prof + (u64)tile * 8 : nullptr;
   if (prof && tid == 0) prof[0] = gtime();
+  if (UNST == 3) {  // the tile as a tile of a virtual array: kin + tile * TILE = its keys, m = its end
+    kin = reinterpret_cast<const u64*>(reinterpret_cast<uintptr_t>(kin) + (s_msrc - (u64)tile * TILE) * 8);
+    m = tile * TILE + s_mcnt;
+  }
   if ((u64)(tile + 1) * TILE <= m)
     onesweep2_tile<THREADS, ITEMS, LBW, true, LATE_LB, S, BAL, TMA, MIX, UNST>(kin, kout, m, shift, bin_base, lookback,
-                                                                             epoch, tile, smem, prof, &ebar);
+                                                                             epoch, tile, smem, prof, &ebar, mp);
   else
     onesweep2_tile<THREADS, ITEMS, LBW, false, LATE_LB, S, BAL, TMA, MIX, UNST>(kin, kout, m, shift, bin_base, lookback,
-                                                                              epoch, tile, smem, prof, &ebar);
+                                                                              epoch, tile, smem, prof, &ebar, mp);
 }
 
 // the measured configuration: 256 x 32 keys, 2 CTAs/SM, look-back after ranking, one rank stream,
@@ -492,6 +534,7 @@ __global__ void __launch_bounds__(THREADS, MINB) onesweep2_kernel(const u64* __r
 constexpr int PT_THREADS = 256, PT_ITEMS = 32, PT_MINB = 2;
 #define OS_UCFG PT_THREADS, PT_ITEMS, PT_MINB, OS_LBW, true, 1, false, 2, 4, 1
 #define OS_UCFG2 PT_THREADS, PT_ITEMS, PT_MINB, OS_LBW, true, 1, false, 2, 4, 2
+#define OS_UCFG3 PT_THREADS, PT_ITEMS, PT_MINB, OS_LBW, true, 1, false, 2, 4, 3
 
 static size_t onesweep2_smem() {
   constexpr int WARPS = OS_THREADS / 32;
@@ -511,11 +554,26 @@ void launch_partition_pass(const u64* kin, u64* kout, u32 m, u32 shift, const u6
   const u32 tiles = (u32)((m + TILE - 1) / TILE);
   if (top) {
     smem_optin((const void*)onesweep2_kernel<OS_UCFG>, sm);
-    onesweep2_kernel<OS_UCFG><<<tiles, PT_THREADS, sm, st>>>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch);
+    onesweep2_kernel<OS_UCFG><<<tiles, PT_THREADS, sm, st>>>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch,
+                                                              MapArgs{});
   } else {
     smem_optin((const void*)onesweep2_kernel<OS_UCFG2>, sm);
-    onesweep2_kernel<OS_UCFG2><<<tiles, PT_THREADS, sm, st>>>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch);
+    onesweep2_kernel<OS_UCFG2><<<tiles, PT_THREADS, sm, st>>>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch,
+                                                               MapArgs{});
   }
+}
+
+// the second partition pass over the fused extents pass's regions (UNST 3): tiles = tprefix[RADIX] (host)
+void launch_partition_regions(const u64* kin, u64* kout, u32 tiles, u32 shift, const u64* bin_base, u64* lookback,
+                              u32* tile_ctr, u32 epoch, const u32* tprefix, const u32* fill, u64 cap, u32 pos_bits,
+                              u32 g0, cudaStream_t st) {
+  if (!tiles) return;
+  constexpr int WARPS = PT_THREADS / 32, TILE = PT_THREADS * PT_ITEMS;
+  const size_t sm = (size_t)TILE * 8 + (size_t)WARPS * RADIX * 4 + RADIX * 4 + (WARPS + 1) * 4;
+  smem_optin((const void*)onesweep2_kernel<OS_UCFG3>, sm);
+  MapArgs mp{tprefix, fill, cap, pos_bits, g0};
+  onesweep2_kernel<OS_UCFG3><<<tiles, PT_THREADS, sm, st>>>(kin, kout, (u32)((u64)tiles * TILE), shift, bin_base,
+                                                            lookback, tile_ctr, epoch, mp);
 }
 
 // bin bases of a digit histogram with every run padded to a multiple of 32 (the bucket path's first pass on a key
@@ -557,7 +615,8 @@ void launch_onesweep(const u64* kin, u64* kout, const u32* vin, u32* vout, u32 m
     const size_t sm = onesweep2_smem();
     smem_optin((const void*)onesweep2_kernel<OS_CFG>, sm);
     const u32 tiles = (u32)((m + OS_TILE - 1) / OS_TILE);
-    onesweep2_kernel<OS_CFG><<<tiles, OS_THREADS, sm, st>>>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch);
+    onesweep2_kernel<OS_CFG><<<tiles, OS_THREADS, sm, st>>>(kin, kout, m, shift, bin_base, lookback, tile_ctr, epoch,
+                                                             MapArgs{});
   }
 }
 

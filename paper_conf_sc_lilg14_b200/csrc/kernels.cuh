@@ -33,6 +33,27 @@ constexpr int CT_TILE = CT_THREADS * CT_ITEMS;
 void launch_extents(const Rec* rec, u64 n, u32 log2G, Summary* d_sum, u32* tile_hist, const Region* regs, u32 nreg,
                     u32 nreg_shared, int grid, cudaStream_t st, u32* gout = nullptr, u32* tile_hist2 = nullptr,
                     u32* wout = nullptr);
+// extents fused with the bucket path's first partition (k_extract.cu "Extents fused with ...")
+struct XPArgs {
+  const Rec* rec;
+  u32 n, log2G, pos_bits;
+  Summary* out;      // initialised like for launch_extents; bhist[3] = raw (g >> 22) & 255 histogram
+  u64* kout;         // RADIX regions of cap keys: region d = kout[d * cap, (d + 1) * cap)
+  u64 cap;
+  u32* gfill;        // [RADIX] zeroed: slots reserved per region (used, sentinel-padded)
+  u32* overflow;     // zeroed; 1 if a region would pass cap
+};
+void launch_extents_part(const XPArgs& A, cudaStream_t st);
+constexpr u32 PART_TILE_KEYS = 256 * 32;  // keys per tile of the partition passes (k_sort.cu PT_*)
+// the second partition pass over launch_extents_part's regions: tprefix[RADIX + 1] = tiles before region r
+// (ceil(fill[r] / PART_TILE_KEYS) per region), keys rebased from raw low-30 granule bits by g0
+void launch_partition_regions(const u64* kin, u64* kout, u32 tiles, u32 shift, const u64* bin_base, u64* lookback,
+                              u32* tile_ctr, u32 epoch, const u32* tprefix, const u32* fill, u64 cap, u32 pos_bits,
+                              u32 g0, cudaStream_t st);
+u64 extents_part_cap(u64 n);
+size_t presample_temp_bytes();
+void launch_presample(const Rec* rec, u32 n, u32 log2G, u32 want, void* temp, unsigned long long* h_ext,
+                      u32* samples, cudaStream_t st);
 void launch_extract_1to1(const Rec* rec, u64 n, const KeyLayout& L, u32 npass, u64* keys, u32* hist, u64 pos_base,
                          int grid, cudaStream_t st);
 void launch_entry_count(const Rec* rec, u64 n, u32 log2G, u32* cnt, cudaStream_t st);

@@ -494,6 +494,118 @@ bool sesa_trace::try_bucket_keys(u64 m, u64** comp, u32* m2, bool* used) {
   return true;
 }
 
+// ---- the bucket path with its first partition fused into the extents pass (k_extract.cu "Extents fused with the
+// bucket path's first partition"): predicted by a sample of 2^20 records before any pass (global, one granule,
+// (block, interval)-ordered, granule span 2^22 .. 2^30, even chunks); then checked exactly on the pass's summary.
+// *used = false (and true returned) when not predicted or not eligible: the caller runs the ordinary path.
+bool sesa_trace::try_extents_part(const Rec* rec, u64 n, u64 index_base, u64** comp, u32* m2, bool* used) {
+  *used = false;
+  if (n < BUCKET_MIN_N || n >= (1ull << 31) || n_regions) return true;
+  const u32 log2G = (u32)__builtin_ctz(cfg.granularity);
+  if (!grow(b_xtmp, presample_temp_bytes() + 256, "presample") || !grow(b_xsmall, 4096, "regions")) return false;
+  unsigned long long ext[4] = {1, 0, 0, 0};
+  u32 samples = 0;
+  LAUNCH("presample", 64.0 * (1 << 20), launch_presample(rec, (u32)n, log2G, 1u << 20, b_xtmp.p, ext, &samples, stream));
+  if (!sync_check("presample")) return false;
+  if (ext[0] || ext[1] > ext[2]) return true;  // a sampled record is shared, multi-granule, invalid or out of order
+  {
+    const u64 G0 = ext[1] & ~((1ull << (HYB_LO + RADIX_BITS)) - 1ull);
+    const u32 nb = bits_of(ext[2] - G0);
+    if (nb <= HYB_LO + RADIX_BITS || nb > HYB_LO + 2 * RADIX_BITS) return true;
+    const double mean = (double)n / (double)(((ext[2] - G0) >> HYB_CHUNK) + 1);
+    const double est_max = (double)ext[3] * (double)n / (double)std::max(1u, samples);
+    if (est_max > 4.0 * mean + 2048.0 || est_max > (double)(1u << 20)) return true;  // (bucket_choose's bound)
+  }
+  // the pass
+  const u32 pos_bits = std::max(1u, bits_of(n - 1));
+  const u64 cap = extents_part_cap(n);
+  if (!grow(b_summary, sizeof(Summary), "summary") || !grow(b_keys[1], (size_t)RADIX * cap * 8 + 64, "keys") ||
+      !grow(b_keys[0], n * 8 + 64, "keys"))
+    return false;
+  Summary init;
+  memset(&init, 0, sizeof init);
+  init.bad_index = ~0ull;
+  init.oob_first = ~0ull;
+  init.gmin[0] = init.gmin[1] = ~0ull;
+  init.bmin[0] = init.bmin[1] = init.imin[0] = init.imin[1] = ~0u;
+  u32* gfill = (u32*)b_xsmall.p;
+  u32* over = gfill + RADIX;
+  u32* tpre = over + 8;
+  if (!cuda_ok(cudaMemcpyAsync(b_summary.p, &init, sizeof(Summary), cudaMemcpyHostToDevice, stream), "summary init"))
+    return false;
+  cudaMemsetAsync(gfill, 0, (RADIX + 8) * 4, stream);
+  XPArgs X{rec, (u32)n, log2G, pos_bits, (Summary*)b_summary.p, (u64*)b_keys[1].p, cap, gfill, over};
+  LAUNCH("extents", 40.0 * n, launch_extents_part(X, stream));
+  std::vector<u32> fill(RADIX + 1);
+  if (!cuda_ok(cudaMemcpyAsync(&h_summary, b_summary.p, sizeof(Summary), cudaMemcpyDeviceToHost, stream), "summary") ||
+      !cuda_ok(cudaMemcpyAsync(fill.data(), gfill, (RADIX + 1) * 4, cudaMemcpyDeviceToHost, stream), "fills") ||
+      !sync_check("extents"))
+    return false;
+  const Summary& S = h_summary;
+  if (S.bad_index != ~0ull) return report_bad(reinterpret_cast<const sesa_access*>(rec), S.bad_index, S.bad_index);
+  const u64 G0 = S.gmin[1] & ~((1ull << (HYB_LO + RADIX_BITS)) - 1ull);
+  const u32 nb = S.count[1] == n ? bits_of(S.gmax[1] - G0) : 0u;
+  if (fill[RADIX] || S.count[0] || S.multi || S.entries != n || S.unsorted || nb <= HYB_LO + RADIX_BITS ||
+      nb > HYB_LO + 2 * RADIX_BITS || nb + pos_bits > 64)
+    return true;  // not the bucket path after all (or a region overflowed): the ordinary path from the start
+  set_oob(reinterpret_cast<const sesa_access*>(rec), 0, 0, index_base);
+  info.n_entries = n;
+  info.sorted_input = 1;
+  if (!make_layout(S, n)) return false;
+  KeyLayout& L = layout;
+  L.gminG = G0;
+  L.gbG = nb;
+  L.sort_bits = nb;
+  info.sort_bits = nb;
+  info.pos_bits = L.pos_bits;
+  info.digit_bits = RADIX_BITS;
+  info.fused_first_pass = 1;
+  info.bucket_path = 1;
+  info.sort_passes = 2;
+  // second pass: digit B = key_hi bits [22, 30) (the raw bits rotated by G0's), over the regions in digit-A order
+  std::vector<u32> row(RADIX), tp(RADIX + 1);
+  const u32 r = (u32)(G0 >> (HYB_LO + RADIX_BITS)) & (RADIX - 1);
+  for (u32 d = 0; d < (u32)RADIX; d++) row[d] = S.bhist[3][(d + r) & (RADIX - 1)];
+  tp[0] = 0;
+  for (u32 d = 0; d < (u32)RADIX; d++) tp[d + 1] = tp[d] + (fill[d] + PART_TILE_KEYS - 1) / PART_TILE_KEYS;
+  const u32 tiles = tp[RADIX];
+  if (!grow(b_hist, 2 * RADIX * 4, "hist") || !grow(b_binbase, 2 * RADIX * 8, "binbase") ||
+      !grow(b_ctotal, 16, "bucket count") || !grow(b_lookback, (size_t)tiles * RADIX * 8, "lookback") ||
+      !grow(b_ctr, 64 * 4, "counters"))
+    return false;
+  if (!cuda_ok(cudaMemcpyAsync(b_hist.p, row.data(), RADIX * 4, cudaMemcpyHostToDevice, stream), "hist") ||
+      !cuda_ok(cudaMemcpyAsync(tpre, tp.data(), (RADIX + 1) * 4, cudaMemcpyHostToDevice, stream), "tile prefix"))
+    return false;
+  LAUNCH("bin_base", 0.0, launch_bin_base((const u32*)b_hist.p, (u64*)b_binbase.p, 1, stream));
+  if (b_lookback.cap != lookback_cleared) {
+    cudaMemsetAsync(b_lookback.p, 0, b_lookback.cap, stream);
+    lookback_cleared = b_lookback.cap;
+    epoch = 0;
+  }
+  cudaMemsetAsync(b_ctr.p, 0, 64 * 4, stream);
+  if (++epoch >= 256) {
+    cudaMemsetAsync(b_lookback.p, 0, b_lookback.cap, stream);
+    epoch = 1;
+  }
+  LAUNCH("partition_pass", 16.0 * n,
+         launch_partition_regions((const u64*)b_keys[1].p, (u64*)b_keys[0].p, tiles, L.pos_bits + HYB_LO + RADIX_BITS,
+                                  (const u64*)b_binbase.p, (u64*)b_lookback.p, (u32*)b_ctr.p, epoch, tpre, gfill, cap,
+                                  L.pos_bits, (u32)(G0 & ((1ull << 30) - 1ull)), stream));
+  // per-chunk bitmap filter + sort of the survivors (k_bucket.cu)
+  const u32 nc = (u32)(((S.gmax[1] - G0) >> HYB_CHUNK) + 1);
+  if (!grow(b_btmp2, bucket_temp_bytes(nc), "bucket temp")) return false;
+  LAUNCH("bucket", 8.0 * n,
+         launches += launch_bucket_compact((u64*)b_keys[0].p, (u64*)b_keys[1].p, (u32)n, L.pos_bits, nc, b_btmp2.p,
+                                           (u32*)b_ctotal.p, stream) - 1);
+  *comp = (u64*)b_keys[0].p;
+  if (!cuda_ok(cudaMemcpyAsync(m2, b_ctotal.p, 4, cudaMemcpyDeviceToHost, stream), "bucket count") ||
+      !sync_check("bucket"))
+    return false;
+  info.n_multi = *m2;
+  *used = true;
+  return true;
+}
+
 // step 2' (distributed): histograms of keys that arrived from the exchange (already in b_keys[0])
 bool sesa_trace::step_hist(u64 m) {
   const u32 npass = (layout.sort_bits + RADIX_BITS - 1) / RADIX_BITS;
@@ -929,6 +1041,17 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
   }
   if (!check_records_ptr(d_rec, n)) return status;
   const Rec* rec = reinterpret_cast<const Rec*>(d_rec);
+#ifndef SESA_NO_XPART
+  {  // C5-like traces: the bucket path with its first partition fused into the extents pass
+    bool used = false;
+    u64* comp = nullptr;
+    u32 m2 = 0;
+    if (!try_extents_part(rec, n, index_base, &comp, &m2, &used)) return status;
+    if (used) return finish_check(comp, m2, rec, index_base);
+    memset(&info, 0, sizeof info);
+    info.n_records = n;
+  }
+#endif
   if (!step_extents(rec, n, true)) return status;
   const Summary& S = h_summary;
   if (S.bad_index != ~0ull) return report_bad(d_rec, S.bad_index, S.bad_index), status;

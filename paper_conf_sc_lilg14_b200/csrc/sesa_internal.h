@@ -44,6 +44,7 @@ struct sesa_trace {
   DevBuf b_races, b_rkeys[2], b_rvals[2], b_races_sorted, b_rhist, b_rbase;
   DevBuf b_eoff, b_ecnt, b_ecell, b_hrec, b_dist_races, b_ctmp, b_ctotal, b_thist, b_ftmp, b_thist2, b_btmp2;
   DevBuf b_wbits;   // per-record write bits from the extents pass (KeyLayout::wbit)
+  DevBuf b_xtmp, b_xsmall;  // fused extents + first partition: record sample; region fills, overflow, tile prefix
   DevBuf b_lraces;  // multi-launch checks: the races of the launches checked so far
   DevBuf b_franges, b_fkeep, b_fcnt2, b_foff2, b_frec, b_forig;  // descriptor-level check (NEXT-2)
   sesa_flow_check_info flow_info{};
@@ -121,6 +122,8 @@ struct sesa_trace {
   bool bucket_choose(uint64_t n, uint64_t* gmin_aligned, uint32_t* nbits, uint32_t* nchunks);
   bool step_bucket(uint64_t n, uint32_t nchunks, uint64_t** comp, uint32_t* m2);
   bool try_bucket_keys(uint64_t m, uint64_t** comp, uint32_t* m2, bool* used);
+  bool try_extents_part(const sesa::Rec* rec, uint64_t n, uint64_t index_base, uint64_t** comp, uint32_t* m2,
+                        bool* used);
   bool step_sort(uint64_t m, int* cur_out, uint32_t first_pass = 0, int cur0 = 0);
   bool step_compact(int cur, uint64_t m, uint64_t** comp, uint32_t* m2);
   bool step_conflict(const uint64_t* comp, uint32_t m2, const sesa::Rec* rec, uint32_t rec_pos_base,
