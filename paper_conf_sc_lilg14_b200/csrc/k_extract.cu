@@ -319,12 +319,17 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
 #define XP_THREADS_ 512
 #endif
 #ifndef XP_ROWS_
-#define XP_ROWS_ 4
+#define XP_ROWS_ 3
 #endif
 #ifndef XP_STAGES_
 #define XP_STAGES_ 3
 #endif
+#ifndef XP_CPP_
+#define XP_CPP_ 2
+#endif
+// XP_TILE records per ring chunk; XP_CPP chunks per partition round (XP_KT keys)
 constexpr int XP_THREADS = XP_THREADS_, XP_ROWS = XP_ROWS_, XP_TILE = XP_THREADS * XP_ROWS, XP_STAGES = XP_STAGES_;
+constexpr int XP_CPP = XP_CPP_, XP_KT = XP_TILE * XP_CPP;
 #ifndef XP_WIN_
 #define XP_WIN_ 256
 #endif
@@ -337,7 +342,7 @@ __global__ void __launch_bounds__(XP_THREADS, 1) extents_part_kernel(XPArgs A) {
   constexpr int THREADS = XP_THREADS, U = XP_ROWS;
   extern __shared__ __align__(128) unsigned char xp_ring[];
   __shared__ u64 bars[XP_STAGES];
-  __shared__ u64 stage[XP_TILE];
+  __shared__ u64 stage[XP_KT];
   __shared__ u32 s_cnt[RADIX], s_base[RADIX], s_hb[RADIX];
   __shared__ uint4 s_wo[RADIX];  // per digit: {d1, split, d2, -} (write-out deltas)
   __shared__ u32 s_tot;
@@ -354,7 +359,17 @@ __global__ void __launch_bounds__(XP_THREADS, 1) extents_part_kernel(XPArgs A) {
   A1.init();
   BulkRing<XP_STAGES> ring(xp_ring, bars, XP_TILE * 32);
   ring.start(A.rec, (u64)n * 32);  // (contains __syncthreads)
-  for (u64 j = 0; ring.next(j); j++) {
+  for (u64 j0 = 0; ring.next(j0); j0 += XP_CPP) {
+  u64 key[XP_CPP * U];
+  u32 rk[XP_CPP * U];
+#pragma unroll
+  for (int cc = 0; cc < XP_CPP; cc++) {
+    const u64 j = j0 + cc;
+    if (!ring.next(j)) {  // (CTA-uniform)
+#pragma unroll
+      for (int u = 0; u < U; u++) rk[cc * U + u] = ~0u;
+      continue;
+    }
     const u32 tile = (u32)ring.chunk_index(j);
     const u32 tb = tile * XP_TILE, r0 = tb + warp * 32 * U;
     // the (block, interval) before the warp's first row: in the ring, or (warp 0) the previous tile's last record
@@ -363,11 +378,10 @@ __global__ void __launch_bounds__(XP_THREADS, 1) extents_part_kernel(XPArgs A) {
     const uint4* R = reinterpret_cast<const uint4*>(ring.wait(j));
     if (warp > 0) pv = R[2 * (warp * 32 * U - 1) + 1];
     u64 prev_bi = ((u64)pv.x << 32) | pv.z;
-    u64 key[U];
-    u32 rk[U];
 #pragma unroll
-    for (int u = 0; u < U; u++) {
-      const u32 i = r0 + u * 32 + lane, li = warp * 32 * U + u * 32 + lane;
+    for (int uu = 0; uu < U; uu++) {
+      const int u = cc * U + uu;
+      const u32 i = r0 + uu * 32 + lane, li = warp * 32 * U + uu * 32 + lane;
       const bool in = i < n;
       const uint4 ca = in ? R[2 * li] : make_uint4(0, 0, 0, 0), cb = in ? R[2 * li + 1] : make_uint4(0, 0, 0, 0);
       const u64 bi = ((u64)cb.x << 32) | cb.z;
@@ -398,6 +412,7 @@ __global__ void __launch_bounds__(XP_THREADS, 1) extents_part_kernel(XPArgs A) {
       }
     }
     ring.release(j);  // (contains __syncthreads: the slot is refilled with tile j + XP_STAGES)
+  }
     // Thread d < RADIX (warps 0-7): the digit's stage base — the counts of the warps before it by one warp
     // reduction each (redux), its own warp by a shuffle scan: no block scan, one barrier less — and this tile's
     // slots in the CTA's windows.  The next window is reserved ahead (its atomic's result is first needed a tile
@@ -441,7 +456,7 @@ __global__ void __launch_bounds__(XP_THREADS, 1) extents_part_kernel(XPArgs A) {
     __syncthreads();
     if (tid < RADIX) s_cnt[tid] = 0;  // (every count was read before the barrier)
 #pragma unroll
-    for (int u = 0; u < U; u++)
+    for (int u = 0; u < XP_CPP * U; u++)
       if (rk[u] != ~0u) stage[s_base[(u32)(key[u] >> (A.pos_bits + HYB_LO)) & (RADIX - 1)] + rk[u]] = key[u];
     __syncthreads();
     // coalesced runs: stage slot jj of digit d goes to its window slot
@@ -480,8 +495,10 @@ void launch_extents_part(const XPArgs& A, cudaStream_t st) {
 
 u64 extents_part_cap(u64 n) {
   // per region: the mean, 1/8 more, a window per CTA and a tile of slack, in whole 32-key rows
+  // (a multiple of the second pass's tile: its tiles read whole tiles inside a region)
   const u64 mean = (n + RADIX - 1) / RADIX;
-  return ((mean + mean / 8 + (u64)XP_WIN * (u64)dev_sm_count() + XP_TILE) + 31) & ~31ull;
+  const u64 c = mean + mean / 8 + 2 * (u64)XP_WIN * (u64)dev_sm_count() + XP_KT;
+  return (c + PART_TILE_KEYS - 1) / PART_TILE_KEYS * PART_TILE_KEYS;
 }
 
 // ---- record sample predicting the fused path (before any pass) -----------------------------------------------

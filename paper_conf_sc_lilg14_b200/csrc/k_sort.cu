@@ -237,12 +237,13 @@ __device__ unsigned long long* g_prof = nullptr;
 
 // UNST == 3 (the second partition pass after the fused extents + first partition, k_extract.cu): the input is
 // RADIX regions of cap keys, region r holding fill[r] keys (sentinel-padded); tiles never straddle regions
-// (tile t of region r: tprefix[r] <= t < tprefix[r + 1]), and each key is rebased on load from raw low-30 granule
-// bits to key_hi = (raw - g0) mod 2^30 (sentinels stay ~0)
+// (tile t belongs to region t / tpr: no lookup before the tile's bulk copy, which reads a whole tile; the keys past
+// the fill are not used), and each key is rebased on load from raw low-30 granule bits to key_hi =
+// (raw - g0) mod 2^30 (sentinels stay ~0)
 struct MapArgs {
-  const u32* tprefix;  // [RADIX + 1]
   const u32* fill;     // [RADIX]
   u64 cap;
+  u32 tpr;             // tiles per region (a tile past a region's fill is empty or partial)
   u32 pos_bits, g0;    // rebase: pos_bits of the layout, low 30 bits of G0
 };
 
@@ -471,30 +472,19 @@ __global__ void __launch_bounds__(THREADS, MINB) onesweep2_kernel(const u64* __r
   u32* wmask = whist + WARPS * S * RADIX + RADIX + WARPS + 1;
   __shared__ u32 s_tile, s_mcnt;
   __shared__ u64 ebar, s_msrc;
-  __shared__ u32 s_tp[UNST == 3 ? RADIX + 1 : 1], s_fill[UNST == 3 ? RADIX : 1];
   const int tid = threadIdx.x;
-  if (UNST == 3) {  // the region map, loaded while thread 0's tile-counter atomic is in flight
-    if (tid <= RADIX) s_tp[tid] = mp.tprefix[tid];
-    if (tid < RADIX) s_fill[tid] = mp.fill[tid];
-    if (tid == 0) s_tile = atomicAdd(tile_ctr, 1u);
-    __syncthreads();
-  }
   if (tid == 0) {
-    const u32 t = UNST == 3 ? s_tile : atomicAdd(tile_ctr, 1u);
+    const u32 t = atomicAdd(tile_ctr, 1u);
     s_tile = t;
     u64 tb = (u64)t * TILE;
     u32 cnt = (u32)min((u64)TILE, (u64)m - tb);
-    if (UNST == 3) {  // region of tile t (binary search of the tile prefix), its keys' offset and count
-      u32 lo = 0, hi = RADIX;  // tprefix[lo] <= t < tprefix[hi]
-      while (hi - lo > 1) {
-        const u32 mid = (lo + hi) >> 1;
-        if (s_tp[mid] <= t) lo = mid;
-        else hi = mid;
-      }
-      const u32 o = (t - s_tp[lo]) * TILE;
-      tb = (u64)lo * mp.cap + o;
-      cnt = min((u32)TILE, s_fill[lo] - o);
-      s_msrc = tb, s_mcnt = cnt;
+    u32 rf = 0, o = 0;
+    if (UNST == 3) {  // region t / tpr; the whole tile is copied, its key count is known when the fill arrives
+      const u32 r = t / mp.tpr;
+      o = (t - r * mp.tpr) * TILE;
+      tb = (u64)r * mp.cap + o;
+      cnt = TILE;
+      rf = mp.fill[r];  // (in flight with the bulk copy)
     }
     if (TMA == 2) {  // start the tile's bulk copies before the counter arrays are cleared
       const u32 bytes = (cnt * 8 + 15) & ~15u;  // key buffers carry >= 16 bytes of slack
@@ -504,6 +494,7 @@ __global__ void __launch_bounds__(THREADS, MINB) onesweep2_kernel(const u64* __r
       for (u32 off = 0; off < bytes; off += 16384)
         bulk_g2s(smem + off, reinterpret_cast<const unsigned char*>(kin + tb) + off, min(16384u, bytes - off), &ebar);
     }
+    if (UNST == 3) s_msrc = tb, s_mcnt = rf > o ? min((u32)TILE, rf - o) : 0u;
   }
   for (int i = tid; i < WARPS * S * RADIX; i += THREADS) whist[i] = 0;
   if (!BAL && !UNST)
@@ -564,14 +555,15 @@ void launch_partition_pass(const u64* kin, u64* kout, u32 m, u32 shift, const u6
 }
 
 // the second partition pass over the fused extents pass's regions (UNST 3): tiles = tprefix[RADIX] (host)
-void launch_partition_regions(const u64* kin, u64* kout, u32 tiles, u32 shift, const u64* bin_base, u64* lookback,
-                              u32* tile_ctr, u32 epoch, const u32* tprefix, const u32* fill, u64 cap, u32 pos_bits,
-                              u32 g0, cudaStream_t st) {
+void launch_partition_regions(const u64* kin, u64* kout, u32 tpr, u32 shift, const u64* bin_base, u64* lookback,
+                              u32* tile_ctr, u32 epoch, const u32* fill, u64 cap, u32 pos_bits, u32 g0,
+                              cudaStream_t st) {
+  const u32 tiles = tpr * RADIX;
   if (!tiles) return;
   constexpr int WARPS = PT_THREADS / 32, TILE = PT_THREADS * PT_ITEMS;
   const size_t sm = (size_t)TILE * 8 + (size_t)WARPS * RADIX * 4 + RADIX * 4 + (WARPS + 1) * 4;
   smem_optin((const void*)onesweep2_kernel<OS_UCFG3>, sm);
-  MapArgs mp{tprefix, fill, cap, pos_bits, g0};
+  MapArgs mp{fill, cap, tpr, pos_bits, g0};
   onesweep2_kernel<OS_UCFG3><<<tiles, PT_THREADS, sm, st>>>(kin, kout, (u32)((u64)tiles * TILE), shift, bin_base,
                                                             lookback, tile_ctr, epoch, mp);
 }

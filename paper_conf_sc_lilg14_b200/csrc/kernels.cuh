@@ -45,11 +45,11 @@ struct XPArgs {
 };
 void launch_extents_part(const XPArgs& A, cudaStream_t st);
 constexpr u32 PART_TILE_KEYS = 256 * 32;  // keys per tile of the partition passes (k_sort.cu PT_*)
-// the second partition pass over launch_extents_part's regions: tprefix[RADIX + 1] = tiles before region r
-// (ceil(fill[r] / PART_TILE_KEYS) per region), keys rebased from raw low-30 granule bits by g0
-void launch_partition_regions(const u64* kin, u64* kout, u32 tiles, u32 shift, const u64* bin_base, u64* lookback,
-                              u32* tile_ctr, u32 epoch, const u32* tprefix, const u32* fill, u64 cap, u32 pos_bits,
-                              u32 g0, cudaStream_t st);
+// the second partition pass over launch_extents_part's regions: tpr tiles per region (cap is a multiple of
+// PART_TILE_KEYS, tpr * PART_TILE_KEYS >= every fill), keys rebased from raw low-30 granule bits by g0
+void launch_partition_regions(const u64* kin, u64* kout, u32 tpr, u32 shift, const u64* bin_base, u64* lookback,
+                              u32* tile_ctr, u32 epoch, const u32* fill, u64 cap, u32 pos_bits, u32 g0,
+                              cudaStream_t st);
 u64 extents_part_cap(u64 n);
 size_t presample_temp_bytes();
 void launch_presample(const Rec* rec, u32 n, u32 log2G, u32 want, void* temp, unsigned long long* h_ext,

@@ -530,7 +530,6 @@ bool sesa_trace::try_extents_part(const Rec* rec, u64 n, u64 index_base, u64** c
   init.bmin[0] = init.bmin[1] = init.imin[0] = init.imin[1] = ~0u;
   u32* gfill = (u32*)b_xsmall.p;
   u32* over = gfill + RADIX;
-  u32* tpre = over + 8;
   if (!cuda_ok(cudaMemcpyAsync(b_summary.p, &init, sizeof(Summary), cudaMemcpyHostToDevice, stream), "summary init"))
     return false;
   cudaMemsetAsync(gfill, 0, (RADIX + 8) * 4, stream);
@@ -563,18 +562,17 @@ bool sesa_trace::try_extents_part(const Rec* rec, u64 n, u64 index_base, u64** c
   info.bucket_path = 1;
   info.sort_passes = 2;
   // second pass: digit B = key_hi bits [22, 30) (the raw bits rotated by G0's), over the regions in digit-A order
-  std::vector<u32> row(RADIX), tp(RADIX + 1);
+  std::vector<u32> row(RADIX);
   const u32 r = (u32)(G0 >> (HYB_LO + RADIX_BITS)) & (RADIX - 1);
   for (u32 d = 0; d < (u32)RADIX; d++) row[d] = S.bhist[3][(d + r) & (RADIX - 1)];
-  tp[0] = 0;
-  for (u32 d = 0; d < (u32)RADIX; d++) tp[d + 1] = tp[d] + (fill[d] + PART_TILE_KEYS - 1) / PART_TILE_KEYS;
-  const u32 tiles = tp[RADIX];
+  // tiles per region from the fullest region (C5: ~1.5% of the tiles are empty or partial)
+  const u32 tpr = (*std::max_element(fill.begin(), fill.begin() + RADIX) + PART_TILE_KEYS - 1) / PART_TILE_KEYS;
+  const u32 tiles = tpr * RADIX;
   if (!grow(b_hist, 2 * RADIX * 4, "hist") || !grow(b_binbase, 2 * RADIX * 8, "binbase") ||
       !grow(b_ctotal, 16, "bucket count") || !grow(b_lookback, (size_t)tiles * RADIX * 8, "lookback") ||
       !grow(b_ctr, 64 * 4, "counters"))
     return false;
-  if (!cuda_ok(cudaMemcpyAsync(b_hist.p, row.data(), RADIX * 4, cudaMemcpyHostToDevice, stream), "hist") ||
-      !cuda_ok(cudaMemcpyAsync(tpre, tp.data(), (RADIX + 1) * 4, cudaMemcpyHostToDevice, stream), "tile prefix"))
+  if (!cuda_ok(cudaMemcpyAsync(b_hist.p, row.data(), RADIX * 4, cudaMemcpyHostToDevice, stream), "hist"))
     return false;
   LAUNCH("bin_base", 0.0, launch_bin_base((const u32*)b_hist.p, (u64*)b_binbase.p, 1, stream));
   if (b_lookback.cap != lookback_cleared) {
@@ -588,8 +586,8 @@ bool sesa_trace::try_extents_part(const Rec* rec, u64 n, u64 index_base, u64** c
     epoch = 1;
   }
   LAUNCH("partition_pass", 16.0 * n,
-         launch_partition_regions((const u64*)b_keys[1].p, (u64*)b_keys[0].p, tiles, L.pos_bits + HYB_LO + RADIX_BITS,
-                                  (const u64*)b_binbase.p, (u64*)b_lookback.p, (u32*)b_ctr.p, epoch, tpre, gfill, cap,
+         launch_partition_regions((const u64*)b_keys[1].p, (u64*)b_keys[0].p, tpr, L.pos_bits + HYB_LO + RADIX_BITS,
+                                  (const u64*)b_binbase.p, (u64*)b_lookback.p, (u32*)b_ctr.p, epoch, gfill, cap,
                                   L.pos_bits, (u32)(G0 & ((1ull << 30) - 1ull)), stream));
   // per-chunk bitmap filter + sort of the survivors (k_bucket.cu)
   const u32 nc = (u32)(((S.gmax[1] - G0) >> HYB_CHUNK) + 1);
