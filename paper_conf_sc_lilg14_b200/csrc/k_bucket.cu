@@ -130,7 +130,7 @@ __global__ void __launch_bounds__(BK_THREADS) bucket_local_kernel(BucketArgs A) 
       for (int u = 0; u < BK_U; u++) k[u] = kn[u];
     }
     __syncthreads();
-    // sweep 2: survivors in order (element order = position); their full keys are read back (few on this path)
+    // sweep 2: the survivors (in element order, which need not be position order); their full keys are read back
     u32 k_total = 0;  // survivors so far (uniform)
     for (u32 b0 = s; b0 < e; b0 += BK_THREADS * BK_U) {
       bool keep[BK_U];
@@ -182,9 +182,11 @@ __global__ void __launch_bounds__(BK_THREADS) bucket_local_kernel(BucketArgs A) 
   }
 }
 
-// ---- overflow chunks: stable LSD radix sort of the survivors by key_hi bits [0, HYB_CHUNK) in global memory ----
-// (they are already ordered by the higher bits and, within equal key_hi, by position), one CTA per chunk, two
-// passes of 8 / 7 bits ping-ponging between the staging range and the chunk's dead range of the sorted keys.
+// ---- overflow chunks: stable LSD radix sort of the survivors by (key_hi bits [0, HYB_CHUNK), position) in global
+// memory, one CTA per chunk: 8-bit passes over the position bits, then two passes of 8 / 7 bits over key_hi,
+// ping-ponging between the staging range and the chunk's dead range of the sorted keys.  (The partition passes
+// before are unstable and the fused extents pass writes its regions in window order, so the survivors of a chunk
+// arrive in no particular position order.)
 __global__ void __launch_bounds__(BK_THREADS) bucket_overflow_kernel(BucketArgs A) {
   __shared__ u32 hist[RADIX], run[RADIX], wc[BK_THREADS / 32][RADIX];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -194,9 +196,16 @@ __global__ void __launch_bounds__(BK_THREADS) bucket_overflow_kernel(BucketArgs 
   const u32 s = A.bounds[c], k = A.cnt[c];
   u64* src = A.stage + s;
   u64* dst = A.spare + s;
-  for (u32 pass = 0; pass < 2; pass++) {
-    const u32 sh = A.pos_bits + pass * RADIX_BITS;
-    const u32 dmask = pass == 0 ? RADIX - 1 : (1u << (HYB_CHUNK - RADIX_BITS)) - 1u;
+  const u32 npos = (A.pos_bits + RADIX_BITS - 1) / RADIX_BITS;
+  for (u32 pass = 0; pass < npos + 2; pass++) {
+    u32 sh, dmask;
+    if (pass < npos) {  // position digits
+      sh = pass * RADIX_BITS;
+      dmask = (1u << min((u32)RADIX_BITS, A.pos_bits - sh)) - 1u;
+    } else {            // key_hi bits [0, 8), [8, HYB_CHUNK)
+      sh = A.pos_bits + (pass - npos) * RADIX_BITS;
+      dmask = pass == npos ? RADIX - 1 : (1u << (HYB_CHUNK - RADIX_BITS)) - 1u;
+    }
     for (int i = tid; i < RADIX; i += BK_THREADS) hist[i] = 0;
     __syncthreads();
     for (u32 i = tid; i < k; i += BK_THREADS) atomicAdd(&hist[(u32)(src[i] >> sh) & dmask], 1u);
@@ -234,7 +243,11 @@ __global__ void __launch_bounds__(BK_THREADS) bucket_overflow_kernel(BucketArgs 
     src = dst;
     dst = t;
   }
-  // two passes: the result is back in the staging range
+  // an odd number of passes leaves the result in the dead range: back to the staging range
+  if ((npos + 2) & 1u) {
+    __syncthreads();
+    for (u32 i = tid; i < k; i += BK_THREADS) dst[i] = src[i];
+  }
   __syncthreads();
   }
 }

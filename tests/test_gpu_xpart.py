@@ -106,3 +106,14 @@ def test_invalid_record_between_samples(S, base_trace):
         t.check(S.to_device(a), len(a))
     t.close()
     assert e.value.status == S.SESA_EINVAL and "record 3000003 " in str(e.value)  # the lowest bad index
+
+
+def test_dense_chunks_overflow_sort(S):
+    # 2^23 words for 2^24 records: almost every entry survives, every chunk has far more than 2,048 survivors,
+    # so each is sorted by the global-memory (key_hi, position) radix sort — the fused pass writes its regions in
+    # window order, so the survivors arrive in no particular position order
+    from sesagen import configs as C
+    a = C.rnd_host(N, 79, blocks=4096, threads=512, intervals=3, words=1 << 23, shared_frac=0.0, sizes=(4,),
+                   unaligned=False, values=3, atomic_frac=0.05, write_frac=0.35)
+    info, names = run(S, a, ls=1)
+    assert info["bucket_path"] == 1 and names["extents"] == 1 and "presample" in names
