@@ -503,18 +503,22 @@ bool sesa_trace::try_extents_part(const Rec* rec, u64 n, u64 index_base, u64** c
   if (n < BUCKET_MIN_N || n >= (1ull << 31) || n_regions) return true;
   const u32 log2G = (u32)__builtin_ctz(cfg.granularity);
   if (!grow(b_xtmp, presample_temp_bytes() + 256, "presample") || !grow(b_xsmall, 4096, "regions")) return false;
-  unsigned long long ext[4] = {1, 0, 0, 0};
-  u32 samples = 0;
-  LAUNCH("presample", 64.0 * (1 << 20), launch_presample(rec, (u32)n, log2G, 1u << 20, b_xtmp.p, ext, &samples, stream));
-  if (!sync_check("presample")) return false;
-  if (ext[0] || ext[1] > ext[2]) return true;  // a sampled record is shared, multi-granule, invalid or out of order
-  {
+  // two stages (bucket_choose's bounds): 2^16 samples reject most other traces at once — a shared or
+  // multi-granule record, an inversion, a hot region (C2-C4) — then 2^20 samples for the tight chunk bound
+  for (u32 want : {1u << 16, 1u << 20}) {
+    unsigned long long ext[4] = {1, 0, 0, 0};
+    u32 samples = 0;
+    LAUNCH("presample", 64.0 * want, launch_presample(rec, (u32)n, log2G, want, b_xtmp.p, ext, &samples, stream));
+    if (!sync_check("presample")) return false;
+    if (ext[0] || ext[1] > ext[2]) return true;  // a sampled record is shared, multi-granule, invalid or out of order
     const u64 G0 = ext[1] & ~((1ull << (HYB_LO + RADIX_BITS)) - 1ull);
     const u32 nb = bits_of(ext[2] - G0);
     if (nb <= HYB_LO + RADIX_BITS || nb > HYB_LO + 2 * RADIX_BITS) return true;
     const double mean = (double)n / (double)(((ext[2] - G0) >> HYB_CHUNK) + 1);
     const double est_max = (double)ext[3] * (double)n / (double)std::max(1u, samples);
-    if (est_max > 4.0 * mean + 2048.0 || est_max > (double)(1u << 20)) return true;  // (bucket_choose's bound)
+    if (want < (1u << 20) ? est_max > 32.0 * mean + 65536.0
+                          : (est_max > 4.0 * mean + 2048.0 || est_max > (double)(1u << 20)))
+      return true;
   }
   // the pass
   const u32 pos_bits = std::max(1u, bits_of(n - 1));

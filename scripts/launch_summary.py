@@ -16,7 +16,11 @@ for r in rows:
         e = L.setdefault(d["ID"], {"name": d["Kernel Name"].split("(")[0].replace("void ", "")})
         e[d["Metric Name"]] = float(d["Metric Value"].replace(",", ""))
 ls = list(L.values())
-last = max(i for i, x in enumerate(ls) if "extents2" in x["name"])
+# a step starts at its first pass over the records: the record sample of the fused path, else the extents pass
+starts = [i for i, x in enumerate(ls) if "presample_kernel" in x["name"]]
+if not starts:
+    starts = [i for i, x in enumerate(ls) if "extents2" in x["name"]]
+last = max(starts)
 step = ls[last:]
 agg = defaultdict(lambda: [0, 0.0, 0.0, 0.0])
 for x in step:
