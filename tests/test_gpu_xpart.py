@@ -65,7 +65,7 @@ def test_c5_recipe_through_the_fused_path(S):
     assert got.tobytes() == C.c5_truth(n).tobytes()
 
 
-@pytest.mark.parametrize("what", ["shared", "two_granules", "inversion"])
+@pytest.mark.parametrize("what", ["shared", "two_granules", "inversion", "far"])
 def test_unsampled_exception_falls_back(S, base_trace, what):
     if what == "inversion":  # (an unsorted trace keys (block, interval) too: a span that fits 64 bits then)
         from sesagen import configs as C
@@ -79,12 +79,14 @@ def test_unsampled_exception_falls_back(S, base_trace, what):
         a["addr"][i] = 64
     elif what == "two_granules":
         a["size"][i] = 8
+    elif what == "far":  # a granule span beyond 2^30 that the sample did not see
+        a["addr"][i] = a["addr"][i] + np.uint64(1 << 40)
     else:
         a["block"][i] = a["block"][i - 1] - 1 if a["block"][i - 1] > 0 else 0
         a["interval"][i] = 0
         a["block"][i - 1] = max(int(a["block"][i - 1]), 1)
     info, names = run(S, a)
-    assert names["presample"] == 1 and names["extents"] == 2  # the fused pass, then the ordinary path
+    assert names["presample"] >= 1 and names["extents"] == 2  # the fused pass, then the ordinary path
 
 
 def test_uneven_first_digit_overflows_and_falls_back(S, base_trace):
@@ -117,3 +119,20 @@ def test_dense_chunks_overflow_sort(S):
                    unaligned=False, values=3, atomic_frac=0.05, write_frac=0.35)
     info, names = run(S, a, ls=1)
     assert info["bucket_path"] == 1 and names["extents"] == 1 and "presample" in names
+
+
+def test_regions_registered_skip_the_fused_pass(S, base_trace):
+    # the out-of-bound check (NEXT-1) runs in the ordinary extents pass: with regions the fused pass is not tried
+    t = S.Trace(32, 0, 4)
+    t.set_profiling(True)
+    lo, hi = int(base_trace["addr"].min()), int(base_trace["addr"].max()) + 4
+    reg = np.zeros(1, S.REGION_DTYPE)
+    reg["base"], reg["size"], reg["space"] = lo, hi - lo, G.GLOBAL
+    t.set_regions(reg)
+    t.check(S.to_device(base_trace), len(base_trace))
+    names = {k["name"]: k["launches"] for k in t.kernel_stats()}
+    got = t.races()
+    assert t.oob()["n_oob"] == 0
+    t.close()
+    assert "presample" not in names
+    assert got.tobytes() == O.check(base_trace, method="partitioned").tobytes()
