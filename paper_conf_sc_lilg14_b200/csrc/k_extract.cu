@@ -615,9 +615,12 @@ __global__ void __launch_bounds__(THREADS) extract_1to1_kernel(const Rec* __rest
       const u32 t = h * THREADS + threadIdx.x;
       if (t >= nr) continue;
       const Rec& x = R[t];
-      const u64 key = (key_hi_of(L, x.space, x.block, x.interval, x.addr >> L.log2G) << L.pos_bits) | (pos_base + c0 + t);
+      // (with KeyLayout::wbit the write bit sits below the position)
+      const u64 key = (key_hi_of(L, x.space, x.block, x.interval, x.addr >> L.log2G) << (L.pos_bits + L.wbit)) |
+                      ((pos_base + c0 + t) << L.wbit) | (L.wbit && x.rw != RW_READ ? 1ull : 0ull);
       __stcs(keys + c0 + t, key);
-      for (u32 p = 0; p < npass; p++) atomicAdd(&wsh[p * RADIX + ((key >> (L.pos_bits + p * RB)) & (RADIX - 1))], 1u);
+      for (u32 p = 0; p < npass; p++)
+        atomicAdd(&wsh[p * RADIX + ((key >> (L.pos_bits + L.wbit + p * RB)) & (RADIX - 1))], 1u);
     }
     ring.release(j);
   }
@@ -665,9 +668,11 @@ __global__ void __launch_bounds__(THREADS) extract_multi_kernel(const Rec* __res
     u64 glo = r.addr >> L.log2G, ghi = (r.addr + (u64)(r.size - 1)) >> L.log2G;
     u64 o = off[k];
     for (u64 g = glo; g <= ghi; g++, o++) {
-      u64 key = (key_hi_of(L, r.space, r.block, r.interval, g) << L.pos_bits) | (pos_base + k);
+      u64 key = (key_hi_of(L, r.space, r.block, r.interval, g) << (L.pos_bits + L.wbit)) | ((pos_base + k) << L.wbit) |
+                (L.wbit && r.rw != RW_READ ? 1ull : 0ull);
       keys[o] = key;
-      for (u32 p = 0; p < npass; p++) atomicAdd(&sh[p * RADIX + ((key >> (L.pos_bits + p * RB)) & (RADIX - 1))], 1u);
+      for (u32 p = 0; p < npass; p++)
+        atomicAdd(&sh[p * RADIX + ((key >> (L.pos_bits + L.wbit + p * RB)) & (RADIX - 1))], 1u);
     }
   }
   __syncthreads();

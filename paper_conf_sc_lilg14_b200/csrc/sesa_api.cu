@@ -1109,6 +1109,13 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
 #endif
     if (!step_extract_fused(rec, n) || !step_sort(m, &cur, 1, 1)) return status;
   } else {
+    // the write bit, unless the key array may still take the bucket path (whose kernels read plain keys)
+    const KeyLayout& L = layout;
+    const bool bucket_ok = !(m < BUCKET_MIN_N || L.both || (L.single_space == SP_GLOBAL && L.lowG) ||
+                             L.sort_bits <= HYB_LO + RADIX_BITS || L.sort_bits > HYB_LO + 2 * RADIX_BITS);
+#ifndef SESA_NO_WBIT
+    layout.wbit = !bucket_ok && layout.sort_bits + layout.pos_bits + 1 <= 64 ? 1u : 0u;
+#endif
     if (!step_extract(rec, n, m, 0, S.multi != 0)) return status;
     bool used = false;
     u64* bcomp = nullptr;
