@@ -325,16 +325,17 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
 #define XP_STAGES_ 3
 #endif
 #ifndef XP_CPP_
-#define XP_CPP_ 2
+#define XP_CPP_ 6
 #endif
 // XP_TILE records per ring chunk; XP_CPP chunks per partition round (XP_KT keys)
 constexpr int XP_THREADS = XP_THREADS_, XP_ROWS = XP_ROWS_, XP_TILE = XP_THREADS * XP_ROWS, XP_STAGES = XP_STAGES_;
 constexpr int XP_CPP = XP_CPP_, XP_KT = XP_TILE * XP_CPP;
 #ifndef XP_WIN_
-#define XP_WIN_ 256
+#define XP_WIN_ 128
 #endif
 constexpr u32 XP_WIN = XP_WIN_;
-constexpr size_t XP_SMEM = (size_t)XP_STAGES * XP_TILE * 32;  // the record ring (dynamic shared memory)
+// dynamic shared memory: the record ring, then the stage of a round's keys (static shared memory stops at 48 KB)
+constexpr size_t XP_RING = (size_t)XP_STAGES * XP_TILE * 32, XP_SMEM = XP_RING + (size_t)XP_KT * 8;
 
 // The tiles' records arrive by TMA bulk copies into a ring of XP_STAGES tiles (192 KB in flight per SM without
 // registers: one CTA of 512 threads per SM would otherwise hold one tile in flight and stall on every barrier).
@@ -342,7 +343,7 @@ __global__ void __launch_bounds__(XP_THREADS, 1) extents_part_kernel(XPArgs A) {
   constexpr int THREADS = XP_THREADS, U = XP_ROWS;
   extern __shared__ __align__(128) unsigned char xp_ring[];
   __shared__ u64 bars[XP_STAGES];
-  __shared__ u64 stage[XP_KT];
+  u64* stage = reinterpret_cast<u64*>(xp_ring + XP_RING);  // [XP_KT]
   __shared__ u32 s_cnt[RADIX], s_base[RADIX], s_hb[RADIX];
   __shared__ uint4 s_wo[RADIX];  // per digit: {d1, split, d2, -} (write-out deltas)
   __shared__ u32 s_tot;
