@@ -316,16 +316,16 @@ __global__ void __launch_bounds__(256) extents2_kernel(const Rec* __restrict__ r
 // (4) keys into shared memory by digit, (5) coalesced write-out.
 // ------------------------------------------------------------------------------------------------------------
 #ifndef XP_THREADS_
-#define XP_THREADS_ 512
+#define XP_THREADS_ 768
 #endif
 #ifndef XP_ROWS_
 #define XP_ROWS_ 3
 #endif
 #ifndef XP_STAGES_
-#define XP_STAGES_ 3
+#define XP_STAGES_ 2
 #endif
 #ifndef XP_CPP_
-#define XP_CPP_ 6
+#define XP_CPP_ 4
 #endif
 // XP_TILE records per ring chunk; XP_CPP chunks per partition round (XP_KT keys)
 constexpr int XP_THREADS = XP_THREADS_, XP_ROWS = XP_ROWS_, XP_TILE = XP_THREADS * XP_ROWS, XP_STAGES = XP_STAGES_;
