@@ -116,34 +116,6 @@ __global__ void __launch_bounds__(256, 4) compact_seg_kernel(const u64* __restri
 #ifndef COMPACT_W_MINB
 #define COMPACT_W_MINB 4
 #endif
-#ifndef COMPACT_W_SKIP
-#define COMPACT_W_SKIP 1
-#endif
-#ifndef COMPACT_W_KS
-#define COMPACT_W_KS 0
-#endif
-// segmented OR over a row's lanes on warp-uniform masks (Kogge-Stone with stop masks): bit l of the result =
-// OR of W over [the head of l's run, l] (fwd) / [l, the last lane of l's run] (bwd); H = heads (lane l starts a
-// run), cin = the carry entering at lane 0 (fwd, if lane 0 is no head) / at lane 31 (bwd, if the run goes on)
-__device__ __forceinline__ unsigned seg_or_fwd(unsigned W, unsigned H, unsigned cin) {
-  unsigned F = W | (cin & ~H & 1u), P = ~H;  // P bit l: l may take from l - 1
-  F |= (F << 1) & P, P &= P << 1;
-  F |= (F << 2) & P, P &= P << 2;
-  F |= (F << 4) & P, P &= P << 4;
-  F |= (F << 8) & P, P &= P << 8;
-  F |= (F << 16) & P;
-  return F;
-}
-__device__ __forceinline__ unsigned seg_or_bwd(unsigned W, unsigned H, unsigned cin) {
-  unsigned Q = ~(H >> 1) & 0x7FFFFFFFu;  // Q bit l: l may take from l + 1 (l + 1 is no head)
-  unsigned B = W | (cin << 31);
-  B |= (B >> 1) & Q, Q &= Q >> 1;
-  B |= (B >> 2) & Q, Q &= Q >> 2;
-  B |= (B >> 4) & Q, Q &= Q >> 4;
-  B |= (B >> 8) & Q, Q &= Q >> 8;
-  B |= (B >> 16) & Q;
-  return B;
-}
 
 template <int U, bool G32>
 __global__ void __launch_bounds__(256, COMPACT_W_MINB) compact_seg_w_kernel(const u64* __restrict__ keys, u32 m, RunKey<G32> R,
@@ -207,7 +179,7 @@ __global__ void __launch_bounds__(256, COMPACT_W_MINB) compact_seg_w_kernel(cons
       wm[u] = __ballot_sync(~0u, i < end && (k[u] & 1ull));
       prevg = __shfl_sync(~0u, g, 31);
       // F masks (kp reused for the keep masks below)
-      kp[u] = COMPACT_W_KS ? seg_or_fwd(wm[u], ~sp[u], fcar) : __ballot_sync(~0u, fwd(sp[u], wm[u], fcar));
+      kp[u] = __ballot_sync(~0u, fwd(sp[u], wm[u], fcar));
       fcar = kp[u] >> 31;
     }
     const unsigned fl = kp[U - 1];  // F mask of the batch's last row (it may become the pending row)
@@ -227,7 +199,7 @@ __global__ void __launch_bounds__(256, COMPACT_W_MINB) compact_seg_w_kernel(cons
     for (int u = 0; u < U; u++)
       if (!(np && u == U - 1)) need |= cand_of(u) & ~kp[u];
     unsigned bnext = 0u;  // B carry into the row from the right (1 = unknown: the next batch)
-    if (!COMPACT_W_SKIP || need) {
+    if (need) {
       bnext = 1u;
       // backward: keep masks, last row first
 #pragma unroll
@@ -242,7 +214,7 @@ __global__ void __launch_bounds__(256, COMPACT_W_MINB) compact_seg_w_kernel(cons
         const unsigned V = (last && end - rb < 32) ? ((1u << (end - rb)) - 1u) : ~0u;
         const unsigned car = last ? succ : bnext;
         // (the lanes past the range's end are no heads: the last run's carry is succ)
-        const unsigned bm = COMPACT_W_KS ? seg_or_bwd(wm[u], ~sp[u] & V, car) : __ballot_sync(~0u, bwd(sp[u], wm[u], V, car));
+        const unsigned bm = __ballot_sync(~0u, bwd(sp[u], wm[u], V, car));
         kp[u] = cand_of(u) & (kp[u] | bm);
         bnext = sp[u] & bm & 1u;
       }
@@ -252,7 +224,7 @@ __global__ void __launch_bounds__(256, COMPACT_W_MINB) compact_seg_w_kernel(cons
     }
     if (pending) {  // the previous batch's last row: its run's backward carry is this batch's row-0 carry
       unsigned bm = 0u;
-      if (pcand & ~pfm) bm = COMPACT_W_KS ? seg_or_bwd(pwm, ~psp, bnext) : __ballot_sync(~0u, bwd(psp, pwm, ~0u, bnext));
+      if (pcand & ~pfm) bm = __ballot_sync(~0u, bwd(psp, pwm, ~0u, bnext));
       write(pk, pcand & (pfm | bm));
     }
 #pragma unroll

@@ -495,7 +495,7 @@ bool sesa_trace::try_bucket_keys(u64 m, u64** comp, u32* m2, bool* used) {
 }
 
 // ---- the bucket path with its first partition fused into the extents pass (k_extract.cu "Extents fused with the
-// bucket path's first partition"): predicted by a sample of 2^20 records before any pass (global, one granule,
+// bucket path's first partition"): predicted by a sample of 2^18 records before any pass (global, one granule,
 // (block, interval)-ordered, granule span 2^22 .. 2^30, even chunks); then checked exactly on the pass's summary.
 // *used = false (and true returned) when not predicted or not eligible: the caller runs the ordinary path.
 bool sesa_trace::try_extents_part(const Rec* rec, u64 n, u64 index_base, u64** comp, u32* m2, bool* used) {
@@ -504,8 +504,9 @@ bool sesa_trace::try_extents_part(const Rec* rec, u64 n, u64 index_base, u64** c
   const u32 log2G = (u32)__builtin_ctz(cfg.granularity);
   if (!grow(b_xtmp, presample_temp_bytes() + 256, "presample") || !grow(b_xsmall, 4096, "regions")) return false;
   // two stages (bucket_choose's bounds): 2^16 samples reject most other traces at once — a shared or
-  // multi-granule record, an inversion, a hot region (C2-C4) — then 2^20 samples for the tight chunk bound
-  for (u32 want : {1u << 16, 1u << 20}) {
+  // multi-granule record, an inversion, a hot region (C2-C4) — then 2^18 samples for the tight chunk bound
+  // (C5: ~8 samples per chunk, the sampled maximum ~2.5x the mean: well inside the 4x bound)
+  for (u32 want : {1u << 16, 1u << 18}) {
     unsigned long long ext[4] = {1, 0, 0, 0};
     u32 samples = 0;
     LAUNCH("presample", 64.0 * want, launch_presample(rec, (u32)n, log2G, want, b_xtmp.p, ext, &samples, stream));
@@ -516,7 +517,7 @@ bool sesa_trace::try_extents_part(const Rec* rec, u64 n, u64 index_base, u64** c
     if (nb <= HYB_LO + RADIX_BITS || nb > HYB_LO + 2 * RADIX_BITS) return true;
     const double mean = (double)n / (double)(((ext[2] - G0) >> HYB_CHUNK) + 1);
     const double est_max = (double)ext[3] * (double)n / (double)std::max(1u, samples);
-    if (want < (1u << 20) ? est_max > 32.0 * mean + 65536.0
+    if (want < (1u << 18) ? est_max > 32.0 * mean + 65536.0
                           : (est_max > 4.0 * mean + 2048.0 || est_max > (double)(1u << 20)))
       return true;
   }

@@ -1,7 +1,7 @@
 """GPU parity of the bucket path with its first partition fused into the extents pass (k_extract.cu
 "Extents fused with the bucket path's first partition", k_sort.cu UNST 3, sesa_api.cu try_extents_part).
 
-The fused pass is speculative: a sample of 2^20 records predicts it, the pass's own summary decides it, and
+The fused pass is speculative: a sample of 2^16 then 2^18 records predicts it, the pass's own summary decides it, and
 anything the sample could not see — a shared record, a two-granule record, a (block, interval) inversion, an
 invalid record between sampled positions, or a first digit so uneven that a region fills up — sends the check
 back to the ordinary path.  Every case must give the oracle's race list byte for byte.
