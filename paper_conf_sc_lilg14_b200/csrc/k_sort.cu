@@ -525,7 +525,7 @@ __global__ void __launch_bounds__(THREADS, MINB) onesweep2_kernel(const u64* __r
 constexpr int PT_THREADS = 256, PT_ITEMS = 32, PT_MINB = 2;
 #define OS_UCFG PT_THREADS, PT_ITEMS, PT_MINB, OS_LBW, true, 1, false, 2, 4, 1
 #define OS_UCFG2 PT_THREADS, PT_ITEMS, PT_MINB, OS_LBW, true, 1, false, 2, 4, 2
-#define OS_UCFG3 PT_THREADS, PT_ITEMS, PT_MINB, OS_LBW, true, 1, false, 2, 4, 3
+#define OS_UCFG3 R3_THREADS_, R3_ITEMS_, R3_MINB_, OS_LBW, true, 1, false, 2, 4, 3
 
 static size_t onesweep2_smem() {
   constexpr int WARPS = OS_THREADS / 32;
@@ -560,11 +560,11 @@ void launch_partition_regions(const u64* kin, u64* kout, u32 tpr, u32 shift, con
                               cudaStream_t st) {
   const u32 tiles = tpr * RADIX;
   if (!tiles) return;
-  constexpr int WARPS = PT_THREADS / 32, TILE = PT_THREADS * PT_ITEMS;
+  constexpr int WARPS = R3_THREADS_ / 32, TILE = R3_THREADS_ * R3_ITEMS_;
   const size_t sm = (size_t)TILE * 8 + (size_t)WARPS * RADIX * 4 + RADIX * 4 + (WARPS + 1) * 4;
   smem_optin((const void*)onesweep2_kernel<OS_UCFG3>, sm);
   MapArgs mp{fill, cap, tpr, pos_bits, g0};
-  onesweep2_kernel<OS_UCFG3><<<tiles, PT_THREADS, sm, st>>>(kin, kout, (u32)((u64)tiles * TILE), shift, bin_base,
+  onesweep2_kernel<OS_UCFG3><<<tiles, R3_THREADS_, sm, st>>>(kin, kout, (u32)((u64)tiles * TILE), shift, bin_base,
                                                             lookback, tile_ctr, epoch, mp);
 }
 

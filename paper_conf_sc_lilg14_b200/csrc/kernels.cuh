@@ -44,7 +44,17 @@ struct XPArgs {
   u32* overflow;     // zeroed; 1 if a region would pass cap
 };
 void launch_extents_part(const XPArgs& A, cudaStream_t st);
-constexpr u32 PART_TILE_KEYS = 256 * 32;  // keys per tile of the partition passes (k_sort.cu PT_*)
+// tile of the second partition pass over the regions (k_sort.cu OS_UCFG3)
+#ifndef R3_THREADS_
+#define R3_THREADS_ 256
+#endif
+#ifndef R3_ITEMS_
+#define R3_ITEMS_ 24
+#endif
+#ifndef R3_MINB_
+#define R3_MINB_ 3
+#endif
+constexpr u32 PART_TILE_KEYS = R3_THREADS_ * R3_ITEMS_;
 // the second partition pass over launch_extents_part's regions: tpr tiles per region (cap is a multiple of
 // PART_TILE_KEYS, tpr * PART_TILE_KEYS >= every fill), keys rebased from raw low-30 granule bits by g0
 void launch_partition_regions(const u64* kin, u64* kout, u32 tpr, u32 shift, const u64* bin_base, u64* lookback,
