@@ -223,7 +223,13 @@ static size_t onesweep_kv_smem() {
 // 4th item by 8 ballots (ALU pipe), the others by shared-memory masks (LSU pipe, the binding one) — measured
 // against all-masks, all-ballots, every 2nd/3rd item by ballots and MATCH.
 // ------------------------------------------------------------------------------------------------------------
-constexpr int OS_THREADS = 256, OS_ITEMS = 32, OS_MINB = 2, OS_LBW = 4, OS_TILE = OS_THREADS * OS_ITEMS;
+#ifndef OS_ITEMS_
+#define OS_ITEMS_ 32
+#endif
+#ifndef OS_MINB_
+#define OS_MINB_ 2
+#endif
+constexpr int OS_THREADS = 256, OS_ITEMS = OS_ITEMS_, OS_MINB = OS_MINB_, OS_LBW = 4, OS_TILE = OS_THREADS * OS_ITEMS;
 
 __device__ __forceinline__ u64 gtime() {
   u64 t;

@@ -6,10 +6,17 @@ namespace sesa {
 
 constexpr int RADIX_BITS = 8;  // onesweep digit width (8-bit digits, 256 bins per pass)
 constexpr int RADIX = 1 << RADIX_BITS;
-// fused key extract + first sort pass (k_fused.cu): tiles of 256 threads x 32 records
+// fused key extract + first sort pass (k_fused.cu): tiles of 256 threads x FUSED_ITEMS records (stable variant,
+// C3/C4: 16 items at 3 CTAs/SM — C3 5.88 -> 5.81 ms, C4 extract 2.10 -> 2.01 ms against 24 at 2; 20 at 3 between)
 // (unstable variant, C5: 24 items at 2 CTAs/SM 3.75 ms; at 3 CTAs/SM 3.72; 16 items at 3-4 CTAs/SM 4.8-5.0;
 // 32 items 3.65 but the extents pass's per-tile histograms slow it by 0.18 ms)
-constexpr int FUSED_THREADS = 256, FUSED_ITEMS = 24, FUSED_MINB = 2, FUSED_TILE = FUSED_THREADS * FUSED_ITEMS;
+#ifndef FUSED_ITEMS_
+#define FUSED_ITEMS_ 16
+#endif
+#ifndef FUSED_MINB_
+#define FUSED_MINB_ 3
+#endif
+constexpr int FUSED_THREADS = 256, FUSED_ITEMS = FUSED_ITEMS_, FUSED_MINB = FUSED_MINB_, FUSED_TILE = FUSED_THREADS * FUSED_ITEMS;
 constexpr int FUSED_UMINB = 2;  // CTAs per SM of the bucket path's unstable variant
 
 // onesweep tile: 256 threads x 16 keys (warp-striped); one lookback word per (tile, bin)
