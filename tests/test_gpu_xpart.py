@@ -136,3 +136,18 @@ def test_regions_registered_skip_the_fused_pass(S, base_trace):
     t.close()
     assert "presample" not in names
     assert got.tobytes() == O.check(base_trace, method="partitioned").tobytes()
+
+
+def test_precise_warp_through_the_fused_path(S, base_trace):
+    # the precise warp model (NEXT-3) on a trace large enough for the fused path: random {pc, div} against the
+    # oracle's precise-warp checker
+    a = base_trace
+    e = G.random_ext(len(a), 5, npc=3, ninst=2, div_frac=0.5)
+    t = S.Trace(32, 1, 4)
+    t.set_profiling(True)
+    t.check_warp(S.to_device(a), torch.from_numpy(np.ascontiguousarray(e).view(np.uint8).reshape(-1)).cuda(), len(a))
+    names = {k["name"] for k in t.kernel_stats()}
+    got = t.races()
+    t.close()
+    assert "presample" in names
+    assert got.tobytes() == O.check_warp(a, e, warp_size=32).tobytes()
