@@ -500,6 +500,7 @@ bool sesa_trace::try_bucket_keys(u64 m, u64** comp, u32* m2, bool* used) {
 // *used = false (and true returned) when not predicted or not eligible: the caller runs the ordinary path.
 bool sesa_trace::try_extents_part(const Rec* rec, u64 n, u64 index_base, u64** comp, u32* m2, bool* used) {
   *used = false;
+  presample_hot = false;
   if (n < BUCKET_MIN_N || n >= (1ull << 31) || n_regions) return true;
   const u32 log2G = (u32)__builtin_ctz(cfg.granularity);
   if (!grow(b_xtmp, presample_temp_bytes() + 256, "presample") || !grow(b_xsmall, 4096, "regions")) return false;
@@ -518,8 +519,10 @@ bool sesa_trace::try_extents_part(const Rec* rec, u64 n, u64 index_base, u64** c
     const double mean = (double)n / (double)(((ext[2] - G0) >> HYB_CHUNK) + 1);
     const double est_max = (double)ext[3] * (double)n / (double)std::max(1u, samples);
     if (want < (1u << 18) ? est_max > 32.0 * mean + 65536.0
-                          : (est_max > 4.0 * mean + 2048.0 || est_max > (double)(1u << 20)))
+                          : (est_max > 4.0 * mean + 2048.0 || est_max > (double)(1u << 20))) {
+      presample_hot = true;  // (bucket_choose's bounds on the same records: it need not sample again)
       return true;
+    }
   }
   // the pass
   const u32 pos_bits = std::max(1u, bits_of(n - 1));
@@ -1074,7 +1077,7 @@ sesa_status sesa_trace::check_device(const sesa_access* d_rec, u64 n, u64 index_
   // bucket path: large traces whose granules spread evenly (k_bucket.cu)
   u64 hyb_g0 = 0;
   u32 hyb_nb = 0, hyb_nc = 0;
-  if (fused && have_thist2 && bucket_choose(n, &hyb_g0, &hyb_nb, &hyb_nc)) {
+  if (fused && have_thist2 && !presample_hot && bucket_choose(n, &hyb_g0, &hyb_nb, &hyb_nc)) {
     layout.gminG = hyb_g0;
     layout.gbG = hyb_nb;
     layout.sort_bits = hyb_nb;

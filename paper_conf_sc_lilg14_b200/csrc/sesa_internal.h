@@ -50,6 +50,7 @@ struct sesa_trace {
   sesa_flow_check_info flow_info{};
   const void* warp_ext = nullptr;  // precise warp model: the {pc, div} extension of the records being checked
   uint32_t conflict_tdiv = 0;      // > 1: conflict tiles with identity = thread / tdiv, lockstep off
+  bool presample_hot = false;  // this check's record sample found a hot chunk: the bucket path cannot pay
   bool have_thist2 = false;  // extents also wrote the per-tile histograms of the bucket path's first digit
   bool have_thist = false;
   bool hist_from_extents = false;  // fused path: later-digit histograms from the extents' raw granule bytes  // extents wrote per-tile raw digit histograms (fused first pass possible)
