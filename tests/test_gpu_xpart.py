@@ -151,3 +151,16 @@ def test_precise_warp_through_the_fused_path(S, base_trace):
     t.close()
     assert "presample" in names
     assert got.tobytes() == O.check_warp(a, e, warp_size=32).tobytes()
+
+
+def test_host_entry_through_the_fused_path(S, base_trace):
+    # sesa_race_check_host (the e2e entry: pageable host records, chunked through pinned staging) takes the same
+    # fused path and returns the oracle's list, index_base applied
+    t = S.Trace(32, 0, 4)
+    t.set_profiling(True)
+    t.check_host(base_trace, index_base=123)
+    names = {k["name"] for k in t.kernel_stats()}
+    got = t.races()
+    t.close()
+    assert "presample" in names and "extract_pass0" not in names
+    assert got.tobytes() == O.check(base_trace, index_base=123, method="partitioned").tobytes()
