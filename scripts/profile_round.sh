@@ -1,5 +1,5 @@
-# round-end evidence: ncu launch lists (C5, C4) and --set full captures of the hot kernels; bash scripts/profile_r2s.sh <tag>
-TAG=${1:-r2s}; OUT=gpurun_out; mkdir -p $OUT
+# round-end evidence: ncu launch lists (C5, C4) and --set full captures of the hot kernels; bash scripts/profile_round.sh <tag>
+TAG=${1:-r2}; OUT=gpurun_out; mkdir -p $OUT
 B="python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu"
 timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv --log-file $OUT/launches_c5_$TAG.csv $B > /dev/null 2>&1
 python scripts/launch_summary.py $OUT/launches_c5_$TAG.csv > $OUT/launches_c5_$TAG.txt 2>&1; head -16 $OUT/launches_c5_$TAG.txt
