@@ -503,6 +503,18 @@ bool sesa_trace::try_extents_part(const Rec* rec, u64 n, u64 index_base, u64** c
   presample_hot = false;
   if (n < BUCKET_MIN_N || n >= (1ull << 31) || n_regions) return true;
   const u32 log2G = (u32)__builtin_ctz(cfg.granularity);
+  {  // a peek at the first 64 records (one small copy): a shared or two-granule record there rules the path out
+     // before any sampling kernel (C2 starts with its shared tiles)
+    sesa_access head[64];
+    const u64 k = std::min<u64>(64, n);
+    if (!cuda_ok(cudaMemcpyAsync(head, rec, k * sizeof(sesa_access), cudaMemcpyDeviceToHost, stream), "peek") ||
+        !sync_check("peek"))
+      return false;
+    for (u64 i = 0; i < k; i++) {
+      const u64 g0 = head[i].addr >> log2G, g1 = (head[i].addr + (u64)head[i].size - 1ull) >> log2G;
+      if (head[i].space != SP_GLOBAL || head[i].size == 0 || g0 != g1) return true;
+    }
+  }
   if (!grow(b_xtmp, presample_temp_bytes() + 256, "presample") || !grow(b_xsmall, 4096, "regions")) return false;
   // two stages (bucket_choose's bounds): 2^16 samples reject most other traces at once — a shared or
   // multi-granule record, an inversion, a hot region (C2-C4) — then 2^18 samples for the tight chunk bound
